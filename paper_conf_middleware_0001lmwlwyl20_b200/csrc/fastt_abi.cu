@@ -1,0 +1,1339 @@
+// fastt_abi.cu -- host side of the C-ABI (include/fastt.h): validation,
+// graph encoding (S1), device memory layout, and the orchestration of the
+// device kernels for rank (S4), batched DPOS (S2-S7), the sweep and OS-DPOS
+// (S8).  Every step of the method itself runs in the kernels of k_prep.cu /
+// k_sim.cu; this file moves data, sizes buffers and sequences launches.
+#include "../../include/fastt.h"
+#include "fastt_internal.cuh"
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <deque>
+#include <mutex>
+#include <string>
+#include <vector>
+
+using namespace fastt;
+
+static thread_local std::string g_err;
+
+static fastt_status fail(fastt_status s, const char *fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return s;
+}
+
+#define CK(x)                                                                                \
+  do {                                                                                       \
+    cudaError_t e_ = (x);                                                                    \
+    if (e_ != cudaSuccess) return fail(FASTT_ECUDA, "%s: %s", #x, cudaGetErrorString(e_));   \
+  } while (0)
+#define TRY(x)                            \
+  do {                                    \
+    fastt_status s_ = (x);                \
+    if (s_ != FASTT_OK) return s_;        \
+  } while (0)
+
+static size_t al16(size_t x) { return (x + 15) & ~(size_t)15; }
+
+// ------------------------------------------------------------------ layouts
+
+struct RawLayout {
+  int64_t vcap = 0, ecap = 0;
+  size_t o[17] = {0};
+  size_t total = 0;
+};
+
+static RawLayout raw_layout(int64_t vcap, int64_t ecap, int G) {
+  RawLayout L;
+  L.vcap = vcap;
+  L.ecap = ecap;
+  size_t sz[17] = {(size_t)vcap * 4, (size_t)vcap * 4, (size_t)vcap * 4, (size_t)vcap * 4,  // off/cnt
+                   (size_t)ecap * 4, (size_t)ecap * 4,                                       // dst, src
+                   (size_t)ecap * 8, (size_t)ecap * 8,                                       // bytes
+                   (size_t)ecap, (size_t)ecap,                                               // param flags
+                   (size_t)vcap * G * 8,                                                     // cost
+                   (size_t)vcap * 8, (size_t)vcap * 8,                                       // mem, param
+                   (size_t)vcap, (size_t)vcap,                                               // split_mask, alive
+                   (size_t)vcap * 4, 16};                                                    // topo, pad
+  size_t off = 0;
+  for (int k = 0; k < 17; k++) {
+    L.o[k] = off;
+    off += al16(sz[k]);
+  }
+  L.total = off;
+  return L;
+}
+
+static RawGraph raw_struct(char *b, const RawLayout &L, int32_t V, int32_t nl, int64_t E) {
+  RawGraph R;
+  R.V = V;
+  R.n_live = nl;
+  R.E = E;
+  R.succ_off = (uint32_t *)(b + L.o[0]);
+  R.succ_cnt = (uint32_t *)(b + L.o[1]);
+  R.pred_off = (uint32_t *)(b + L.o[2]);
+  R.pred_cnt = (uint32_t *)(b + L.o[3]);
+  R.succ_dst = (int32_t *)(b + L.o[4]);
+  R.pred_src = (int32_t *)(b + L.o[5]);
+  R.succ_bytes = (int64_t *)(b + L.o[6]);
+  R.pred_bytes = (int64_t *)(b + L.o[7]);
+  R.succ_param = (uint8_t *)(b + L.o[8]);
+  R.pred_param = (uint8_t *)(b + L.o[9]);
+  R.cost = (int64_t *)(b + L.o[10]);
+  R.mem = (int64_t *)(b + L.o[11]);
+  R.param = (int64_t *)(b + L.o[12]);
+  R.split_mask = (uint8_t *)(b + L.o[13]);
+  R.alive = (uint8_t *)(b + L.o[14]);
+  R.topo = (int32_t *)(b + L.o[15]);
+  return R;
+}
+
+struct PrepLayout {
+  int64_t ncap = 0, ecap = 0;
+  size_t o[19] = {0};
+  size_t total = 0;
+};
+
+static PrepLayout prep_layout(int64_t ncap, int64_t ecap, int G, int K, int tbytes) {
+  PrepLayout L;
+  L.ncap = ncap;
+  L.ecap = ecap;
+  size_t sz[19] = {(size_t)ncap * CARD_WORDS * 4,        // card
+                   (size_t)ncap * G * tbytes,           // costp
+                   (size_t)ecap * 4,                    // pe_src
+                   (size_t)ecap * K * tbytes,           // pe_comm
+                   (size_t)ecap * 4, (size_t)ecap * 4,  // se_dst, se_pe
+                   (size_t)ncap * 4,                    // npred
+                   (size_t)(ncap / 32 + 2) * 4,         // srcbits
+                   (size_t)ncap * 4,                    // pos (V <= ncap)
+                   (size_t)ncap * 4,                    // uid
+                   (size_t)ncap * 8,                    // rank
+                   (size_t)ncap * 4,                    // cp
+                   (size_t)(ncap + 1) * 8,              // pmem
+                   (size_t)(ncap + 1) * G * 8,          // pcost
+                   (size_t)ncap * 8, (size_t)ncap * 8,  // keys
+                   (size_t)ncap * 4, (size_t)ncap * 4,  // vals
+                   16};
+  size_t off = 0;
+  for (int k = 0; k < 19; k++) {
+    L.o[k] = off;
+    off += al16(sz[k]);
+  }
+  L.total = off;
+  return L;
+}
+
+static PrepGraph prep_struct(char *b, const PrepLayout &L, int tbits) {
+  PrepGraph P;
+  memset(&P, 0, sizeof P);
+  P.tbits = tbits;
+  P.card = (uint32_t *)(b + L.o[0]);
+  P.costp = (void *)(b + L.o[1]);
+  P.pe_src = (uint32_t *)(b + L.o[2]);
+  P.pe_comm = (void *)(b + L.o[3]);
+  P.se_dst = (uint32_t *)(b + L.o[4]);
+  P.se_pe = (uint32_t *)(b + L.o[5]);
+  P.npred = (uint32_t *)(b + L.o[6]);
+  P.srcbits = (uint32_t *)(b + L.o[7]);
+  P.pos = (uint32_t *)(b + L.o[8]);
+  P.uid = (uint32_t *)(b + L.o[9]);
+  P.rank = (uint64_t *)(b + L.o[10]);
+  P.cp = (uint32_t *)(b + L.o[11]);
+  P.pmem = (int64_t *)(b + L.o[12]);
+  P.pcost = (int64_t *)(b + L.o[13]);
+  P.key0 = (uint64_t *)(b + L.o[14]);
+  P.key1 = (uint64_t *)(b + L.o[15]);
+  P.val0 = (uint32_t *)(b + L.o[16]);
+  P.val1 = (uint32_t *)(b + L.o[17]);
+  return P;
+}
+
+// ----------------------------------------------------------------- graph
+
+// A "base": a raw graph in HBM plus its prepared (priority-ordered) form.
+// The loaded graph is one; OS-DPOS creates more as it accepts splits.
+struct Base {
+  int32_t V = 0, n_live = 0, n = 0, cp_len = 0;
+  int64_t E = 0;  // edge slots used
+  RawLayout rl;
+  PrepLayout pl;
+  char *raw_block = nullptr;
+  RawGraph *raw_dev = nullptr;
+  char *prep_block = nullptr;
+  PrepGraph *pg_dev = nullptr;
+  int tbits = 64, key_bits = 64;
+  unsigned long long bound = 0, maxextra = 0;
+  void release() {
+    cudaFree(raw_block);
+    cudaFree(raw_dev);
+    cudaFree(prep_block);
+    cudaFree(pg_dev);
+    raw_block = prep_block = nullptr;
+    raw_dev = nullptr;
+    pg_dev = nullptr;
+  }
+};
+
+struct StreamCache {
+  bool valid = false;
+  uint8_t *base_place = nullptr;
+  int32_t *live = nullptr;
+  int32_t n_live = 0;
+  int64_t n_split = 0;
+  int32_t *split_op = nullptr;
+  uint8_t *split_dim = nullptr, *split_n = nullptr;
+  void release() {
+    cudaFree(base_place);
+    cudaFree(live);
+    cudaFree(split_op);
+    cudaFree(split_dim);
+    cudaFree(split_n);
+    *this = StreamCache();
+  }
+};
+
+struct fastt_graph {
+  int dev = 0;
+  int32_t V = 0, G = 1, K = 1;
+  int64_t E = 0;
+  int32_t maxP = 0, maxS = 0;
+  int32_t v_max = 0;  // V + largest single-split overlay (user-facing per-op array size)
+  GraphConst gch;
+  GraphConst *gc_dev = nullptr;
+  uint8_t *split_mask_dev = nullptr;
+  Base base;
+  std::vector<uint8_t> split_mask_h;
+  StreamCache streams[4];
+  // arena (per base layout)
+  size_t arena_raw_total = 0, arena_prep_total = 0;
+  int arena_slots = 0;
+  char *arena = nullptr;
+  RawGraph *tmpl_dev = nullptr, *slot_raws_dev = nullptr;
+  PrepGraph *slot_pgs_dev = nullptr;
+  Cand *slot_cands = nullptr;
+  int64_t *slot_result = nullptr, *slot_index = nullptr;
+  // simulation workspace
+  int sms = 148, sim_block = 256, sim_grid = 0, sim_tbits = 0;
+  int64_t sim_ncap = 0;
+  size_t sim_smem = 0;
+  void *slab = nullptr;
+  int64_t *wbest = nullptr, *best_dev = nullptr;
+  unsigned long long *counters = nullptr;  // [0] work counter, [1] deferred count
+  int64_t *defer_q = nullptr;
+  int64_t defer_cap = 0;
+  // misc scratch
+  int64_t *scratch_rank = nullptr;
+  int32_t *scratch_cp = nullptr, *scratch_list = nullptr, *scratch_n = nullptr;
+  std::mutex mu;
+};
+
+static int64_t overlay_v(const fastt_graph *g) { return (int64_t)g->maxP + g->G + g->maxS + 1; }
+static int64_t overlay_e(const fastt_graph *g) {
+  return (int64_t)g->maxP * (2 + g->G) + (int64_t)g->maxS * (2 + g->G) + (int64_t)g->G + 16;
+}
+
+struct Dev {  // RAII device guard
+  int prev = -1;
+  explicit Dev(int d) {
+    cudaGetDevice(&prev);
+    cudaSetDevice(d);
+  }
+  ~Dev() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+static cudaStream_t stream_of(const fastt_opts *o) { return o ? (cudaStream_t)o->cuda_stream : (cudaStream_t)0; }
+static uint32_t flags_of(const fastt_opts *o) { return o ? o->flags : 0u; }
+
+// ------------------------------------------------------ base preparation
+
+static int bits_for(unsigned long long v) {
+  int b = 1;
+  while (b < 64 && (v >> b) != 0) b++;
+  return b;
+}
+
+// bound -> time type; rank, sort, cards, CP for a base whose raw graph is in place
+static fastt_status prepare_base(fastt_graph *g, Base &B, cudaStream_t st) {
+  unsigned long long *d_b = nullptr;
+  CK(cudaMalloc(&d_b, 16));
+  CK(cudaMemsetAsync(d_b, 0, 16, st));
+  launch_bound(B.raw_dev, g->gc_dev, g->G, d_b, st);
+  unsigned long long hb[2];
+  CK(cudaMemcpyAsync(hb, d_b, 16, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  cudaFree(d_b);
+  B.bound = hb[0];
+  B.maxextra = hb[1];
+  unsigned long long tot = hb[0] + hb[1];
+  B.tbits = tot < (1ull << 32) ? 32 : 64;
+  B.key_bits = B.tbits == 32 ? 32 : bits_for(tot);
+  // prepared block (capacity = raw capacity)
+  B.pl = prep_layout(B.rl.vcap, B.rl.ecap, g->G, g->K, B.tbits / 8);
+  CK(cudaMalloc(&B.prep_block, B.pl.total));
+  CK(cudaMalloc(&B.pg_dev, sizeof(PrepGraph)));
+  PrepGraph P = prep_struct(B.prep_block, B.pl, B.tbits);
+  P.V = B.V;
+  CK(cudaMemcpyAsync(B.pg_dev, &P, sizeof P, cudaMemcpyHostToDevice, st));
+  launch_rank(B.raw_dev, B.pg_dev, g->gc_dev, nullptr, 1, g->G, st);
+  launch_sort(B.pg_dev, B.raw_dev, 1, B.key_bits, B.n_live, st);
+  launch_cards(B.raw_dev, B.pg_dev, g->gc_dev, 1, B.n_live, g->G, g->K, B.tbits, st);
+  launch_cp(B.pg_dev, 1, g->G, B.tbits, st);
+  CK(cudaGetLastError());
+  CK(cudaMemcpyAsync(&P, B.pg_dev, sizeof P, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  B.n = P.n;
+  B.cp_len = P.cp_len;
+  return FASTT_OK;
+}
+
+// ------------------------------------------------------------- workspaces
+
+static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st) {
+  size_t rt = B.rl.total, pt = B.pl.total;
+  if (g->arena && g->arena_raw_total == rt && g->arena_prep_total == pt) return FASTT_OK;
+  cudaFree(g->arena);
+  cudaFree(g->tmpl_dev);
+  cudaFree(g->slot_raws_dev);
+  cudaFree(g->slot_pgs_dev);
+  cudaFree(g->slot_cands);
+  cudaFree(g->slot_result);
+  cudaFree(g->slot_index);
+  g->arena = nullptr;
+  size_t freeb = 0, totb = 0;
+  CK(cudaMemGetInfo(&freeb, &totb));
+  size_t per = rt + pt;
+  int64_t slots = (int64_t)(freeb / 4 / per);
+  if (slots > 512) slots = 512;
+  if (slots < 1) return fail(FASTT_ENOMEM, "device memory too small for one preparation slot (%zu bytes)", per);
+  g->arena_slots = (int)slots;
+  CK(cudaMalloc(&g->arena, per * slots));
+  std::vector<RawGraph> tm(slots);
+  std::vector<PrepGraph> pg(slots);
+  for (int64_t k = 0; k < slots; k++) {
+    char *b = g->arena + per * k;
+    tm[k] = raw_struct(b, B.rl, 0, 0, 0);
+    pg[k] = prep_struct(b + rt, B.pl, B.tbits);
+  }
+  CK(cudaMalloc(&g->tmpl_dev, sizeof(RawGraph) * slots));
+  CK(cudaMalloc(&g->slot_raws_dev, sizeof(RawGraph) * slots));
+  CK(cudaMalloc(&g->slot_pgs_dev, sizeof(PrepGraph) * slots));
+  CK(cudaMalloc(&g->slot_cands, sizeof(Cand) * slots));
+  CK(cudaMalloc(&g->slot_result, sizeof(int64_t) * slots));
+  CK(cudaMalloc(&g->slot_index, sizeof(int64_t) * slots));
+  CK(cudaMemcpyAsync(g->tmpl_dev, tm.data(), sizeof(RawGraph) * slots, cudaMemcpyHostToDevice, st));
+  CK(cudaMemcpyAsync(g->slot_pgs_dev, pg.data(), sizeof(PrepGraph) * slots, cudaMemcpyHostToDevice, st));
+  CK(cudaStreamSynchronize(st));
+  g->arena_raw_total = rt;
+  g->arena_prep_total = pt;
+  return FASTT_OK;
+}
+
+static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need) {
+  int64_t ncap = B.pl.ncap;
+  if (!g->slab || g->sim_tbits != B.tbits || g->sim_ncap < ncap) {
+    cudaFree(g->slab);
+    cudaFree(g->wbest);
+    g->slab = nullptr;
+    g->wbest = nullptr;
+    int leaf = (int)((ncap + 31) / 32);
+    size_t smem = (size_t)(g->sim_block / 32) * (leaf + 32) * 4;
+    if (smem > 48 * 1024) CK(sim_set_smem(B.tbits, smem));
+    int per_sm = sim_occupancy(B.tbits, g->sim_block, smem);
+    if (per_sm < 1) return fail(FASTT_EUNSUP, "simulation kernel does not fit on an SM (smem %zu)", smem);
+    g->sim_grid = g->sms * per_sm;
+    g->sim_smem = smem;
+    int64_t nwarps = (int64_t)g->sim_grid * (g->sim_block / 32);
+    size_t rec = B.tbits == 32 ? 8 : 16;
+    CK(cudaMalloc(&g->slab, (size_t)nwarps * ncap * rec));
+    CK(cudaMalloc(&g->wbest, sizeof(int64_t) * 2 * nwarps));
+    g->sim_tbits = B.tbits;
+    g->sim_ncap = ncap;
+  }
+  if (!g->counters) {
+    CK(cudaMalloc(&g->counters, 2 * sizeof(unsigned long long)));
+    CK(cudaMalloc(&g->best_dev, 2 * sizeof(int64_t)));
+  }
+  if (g->defer_cap < defer_need) {
+    cudaFree(g->defer_q);
+    int64_t cap = std::max<int64_t>(defer_need, 1024);
+    CK(cudaMalloc(&g->defer_q, sizeof(int64_t) * cap));
+    g->defer_cap = cap;
+  }
+  return FASTT_OK;
+}
+
+static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
+  SimArgs a;
+  memset(&a, 0, sizeof a);
+  a.flags = flags;
+  a.base = B.pg_dev;
+  a.slots = g->slot_pgs_dev;
+  a.gc = g->gc_dev;
+  a.split_mask = B.raw_block ? raw_struct(B.raw_block, B.rl, 0, 0, 0).split_mask : nullptr;
+  a.counter = g->counters;
+  a.ndefer = g->counters + 1;
+  a.defer_q = g->defer_q;
+  a.wbest = g->wbest;
+  a.slab = g->slab;
+  a.slab_stride = g->sim_ncap;
+  a.leaf_words = (int32_t)((g->sim_ncap + 31) / 32);
+  a.G = g->G;
+  return a;
+}
+
+// Preparation pipeline for nslots deferred candidates already in slot_cands
+// (SURVEY 8(a) S3 + S4 + S5 per candidate): materialise splits, ranks with
+// the candidate's allowed sets, priority sort, cards, critical path.
+static fastt_status run_prep(fastt_graph *g, const Base &B, int nslots, cudaStream_t st) {
+  launch_slot_setup(g->slot_cands, g->tmpl_dev, B.raw_dev, g->slot_raws_dev, nslots, st);
+  launch_copy_block(B.raw_block, g->arena, (int64_t)(g->arena_raw_total + g->arena_prep_total), (int64_t)B.rl.total,
+                    g->slot_cands, nslots, st);
+  launch_patch_split(B.raw_dev, g->slot_raws_dev, g->gc_dev, g->slot_cands, nslots, st);
+  launch_rank(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, g->slot_cands, nslots, g->G, st);
+  launch_sort(g->slot_pgs_dev, g->slot_raws_dev, nslots, B.key_bits, (int)B.rl.vcap, st);
+  launch_cards(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, nslots, (int)B.rl.vcap, g->G, g->K, B.tbits, st);
+  launch_cp(g->slot_pgs_dev, nslots, g->G, B.tbits, st);
+  CK(cudaGetLastError());
+  return FASTT_OK;
+}
+
+struct DevOut {
+  int64_t *makespan = nullptr;
+  uint8_t *status = nullptr;
+  int64_t *peak = nullptr;
+  uint8_t *place = nullptr;
+  int64_t *start = nullptr;
+  int32_t *deq = nullptr;
+  int32_t *order = nullptr;
+  int64_t vmax = 0;
+};
+
+// DPOS of n candidates (device array) on base B.  Outputs: device pointers.
+static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int64_t n, uint32_t flags,
+                               cudaStream_t st, DevOut o) {
+  if (n <= 0) return FASTT_OK;
+  TRY(ensure_sim(g, B, n));
+  if (o.place) CK(cudaMemsetAsync(o.place, 0xFF, (size_t)n * o.vmax, st));
+  if (o.start) launch_fill_i64(o.start, n * o.vmax, -1, st);
+  if (o.deq) CK(cudaMemsetAsync(o.deq, 0xFF, (size_t)n * o.vmax * 4, st));
+  CK(cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), st));
+  SimArgs a = sim_args(g, B, flags);
+  a.mode = 1;
+  a.cands = d_cands;
+  a.n = n;
+  a.out.makespan = o.makespan;
+  a.out.status = o.status;
+  a.out.peak = o.peak;
+  a.out.place = o.place;
+  a.out.start = o.start;
+  a.out.deq = o.deq;
+  a.out.vmax = (int32_t)o.vmax;
+  launch_sim(a, B.tbits, g->sim_grid, g->sim_block, g->sim_smem, st);
+  CK(cudaGetLastError());
+  unsigned long long nd = 0;
+  CK(cudaMemcpyAsync(&nd, g->counters + 1, sizeof nd, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  if (nd > 0) {
+    TRY(ensure_arena(g, B, st));
+    for (int64_t c0 = 0; c0 < (int64_t)nd; c0 += g->arena_slots) {
+      int nc = (int)std::min<int64_t>(g->arena_slots, (int64_t)nd - c0);
+      launch_gather_cands(d_cands, g->defer_q + c0, nc, g->slot_cands, g->slot_result, st);
+      TRY(run_prep(g, B, nc, st));
+      CK(cudaMemsetAsync(g->counters, 0, sizeof(unsigned long long), st));
+      SimArgs b = a;
+      b.slots = g->slot_pgs_dev;
+      b.mode = 2;
+      b.cands = g->slot_cands;
+      b.slot_result = g->slot_result;
+      b.slot_index = nullptr;
+      b.n = nc;
+      launch_sim(b, B.tbits, std::min(g->sim_grid, (nc + 7) / 8 + 1), g->sim_block, g->sim_smem, st);
+      CK(cudaGetLastError());
+    }
+  }
+  if (o.order) {
+    // execution order list A (R17): per-result stable sort of the dequeue list by start
+    int64_t chunk = 256;
+    uint64_t *k0, *k1;
+    uint32_t *v0, *v1;
+    CK(cudaMalloc(&k0, (size_t)chunk * o.vmax * 8));
+    CK(cudaMalloc(&k1, (size_t)chunk * o.vmax * 8));
+    CK(cudaMalloc(&v0, (size_t)chunk * o.vmax * 4));
+    CK(cudaMalloc(&v1, (size_t)chunk * o.vmax * 4));
+    std::vector<int64_t> idx(chunk);
+    int64_t *d_idx;
+    CK(cudaMalloc(&d_idx, sizeof(int64_t) * chunk));
+    for (int64_t c0 = 0; c0 < n; c0 += chunk) {
+      int64_t nc = std::min(chunk, n - c0);
+      for (int64_t k = 0; k < nc; k++) idx[k] = c0 + k;
+      CK(cudaMemcpyAsync(d_idx, idx.data(), sizeof(int64_t) * nc, cudaMemcpyHostToDevice, st));
+      launch_order_chunk(o.deq, o.start, o.order, d_idx, nc, o.vmax, B.key_bits, k0, k1, v0, v1, st);
+      CK(cudaStreamSynchronize(st));
+    }
+    cudaFree(k0);
+    cudaFree(k1);
+    cudaFree(v0);
+    cudaFree(v1);
+    cudaFree(d_idx);
+  }
+  CK(cudaStreamSynchronize(st));
+  return FASTT_OK;
+}
+
+// ----------------------------------------------------------------- stream
+
+static int split_counts(int G, int pow2, int *ns) {
+  int c = 0;
+  for (int n = 2; n <= G; n++)
+    if (!pow2 || (n & (n - 1)) == 0) ns[c++] = n;
+  return c;
+}
+
+// split-eligible placement-aware CP of a placement (Alg. 2 lines 4-5) -> host list
+static fastt_status split_list(fastt_graph *g, Base &B, const uint8_t *d_place, std::vector<int32_t> &out,
+                               cudaStream_t st) {
+  if (!g->scratch_rank) {
+    CK(cudaMalloc(&g->scratch_n, 16));
+  }
+  cudaFree(g->scratch_rank);
+  cudaFree(g->scratch_cp);
+  cudaFree(g->scratch_list);
+  CK(cudaMalloc(&g->scratch_rank, sizeof(int64_t) * (B.V + 1)));
+  CK(cudaMalloc(&g->scratch_cp, sizeof(int32_t) * (B.V + 1)));
+  CK(cudaMalloc(&g->scratch_list, sizeof(int32_t) * (B.V + 1)));
+  launch_splitlist(B.raw_dev, g->gc_dev, d_place, g->scratch_list, g->scratch_n, g->scratch_rank, g->scratch_cp,
+                   g->G, st);
+  CK(cudaGetLastError());
+  int32_t m = 0;
+  CK(cudaMemcpyAsync(&m, g->scratch_n, 4, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  out.resize(m);
+  if (m) CK(cudaMemcpy(out.data(), g->scratch_list, sizeof(int32_t) * m, cudaMemcpyDeviceToHost));
+  return FASTT_OK;
+}
+
+static fastt_status ensure_stream(fastt_graph *g, uint32_t flags, int pow2, cudaStream_t st, StreamCache **out) {
+  int key = (int)(flags & FASTT_F_CP_PIN) | (pow2 ? 2 : 0);
+  StreamCache &S = g->streams[key];
+  *out = &S;
+  if (S.valid) return FASTT_OK;
+  Base &B = g->base;
+  const int64_t vm = B.rl.vcap;
+  // one DPOS run of BASE (R21)
+  Cand c;
+  memset(&c, 0, sizeof c);
+  c.split_op = -1;
+  for (int k = 0; k < 4; k++) c.pin_op[k] = -1;
+  Cand *d_c;
+  int64_t *d_ms;
+  uint8_t *d_st;
+  CK(cudaMalloc(&d_c, sizeof c));
+  CK(cudaMalloc(&d_ms, 8));
+  CK(cudaMalloc(&d_st, 1));
+  CK(cudaMalloc(&S.base_place, vm));
+  CK(cudaMemcpyAsync(d_c, &c, sizeof c, cudaMemcpyHostToDevice, st));
+  DevOut o;
+  o.makespan = d_ms;
+  o.status = d_st;
+  o.place = S.base_place;
+  o.vmax = vm;
+  TRY(eval_batch(g, B, d_c, 1, flags, st, o));
+  uint8_t hst = 0;
+  CK(cudaMemcpy(&hst, d_st, 1, cudaMemcpyDeviceToHost));
+  std::vector<int32_t> list;
+  if (hst != FASTT_CAND_OK) {
+    CK(cudaMemsetAsync(S.base_place, 0, vm, st));
+  } else {
+    TRY(split_list(g, B, S.base_place, list, st));
+  }
+  cudaFree(d_c);
+  cudaFree(d_ms);
+  cudaFree(d_st);
+  int ns[MAXG];
+  int nns = split_counts(g->G, pow2, ns);
+  std::vector<int32_t> so;
+  std::vector<uint8_t> sd, sn;
+  for (int32_t op : list)
+    for (int dim = 0; dim < 2; dim++) {
+      if (!(g->split_mask_h[op] & (1u << dim))) continue;
+      for (int q = 0; q < nns; q++) {
+        so.push_back(op);
+        sd.push_back((uint8_t)dim);
+        sn.push_back((uint8_t)ns[q]);
+      }
+    }
+  S.n_split = (int64_t)so.size();
+  CK(cudaMalloc(&S.split_op, sizeof(int32_t) * (so.size() + 1)));
+  CK(cudaMalloc(&S.split_dim, so.size() + 1));
+  CK(cudaMalloc(&S.split_n, so.size() + 1));
+  if (!so.empty()) {
+    CK(cudaMemcpy(S.split_op, so.data(), sizeof(int32_t) * so.size(), cudaMemcpyHostToDevice));
+    CK(cudaMemcpy(S.split_dim, sd.data(), sd.size(), cudaMemcpyHostToDevice));
+    CK(cudaMemcpy(S.split_n, sn.data(), sn.size(), cudaMemcpyHostToDevice));
+  }
+  std::vector<int32_t> live(g->V);
+  for (int32_t i = 0; i < g->V; i++) live[i] = i;
+  S.n_live = g->V;
+  CK(cudaMalloc(&S.live, sizeof(int32_t) * (g->V + 1)));
+  if (g->V) CK(cudaMemcpy(S.live, live.data(), sizeof(int32_t) * g->V, cudaMemcpyHostToDevice));
+  S.valid = true;
+  return FASTT_OK;
+}
+
+static StreamState stream_state(const fastt_graph *g, const StreamCache &S, const fastt_gen_params *gp) {
+  StreamState s;
+  s.base_place = S.base_place;
+  s.live = S.live;
+  s.n_live = S.n_live;
+  s.n_split = S.n_split;
+  s.split_op = S.split_op;
+  s.split_dim = S.split_dim;
+  s.split_n = S.split_n;
+  s.seed = gp->seed;
+  s.kmin = gp->pin_k_min;
+  s.kmax = gp->pin_k_max;
+  s.G = g->G;
+  return s;
+}
+
+static fastt_status check_gen(const fastt_graph *g, const StreamCache &S, const fastt_gen_params *gp, int64_t first,
+                              int64_t n, int64_t stride) {
+  if (!gp) return fail(FASTT_EINVAL, "gen params are NULL");
+  if (gp->pin_k_min < 1 || gp->pin_k_max > 4 || gp->pin_k_min > gp->pin_k_max)
+    return fail(FASTT_EINVAL, "need 1 <= pin_k_min <= pin_k_max <= 4");
+  if (first < 0 || n < 0 || stride < 1) return fail(FASTT_EINVAL, "need first >= 0, n >= 0, stride >= 1");
+  if (n > 0 && (g->G == 1 || S.n_live == 0) && first + (n - 1) * stride > S.n_split)
+    return fail(FASTT_EINVAL, "the stream has no PIN candidates (G == 1 or no ops)");
+  return FASTT_OK;
+}
+
+// =================================================================== ABI
+
+extern "C" {
+
+const char *fastt_last_error(void) { return g_err.c_str(); }
+const char *fastt_version(void) { return "fastt-b200 0.1 (sm_100a)"; }
+
+fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_graph **out) {
+  g_err.clear();
+  if (!d || !out) return fail(FASTT_EINVAL, "NULL argument");
+  *out = nullptr;
+  const int32_t V = d->n_ops, G = d->n_devices, K = d->n_link_classes;
+  if (V < 0) return fail(FASTT_EINVAL, "n_ops < 0");
+  if (G < 1 || G > MAXG) return fail(FASTT_EINVAL, "n_devices must be 1..32");
+  if (K < 1 || K > MAXK) return fail(FASTT_EINVAL, "n_link_classes must be 1..16");
+  if (!d->succ_off || !d->dev_mem_cap || !d->link_class || !d->link_alpha_ns || !d->link_beta_fs_per_byte)
+    return fail(FASTT_EINVAL, "NULL array");
+  if (V > 0 && (!d->cost_ns || !d->mem_bytes || !d->param_bytes || !d->split_mask))
+    return fail(FASTT_EINVAL, "NULL per-op array");
+  if (d->succ_off[0] != 0) return fail(FASTT_EINVAL, "succ_off[0] != 0");
+  for (int32_t i = 0; i < V; i++)
+    if (d->succ_off[i + 1] < d->succ_off[i]) return fail(FASTT_EINVAL, "succ_off not monotone at %d", i);
+  const int64_t E = d->succ_off[V];
+  if (E > 0 && (!d->succ_dst || !d->edge_bytes || !d->edge_param)) return fail(FASTT_EINVAL, "NULL edge array");
+  if (d->split_copy_fs_per_byte < 0) return fail(FASTT_EINVAL, "split_copy_fs_per_byte < 0");
+  for (int32_t k = 0; k < K; k++)
+    if (d->link_alpha_ns[k] < 0 || d->link_beta_fs_per_byte[k] < 0) return fail(FASTT_EINVAL, "negative link model");
+  for (int32_t q = 0; q < G * G; q++)
+    if (d->link_class[q] >= K) return fail(FASTT_EINVAL, "link_class out of range");
+  for (int32_t q = 0; q < G; q++)
+    if (d->dev_mem_cap[q] < 0) return fail(FASTT_EINVAL, "negative memory cap");
+  for (int64_t q = 0; q < (int64_t)V * G; q++)
+    if (d->cost_ns[q] < 0) return fail(FASTT_EINVAL, "negative cost");
+  for (int32_t i = 0; i < V; i++)
+    if (d->mem_bytes[i] < 0 || d->param_bytes[i] < 0 || d->param_bytes[i] > d->mem_bytes[i])
+      return fail(FASTT_EINVAL, "need 0 <= param_bytes <= mem_bytes (op %d)", i);
+  // edges: validate, merge parallel edges (R11), sort both adjacency lists
+  struct Ed { int32_t s, t; int64_t b; uint8_t p; };
+  std::vector<Ed> ed;
+  ed.reserve(E);
+  for (int32_t i = 0; i < V; i++)
+    for (int64_t e = d->succ_off[i]; e < d->succ_off[i + 1]; e++) {
+      int32_t t = d->succ_dst[e];
+      if (t < 0 || t >= V) return fail(FASTT_EINVAL, "edge destination out of range");
+      if (t == i) return fail(FASTT_ECYCLE, "self loop at op %d", i);
+      if (d->edge_bytes[e] < 0) return fail(FASTT_EINVAL, "negative edge bytes");
+      ed.push_back({i, t, d->edge_bytes[e], (uint8_t)(d->edge_param[e] ? 1 : 0)});
+    }
+  std::sort(ed.begin(), ed.end(), [](const Ed &a, const Ed &b) { return a.s != b.s ? a.s < b.s : a.t < b.t; });
+  size_t m = 0;
+  for (size_t e = 0; e < ed.size(); e++) {
+    if (m > 0 && ed[m - 1].s == ed[e].s && ed[m - 1].t == ed[e].t) {
+      if (ed[m - 1].b > INT64_MAX / 4 - ed[e].b) return fail(FASTT_ERANGE, "merged edge bytes overflow");
+      ed[m - 1].b += ed[e].b;
+      ed[m - 1].p |= ed[e].p;
+    } else {
+      ed[m++] = ed[e];
+    }
+  }
+  ed.resize(m);
+  const int64_t Em = (int64_t)m;
+  for (auto &x : ed)
+    for (int k = 0; k < K; k++)
+      if (d->link_beta_fs_per_byte[k] && x.b > (INT64_MAX / 4) / d->link_beta_fs_per_byte[k])
+        return fail(FASTT_ERANGE, "bytes * beta overflows int64");
+  std::vector<uint32_t> so(V), sc(V, 0), po(V), pc(V, 0);
+  std::vector<int32_t> sdst(Em), psrc(Em);
+  std::vector<int64_t> sb(Em), pb(Em);
+  std::vector<uint8_t> sp(Em), pp(Em);
+  for (auto &x : ed) sc[x.s]++, pc[x.t]++;
+  {
+    uint32_t a = 0, b = 0;
+    for (int32_t i = 0; i < V; i++) {
+      so[i] = a;
+      a += sc[i];
+      po[i] = b;
+      b += pc[i];
+    }
+  }
+  {
+    std::vector<uint32_t> fs(so), fp(po);
+    for (auto &x : ed) {  // ed sorted by (s, t): succ lists ascending
+      uint32_t q = fs[x.s]++;
+      sdst[q] = x.t;
+      sb[q] = x.b;
+      sp[q] = x.p;
+    }
+    std::vector<Ed> byt(ed);
+    std::sort(byt.begin(), byt.end(), [](const Ed &a, const Ed &b) { return a.t != b.t ? a.t < b.t : a.s < b.s; });
+    for (auto &x : byt) {
+      uint32_t q = fp[x.t]++;
+      psrc[q] = x.s;
+      pb[q] = x.b;
+      pp[q] = x.p;
+    }
+  }
+  int32_t maxdeg = 0, maxP = 0, maxS = 0, maxov = 0;
+  for (int32_t i = 0; i < V; i++) {
+    maxdeg = std::max<int32_t>(maxdeg, (int32_t)std::max(sc[i], pc[i]));
+    if (d->split_mask[i]) {
+      maxov = std::max<int32_t>(maxov, (int32_t)(pc[i] + G + sc[i]));
+      maxP = std::max<int32_t>(maxP, (int32_t)pc[i]);
+      maxS = std::max<int32_t>(maxS, (int32_t)sc[i]);
+    }
+  }
+  if (maxdeg >= 65535) return fail(FASTT_EUNSUP, "an op has >= 65535 neighbours");
+  // Kahn: acyclicity and a topological order
+  std::vector<int32_t> topo;
+  topo.reserve(V);
+  {
+    std::vector<uint32_t> deg(pc);
+    for (int32_t i = 0; i < V; i++)
+      if (deg[i] == 0) topo.push_back(i);
+    for (size_t h = 0; h < topo.size(); h++) {
+      int32_t i = topo[h];
+      for (uint32_t q = so[i]; q < so[i] + sc[i]; q++)
+        if (--deg[sdst[q]] == 0) topo.push_back(sdst[q]);
+    }
+    if ((int32_t)topo.size() != V) return fail(FASTT_ECYCLE, "the graph has a cycle (R22)");
+  }
+  // link-class masks and the int64 guard (same rule as the oracle's loader)
+  GraphConst gc;
+  memset(&gc, 0, sizeof gc);
+  gc.G = G;
+  gc.K = K;
+  gc.copy_fs = d->split_copy_fs_per_byte;
+  for (int q = 0; q < G; q++) gc.cap[q] = d->dev_mem_cap[q];
+  for (int k = 0; k < K; k++) {
+    gc.alpha[k] = d->link_alpha_ns[k];
+    gc.beta[k] = d->link_beta_fs_per_byte[k];
+  }
+  for (int s = 0; s < G; s++)
+    for (int t = 0; t < G; t++) {
+      gc.link_class[s * G + t] = d->link_class[s * G + t];
+      if (s != t) {
+        uint32_t bit = 1u << d->link_class[s * G + t];
+        gc.offdiag_mask |= bit;
+        gc.row_mask[s] |= bit;
+        gc.col_mask[t] |= bit;
+      }
+    }
+  {
+    __int128 tot = 0, totm = 0;
+    for (int32_t i = 0; i < V; i++) {
+      int64_t mx = 0;
+      for (int q = 0; q < G; q++) mx = std::max(mx, d->cost_ns[(int64_t)i * G + q]);
+      tot += mx + G;
+      totm += (__int128)d->mem_bytes[i] * (G + 1);
+    }
+    for (auto &x : ed) {
+      int64_t mx = 0;
+      for (int k = 0; k < K; k++) mx = std::max(mx, comm_class(gc, x.b, k));
+      int64_t cc = gc.copy_fs ? ceil_div64(x.b * gc.copy_fs, 1000000) : 0;
+      tot += (__int128)(mx + cc) * (G + 2);
+    }
+    if (tot >= ((__int128)1 << 58) || totm >= ((__int128)1 << 60))
+      return fail(FASTT_ERANGE, "costs/bytes exceed the int64 envelope");
+  }
+  fastt_graph *g = new (std::nothrow) fastt_graph();
+  if (!g) return fail(FASTT_ENOMEM, "host allocation");
+  g->dev = cuda_device;
+  g->V = V;
+  g->G = G;
+  g->K = K;
+  g->E = Em;
+  g->maxP = maxP;
+  g->maxS = maxS;
+  g->v_max = V + maxov;
+  g->gch = gc;
+  g->split_mask_h.assign(d->split_mask, d->split_mask + V);
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || cuda_device < 0 || cuda_device >= ndev) {
+    delete g;
+    return fail(FASTT_ECUDA, "no CUDA device %d", cuda_device);
+  }
+  Dev guard(cuda_device);
+  int sms = 0;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cuda_device);
+  g->sms = sms > 0 ? sms : 148;
+  const int64_t vcap = (int64_t)V + overlay_v(g);
+  const int64_t ecap = Em + overlay_e(g);
+  if (vcap > 32768) {
+    delete g;
+    return fail(FASTT_EUNSUP, "graphs above 32768 ops (+ split overlay) are not supported yet (V=%d)", V);
+  }
+  Base &B = g->base;
+  B.V = V;
+  B.n_live = V;
+  B.E = Em;
+  B.rl = raw_layout(vcap, ecap, G);
+  // host image of the raw block, one H2D copy
+  std::vector<char> img(B.rl.total, 0);
+  auto put = [&](int k, const void *src, size_t bytes) {
+    if (bytes) memcpy(img.data() + B.rl.o[k], src, bytes);
+  };
+  put(0, so.data(), 4 * (size_t)V);
+  put(1, sc.data(), 4 * (size_t)V);
+  put(2, po.data(), 4 * (size_t)V);
+  put(3, pc.data(), 4 * (size_t)V);
+  put(4, sdst.data(), 4 * (size_t)Em);
+  put(5, psrc.data(), 4 * (size_t)Em);
+  put(6, sb.data(), 8 * (size_t)Em);
+  put(7, pb.data(), 8 * (size_t)Em);
+  put(8, sp.data(), (size_t)Em);
+  put(9, pp.data(), (size_t)Em);
+  put(10, d->cost_ns, 8 * (size_t)V * G);
+  put(11, d->mem_bytes, 8 * (size_t)V);
+  put(12, d->param_bytes, 8 * (size_t)V);
+  put(13, d->split_mask, (size_t)V);
+  {
+    std::vector<uint8_t> alive(V, 1);
+    put(14, alive.data(), (size_t)V);
+  }
+  put(15, topo.data(), 4 * (size_t)V);
+  cudaStream_t st = 0;
+  fastt_status rc = FASTT_OK;
+  do {
+    if (cudaMalloc(&g->gc_dev, sizeof gc) != cudaSuccess || cudaMalloc(&B.raw_block, B.rl.total) != cudaSuccess ||
+        cudaMalloc(&B.raw_dev, sizeof(RawGraph)) != cudaSuccess) {
+      rc = fail(FASTT_ENOMEM, "device allocation for the graph");
+      break;
+    }
+    RawGraph R = raw_struct(B.raw_block, B.rl, V, V, Em);
+    if (cudaMemcpy(g->gc_dev, &gc, sizeof gc, cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemcpy(B.raw_block, img.data(), B.rl.total, cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemcpy(B.raw_dev, &R, sizeof R, cudaMemcpyHostToDevice) != cudaSuccess) {
+      rc = fail(FASTT_ECUDA, "upload: %s", cudaGetErrorString(cudaGetLastError()));
+      break;
+    }
+    rc = prepare_base(g, B, st);
+  } while (0);
+  if (rc != FASTT_OK) {
+    fastt_free_graph(g);
+    return rc;
+  }
+  *out = g;
+  return FASTT_OK;
+}
+
+void fastt_free_graph(fastt_graph *g) {
+  if (!g) return;
+  {
+    Dev guard(g->dev);
+    g->base.release();
+    for (auto &s : g->streams) s.release();
+    cudaFree(g->gc_dev);
+    cudaFree(g->arena);
+    cudaFree(g->tmpl_dev);
+    cudaFree(g->slot_raws_dev);
+    cudaFree(g->slot_pgs_dev);
+    cudaFree(g->slot_cands);
+    cudaFree(g->slot_result);
+    cudaFree(g->slot_index);
+    cudaFree(g->slab);
+    cudaFree(g->wbest);
+    cudaFree(g->best_dev);
+    cudaFree(g->counters);
+    cudaFree(g->defer_q);
+    cudaFree(g->scratch_rank);
+    cudaFree(g->scratch_cp);
+    cudaFree(g->scratch_list);
+    cudaFree(g->scratch_n);
+  }
+  delete g;
+}
+
+fastt_status fastt_graph_info(const fastt_graph *g, int32_t *n_ops, int32_t *v_max, int32_t *cp_len,
+                              int32_t *time_bits) {
+  if (!g) return fail(FASTT_EINVAL, "NULL graph");
+  if (n_ops) *n_ops = g->V;
+  if (v_max) *v_max = g->v_max;
+  if (cp_len) *cp_len = g->base.cp_len;
+  if (time_bits) *time_bits = g->base.tbits;
+  return FASTT_OK;
+}
+
+// host or device candidates -> device array
+static fastt_status upload_cands(const fastt_candidate *cands, int64_t n, uint32_t flags, Cand **d, bool *owned,
+                                 cudaStream_t st) {
+  *owned = false;
+  if (flags & FASTT_F_IN_DEVICE) {
+    *d = (Cand *)cands;
+    return FASTT_OK;
+  }
+  CK(cudaMalloc(d, sizeof(Cand) * (n + 1)));
+  *owned = true;
+  if (n) CK(cudaMemcpyAsync(*d, cands, sizeof(Cand) * n, cudaMemcpyHostToDevice, st));
+  return FASTT_OK;
+}
+
+fastt_status fastt_rank(const fastt_graph *gc_, const fastt_candidate *cand, const fastt_opts *opts,
+                        int64_t *rank_out) {
+  fastt_graph *g = (fastt_graph *)gc_;
+  if (!g || !rank_out) return fail(FASTT_EINVAL, "NULL argument");
+  std::lock_guard<std::mutex> lk(g->mu);
+  Dev guard(g->dev);
+  cudaStream_t st = stream_of(opts);
+  Base &B = g->base;
+  const int64_t vm = g->v_max;
+  std::vector<uint64_t> r(B.rl.vcap, ~0ull);
+  if (!cand || cand->kind == FASTT_KIND_BASE) {
+    if (B.V) CK(cudaMemcpy(r.data(), prep_struct(B.prep_block, B.pl, B.tbits).rank, 8 * (size_t)B.V,
+                           cudaMemcpyDeviceToHost));
+  } else {
+    // validate like the simulator does
+    const Cand &c = *(const Cand *)cand;
+    bool bad = false;
+    if (c.kind == FASTT_KIND_PIN) {
+      if (c.n_pins < 1 || c.n_pins > 4) bad = true;
+      for (int k = 0; k < c.n_pins && !bad; k++) {
+        if (c.pin_op[k] < 0 || c.pin_op[k] >= B.V || c.pin_dev[k] >= g->G) bad = true;
+        for (int k2 = 0; k2 < k; k2++) bad |= c.pin_op[k2] == c.pin_op[k];
+      }
+    } else if (c.kind == FASTT_KIND_SPLIT) {
+      if (c.split_op < 0 || c.split_op >= B.V || c.split_dim > 1 ||
+          !(g->split_mask_h[c.split_op] & (1u << c.split_dim)) || c.split_n < 2 || c.split_n > g->G)
+        bad = true;
+    } else {
+      bad = true;
+    }
+    if (bad) return fail(FASTT_EINVAL, "invalid candidate");
+    TRY(ensure_arena(g, B, st));
+    CK(cudaMemcpyAsync(g->slot_cands, &c, sizeof c, cudaMemcpyHostToDevice, st));
+    launch_slot_setup(g->slot_cands, g->tmpl_dev, B.raw_dev, g->slot_raws_dev, 1, st);
+    launch_copy_block(B.raw_block, g->arena, (int64_t)(g->arena_raw_total + g->arena_prep_total),
+                      (int64_t)B.rl.total, g->slot_cands, 1, st);
+    launch_patch_split(B.raw_dev, g->slot_raws_dev, g->gc_dev, g->slot_cands, 1, st);
+    launch_rank(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, g->slot_cands, 1, g->G, st);
+    CK(cudaGetLastError());
+    RawGraph R;
+    PrepGraph P;
+    CK(cudaMemcpyAsync(&R, g->slot_raws_dev, sizeof R, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&P, g->slot_pgs_dev, sizeof P, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    CK(cudaMemcpy(r.data(), P.rank, 8 * (size_t)R.V, cudaMemcpyDeviceToHost));
+  }
+  std::vector<int64_t> ro(vm);
+  for (int64_t i = 0; i < vm; i++) ro[i] = r[i] == ~0ull ? -1 : (int64_t)r[i];
+  if (flags_of(opts) & FASTT_F_OUT_DEVICE) CK(cudaMemcpy(rank_out, ro.data(), 8 * vm, cudaMemcpyHostToDevice));
+  else memcpy(rank_out, ro.data(), 8 * vm);
+  return FASTT_OK;
+}
+
+fastt_status fastt_schedule_batch(const fastt_graph *gc_, const fastt_candidate *cands, int64_t n,
+                                  const fastt_opts *opts, int64_t *makespan, int64_t *peak_mem, uint8_t *status,
+                                  uint8_t *placement, int32_t *order, int64_t *start_ns) {
+  fastt_graph *g = (fastt_graph *)gc_;
+  if (!g || n < 0 || (n > 0 && (!cands || !makespan || !status))) return fail(FASTT_EINVAL, "bad argument");
+  const uint32_t flags = flags_of(opts);
+  if (flags & FASTT_F_POLICY_INSERT) return fail(FASTT_EUNSUP, "FASTT_F_POLICY_INSERT is not implemented yet");
+  if (n == 0) return FASTT_OK;
+  std::lock_guard<std::mutex> lk(g->mu);
+  Dev guard(g->dev);
+  cudaStream_t st = stream_of(opts);
+  Base &B = g->base;
+  const int64_t vm = g->v_max;
+  const bool outdev = (flags & FASTT_F_OUT_DEVICE) != 0;
+  Cand *d_c;
+  bool own_c;
+  TRY(upload_cands(cands, n, flags, &d_c, &own_c, st));
+  DevOut o;
+  o.vmax = vm;
+  std::vector<void *> tmp;
+  auto dalloc = [&](void *user, size_t bytes, bool need) -> void * {
+    if (!need) return nullptr;
+    if (outdev && user) return user;
+    void *p = nullptr;
+    if (cudaMalloc(&p, bytes) != cudaSuccess) return nullptr;
+    tmp.push_back(p);
+    return p;
+  };
+  o.makespan = (int64_t *)dalloc(makespan, 8 * (size_t)n, true);
+  o.status = (uint8_t *)dalloc(status, (size_t)n, true);
+  o.peak = (int64_t *)dalloc(peak_mem, 8 * (size_t)n * g->G, peak_mem != nullptr);
+  const bool want_sched = placement || order || start_ns;
+  o.place = (uint8_t *)dalloc(placement, (size_t)n * vm, want_sched);
+  o.start = (int64_t *)dalloc(start_ns, 8 * (size_t)n * vm, want_sched);
+  o.deq = (int32_t *)dalloc(nullptr, 4 * (size_t)n * vm, order != nullptr);
+  o.order = (int32_t *)dalloc(order, 4 * (size_t)n * vm, order != nullptr);
+  fastt_status rc = FASTT_OK;
+  if (!o.makespan || !o.status || (peak_mem && !o.peak) || (want_sched && (!o.place || !o.start)) ||
+      (order && (!o.deq || !o.order)))
+    rc = fail(FASTT_ENOMEM, "device output buffers");
+  if (rc == FASTT_OK) rc = eval_batch(g, B, d_c, n, flags, st, o);
+  if (rc == FASTT_OK && !outdev) {
+    auto back = [&](void *h, void *dd, size_t bytes) {
+      if (h && dd && cudaMemcpy(h, dd, bytes, cudaMemcpyDeviceToHost) != cudaSuccess)
+        rc = fail(FASTT_ECUDA, "download");
+    };
+    back(makespan, o.makespan, 8 * (size_t)n);
+    back(status, o.status, (size_t)n);
+    back(peak_mem, o.peak, 8 * (size_t)n * g->G);
+    back(placement, o.place, (size_t)n * vm);
+    back(start_ns, o.start, 8 * (size_t)n * vm);
+    back(order, o.order, 4 * (size_t)n * vm);
+  }
+  for (void *p : tmp) cudaFree(p);
+  if (own_c) cudaFree(d_c);
+  return rc;
+}
+
+fastt_status fastt_stream_info(const fastt_graph *gc_, const fastt_gen_params *gen, const fastt_opts *opts,
+                               int64_t *n_split) {
+  fastt_graph *g = (fastt_graph *)gc_;
+  if (!g || !gen || !n_split) return fail(FASTT_EINVAL, "NULL argument");
+  std::lock_guard<std::mutex> lk(g->mu);
+  Dev guard(g->dev);
+  StreamCache *S;
+  TRY(ensure_stream(g, flags_of(opts), gen->n_pow2_only, stream_of(opts), &S));
+  *n_split = S->n_split;
+  return FASTT_OK;
+}
+
+fastt_status fastt_generate_candidates(const fastt_graph *gc_, const fastt_gen_params *gen, const fastt_opts *opts,
+                                       int64_t first, int64_t n, fastt_candidate *out) {
+  fastt_graph *g = (fastt_graph *)gc_;
+  if (!g || !gen || (n > 0 && !out)) return fail(FASTT_EINVAL, "NULL argument");
+  std::lock_guard<std::mutex> lk(g->mu);
+  Dev guard(g->dev);
+  cudaStream_t st = stream_of(opts);
+  StreamCache *S;
+  TRY(ensure_stream(g, flags_of(opts), gen->n_pow2_only, st, &S));
+  TRY(check_gen(g, *S, gen, first, n, 1));
+  if (n == 0) return FASTT_OK;
+  StreamState ss = stream_state(g, *S, gen);
+  const bool outdev = (flags_of(opts) & FASTT_F_OUT_DEVICE) != 0;
+  Cand *d = (Cand *)out;
+  if (!outdev) CK(cudaMalloc(&d, sizeof(Cand) * n));
+  launch_candgen(ss, first, n, d, st);
+  CK(cudaGetLastError());
+  CK(cudaStreamSynchronize(st));
+  if (!outdev) {
+    CK(cudaMemcpy(out, d, sizeof(Cand) * n, cudaMemcpyDeviceToHost));
+    cudaFree(d);
+  }
+  return FASTT_OK;
+}
+
+fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *gen, const fastt_opts *opts,
+                              int64_t first, int64_t n, int64_t stride, int64_t *best) {
+  fastt_graph *g = (fastt_graph *)gc_;
+  if (!g || !gen || !best) return fail(FASTT_EINVAL, "NULL argument");
+  const uint32_t flags = flags_of(opts);
+  if (flags & FASTT_F_POLICY_INSERT) return fail(FASTT_EUNSUP, "FASTT_F_POLICY_INSERT is not implemented yet");
+  std::lock_guard<std::mutex> lk(g->mu);
+  Dev guard(g->dev);
+  cudaStream_t st = stream_of(opts);
+  StreamCache *S;
+  TRY(ensure_stream(g, flags, gen->n_pow2_only, st, &S));
+  TRY(check_gen(g, *S, gen, first, n, stride));
+  Base &B = g->base;
+  TRY(ensure_sim(g, B, n));
+  const int64_t nwarps = (int64_t)g->sim_grid * (g->sim_block / 32);
+  {
+    std::vector<int64_t> init(2 * nwarps);
+    for (int64_t w = 0; w < nwarps; w++) {
+      init[2 * w] = I64MAX;
+      init[2 * w + 1] = -1;
+    }
+    CK(cudaMemcpyAsync(g->wbest, init.data(), 16 * nwarps, cudaMemcpyHostToDevice, st));
+  }
+  if (n > 0) {
+    CK(cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), st));
+    SimArgs a = sim_args(g, B, flags);
+    a.mode = 0;
+    a.stream = stream_state(g, *S, gen);
+    a.first = first;
+    a.n = n;
+    a.stride = stride;
+    a.track_best = 1;
+    launch_sim(a, B.tbits, g->sim_grid, g->sim_block, g->sim_smem, st);
+    CK(cudaGetLastError());
+    unsigned long long nd = 0;
+    CK(cudaMemcpyAsync(&nd, g->counters + 1, sizeof nd, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (nd > 0) {
+      TRY(ensure_arena(g, B, st));
+      for (int64_t c0 = 0; c0 < (int64_t)nd; c0 += g->arena_slots) {
+        int nc = (int)std::min<int64_t>(g->arena_slots, (int64_t)nd - c0);
+        launch_candgen_idx(a.stream, first, stride, g->defer_q + c0, nc, g->slot_cands, g->slot_index, st);
+        TRY(run_prep(g, B, nc, st));
+        CK(cudaMemsetAsync(g->counters, 0, sizeof(unsigned long long), st));
+        SimArgs b = a;
+        b.slots = g->slot_pgs_dev;
+        b.mode = 2;
+        b.cands = g->slot_cands;
+        b.slot_result = nullptr;
+        b.slot_index = g->slot_index;
+        b.n = nc;
+        launch_sim(b, B.tbits, g->sim_grid, g->sim_block, g->sim_smem, st);
+        CK(cudaGetLastError());
+      }
+    }
+  }
+  launch_argmin(g->wbest, nwarps, g->best_dev, st);
+  CK(cudaGetLastError());
+  if (flags & FASTT_F_OUT_DEVICE) {
+    CK(cudaMemcpyAsync(best, g->best_dev, 16, cudaMemcpyDeviceToDevice, st));
+    CK(cudaStreamSynchronize(st));
+  } else {
+    CK(cudaMemcpyAsync(best, g->best_dev, 16, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+  }
+  return FASTT_OK;
+}
+
+// materialise an accepted split into a new base with room for one more split
+static fastt_status materialize_base(fastt_graph *g, Base &from, const Cand &c, Base &to, cudaStream_t st) {
+  RawGraph Rf = raw_struct(from.raw_block, from.rl, from.V, from.n_live, from.E);
+  (void)Rf;
+  // sizes of the new graph
+  std::vector<uint32_t> cnt(2);
+  uint32_t P = 0, S = 0;
+  {
+    RawGraph R = raw_struct(from.raw_block, from.rl, 0, 0, 0);
+    CK(cudaMemcpy(&P, R.pred_cnt + c.split_op, 4, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(&S, R.succ_cnt + c.split_op, 4, cudaMemcpyDeviceToHost));
+  }
+  to.V = from.V + (int32_t)(P + c.split_n + S);
+  to.n_live = from.n_live - 1 + (int32_t)(P + c.split_n + S);
+  const int64_t newE = from.E + (int64_t)P + (int64_t)P * c.split_n * 2 + (int64_t)S * c.split_n * 2 + S + 16;
+  to.rl = raw_layout((int64_t)to.V + overlay_v(g), newE + overlay_e(g), g->G);
+  if (to.rl.vcap > 32768) return fail(FASTT_EUNSUP, "split search grew the graph above 32768 ops");
+  CK(cudaMalloc(&to.raw_block, to.rl.total));
+  CK(cudaMalloc(&to.raw_dev, sizeof(RawGraph)));
+  CK(cudaMemsetAsync(to.raw_block, 0, to.rl.total, st));
+  // array-wise copy (capacities differ)
+  const int64_t vf = from.rl.vcap, ef = from.rl.ecap;
+  size_t sz[16] = {(size_t)vf * 4, (size_t)vf * 4, (size_t)vf * 4, (size_t)vf * 4, (size_t)ef * 4, (size_t)ef * 4,
+                   (size_t)ef * 8, (size_t)ef * 8, (size_t)ef, (size_t)ef, (size_t)vf * g->G * 8, (size_t)vf * 8,
+                   (size_t)vf * 8, (size_t)vf, (size_t)vf, (size_t)vf * 4};
+  for (int k = 0; k < 16; k++)
+    CK(cudaMemcpyAsync(to.raw_block + to.rl.o[k], from.raw_block + from.rl.o[k], sz[k], cudaMemcpyDeviceToDevice, st));
+  RawGraph Rt = raw_struct(to.raw_block, to.rl, from.V, from.n_live, from.E);
+  CK(cudaMemcpyAsync(to.raw_dev, &Rt, sizeof Rt, cudaMemcpyHostToDevice, st));
+  Cand *d_c;
+  CK(cudaMalloc(&d_c, sizeof c));
+  CK(cudaMemcpyAsync(d_c, &c, sizeof c, cudaMemcpyHostToDevice, st));
+  launch_patch_split(from.raw_dev, to.raw_dev, g->gc_dev, d_c, 1, st);
+  CK(cudaGetLastError());
+  CK(cudaMemcpyAsync(&Rt, to.raw_dev, sizeof Rt, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  cudaFree(d_c);
+  to.E = Rt.E;
+  return prepare_base(g, to, st);
+}
+
+fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, int32_t n_pow2_only,
+                                fastt_split_result *out) {
+  fastt_graph *g = (fastt_graph *)gc_;
+  if (!g || !out) return fail(FASTT_EINVAL, "NULL argument");
+  const uint32_t flags = flags_of(opts) & FASTT_F_CP_PIN;
+  if (flags_of(opts) & FASTT_F_POLICY_INSERT) return fail(FASTT_EUNSUP, "FASTT_F_POLICY_INSERT is not implemented yet");
+  memset(out, 0, sizeof *out);
+  std::lock_guard<std::mutex> lk(g->mu);
+  Dev guard(g->dev);
+  cudaStream_t st = stream_of(opts);
+  std::deque<Base> owned;  // bases created by accepted splits (stable addresses)
+  Base *cur = &g->base;
+  // Alg. 2 line 3: DPOS of the input graph
+  int64_t vm = cur->rl.vcap;
+  const int maxc = 2 * MAXG;
+  Cand *d_c;
+  int64_t *d_ms, *d_start;
+  uint8_t *d_st, *d_place;
+  int32_t *d_deq, *d_order;
+  int64_t cap_v = 32768 + 64;
+  CK(cudaMalloc(&d_c, sizeof(Cand) * maxc));
+  CK(cudaMalloc(&d_ms, 8 * maxc));
+  CK(cudaMalloc(&d_st, maxc));
+  CK(cudaMalloc(&d_place, (size_t)maxc * cap_v));
+  CK(cudaMalloc(&d_start, 8 * (size_t)maxc * cap_v));
+  CK(cudaMalloc(&d_deq, 4 * (size_t)maxc * cap_v));
+  CK(cudaMalloc(&d_order, 4 * (size_t)maxc * cap_v));
+  auto cleanup = [&]() {
+    cudaFree(d_c);
+    cudaFree(d_ms);
+    cudaFree(d_st);
+    cudaFree(d_place);
+    cudaFree(d_start);
+    cudaFree(d_deq);
+    cudaFree(d_order);
+    for (auto &b : owned) b.release();
+    if (g->arena_raw_total != g->base.rl.total) {  // arena was sized for a split-search base
+      cudaFree(g->arena);
+      g->arena = nullptr;
+      g->arena_raw_total = g->arena_prep_total = 0;
+    }
+  };
+  Cand base;
+  memset(&base, 0, sizeof base);
+  base.split_op = -1;
+  for (int k = 0; k < 4; k++) base.pin_op[k] = -1;
+  CK(cudaMemcpy(d_c, &base, sizeof base, cudaMemcpyHostToDevice));
+  DevOut o;
+  o.makespan = d_ms;
+  o.status = d_st;
+  o.place = d_place;
+  o.start = d_start;
+  o.deq = d_deq;
+  o.order = d_order;
+  o.vmax = vm;
+  fastt_status rc = eval_batch(g, *cur, d_c, 1, flags, st, o);
+  if (rc != FASTT_OK) {
+    cleanup();
+    return rc;
+  }
+  int64_t ft_old = 0;
+  uint8_t s0 = 0;
+  CK(cudaMemcpy(&ft_old, d_ms, 8, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(&s0, d_st, 1, cudaMemcpyDeviceToHost));
+  std::vector<uint8_t> bplace(vm);
+  std::vector<int64_t> bstart(vm);
+  std::vector<int32_t> border(vm);
+  CK(cudaMemcpy(bplace.data(), d_place, vm, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(bstart.data(), d_start, 8 * vm, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(border.data(), d_order, 4 * vm, cudaMemcpyDeviceToHost));
+  std::vector<int32_t> sp_op;
+  std::vector<uint8_t> sp_dim, sp_n;
+  int32_t vfinal = g->V;
+  if (s0 == FASTT_CAND_OK) {
+    // Alg. 2 lines 4-5
+    std::vector<int32_t> list;
+    rc = split_list(g, *cur, d_place, list, st);
+    if (rc != FASTT_OK) {
+      cleanup();
+      return rc;
+    }
+    int ns[MAXG];
+    int nns = split_counts(g->G, n_pow2_only, ns);
+    // Alg. 2 lines 7-14
+    for (int32_t op : list) {
+      std::vector<Cand> cs;
+      for (int dim = 0; dim < 2; dim++) {
+        if (!(g->split_mask_h[op] & (1u << dim))) continue;
+        for (int q = 0; q < nns; q++) {
+          Cand c;
+          memset(&c, 0, sizeof c);
+          c.kind = FASTT_KIND_SPLIT;
+          c.split_op = op;
+          c.split_dim = (uint8_t)dim;
+          c.split_n = (uint8_t)ns[q];
+          for (int k = 0; k < 4; k++) c.pin_op[k] = -1;
+          cs.push_back(c);
+        }
+      }
+      if (cs.empty()) continue;
+      CK(cudaMemcpy(d_c, cs.data(), sizeof(Cand) * cs.size(), cudaMemcpyHostToDevice));
+      vm = cur->rl.vcap;
+      o.vmax = vm;
+      rc = eval_batch(g, *cur, d_c, (int64_t)cs.size(), flags, st, o);
+      if (rc != FASTT_OK) {
+        cleanup();
+        return rc;
+      }
+      std::vector<int64_t> ms(cs.size());
+      std::vector<uint8_t> sts(cs.size());
+      CK(cudaMemcpy(ms.data(), d_ms, 8 * cs.size(), cudaMemcpyDeviceToHost));
+      CK(cudaMemcpy(sts.data(), d_st, cs.size(), cudaMemcpyDeviceToHost));
+      int bi = -1;
+      for (size_t q = 0; q < cs.size(); q++)
+        if (sts[q] == FASTT_CAND_OK && (bi < 0 || ms[q] < ms[bi])) bi = (int)q;
+      if (bi < 0 || ms[bi] >= ft_old) break;
+      // accept: Alg. 2 line 10
+      owned.emplace_back();
+      Base &nb = owned.back();
+      rc = materialize_base(g, *cur, cs[bi], nb, st);
+      if (rc != FASTT_OK) {
+        cleanup();
+        return rc;
+      }
+      ft_old = ms[bi];
+      sp_op.push_back(op);
+      sp_dim.push_back(cs[bi].split_dim);
+      sp_n.push_back(cs[bi].split_n);
+      vfinal = nb.V;
+      bplace.resize(vm);
+      bstart.resize(vm);
+      border.resize(vm);
+      CK(cudaMemcpy(bplace.data(), d_place + (size_t)bi * vm, vm, cudaMemcpyDeviceToHost));
+      CK(cudaMemcpy(bstart.data(), d_start + (size_t)bi * vm, 8 * vm, cudaMemcpyDeviceToHost));
+      CK(cudaMemcpy(border.data(), d_order + (size_t)bi * vm, 4 * vm, cudaMemcpyDeviceToHost));
+      cur = &nb;
+    }
+  }
+  out->status = s0;
+  out->makespan = s0 == FASTT_CAND_OK ? ft_old : I64MAX;
+  out->n_splits = (int32_t)sp_op.size();
+  out->op = (int32_t *)malloc(sizeof(int32_t) * (sp_op.size() + 1));
+  out->dim = (uint8_t *)malloc(sp_op.size() + 1);
+  out->n = (uint8_t *)malloc(sp_op.size() + 1);
+  for (size_t q = 0; q < sp_op.size(); q++) {
+    out->op[q] = sp_op[q];
+    out->dim[q] = sp_dim[q];
+    out->n[q] = sp_n[q];
+  }
+  out->n_ops_final = vfinal;
+  out->placement = (uint8_t *)malloc(vfinal + 1);
+  out->order = (int32_t *)malloc(sizeof(int32_t) * (vfinal + 1));
+  out->start_ns = (int64_t *)malloc(sizeof(int64_t) * (vfinal + 1));
+  for (int32_t i = 0; i < vfinal; i++) {
+    out->placement[i] = i < (int32_t)bplace.size() ? bplace[i] : 0xFF;
+    out->start_ns[i] = i < (int32_t)bstart.size() ? bstart[i] : -1;
+    out->order[i] = i < (int32_t)border.size() ? border[i] : -1;
+  }
+  cleanup();
+  return FASTT_OK;
+}
+
+void fastt_free_split_result(fastt_split_result *r) {
+  if (!r) return;
+  free(r->op);
+  free(r->dim);
+  free(r->n);
+  free(r->placement);
+  free(r->order);
+  free(r->start_ns);
+  memset(r, 0, sizeof *r);
+}
+
+}  // extern "C"

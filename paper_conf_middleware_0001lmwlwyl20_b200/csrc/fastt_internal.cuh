@@ -1,0 +1,181 @@
+// fastt_internal.cuh -- device-side data layout of the B200 FastT library.
+//
+// Two graph forms live in HBM:
+//  * RawGraph  -- the problem graph in the caller's id space:
+//    both CSRs with per-op (offset, count) so a split can be patched in place
+//    and appended to (R13), per-edge bytes/param flags, cost/mem tables and a
+//    topological order.  One for the loaded graph; one per SPLIT candidate
+//    slot (materialised SplitOperation, Alg. 2 lines 16-30).
+//  * PrepGraph -- what the schedule simulator reads.  Ops are renumbered by
+//    their priority (rank_u desc, id asc; R2/R3), so a ready set is a bitmap
+//    over positions and "pop max priority" is find-first-set.  Each op has a
+//    128-byte CARD (header + up to 12 predecessor and 12 successor positions)
+//    that one coalesced warp load brings in; costs are a [pos][G] table in
+//    the time type T (uint32 when the schedule bound fits, else uint64).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace fastt {
+
+constexpr int MAXG = 32;
+constexpr int MAXK = 16;
+constexpr int MAXPINS = 4;
+constexpr int CARD_WORDS = 32;
+constexpr int CARD_HDR = 8;
+constexpr int P_IN = 12;  // inline predecessor positions in a card
+constexpr int S_IN = 12;  // inline successor positions in a card
+constexpr uint32_t NONE = 0xFFFFFFFFu;
+constexpr int64_t I64MAX = INT64_MAX;
+
+// card header words
+enum { CW_DEG = 0, CW_PBASE = 1, CW_SBASE = 2, CW_CPIDX = 3, CW_MEMLO = 4, CW_MEMHI = 5, CW_UID = 6, CW_FLAGS = 7 };
+
+struct GraphConst {
+  int32_t G, K;
+  int64_t copy_fs;
+  int64_t cap[MAXG];
+  int64_t alpha[MAXK], beta[MAXK];
+  uint8_t link_class[MAXG * MAXG];
+  uint32_t offdiag_mask;          // classes k with some s != t, class[s][t] == k
+  uint32_t row_mask[MAXG];        // classes in row s (t != s)
+  uint32_t col_mask[MAXG];        // classes in column t (s != t)
+};
+
+struct RawGraph {
+  int32_t V;       // op slots (dead ops included)
+  int32_t n_live;  // live ops
+  int64_t E;       // edge slots per side
+  uint32_t *succ_off, *succ_cnt, *pred_off, *pred_cnt;
+  int32_t *succ_dst, *pred_src;
+  int64_t *succ_bytes, *pred_bytes;
+  uint8_t *succ_param, *pred_param;
+  int64_t *cost;   // V*G
+  int64_t *mem, *param;
+  uint8_t *split_mask, *alive;
+  int32_t *topo;   // n_live, a topological order of the live ops
+};
+
+struct PrepGraph {
+  int32_t n;        // positions (= live ops)
+  int32_t V;        // raw op slots
+  int64_t E;        // live edges
+  int32_t cp_len;   // written by the CP kernel
+  int32_t tbits;    // 32 or 64
+  uint32_t *card;   // n * CARD_WORDS
+  void *costp;      // n * G of T
+  uint32_t *pe_src; // E: predecessor position, grouped by consumer position
+  void *pe_comm;    // E * K of T: comm(bytes, k) of that edge per link class
+  uint32_t *se_dst; // E: successor position, grouped by producer position
+  uint32_t *se_pe;  // E: index of the same edge in pe_*
+  uint32_t *npred;  // n
+  uint32_t *srcbits;// ceil(n/32): positions with no predecessor
+  uint32_t *pos;    // V: uid -> position (NONE for dead)
+  uint32_t *uid;    // n: position -> uid
+  uint64_t *rank;   // V: rank_u by uid (~0 for dead)
+  uint32_t *cp;     // critical path (positions)
+  int64_t *pmem;    // cp prefix sums of mem, cp_len+1
+  int64_t *pcost;   // cp prefix sums of cost, (cp_len+1)*G
+  // scratch for the sort / scans
+  uint64_t *key0, *key1;
+  uint32_t *val0, *val1;
+};
+
+// the candidate record of the ABI (32 bytes)
+struct Cand {
+  uint8_t kind, n_pins, split_dim, split_n;
+  int32_t split_op;
+  int32_t pin_op[4];
+  uint8_t pin_dev[4];
+  uint8_t pad[4];
+};
+static_assert(sizeof(Cand) == 32, "candidate record is 32 bytes");
+
+// the sweep's candidate stream (R21)
+struct StreamState {
+  uint8_t *base_place;  // V
+  int32_t *live;        // n_live uids
+  int32_t n_live;
+  int64_t n_split;
+  int32_t *split_op;    // n_split
+  uint8_t *split_dim, *split_n;
+  uint64_t seed;
+  int32_t kmin, kmax;
+  int32_t G;
+};
+
+__host__ __device__ inline int64_t comm_class(const GraphConst &c, int64_t bytes, int k) {
+  int64_t num = bytes * c.beta[k];
+  return c.alpha[k] + (num + 999999) / 1000000;
+}
+__host__ __device__ inline int64_t ceil_div64(int64_t a, int64_t b) { return (a + b - 1) / b; }
+__host__ __device__ inline int64_t part_bytes(int64_t b, int n, int k) { return b / n + (k < b % n ? 1 : 0); }
+
+// ------------------------------------------------------------ launchers
+// (defined in k_prep.cu / k_sim.cu; all asynchronous on `st`)
+
+void launch_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, const Cand *cands, int nslots,
+                 int G, cudaStream_t st);
+void launch_sort(PrepGraph *pgs, const RawGraph *raws, int nslots, int key_bits, int max_n, cudaStream_t st);
+void launch_cards(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, int nslots, int max_n, int G, int K,
+                  int tbits, cudaStream_t st);
+void launch_cp(PrepGraph *pgs, int nslots, int G, int tbits, cudaStream_t st);
+void launch_copy_block(const void *src, void *dst, int64_t slot_stride_bytes, int64_t bytes, const Cand *cands,
+                       int nslots, cudaStream_t st);
+void launch_patch_split(const RawGraph *base, RawGraph *raws, const GraphConst *gc, const Cand *cands, int nslots,
+                        cudaStream_t st);
+void launch_bound(const RawGraph *raw, const GraphConst *gc, int G, unsigned long long *out /* [2] */,
+                  cudaStream_t st);
+void launch_splitlist(const RawGraph *raw, const GraphConst *gc, const uint8_t *place, int32_t *list,
+                      int32_t *nlist, int64_t *scratch_rank, int32_t *scratch_cp, int G, cudaStream_t st);
+
+struct SimOut {
+  int64_t *makespan;   // per result index
+  uint8_t *status;
+  int64_t *peak;       // per result * G (nullable)
+  uint8_t *place;      // per result * vmax (nullable)
+  int64_t *start;      // per result * vmax (nullable)
+  int32_t *deq;        // per result * vmax (nullable): uids in dequeue order
+  int32_t vmax;
+};
+
+struct SimArgs {
+  int mode;              // 0 sweep, 1 list, 2 prepared slots
+  uint32_t flags;
+  const PrepGraph *base; // base prepared graph (modes 0, 1)
+  const PrepGraph *slots;// prepared slot graphs (mode 2)
+  const Cand *cands;     // mode 1: candidate list; mode 2: candidate per slot
+  const int64_t *slot_result; // mode 2: result index per slot
+  const int64_t *slot_index;  // mode 2: stream index per slot (sweep bests)
+  const GraphConst *gc;
+  const uint8_t *split_mask; // raw split masks of the base graph (validation)
+  StreamState stream;    // mode 0
+  int64_t first, n, stride;
+  unsigned long long *counter;  // work counter
+  int64_t *defer_q;      // deferred work items (q)
+  unsigned long long *ndefer;
+  int64_t *wbest;        // per-warp (makespan, index) pairs, 2 per warp
+  SimOut out;
+  void *slab;            // per-warp state slabs
+  int64_t slab_stride;   // elements (records) per warp
+  int32_t leaf_words;    // bitmap words per warp in smem
+  int32_t G;
+  int32_t track_best;
+};
+
+void launch_sim(const SimArgs &a, int tbits, int grid, int block, size_t smem, cudaStream_t st);
+void launch_argmin(const int64_t *wbest, int64_t nwarps, int64_t *best_dev, cudaStream_t st);
+void launch_order_chunk(const int32_t *deq, const int64_t *start, int32_t *order, const int64_t *results, int64_t n,
+                        int64_t vmax, int key_bits, uint64_t *k0, uint64_t *k1, uint32_t *v0, uint32_t *v1,
+                        cudaStream_t st);
+void launch_candgen(const StreamState &s, int64_t first, int64_t n, Cand *out, cudaStream_t st);
+void launch_candgen_idx(const StreamState &s, int64_t first, int64_t stride, const int64_t *qlist, int64_t n,
+                        Cand *out, int64_t *out_index, cudaStream_t st);
+void launch_slot_setup(const Cand *cands, const RawGraph *tmpl, const RawGraph *base, RawGraph *raws, int nslots,
+                       cudaStream_t st);
+void launch_gather_cands(const Cand *src, const int64_t *idx, int64_t n, Cand *dst, int64_t *res, cudaStream_t st);
+int sim_occupancy(int tbits, int block, size_t smem);
+cudaError_t sim_set_smem(int tbits, size_t smem);
+void launch_fill_i64(int64_t *p, int64_t n, int64_t v, cudaStream_t st);
+
+}  // namespace fastt

