@@ -75,7 +75,8 @@ enum {
   FASTT_F_CP_PIN = 1u << 0,        /* pin critical-path ops to CP devices (Alg. 1 lines 4-5, 9-10) */
   FASTT_F_POLICY_INSERT = 1u << 1, /* insertion-based avail[j]; NOT YET SUPPORTED -> EUNSUP */
   FASTT_F_OUT_DEVICE = 1u << 2,    /* output pointers are device pointers */
-  FASTT_F_IN_DEVICE = 1u << 3      /* candidate input pointer is a device pointer */
+  FASTT_F_IN_DEVICE = 1u << 3,     /* candidate input pointer is a device pointer */
+  FASTT_F_TIMING = 1u << 4         /* record CUDA events around the kernels of this call (fastt_last_timing) */
 };
 
 /* The problem input of P:321-328.  Edges are a CSR by source: the edges of
@@ -142,8 +143,10 @@ typedef struct {
 /* Load + encode: validates (acyclic, ranges), merges
  * parallel edges, builds both CSRs, computes the device-side base ranks and
  * priority order.  Supported envelope: G <= 32, K <= 16, in/out degree
- * < 65536, V + overlay <= 2^24 ops (EUNSUP beyond); int64 bound
- * sum_i(max cost + max in-edge comm) * (G+2) < 2^58 (ERANGE beyond).
+ * < 65535, V + largest split overlay <= 32768 ops (EUNSUP beyond: the ready
+ * set bitmap of one candidate lives in shared memory); int64 guard
+ * sum_i (max cost + G) + sum_e (max comm + copy cost) * (G+2) < 2^58 and
+ * sum_i mem * (G+1) < 2^60 (ERANGE beyond; the oracle applies the same rule).
  * cuda_device: the CUDA device ordinal to use. */
 fastt_status fastt_load_graph(const fastt_graph_desc *desc, int cuda_device, fastt_graph **out);
 void fastt_free_graph(fastt_graph *g);
@@ -199,6 +202,21 @@ typedef struct {
 fastt_status fastt_split_search(const fastt_graph *g, const fastt_opts *opts, int32_t n_pow2_only,
                                 fastt_split_result *out);
 void fastt_free_split_result(fastt_split_result *r);
+
+/* Instrumentation of the last fastt_schedule_batch / fastt_sweep_best call on
+ * this graph.  launches: kernels the library launched (always counted).
+ * The *_ms fields are CUDA-event times on the call's stream, filled only when
+ * that call had FASTT_F_TIMING: ms_sim = the main simulation kernel (S2-S7 for
+ * the candidates whose ranks equal the base ranks), ms_prep = the
+ * per-candidate preparation pipeline plus its simulation launches, ms_total =
+ * the whole call on the device. */
+typedef struct {
+  int64_t launches;
+  int64_t candidates;   /* candidates evaluated */
+  int64_t deferred;     /* of which went through the preparation pipeline */
+  float ms_sim, ms_prep, ms_total;
+} fastt_timing;
+fastt_status fastt_last_timing(const fastt_graph *g, fastt_timing *out);
 
 const char *fastt_last_error(void); /* thread-local; valid until the next call on this thread */
 const char *fastt_version(void);

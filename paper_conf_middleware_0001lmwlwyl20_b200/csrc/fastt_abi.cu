@@ -108,7 +108,7 @@ static PrepLayout prep_layout(int64_t ncap, int64_t ecap, int G, int K, int tbyt
   size_t sz[19] = {(size_t)ncap * CARD_WORDS * 4,        // card
                    (size_t)ncap * G * tbytes,           // costp
                    (size_t)ecap * 4,                    // pe_src
-                   (size_t)ecap * K * tbytes,           // pe_comm
+                   (size_t)(ecap + 64) * K * tbytes,    // pe_comm (+ padding for speculative reads)
                    (size_t)ecap * 4, (size_t)ecap * 4,  // se_dst, se_pe
                    (size_t)ncap * 4,                    // npred
                    (size_t)(ncap / 32 + 2) * 4,         // srcbits
@@ -231,8 +231,44 @@ struct fastt_graph {
   // misc scratch
   int64_t *scratch_rank = nullptr;
   int32_t *scratch_cp = nullptr, *scratch_list = nullptr, *scratch_n = nullptr;
+  // instrumentation
+  int64_t launches = 0;
+  fastt_timing last;
+  cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
   std::mutex mu;
 };
+
+// kernels each launcher issues (for the launch count of fastt_last_timing)
+enum { NL_SIM = 1, NL_PREP = 8, NL_ARGMIN = 1, NL_GATHER = 1, NL_CANDGEN = 1, NL_ORDER = 1, NL_FILL = 1 };
+
+static fastt_status timing_begin(fastt_graph *g, uint32_t flags, cudaStream_t st) {
+  g->launches = 0;
+  memset(&g->last, 0, sizeof g->last);
+  if (!(flags & FASTT_F_TIMING)) return FASTT_OK;
+  for (auto &e : g->ev)
+    if (!e) CK(cudaEventCreate(&e));
+  CK(cudaEventRecord(g->ev[0], st));
+  return FASTT_OK;
+}
+static void timing_mark(fastt_graph *g, uint32_t flags, int k, cudaStream_t st) {
+  if (flags & FASTT_F_TIMING) cudaEventRecord(g->ev[k], st);
+}
+static fastt_status timing_end(fastt_graph *g, uint32_t flags, cudaStream_t st, int64_t cands, int64_t deferred) {
+  g->last.launches = g->launches;
+  g->last.candidates = cands;
+  g->last.deferred = deferred;
+  if (!(flags & FASTT_F_TIMING)) return FASTT_OK;
+  CK(cudaEventRecord(g->ev[3], st));
+  CK(cudaEventSynchronize(g->ev[3]));
+  float a = 0, b = 0, c = 0;
+  CK(cudaEventElapsedTime(&a, g->ev[0], g->ev[1]));
+  CK(cudaEventElapsedTime(&b, g->ev[1], g->ev[2]));
+  CK(cudaEventElapsedTime(&c, g->ev[0], g->ev[3]));
+  g->last.ms_sim = a;
+  g->last.ms_prep = b;
+  g->last.ms_total = c;
+  return FASTT_OK;
+}
 
 static int64_t overlay_v(const fastt_graph *g) { return (int64_t)g->maxP + g->G + g->maxS + 1; }
 static int64_t overlay_e(const fastt_graph *g) {
@@ -311,8 +347,10 @@ static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st)
   size_t freeb = 0, totb = 0;
   CK(cudaMemGetInfo(&freeb, &totb));
   size_t per = rt + pt;
-  int64_t slots = (int64_t)(freeb / 4 / per);
-  if (slots > 512) slots = 512;
+  // up to 8192 slots within 40% of free HBM: a C5 sweep's ~4k split
+  // candidates then prepare in one wave instead of many sequential chunks
+  int64_t slots = (int64_t)(freeb * 2 / 5 / per);
+  if (slots > 8192) slots = 8192;
   if (slots < 1) return fail(FASTT_ENOMEM, "device memory too small for one preparation slot (%zu bytes)", per);
   g->arena_slots = (int)slots;
   CK(cudaMalloc(&g->arena, per * slots));
@@ -346,8 +384,10 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     g->wbest = nullptr;
     int leaf = (int)((ncap + 31) / 32);
     size_t smem = (size_t)(g->sim_block / 32) * (leaf + 32) * 4;
-    if (smem > 48 * 1024) CK(sim_set_smem(B.tbits, smem));
-    int per_sm = sim_occupancy(B.tbits, g->sim_block, smem);
+    int gsh = 0;
+    while ((1 << gsh) < g->G) gsh++;
+    if (smem > 48 * 1024) CK(sim_set_smem(B.tbits, gsh, smem));
+    int per_sm = sim_occupancy(B.tbits, gsh, g->sim_block, smem);
     if (per_sm < 1) return fail(FASTT_EUNSUP, "simulation kernel does not fit on an SM (smem %zu)", smem);
     g->sim_grid = g->sms * per_sm;
     g->sim_smem = smem;
@@ -387,6 +427,10 @@ static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
   a.slab_stride = g->sim_ncap;
   a.leaf_words = (int32_t)((g->sim_ncap + 31) / 32);
   a.G = g->G;
+  while ((1 << a.gshift) < g->G) a.gshift++;
+  for (int d = 0; d < g->G; d++)
+    if (g->gch.cap[d] != I64MAX) a.cap_check = 1;
+  a.need_mem = a.cap_check;
   return a;
 }
 
@@ -394,6 +438,7 @@ static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
 // (SURVEY 8(a) S3 + S4 + S5 per candidate): materialise splits, ranks with
 // the candidate's allowed sets, priority sort, cards, critical path.
 static fastt_status run_prep(fastt_graph *g, const Base &B, int nslots, cudaStream_t st) {
+  g->launches += NL_PREP;
   launch_slot_setup(g->slot_cands, g->tmpl_dev, B.raw_dev, g->slot_raws_dev, nslots, st);
   launch_copy_block(B.raw_block, g->arena, (int64_t)(g->arena_raw_total + g->arena_prep_total), (int64_t)B.rl.total,
                     g->slot_cands, nslots, st);
@@ -423,7 +468,10 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
   if (n <= 0) return FASTT_OK;
   TRY(ensure_sim(g, B, n));
   if (o.place) CK(cudaMemsetAsync(o.place, 0xFF, (size_t)n * o.vmax, st));
-  if (o.start) launch_fill_i64(o.start, n * o.vmax, -1, st);
+  if (o.start) {
+    launch_fill_i64(o.start, n * o.vmax, -1, st);
+    g->launches += NL_FILL;
+  }
   if (o.deq) CK(cudaMemsetAsync(o.deq, 0xFF, (size_t)n * o.vmax * 4, st));
   CK(cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), st));
   SimArgs a = sim_args(g, B, flags);
@@ -433,12 +481,15 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
   a.out.makespan = o.makespan;
   a.out.status = o.status;
   a.out.peak = o.peak;
+  if (o.peak) a.need_mem = 1;
   a.out.place = o.place;
   a.out.start = o.start;
   a.out.deq = o.deq;
   a.out.vmax = (int32_t)o.vmax;
   launch_sim(a, B.tbits, g->sim_grid, g->sim_block, g->sim_smem, st);
+  g->launches += NL_SIM;
   CK(cudaGetLastError());
+  timing_mark(g, flags, 1, st);
   unsigned long long nd = 0;
   CK(cudaMemcpyAsync(&nd, g->counters + 1, sizeof nd, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
@@ -447,6 +498,7 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
     for (int64_t c0 = 0; c0 < (int64_t)nd; c0 += g->arena_slots) {
       int nc = (int)std::min<int64_t>(g->arena_slots, (int64_t)nd - c0);
       launch_gather_cands(d_cands, g->defer_q + c0, nc, g->slot_cands, g->slot_result, st);
+      g->launches += NL_GATHER + NL_SIM;
       TRY(run_prep(g, B, nc, st));
       CK(cudaMemsetAsync(g->counters, 0, sizeof(unsigned long long), st));
       SimArgs b = a;
@@ -460,6 +512,7 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
       CK(cudaGetLastError());
     }
   }
+  timing_mark(g, flags, 2, st);
   if (o.order) {
     // execution order list A (R17): per-result stable sort of the dequeue list by start
     int64_t chunk = 256;
@@ -477,6 +530,7 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
       for (int64_t k = 0; k < nc; k++) idx[k] = c0 + k;
       CK(cudaMemcpyAsync(d_idx, idx.data(), sizeof(int64_t) * nc, cudaMemcpyHostToDevice, st));
       launch_order_chunk(o.deq, o.start, o.order, d_idx, nc, o.vmax, B.key_bits, k0, k1, v0, v1, st);
+      g->launches += NL_ORDER;
       CK(cudaStreamSynchronize(st));
     }
     cudaFree(k0);
@@ -878,6 +932,8 @@ void fastt_free_graph(fastt_graph *g) {
     cudaFree(g->scratch_cp);
     cudaFree(g->scratch_list);
     cudaFree(g->scratch_n);
+    for (auto &e : g->ev)
+      if (e) cudaEventDestroy(e);
   }
   delete g;
 }
@@ -999,7 +1055,10 @@ fastt_status fastt_schedule_batch(const fastt_graph *gc_, const fastt_candidate 
   if (!o.makespan || !o.status || (peak_mem && !o.peak) || (want_sched && (!o.place || !o.start)) ||
       (order && (!o.deq || !o.order)))
     rc = fail(FASTT_ENOMEM, "device output buffers");
+  unsigned long long nd0 = 0;
+  if (rc == FASTT_OK) rc = timing_begin(g, flags, st);
   if (rc == FASTT_OK) rc = eval_batch(g, B, d_c, n, flags, st, o);
+  if (rc == FASTT_OK) cudaMemcpy(&nd0, g->counters + 1, sizeof nd0, cudaMemcpyDeviceToHost);
   if (rc == FASTT_OK && !outdev) {
     auto back = [&](void *h, void *dd, size_t bytes) {
       if (h && dd && cudaMemcpy(h, dd, bytes, cudaMemcpyDeviceToHost) != cudaSuccess)
@@ -1012,6 +1071,7 @@ fastt_status fastt_schedule_batch(const fastt_graph *gc_, const fastt_candidate 
     back(start_ns, o.start, 8 * (size_t)n * vm);
     back(order, o.order, 4 * (size_t)n * vm);
   }
+  if (rc == FASTT_OK) rc = timing_end(g, flags, st, n, (int64_t)nd0);
   for (void *p : tmp) cudaFree(p);
   if (own_c) cudaFree(d_c);
   return rc;
@@ -1077,6 +1137,8 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
     }
     CK(cudaMemcpyAsync(g->wbest, init.data(), 16 * nwarps, cudaMemcpyHostToDevice, st));
   }
+  TRY(timing_begin(g, flags, st));
+  unsigned long long nd = 0;
   if (n > 0) {
     CK(cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), st));
     SimArgs a = sim_args(g, B, flags);
@@ -1087,8 +1149,9 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
     a.stride = stride;
     a.track_best = 1;
     launch_sim(a, B.tbits, g->sim_grid, g->sim_block, g->sim_smem, st);
+    g->launches += NL_SIM;
     CK(cudaGetLastError());
-    unsigned long long nd = 0;
+    timing_mark(g, flags, 1, st);
     CK(cudaMemcpyAsync(&nd, g->counters + 1, sizeof nd, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     if (nd > 0) {
@@ -1096,6 +1159,7 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
       for (int64_t c0 = 0; c0 < (int64_t)nd; c0 += g->arena_slots) {
         int nc = (int)std::min<int64_t>(g->arena_slots, (int64_t)nd - c0);
         launch_candgen_idx(a.stream, first, stride, g->defer_q + c0, nc, g->slot_cands, g->slot_index, st);
+        g->launches += NL_CANDGEN + NL_SIM;
         TRY(run_prep(g, B, nc, st));
         CK(cudaMemsetAsync(g->counters, 0, sizeof(unsigned long long), st));
         SimArgs b = a;
@@ -1110,15 +1174,18 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
       }
     }
   }
+  else timing_mark(g, flags, 1, st);
+  timing_mark(g, flags, 2, st);
   launch_argmin(g->wbest, nwarps, g->best_dev, st);
+  g->launches += NL_ARGMIN;
   CK(cudaGetLastError());
   if (flags & FASTT_F_OUT_DEVICE) {
     CK(cudaMemcpyAsync(best, g->best_dev, 16, cudaMemcpyDeviceToDevice, st));
-    CK(cudaStreamSynchronize(st));
   } else {
     CK(cudaMemcpyAsync(best, g->best_dev, 16, cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
   }
+  TRY(timing_end(g, flags, st, n, (int64_t)nd));
+  CK(cudaStreamSynchronize(st));
   return FASTT_OK;
 }
 
@@ -1322,6 +1389,12 @@ fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, 
     out->order[i] = i < (int32_t)border.size() ? border[i] : -1;
   }
   cleanup();
+  return FASTT_OK;
+}
+
+fastt_status fastt_last_timing(const fastt_graph *g, fastt_timing *out) {
+  if (!g || !out) return fail(FASTT_EINVAL, "NULL argument");
+  *out = g->last;
   return FASTT_OK;
 }
 

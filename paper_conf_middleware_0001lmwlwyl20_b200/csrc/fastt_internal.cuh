@@ -160,7 +160,10 @@ struct SimArgs {
   int64_t slab_stride;   // elements (records) per warp
   int32_t leaf_words;    // bitmap words per warp in smem
   int32_t G;
+  int32_t gshift;        // ceil(log2(G)): lanes per predecessor group = 1 << gshift
   int32_t track_best;
+  int32_t need_mem;      // track per-device memory (caps present or peak output)
+  int32_t cap_check;     // some device has a finite memory cap (R8)
 };
 
 void launch_sim(const SimArgs &a, int tbits, int grid, int block, size_t smem, cudaStream_t st);
@@ -174,8 +177,8 @@ void launch_candgen_idx(const StreamState &s, int64_t first, int64_t stride, con
 void launch_slot_setup(const Cand *cands, const RawGraph *tmpl, const RawGraph *base, RawGraph *raws, int nslots,
                        cudaStream_t st);
 void launch_gather_cands(const Cand *src, const int64_t *idx, int64_t n, Cand *dst, int64_t *res, cudaStream_t st);
-int sim_occupancy(int tbits, int block, size_t smem);
-cudaError_t sim_set_smem(int tbits, size_t smem);
+int sim_occupancy(int tbits, int gshift, int block, size_t smem);
+cudaError_t sim_set_smem(int tbits, int gshift, size_t smem);
 void launch_fill_i64(int64_t *p, int64_t n, int64_t v, cudaStream_t st);
 
 }  // namespace fastt

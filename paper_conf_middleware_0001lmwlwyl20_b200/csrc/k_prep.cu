@@ -495,6 +495,9 @@ __global__ void k_cards_edges(const RawGraph *raws, PrepGraph *pgs, const GraphC
       P.se_pe[sb + j] = P.card[(int64_t)dp * CARD_WORDS + CW_PBASE] + q;
       if (j < S_IN) c[CARD_HDR + P_IN + j] = dp;
     }
+    // unused inline slots hold position 0 so the simulator may load them speculatively
+    if (lane >= np_ && lane < P_IN) c[CARD_HDR + lane] = 0;
+    if (lane >= ns_ && lane < S_IN) c[CARD_HDR + P_IN + lane] = 0;
   }
   (void)max_n;
 }

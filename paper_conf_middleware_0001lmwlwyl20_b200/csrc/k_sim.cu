@@ -176,33 +176,394 @@ __device__ __forceinline__ bool lt_cross(uint64_t a, uint64_t mb, uint64_t b, ui
   return h1 < h2 || (h1 == h2 && l1 < l2);
 }
 
+
+// A PIN candidate keeps the base ranks iff w of each pinned op and
+// c of every edge touching one are unchanged under R5's allowed
+// sets; otherwise it is deferred to the per-candidate preparation pipeline.
 template <typename T>
-__global__ void __launch_bounds__(256, 4) k_sim(SimArgs a) {
+__device__ __noinline__ bool pin_changes_ranks(const PrepGraph *pg, const GraphConst &gc, const Cand &c, int np,
+                                               uint32_t i, int di, int G, int K) {
+  const T *costp = (const T *)pg->costp;
+  const T *pe_comm = (const T *)pg->pe_comm;
+  const uint32_t *posm = pg->pos;
+  bool changed = false;
+  T wmax = 0;
+  for (int d = 0; d < G; d++) {
+    T v = costp[(int64_t)i * G + d];
+    wmax = v > wmax ? v : wmax;
+  }
+  changed |= costp[(int64_t)i * G + di] != wmax;
+  const uint32_t *ci = pg->card + (int64_t)i * CARD_WORDS;
+  uint32_t deg = ci[CW_DEG], pb = ci[CW_PBASE], sbb = ci[CW_SBASE];
+  for (uint32_t j = 0; j < (deg & 0xFFFF) && !changed; j++) {
+    uint32_t e = pb + j, o = pg->pe_src[e];
+    int po = -1;
+    for (int k = 0; k < np; k++)
+      if (posm[c.pin_op[k]] == o) po = c.pin_dev[k];
+    const T *pc = pe_comm + (int64_t)e * K;
+    changed |= c_allowed_t<T>(gc, pc, -1, -1) != c_allowed_t<T>(gc, pc, po, di);
+  }
+  for (uint32_t j = 0; j < (deg >> 16) && !changed; j++) {
+    uint32_t o = pg->se_dst[sbb + j], e = pg->se_pe[sbb + j];
+    int po = -1;
+    for (int k = 0; k < np; k++)
+      if (posm[c.pin_op[k]] == o) po = c.pin_dev[k];
+    const T *pc = pe_comm + (int64_t)e * K;
+    changed |= c_allowed_t<T>(gc, pc, -1, -1) != c_allowed_t<T>(gc, pc, di, po);
+  }
+  return changed;
+}
+
+// CP devices (Alg. 1 line 5, R9): repeatedly give the
+// device with the smallest exact average cost the longest prefix of the
+// remaining free CP ops that fits its memory; perturbation-pinned CP ops are
+// excluded (free-index space).  Lane r < nrounds receives round r.
+template <typename T>
+__device__ __noinline__ void cp_rounds(const PrepGraph *pg, int np, uint32_t my_pos, int lane, int dl, int G,
+                                       int64_t cap_d, uint32_t &r_lo, uint32_t &r_hi, int &r_dev, int &nrounds,
+                                       uint32_t &my_pcp, int64_t &reserved) {
+  const uint32_t *card = pg->card;
+  const T *costp = (const T *)pg->costp;
+  const int32_t L = pg->cp_len;
+  int64_t my_pmem = 0;
+  if (lane < np) {
+    const uint32_t *ci = card + (int64_t)my_pos * CARD_WORDS;
+    my_pcp = ci[CW_CPIDX];
+    my_pmem = (int64_t)(((uint64_t)ci[CW_MEMHI] << 32) | ci[CW_MEMLO]);
+  }
+  // pinned CP indices sorted ascending (uniform registers)
+  uint32_t pcs[MAXPINS];
+  int64_t pms[MAXPINS];
+  int64_t pcd[MAXPINS];  // cost on this lane's device
+  bool oncp = lane < np && my_pcp != NONE;
+  unsigned oncp_m = __ballot_sync(FULL, oncp);
+  int my_rank = 0;
+  for (int k = 0; k < np; k++) {
+    uint32_t ok_ = __shfl_sync(FULL, my_pcp, k);
+    bool okon = (oncp_m >> k) & 1;
+    if (okon && ok_ < my_pcp) my_rank++;
+  }
+  const int m = __popc(oncp_m);
+#pragma unroll
+  for (int j = 0; j < MAXPINS; j++) {
+    unsigned who = __ballot_sync(FULL, oncp && my_rank == j);
+    int src = who ? __ffs(who) - 1 : 0;
+    uint32_t pv = __shfl_sync(FULL, my_pcp, src);
+    int64_t mv = __shfl_sync(FULL, my_pmem, src);
+    uint32_t ppos = __shfl_sync(FULL, my_pos, src);
+    pcs[j] = (j < m) ? pv : NONE;
+    pms[j] = (j < m) ? mv : 0;
+    pcd[j] = (j < m && dl < G) ? (int64_t)costp[(int64_t)ppos * G + dl] : 0;
+  }
+  const int32_t Lf = L - m;
+  auto raw_end = [&](int32_t f) -> int32_t {  // raw index just after the f-th free op (f >= 1)
+    int32_t r = f - 1;
+#pragma unroll
+    for (int j = 0; j < MAXPINS; j++)
+      if (j < m && (int32_t)pcs[j] <= r) r++;
+    return r + 1;
+  };
+  auto fp_mem = [&](int32_t f) -> int64_t {
+    if (f <= 0) return 0;
+    int32_t re = raw_end(f);
+    int64_t v = pg->pmem[re];
+#pragma unroll
+    for (int j = 0; j < MAXPINS; j++)
+      if (j < m && (int32_t)pcs[j] < re) v -= pms[j];
+    return v;
+  };
+  auto fp_cost = [&](int32_t f) -> int64_t {  // for device dl
+    if (f <= 0) return 0;
+    int32_t re = raw_end(f);
+    int64_t v = pg->pcost[(int64_t)re * G + dl];
+#pragma unroll
+    for (int j = 0; j < MAXPINS; j++)
+      if (j < m && (int32_t)pcs[j] < re) v -= pcd[j];
+    return v;
+  };
+  uint32_t devs = G == 32 ? FULL : ((1u << G) - 1);
+  int32_t k = 0;
+  while (k < Lf && devs) {
+    int32_t t = 0;
+    int64_t S = 0;
+    if (lane < G && ((devs >> lane) & 1)) {
+      int64_t bm = fp_mem(k);
+      int64_t tot = fp_mem(Lf) - bm;
+      if (tot <= cap_d) t = Lf - k;
+      else {
+        int32_t lo = 0, hi = Lf - k;
+        while (hi - lo > 1) {
+          int32_t mid = (lo + hi) >> 1;
+          if (fp_mem(k + mid) - bm <= cap_d) lo = mid;
+          else hi = mid;
+        }
+        t = lo;
+      }
+      if (t > 0) S = fp_cost(k + t) - fp_cost(k);
+    }
+    int best = -1;
+    int32_t tb = 0;
+    int64_t Sb = 0;
+    for (int d = 0; d < G; d++) {
+      int32_t td = __shfl_sync(FULL, t, d);
+      int64_t Sd = __shfl_sync(FULL, S, d);
+      if (td > 0 && (best < 0 || lt_cross((uint64_t)Sd, (uint64_t)tb, (uint64_t)Sb, (uint64_t)td))) {
+        best = d;
+        tb = td;
+        Sb = Sd;
+      }
+    }
+    if (best < 0) break;
+    int64_t resv = fp_mem(k + tb) - fp_mem(k);
+    if (lane == nrounds) {
+      r_lo = (uint32_t)k;
+      r_hi = (uint32_t)(k + tb);
+      r_dev = best;
+    }
+    if (dl == best) reserved += resv;
+    devs &= ~(1u << best);
+    k += tb;
+    nrounds++;
+  }
+}
+
+// general predecessor max for ops with more predecessors than one lane pass
+// holds (or beyond the inline card entries): chunks of 32 via pe_src.
+template <typename T, int GSH>
+__device__ __forceinline__ T pred_max_general(const typename Slab<T>::W *slab, const uint32_t *pe_src, const T *pe_comm,
+                                           const GraphConst &gc, uint32_t npred, uint32_t pbase, int lane, int G,
+                                           int K) {
+  constexpr int GP = 1 << GSH, PPP = 32 >> GSH;
+  const int dl = lane & (GP - 1), ql = lane >> GSH;
+  T estp = 0;
+  for (uint32_t pb0 = 0; pb0 < npred; pb0 += 32) {
+    const uint32_t pj = pb0 + lane;
+    T ftv = 0, cm = 0;
+    uint32_t plc = 0;
+    if (pj < npred) {
+      const uint32_t src = __ldg(pe_src + pbase + pj);
+      Slab<T>::load(slab, src, ftv, plc);
+      if (K == 1) cm = __ldg(pe_comm + pbase + pj);
+    }
+    const uint32_t cnt = npred - pb0 < 32 ? npred - pb0 : 32;
+    for (uint32_t q0 = 0; q0 < cnt; q0 += PPP) {
+      const uint32_t qi = q0 + ql;
+      const T f = __shfl_sync(FULL, ftv, qi & 31);
+      const uint32_t pl = __shfl_sync(FULL, plc, qi & 31);
+      T cmm = __shfl_sync(FULL, cm, qi & 31);
+      if (qi < cnt) {
+        if (K > 1 && pl != (uint32_t)dl && dl < G)
+          cmm = __ldg(pe_comm + (size_t)(pbase + pb0 + qi) * K + gc.link_class[pl * G + dl]);
+        const T term = f + ((pl == (uint32_t)dl) ? (T)0 : cmm);
+        estp = term > estp ? term : estp;
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o >= GP; o >>= 1) {
+    T x = __shfl_xor_sync(FULL, estp, o);
+    estp = x > estp ? x : estp;
+  }
+  return estp;
+}
+
+
+struct LoopOut {
+  uint64_t makespan;
+  int64_t used;
+  int32_t infeasible;
+};
+
+// The hot loop of DPOS (Alg. 1 lines 6-22) for one candidate, isolated so
+// its register allocation holds only loop state.
+template <typename T, int GSH, bool MEM>
+__device__ __noinline__ LoopOut sim_loop(uint32_t *leaf, uint32_t *summ, uint32_t top, typename Slab<T>::W *slab,
+                                         const uint32_t *__restrict__ card, const T *__restrict__ costp,
+                                         const T *__restrict__ pe_comm, const PrepGraph *pg, const GraphConst *gcp,
+                                         const int G, const int K, const uint32_t my_pos, const int my_dev,
+                                         const int np, const uint32_t r_lo, const uint32_t r_hi, const int r_dev,
+                                         const int nrounds, const uint32_t my_pcp, const int64_t cap_d,
+                                         int64_t used, int64_t reserved, const bool cap_chk, uint8_t *out_place,
+                                         int64_t *out_start, int32_t *out_deq) {
+  constexpr int GP = 1 << GSH;
+  constexpr int PPP = 32 >> GSH;
+  constexpr int PFAST = PPP < P_IN ? PPP : P_IN;
+  constexpr bool need_mem = MEM;
+  const int lane = threadIdx.x & 31;
+  const int dl = lane & (GP - 1);
+  const int ql = lane >> GSH;
+  const bool want_out = out_place != nullptr;
+  T avail = 0, makespan = 0;
+  int32_t seq = 0;
+  bool infeasible = false;
+  while (top) {
+    // pop: highest priority = lowest position = lowest set bit
+    const int s = __ffs(top) - 1;
+    const uint32_t m = summ[s];
+    const int b = __ffs(m) - 1;
+    const int w = (s << 5) + b;
+    const uint32_t lw = leaf[w];
+    const uint32_t i = ((uint32_t)w << 5) + (__ffs(lw) - 1);
+    const uint32_t nlw = lw & (lw - 1);
+    const uint32_t nm = nlw ? m : (m & (m - 1));
+    __syncwarp();
+    if (lane == 0) {
+      leaf[w] = nlw;
+      summ[s] = nm;
+    }
+    if (!nm) top &= top - 1;
+
+    // round 1: the card (zero-padded inline entries make every slot a
+    // valid index), this lane's predecessor slot, successor slot, cost
+    const uint32_t *cd = card + (size_t)i * CARD_WORDS;
+    const uint4 h0 = __ldg((const uint4 *)cd);  // deg, pbase, sbase, cpidx
+    const uint32_t psrc = __ldg(cd + CARD_HDR + (ql < P_IN ? ql : 0));
+    const uint32_t sdst = __ldg(cd + CARD_HDR + P_IN + (lane < S_IN ? lane : 0));
+    const T cst = __ldg(costp + (size_t)i * G + (dl < G ? dl : 0));
+    // round 2 (speculative): predecessor record, edge comm, successor indegree
+    T ftv;
+    uint32_t plc;
+    Slab<T>::load(slab, psrc, ftv, plc);
+    const uint32_t sdeg = Slab<T>::indeg(slab, sdst);
+    const uint32_t npred = h0.x & 0xFFFF, nsucc = h0.x >> 16;
+    T estp;
+    if (npred <= (uint32_t)PFAST) {
+      T term = 0;
+      if ((uint32_t)ql < npred) {
+        T cm;
+        if (K == 1) cm = __ldg(pe_comm + h0.y + ql);
+        else cm = (plc != (uint32_t)dl && dl < G) ? __ldg(pe_comm + (size_t)(h0.y + ql) * K + gcp->link_class[plc * G + dl]) : (T)0;
+        term = ftv + (plc == (uint32_t)dl ? (T)0 : cm);
+      }
+#pragma unroll
+      for (int o = 16; o >= GP; o >>= 1) {
+        T x = __shfl_xor_sync(FULL, term, o);
+        term = x > term ? x : term;
+      }
+      estp = term;
+    } else {
+      estp = pred_max_general<T, GSH>(slab, pg->pe_src, pe_comm, *gcp, npred, h0.y, lane, G, K);
+    }
+    const T est = estp > avail ? estp : avail;
+    const T eft = est + cst;
+
+    // device forced by a perturbation pin or a CP pin
+    int forced = -1;
+    bool pert = false;
+    if (np) {
+      const unsigned pmk = __ballot_sync(FULL, my_pos == i);
+      if (pmk) {
+        forced = __shfl_sync(FULL, my_dev, __ffs(pmk) - 1);
+        pert = true;
+      }
+    }
+    if (forced < 0 && nrounds > 0 && h0.w != NONE) {
+      const uint32_t fi = h0.w - __popc(__ballot_sync(FULL, lane < np && my_pcp < h0.w));
+      const unsigned rm = __ballot_sync(FULL, lane < nrounds && fi >= r_lo && fi < r_hi);
+      if (rm) forced = __shfl_sync(FULL, r_dev, __ffs(rm) - 1);
+    }
+    int64_t mem = 0;
+    if (need_mem) mem = (int64_t)(((uint64_t)__ldg(cd + CW_MEMHI) << 32) | __ldg(cd + CW_MEMLO));
+    bool feas = lane < G;
+    if (forced >= 0) feas = feas && lane == forced;
+    if (cap_chk && (forced < 0 || pert)) feas = feas && (used + reserved + mem <= cap_d);
+    const T key = feas ? eft : TT<T>::MAXV;
+    const T mn = TT<T>::wmin(key);
+    const unsigned fm = __ballot_sync(FULL, feas && key == mn);
+    if (!fm) {
+      infeasible = true;
+      break;
+    }
+    const int dsel = __ffs(fm) - 1;
+    if (dl == dsel) {
+      avail = mn;
+      if (need_mem) {
+        used += mem;
+        if (forced >= 0 && !pert) reserved -= mem;
+      }
+    }
+    makespan = mn > makespan ? mn : makespan;
+    if (lane == 0) Slab<T>::sched(slab, i, mn, (uint32_t)dsel);
+    if (want_out) {
+      const T stt = __shfl_sync(FULL, est, dsel);
+      const uint32_t u = __ldg(cd + CW_UID);
+      if (lane == 0) {
+        out_place[u] = (uint8_t)dsel;
+        if (out_start) out_start[u] = (int64_t)stt;
+        if (out_deq) out_deq[seq] = (int32_t)u;
+      }
+      seq++;
+    }
+    // release successors
+    if (nsucc <= (uint32_t)S_IN) {
+      bool push = false;
+      if ((uint32_t)lane < nsucc) {
+        const uint32_t dg = sdeg - 1;
+        Slab<T>::set_indeg(slab, sdst, dg);
+        push = dg == 0;
+      }
+      if (push) {
+        atomicOr(&leaf[sdst >> 5], 1u << (sdst & 31));
+        atomicOr(&summ[sdst >> 10], 1u << ((sdst >> 5) & 31));
+      }
+      top |= __reduce_or_sync(FULL, push ? (1u << (sdst >> 10)) : 0u);
+    } else {
+      for (uint32_t sb0 = 0; sb0 < nsucc; sb0 += 32) {
+        const uint32_t sj = sb0 + lane;
+        bool push = false;
+        uint32_t dst = 0;
+        if (sj < nsucc) {
+          dst = __ldg(pg->se_dst + h0.z + sj);
+          const uint32_t dg = Slab<T>::indeg(slab, dst) - 1;
+          Slab<T>::set_indeg(slab, dst, dg);
+          push = dg == 0;
+        }
+        if (push) {
+          atomicOr(&leaf[dst >> 5], 1u << (dst & 31));
+          atomicOr(&summ[dst >> 10], 1u << ((dst >> 5) & 31));
+        }
+        top |= __reduce_or_sync(FULL, push ? (1u << (dst >> 10)) : 0u);
+      }
+    }
+    __syncwarp();
+  }
+  __syncwarp();
+LoopOut r;
+r.makespan = (uint64_t)makespan;
+r.used = used;
+r.infeasible = infeasible ? 1 : 0;
+return r;
+}
+
+// One warp simulates one candidate at a time.  T: time type; GSH: log2 of the
+// lanes per predecessor group (the device count rounded up to a power of 2).
+template <typename T, int GSH, bool MEM>
+__global__ void __launch_bounds__(256, SIM_MINB) k_sim(SimArgs a) {
   typedef typename Slab<T>::W W;
+  constexpr int GP = 1 << GSH;   // lanes per predecessor (>= G)
   extern __shared__ uint32_t smem[];
   const int lane = threadIdx.x & 31;
   const int wib = threadIdx.x >> 5;
   const int64_t gwarp = (int64_t)blockIdx.x * (blockDim.x >> 5) + wib;
   uint32_t *leaf = smem + wib * (a.leaf_words + 32);
   uint32_t *summ = leaf + a.leaf_words;
-  W *slab = (W *)a.slab + gwarp * a.slab_stride;
+  W *slab = (W *)a.slab + (uint32_t)(gwarp * a.slab_stride);
   const GraphConst &gc = *a.gc;
   const int G = a.G;
   const int K = gc.K;
-  int gshift = 0;
-  while ((1 << gshift) < G) gshift++;
-  const int GP = 1 << gshift;
   const int dl = lane & (GP - 1);
-  const int ql = lane >> gshift;
-  const int PPP = 32 >> gshift;
   const int64_t cap_d = dl < G ? gc.cap[dl] : 0;
   const bool cp_on = (a.flags & 1u) != 0;
-
-  int64_t best_ms = I64MAX, best_idx = -1;
-  if (a.track_best) {
-    best_ms = a.wbest[2 * gwarp];
-    best_idx = a.wbest[2 * gwarp + 1];
+  const bool cap_chk = MEM && a.cap_check != 0;
+  // per-warp bookkeeping kept in shared memory (frees registers for the loop)
+  __shared__ int64_t s_best[8][2];
+  __shared__ int64_t s_res[8], s_sidx[8];
+  __shared__ const PrepGraph *s_pg[8];
+  if (lane == 0) {
+    s_best[wib][0] = a.track_best ? a.wbest[2 * gwarp] : I64MAX;
+    s_best[wib][1] = a.track_best ? a.wbest[2 * gwarp + 1] : -1;
   }
+  __syncwarp();
 
   for (;;) {
     unsigned long long qq = 0;
@@ -229,12 +590,10 @@ __global__ void __launch_bounds__(256, 4) k_sim(SimArgs a) {
     }
     const int32_t n = pg->n;
     const int32_t Vraw = pg->V;
-    const uint32_t *card = pg->card;
-    const T *costp = (const T *)pg->costp;
-    const uint32_t *pe_src = pg->pe_src;
-    const T *pe_comm = (const T *)pg->pe_comm;
-    const uint32_t *se_dst = pg->se_dst;
-    const uint32_t *posm = pg->pos;
+    const uint32_t *__restrict__ card = pg->card;
+    const T *__restrict__ costp = (const T *)pg->costp;
+    const T *__restrict__ pe_comm = (const T *)pg->pe_comm;
+    const uint32_t *__restrict__ posm = pg->pos;
 
     // ---------------------------------------------------------- validate
     int np = 0;
@@ -266,7 +625,7 @@ __global__ void __launch_bounds__(256, 4) k_sim(SimArgs a) {
     } else {
       np = c.kind == 1 ? c.n_pins : 0;
     }
-    // pins of this candidate, lane k < np holds pin k (as positions)
+    // pins of this candidate: lane k < np holds pin k (as a position)
     uint32_t my_pos = NONE;
     int my_dev = 0;
     if (st == 0 && lane < np) {
@@ -274,39 +633,8 @@ __global__ void __launch_bounds__(256, 4) k_sim(SimArgs a) {
       my_dev = c.pin_dev[lane];
     }
     // ------------------------------------------- classify (modes 0 and 1)
-    if (st == 0 && !defer && a.mode != 2 && np > 0) {
-      bool changed = false;
-      if (lane < np) {
-        const uint32_t i = my_pos;
-        const int di = my_dev;
-        T wmax = 0;
-        for (int d = 0; d < G; d++) {
-          T v = costp[(int64_t)i * G + d];
-          wmax = v > wmax ? v : wmax;
-        }
-        changed |= costp[(int64_t)i * G + di] != wmax;
-        const uint32_t *ci = card + (int64_t)i * CARD_WORDS;
-        uint32_t deg = ci[CW_DEG], pb = ci[CW_PBASE], sbb = ci[CW_SBASE];
-        for (uint32_t j = 0; j < (deg & 0xFFFF) && !changed; j++) {
-          uint32_t e = pb + j, o = pe_src[e];
-          // the other endpoint's pin, if any (pins are few; read them from the record)
-          int po = -1;
-          for (int k = 0; k < np; k++)
-            if (posm[c.pin_op[k]] == o) po = c.pin_dev[k];
-          const T *pc = pe_comm + (int64_t)e * K;
-          changed |= c_allowed_t<T>(gc, pc, -1, -1) != c_allowed_t<T>(gc, pc, po, di);
-        }
-        for (uint32_t j = 0; j < (deg >> 16) && !changed; j++) {
-          uint32_t o = se_dst[sbb + j], e = pg->se_pe[sbb + j];
-          int po = -1;
-          for (int k = 0; k < np; k++)
-            if (posm[c.pin_op[k]] == o) po = c.pin_dev[k];
-          const T *pc = pe_comm + (int64_t)e * K;
-          changed |= c_allowed_t<T>(gc, pc, -1, -1) != c_allowed_t<T>(gc, pc, di, po);
-        }
-      }
-      defer = __any_sync(FULL, changed);
-    }
+    if (st == 0 && !defer && a.mode != 2 && np > 0)
+      defer = __any_sync(FULL, lane < np && pin_changes_ranks<T>(pg, gc, c, np, my_pos, my_dev, G, K));
     if (defer) {
       if (lane == 0) {
         unsigned long long k = atomicAdd(a.ndefer, 1ull);
@@ -329,17 +657,15 @@ __global__ void __launch_bounds__(256, 4) k_sim(SimArgs a) {
     uint32_t top = 0;
     for (int32_t s = 0; s < nsumm; s++) {
       int32_t w = s * 32 + lane;
-      uint32_t word = w < nwords ? pg->srcbits[w] : 0u;
+      uint32_t word = w < nwords ? __ldg(pg->srcbits + w) : 0u;
       if (w < nwords) leaf[w] = word;
       unsigned m = __ballot_sync(FULL, word != 0);
       if (lane == 0) summ[s] = m;
       if (m) top |= 1u << s;
     }
-    for (int32_t p = lane; p < n; p += 32) Slab<T>::init(slab, (uint32_t)p, pg->npred[p]);
-    T avail = 0;
+    for (int32_t p = lane; p < n; p += 32) Slab<T>::init(slab, (uint32_t)p, __ldg(pg->npred + p));
     int64_t used = 0, reserved = 0;
     T makespan = 0;
-    int32_t seq = 0;
     bool infeasible = false;
 
     // CP devices (Alg. 1 line 5, R9) in free-index space
@@ -347,264 +673,40 @@ __global__ void __launch_bounds__(256, 4) k_sim(SimArgs a) {
     int r_dev = -1;
     int nrounds = 0;
     uint32_t my_pcp = NONE;  // CP index of this lane's pinned op
-    if (cp_on && pg->cp_len > 0) {
-      const int32_t L = pg->cp_len;
-      int64_t my_pmem = 0;
-      if (lane < np) {
-        const uint32_t *ci = card + (int64_t)my_pos * CARD_WORDS;
-        my_pcp = ci[CW_CPIDX];
-        my_pmem = (int64_t)(((uint64_t)ci[CW_MEMHI] << 32) | ci[CW_MEMLO]);
-      }
-      // pinned CP indices sorted ascending (uniform registers)
-      uint32_t pcs[MAXPINS];
-      int64_t pms[MAXPINS];
-      int64_t pcd[MAXPINS];  // cost on this lane's device
-      int m = 0;
-      bool oncp = lane < np && my_pcp != NONE;
-      unsigned oncp_m = __ballot_sync(FULL, oncp);
-      int my_rank = 0;
-      {
-        // rank of each on-CP pinned op among the on-CP pinned ops
-        int r = 0;
-        for (int k = 0; k < np; k++) {
-          uint32_t ok_ = __shfl_sync(FULL, my_pcp, k);
-          bool okon = (oncp_m >> k) & 1;
-          if (okon && ok_ < my_pcp) r++;
-        }
-        my_rank = r;
-      }
-      m = __popc(oncp_m);
-      for (int j = 0; j < MAXPINS; j++) {
-        unsigned who = __ballot_sync(FULL, oncp && my_rank == j);
-        int src = who ? __ffs(who) - 1 : 0;
-        uint32_t pv = __shfl_sync(FULL, my_pcp, src);
-        int64_t mv = __shfl_sync(FULL, my_pmem, src);
-        uint32_t ppos = __shfl_sync(FULL, my_pos, src);
-        pcs[j] = (j < m) ? pv : NONE;
-        pms[j] = (j < m) ? mv : 0;
-        pcd[j] = (j < m && dl < G) ? (int64_t)costp[(int64_t)ppos * G + dl] : 0;
-      }
-      const int32_t Lf = L - m;
-      auto raw_end = [&](int32_t f) -> int32_t {  // raw index just after the f-th free op (f >= 1)
-        int32_t r = f - 1;
-        for (int j = 0; j < MAXPINS; j++)
-          if (j < m && (int32_t)pcs[j] <= r) r++;
-        return r + 1;
-      };
-      auto fp_mem = [&](int32_t f) -> int64_t {
-        if (f <= 0) return 0;
-        int32_t re = raw_end(f);
-        int64_t v = pg->pmem[re];
-        for (int j = 0; j < MAXPINS; j++)
-          if (j < m && (int32_t)pcs[j] < re) v -= pms[j];
-        return v;
-      };
-      auto fp_cost = [&](int32_t f) -> int64_t {  // for device dl
-        if (f <= 0) return 0;
-        int32_t re = raw_end(f);
-        int64_t v = pg->pcost[(int64_t)re * G + dl];
-        for (int j = 0; j < MAXPINS; j++)
-          if (j < m && (int32_t)pcs[j] < re) v -= pcd[j];
-        return v;
-      };
-      uint32_t devs = G == 32 ? FULL : ((1u << G) - 1);
-      int32_t k = 0;
-      while (k < Lf && devs) {
-        int32_t t = 0;
-        int64_t S = 0;
-        if (lane < G && ((devs >> lane) & 1)) {
-          int64_t bm = fp_mem(k);
-          int64_t tot = fp_mem(Lf) - bm;
-          if (tot <= cap_d) t = Lf - k;
-          else {
-            int32_t lo = 0, hi = Lf - k;
-            while (hi - lo > 1) {
-              int32_t mid = (lo + hi) >> 1;
-              if (fp_mem(k + mid) - bm <= cap_d) lo = mid;
-              else hi = mid;
-            }
-            t = lo;
-          }
-          if (t > 0) S = fp_cost(k + t) - fp_cost(k);
-        }
-        int best = -1;
-        int32_t tb = 0;
-        int64_t Sb = 0;
-        for (int d = 0; d < G; d++) {
-          int32_t td = __shfl_sync(FULL, t, d);
-          int64_t Sd = __shfl_sync(FULL, S, d);
-          if (td > 0 && (best < 0 || lt_cross((uint64_t)Sd, (uint64_t)tb, (uint64_t)Sb, (uint64_t)td))) {
-            best = d;
-            tb = td;
-            Sb = Sd;
-          }
-        }
-        if (best < 0) break;
-        int64_t resv = fp_mem(k + tb) - fp_mem(k);
-        if (lane == nrounds) {
-          r_lo = (uint32_t)k;
-          r_hi = (uint32_t)(k + tb);
-          r_dev = best;
-        }
-        if (dl == best) reserved += resv;
-        devs &= ~(1u << best);
-        k += tb;
-        nrounds++;
-      }
-    }
+    if (cp_on && pg->cp_len > 0)
+      cp_rounds<T>(pg, np, my_pos, lane, dl, G, cap_d, r_lo, r_hi, r_dev, nrounds, my_pcp, reserved);
     __syncwarp();
 
     // ---------------------------------------------------------- main loop
-    const bool want_out = res_idx >= 0 && a.out.place != nullptr;
-    const int64_t obase = res_idx >= 0 ? res_idx * (int64_t)a.out.vmax : 0;
-    while (top) {
-      // pop: highest priority = lowest position
-      const int s = __ffs(top) - 1;
-      const uint32_t m = summ[s];
-      const int b = __ffs(m) - 1;
-      const int w = s * 32 + b;
-      const uint32_t lw = leaf[w];
-      const int jb = __ffs(lw) - 1;
-      const uint32_t i = (uint32_t)w * 32 + jb;
-      const uint32_t nlw = lw & ~(1u << jb);
-      const uint32_t nm = nlw ? m : (m & ~(1u << b));
-      __syncwarp();
-      if (lane == 0) {
-        leaf[w] = nlw;
-        summ[s] = nm;
-      }
-      if (!nm) top &= ~(1u << s);
-
-      const uint32_t cw = card[(int64_t)i * CARD_WORDS + lane];
-      const T cst = dl < G ? costp[(int64_t)i * G + dl] : (T)0;
-      const uint32_t deg = __shfl_sync(FULL, cw, CW_DEG);
-      const uint32_t npred = deg & 0xFFFF, nsucc = deg >> 16;
-      const uint32_t pbase = __shfl_sync(FULL, cw, CW_PBASE);
-      const uint32_t sbase = __shfl_sync(FULL, cw, CW_SBASE);
-      const uint32_t cpidx = __shfl_sync(FULL, cw, CW_CPIDX);
-      const int64_t mem =
-          (int64_t)(((uint64_t)__shfl_sync(FULL, cw, CW_MEMHI) << 32) | __shfl_sync(FULL, cw, CW_MEMLO));
-      const uint32_t psrc = __shfl_sync(FULL, cw, CARD_HDR + (lane < P_IN ? lane : 0));
-      const uint32_t sdst = __shfl_sync(FULL, cw, CARD_HDR + P_IN + (lane < S_IN ? lane : 0));
-
-      // device forced by a perturbation pin or a CP pin
-      int forced = -1;
-      bool pert = false;
-      const unsigned pmk = __ballot_sync(FULL, my_pos == i);
-      if (pmk) {
-        forced = __shfl_sync(FULL, my_dev, __ffs(pmk) - 1);
-        pert = true;
-      } else if (nrounds > 0 && cpidx != NONE) {
-        const uint32_t fi = cpidx - __popc(__ballot_sync(FULL, lane < np && my_pcp < cpidx));
-        const unsigned rm = __ballot_sync(FULL, lane < nrounds && fi >= r_lo && fi < r_hi);
-        if (rm) forced = __shfl_sync(FULL, r_dev, __ffs(rm) - 1);
-      }
-
-      // successor indegrees (independent of this step's result: prefetch)
-      uint32_t s0dst = 0, s0deg = 0;
-      if (lane < nsucc) {
-        s0dst = lane < S_IN ? sdst : se_dst[sbase + lane];
-        s0deg = Slab<T>::indeg(slab, s0dst);
-      }
-
-      // EST over predecessors for this lane's device dl
-      T estp = 0;
-      for (uint32_t pb0 = 0; pb0 < npred; pb0 += 32) {
-        const uint32_t pj = pb0 + lane;
-        T ftv = 0, cm = 0;
-        uint32_t plc = 0;
-        if (pj < npred) {
-          const uint32_t src = pj < P_IN ? psrc : pe_src[pbase + pj];
-          Slab<T>::load(slab, src, ftv, plc);
-          if (K == 1) cm = pe_comm[pbase + pj];
-        }
-        const uint32_t cnt = npred - pb0 < 32 ? npred - pb0 : 32;
-        for (uint32_t q0 = 0; q0 < cnt; q0 += PPP) {
-          const uint32_t qi = q0 + ql;
-          const T f = __shfl_sync(FULL, ftv, qi & 31);
-          const uint32_t pl = __shfl_sync(FULL, plc, qi & 31);
-          T cmm = __shfl_sync(FULL, cm, qi & 31);
-          if (qi < cnt) {
-            if (K > 1 && pl != (uint32_t)dl && dl < G)
-              cmm = pe_comm[(int64_t)(pbase + pb0 + qi) * K + gc.link_class[pl * G + dl]];
-            const T term = f + ((pl == (uint32_t)dl) ? (T)0 : cmm);
-            estp = term > estp ? term : estp;
-          }
-        }
-      }
-#pragma unroll
-      for (int o = 16; o >= 1; o >>= 1)
-        if (o >= GP) {
-          T x = __shfl_xor_sync(FULL, estp, o);
-          estp = x > estp ? x : estp;
-        }
-      const T est = estp > avail ? estp : avail;
-      const T eft = est + cst;
-      bool feas = lane < G;
-      if (forced >= 0) feas = feas && lane == forced;
-      if (forced < 0 || pert) feas = feas && (used + reserved + mem <= cap_d);
-      const T key = feas ? eft : TT<T>::MAXV;
-      const T mn = TT<T>::wmin(key);
-      const unsigned fm = __ballot_sync(FULL, feas && key == mn);
-      if (!fm) {
-        infeasible = true;
-        break;
-      }
-      const int dsel = __ffs(fm) - 1;
-      const T stt = __shfl_sync(FULL, est, dsel);
-      if (dl == dsel) {
-        avail = mn;
-        used += mem;
-        if (forced >= 0 && !pert) reserved -= mem;
-      }
-      makespan = mn > makespan ? mn : makespan;
-      if (lane == 0) Slab<T>::sched(slab, i, mn, (uint32_t)dsel);
-      if (want_out) {
-        const uint32_t u = __shfl_sync(FULL, cw, CW_UID);
-        if (lane == 0) {
-          a.out.place[obase + u] = (uint8_t)dsel;
-          if (a.out.start) a.out.start[obase + u] = (int64_t)stt;
-          if (a.out.deq) a.out.deq[obase + seq] = (int32_t)u;
-        }
-      }
-      seq++;
-      // release successors
-      for (uint32_t sb0 = 0; sb0 < nsucc; sb0 += 32) {
-        const uint32_t sj = sb0 + lane;
-        bool push = false;
-        uint32_t dst = 0;
-        if (sj < nsucc) {
-          uint32_t dg;
-          if (sb0 == 0) {
-            dst = s0dst;
-            dg = s0deg;
-          } else {
-            dst = se_dst[sbase + sj];
-            dg = Slab<T>::indeg(slab, dst);
-          }
-          dg -= 1;
-          Slab<T>::set_indeg(slab, dst, dg);
-          push = dg == 0;
-        }
-        if (push) {
-          atomicOr(&leaf[dst >> 5], 1u << (dst & 31));
-          atomicOr(&summ[dst >> 10], 1u << ((dst >> 5) & 31));
-        }
-        top |= __reduce_or_sync(FULL, push ? (1u << (dst >> 10)) : 0u);
-      }
-      __syncwarp();
+    if (lane == 0) {
+      s_res[wib] = res_idx;
+      s_sidx[wib] = sidx;
+      s_pg[wib] = pg;
     }
     __syncwarp();
-
+    {
+      const bool want_out = res_idx >= 0 && a.out.place != nullptr;
+      const int64_t ob = want_out ? res_idx * (int64_t)a.out.vmax : 0;
+      LoopOut lo = sim_loop<T, GSH, MEM>(leaf, summ, top, slab, card, costp, pe_comm, pg, a.gc, G, K, my_pos, my_dev,
+                                         np, r_lo, r_hi, r_dev, nrounds, my_pcp, cap_d, used, reserved, cap_chk,
+                                         want_out ? a.out.place + ob : nullptr,
+                                         want_out && a.out.start ? a.out.start + ob : nullptr,
+                                         want_out && a.out.deq ? a.out.deq + ob : nullptr);
+      makespan = (T)lo.makespan;
+      infeasible = lo.infeasible != 0;
+      used = lo.used;
+    }
     // ------------------------------------------------------------ epilogue
     int64_t ms64 = infeasible ? I64MAX : (int64_t)makespan;
-    if (res_idx >= 0) {
+    const int64_t res_idx2 = s_res[wib], sidx2 = s_sidx[wib];
+    const int64_t obase = res_idx2 >= 0 ? res_idx2 * (int64_t)a.out.vmax : 0;
+    if (res_idx2 >= 0) {
       if (lane == 0) {
-        a.out.makespan[res_idx] = ms64;
-        a.out.status[res_idx] = infeasible ? 1 : 0;
+        a.out.makespan[res_idx2] = ms64;
+        a.out.status[res_idx2] = infeasible ? 1 : 0;
       }
-      if (a.out.peak && lane < G) a.out.peak[res_idx * G + lane] = infeasible ? -1 : used;
-      if (infeasible && want_out) {
+      if (a.out.peak && lane < G) a.out.peak[res_idx2 * G + lane] = infeasible ? -1 : used;
+      if (infeasible && a.out.place != nullptr) {
         for (int32_t u = lane; u < a.out.vmax; u += 32) {
           a.out.place[obase + u] = 0xFF;
           if (a.out.start) a.out.start[obase + u] = -1;
@@ -612,37 +714,59 @@ __global__ void __launch_bounds__(256, 4) k_sim(SimArgs a) {
         }
       }
     }
-    if (!infeasible && (ms64 < best_ms || (ms64 == best_ms && sidx < best_idx))) {
-      best_ms = ms64;
-      best_idx = sidx;
+    if (lane == 0 && !infeasible && (ms64 < s_best[wib][0] || (ms64 == s_best[wib][0] && sidx2 < s_best[wib][1]))) {
+      s_best[wib][0] = ms64;
+      s_best[wib][1] = sidx2;
     }
-    // clear the smem bitmap state left by an aborted (infeasible) run
+    // clear the smem bitmap left by an aborted (infeasible) run
     if (infeasible) {
-      for (int32_t w = lane; w < nwords; w += 32) leaf[w] = 0;
-      if (lane < 32) summ[lane] = 0;
+      for (int32_t w = lane; w < a.leaf_words; w += 32) leaf[w] = 0;
+      summ[lane] = 0;
     }
     __syncwarp();
   }
+  __syncwarp();
   if (a.track_best && lane == 0) {
-    a.wbest[2 * gwarp] = best_ms;
-    a.wbest[2 * gwarp + 1] = best_idx;
+    a.wbest[2 * gwarp] = s_best[wib][0];
+    a.wbest[2 * gwarp + 1] = s_best[wib][1];
   }
 }
 
-void launch_sim(const SimArgs &a, int tbits, int grid, int block, size_t smem, cudaStream_t st) {
-  if (tbits == 32) k_sim<uint32_t><<<grid, block, smem, st>>>(a);
-  else k_sim<uint64_t><<<grid, block, smem, st>>>(a);
+template <typename T, bool MEM>
+static const void *sim_fn_t(int gshift) {
+  switch (gshift) {
+    case 0: return (const void *)k_sim<T, 0, MEM>;
+    case 1: return (const void *)k_sim<T, 1, MEM>;
+    case 2: return (const void *)k_sim<T, 2, MEM>;
+    case 3: return (const void *)k_sim<T, 3, MEM>;
+    case 4: return (const void *)k_sim<T, 4, MEM>;
+    default: return (const void *)k_sim<T, 5, MEM>;
+  }
+}
+static const void *sim_fn(int tbits, int gshift, bool mem) {
+  if (tbits == 32) return mem ? sim_fn_t<uint32_t, true>(gshift) : sim_fn_t<uint32_t, false>(gshift);
+  return mem ? sim_fn_t<uint64_t, true>(gshift) : sim_fn_t<uint64_t, false>(gshift);
 }
 
-int sim_occupancy(int tbits, int block, size_t smem) {
-  int nb = 0;
-  if (tbits == 32) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_sim<uint32_t>, block, smem);
-  else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_sim<uint64_t>, block, smem);
+void launch_sim(const SimArgs &a, int tbits, int grid, int block, size_t smem, cudaStream_t st) {
+  const void *f = sim_fn(tbits, a.gshift, a.need_mem != 0);
+  SimArgs aa = a;
+  void *args[] = {&aa};
+  cudaLaunchKernel(f, dim3(grid), dim3(block), args, smem, st);
+}
+
+int sim_occupancy(int tbits, int gshift, int block, size_t smem) {
+  int nb = 1 << 30, x = 0;
+  for (int mem = 0; mem < 2; mem++) {
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, sim_fn(tbits, gshift, mem), block, smem);
+    nb = x < nb ? x : nb;
+  }
   return nb;
 }
-cudaError_t sim_set_smem(int tbits, size_t smem) {
-  if (tbits == 32) return cudaFuncSetAttribute(k_sim<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  return cudaFuncSetAttribute(k_sim<uint64_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+cudaError_t sim_set_smem(int tbits, int gshift, size_t smem) {
+  cudaError_t e = cudaFuncSetAttribute(sim_fn(tbits, gshift, false), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(sim_fn(tbits, gshift, true), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
 }
 
 // ------------------------------------------------------------------ argmin

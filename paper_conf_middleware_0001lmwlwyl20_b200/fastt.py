@@ -15,7 +15,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libfastt.so")
+LIB_PATH = os.environ.get("FASTT_LIB") or os.path.join(_HERE, "libfastt.so")
 
 OK, EINVAL, ECYCLE, ENOMEM, ECUDA, ERANGE, EUNSUP = 0, -1, -2, -3, -4, -5, -6
 CAND_OK, CAND_INFEASIBLE, CAND_BADSPEC = 0, 1, 2
@@ -57,9 +57,15 @@ class fastt_split_result(C.Structure):
                 ("status", C.c_uint8)]
 
 
+class fastt_timing(C.Structure):
+    _fields_ = [("launches", C.c_int64), ("candidates", C.c_int64), ("deferred", C.c_int64),
+                ("ms_sim", C.c_float), ("ms_prep", C.c_float), ("ms_total", C.c_float)]
+
+
 SYMBOLS = ["fastt_load_graph", "fastt_free_graph", "fastt_graph_info", "fastt_rank", "fastt_schedule_batch",
            "fastt_stream_info", "fastt_generate_candidates", "fastt_sweep_best", "fastt_split_search",
-           "fastt_free_split_result", "fastt_last_error", "fastt_version"]
+           "fastt_free_split_result", "fastt_last_timing", "fastt_last_error", "fastt_version"]
+F_TIMING = 16
 
 _lib = None
 
@@ -91,6 +97,8 @@ def lib():
     L.fastt_split_search.restype = i32
     L.fastt_split_search.argtypes = [P, C.POINTER(fastt_opts), i32, C.POINTER(fastt_split_result)]
     L.fastt_free_split_result.argtypes = [C.POINTER(fastt_split_result)]
+    L.fastt_last_timing.restype = i32
+    L.fastt_last_timing.argtypes = [P, C.POINTER(fastt_timing)]
     L.fastt_last_error.restype = C.c_char_p
     L.fastt_version.restype = C.c_char_p
     _lib = L
@@ -279,6 +287,12 @@ class Graph:
         if out is not None:
             return out
         return int(buf[0]), int(buf[1])
+
+    def last_timing(self):
+        t = fastt_timing()
+        _check(lib().fastt_last_timing(self.h, C.byref(t)))
+        return {"launches": int(t.launches), "candidates": int(t.candidates), "deferred": int(t.deferred),
+                "ms_sim": float(t.ms_sim), "ms_prep": float(t.ms_prep), "ms_total": float(t.ms_total)}
 
     def split_search(self, flags=0, n_pow2_only=False, stream=None):
         r = fastt_split_result()
