@@ -10,8 +10,10 @@ SRCS = [os.path.join(HERE, "csrc", f) for f in ("fastt_abi.cu", "k_prep.cu", "k_
 DEPS = SRCS + [os.path.join(HERE, "csrc", "fastt_internal.cuh"), os.path.join(ROOT, "include", "fastt.h")]
 OUT = os.path.join(HERE, "libfastt.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17", "-Xcompiler", "-fPIC", "-DSIM_MINB=" + os.environ.get("SIM_MINB", "4"),
+FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17", "-Xcompiler", "-fPIC",
          "-shared", "-I" + os.path.join(ROOT, "include")]
+# launch-shape overrides for tuning experiments (defaults live in fastt_internal.cuh)
+FLAGS += ["-D%s=%s" % (k, os.environ[k]) for k in ("SIM_MINB", "SIM_BLOCK") if os.environ.get(k)]
 
 
 def build(force: bool = False, verbose: bool = False) -> str:

@@ -120,7 +120,7 @@ static PrepLayout prep_layout(int64_t ncap, int64_t ecap, int G, int K, int tbyt
                    (size_t)(ncap + 1) * G * 8,          // pcost
                    (size_t)ncap * 8, (size_t)ncap * 8,  // keys
                    (size_t)ncap * 4, (size_t)ncap * 4,  // vals
-                   16};
+                   33 * 4};                             // srcsumm
   size_t off = 0;
   for (int k = 0; k < 19; k++) {
     L.o[k] = off;
@@ -152,6 +152,7 @@ static PrepGraph prep_struct(char *b, const PrepLayout &L, int tbits) {
   P.key1 = (uint64_t *)(b + L.o[15]);
   P.val0 = (uint32_t *)(b + L.o[16]);
   P.val1 = (uint32_t *)(b + L.o[17]);
+  P.srcsumm = (uint32_t *)(b + L.o[18]);
   return P;
 }
 
@@ -220,7 +221,7 @@ struct fastt_graph {
   Cand *slot_cands = nullptr;
   int64_t *slot_result = nullptr, *slot_index = nullptr;
   // simulation workspace
-  int sms = 148, sim_block = 256, sim_grid = 0, sim_tbits = 0;
+  int sms = 148, sim_block = SIM_BLOCK, sim_grid = 0, sim_tbits = 0, sim_cpw = 1, sim_bm_stride = 0;
   int64_t sim_ncap = 0;
   size_t sim_smem = 0;
   void *slab = nullptr;
@@ -375,6 +376,14 @@ static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st)
   return FASTT_OK;
 }
 
+static int gshift_of(int G) {
+  int gsh = 0;
+  while ((1 << gsh) < G) gsh++;
+  return gsh;
+}
+
+// simulation workspace: one candidate per lane group (32 >> gshift per warp),
+// each with a ready bitmap in shared memory and an 8/16 B-per-op slab in HBM
 static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need) {
   int64_t ncap = B.pl.ncap;
   if (!g->slab || g->sim_tbits != B.tbits || g->sim_ncap < ncap) {
@@ -382,19 +391,23 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     cudaFree(g->wbest);
     g->slab = nullptr;
     g->wbest = nullptr;
+    const int gsh = gshift_of(g->G);
+    const int cpw = 32 >> gsh;
     int leaf = (int)((ncap + 31) / 32);
-    size_t smem = (size_t)(g->sim_block / 32) * (leaf + 32) * 4;
-    int gsh = 0;
-    while ((1 << gsh) < g->G) gsh++;
+    int stride = leaf + 32;
+    while (stride % 32 != 8) stride++;  // candidates of one warp start on different banks
+    size_t smem = (size_t)(g->sim_block / 32) * cpw * stride * 4;
     if (smem > 48 * 1024) CK(sim_set_smem(B.tbits, gsh, smem));
     int per_sm = sim_occupancy(B.tbits, gsh, g->sim_block, smem);
     if (per_sm < 1) return fail(FASTT_EUNSUP, "simulation kernel does not fit on an SM (smem %zu)", smem);
     g->sim_grid = g->sms * per_sm;
     g->sim_smem = smem;
-    int64_t nwarps = (int64_t)g->sim_grid * (g->sim_block / 32);
+    g->sim_cpw = cpw;
+    g->sim_bm_stride = stride;
+    int64_t nslot = (int64_t)g->sim_grid * (g->sim_block / 32) * cpw;
     size_t rec = B.tbits == 32 ? 8 : 16;
-    CK(cudaMalloc(&g->slab, (size_t)nwarps * ncap * rec));
-    CK(cudaMalloc(&g->wbest, sizeof(int64_t) * 2 * nwarps));
+    CK(cudaMalloc(&g->slab, (size_t)nslot * ncap * rec));
+    CK(cudaMalloc(&g->wbest, sizeof(int64_t) * 2 * nslot));
     g->sim_tbits = B.tbits;
     g->sim_ncap = ncap;
   }
@@ -426,6 +439,7 @@ static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
   a.slab = g->slab;
   a.slab_stride = g->sim_ncap;
   a.leaf_words = (int32_t)((g->sim_ncap + 31) / 32);
+  a.bm_stride = g->sim_bm_stride;
   a.G = g->G;
   while ((1 << a.gshift) < g->G) a.gshift++;
   for (int d = 0; d < g->G; d++)
@@ -508,7 +522,8 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
       b.slot_result = g->slot_result;
       b.slot_index = nullptr;
       b.n = nc;
-      launch_sim(b, B.tbits, std::min(g->sim_grid, (nc + 7) / 8 + 1), g->sim_block, g->sim_smem, st);
+      launch_sim(b, B.tbits, std::min<int64_t>(g->sim_grid, nc / ((g->sim_block / 32) * g->sim_cpw) + 1), g->sim_block,
+                 g->sim_smem, st);
       CK(cudaGetLastError());
     }
   }
@@ -1128,7 +1143,7 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
   TRY(check_gen(g, *S, gen, first, n, stride));
   Base &B = g->base;
   TRY(ensure_sim(g, B, n));
-  const int64_t nwarps = (int64_t)g->sim_grid * (g->sim_block / 32);
+  const int64_t nwarps = (int64_t)g->sim_grid * (g->sim_block / 32) * g->sim_cpw;  // candidate slots
   {
     std::vector<int64_t> init(2 * nwarps);
     for (int64_t w = 0; w < nwarps; w++) {

@@ -16,6 +16,14 @@
 #include <cstdint>
 #include <cuda_runtime.h>
 
+// simulation kernel launch shape (threads per block, min blocks per SM)
+#ifndef SIM_BLOCK
+#define SIM_BLOCK 128
+#endif
+#ifndef SIM_MINB
+#define SIM_MINB 5
+#endif
+
 namespace fastt {
 
 constexpr int MAXG = 32;
@@ -23,8 +31,12 @@ constexpr int MAXK = 16;
 constexpr int MAXPINS = 4;
 constexpr int CARD_WORDS = 32;
 constexpr int CARD_HDR = 8;
-constexpr int P_IN = 12;  // inline predecessor positions in a card
-constexpr int S_IN = 12;  // inline successor positions in a card
+// card words 8..11: up to 4 predecessor positions; 12..15: their comm
+// values (uint32 time, one link class); 16..31: up to 16 successor positions
+constexpr int P_IN = 4;   // inline predecessor positions in a card
+constexpr int S_IN = 16;  // inline successor positions in a card
+constexpr int CW_PCOMM = CARD_HDR + P_IN;  // inline comm values
+constexpr int CW_SUCC = CW_PCOMM + P_IN;   // inline successor positions
 constexpr uint32_t NONE = 0xFFFFFFFFu;
 constexpr int64_t I64MAX = INT64_MAX;
 
@@ -70,6 +82,7 @@ struct PrepGraph {
   uint32_t *se_pe;  // E: index of the same edge in pe_*
   uint32_t *npred;  // n
   uint32_t *srcbits;// ceil(n/32): positions with no predecessor
+  uint32_t *srcsumm;// 33 words: summary of srcbits (bit b of word s = leaf word 32s+b nonzero), [32] = top
   uint32_t *pos;    // V: uid -> position (NONE for dead)
   uint32_t *uid;    // n: position -> uid
   uint64_t *rank;   // V: rank_u by uid (~0 for dead)
@@ -154,11 +167,12 @@ struct SimArgs {
   unsigned long long *counter;  // work counter
   int64_t *defer_q;      // deferred work items (q)
   unsigned long long *ndefer;
-  int64_t *wbest;        // per-warp (makespan, index) pairs, 2 per warp
+  int64_t *wbest;        // per candidate slot (makespan, index) pairs
   SimOut out;
   void *slab;            // per-warp state slabs
   int64_t slab_stride;   // elements (records) per warp
-  int32_t leaf_words;    // bitmap words per warp in smem
+  int32_t leaf_words;    // ready-bitmap leaf words per candidate (smem)
+  int32_t bm_stride;     // smem words per candidate: leaf_words + 32 summary words, padded
   int32_t G;
   int32_t gshift;        // ceil(log2(G)): lanes per predecessor group = 1 << gshift
   int32_t track_best;

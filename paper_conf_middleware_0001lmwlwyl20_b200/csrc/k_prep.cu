@@ -455,6 +455,19 @@ __global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, Prep
     runs += tots;
   }
   if (threadIdx.x == 0) P.E = runp;
+  __syncthreads();
+  // summary level of the source bitmap (read by the simulator's prologue)
+  if (threadIdx.x < 32) {
+    const int32_t nw = (n + 31) / 32;
+    uint32_t sw = 0;
+    for (int b = 0; b < 32; b++) {
+      int32_t w = (int32_t)threadIdx.x * 32 + b;
+      if (w < nw && P.srcbits[w]) sw |= 1u << b;
+    }
+    P.srcsumm[threadIdx.x] = sw;
+    unsigned top = __ballot_sync(0xFFFFFFFFu, sw != 0);
+    if (threadIdx.x == 0) P.srcsumm[32] = top;
+  }
 }
 
 // One warp per position: edge arrays, inline card entries and the cost row.
@@ -483,7 +496,10 @@ __global__ void k_cards_edges(const RawGraph *raws, PrepGraph *pgs, const GraphC
       uint32_t sp = P.pos[s];
       P.pe_src[pb + j] = sp;
       for (int k = 0; k < K; k++) pec[(int64_t)(pb + j) * K + k] = (T)comm_class(gc, b, k);
-      if (j < P_IN) c[CARD_HDR + j] = sp;
+      if (j < P_IN) {
+        c[CARD_HDR + j] = sp;
+        c[CW_PCOMM + j] = (uint32_t)comm_class(gc, b, 0);  // used only for uint32 time, one class
+      }
     }
     for (uint32_t j = lane; j < ns_; j += 32) {
       int32_t d = R.succ_dst[so + j];
@@ -493,11 +509,14 @@ __global__ void k_cards_edges(const RawGraph *raws, PrepGraph *pgs, const GraphC
       uint32_t dpo = R.pred_off[d], dcnt = R.pred_cnt[d], q = 0;
       while (q < dcnt && R.pred_src[dpo + q] != (int32_t)u) q++;
       P.se_pe[sb + j] = P.card[(int64_t)dp * CARD_WORDS + CW_PBASE] + q;
-      if (j < S_IN) c[CARD_HDR + P_IN + j] = dp;
+      if (j < S_IN) c[CW_SUCC + j] = dp;
     }
     // unused inline slots hold position 0 so the simulator may load them speculatively
-    if (lane >= np_ && lane < P_IN) c[CARD_HDR + lane] = 0;
-    if (lane >= ns_ && lane < S_IN) c[CARD_HDR + P_IN + lane] = 0;
+    if (lane >= np_ && lane < P_IN) {
+      c[CARD_HDR + lane] = 0;
+      c[CW_PCOMM + lane] = 0;
+    }
+    if (lane >= ns_ && lane < S_IN) c[CW_SUCC + lane] = 0;
   }
   (void)max_n;
 }
@@ -563,7 +582,7 @@ __global__ void k_cp(PrepGraph *pgs, int nslots, int G) {
     uint32_t ns_ = deg >> 16, sb = c[CW_SBASE];
     uint32_t best = NONE;
     for (uint32_t j = lane; j < ns_; j += 32) {
-      uint32_t d = j < S_IN ? c[CARD_HDR + P_IN + j] : P.se_dst[sb + j];
+      uint32_t d = j < S_IN ? c[CW_SUCC + j] : P.se_dst[sb + j];
       best = d < best ? d : best;
     }
     best = warp_min_u32(best);

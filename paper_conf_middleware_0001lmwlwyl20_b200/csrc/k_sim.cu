@@ -1,23 +1,25 @@
 // k_sim.cu -- batched DPOS list-scheduling simulation.
 //
-// One warp owns one candidate at a time (persistent kernel, work fetched
-// from a global counter).  Per candidate:
+// Persistent kernel; a warp holds 32/GP candidates, one per group of GP
+// lanes (GP = the device count rounded up to a power of two; lane d of a
+// group is device d).  Work is fetched from a global counter.  Per candidate:
 //   prologue : decode (stream R21 / list), validate, classify (do its ranks
 //              equal the base ranks? else defer to the per-candidate
 //              preparation pipeline), CP-device rounds (R9),
 //              ready-set bitmap from the source bitmap, indegrees into the
-//              warp's slab.
+//              candidate's slab.
 //   loop     : pop the max-priority ready op = find-first-set over the
 //              position bitmap (2 levels in smem + 1 in a register);
-//              one coalesced 128-B card load + the cost row; lanes
-//              (pred q, device d) form FT(pred)+comm (R6), a
-//              shuffle max over q, EST = max(avail[d], .) (R1 append),
-//              EFT = EST + cost; memory-feasible argmin over d with ties to
-//              the lowest device (Alg. 1 lines 12-19, R3, R8); CP pins
-//              (lines 9-10) and perturbation pins override the argmin;
-//              release successors (indegree in the slab) into the bitmap.
+//              loads from the op's 128-B card (predecessor positions and
+//              comm, successors) + the cost row, then the predecessor
+//              records; lane d forms EST(d) = max(avail[d], max_pred FT +
+//              comm) (R1, R6), EFT = EST + cost; memory-feasible
+//              argmin over the group with ties to the lowest device
+//              (Alg. 1 lines 12-19, R3, R8); CP pins (lines 9-10) and
+//              perturbation pins override it; release successors
+//              (indegree in the slab) into the bitmap.
 //   epilogue : makespan = max FT (R16), peak memory per device, outputs,
-//              per-warp best (makespan, index) for the sweep argmin (S7).
+//              per-slot best (makespan, index) for the sweep argmin (S7).
 // Time arithmetic runs in T = uint32 when the load-time bound proves every
 // schedule fits (R18), else uint64; results are identical.
 #include "fastt_internal.cuh"
@@ -176,7 +178,6 @@ __device__ __forceinline__ bool lt_cross(uint64_t a, uint64_t mb, uint64_t b, ui
   return h1 < h2 || (h1 == h2 && l1 < l2);
 }
 
-
 // A PIN candidate keeps the base ranks iff w of each pinned op and
 // c of every edge touching one are unchanged under R5's allowed
 // sets; otherwise it is deferred to the per-candidate preparation pipeline.
@@ -214,46 +215,46 @@ __device__ __noinline__ bool pin_changes_ranks(const PrepGraph *pg, const GraphC
   return changed;
 }
 
-// CP devices (Alg. 1 line 5, R9): repeatedly give the
-// device with the smallest exact average cost the longest prefix of the
-// remaining free CP ops that fits its memory; perturbation-pinned CP ops are
-// excluded (free-index space).  Lane r < nrounds receives round r.
+// CP devices (Alg. 1 line 5, R9) for one candidate,
+// executed by its lane group (gm = group mask, gb = first lane, d = device
+// lane): repeatedly give the device with the smallest exact average cost the
+// longest prefix of the remaining free CP ops that fits its memory;
+// perturbation-pinned CP ops are excluded (free-index space).  Lane gb + r
+// receives round r.
 template <typename T>
-__device__ __noinline__ void cp_rounds(const PrepGraph *pg, int np, uint32_t my_pos, int lane, int dl, int G,
-                                       int64_t cap_d, uint32_t &r_lo, uint32_t &r_hi, int &r_dev, int &nrounds,
-                                       uint32_t &my_pcp, int64_t &reserved) {
+__device__ __noinline__ void cp_rounds_g(const PrepGraph *pg, int np, const uint32_t *pp, unsigned gm, int gb, int d,
+                                         int G, int64_t cap_d, uint32_t &r_lo, uint32_t &r_hi, int &r_dev,
+                                         int &nrounds, uint32_t *pcp, int64_t &reserved) {
   const uint32_t *card = pg->card;
   const T *costp = (const T *)pg->costp;
   const int32_t L = pg->cp_len;
-  int64_t my_pmem = 0;
-  if (lane < np) {
-    const uint32_t *ci = card + (int64_t)my_pos * CARD_WORDS;
-    my_pcp = ci[CW_CPIDX];
-    my_pmem = (int64_t)(((uint64_t)ci[CW_MEMHI] << 32) | ci[CW_MEMLO]);
-  }
-  // pinned CP indices sorted ascending (uniform registers)
+  // CP index / memory of each pinned op; the on-CP ones sorted ascending
   uint32_t pcs[MAXPINS];
   int64_t pms[MAXPINS];
   int64_t pcd[MAXPINS];  // cost on this lane's device
-  bool oncp = lane < np && my_pcp != NONE;
-  unsigned oncp_m = __ballot_sync(FULL, oncp);
-  int my_rank = 0;
-  for (int k = 0; k < np; k++) {
-    uint32_t ok_ = __shfl_sync(FULL, my_pcp, k);
-    bool okon = (oncp_m >> k) & 1;
-    if (okon && ok_ < my_pcp) my_rank++;
+  int m = 0;
+  for (int k = 0; k < MAXPINS; k++) {
+    pcp[k] = NONE;
+    pcs[k] = NONE;
+    pms[k] = 0;
+    pcd[k] = 0;
   }
-  const int m = __popc(oncp_m);
-#pragma unroll
-  for (int j = 0; j < MAXPINS; j++) {
-    unsigned who = __ballot_sync(FULL, oncp && my_rank == j);
-    int src = who ? __ffs(who) - 1 : 0;
-    uint32_t pv = __shfl_sync(FULL, my_pcp, src);
-    int64_t mv = __shfl_sync(FULL, my_pmem, src);
-    uint32_t ppos = __shfl_sync(FULL, my_pos, src);
-    pcs[j] = (j < m) ? pv : NONE;
-    pms[j] = (j < m) ? mv : 0;
-    pcd[j] = (j < m && dl < G) ? (int64_t)costp[(int64_t)ppos * G + dl] : 0;
+  for (int k = 0; k < np; k++) {
+    const uint32_t *ci = card + (int64_t)pp[k] * CARD_WORDS;
+    pcp[k] = ci[CW_CPIDX];
+    if (pcp[k] == NONE) continue;
+    int j = m++;
+    const int64_t mv = (int64_t)(((uint64_t)ci[CW_MEMHI] << 32) | ci[CW_MEMLO]);
+    const int64_t cv = d < G ? (int64_t)costp[(int64_t)pp[k] * G + d] : 0;
+    while (j > 0 && pcs[j - 1] > pcp[k]) {
+      pcs[j] = pcs[j - 1];
+      pms[j] = pms[j - 1];
+      pcd[j] = pcd[j - 1];
+      j--;
+    }
+    pcs[j] = pcp[k];
+    pms[j] = mv;
+    pcd[j] = cv;
   }
   const int32_t Lf = L - m;
   auto raw_end = [&](int32_t f) -> int32_t {  // raw index just after the f-th free op (f >= 1)
@@ -272,10 +273,10 @@ __device__ __noinline__ void cp_rounds(const PrepGraph *pg, int np, uint32_t my_
       if (j < m && (int32_t)pcs[j] < re) v -= pms[j];
     return v;
   };
-  auto fp_cost = [&](int32_t f) -> int64_t {  // for device dl
+  auto fp_cost = [&](int32_t f) -> int64_t {  // for device d
     if (f <= 0) return 0;
     int32_t re = raw_end(f);
-    int64_t v = pg->pcost[(int64_t)re * G + dl];
+    int64_t v = pg->pcost[(int64_t)re * G + d];
 #pragma unroll
     for (int j = 0; j < MAXPINS; j++)
       if (j < m && (int32_t)pcs[j] < re) v -= pcd[j];
@@ -286,7 +287,7 @@ __device__ __noinline__ void cp_rounds(const PrepGraph *pg, int np, uint32_t my_
   while (k < Lf && devs) {
     int32_t t = 0;
     int64_t S = 0;
-    if (lane < G && ((devs >> lane) & 1)) {
+    if (d < G && ((devs >> d) & 1)) {
       int64_t bm = fp_mem(k);
       int64_t tot = fp_mem(Lf) - bm;
       if (tot <= cap_d) t = Lf - k;
@@ -304,431 +305,396 @@ __device__ __noinline__ void cp_rounds(const PrepGraph *pg, int np, uint32_t my_
     int best = -1;
     int32_t tb = 0;
     int64_t Sb = 0;
-    for (int d = 0; d < G; d++) {
-      int32_t td = __shfl_sync(FULL, t, d);
-      int64_t Sd = __shfl_sync(FULL, S, d);
+    for (int dd = 0; dd < G; dd++) {
+      int32_t td = __shfl_sync(gm, t, gb + dd);
+      int64_t Sd = __shfl_sync(gm, S, gb + dd);
       if (td > 0 && (best < 0 || lt_cross((uint64_t)Sd, (uint64_t)tb, (uint64_t)Sb, (uint64_t)td))) {
-        best = d;
+        best = dd;
         tb = td;
         Sb = Sd;
       }
     }
     if (best < 0) break;
     int64_t resv = fp_mem(k + tb) - fp_mem(k);
-    if (lane == nrounds) {
+    if (d == nrounds) {
       r_lo = (uint32_t)k;
       r_hi = (uint32_t)(k + tb);
       r_dev = best;
     }
-    if (dl == best) reserved += resv;
+    if (d == best) reserved += resv;
     devs &= ~(1u << best);
     k += tb;
     nrounds++;
   }
 }
 
-// general predecessor max for ops with more predecessors than one lane pass
-// holds (or beyond the inline card entries): chunks of 32 via pe_src.
-template <typename T, int GSH>
-__device__ __forceinline__ T pred_max_general(const typename Slab<T>::W *slab, const uint32_t *pe_src, const T *pe_comm,
-                                           const GraphConst &gc, uint32_t npred, uint32_t pbase, int lane, int G,
-                                           int K) {
-  constexpr int GP = 1 << GSH, PPP = 32 >> GSH;
-  const int dl = lane & (GP - 1), ql = lane >> GSH;
-  T estp = 0;
-  for (uint32_t pb0 = 0; pb0 < npred; pb0 += 32) {
-    const uint32_t pj = pb0 + lane;
-    T ftv = 0, cm = 0;
-    uint32_t plc = 0;
-    if (pj < npred) {
-      const uint32_t src = __ldg(pe_src + pbase + pj);
-      Slab<T>::load(slab, src, ftv, plc);
-      if (K == 1) cm = __ldg(pe_comm + pbase + pj);
-    }
-    const uint32_t cnt = npred - pb0 < 32 ? npred - pb0 : 32;
-    for (uint32_t q0 = 0; q0 < cnt; q0 += PPP) {
-      const uint32_t qi = q0 + ql;
-      const T f = __shfl_sync(FULL, ftv, qi & 31);
-      const uint32_t pl = __shfl_sync(FULL, plc, qi & 31);
-      T cmm = __shfl_sync(FULL, cm, qi & 31);
-      if (qi < cnt) {
-        if (K > 1 && pl != (uint32_t)dl && dl < G)
-          cmm = __ldg(pe_comm + (size_t)(pbase + pb0 + qi) * K + gc.link_class[pl * G + dl]);
-        const T term = f + ((pl == (uint32_t)dl) ? (T)0 : cmm);
-        estp = term > estp ? term : estp;
-      }
-    }
-  }
-#pragma unroll
-  for (int o = 16; o >= GP; o >>= 1) {
-    T x = __shfl_xor_sync(FULL, estp, o);
-    estp = x > estp ? x : estp;
-  }
-  return estp;
-}
-
-
-struct LoopOut {
-  uint64_t makespan;
-  int64_t used;
-  int32_t infeasible;
-};
-
-// The hot loop of DPOS (Alg. 1 lines 6-22) for one candidate, isolated so
-// its register allocation holds only loop state.
+// Several candidates per warp: lane group g (GP = 2^GSH lanes, GP >= G) owns
+// one candidate; lane d of the group is device d.  The main loop keeps the
+// warp converged (groups that finished idle) so every shuffle/vote is a
+// full-warp instruction.  T: time type; MEM: track per-device memory.
 template <typename T, int GSH, bool MEM>
-__device__ __noinline__ LoopOut sim_loop(uint32_t *leaf, uint32_t *summ, uint32_t top, typename Slab<T>::W *slab,
-                                         const uint32_t *__restrict__ card, const T *__restrict__ costp,
-                                         const T *__restrict__ pe_comm, const PrepGraph *pg, const GraphConst *gcp,
-                                         const int G, const int K, const uint32_t my_pos, const int my_dev,
-                                         const int np, const uint32_t r_lo, const uint32_t r_hi, const int r_dev,
-                                         const int nrounds, const uint32_t my_pcp, const int64_t cap_d,
-                                         int64_t used, int64_t reserved, const bool cap_chk, uint8_t *out_place,
-                                         int64_t *out_start, int32_t *out_deq) {
-  constexpr int GP = 1 << GSH;
-  constexpr int PPP = 32 >> GSH;
-  constexpr int PFAST = PPP < P_IN ? PPP : P_IN;
-  constexpr bool need_mem = MEM;
-  const int lane = threadIdx.x & 31;
-  const int dl = lane & (GP - 1);
-  const int ql = lane >> GSH;
-  const bool want_out = out_place != nullptr;
-  T avail = 0, makespan = 0;
-  int32_t seq = 0;
-  bool infeasible = false;
-  while (top) {
-    // pop: highest priority = lowest position = lowest set bit
-    const int s = __ffs(top) - 1;
-    const uint32_t m = summ[s];
-    const int b = __ffs(m) - 1;
-    const int w = (s << 5) + b;
-    const uint32_t lw = leaf[w];
-    const uint32_t i = ((uint32_t)w << 5) + (__ffs(lw) - 1);
-    const uint32_t nlw = lw & (lw - 1);
-    const uint32_t nm = nlw ? m : (m & (m - 1));
-    __syncwarp();
-    if (lane == 0) {
-      leaf[w] = nlw;
-      summ[s] = nm;
-    }
-    if (!nm) top &= top - 1;
-
-    // round 1: the card (zero-padded inline entries make every slot a
-    // valid index), this lane's predecessor slot, successor slot, cost
-    const uint32_t *cd = card + (size_t)i * CARD_WORDS;
-    const uint4 h0 = __ldg((const uint4 *)cd);  // deg, pbase, sbase, cpidx
-    const uint32_t psrc = __ldg(cd + CARD_HDR + (ql < P_IN ? ql : 0));
-    const uint32_t sdst = __ldg(cd + CARD_HDR + P_IN + (lane < S_IN ? lane : 0));
-    const T cst = __ldg(costp + (size_t)i * G + (dl < G ? dl : 0));
-    // round 2 (speculative): predecessor record, edge comm, successor indegree
-    T ftv;
-    uint32_t plc;
-    Slab<T>::load(slab, psrc, ftv, plc);
-    const uint32_t sdeg = Slab<T>::indeg(slab, sdst);
-    const uint32_t npred = h0.x & 0xFFFF, nsucc = h0.x >> 16;
-    T estp;
-    if (npred <= (uint32_t)PFAST) {
-      T term = 0;
-      if ((uint32_t)ql < npred) {
-        T cm;
-        if (K == 1) cm = __ldg(pe_comm + h0.y + ql);
-        else cm = (plc != (uint32_t)dl && dl < G) ? __ldg(pe_comm + (size_t)(h0.y + ql) * K + gcp->link_class[plc * G + dl]) : (T)0;
-        term = ftv + (plc == (uint32_t)dl ? (T)0 : cm);
-      }
-#pragma unroll
-      for (int o = 16; o >= GP; o >>= 1) {
-        T x = __shfl_xor_sync(FULL, term, o);
-        term = x > term ? x : term;
-      }
-      estp = term;
-    } else {
-      estp = pred_max_general<T, GSH>(slab, pg->pe_src, pe_comm, *gcp, npred, h0.y, lane, G, K);
-    }
-    const T est = estp > avail ? estp : avail;
-    const T eft = est + cst;
-
-    // device forced by a perturbation pin or a CP pin
-    int forced = -1;
-    bool pert = false;
-    if (np) {
-      const unsigned pmk = __ballot_sync(FULL, my_pos == i);
-      if (pmk) {
-        forced = __shfl_sync(FULL, my_dev, __ffs(pmk) - 1);
-        pert = true;
-      }
-    }
-    if (forced < 0 && nrounds > 0 && h0.w != NONE) {
-      const uint32_t fi = h0.w - __popc(__ballot_sync(FULL, lane < np && my_pcp < h0.w));
-      const unsigned rm = __ballot_sync(FULL, lane < nrounds && fi >= r_lo && fi < r_hi);
-      if (rm) forced = __shfl_sync(FULL, r_dev, __ffs(rm) - 1);
-    }
-    int64_t mem = 0;
-    if (need_mem) mem = (int64_t)(((uint64_t)__ldg(cd + CW_MEMHI) << 32) | __ldg(cd + CW_MEMLO));
-    bool feas = lane < G;
-    if (forced >= 0) feas = feas && lane == forced;
-    if (cap_chk && (forced < 0 || pert)) feas = feas && (used + reserved + mem <= cap_d);
-    const T key = feas ? eft : TT<T>::MAXV;
-    const T mn = TT<T>::wmin(key);
-    const unsigned fm = __ballot_sync(FULL, feas && key == mn);
-    if (!fm) {
-      infeasible = true;
-      break;
-    }
-    const int dsel = __ffs(fm) - 1;
-    if (dl == dsel) {
-      avail = mn;
-      if (need_mem) {
-        used += mem;
-        if (forced >= 0 && !pert) reserved -= mem;
-      }
-    }
-    makespan = mn > makespan ? mn : makespan;
-    if (lane == 0) Slab<T>::sched(slab, i, mn, (uint32_t)dsel);
-    if (want_out) {
-      const T stt = __shfl_sync(FULL, est, dsel);
-      const uint32_t u = __ldg(cd + CW_UID);
-      if (lane == 0) {
-        out_place[u] = (uint8_t)dsel;
-        if (out_start) out_start[u] = (int64_t)stt;
-        if (out_deq) out_deq[seq] = (int32_t)u;
-      }
-      seq++;
-    }
-    // release successors
-    if (nsucc <= (uint32_t)S_IN) {
-      bool push = false;
-      if ((uint32_t)lane < nsucc) {
-        const uint32_t dg = sdeg - 1;
-        Slab<T>::set_indeg(slab, sdst, dg);
-        push = dg == 0;
-      }
-      if (push) {
-        atomicOr(&leaf[sdst >> 5], 1u << (sdst & 31));
-        atomicOr(&summ[sdst >> 10], 1u << ((sdst >> 5) & 31));
-      }
-      top |= __reduce_or_sync(FULL, push ? (1u << (sdst >> 10)) : 0u);
-    } else {
-      for (uint32_t sb0 = 0; sb0 < nsucc; sb0 += 32) {
-        const uint32_t sj = sb0 + lane;
-        bool push = false;
-        uint32_t dst = 0;
-        if (sj < nsucc) {
-          dst = __ldg(pg->se_dst + h0.z + sj);
-          const uint32_t dg = Slab<T>::indeg(slab, dst) - 1;
-          Slab<T>::set_indeg(slab, dst, dg);
-          push = dg == 0;
-        }
-        if (push) {
-          atomicOr(&leaf[dst >> 5], 1u << (dst & 31));
-          atomicOr(&summ[dst >> 10], 1u << ((dst >> 5) & 31));
-        }
-        top |= __reduce_or_sync(FULL, push ? (1u << (dst >> 10)) : 0u);
-      }
-    }
-    __syncwarp();
-  }
-  __syncwarp();
-LoopOut r;
-r.makespan = (uint64_t)makespan;
-r.used = used;
-r.infeasible = infeasible ? 1 : 0;
-return r;
-}
-
-// One warp simulates one candidate at a time.  T: time type; GSH: log2 of the
-// lanes per predecessor group (the device count rounded up to a power of 2).
-template <typename T, int GSH, bool MEM>
-__global__ void __launch_bounds__(256, SIM_MINB) k_sim(SimArgs a) {
+__global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
   typedef typename Slab<T>::W W;
-  constexpr int GP = 1 << GSH;   // lanes per predecessor (>= G)
+  constexpr int GP = 1 << GSH;   // lanes per candidate (>= G)
+  constexpr int CPW = 32 >> GSH; // candidates per warp
   extern __shared__ uint32_t smem[];
+  __shared__ int64_t s_best[SIM_BLOCK][2];      // per group leader
+  __shared__ int64_t s_res[SIM_BLOCK], s_sidx[SIM_BLOCK];
   const int lane = threadIdx.x & 31;
   const int wib = threadIdx.x >> 5;
+  const int grp = lane >> GSH;
+  const int d = lane & (GP - 1);
+  const int gb = grp << GSH;
+  const unsigned gm = GP == 32 ? FULL : (((1u << GP) - 1u) << gb);
+  const int lead = threadIdx.x - d;  // group leader thread (s_* index)
   const int64_t gwarp = (int64_t)blockIdx.x * (blockDim.x >> 5) + wib;
-  uint32_t *leaf = smem + wib * (a.leaf_words + 32);
+  const int64_t cslot = gwarp * CPW + grp;
+  uint32_t *leaf = smem + (uint32_t)(wib * CPW + grp) * (uint32_t)a.bm_stride;
   uint32_t *summ = leaf + a.leaf_words;
-  W *slab = (W *)a.slab + (uint32_t)(gwarp * a.slab_stride);
+  W *slab = (W *)a.slab + (size_t)cslot * (size_t)a.slab_stride;
   const GraphConst &gc = *a.gc;
   const int G = a.G;
   const int K = gc.K;
-  const int dl = lane & (GP - 1);
-  const int64_t cap_d = dl < G ? gc.cap[dl] : 0;
+  const int64_t cap_d = d < G ? gc.cap[d] : 0;
   const bool cp_on = (a.flags & 1u) != 0;
   const bool cap_chk = MEM && a.cap_check != 0;
-  // per-warp bookkeeping kept in shared memory (frees registers for the loop)
-  __shared__ int64_t s_best[8][2];
-  __shared__ int64_t s_res[8], s_sidx[8];
-  __shared__ const PrepGraph *s_pg[8];
-  if (lane == 0) {
-    s_best[wib][0] = a.track_best ? a.wbest[2 * gwarp] : I64MAX;
-    s_best[wib][1] = a.track_best ? a.wbest[2 * gwarp + 1] : -1;
+  const bool fastcomm = sizeof(T) == 4 && K == 1;
+  if (d == 0) {
+    s_best[lead][0] = a.track_best ? a.wbest[2 * cslot] : I64MAX;
+    s_best[lead][1] = a.track_best ? a.wbest[2 * cslot + 1] : -1;
   }
   __syncwarp();
 
   for (;;) {
-    unsigned long long qq = 0;
-    if (lane == 0) qq = atomicAdd(a.counter, 1ull);
-    qq = __shfl_sync(FULL, qq, 0);
-    if ((int64_t)qq >= a.n) break;
-    const int64_t q = (int64_t)qq;
+    unsigned long long q0 = 0;
+    if (lane == 0) q0 = atomicAdd(a.counter, (unsigned long long)CPW);
+    q0 = __shfl_sync(FULL, q0, 0);
+    if ((int64_t)q0 >= a.n) break;
+    const int64_t q = (int64_t)q0 + grp;
+    const bool active = q < a.n;
     Cand c;
-    const PrepGraph *pg;
+    c.kind = 0; c.n_pins = 0; c.split_op = -1;
+    const PrepGraph *pg = a.base;
     int64_t res_idx = -1, sidx = q;
-    if (a.mode == 0) {
-      sidx = a.first + q * a.stride;
-      c = stream_cand(a.stream, sidx);
-      pg = a.base;
-    } else if (a.mode == 1) {
-      c = a.cands[q];
-      pg = a.base;
-      res_idx = q;
-    } else {
-      c = a.cands[q];
-      pg = a.slots + q;
-      res_idx = a.slot_result ? a.slot_result[q] : -1;
-      sidx = a.slot_index ? a.slot_index[q] : q;
+    if (active) {
+      if (a.mode == 0) {
+        sidx = a.first + q * a.stride;
+        c = stream_cand(a.stream, sidx);
+      } else if (a.mode == 1) {
+        c = a.cands[q];
+        res_idx = q;
+      } else {
+        c = a.cands[q];
+        pg = a.slots + q;
+        res_idx = a.slot_result ? a.slot_result[q] : -1;
+        sidx = a.slot_index ? a.slot_index[q] : q;
+      }
     }
-    const int32_t n = pg->n;
-    const int32_t Vraw = pg->V;
     const uint32_t *__restrict__ card = pg->card;
     const T *__restrict__ costp = (const T *)pg->costp;
     const T *__restrict__ pe_comm = (const T *)pg->pe_comm;
+    const int32_t n = pg->n;
+    const int32_t Vraw = pg->V;
     const uint32_t *__restrict__ posm = pg->pos;
 
     // ---------------------------------------------------------- validate
     int np = 0;
-    uint8_t st = 0;  // candidate status
+    uint8_t st = 0;
     bool defer = false;
-    if (a.mode != 2) {
-      if (c.kind == 0) {
-      } else if (c.kind == 1) {
-        np = c.n_pins;
-        if (np < 1 || np > MAXPINS) st = 2;
-        else {
-          bool bad = false;
-          for (int k = 0; k < np; k++) {
-            int32_t o = c.pin_op[k];
-            if (o < 0 || o >= Vraw || posm[o] == NONE || c.pin_dev[k] >= G) bad = true;
-            for (int k2 = 0; k2 < k; k2++) bad |= c.pin_op[k2] == o;
+    if (active) {
+      if (a.mode != 2) {
+        if (c.kind == 0) {
+        } else if (c.kind == 1) {
+          np = c.n_pins;
+          if (np < 1 || np > MAXPINS) st = 2;
+          else {
+            bool bad = false;
+            for (int k = 0; k < np; k++) {
+              int32_t o = c.pin_op[k];
+              if (o < 0 || o >= Vraw || posm[o] == NONE || c.pin_dev[k] >= G) bad = true;
+              for (int k2 = 0; k2 < k; k2++) bad |= c.pin_op[k2] == o;
+            }
+            if (bad) st = 2;
           }
-          if (bad) st = 2;
-        }
-      } else if (c.kind == 2) {
-        int32_t o = c.split_op;
-        if (o < 0 || o >= Vraw || posm[o] == NONE || c.split_dim > 1 || !(a.split_mask[o] & (1u << c.split_dim)) ||
-            c.split_n < 2 || c.split_n > G)
+        } else if (c.kind == 2) {
+          int32_t o = c.split_op;
+          if (o < 0 || o >= Vraw || posm[o] == NONE || c.split_dim > 1 ||
+              !(a.split_mask[o] & (1u << c.split_dim)) || c.split_n < 2 || c.split_n > G)
+            st = 2;
+          else defer = true;
+        } else {
           st = 2;
-        else defer = true;
+        }
       } else {
-        st = 2;
+        np = c.kind == 1 ? c.n_pins : 0;
       }
-    } else {
-      np = c.kind == 1 ? c.n_pins : 0;
     }
-    // pins of this candidate: lane k < np holds pin k (as a position)
-    uint32_t my_pos = NONE;
-    int my_dev = 0;
-    if (st == 0 && lane < np) {
-      my_pos = posm[c.pin_op[lane]];
-      my_dev = c.pin_dev[lane];
-    }
-    // ------------------------------------------- classify (modes 0 and 1)
-    if (st == 0 && !defer && a.mode != 2 && np > 0)
-      defer = __any_sync(FULL, lane < np && pin_changes_ranks<T>(pg, gc, c, np, my_pos, my_dev, G, K));
-    if (defer) {
-      if (lane == 0) {
-        unsigned long long k = atomicAdd(a.ndefer, 1ull);
-        a.defer_q[k] = q;
+    if (st) np = 0;
+    // the candidate's pins as group-uniform arrays (positions, packed devices)
+    uint32_t pp[MAXPINS] = {NONE, NONE, NONE, NONE};
+    uint32_t pdv = 0;
+    if (active && !defer)
+      for (int k = 0; k < np; k++) {
+        pp[k] = posm[c.pin_op[k]];
+        pdv |= (uint32_t)c.pin_dev[k] << (8 * k);
       }
-      continue;
+    // classify (modes 0, 1): pins that change w or c send the candidate to
+    // the preparation pipeline
+    {
+      bool chg = false;
+      if (active && !defer && a.mode != 2)
+        for (int k = d; k < np; k += GP) chg |= pin_changes_ranks<T>(pg, gc, c, np, posm[c.pin_op[k]], c.pin_dev[k], G, K);
+      if ((__ballot_sync(FULL, chg) & gm) != 0) defer = true;
     }
-    if (st != 0) {
-      if (lane == 0 && res_idx >= 0) {
-        a.out.makespan[res_idx] = I64MAX;
-        a.out.status[res_idx] = st;
-      }
-      if (a.out.peak && res_idx >= 0 && lane < G) a.out.peak[res_idx * G + lane] = -1;
-      continue;
+    if (active && defer && d == 0) {
+      unsigned long long k = atomicAdd(a.ndefer, 1ull);
+      a.defer_q[k] = q;
     }
+    if (active && !defer && st && d == 0 && res_idx >= 0) {
+      a.out.makespan[res_idx] = I64MAX;
+      a.out.status[res_idx] = st;
+    }
+    if (active && !defer && st && res_idx >= 0 && a.out.peak && d < G) a.out.peak[res_idx * G + d] = -1;
+    const bool run = active && !defer && st == 0;
 
     // ------------------------------------------------------ prologue
-    const int32_t nwords = (n + 31) >> 5;
-    const int32_t nsumm = (nwords + 31) >> 5;
     uint32_t top = 0;
-    for (int32_t s = 0; s < nsumm; s++) {
-      int32_t w = s * 32 + lane;
-      uint32_t word = w < nwords ? __ldg(pg->srcbits + w) : 0u;
-      if (w < nwords) leaf[w] = word;
-      unsigned m = __ballot_sync(FULL, word != 0);
-      if (lane == 0) summ[s] = m;
-      if (m) top |= 1u << s;
+    if (run) {
+      const int32_t nwords = (n + 31) >> 5;
+      for (int32_t w = d; w < nwords; w += GP) leaf[w] = __ldg(pg->srcbits + w);
+      for (int32_t s = d; s < 32; s += GP) summ[s] = __ldg(pg->srcsumm + s);
+      top = __ldg(pg->srcsumm + 32);
+      for (int32_t p = d; p < n; p += GP) Slab<T>::init(slab, (uint32_t)p, __ldg(pg->npred + p));
     }
-    for (int32_t p = lane; p < n; p += 32) Slab<T>::init(slab, (uint32_t)p, __ldg(pg->npred + p));
     int64_t used = 0, reserved = 0;
-    T makespan = 0;
-    bool infeasible = false;
-
-    // CP devices (Alg. 1 line 5, R9) in free-index space
     uint32_t r_lo = 0, r_hi = 0;
-    int r_dev = -1;
-    int nrounds = 0;
-    uint32_t my_pcp = NONE;  // CP index of this lane's pinned op
-    if (cp_on && pg->cp_len > 0)
-      cp_rounds<T>(pg, np, my_pos, lane, dl, G, cap_d, r_lo, r_hi, r_dev, nrounds, my_pcp, reserved);
+    int r_dev = -1, nrounds = 0;
+    uint32_t pcp[MAXPINS] = {NONE, NONE, NONE, NONE};
+    if (run && cp_on && pg->cp_len > 0)
+      cp_rounds_g<T>(pg, np, pp, gm, gb, d, G, cap_d, r_lo, r_hi, r_dev, nrounds, pcp, reserved);
+    // groups of >= 4 lanes hold pin k in lane k; narrower groups keep the arrays
+    uint32_t my_pos = NONE, my_pcp = NONE;
+    int my_dev = 0;
+    if (GP >= 4) {
+      my_pos = d == 0 ? pp[0] : d == 1 ? pp[1] : d == 2 ? pp[2] : d == 3 ? pp[3] : NONE;
+      my_pcp = d == 0 ? pcp[0] : d == 1 ? pcp[1] : d == 2 ? pcp[2] : d == 3 ? pcp[3] : NONE;
+      my_dev = d < 4 ? (int)((pdv >> (8 * d)) & 0xFF) : 0;
+    }
+    if (d == 0) {
+      s_res[lead] = res_idx;
+      s_sidx[lead] = sidx;
+    }
     __syncwarp();
+    const bool any_pins = __any_sync(FULL, np > 0);
+    const bool any_cp = __any_sync(FULL, nrounds > 0);
+    const bool want_out = run && res_idx >= 0 && a.out.place != nullptr;
+    const bool any_out = __any_sync(FULL, want_out);
+    const int64_t ob = want_out ? res_idx * (int64_t)a.out.vmax : 0;
 
     // ---------------------------------------------------------- main loop
-    if (lane == 0) {
-      s_res[wib] = res_idx;
-      s_sidx[wib] = sidx;
-      s_pg[wib] = pg;
-    }
-    __syncwarp();
-    {
-      const bool want_out = res_idx >= 0 && a.out.place != nullptr;
-      const int64_t ob = want_out ? res_idx * (int64_t)a.out.vmax : 0;
-      LoopOut lo = sim_loop<T, GSH, MEM>(leaf, summ, top, slab, card, costp, pe_comm, pg, a.gc, G, K, my_pos, my_dev,
-                                         np, r_lo, r_hi, r_dev, nrounds, my_pcp, cap_d, used, reserved, cap_chk,
-                                         want_out ? a.out.place + ob : nullptr,
-                                         want_out && a.out.start ? a.out.start + ob : nullptr,
-                                         want_out && a.out.deq ? a.out.deq + ob : nullptr);
-      makespan = (T)lo.makespan;
-      infeasible = lo.infeasible != 0;
-      used = lo.used;
-    }
-    // ------------------------------------------------------------ epilogue
-    int64_t ms64 = infeasible ? I64MAX : (int64_t)makespan;
-    const int64_t res_idx2 = s_res[wib], sidx2 = s_sidx[wib];
-    const int64_t obase = res_idx2 >= 0 ? res_idx2 * (int64_t)a.out.vmax : 0;
-    if (res_idx2 >= 0) {
-      if (lane == 0) {
-        a.out.makespan[res_idx2] = ms64;
-        a.out.status[res_idx2] = infeasible ? 1 : 0;
+    T avail = 0, makespan = 0;
+    int32_t seq = 0;
+    bool infeas = false;
+    while (__any_sync(FULL, top != 0)) {
+      const bool live = top != 0;
+      // pop: highest priority = lowest position = lowest set bit
+      const int s = live ? __ffs(top) - 1 : 0;
+      const uint32_t m = summ[s];
+      const int b = m ? __ffs(m) - 1 : 0;
+      const int w = (s << 5) + b;
+      const uint32_t lw = leaf[w];
+      const uint32_t i = live ? ((uint32_t)w << 5) + (__ffs(lw) - 1) : 0u;
+      const uint32_t nlw = lw & (lw - 1);
+      const uint32_t nm = nlw ? m : (m & (m - 1));
+      __syncwarp();
+      if (live && d == 0) {
+        leaf[w] = nlw;
+        summ[s] = nm;
       }
-      if (a.out.peak && lane < G) a.out.peak[res_idx2 * G + lane] = infeasible ? -1 : used;
-      if (infeasible && a.out.place != nullptr) {
-        for (int32_t u = lane; u < a.out.vmax; u += 32) {
-          a.out.place[obase + u] = 0xFF;
-          if (a.out.start) a.out.start[obase + u] = -1;
-          if (a.out.deq) a.out.deq[obase + u] = -1;
+      if (live && !nm) top &= top - 1;
+
+      // round 1 (all from the op's card line): header, predecessor
+      // positions and comm, this lane's successor, cost on this lane's device
+      const uint32_t *cd = card + (size_t)i * CARD_WORDS;
+      const uint4 h0 = __ldg((const uint4 *)cd);
+      const uint4 hs = __ldg((const uint4 *)(cd + CARD_HDR));
+      uint4 hc = make_uint4(0, 0, 0, 0);
+      if (fastcomm) hc = __ldg((const uint4 *)(cd + CW_PCOMM));
+      const T cst = __ldg(costp + (size_t)i * G + (d < G ? d : 0));
+      const uint32_t s0 = __ldg(cd + CW_SUCC + (d < S_IN ? d : 0));
+      const uint32_t npred = live ? (h0.x & 0xFFFF) : 0u;
+      const uint32_t nsucc = live ? (h0.x >> 16) : 0u;
+      // round 2: predecessor records, successor indegree
+      const uint32_t src[4] = {hs.x, hs.y, hs.z, hs.w};
+      const uint32_t cmi[4] = {hc.x, hc.y, hc.z, hc.w};
+      T ft[4];
+      uint32_t pl[4];
+#pragma unroll
+      for (int k = 0; k < 4; k++) {
+        ft[k] = 0;
+        pl[k] = (uint32_t)d;
+        if ((uint32_t)k < npred) Slab<T>::load(slab, src[k], ft[k], pl[k]);
+      }
+      const uint32_t sdeg = ((uint32_t)d < nsucc) ? Slab<T>::indeg(slab, s0) : 1u;
+      // EST = max(avail[d], max_pred FT + c(pred -> i on d))   (R1, R6)
+      T est = avail;
+#pragma unroll
+      for (int k = 0; k < 4; k++) {
+        T cm;
+        if (fastcomm) cm = (T)cmi[k];
+        else cm = ((uint32_t)k < npred && pl[k] != (uint32_t)d && d < G)
+                      ? __ldg(pe_comm + (size_t)(h0.y + k) * K + gc.link_class[pl[k] * G + d])
+                      : (T)0;
+        const T term = ft[k] + (pl[k] == (uint32_t)d ? (T)0 : cm);
+        est = term > est ? term : est;
+      }
+      if (__any_sync(FULL, npred > 4u)) {
+        const uint32_t *pe_src = pg->pe_src;
+        for (uint32_t k = 4; __any_sync(FULL, k < npred); k++) {
+          if (k < npred) {
+            T f;
+            uint32_t p;
+            Slab<T>::load(slab, __ldg(pe_src + h0.y + k), f, p);
+            T cm = 0;
+            if (p != (uint32_t)d && d < G)
+              cm = K == 1 ? __ldg(pe_comm + h0.y + k) : __ldg(pe_comm + (size_t)(h0.y + k) * K + gc.link_class[p * G + d]);
+            const T term = f + cm;
+            est = term > est ? term : est;
+          }
         }
       }
+      const T eft = est + cst;
+
+      // device forced by a perturbation pin (hard) or a CP pin (Alg. 1 l.9-10)
+      int forced = -1;
+      bool pert = false;
+      if (any_pins) {
+        if (GP >= 4) {
+          const unsigned pm = __ballot_sync(FULL, live && my_pos == i) & gm;
+          const int fd = __shfl_sync(FULL, my_dev, pm ? __ffs(pm) - 1 : lane);
+          if (pm) {
+            forced = fd;
+            pert = true;
+          }
+        } else {
+#pragma unroll
+          for (int k = 0; k < MAXPINS; k++)
+            if (live && pp[k] == i) {
+              forced = (int)((pdv >> (8 * k)) & 0xFF);
+              pert = true;
+            }
+        }
+      }
+      if (any_cp) {
+        const uint32_t cpidx = h0.w;
+        uint32_t below;
+        if (GP >= 4) below = __popc(__ballot_sync(FULL, d < np && my_pcp < cpidx) & gm);
+        else below = (pcp[0] < cpidx) + (pcp[1] < cpidx) + (pcp[2] < cpidx) + (pcp[3] < cpidx);
+        const uint32_t fi = cpidx - below;
+        const unsigned rm = __ballot_sync(FULL, live && forced < 0 && cpidx != NONE && d < nrounds && fi >= r_lo &&
+                                                    fi < r_hi) & gm;
+        const int rd = __shfl_sync(FULL, r_dev, rm ? __ffs(rm) - 1 : lane);
+        if (rm) forced = rd;
+      }
+      int64_t mem = 0;
+      if (MEM) mem = (int64_t)(((uint64_t)__ldg(cd + CW_MEMHI) << 32) | __ldg(cd + CW_MEMLO));
+      bool feas = live && d < G && (forced < 0 || d == forced);
+      if (cap_chk && (forced < 0 || pert)) feas = feas && (used + reserved + mem <= cap_d);
+      // argmin EFT over feasible devices, ties -> lowest device (Alg. 1 l.12-19, R3, R8)
+      const T key = feas ? eft : TT<T>::MAXV;
+      T mn = key;
+#pragma unroll
+      for (int o = GP >> 1; o >= 1; o >>= 1) {
+        const T x = __shfl_xor_sync(FULL, mn, o);
+        mn = x < mn ? x : mn;
+      }
+      const unsigned fm = __ballot_sync(FULL, feas && key == mn) & gm;
+      if (live && !fm) {
+        infeas = true;
+        top = 0;
+      }
+      const bool go = live && fm != 0;
+      const int dsel = fm ? __ffs(fm) - 1 - gb : 0;
+      if (go && d == dsel) {
+        avail = mn;
+        if (MEM) {
+          used += mem;
+          if (forced >= 0 && !pert) reserved -= mem;
+        }
+      }
+      if (go) makespan = mn > makespan ? mn : makespan;
+      if (go && d == 0) Slab<T>::sched(slab, i, mn, (uint32_t)dsel);
+      if (any_out) {
+        const T stt = __shfl_sync(FULL, est, gb + dsel);
+        if (go && want_out && d == 0) {
+          const uint32_t u = __ldg(cd + CW_UID);
+          a.out.place[ob + u] = (uint8_t)dsel;
+          if (a.out.start) a.out.start[ob + u] = (int64_t)stt;
+          if (a.out.deq) a.out.deq[ob + seq] = (int32_t)u;
+        }
+        seq++;
+      }
+      // release successors into the ready bitmap
+      uint32_t bits = 0;
+      if (go && (uint32_t)d < nsucc) {
+        const uint32_t dg = sdeg - 1;
+        Slab<T>::set_indeg(slab, s0, dg);
+        if (dg == 0) {
+          atomicOr(&leaf[s0 >> 5], 1u << (s0 & 31));
+          atomicOr(&summ[s0 >> 10], 1u << ((s0 >> 5) & 31));
+          bits = 1u << (s0 >> 10);
+        }
+      }
+      if (__any_sync(FULL, go && nsucc > (uint32_t)GP)) {
+        for (uint32_t kk = GP + d; __any_sync(FULL, go && kk - d < nsucc); kk += GP) {
+          if (go && kk < nsucc) {
+            const uint32_t dst = kk < (uint32_t)S_IN ? __ldg(cd + CW_SUCC + kk) : __ldg(pg->se_dst + h0.z + kk);
+            const uint32_t dg = Slab<T>::indeg(slab, dst) - 1;
+            Slab<T>::set_indeg(slab, dst, dg);
+            if (dg == 0) {
+              atomicOr(&leaf[dst >> 5], 1u << (dst & 31));
+              atomicOr(&summ[dst >> 10], 1u << ((dst >> 5) & 31));
+              bits |= 1u << (dst >> 10);
+            }
+          }
+        }
+      }
+#pragma unroll
+      for (int o = GP >> 1; o >= 1; o >>= 1) bits |= __shfl_xor_sync(FULL, bits, o);
+      top |= bits;
+      __syncwarp();
     }
-    if (lane == 0 && !infeasible && (ms64 < s_best[wib][0] || (ms64 == s_best[wib][0] && sidx2 < s_best[wib][1]))) {
-      s_best[wib][0] = ms64;
-      s_best[wib][1] = sidx2;
-    }
-    // clear the smem bitmap left by an aborted (infeasible) run
-    if (infeasible) {
-      for (int32_t w = lane; w < a.leaf_words; w += 32) leaf[w] = 0;
-      summ[lane] = 0;
+
+    // ------------------------------------------------------------ epilogue
+    if (run) {
+      const int64_t ms64 = infeas ? I64MAX : (int64_t)makespan;
+      const int64_t ri = s_res[lead], si = s_sidx[lead];
+      if (ri >= 0) {
+        if (d == 0) {
+          a.out.makespan[ri] = ms64;
+          a.out.status[ri] = infeas ? 1 : 0;
+        }
+        if (a.out.peak && d < G) a.out.peak[ri * G + d] = infeas ? -1 : used;
+        if (infeas && a.out.place != nullptr) {
+          const int64_t o2 = ri * (int64_t)a.out.vmax;
+          for (int32_t u = d; u < a.out.vmax; u += GP) {
+            a.out.place[o2 + u] = 0xFF;
+            if (a.out.start) a.out.start[o2 + u] = -1;
+            if (a.out.deq) a.out.deq[o2 + u] = -1;
+          }
+        }
+      }
+      if (d == 0 && !infeas && (ms64 < s_best[lead][0] || (ms64 == s_best[lead][0] && si < s_best[lead][1]))) {
+        s_best[lead][0] = ms64;
+        s_best[lead][1] = si;
+      }
     }
     __syncwarp();
   }
   __syncwarp();
-  if (a.track_best && lane == 0) {
-    a.wbest[2 * gwarp] = s_best[wib][0];
-    a.wbest[2 * gwarp + 1] = s_best[wib][1];
+  if (a.track_best && d == 0) {
+    a.wbest[2 * cslot] = s_best[lead][0];
+    a.wbest[2 * cslot + 1] = s_best[lead][1];
   }
 }
 
@@ -764,9 +730,11 @@ int sim_occupancy(int tbits, int gshift, int block, size_t smem) {
   return nb;
 }
 cudaError_t sim_set_smem(int tbits, int gshift, size_t smem) {
-  cudaError_t e = cudaFuncSetAttribute(sim_fn(tbits, gshift, false), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(sim_fn(tbits, gshift, true), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  for (int mem = 0; mem < 2; mem++) {
+    cudaError_t e = cudaFuncSetAttribute(sim_fn(tbits, gshift, mem), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
 }
 
 // ------------------------------------------------------------------ argmin
