@@ -9,6 +9,7 @@
 #include <algorithm>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <deque>
 #include <mutex>
@@ -171,11 +172,24 @@ struct Base {
   PrepGraph *pg_dev = nullptr;
   int tbits = 64, key_bits = 64;
   unsigned long long bound = 0, maxextra = 0;
+  // recorded BASE schedule for prefix sharing, per CP-pin flag value
+  struct Snap {
+    bool valid = false;
+    int round_dev = -1;
+    char *buf = nullptr;  // dq | avail | ms | rec | rounds
+    uint32_t *dq = nullptr;
+    void *avail = nullptr, *ms = nullptr, *rec = nullptr;
+    int32_t *rounds = nullptr;
+  } snap[2];
   void release() {
     cudaFree(raw_block);
     cudaFree(raw_dev);
     cudaFree(prep_block);
     cudaFree(pg_dev);
+    for (auto &x : snap) {
+      cudaFree(x.buf);
+      x = Snap();
+    }
     raw_block = prep_block = nullptr;
     raw_dev = nullptr;
     pg_dev = nullptr;
@@ -235,6 +249,13 @@ struct fastt_graph {
   // instrumentation
   int64_t launches = 0;
   fastt_timing last;
+  bool share = true;  // BASE-schedule prefix sharing (env FASTT_NO_SHARE=1 disables, for A/B checks)
+  // start-step sorted candidate lists for prefix sharing
+  char *sort_buf = nullptr;
+  int64_t sort_cap = 0;
+  Cand *srt_tmp_c = nullptr, *srt_c = nullptr;
+  int64_t *srt_tmp_i = nullptr, *srt_i = nullptr, *srt_res = nullptr;
+  uint32_t *srt_key = nullptr, *srt_hist = nullptr;
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
   std::mutex mu;
 };
@@ -465,6 +486,97 @@ static fastt_status run_prep(fastt_graph *g, const Base &B, int nslots, cudaStre
   return FASTT_OK;
 }
 
+// Record the BASE schedule of base B under `flags` (one BASE run in
+// snap_mode 1): per-position dequeue index, final records, avail and
+// makespan before every step, the base CP rounds.
+static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cudaStream_t st) {
+  Base::Snap &S = B.snap[flags & FASTT_F_CP_PIN ? 1 : 0];
+  if (S.valid) return FASTT_OK;
+  for (int d = 0; d < g->G; d++)
+    if (g->gch.cap[d] != I64MAX) return FASTT_OK;  // sharing needs unlimited memory
+  const size_t tb = B.tbits / 8, n = (size_t)B.pl.ncap;
+  const size_t o_dq = 0, o_av = al16(4 * n), o_ms = o_av + al16(tb * (n + 1) * g->G),
+               o_rec = o_ms + al16(tb * (n + 1)), o_rd = o_rec + al16((B.tbits == 32 ? 8 : 16) * n),
+               tot = o_rd + 64;
+  CK(cudaMalloc(&S.buf, tot));
+  S.dq = (uint32_t *)(S.buf + o_dq);
+  S.avail = S.buf + o_av;
+  S.ms = S.buf + o_ms;
+  S.rec = S.buf + o_rec;
+  S.rounds = (int32_t *)(S.buf + o_rd);
+  CK(cudaMemsetAsync(S.rounds, 0, 16, st));
+  Cand c;
+  memset(&c, 0, sizeof c);
+  c.split_op = -1;
+  for (int k = 0; k < 4; k++) c.pin_op[k] = -1;
+  Cand *d_c;
+  int64_t *d_ms;
+  uint8_t *d_st;
+  CK(cudaMalloc(&d_c, sizeof c));
+  CK(cudaMalloc(&d_ms, 8));
+  CK(cudaMalloc(&d_st, 8));
+  CK(cudaMemcpyAsync(d_c, &c, sizeof c, cudaMemcpyHostToDevice, st));
+  TRY(ensure_sim(g, B, 1));
+  CK(cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), st));
+  SimArgs a = sim_args(g, B, flags);
+  a.mode = 1;
+  a.cands = d_c;
+  a.n = 1;
+  a.out.makespan = d_ms;
+  a.out.status = d_st;
+  a.snap_mode = 1;
+  a.snap_dq = S.dq;
+  a.snap_avail = S.avail;
+  a.snap_ms = S.ms;
+  a.snap_rec = S.rec;
+  a.snap_rounds = S.rounds;
+  launch_sim(a, B.tbits, 1, g->sim_block, g->sim_smem, st);
+  g->launches += NL_SIM;
+  CK(cudaGetLastError());
+  int32_t rd[4];
+  uint8_t hst = 0;
+  CK(cudaMemcpyAsync(rd, S.rounds, 16, cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(&hst, d_st, 1, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  cudaFree(d_c);
+  cudaFree(d_ms);
+  cudaFree(d_st);
+  if (hst != FASTT_CAND_OK) return FASTT_OK;  // (cannot happen without caps)
+  S.round_dev = (rd[0] == 1 && rd[2] == 0 && rd[3] == B.cp_len) ? rd[1] : -1;
+  S.valid = true;
+  return FASTT_OK;
+}
+
+// enable prefix sharing on a launch when the snapshot exists
+static void use_snapshot(const Base &B, uint32_t flags, SimArgs &a) {
+  const Base::Snap &S = B.snap[flags & FASTT_F_CP_PIN ? 1 : 0];
+  if (!S.valid || a.need_mem || a.out.place) return;
+  a.snap_mode = 2;
+  a.snap_round_dev = S.round_dev;
+  a.snap_dq = S.dq;
+  a.snap_avail = S.avail;
+  a.snap_ms = S.ms;
+  a.snap_rec = S.rec;
+}
+
+static fastt_status ensure_sort_buf(fastt_graph *g, int64_t n) {
+  if (g->sort_cap >= n) return FASTT_OK;
+  cudaFree(g->sort_buf);
+  const int64_t c = std::max<int64_t>(n, 4096);
+  const size_t oc = 0, oc2 = al16(32 * c), oi = oc2 + al16(32 * c), oi2 = oi + al16(8 * c), ores = oi2 + al16(8 * c),
+               ok = ores + al16(8 * c), oh = ok + al16(4 * c), tot = oh + 4096;
+  CK(cudaMalloc(&g->sort_buf, tot));
+  g->srt_tmp_c = (Cand *)(g->sort_buf + oc);
+  g->srt_c = (Cand *)(g->sort_buf + oc2);
+  g->srt_tmp_i = (int64_t *)(g->sort_buf + oi);
+  g->srt_i = (int64_t *)(g->sort_buf + oi2);
+  g->srt_res = (int64_t *)(g->sort_buf + ores);
+  g->srt_key = (uint32_t *)(g->sort_buf + ok);
+  g->srt_hist = (uint32_t *)(g->sort_buf + oh);
+  g->sort_cap = c;
+  return FASTT_OK;
+}
+
 struct DevOut {
   int64_t *makespan = nullptr;
   uint8_t *status = nullptr;
@@ -481,6 +593,8 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
                                cudaStream_t st, DevOut o) {
   if (n <= 0) return FASTT_OK;
   TRY(ensure_sim(g, B, n));
+  const bool sharing = g->share && !o.peak && !o.place && n >= 64;
+  if (sharing) TRY(ensure_snapshot(g, B, flags, st));  // before the work counters are reset
   if (o.place) CK(cudaMemsetAsync(o.place, 0xFF, (size_t)n * o.vmax, st));
   if (o.start) {
     launch_fill_i64(o.start, n * o.vmax, -1, st);
@@ -500,6 +614,22 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
   a.out.start = o.start;
   a.out.deq = o.deq;
   a.out.vmax = (int32_t)o.vmax;
+  if (sharing) use_snapshot(B, flags, a);
+  const bool sorted = a.snap_mode == 2;
+  if (sorted) {
+    // order the list by BASE-prefix start step (results keep their index)
+    TRY(ensure_sort_buf(g, n));
+    const PrepGraph P = prep_struct(B.prep_block, B.pl, B.tbits);
+    StreamState dummy;
+    memset(&dummy, 0, sizeof dummy);
+    launch_t0_sort(0, dummy, 0, 1, d_cands, n, P.pos, a.snap_dq, B.n, B.V, g->G, g->srt_tmp_c, g->srt_tmp_i,
+                   g->srt_key, g->srt_hist, g->srt_c, g->srt_i, g->srt_res, st);
+    g->launches += 4;
+    a.mode = 3;
+    a.cands = g->srt_c;
+    a.slot_index = g->srt_i;
+    a.slot_result = g->srt_res;
+  }
   launch_sim(a, B.tbits, g->sim_grid, g->sim_block, g->sim_smem, st);
   g->launches += NL_SIM;
   CK(cudaGetLastError());
@@ -511,7 +641,9 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
     TRY(ensure_arena(g, B, st));
     for (int64_t c0 = 0; c0 < (int64_t)nd; c0 += g->arena_slots) {
       int nc = (int)std::min<int64_t>(g->arena_slots, (int64_t)nd - c0);
-      launch_gather_cands(d_cands, g->defer_q + c0, nc, g->slot_cands, g->slot_result, st);
+      if (sorted) launch_gather_sorted(g->srt_c, g->srt_i, g->srt_res, g->defer_q + c0, nc, g->slot_cands, nullptr,
+                                       g->slot_result, st);
+      else launch_gather_cands(d_cands, g->defer_q + c0, nc, g->slot_cands, g->slot_result, st);
       g->launches += NL_GATHER + NL_SIM;
       TRY(run_prep(g, B, nc, st));
       CK(cudaMemsetAsync(g->counters, 0, sizeof(unsigned long long), st));
@@ -855,6 +987,10 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
   g->v_max = V + maxov;
   g->gch = gc;
   g->split_mask_h.assign(d->split_mask, d->split_mask + V);
+  {
+    const char *e = getenv("FASTT_NO_SHARE");
+    g->share = !(e && e[0] == '1');
+  }
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || cuda_device < 0 || cuda_device >= ndev) {
     delete g;
@@ -947,6 +1083,7 @@ void fastt_free_graph(fastt_graph *g) {
     cudaFree(g->scratch_cp);
     cudaFree(g->scratch_list);
     cudaFree(g->scratch_n);
+    cudaFree(g->sort_buf);
     for (auto &e : g->ev)
       if (e) cudaEventDestroy(e);
   }
@@ -1152,6 +1289,7 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
     }
     CK(cudaMemcpyAsync(g->wbest, init.data(), 16 * nwarps, cudaMemcpyHostToDevice, st));
   }
+  if (g->share) TRY(ensure_snapshot(g, B, flags, st));
   TRY(timing_begin(g, flags, st));
   unsigned long long nd = 0;
   if (n > 0) {
@@ -1163,6 +1301,18 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
     a.n = n;
     a.stride = stride;
     a.track_best = 1;
+    if (g->share) use_snapshot(B, flags, a);
+    if (a.snap_mode == 2) {
+      TRY(ensure_sort_buf(g, n));
+      const PrepGraph P = prep_struct(B.prep_block, B.pl, B.tbits);
+      launch_t0_sort(1, a.stream, first, stride, nullptr, n, P.pos, a.snap_dq, B.n, B.V, g->G, g->srt_tmp_c,
+                     g->srt_tmp_i, g->srt_key, g->srt_hist, g->srt_c, g->srt_i, nullptr, st);
+      g->launches += 4;
+      a.mode = 3;
+      a.cands = g->srt_c;
+      a.slot_index = g->srt_i;
+      a.slot_result = nullptr;
+    }
     launch_sim(a, B.tbits, g->sim_grid, g->sim_block, g->sim_smem, st);
     g->launches += NL_SIM;
     CK(cudaGetLastError());
@@ -1173,7 +1323,9 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
       TRY(ensure_arena(g, B, st));
       for (int64_t c0 = 0; c0 < (int64_t)nd; c0 += g->arena_slots) {
         int nc = (int)std::min<int64_t>(g->arena_slots, (int64_t)nd - c0);
-        launch_candgen_idx(a.stream, first, stride, g->defer_q + c0, nc, g->slot_cands, g->slot_index, st);
+        if (a.mode == 3) launch_gather_sorted(g->srt_c, g->srt_i, nullptr, g->defer_q + c0, nc, g->slot_cands,
+                                              g->slot_index, nullptr, st);
+        else launch_candgen_idx(a.stream, first, stride, g->defer_q + c0, nc, g->slot_cands, g->slot_index, st);
         g->launches += NL_CANDGEN + NL_SIM;
         TRY(run_prep(g, B, nc, st));
         CK(cudaMemsetAsync(g->counters, 0, sizeof(unsigned long long), st));

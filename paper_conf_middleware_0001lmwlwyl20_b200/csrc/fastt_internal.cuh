@@ -153,7 +153,7 @@ struct SimOut {
 };
 
 struct SimArgs {
-  int mode;              // 0 sweep, 1 list, 2 prepared slots
+  int mode;              // 0 sweep, 1 list, 2 prepared slots, 3 permuted list (slot_index/slot_result)
   uint32_t flags;
   const PrepGraph *base; // base prepared graph (modes 0, 1)
   const PrepGraph *slots;// prepared slot graphs (mode 2)
@@ -178,6 +178,15 @@ struct SimArgs {
   int32_t track_best;
   int32_t need_mem;      // track per-device memory (caps present or peak output)
   int32_t cap_check;     // some device has a finite memory cap (R8)
+  // BASE-schedule prefix sharing: 1 = record the snapshot (one BASE run),
+  // 2 = start eligible PIN candidates from it at their first pinned op
+  int32_t snap_mode;
+  int32_t snap_round_dev;  // device of the base's single CP round covering the whole CP, else -1
+  uint32_t *snap_dq;       // [n] dequeue index of each position in the BASE schedule
+  void *snap_avail;        // [(n+1)*G] T: avail[d] before step t
+  void *snap_ms;           // [n+1] T: makespan before step t
+  void *snap_rec;          // [n] final slab records of the BASE schedule
+  int32_t *snap_rounds;    // [4] base CP rounds: count, dev0, lo0, hi0 (written when recording)
 };
 
 void launch_sim(const SimArgs &a, int tbits, int grid, int block, size_t smem, cudaStream_t st);
@@ -191,6 +200,12 @@ void launch_candgen_idx(const StreamState &s, int64_t first, int64_t stride, con
 void launch_slot_setup(const Cand *cands, const RawGraph *tmpl, const RawGraph *base, RawGraph *raws, int nslots,
                        cudaStream_t st);
 void launch_gather_cands(const Cand *src, const int64_t *idx, int64_t n, Cand *dst, int64_t *res, cudaStream_t st);
+void launch_t0_sort(int from_stream, const StreamState &S, int64_t first, int64_t stride, const Cand *list, int64_t n,
+                    const uint32_t *pos, const uint32_t *snap_dq, int32_t nops, int32_t vraw, int G, Cand *tmp_c,
+                    int64_t *tmp_i, uint32_t *key, uint32_t *hist, Cand *out_c, int64_t *out_i, int64_t *out_res,
+                    cudaStream_t st);
+void launch_gather_sorted(const Cand *src, const int64_t *sidx, const int64_t *sres, const int64_t *qs, int64_t n,
+                          Cand *dst, int64_t *didx, int64_t *dres, cudaStream_t st);
 int sim_occupancy(int tbits, int gshift, int block, size_t smem);
 cudaError_t sim_set_smem(int tbits, int gshift, size_t smem);
 void launch_fill_i64(int64_t *p, int64_t n, int64_t v, cudaStream_t st);

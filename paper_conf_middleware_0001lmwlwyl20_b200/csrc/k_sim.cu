@@ -61,6 +61,7 @@ template <> struct Slab<uint32_t> {
   __device__ static void sched(W *s, uint32_t p, uint32_t ft, uint32_t plc) {
     s[p] = ((unsigned long long)plc << 32) | ft;
   }
+  __device__ static void make(W &w, uint32_t ft, uint32_t plc) { w = ((unsigned long long)plc << 32) | ft; }
 };
 template <> struct Slab<uint64_t> {
   typedef ulonglong2 W;
@@ -85,6 +86,10 @@ template <> struct Slab<uint64_t> {
     w.y = plc;
     s[p] = w;
   }
+  __device__ static void make(W &w, uint64_t ft, uint32_t plc) {
+    w.x = ft;
+    w.y = plc;
+  }
 };
 
 __device__ __forceinline__ uint64_t splitmix64(uint64_t &s) {
@@ -94,6 +99,35 @@ __device__ __forceinline__ uint64_t splitmix64(uint64_t &s) {
   z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
   return z ^ (z >> 31);
 }
+
+
+#ifndef SIM_PEEK
+#define SIM_PEEK 0
+#endif
+#ifndef SIM_ASM_SMEM
+#define SIM_ASM_SMEM 0
+#endif
+// 32-bit shared-memory accessors for the ready bitmap
+#if SIM_ASM_SMEM
+__device__ __forceinline__ uint32_t lds32(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts32(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void red_or_s(uint32_t a, uint32_t v) {
+  asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+#else
+extern __shared__ uint32_t smem[];
+__device__ __forceinline__ uint32_t *sptr(uint32_t a) { return (uint32_t *)__cvta_shared_to_generic(a); }
+__device__ __forceinline__ uint32_t lds32(uint32_t a) { return *sptr(a); }
+__device__ __forceinline__ void sts32(uint32_t a, uint32_t v) { *sptr(a) = v; }
+__device__ __forceinline__ void red_or_s(uint32_t a, uint32_t v) { atomicOr(sptr(a), v); }
+#endif
+__device__ __forceinline__ void prefetch_l2(const void *p) { asm volatile("prefetch.global.L2 [%0];" ::"l"(p)); }
 
 // R21: the c-th candidate of the sweep stream
 __device__ Cand stream_cand(const StreamState &S, int64_t c) {
@@ -351,7 +385,11 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
   const int64_t cslot = gwarp * CPW + grp;
   uint32_t *leaf = smem + (uint32_t)(wib * CPW + grp) * (uint32_t)a.bm_stride;
   uint32_t *summ = leaf + a.leaf_words;
-  W *slab = (W *)a.slab + (size_t)cslot * (size_t)a.slab_stride;
+  const uint32_t leaf_sa = (uint32_t)__cvta_generic_to_shared(leaf);
+  const uint32_t summ_sa = (uint32_t)__cvta_generic_to_shared(summ);
+  W *const slab0 = (W *)a.slab;                                  // all slabs
+  const uint32_t sb = (uint32_t)(cslot * a.slab_stride);         // this candidate's slab (elements)
+  W *slab = slab0 + sb;
   const GraphConst &gc = *a.gc;
   const int G = a.G;
   const int K = gc.K;
@@ -383,6 +421,10 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       } else if (a.mode == 1) {
         c = a.cands[q];
         res_idx = q;
+      } else if (a.mode == 3) {  // candidate list ordered by BASE-prefix start step
+        c = a.cands[q];
+        res_idx = a.slot_result ? a.slot_result[q] : -1;
+        sidx = a.slot_index[q];
       } else {
         c = a.cands[q];
         pg = a.slots + q;
@@ -458,20 +500,102 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
     const bool run = active && !defer && st == 0;
 
     // ------------------------------------------------------ prologue
-    uint32_t top = 0;
-    if (run) {
-      const int32_t nwords = (n + 31) >> 5;
-      for (int32_t w = d; w < nwords; w += GP) leaf[w] = __ldg(pg->srcbits + w);
-      for (int32_t s = d; s < 32; s += GP) summ[s] = __ldg(pg->srcsumm + s);
-      top = __ldg(pg->srcsumm + 32);
-      for (int32_t p = d; p < n; p += GP) Slab<T>::init(slab, (uint32_t)p, __ldg(pg->npred + p));
-    }
     int64_t used = 0, reserved = 0;
     uint32_t r_lo = 0, r_hi = 0;
     int r_dev = -1, nrounds = 0;
     uint32_t pcp[MAXPINS] = {NONE, NONE, NONE, NONE};
     if (run && cp_on && pg->cp_len > 0)
       cp_rounds_g<T>(pg, np, pp, gm, gb, d, G, cap_d, r_lo, r_hi, r_dev, nrounds, pcp, reserved);
+    if (d == 0) {
+      s_res[lead] = res_idx;
+      s_sidx[lead] = sidx;
+    }
+    const bool want_out = run && res_idx >= 0 && a.out.place != nullptr;
+    // BASE-schedule prefix sharing: with the base ranks, the base CP devices
+    // for every free CP op and no memory caps, the candidate's schedule is the
+    // BASE schedule until its first pinned op is dequeued (step t0), so it
+    // starts from the recorded BASE state at t0 (exact)
+    int32_t t0 = 0;
+    bool share = false;
+    if (run && !MEM && !want_out && a.snap_mode == 2 && a.mode != 2) {
+      t0 = n;
+      for (int k = 0; k < np; k++) {
+        const int32_t dq = (int32_t)__ldg(a.snap_dq + pp[k]);
+        t0 = dq < t0 ? dq : t0;
+      }
+      share = true;
+      if (cp_on && pg->cp_len > 0) {
+        int m = 0;
+        for (int k = 0; k < np; k++) m += pcp[k] != NONE;
+        if (m > 0) {
+          // pinned CP ops change the free list: accept only one round over
+          // every free CP op on the base's single-round device
+          const uint32_t lo0 = __shfl_sync(gm, r_lo, gb), hi0 = __shfl_sync(gm, r_hi, gb);
+          const int dv0 = __shfl_sync(gm, r_dev, gb);
+          share = a.snap_round_dev >= 0 && nrounds == 1 && lo0 == 0 && (int32_t)hi0 == pg->cp_len - m &&
+                  dv0 == a.snap_round_dev;
+        }
+      }
+    }
+    uint32_t top = 0;
+    T avail = 0, makespan = 0;
+    if (run && share) {
+      avail = d < G ? __ldg((const T *)a.snap_avail + (size_t)t0 * G + d) : (T)0;
+      makespan = __ldg((const T *)a.snap_ms + t0);
+      if (t0 < n) {
+        const int32_t nwords = (n + 31) >> 5;
+        for (int32_t w = d; w < nwords; w += GP) leaf[w] = 0;
+        __syncwarp(gm);
+        const W *rec0 = (const W *)a.snap_rec;
+        for (int32_t p = d; p < n; p += GP) {
+          const uint32_t dq = __ldg(a.snap_dq + p);
+          if ((int32_t)dq < t0) {
+            slab[p] = rec0[p];
+          } else {
+            const uint32_t *cp_ = card + (size_t)p * CARD_WORDS;
+            const uint32_t npr = __ldg(cp_ + CW_DEG) & 0xFFFF;
+            const uint4 ps = __ldg((const uint4 *)(cp_ + CARD_HDR));
+            uint32_t cnt = 0;
+            if (npr > 0) cnt += (int32_t)__ldg(a.snap_dq + ps.x) >= t0;
+            if (npr > 1) cnt += (int32_t)__ldg(a.snap_dq + ps.y) >= t0;
+            if (npr > 2) cnt += (int32_t)__ldg(a.snap_dq + ps.z) >= t0;
+            if (npr > 3) cnt += (int32_t)__ldg(a.snap_dq + ps.w) >= t0;
+            if (npr > 4) {
+              const uint32_t pb = __ldg(cp_ + CW_PBASE);
+              for (uint32_t k = 4; k < npr; k++) cnt += (int32_t)__ldg(a.snap_dq + __ldg(pg->pe_src + pb + k)) >= t0;
+            }
+            Slab<T>::init(slab, (uint32_t)p, cnt);
+            if (cnt == 0) atomicOr(&leaf[p >> 5], 1u << (p & 31));
+          }
+        }
+        __syncwarp(gm);
+        uint32_t tb = 0;
+        for (int32_t sw = d; sw < 32; sw += GP) {
+          uint32_t word = 0;
+          for (int b = 0; b < 32; b++) {
+            const int32_t w = sw * 32 + b;
+            if (w < nwords && leaf[w]) word |= 1u << b;
+          }
+          summ[sw] = word;
+          if (word) tb |= 1u << sw;
+        }
+#pragma unroll
+        for (int o = GP >> 1; o >= 1; o >>= 1) tb |= __shfl_xor_sync(gm, tb, o);
+        top = tb;
+      }
+    } else if (run) {
+      const int32_t nwords = (n + 31) >> 5;
+      for (int32_t w = d; w < nwords; w += GP) leaf[w] = __ldg(pg->srcbits + w);
+      for (int32_t s = d; s < 32; s += GP) summ[s] = __ldg(pg->srcsumm + s);
+      top = __ldg(pg->srcsumm + 32);
+      for (int32_t p = d; p < n; p += GP) Slab<T>::init(slab, (uint32_t)p, __ldg(pg->npred + p));
+    }
+    if (a.snap_mode == 1 && run && d == 0) {
+      a.snap_rounds[0] = nrounds;
+      a.snap_rounds[1] = r_dev;
+      a.snap_rounds[2] = (int32_t)r_lo;
+      a.snap_rounds[3] = (int32_t)r_hi;
+    }
     // groups of >= 4 lanes hold pin k in lane k; narrower groups keep the arrays
     uint32_t my_pos = NONE, my_pcp = NONE;
     int my_dev = 0;
@@ -480,38 +604,29 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       my_pcp = d == 0 ? pcp[0] : d == 1 ? pcp[1] : d == 2 ? pcp[2] : d == 3 ? pcp[3] : NONE;
       my_dev = d < 4 ? (int)((pdv >> (8 * d)) & 0xFF) : 0;
     }
-    if (d == 0) {
-      s_res[lead] = res_idx;
-      s_sidx[lead] = sidx;
-    }
     __syncwarp();
     const bool any_pins = __any_sync(FULL, np > 0);
     const bool any_cp = __any_sync(FULL, nrounds > 0);
-    const bool want_out = run && res_idx >= 0 && a.out.place != nullptr;
     const bool any_out = __any_sync(FULL, want_out);
     const int64_t ob = want_out ? res_idx * (int64_t)a.out.vmax : 0;
+    const bool snap_rec_on = a.snap_mode == 1;
+    int32_t tstep = 0;
 
     // ---------------------------------------------------------- main loop
-    T avail = 0, makespan = 0;
     int32_t seq = 0;
     bool infeas = false;
+    const uint32_t la = leaf_sa, sa = summ_sa;  // shared-memory byte addresses
     while (__any_sync(FULL, top != 0)) {
       const bool live = top != 0;
       // pop: highest priority = lowest position = lowest set bit
       const int s = live ? __ffs(top) - 1 : 0;
-      const uint32_t m = summ[s];
+      const uint32_t m = lds32(sa + 4u * s);
       const int b = m ? __ffs(m) - 1 : 0;
       const int w = (s << 5) + b;
-      const uint32_t lw = leaf[w];
+      const uint32_t lw = lds32(la + 4u * w);
       const uint32_t i = live ? ((uint32_t)w << 5) + (__ffs(lw) - 1) : 0u;
       const uint32_t nlw = lw & (lw - 1);
       const uint32_t nm = nlw ? m : (m & (m - 1));
-      __syncwarp();
-      if (live && d == 0) {
-        leaf[w] = nlw;
-        summ[s] = nm;
-      }
-      if (live && !nm) top &= top - 1;
 
       // round 1 (all from the op's card line): header, predecessor
       // positions and comm, this lane's successor, cost on this lane's device
@@ -522,6 +637,24 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       if (fastcomm) hc = __ldg((const uint4 *)(cd + CW_PCOMM));
       const T cst = __ldg(costp + (size_t)i * G + (d < G ? d : 0));
       const uint32_t s0 = __ldg(cd + CW_SUCC + (d < S_IN ? d : 0));
+      // peek the next ready op (88% of pops on C5 are the op that was
+      // already next): its card now, its predecessor records prefetched
+      // into L2 at the end of this step
+      uint32_t jn = NONE;
+      if (SIM_PEEK && nlw) jn = ((uint32_t)w << 5) + (__ffs(nlw) - 1);
+      else if (SIM_PEEK && nm) {
+        const int w2 = (s << 5) + __ffs(nm) - 1;
+        const uint32_t l2 = lds32(la + 4u * w2);
+        jn = ((uint32_t)w2 << 5) + (__ffs(l2) - 1);
+      }
+      uint4 hn = make_uint4(0, 0, 0, 0);
+      if (SIM_PEEK && live && jn != NONE) hn = __ldg((const uint4 *)(card + (size_t)jn * CARD_WORDS + CARD_HDR));
+      __syncwarp();
+      if (live && d == 0) {
+        sts32(la + 4u * w, nlw);
+        sts32(sa + 4u * s, nm);
+      }
+      if (live && !nm) top &= top - 1;
       const uint32_t npred = live ? (h0.x & 0xFFFF) : 0u;
       const uint32_t nsucc = live ? (h0.x >> 16) : 0u;
       // round 2: predecessor records, successor indegree
@@ -533,9 +666,9 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       for (int k = 0; k < 4; k++) {
         ft[k] = 0;
         pl[k] = (uint32_t)d;
-        if ((uint32_t)k < npred) Slab<T>::load(slab, src[k], ft[k], pl[k]);
+        if ((uint32_t)k < npred) Slab<T>::load(slab0, sb + src[k], ft[k], pl[k]);
       }
-      const uint32_t sdeg = ((uint32_t)d < nsucc) ? Slab<T>::indeg(slab, s0) : 1u;
+      const uint32_t sdeg = ((uint32_t)d < nsucc) ? Slab<T>::indeg(slab0, sb + s0) : 1u;
       // EST = max(avail[d], max_pred FT + c(pred -> i on d))   (R1, R6)
       T est = avail;
 #pragma unroll
@@ -554,7 +687,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
           if (k < npred) {
             T f;
             uint32_t p;
-            Slab<T>::load(slab, __ldg(pe_src + h0.y + k), f, p);
+            Slab<T>::load(slab0, sb + __ldg(pe_src + h0.y + k), f, p);
             T cm = 0;
             if (p != (uint32_t)d && d < G)
               cm = K == 1 ? __ldg(pe_comm + h0.y + k) : __ldg(pe_comm + (size_t)(h0.y + k) * K + gc.link_class[p * G + d]);
@@ -585,7 +718,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
             }
         }
       }
-      if (any_cp) {
+      if (any_cp && __any_sync(FULL, live && h0.w != NONE)) {
         const uint32_t cpidx = h0.w;
         uint32_t below;
         if (GP >= 4) below = __popc(__ballot_sync(FULL, d < np && my_pcp < cpidx) & gm);
@@ -615,6 +748,17 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       }
       const bool go = live && fm != 0;
       const int dsel = fm ? __ffs(fm) - 1 - gb : 0;
+      if (snap_rec_on && go) {
+        if (d < G) ((T *)a.snap_avail)[(size_t)tstep * G + d] = avail;
+        if (d == 0) {
+          ((T *)a.snap_ms)[tstep] = makespan;
+          a.snap_dq[i] = (uint32_t)tstep;
+          W rw;
+          Slab<T>::make(rw, mn, (uint32_t)dsel);
+          ((W *)a.snap_rec)[i] = rw;
+        }
+      }
+      tstep++;
       if (go && d == dsel) {
         avail = mn;
         if (MEM) {
@@ -623,7 +767,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
         }
       }
       if (go) makespan = mn > makespan ? mn : makespan;
-      if (go && d == 0) Slab<T>::sched(slab, i, mn, (uint32_t)dsel);
+      if (go && d == 0) Slab<T>::sched(slab0, sb + i, mn, (uint32_t)dsel);
       if (any_out) {
         const T stt = __shfl_sync(FULL, est, gb + dsel);
         if (go && want_out && d == 0) {
@@ -638,10 +782,10 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       uint32_t bits = 0;
       if (go && (uint32_t)d < nsucc) {
         const uint32_t dg = sdeg - 1;
-        Slab<T>::set_indeg(slab, s0, dg);
+        Slab<T>::set_indeg(slab0, sb + s0, dg);
         if (dg == 0) {
-          atomicOr(&leaf[s0 >> 5], 1u << (s0 & 31));
-          atomicOr(&summ[s0 >> 10], 1u << ((s0 >> 5) & 31));
+          red_or_s(la + 4u * (s0 >> 5), 1u << (s0 & 31));
+          red_or_s(sa + 4u * (s0 >> 10), 1u << ((s0 >> 5) & 31));
           bits = 1u << (s0 >> 10);
         }
       }
@@ -649,11 +793,11 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
         for (uint32_t kk = GP + d; __any_sync(FULL, go && kk - d < nsucc); kk += GP) {
           if (go && kk < nsucc) {
             const uint32_t dst = kk < (uint32_t)S_IN ? __ldg(cd + CW_SUCC + kk) : __ldg(pg->se_dst + h0.z + kk);
-            const uint32_t dg = Slab<T>::indeg(slab, dst) - 1;
-            Slab<T>::set_indeg(slab, dst, dg);
+            const uint32_t dg = Slab<T>::indeg(slab0, sb + dst) - 1;
+            Slab<T>::set_indeg(slab0, sb + dst, dg);
             if (dg == 0) {
-              atomicOr(&leaf[dst >> 5], 1u << (dst & 31));
-              atomicOr(&summ[dst >> 10], 1u << ((dst >> 5) & 31));
+              red_or_s(la + 4u * (dst >> 5), 1u << (dst & 31));
+              red_or_s(sa + 4u * (dst >> 10), 1u << ((dst >> 5) & 31));
               bits |= 1u << (dst >> 10);
             }
           }
@@ -662,10 +806,21 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
 #pragma unroll
       for (int o = GP >> 1; o >= 1; o >>= 1) bits |= __shfl_xor_sync(FULL, bits, o);
       top |= bits;
+      // prefetch the peeked op's predecessor records (lane k of the group takes pred k)
+      if (SIM_PEEK && go && jn != NONE) {
+        const uint32_t npn = hn.x;  // hn = words 8..11 of the peeked card: its predecessor positions
+        (void)npn;
+        const uint32_t ps = d == 0 ? hn.x : d == 1 ? hn.y : d == 2 ? hn.z : hn.w;
+        if (d < 4) prefetch_l2(slab0 + (sb + ps));
+      }
       __syncwarp();
     }
 
     // ------------------------------------------------------------ epilogue
+    if (snap_rec_on && run && !infeas) {
+      if (d < G) ((T *)a.snap_avail)[(size_t)tstep * G + d] = avail;
+      if (d == 0) ((T *)a.snap_ms)[tstep] = makespan;
+    }
     if (run) {
       const int64_t ms64 = infeas ? I64MAX : (int64_t)makespan;
       const int64_t ri = s_res[lead], si = s_sidx[lead];
@@ -735,6 +890,116 @@ cudaError_t sim_set_smem(int tbits, int gshift, size_t smem) {
     if (e != cudaSuccess) return e;
   }
   return cudaSuccess;
+}
+
+// ------------------------------------------------- start-step bucketing
+// Key of a candidate for prefix sharing: the BASE dequeue step of its first
+// pinned op (n for BASE, 0 otherwise).  Candidates are bucket-sorted by it so
+// the lane groups of a warp start at similar steps.
+__global__ void k_t0_keys(int from_stream, StreamState S, int64_t first, int64_t stride, const Cand *list, int64_t n,
+                          const uint32_t *pos, const uint32_t *snap_dq, int32_t nops, int32_t vraw, int G, Cand *out,
+                          int64_t *oidx, uint32_t *key) {
+  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x) {
+    Cand c;
+    int64_t ix;
+    if (from_stream) {
+      ix = first + q * stride;
+      c = stream_cand(S, ix);
+    } else {
+      ix = q;
+      c = list[q];
+    }
+    uint32_t k = 0;
+    if (c.kind == 0) k = (uint32_t)nops;
+    else if (c.kind == 1 && c.n_pins >= 1 && c.n_pins <= MAXPINS) {
+      k = (uint32_t)nops;
+      for (int j = 0; j < c.n_pins; j++) {
+        const int32_t o = c.pin_op[j];
+        if (o < 0 || o >= vraw || pos[o] == NONE || c.pin_dev[j] >= G) {
+          k = 0;
+          break;
+        }
+        const uint32_t t = snap_dq[pos[o]];
+        k = t < k ? t : k;
+      }
+    }
+    out[q] = c;
+    oidx[q] = ix;
+    key[q] = k;
+  }
+}
+
+__global__ void k_bucket_hist(const uint32_t *key, int64_t n, int shift, uint32_t *hist) {
+  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(&hist[key[q] >> shift], 1u);
+}
+
+// exclusive scan of nb <= 1024 bucket counts, in place (one block of 1024)
+__global__ void k_bucket_scan(uint32_t *hist, int nb) {
+  __shared__ uint32_t sw[33];
+  const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+  uint32_t v = t < nb ? hist[t] : 0, x = v;
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t y = __shfl_up_sync(FULL, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) sw[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    uint32_t z = sw[lane], zz = z;
+    for (int o = 1; o < 32; o <<= 1) {
+      uint32_t y = __shfl_up_sync(FULL, zz, o);
+      if (lane >= o) zz += y;
+    }
+    sw[lane] = zz - z;
+  }
+  __syncthreads();
+  if (t < nb) hist[t] = sw[w] + x - v;
+}
+
+__global__ void k_bucket_scatter(const uint32_t *key, const Cand *in, const int64_t *iidx, int64_t n, int shift,
+                                 int nb, uint32_t *cursor, Cand *out, int64_t *oidx, int64_t *ores) {
+  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x) {
+    // ascending start step = longest remaining simulation first
+    const uint32_t b = key[q] >> shift;
+    const uint32_t dst = atomicAdd(&cursor[b], 1u);
+    out[dst] = in[q];
+    oidx[dst] = iidx[q];
+    if (ores) ores[dst] = iidx[q];
+  }
+  (void)nb;
+}
+
+void launch_t0_sort(int from_stream, const StreamState &S, int64_t first, int64_t stride, const Cand *list, int64_t n,
+                    const uint32_t *pos, const uint32_t *snap_dq, int32_t nops, int32_t vraw, int G, Cand *tmp_c,
+                    int64_t *tmp_i, uint32_t *key, uint32_t *hist, Cand *out_c, int64_t *out_i, int64_t *out_res,
+                    cudaStream_t st) {
+  if (n <= 0) return;
+  int shift = 0;
+  while ((nops >> shift) >= 1023) shift++;
+  const int nb = (nops >> shift) + 1;
+  const int blocks = (int)((n + 255) / 256 < 2048 ? (n + 255) / 256 : 2048);
+  k_t0_keys<<<blocks, 256, 0, st>>>(from_stream, S, first, stride, list, n, pos, snap_dq, nops, vraw, G, tmp_c, tmp_i,
+                                    key);
+  cudaMemsetAsync(hist, 0, sizeof(uint32_t) * 1024, st);
+  k_bucket_hist<<<blocks, 256, 0, st>>>(key, n, shift, hist);
+  k_bucket_scan<<<1, 1024, 0, st>>>(hist, nb);
+  k_bucket_scatter<<<blocks, 256, 0, st>>>(key, tmp_c, tmp_i, n, shift, nb, hist, out_c, out_i, out_res);
+}
+
+__global__ void k_gather_sorted(const Cand *src, const int64_t *sidx, const int64_t *sres, const int64_t *qs, int64_t n,
+                                Cand *dst, int64_t *didx, int64_t *dres) {
+  int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= n) return;
+  const int64_t q = qs[k];
+  dst[k] = src[q];
+  if (didx) didx[k] = sidx[q];
+  if (dres) dres[k] = sres ? sres[q] : -1;
+}
+void launch_gather_sorted(const Cand *src, const int64_t *sidx, const int64_t *sres, const int64_t *qs, int64_t n,
+                          Cand *dst, int64_t *didx, int64_t *dres, cudaStream_t st) {
+  if (n <= 0) return;
+  k_gather_sorted<<<(unsigned)((n + 127) / 128), 128, 0, st>>>(src, sidx, sres, qs, n, dst, didx, dres);
 }
 
 // ------------------------------------------------------------------ argmin

@@ -278,3 +278,47 @@ def test_bench_config_c5_size_and_32bit():
     desc = synth.config("C5")
     gg = F.Graph(desc)
     assert gg.time_bits == 32, "C5 should run the 32-bit time path"
+
+
+# ------------------------------------------------ BASE-schedule prefix sharing
+
+def _graph_noshare(desc):
+    os.environ["FASTT_NO_SHARE"] = "1"
+    try:
+        return F.Graph(desc)
+    finally:
+        del os.environ["FASTT_NO_SHARE"]
+
+
+@pytest.mark.parametrize("seed", range(16))
+def test_prefix_sharing_random(seed):
+    """makespan-only batches take the prefix-sharing path (no caps, no
+    outputs): they must equal the oracle and the non-sharing path."""
+    desc = synth.random_dag(seed + 1300, V=int(np.random.default_rng(seed).integers(20, 400)), caps="none",
+                            homogeneous=bool(seed % 2))
+    gg, og, g0 = F.Graph(desc), O.OracleGraph(desc), _graph_noshare(desc)
+    cands = random_cands(desc, np.random.default_rng(seed), 96, split_frac=0.1, bad_frac=0.02)
+    for flags in (0, F.F_CP_PIN):
+        r = gg.schedule_batch(cands, flags=flags, peak=False)
+        r0 = g0.schedule_batch(cands, flags=flags, peak=False)
+        assert (r["makespan"] == r0["makespan"]).all() and (r["status"] == r0["status"]).all()
+        for k, c in enumerate(cands):
+            o = og.schedule(c, flags=flags, outputs=False)
+            assert int(r["makespan"][k]) == o["makespan"] and int(r["status"][k]) == o["status"], (seed, k, flags)
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C3", "C5"])
+def test_prefix_sharing_configs(name):
+    desc = synth.config(name)
+    gg, og, g0 = F.Graph(desc), O.OracleGraph(desc), _graph_noshare(desc)
+    gen = F.gen_params(seed=0xFA57)
+    ns = gg.stream_info(gen, flags=F.F_CP_PIN)
+    n = 2000 if name in ("C1",) else 600
+    c = gg.generate_candidates(gen, 0, ns + n, flags=F.F_CP_PIN)
+    r = gg.schedule_batch(c, flags=F.F_CP_PIN, peak=False)
+    r0 = g0.schedule_batch(c, flags=F.F_CP_PIN, peak=False)
+    assert (r["makespan"] == r0["makespan"]).all()
+    step = 1 if name == "C1" else 97
+    for k in list(range(0, len(c), step)) + [0, len(c) - 1]:
+        assert int(r["makespan"][k]) == og.schedule(c[k], flags=F.F_CP_PIN, outputs=False)["makespan"], (name, k)
+    assert gg.sweep_best(gen, 0, ns + n, flags=F.F_CP_PIN) == g0.sweep_best(gen, 0, ns + n, flags=F.F_CP_PIN)
