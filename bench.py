@@ -186,6 +186,11 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # test hook: FASTT_DIST_BACKEND=gloo runs the multi-rank flow on one GPU
+    # (all ranks on cuda:0, collectives on CPU copies); the driver uses NCCL
+    backend = os.environ.get("FASTT_DIST_BACKEND", "nccl")
+    if backend == "gloo":
+        local = 0
     if args.impl == "reference":
         return run_reference(args, rank, world)
 
@@ -193,7 +198,18 @@ def main():
     import torch.distributed as dist
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+
+    def allreduce(t, op):
+        if backend == "nccl":
+            dist.all_reduce(t, op=op)
+        else:
+            c = t.cpu()
+            dist.all_reduce(c, op=op)
+            t.copy_(c)
     from paper_conf_middleware_0001lmwlwyl20_b200 import build as B
     B.build()
     from paper_conf_middleware_0001lmwlwyl20_b200 import fastt as F
@@ -213,7 +229,12 @@ def main():
         g.sweep_best(gen, rank, S, stride=world, flags=fl, stream=st, out=best_dev)
         tm = g.last_timing()
         if world > 1:
-            combine_best(best_dev)
+            if backend == "nccl":
+                combine_best(best_dev)
+            else:
+                c = best_dev.cpu()
+                combine_best(c)
+                best_dev.copy_(c)
         return tm
 
     for _ in range(args.warmup):
@@ -237,7 +258,7 @@ def main():
     ms = ev0.elapsed_time(ev1)
     t = torch.tensor([ms], dtype=torch.float64, device="cuda")
     if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        allreduce(t, dist.ReduceOp.MAX)
     ms_max = float(t.item())
     ms_step = ms_max / args.steps
     value = world * S / (ms_step / 1000.0)
@@ -262,7 +283,7 @@ def main():
     # end to end through the public API with host buffers
     e2e = None
     if not args.no_e2e:
-        cands = g.generate_candidates(gen, 0, world * S, flags=FLAGS_CP)[rank::world]
+        cands = np.ascontiguousarray(g.generate_candidates(gen, 0, world * S, flags=FLAGS_CP)[rank::world])
         n = len(cands)
         hc = torch.from_numpy(cands.view(np.uint8).reshape(-1, 32).copy()).pin_memory()
         # a search needs each candidate's makespan and status (per-device peak
@@ -286,7 +307,7 @@ def main():
         torch.cuda.synchronize()
         t2 = torch.tensor([ev2.elapsed_time(ev3)], dtype=torch.float64, device="cuda")
         if world > 1:
-            dist.all_reduce(t2, op=dist.ReduceOp.MAX)
+            allreduce(t2, dist.ReduceOp.MAX)
         e2e_ms = float(t2.item()) / args.steps
         e2e = {"value": world * n / (e2e_ms / 1000.0), "unit": UNIT, "h2d_bytes_per_step": int(32 * n),
                "d2h_bytes_per_step": int(n * (8 + 1)), "ms_per_step": e2e_ms,
