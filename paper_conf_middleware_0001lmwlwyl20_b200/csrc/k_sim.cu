@@ -387,9 +387,12 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
   uint32_t *summ = leaf + a.leaf_words;
   const uint32_t leaf_sa = (uint32_t)__cvta_generic_to_shared(leaf);
   const uint32_t summ_sa = (uint32_t)__cvta_generic_to_shared(summ);
-  W *const slab0 = (W *)a.slab;                                  // all slabs
-  const uint32_t sb = (uint32_t)(cslot * a.slab_stride);         // this candidate's slab (elements)
-  W *slab = slab0 + sb;
+  // state slabs: the CPW candidates of a warp are interleaved by position
+  // ([position][candidate], 32 B per position at CPW = 4), so groups that pop
+  // the same or nearby ops (they follow nearly the BASE order) share sectors
+  W *const slab0 = (W *)a.slab;
+  const uint32_t sb = (uint32_t)(gwarp * a.slab_stride * CPW + grp);
+#define SLOT(p) (sb + (uint32_t)(p) * (uint32_t)CPW)
   const GraphConst &gc = *a.gc;
   const int G = a.G;
   const int K = gc.K;
@@ -550,7 +553,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
         for (int32_t p = d; p < n; p += GP) {
           const uint32_t dq = __ldg(a.snap_dq + p);
           if ((int32_t)dq < t0) {
-            slab[p] = rec0[p];
+            slab0[SLOT(p)] = rec0[p];
           } else {
             const uint32_t *cp_ = card + (size_t)p * CARD_WORDS;
             const uint32_t npr = __ldg(cp_ + CW_DEG) & 0xFFFF;
@@ -564,7 +567,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
               const uint32_t pb = __ldg(cp_ + CW_PBASE);
               for (uint32_t k = 4; k < npr; k++) cnt += (int32_t)__ldg(a.snap_dq + __ldg(pg->pe_src + pb + k)) >= t0;
             }
-            Slab<T>::init(slab, (uint32_t)p, cnt);
+            Slab<T>::init(slab0, SLOT(p), cnt);
             if (cnt == 0) atomicOr(&leaf[p >> 5], 1u << (p & 31));
           }
         }
@@ -588,7 +591,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       for (int32_t w = d; w < nwords; w += GP) leaf[w] = __ldg(pg->srcbits + w);
       for (int32_t s = d; s < 32; s += GP) summ[s] = __ldg(pg->srcsumm + s);
       top = __ldg(pg->srcsumm + 32);
-      for (int32_t p = d; p < n; p += GP) Slab<T>::init(slab, (uint32_t)p, __ldg(pg->npred + p));
+      for (int32_t p = d; p < n; p += GP) Slab<T>::init(slab0, SLOT(p), __ldg(pg->npred + p));
     }
     if (a.snap_mode == 1 && run && d == 0) {
       a.snap_rounds[0] = nrounds;
@@ -666,9 +669,9 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       for (int k = 0; k < 4; k++) {
         ft[k] = 0;
         pl[k] = (uint32_t)d;
-        if ((uint32_t)k < npred) Slab<T>::load(slab0, sb + src[k], ft[k], pl[k]);
+        if ((uint32_t)k < npred) Slab<T>::load(slab0, SLOT(src[k]), ft[k], pl[k]);
       }
-      const uint32_t sdeg = ((uint32_t)d < nsucc) ? Slab<T>::indeg(slab0, sb + s0) : 1u;
+      const uint32_t sdeg = ((uint32_t)d < nsucc) ? Slab<T>::indeg(slab0, SLOT(s0)) : 1u;
       // EST = max(avail[d], max_pred FT + c(pred -> i on d))   (R1, R6)
       T est = avail;
 #pragma unroll
@@ -687,7 +690,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
           if (k < npred) {
             T f;
             uint32_t p;
-            Slab<T>::load(slab0, sb + __ldg(pe_src + h0.y + k), f, p);
+            Slab<T>::load(slab0, SLOT(__ldg(pe_src + h0.y + k)), f, p);
             T cm = 0;
             if (p != (uint32_t)d && d < G)
               cm = K == 1 ? __ldg(pe_comm + h0.y + k) : __ldg(pe_comm + (size_t)(h0.y + k) * K + gc.link_class[p * G + d]);
@@ -767,7 +770,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
         }
       }
       if (go) makespan = mn > makespan ? mn : makespan;
-      if (go && d == 0) Slab<T>::sched(slab0, sb + i, mn, (uint32_t)dsel);
+      if (go && d == 0) Slab<T>::sched(slab0, SLOT(i), mn, (uint32_t)dsel);
       if (any_out) {
         const T stt = __shfl_sync(FULL, est, gb + dsel);
         if (go && want_out && d == 0) {
@@ -782,7 +785,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       uint32_t bits = 0;
       if (go && (uint32_t)d < nsucc) {
         const uint32_t dg = sdeg - 1;
-        Slab<T>::set_indeg(slab0, sb + s0, dg);
+        Slab<T>::set_indeg(slab0, SLOT(s0), dg);
         if (dg == 0) {
           red_or_s(la + 4u * (s0 >> 5), 1u << (s0 & 31));
           red_or_s(sa + 4u * (s0 >> 10), 1u << ((s0 >> 5) & 31));
@@ -793,8 +796,8 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
         for (uint32_t kk = GP + d; __any_sync(FULL, go && kk - d < nsucc); kk += GP) {
           if (go && kk < nsucc) {
             const uint32_t dst = kk < (uint32_t)S_IN ? __ldg(cd + CW_SUCC + kk) : __ldg(pg->se_dst + h0.z + kk);
-            const uint32_t dg = Slab<T>::indeg(slab0, sb + dst) - 1;
-            Slab<T>::set_indeg(slab0, sb + dst, dg);
+            const uint32_t dg = Slab<T>::indeg(slab0, SLOT(dst)) - 1;
+            Slab<T>::set_indeg(slab0, SLOT(dst), dg);
             if (dg == 0) {
               red_or_s(la + 4u * (dst >> 5), 1u << (dst & 31));
               red_or_s(sa + 4u * (dst >> 10), 1u << ((dst >> 5) & 31));
@@ -811,7 +814,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
         const uint32_t npn = hn.x;  // hn = words 8..11 of the peeked card: its predecessor positions
         (void)npn;
         const uint32_t ps = d == 0 ? hn.x : d == 1 ? hn.y : d == 2 ? hn.z : hn.w;
-        if (d < 4) prefetch_l2(slab0 + (sb + ps));
+        if (d < 4) prefetch_l2(slab0 + SLOT(ps));
       }
       __syncwarp();
     }
