@@ -47,7 +47,7 @@ static size_t al16(size_t x) { return (x + 15) & ~(size_t)15; }
 
 struct RawLayout {
   int64_t vcap = 0, ecap = 0;
-  size_t o[17] = {0};
+  size_t o[20] = {0};
   size_t total = 0;
 };
 
@@ -55,16 +55,18 @@ static RawLayout raw_layout(int64_t vcap, int64_t ecap, int G) {
   RawLayout L;
   L.vcap = vcap;
   L.ecap = ecap;
-  size_t sz[17] = {(size_t)vcap * 4, (size_t)vcap * 4, (size_t)vcap * 4, (size_t)vcap * 4,  // off/cnt
+  size_t sz[20] = {(size_t)vcap * 4, (size_t)vcap * 4, (size_t)vcap * 4, (size_t)vcap * 4,  // off/cnt
                    (size_t)ecap * 4, (size_t)ecap * 4,                                       // dst, src
                    (size_t)ecap * 8, (size_t)ecap * 8,                                       // bytes
                    (size_t)ecap, (size_t)ecap,                                               // param flags
                    (size_t)vcap * G * 8,                                                     // cost
                    (size_t)vcap * 8, (size_t)vcap * 8,                                       // mem, param
                    (size_t)vcap, (size_t)vcap,                                               // split_mask, alive
-                   (size_t)vcap * 4, 16};                                                    // topo, pad
+                   (size_t)vcap * 4,                                                         // topo
+                   (size_t)vcap * 4, (size_t)(vcap + 2) * 4, (size_t)vcap * 4,               // height, levels
+                   16};
   size_t off = 0;
-  for (int k = 0; k < 17; k++) {
+  for (int k = 0; k < 20; k++) {
     L.o[k] = off;
     off += al16(sz[k]);
   }
@@ -93,6 +95,12 @@ static RawGraph raw_struct(char *b, const RawLayout &L, int32_t V, int32_t nl, i
   R.split_mask = (uint8_t *)(b + L.o[13]);
   R.alive = (uint8_t *)(b + L.o[14]);
   R.topo = (int32_t *)(b + L.o[15]);
+  R.height = (int32_t *)(b + L.o[16]);
+  R.lvl_off = (int32_t *)(b + L.o[17]);
+  R.lvl_ops = (int32_t *)(b + L.o[18]);
+  R.H = 0;
+  R.ov_o = R.ov_base = R.ov_n = R.ov_S = 0;
+  R.ov_P = -1;
   return R;
 }
 
@@ -321,6 +329,14 @@ static int bits_for(unsigned long long v) {
 
 // bound -> time type; rank, sort, cards, CP for a base whose raw graph is in place
 static fastt_status prepare_base(fastt_graph *g, Base &B, cudaStream_t st) {
+  {
+    int32_t *scratch = nullptr;
+    CK(cudaMalloc(&scratch, sizeof(int32_t) * (3 * B.rl.vcap + 64)));
+    launch_heights(B.raw_dev, scratch, B.rl.vcap, st);
+    CK(cudaGetLastError());
+    CK(cudaStreamSynchronize(st));
+    cudaFree(scratch);
+  }
   unsigned long long *d_b = nullptr;
   CK(cudaMalloc(&d_b, 16));
   CK(cudaMemsetAsync(d_b, 0, 16, st));
@@ -355,9 +371,13 @@ static fastt_status prepare_base(fastt_graph *g, Base &B, cudaStream_t st) {
 
 // ------------------------------------------------------------- workspaces
 
-static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st) {
+// preparation slots for `need` deferred candidates: sized to the batch (a
+// C5 sweep's ~4k split candidates prepare in one wave), capped at 8192 slots
+// and 40 % of free HBM, and kept for later calls with the same layout
+static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st, int64_t need) {
   size_t rt = B.rl.total, pt = B.pl.total;
-  if (g->arena && g->arena_raw_total == rt && g->arena_prep_total == pt) return FASTT_OK;
+  const int64_t want = std::min<int64_t>(std::max<int64_t>(need, 64), 8192);
+  if (g->arena && g->arena_raw_total == rt && g->arena_prep_total == pt && g->arena_slots >= want) return FASTT_OK;
   cudaFree(g->arena);
   cudaFree(g->tmpl_dev);
   cudaFree(g->slot_raws_dev);
@@ -369,10 +389,8 @@ static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st)
   size_t freeb = 0, totb = 0;
   CK(cudaMemGetInfo(&freeb, &totb));
   size_t per = rt + pt;
-  // up to 8192 slots within 40% of free HBM: a C5 sweep's ~4k split
-  // candidates then prepare in one wave instead of many sequential chunks
-  int64_t slots = (int64_t)(freeb * 2 / 5 / per);
-  if (slots > 8192) slots = 8192;
+  // at most 40 % of the free and 25 % of the total device memory per graph
+  int64_t slots = std::min<int64_t>(want, (int64_t)(std::min(freeb * 2 / 5, totb / 4) / per));
   if (slots < 1) return fail(FASTT_ENOMEM, "device memory too small for one preparation slot (%zu bytes)", per);
   g->arena_slots = (int)slots;
   CK(cudaMalloc(&g->arena, per * slots));
@@ -638,7 +656,7 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
   CK(cudaMemcpyAsync(&nd, g->counters + 1, sizeof nd, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
   if (nd > 0) {
-    TRY(ensure_arena(g, B, st));
+    TRY(ensure_arena(g, B, st, (int64_t)nd));
     for (int64_t c0 = 0; c0 < (int64_t)nd; c0 += g->arena_slots) {
       int nc = (int)std::min<int64_t>(g->arena_slots, (int64_t)nd - c0);
       if (sorted) launch_gather_sorted(g->srt_c, g->srt_i, g->srt_res, g->defer_q + c0, nc, g->slot_cands, nullptr,
@@ -1145,7 +1163,7 @@ fastt_status fastt_rank(const fastt_graph *gc_, const fastt_candidate *cand, con
       bad = true;
     }
     if (bad) return fail(FASTT_EINVAL, "invalid candidate");
-    TRY(ensure_arena(g, B, st));
+    TRY(ensure_arena(g, B, st, 1));
     CK(cudaMemcpyAsync(g->slot_cands, &c, sizeof c, cudaMemcpyHostToDevice, st));
     launch_slot_setup(g->slot_cands, g->tmpl_dev, B.raw_dev, g->slot_raws_dev, 1, st);
     launch_copy_block(B.raw_block, g->arena, (int64_t)(g->arena_raw_total + g->arena_prep_total),
@@ -1320,7 +1338,7 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
     CK(cudaMemcpyAsync(&nd, g->counters + 1, sizeof nd, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     if (nd > 0) {
-      TRY(ensure_arena(g, B, st));
+      TRY(ensure_arena(g, B, st, (int64_t)nd));
       for (int64_t c0 = 0; c0 < (int64_t)nd; c0 += g->arena_slots) {
         int nc = (int)std::min<int64_t>(g->arena_slots, (int64_t)nd - c0);
         if (a.mode == 3) launch_gather_sorted(g->srt_c, g->srt_i, nullptr, g->defer_q + c0, nc, g->slot_cands,
@@ -1394,6 +1412,8 @@ static fastt_status materialize_base(fastt_graph *g, Base &from, const Cand &c, 
   CK(cudaStreamSynchronize(st));
   cudaFree(d_c);
   to.E = Rt.E;
+  Rt.ov_P = -1;  // a materialised base, not a slot: its levels are recomputed by prepare_base
+  CK(cudaMemcpy(to.raw_dev, &Rt, sizeof Rt, cudaMemcpyHostToDevice));
   return prepare_base(g, to, st);
 }
 

@@ -66,6 +66,15 @@ struct RawGraph {
   int64_t *mem, *param;
   uint8_t *split_mask, *alive;
   int32_t *topo;   // n_live, a topological order of the live ops
+  // levels for the level-synchronous rank sweep (heights of the base graph;
+  // a split slot keeps its base's levels and places its overlay nodes at
+  // labels 4h(o)-2 (concat), 4h(o) (sub-ops), 4h(o)+2 (split nodes))
+  int32_t *height;  // V: longest path (in edges) to a sink; -1 for dead ops
+  int32_t *lvl_off; // H+2
+  int32_t *lvl_ops; // n_live ops ordered by height
+  int32_t H;        // max height
+  // split overlay of a slot (ov_P < 0: none)
+  int32_t ov_o, ov_base, ov_P, ov_n, ov_S;
 };
 
 struct PrepGraph {
@@ -129,6 +138,7 @@ __host__ __device__ inline int64_t part_bytes(int64_t b, int n, int k) { return 
 
 void launch_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, const Cand *cands, int nslots,
                  int G, cudaStream_t st);
+void launch_heights(RawGraph *raw_dev, int32_t *scratch, int64_t vcap, cudaStream_t st);
 void launch_sort(PrepGraph *pgs, const RawGraph *raws, int nslots, int key_bits, int max_n, cudaStream_t st);
 void launch_cards(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, int nslots, int max_n, int G, int K,
                   int tbits, cudaStream_t st);

@@ -163,6 +163,12 @@ __global__ void k_patch_split(const RawGraph *base_p, RawGraph *raws, const Grap
     R.V = V + P + n + S;
     R.n_live = B.n_live - 1 + P + n + S;
     R.E = ecur > ecur_s ? ecur : ecur_s;
+    R.H = B.H;
+    R.ov_o = o;
+    R.ov_base = V;
+    R.ov_P = (int32_t)P;
+    R.ov_n = n;
+    R.ov_S = (int32_t)S;
     s_to = -1;
   }
   __syncthreads();
@@ -224,7 +230,33 @@ __device__ __forceinline__ int pin_of(int32_t u, const int32_t *po, const int32_
   return r;
 }
 
-// One warp per slot: rank_u in reverse topological order.
+// rank of one op u evaluated by one lane: w_u over the allowed
+// devices + max over successors of (c_uv + rank_v)
+__device__ __forceinline__ void rank_one(const RawGraph &R, const GraphConst &gc, uint64_t *rank, int32_t u,
+                                         const int32_t *po, const int32_t *pd, int np) {
+  const int G = gc.G;
+  const int pu = pin_of(u, po, pd, np);
+  int64_t w = 0;
+  if (pu >= 0) w = R.cost[(int64_t)u * G + pu];
+  else
+    for (int d = 0; d < G; d++) {
+      const int64_t c = R.cost[(int64_t)u * G + d];
+      w = c > w ? c : w;
+    }
+  const uint32_t off = R.succ_off[u], cnt_s = R.succ_cnt[u];
+  uint64_t best = 0;
+  for (uint32_t j = 0; j < cnt_s; j++) {
+    const int32_t s = R.succ_dst[off + j];
+    const uint64_t v = (uint64_t)c_allowed(gc, R.succ_bytes[off + j], pu, pin_of(s, po, pd, np)) + rank[s];
+    best = v > best ? v : best;
+  }
+  rank[u] = (uint64_t)w + best;
+}
+
+// One warp per slot: rank_u level by level (increasing height: every
+// successor of an op sits on a lower level); the ops of a level are
+// independent, one lane each.  A split slot inserts its concat nodes before
+// level h(o), its sub-ops with level h(o) and its split nodes after it.
 __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gcp, const Cand *cands, int nslots) {
   const int lane = threadIdx.x & 31;
   const int slot = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -232,7 +264,6 @@ __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *g
   const RawGraph &R = raws[slot];
   PrepGraph &P = pgs[slot];
   const GraphConst &gc = *gcp;
-  const int G = gc.G;
   int32_t po[MAXPINS], pd[MAXPINS];
   int np = 0;
   if (cands) {
@@ -246,35 +277,27 @@ __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *g
   uint64_t *rank = P.rank;
   for (int32_t u = lane; u < R.V; u += 32) rank[u] = ~0ull;
   __syncwarp();
-  const int32_t nl = R.n_live;
-  for (int32_t base = nl - 1; base >= 0; base -= 32) {
-    int32_t tl = base - lane;
-    int32_t mine = tl >= 0 ? R.topo[tl] : -1;
-    int cnt = base + 1 < 32 ? base + 1 : 32;
-    for (int q = 0; q < cnt; q++) {
-      int32_t u = __shfl_sync(FULL, mine, q);
-      int pu = pin_of(u, po, pd, np);
-      // w_i: max over allowed devices
-      int64_t w;
-      if (pu >= 0) w = R.cost[(int64_t)u * G + pu];
-      else {
-        int64_t cv = lane < G ? R.cost[(int64_t)u * G + lane] : 0;
-        w = (int64_t)warp_max_u64((uint64_t)cv);
+  const bool split = R.ov_P >= 0;
+  const int32_t ho = split ? R.height[R.ov_o] : -1;
+  for (int32_t lev = 0; lev <= R.H; lev++) {
+    for (int phase = 0; phase < 3; phase++) {
+      // phase 0: concat nodes (label 4h(o)-2), 1: the level (+ sub-ops at h(o)), 2: split nodes (4h(o)+2)
+      int32_t lo, cnt;
+      const int32_t *list = nullptr;
+      if (phase == 1) {
+        lo = R.lvl_off[lev];
+        cnt = R.lvl_off[lev + 1] - lo;
+        list = R.lvl_ops + lo;
+      } else {
+        if (!split || lev != ho) continue;
+        lo = phase == 0 ? R.ov_base + R.ov_P + R.ov_n : R.ov_base;
+        cnt = phase == 0 ? R.ov_S : R.ov_P;
       }
-      uint32_t off = R.succ_off[u], cnt_s = R.succ_cnt[u];
-      uint64_t best = 0;
-      for (uint32_t j0 = 0; j0 < cnt_s; j0 += 32) {
-        uint64_t v = 0;
-        if (j0 + lane < cnt_s) {
-          int32_t s = R.succ_dst[off + j0 + lane];
-          int64_t b = R.succ_bytes[off + j0 + lane];
-          int ps = pin_of(s, po, pd, np);
-          v = (uint64_t)c_allowed(gc, b, pu, ps) + rank[s];
-        }
-        v = warp_max_u64(v);
-        best = v > best ? v : best;
+      const int32_t extra = (phase == 1 && split && lev == ho) ? R.ov_n : 0;
+      for (int32_t q = lane; q < cnt + extra; q += 32) {
+        int32_t u = q < cnt ? (list ? list[q] : lo + q) : R.ov_base + R.ov_P + (q - cnt);
+        if (R.alive[u]) rank_one(R, gc, rank, u, po, pd, np);
       }
-      if (lane == 0) rank[u] = (uint64_t)w + best;
       __syncwarp();
     }
   }
@@ -286,6 +309,81 @@ void launch_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, con
   int warps_per_block = 4;
   int blocks = (nslots + warps_per_block - 1) / warps_per_block;
   k_rank<<<blocks, warps_per_block * 32, 0, st>>>(raws, pgs, gc, cands, nslots);
+}
+
+__device__ uint32_t cta_exscan(uint32_t v, uint32_t *total, uint32_t *s_w);
+
+// Heights (edges on the longest path to a sink) and the per-height op lists of
+// a base graph: a frontier peel from the sinks (one CTA), then a counting sort.
+__global__ void __launch_bounds__(1024) k_heights(RawGraph *Rp, int32_t *scratch, int64_t vcap) {
+  RawGraph &R = *Rp;
+  int32_t *rem = scratch, *fa = scratch + vcap, *fb = scratch + 2 * vcap;
+  __shared__ int32_t s_na, s_nb, s_H;
+  __shared__ uint32_t s_w[33];
+  const int tid = threadIdx.x;
+  if (tid == 0) { s_na = 0; s_nb = 0; s_H = -1; }  // H = -1: no live op
+  __syncthreads();
+  for (int32_t u = tid; u < R.V; u += blockDim.x) {
+    R.height[u] = -1;
+    rem[u] = (int32_t)R.succ_cnt[u];
+    if (R.alive[u] && R.succ_cnt[u] == 0) {
+      R.height[u] = 0;
+      fa[atomicAdd(&s_na, 1)] = u;
+    }
+  }
+  __syncthreads();
+  int32_t lev = 0;
+  int32_t *cur = fa, *nxt = fb;
+  while (true) {
+    const int32_t nc = s_na;
+    if (nc == 0) break;
+    for (int32_t k = tid; k < nc; k += blockDim.x) {
+      const int32_t u = cur[k];
+      for (uint32_t j = 0; j < R.pred_cnt[u]; j++) {
+        const int32_t p = R.pred_src[R.pred_off[u] + j];
+        if (atomicSub(&rem[p], 1) == 1) {
+          R.height[p] = lev + 1;
+          nxt[atomicAdd(&s_nb, 1)] = p;
+        }
+      }
+    }
+    __syncthreads();
+    if (tid == 0) {
+      s_na = s_nb;
+      s_nb = 0;
+      s_H = lev;
+    }
+    int32_t *t = cur; cur = nxt; nxt = t;
+    lev++;
+    __syncthreads();
+  }
+  const int32_t H = s_H;
+  // counting sort by height: counts -> exclusive offsets -> scatter
+  for (int32_t h = tid; h <= H + 1; h += blockDim.x) R.lvl_off[h] = 0;
+  __syncthreads();
+  for (int32_t u = tid; u < R.V; u += blockDim.x)
+    if (R.height[u] >= 0) atomicAdd(&R.lvl_off[R.height[u] + 1], 1);
+  __syncthreads();
+  uint32_t run = 0;
+  for (int32_t t0 = 0; t0 <= H + 1; t0 += blockDim.x) {
+    const int32_t h = t0 + tid;
+    const uint32_t v = h <= H + 1 ? (uint32_t)R.lvl_off[h] : 0u;
+    uint32_t tot;
+    const uint32_t pre = cta_exscan(v, &tot, s_w);
+    if (h <= H + 1) R.lvl_off[h] = (int32_t)(run + pre + v);  // inclusive: lvl_off[h] = end of level h-1
+    run += tot;
+  }
+  __syncthreads();
+  // lvl_off[h] now holds the start of level h (level counts were shifted by one)
+  for (int32_t h = tid; h <= H; h += blockDim.x) rem[h] = R.lvl_off[h];
+  __syncthreads();
+  for (int32_t u = tid; u < R.V; u += blockDim.x)
+    if (R.height[u] >= 0) R.lvl_ops[atomicAdd(&rem[R.height[u]], 1)] = u;
+  if (tid == 0) R.H = H;
+}
+
+void launch_heights(RawGraph *raw_dev, int32_t *scratch, int64_t vcap, cudaStream_t st) {
+  k_heights<<<1, 1024, 0, st>>>(raw_dev, scratch, vcap);
 }
 
 // ------------------------------------------------------------- radix sort

@@ -247,7 +247,7 @@ def test_split_search_random(seed):
         assert (a["order"] == b["order"]).all()
 
 
-@pytest.mark.parametrize("name", ["C1", "C4"])
+@pytest.mark.parametrize("name", ["C1", "C2", "C3", "C4", "C5"])
 def test_split_search_configs(name):
     desc = synth.config(name)
     gg, og = F.Graph(desc), O.OracleGraph(desc)
