@@ -76,7 +76,8 @@ enum {
   FASTT_F_POLICY_INSERT = 1u << 1, /* insertion-based avail[j]; NOT YET SUPPORTED -> EUNSUP */
   FASTT_F_OUT_DEVICE = 1u << 2,    /* output pointers are device pointers */
   FASTT_F_IN_DEVICE = 1u << 3,     /* candidate input pointer is a device pointer */
-  FASTT_F_TIMING = 1u << 4         /* record CUDA events around the kernels of this call (fastt_last_timing) */
+  FASTT_F_TIMING = 1u << 4,        /* record CUDA events around the kernels of this call (fastt_last_timing) */
+  FASTT_F_SPLIT_BEST = 1u << 5     /* fastt_split_search: best-improvement rounds */
 };
 
 /* The problem input of P:321-328.  Edges are a CSR by source: the edges of
@@ -187,7 +188,13 @@ fastt_status fastt_generate_candidates(const fastt_graph *g, const fastt_gen_par
 fastt_status fastt_sweep_best(const fastt_graph *g, const fastt_gen_params *gen, const fastt_opts *opts,
                               int64_t first, int64_t n, int64_t stride, int64_t *best);
 
-/* OS-DPOS (Alg. 2, S8). */
+/* OS-DPOS (Alg. 2, S8): DPOS of the graph, the placement-aware critical path
+ * (lines 4-5, R15), then for each split-eligible CP op in descending cost the
+ * best of its splits (dims asc, n asc; n in 2..G or powers of two with
+ * n_pow2_only) is accepted if strictly better, else the search stops.
+ * With FASTT_F_SPLIT_BEST (NEXT row N2, a variant): every round evaluates all
+ * splits of all not-yet-split list ops in one batch and accepts the best
+ * (ties: list order, dim, n) while it strictly improves. */
 typedef struct {
   int32_t n_splits; /* SP list */
   int32_t *op;

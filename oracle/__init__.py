@@ -68,6 +68,8 @@ def lib():
         _lib.fastt_ref_rank.argtypes = [P, i32, i32, P, P, i32, i32, i32, P]
         _lib.fastt_ref_split_search.restype = i32
         _lib.fastt_ref_split_search.argtypes = [P, u32, i32, i32, P, P, P, P, i32, P, P, P, P, P, P]
+        _lib.fastt_ref_split_search_bi.restype = i32
+        _lib.fastt_ref_split_search_bi.argtypes = [P, u32, i32, i32, P, P, P, P, i32, P, P, P, P, P, P]
         _lib.fastt_ref_stream_info.restype = i32
         _lib.fastt_ref_stream_info.argtypes = [P, u32, i32, P, P]
         _lib.fastt_ref_generate.restype = i32
@@ -204,7 +206,7 @@ class OracleGraph:
         n = lib().fastt_ref_cp(self.h, _p(cp))
         return cp[:n]
 
-    def split_search(self, flags=0, pow2_only=False, out_cap=None):
+    def split_search(self, flags=0, pow2_only=False, out_cap=None, best_improvement=False):
         cap = out_cap or (self.V + 64 * (self.G + 64) + 1024)
         sp_n = np.zeros(1, np.int32)
         spc = 4096
@@ -217,14 +219,15 @@ class OracleGraph:
         start = np.zeros(cap, np.int64)
         ms = np.zeros(1, np.int64)
         st = np.zeros(1, np.uint8)
-        rc = lib().fastt_ref_split_search(self.h, flags, int(bool(pow2_only)), spc, _p(sp_n), _p(sp_op), _p(sp_dim),
-                                          _p(sp_cnt), cap, _p(nfin), _p(place), _p(order), _p(start), _p(ms), _p(st))
+        fn = lib().fastt_ref_split_search_bi if best_improvement else lib().fastt_ref_split_search
+        rc = fn(self.h, flags, int(bool(pow2_only)), spc, _p(sp_n), _p(sp_op), _p(sp_dim),
+                _p(sp_cnt), cap, _p(nfin), _p(place), _p(order), _p(start), _p(ms), _p(st))
         if rc != 0:
             raise OracleError(rc)
         n = int(sp_n[0])
         nf = int(nfin[0])
         if nf > cap:
-            return self.split_search(flags, pow2_only, out_cap=nf + 16)
+            return self.split_search(flags, pow2_only, out_cap=nf + 16, best_improvement=best_improvement)
         return {"sp": [(int(sp_op[q]), int(sp_dim[q]), int(sp_cnt[q])) for q in range(n)], "n_ops_final": nf,
                 "placement": place[:nf], "order": order[:nf], "start": start[:nf], "makespan": int(ms[0]),
                 "status": int(st[0])}

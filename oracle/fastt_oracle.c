@@ -847,6 +847,94 @@ int32_t fastt_ref_split_search(const fo_graph *g0, uint32_t flags, int32_t pow2_
   return FO_OK;
 }
 
+/* NEXT row N2: best-improvement OS-DPOS.  Same input and CP
+ * list as Alg. 2 (lines 3-5), but every round evaluates every split (op, dim,
+ * n) of every not-yet-split op of the list on the current graph and accepts
+ * the one with the smallest FT (ties: list order, dim asc, n asc) if it is
+ * strictly better; stops when no split improves.  (A variant of Alg. 2,
+ * the paper stops at the first op that does not improve.) */
+int32_t fastt_ref_split_search_bi(const fo_graph *g0, uint32_t flags, int32_t pow2_only, int32_t sp_cap,
+                                  int32_t *sp_n, int32_t *sp_op, uint8_t *sp_dim, uint8_t *sp_cnt,
+                                  int32_t out_cap, int32_t *n_ops_final, uint8_t *placement, int32_t *order,
+                                  int64_t *start, int64_t *makespan, uint8_t *status) {
+  int32_t G = g0->G;
+  fo_graph *cur = (fo_graph *)g0;
+  fo_result best_r;
+  fo_result_alloc(&best_r, g0->V, G);
+  int64_t *rank = malloc(sizeof(int64_t) * ((size_t)g0->V + 1));
+  fo_dpos(cur, NULL, flags, rank, &best_r);
+  free(rank);
+  *sp_n = 0;
+  if (best_r.status != FO_CAND_OK) {
+    *makespan = FO_INF; *status = best_r.status; *n_ops_final = g0->V;
+    fo_result_free(&best_r);
+    return FO_OK;
+  }
+  int64_t ft_old = best_r.makespan;
+  int32_t *list = malloc(sizeof(int32_t) * ((size_t)g0->V + 1));
+  int32_t nl = fo_split_list(g0, best_r.place, list);
+  uint8_t *done = calloc((size_t)nl + 1, 1);
+  int ns[FO_MAXG];
+  int nns = fo_split_ns(G, pow2_only, ns);
+  for (;;) {
+    int64_t bft = FO_INF;
+    int32_t bli = -1;
+    int bdim = -1, bn = -1;
+    fo_graph *bg = NULL;
+    fo_result br;
+    memset(&br, 0, sizeof(br));
+    for (int32_t li = 0; li < nl; li++) {
+      if (done[li]) continue;
+      int32_t op = list[li];
+      for (int dim = 0; dim < 2; dim++) {
+        if (!(cur->split_mask[op] & (1u << dim))) continue;
+        for (int q = 0; q < nns; q++) {
+          fo_graph *sv;
+          if (fo_split_view(cur, op, dim, ns[q], &sv) != FO_OK) continue;
+          fo_result r;
+          fo_result_alloc(&r, sv->V, G);
+          int64_t *rk = malloc(sizeof(int64_t) * ((size_t)sv->V + 1));
+          fo_dpos(sv, NULL, flags, rk, &r);
+          free(rk);
+          if (r.status == FO_CAND_OK && r.makespan < bft) {
+            if (bg) { fo_graph_free(bg); fo_result_free(&br); }
+            bg = sv; br = r; bft = r.makespan; bli = li; bdim = dim; bn = ns[q];
+          } else {
+            fo_graph_free(sv);
+            fo_result_free(&r);
+          }
+        }
+      }
+    }
+    if (!bg || bft >= ft_old) {
+      if (bg) { fo_graph_free(bg); fo_result_free(&br); }
+      break;
+    }
+    if (*sp_n < sp_cap) { sp_op[*sp_n] = list[bli]; sp_dim[*sp_n] = (uint8_t)bdim; sp_cnt[*sp_n] = (uint8_t)bn; }
+    (*sp_n)++;
+    done[bli] = 1;
+    ft_old = bft;
+    if (cur != g0) fo_graph_free(cur);
+    cur = bg;
+    fo_result_free(&best_r);
+    best_r = br;
+  }
+  *makespan = ft_old;
+  *status = FO_CAND_OK;
+  *n_ops_final = cur->V;
+  int32_t n = cur->V < out_cap ? cur->V : out_cap;
+  for (int32_t i = 0; i < out_cap; i++) {
+    if (placement) placement[i] = i < n ? best_r.place[i] : 0xFF;
+    if (order) order[i] = i < n ? best_r.order[i] : -1;
+    if (start) start[i] = i < n ? best_r.start[i] : -1;
+  }
+  fo_result_free(&best_r);
+  free(list);
+  free(done);
+  if (cur != g0) fo_graph_free(cur);
+  return FO_OK;
+}
+
 /* ------------------------------------- the sweep's candidate stream (R21) */
 
 typedef struct {

@@ -1422,6 +1422,7 @@ fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, 
   fastt_graph *g = (fastt_graph *)gc_;
   if (!g || !out) return fail(FASTT_EINVAL, "NULL argument");
   const uint32_t flags = flags_of(opts) & FASTT_F_CP_PIN;
+  const bool best_mode = (flags_of(opts) & FASTT_F_SPLIT_BEST) != 0;
   if (flags_of(opts) & FASTT_F_POLICY_INSERT) return fail(FASTT_EUNSUP, "FASTT_F_POLICY_INSERT is not implemented yet");
   memset(out, 0, sizeof *out);
   std::lock_guard<std::mutex> lk(g->mu);
@@ -1500,6 +1501,95 @@ fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, 
     }
     int ns[MAXG];
     int nns = split_counts(g->G, n_pow2_only, ns);
+    if (best_mode) {
+      // NEXT N2: best-improvement rounds -- every remaining split of every
+      // not-yet-split list op in one batch, accept the best if it improves
+      std::vector<char> done(list.size(), 0);
+      const size_t cap_round = list.size() * 2 * (size_t)nns + 1;
+      Cand *d_round = nullptr;
+      int64_t *d_rms = nullptr;
+      uint8_t *d_rst = nullptr;
+      if (cudaMalloc(&d_round, sizeof(Cand) * cap_round) != cudaSuccess ||
+          cudaMalloc(&d_rms, 8 * cap_round) != cudaSuccess || cudaMalloc(&d_rst, cap_round) != cudaSuccess) {
+        cudaFree(d_round);
+        cudaFree(d_rms);
+        cleanup();
+        return fail(FASTT_ENOMEM, "split-search round buffers");
+      }
+      for (;;) {
+        std::vector<Cand> cs;
+        std::vector<size_t> li_of;
+        for (size_t li = 0; li < list.size(); li++) {
+          if (done[li]) continue;
+          const int32_t op = list[li];
+          for (int dim = 0; dim < 2; dim++) {
+            if (!(g->split_mask_h[op] & (1u << dim))) continue;
+            for (int q = 0; q < nns; q++) {
+              Cand c;
+              memset(&c, 0, sizeof c);
+              c.kind = FASTT_KIND_SPLIT;
+              c.split_op = op;
+              c.split_dim = (uint8_t)dim;
+              c.split_n = (uint8_t)ns[q];
+              for (int k = 0; k < 4; k++) c.pin_op[k] = -1;
+              cs.push_back(c);
+              li_of.push_back(li);
+            }
+          }
+        }
+        if (cs.empty()) break;
+        CK(cudaMemcpy(d_round, cs.data(), sizeof(Cand) * cs.size(), cudaMemcpyHostToDevice));
+        DevOut mo;
+        mo.makespan = d_rms;
+        mo.status = d_rst;
+        mo.vmax = cur->rl.vcap;
+        rc = eval_batch(g, *cur, d_round, (int64_t)cs.size(), flags, st, mo);
+        std::vector<int64_t> ms(cs.size());
+        std::vector<uint8_t> sts(cs.size());
+        if (rc == FASTT_OK && (cudaMemcpy(ms.data(), d_rms, 8 * cs.size(), cudaMemcpyDeviceToHost) != cudaSuccess ||
+                               cudaMemcpy(sts.data(), d_rst, cs.size(), cudaMemcpyDeviceToHost) != cudaSuccess))
+          rc = fail(FASTT_ECUDA, "download round results");
+        int bi = -1;
+        for (size_t q = 0; rc == FASTT_OK && q < cs.size(); q++)
+          if (sts[q] == FASTT_CAND_OK && (bi < 0 || ms[q] < ms[bi])) bi = (int)q;
+        if (rc == FASTT_OK && bi >= 0 && ms[bi] < ft_old) {
+          // the winner's placement / order / start (one more evaluation with outputs)
+          vm = cur->rl.vcap;
+          o.vmax = vm;
+          CK(cudaMemcpy(d_c, &cs[bi], sizeof(Cand), cudaMemcpyHostToDevice));
+          rc = eval_batch(g, *cur, d_c, 1, flags, st, o);
+          if (rc == FASTT_OK) {
+            owned.emplace_back();
+            Base &nb = owned.back();
+            rc = materialize_base(g, *cur, cs[bi], nb, st);
+            if (rc == FASTT_OK) {
+              ft_old = ms[bi];
+              done[li_of[bi]] = 1;
+              sp_op.push_back(cs[bi].split_op);
+              sp_dim.push_back(cs[bi].split_dim);
+              sp_n.push_back(cs[bi].split_n);
+              vfinal = nb.V;
+              bplace.resize(vm);
+              bstart.resize(vm);
+              border.resize(vm);
+              CK(cudaMemcpy(bplace.data(), d_place, vm, cudaMemcpyDeviceToHost));
+              CK(cudaMemcpy(bstart.data(), d_start, 8 * vm, cudaMemcpyDeviceToHost));
+              CK(cudaMemcpy(border.data(), d_order, 4 * vm, cudaMemcpyDeviceToHost));
+              cur = &nb;
+              continue;
+            }
+          }
+        }
+        cudaFree(d_round);
+        cudaFree(d_rms);
+        cudaFree(d_rst);
+        if (rc != FASTT_OK) {
+          cleanup();
+          return rc;
+        }
+        break;
+      }
+    } else
     // Alg. 2 lines 7-14
     for (int32_t op : list) {
       std::vector<Cand> cs;

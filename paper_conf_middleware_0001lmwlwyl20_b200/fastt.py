@@ -66,6 +66,7 @@ SYMBOLS = ["fastt_load_graph", "fastt_free_graph", "fastt_graph_info", "fastt_ra
            "fastt_stream_info", "fastt_generate_candidates", "fastt_sweep_best", "fastt_split_search",
            "fastt_free_split_result", "fastt_last_timing", "fastt_last_error", "fastt_version"]
 F_TIMING = 16
+F_SPLIT_BEST = 32
 
 _lib = None
 
@@ -294,9 +295,9 @@ class Graph:
         return {"launches": int(t.launches), "candidates": int(t.candidates), "deferred": int(t.deferred),
                 "ms_sim": float(t.ms_sim), "ms_prep": float(t.ms_prep), "ms_total": float(t.ms_total)}
 
-    def split_search(self, flags=0, n_pow2_only=False, stream=None):
+    def split_search(self, flags=0, n_pow2_only=False, stream=None, best_improvement=False):
         r = fastt_split_result()
-        o = _opts(flags, stream)
+        o = _opts(flags | (F_SPLIT_BEST if best_improvement else 0), stream)
         _check(lib().fastt_split_search(self.h, C.byref(o), 1 if n_pow2_only else 0, C.byref(r)))
         try:
             n = r.n_splits

@@ -257,6 +257,54 @@ def test_split_search_configs(name):
     assert (a["placement"] == b["placement"]).all() and (a["order"] == b["order"]).all()
 
 
+@pytest.mark.parametrize("seed", [4, 13, 21, 32, 34, 39, 116, 122, 214, 1, 3])
+def test_split_search_best_random(seed):
+    desc = synth.random_dag(seed, V=40, G=4, caps="none", max_in=2)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    for flags in (0, F.F_CP_PIN):
+        a = gg.split_search(flags=flags, best_improvement=True)
+        b = og.split_search(flags=flags, best_improvement=True)
+        assert a["sp"] == b["sp"] and a["makespan"] == b["makespan"] and a["n_ops_final"] == b["n_ops_final"]
+        assert (a["placement"] == b["placement"]).all()
+        assert (a["start"] == b["start"]).all()
+        assert (a["order"] == b["order"]).all()
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C4"])
+def test_split_search_best_configs(name):
+    desc = synth.config(name)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    a = gg.split_search(flags=F.F_CP_PIN, n_pow2_only=(name == "C4"), best_improvement=True)
+    b = og.split_search(flags=O.F_CP_PIN, pow2_only=(name == "C4"), best_improvement=True)
+    assert a["sp"] == b["sp"] and a["makespan"] == b["makespan"]
+    assert (a["placement"] == b["placement"]).all() and (a["order"] == b["order"]).all()
+
+
+@pytest.mark.parametrize("name", ["C3", "C5"])
+def test_split_search_best_large_properties(name):
+    """C3/C5 best-improvement is minutes of oracle time, so check properties:
+    the sweep stream's SPLIT block (R21) is exactly round 1's batch in the
+    same enumeration order, so round 1 accepts its first argmin if it beats
+    BASE; the result never exceeds BASE; no op is split twice."""
+    desc = synth.config(name)
+    gg = F.Graph(desc)
+    a = gg.split_search(flags=F.F_CP_PIN, best_improvement=True)
+    gen = F.gen_params(seed=0)
+    n_split = gg.stream_info(gen, flags=F.F_CP_PIN)
+    c = gg.generate_candidates(gen, 0, n_split + 1, flags=F.F_CP_PIN)
+    r = gg.schedule_batch(c, flags=F.F_CP_PIN)
+    base = int(r["makespan"][0])
+    ms = np.where(r["status"][1:] == F.CAND_OK, r["makespan"][1:], F.INT64_MAX)
+    ops = [x[0] for x in a["sp"]]
+    assert len(set(ops)) == len(ops)
+    if len(ms) and ms.min() < base:
+        k = 1 + int(np.argmin(ms))
+        assert a["sp"][0] == (int(c[k]["split_op"]), int(c[k]["split_dim"]), int(c[k]["split_n"]))
+        assert a["makespan"] <= int(ms.min())
+    else:
+        assert a["sp"] == [] and a["makespan"] == base
+
+
 # ------------------------------------------------------------- device buffers
 
 def test_device_buffers_roundtrip():

@@ -297,19 +297,11 @@ def test_split_operation_properties(seed):
             O.OracleGraph(sd)
 
 
-@pytest.mark.parametrize("seed", range(8))
-def test_split_search_monotone(seed):
-    d = synth.random_dag(seed + 900, V=60, G=4, caps="none")
-    g = O.OracleGraph(d)
-    base = g.schedule(flags=O.F_CP_PIN)
-    ss = g.split_search(flags=O.F_CP_PIN)
-    assert ss["makespan"] <= base["makespan"]
-    if ss["sp"]:
-        assert ss["makespan"] < base["makespan"]
-    # SP ops come from the placement-aware CP of the initial DPOS (R15),
-    # recomputed here independently
+def _placed_cp(d, place):
+    """The placement-aware critical path of R15 (Alg. 2 lines 4-5), recomputed
+    here independently of the oracle: longest cost+comm path under `place`,
+    ties to the lower id."""
     rg = RC.G(d)
-    place = base["placement"][: d.n_ops].tolist()
     memo = {}
 
     def rk(i):
@@ -324,8 +316,78 @@ def test_split_search_monotone(seed):
     while rg.succ[cur]:
         cur = max([j for (j, _) in rg.succ[cur]], key=lambda j: (rk(j), -j))
         cp.append(cur)
+    return cp
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_split_search_monotone(seed):
+    d = synth.random_dag(seed + 900, V=60, G=4, caps="none")
+    g = O.OracleGraph(d)
+    base = g.schedule(flags=O.F_CP_PIN)
+    ss = g.split_search(flags=O.F_CP_PIN)
+    assert ss["makespan"] <= base["makespan"]
+    if ss["sp"]:
+        assert ss["makespan"] < base["makespan"]
+    # SP ops come from the placement-aware CP of the initial DPOS (R15)
+    cp = _placed_cp(d, base["placement"][: d.n_ops].tolist())
     for (op, dim, n) in ss["sp"]:
         assert op in cp and d.split_mask[op] & (1 << dim) and 2 <= n <= d.n_devices
+
+
+# ------------------------------------- best-improvement split search (NEXT N2)
+
+def test_split_search_best_a2_golden():
+    """A.2: X is the only splittable op and G=2 allows only n=2, so both
+    searches accept exactly that split (golden a2 "split_search")."""
+    gd = gold("a2_split_chain.json")
+    ss = O.OracleGraph(synth.split_chain()).split_search(flags=O.F_CP_PIN, best_improvement=True)
+    assert [list(x) for x in ss["sp"]] == gd["split_search"]["sp"]
+    assert ss["makespan"] == gd["split_search"]["makespan"]
+
+
+# seeds where the best-improvement search differs from Alg. 2 or splits twice
+BI_SEEDS = [4, 13, 21, 32, 34, 39, 116, 122, 214, 1, 3]
+
+
+@pytest.mark.parametrize("seed", BI_SEEDS)
+def test_split_search_best_first_round_is_brute_force_min(seed):
+    """Round 1 of the best-improvement search is the minimum over every single
+    split of every split-eligible CP op of G0 (brute force through SPLIT
+    candidates); later rounds only lower the makespan; no op is split twice;
+    the emitted schedule respects every surviving original edge."""
+    d = synth.random_dag(seed, V=40, G=4, caps="none", max_in=2)
+    g = O.OracleGraph(d)
+    rg = RC.G(d)
+    base = g.schedule(flags=O.F_CP_PIN)
+    bi = g.split_search(flags=O.F_CP_PIN, best_improvement=True)
+    cp = _placed_cp(d, base["placement"][: d.n_ops].tolist())
+    singles = {}
+    for op in cp:
+        for dim in (0, 1):
+            if d.split_mask[op] & (1 << dim):
+                for n in range(2, d.n_devices + 1):
+                    r = g.schedule(O.make_cand(O.KIND_SPLIT, split=(op, dim, n)), flags=O.F_CP_PIN)
+                    if r["status"] == O.CAND_OK:
+                        singles[(op, dim, n)] = r["makespan"]
+    m1 = min(singles.values(), default=None)
+    if m1 is not None and m1 < base["makespan"]:
+        assert bi["sp"] and singles[tuple(bi["sp"][0])] == m1
+        assert bi["makespan"] <= m1 < base["makespan"]
+    else:
+        assert bi["sp"] == [] and bi["makespan"] == base["makespan"]
+    ops = [x[0] for x in bi["sp"]]
+    assert len(set(ops)) == len(ops) and set(ops) <= set(cp)
+    split = set(ops)
+    place, start = bi["placement"], bi["start"]
+    for i in range(d.n_ops):
+        if i in split:
+            assert place[i] == 0xFF and start[i] == -1
+            continue
+        fi = start[i] + d.cost[i][place[i]]
+        assert 0 <= start[i] and fi <= bi["makespan"]
+        for (j, b) in rg.succ[i]:
+            if j not in split:
+                assert start[j] >= fi + rg.comm(b, place[i], place[j])
 
 
 # ------------------------------------------------------ memory / statuses
