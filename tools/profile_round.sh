@@ -1,0 +1,14 @@
+#!/bin/bash
+# One GPU call's worth of round measurements (run under gpurun from the repo root):
+#   1. the bench line (no profiler), 2. the ncu launch list of a short bench,
+#   3. one `ncu --set full` capture of the main k_sim sweep launch.
+# usage: tools/profile_round.sh <tag>
+set -u
+tag=${1:-r01}
+mkdir -p gpurun_out
+python bench.py > gpurun_out/${tag}_bench.json 2> gpurun_out/${tag}_bench.err
+ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/${tag}_launches.csv \
+    python bench.py --steps 1 --warmup 3 --candidates 200000 --no-e2e --no-cpu > gpurun_out/${tag}_ncu_bench.log 2>&1
+ncu --set full --clock-control none --import-source on -k regex:k_sim -c 4 -o gpurun_out/${tag}_k_sim -f \
+    python tools/ncu_sim.py 20000 > gpurun_out/${tag}_ncu_full.log 2>&1
+ls -la gpurun_out
