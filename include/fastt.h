@@ -73,7 +73,7 @@ enum { FASTT_DIM_BATCH = 0, FASTT_DIM_CHANNEL = 1 };
 /* option flags */
 enum {
   FASTT_F_CP_PIN = 1u << 0,        /* pin critical-path ops to CP devices (Alg. 1 lines 4-5, 9-10) */
-  FASTT_F_POLICY_INSERT = 1u << 1, /* insertion-based avail[j]; NOT YET SUPPORTED -> EUNSUP */
+  FASTT_F_POLICY_INSERT = 1u << 1, /* insertion-based avail[j] (R1i; NEXT N1): earliest idle slot that fits */
   FASTT_F_OUT_DEVICE = 1u << 2,    /* output pointers are device pointers */
   FASTT_F_IN_DEVICE = 1u << 3,     /* candidate input pointer is a device pointer */
   FASTT_F_TIMING = 1u << 4,        /* record CUDA events around the kernels of this call (fastt_last_timing) */

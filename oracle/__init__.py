@@ -25,6 +25,7 @@ CAND_OK, CAND_INFEASIBLE, CAND_BADSPEC = 0, 1, 2
 KIND_BASE, KIND_PIN, KIND_SPLIT = 0, 1, 2
 DIM_BATCH, DIM_CHANNEL = 0, 1
 F_CP_PIN = 1
+F_POLICY_INSERT = 2
 
 CAND_DTYPE = np.dtype(
     [("kind", "u1"), ("n_pins", "u1"), ("split_dim", "u1"), ("split_n", "u1"),

@@ -44,6 +44,7 @@
 #define FO_DIM_CHANNEL 1
 
 #define FO_F_CP_PIN 1u
+#define FO_F_POLICY_INSERT 2u
 
 #define FO_INF INT64_MAX
 #define FO_MAXG 32
@@ -471,6 +472,28 @@ static int32_t fo_critical_path(const fo_graph *g, const int64_t *rank, int32_t 
   return n;
 }
 
+/* INSERT policy (reading R1i): "avail[j] is the start time of"
+ * the earliest idle time slot on d_j whose length suffices for the op and
+ * which preserves precedence.  The ops already placed on d_j (zero-length
+ * ones included) form a sequence sorted by (ST, FT); its idle time slots are
+ * the gaps of positive length between consecutive ops -- [0, s_1),
+ * [f_1, s_2), ... -- and the open-ended slot [f_last, inf) after the last
+ * op.  The op, ready at r (its predecessors' data arrived), fits slot
+ * [a, b) iff max(a, r) + w <= b; EST = max(a, r) of the first slot that
+ * fits. */
+static int64_t fo_idle_slot(const int64_t *s, const int64_t *f, int32_t n, int64_t r, int64_t w) {
+  int64_t a = 0;
+  for (int32_t k = 0; k < n; k++) {
+    int64_t b = s[k];
+    if (b > a) {
+      int64_t t = a > r ? a : r;
+      if (t + w <= b) return t;
+    }
+    a = f[k];
+  }
+  return a > r ? a : r;
+}
+
 /* DPOS (Alg. 1) for one candidate: graph g (already split if the
  * candidate splits), perturbation pins pin[] (-1 = free), flags.
  * Ranks are written to rank[] (V entries). */
@@ -530,6 +553,16 @@ static void fo_dpos(const fo_graph *g, const int32_t *pin, uint32_t flags, int64
   int32_t *indeg = malloc(sizeof(int32_t) * ((size_t)V + 1));
   int32_t *ready = malloc(sizeof(int32_t) * ((size_t)V + 1));
   int32_t nready = 0, seq = 0;
+  /* INSERT (R1i): per device the [ST, FT] of the ops placed on it,
+   * kept sorted by (ST, FT) */
+  const int insert = (flags & FO_F_POLICY_INSERT) != 0;
+  int64_t *bs = NULL, *bf = NULL;
+  int32_t nb[FO_MAXG];
+  for (int d = 0; d < G; d++) nb[d] = 0;
+  if (insert) {
+    bs = malloc(sizeof(int64_t) * ((size_t)V * G + 1));
+    bf = malloc(sizeof(int64_t) * ((size_t)V * G + 1));
+  }
   for (int d = 0; d < G; d++) r->peak[d] = 0;
   for (int32_t i = 0; i < V; i++) {
     indeg[i] = g->pred_off[i + 1] - g->pred_off[i];
@@ -551,12 +584,14 @@ static void fo_dpos(const fo_graph *g, const int32_t *pin, uint32_t flags, int64
      * (R1 append, R6 actual transfer time, 0 when co-located) */
 #define FO_EST(dev, outv)                                                          \
   do {                                                                             \
-    int64_t est_ = avail[dev];                                                     \
+    int64_t est_ = insert ? 0 : avail[dev];                                        \
     for (int32_t e_ = g->pred_off[i]; e_ < g->pred_off[i + 1]; e_++) {             \
       int32_t m_ = g->pred_src[e_];                                                \
       int64_t t_ = r->finish[m_] + fo_comm(g, g->pred_bytes[e_], r->place[m_], dev); \
       if (t_ > est_) est_ = t_;                                                    \
     }                                                                              \
+    if (insert) est_ = fo_idle_slot(bs + (int64_t)(dev) * V, bf + (int64_t)(dev) * V, nb[dev], est_, \
+                                    g->cost[(int64_t)i * G + (dev)]);             \
     (outv) = est_;                                                                 \
   } while (0)
     if (pin && pin[i] >= 0) {
@@ -594,6 +629,19 @@ static void fo_dpos(const fo_graph *g, const int32_t *pin, uint32_t flags, int64
     r->finish[i] = est_sel + g->cost[(int64_t)i * G + dsel];
     r->place[i] = (uint8_t)dsel;
     avail[dsel] = r->finish[i];
+    if (insert) {
+      /* keep the device's op sequence sorted by (ST, FT) */
+      int64_t *s_ = bs + (int64_t)dsel * V, *f_ = bf + (int64_t)dsel * V;
+      int32_t pos = nb[dsel];
+      while (pos > 0 && (s_[pos - 1] > r->start[i] || (s_[pos - 1] == r->start[i] && f_[pos - 1] > r->finish[i]))) {
+        s_[pos] = s_[pos - 1];
+        f_[pos] = f_[pos - 1];
+        pos--;
+      }
+      s_[pos] = r->start[i];
+      f_[pos] = r->finish[i];
+      nb[dsel]++;
+    }
     used[dsel] += mi;
     r->dq[i] = seq;
     r->deq[seq] = i;
@@ -623,6 +671,7 @@ static void fo_dpos(const fo_graph *g, const int32_t *pin, uint32_t flags, int64
   for (int d = 0; d < G; d++) r->peak[d] = used[d];
 done:
   free(cpdev); free(indeg); free(ready);
+  free(bs); free(bf);
 }
 
 /* ----------------------------------------------------- candidate handling */

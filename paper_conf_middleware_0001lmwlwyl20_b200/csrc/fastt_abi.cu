@@ -233,7 +233,7 @@ struct fastt_graph {
   uint8_t *split_mask_dev = nullptr;
   Base base;
   std::vector<uint8_t> split_mask_h;
-  StreamCache streams[4];
+  StreamCache streams[8];
   // arena (per base layout)
   size_t arena_raw_total = 0, arena_prep_total = 0;
   int arena_slots = 0;
@@ -247,6 +247,8 @@ struct fastt_graph {
   int64_t sim_ncap = 0;
   size_t sim_smem = 0;
   void *slab = nullptr;
+  void *gap = nullptr;  // INSERT idle-slot pools, one per candidate slot (lazy)
+  int64_t gap_stride = 0;
   int64_t *wbest = nullptr, *best_dev = nullptr;
   unsigned long long *counters = nullptr;  // [0] work counter, [1] deferred count
   int64_t *defer_q = nullptr;
@@ -423,13 +425,15 @@ static int gshift_of(int G) {
 
 // simulation workspace: one candidate per lane group (32 >> gshift per warp),
 // each with a ready bitmap in shared memory and an 8/16 B-per-op slab in HBM
-static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need) {
+static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need, uint32_t flags = 0) {
   int64_t ncap = B.pl.ncap;
   if (!g->slab || g->sim_tbits != B.tbits || g->sim_ncap < ncap) {
     cudaFree(g->slab);
     cudaFree(g->wbest);
+    cudaFree(g->gap);
     g->slab = nullptr;
     g->wbest = nullptr;
+    g->gap = nullptr;
     const int gsh = gshift_of(g->G);
     const int cpw = 32 >> gsh;
     int leaf = (int)((ncap + 31) / 32);
@@ -449,6 +453,17 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     CK(cudaMalloc(&g->wbest, sizeof(int64_t) * 2 * nslot));
     g->sim_tbits = B.tbits;
     g->sim_ncap = ncap;
+  }
+  if ((flags & FASTT_F_POLICY_INSERT) && !g->gap) {
+    // INSERT: at most one idle-slot record per placed op per candidate
+    const int64_t nslot = (int64_t)g->sim_grid * (g->sim_block / 32) * g->sim_cpw;
+    g->gap_stride = g->sim_ncap + 1;
+    const size_t rec = B.tbits == 32 ? sizeof(GapRec<uint32_t>) : sizeof(GapRec<uint64_t>);
+    if (cudaMalloc(&g->gap, (size_t)nslot * g->gap_stride * rec) != cudaSuccess) {
+      cudaGetLastError();
+      g->gap = nullptr;
+      return fail(FASTT_ENOMEM, "INSERT idle-slot pools (%lld slots)", (long long)nslot);
+    }
   }
   if (!g->counters) {
     CK(cudaMalloc(&g->counters, 2 * sizeof(unsigned long long)));
@@ -484,6 +499,11 @@ static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
   for (int d = 0; d < g->G; d++)
     if (g->gch.cap[d] != I64MAX) a.cap_check = 1;
   a.need_mem = a.cap_check;
+  if (flags & FASTT_F_POLICY_INSERT) {
+    a.ins = 1;
+    a.gap = g->gap;
+    a.gap_stride = g->gap_stride;
+  }
   return a;
 }
 
@@ -509,7 +529,7 @@ static fastt_status run_prep(fastt_graph *g, const Base &B, int nslots, cudaStre
 // makespan before every step, the base CP rounds.
 static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cudaStream_t st) {
   Base::Snap &S = B.snap[flags & FASTT_F_CP_PIN ? 1 : 0];
-  if (S.valid) return FASTT_OK;
+  if (S.valid || (flags & FASTT_F_POLICY_INSERT)) return FASTT_OK;  // (no sharing under INSERT)
   for (int d = 0; d < g->G; d++)
     if (g->gch.cap[d] != I64MAX) return FASTT_OK;  // sharing needs unlimited memory
   const size_t tb = B.tbits / 8, n = (size_t)B.pl.ncap;
@@ -568,7 +588,7 @@ static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cud
 // enable prefix sharing on a launch when the snapshot exists
 static void use_snapshot(const Base &B, uint32_t flags, SimArgs &a) {
   const Base::Snap &S = B.snap[flags & FASTT_F_CP_PIN ? 1 : 0];
-  if (!S.valid || a.need_mem || a.out.place) return;
+  if (!S.valid || a.need_mem || a.out.place || a.ins) return;
   a.snap_mode = 2;
   a.snap_round_dev = S.round_dev;
   a.snap_dq = S.dq;
@@ -610,8 +630,8 @@ struct DevOut {
 static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int64_t n, uint32_t flags,
                                cudaStream_t st, DevOut o) {
   if (n <= 0) return FASTT_OK;
-  TRY(ensure_sim(g, B, n));
-  const bool sharing = g->share && !o.peak && !o.place && n >= 64;
+  TRY(ensure_sim(g, B, n, flags));
+  const bool sharing = g->share && !o.peak && !o.place && n >= 64 && !(flags & FASTT_F_POLICY_INSERT);
   if (sharing) TRY(ensure_snapshot(g, B, flags, st));  // before the work counters are reset
   if (o.place) CK(cudaMemsetAsync(o.place, 0xFF, (size_t)n * o.vmax, st));
   if (o.start) {
@@ -741,7 +761,7 @@ static fastt_status split_list(fastt_graph *g, Base &B, const uint8_t *d_place, 
 }
 
 static fastt_status ensure_stream(fastt_graph *g, uint32_t flags, int pow2, cudaStream_t st, StreamCache **out) {
-  int key = (int)(flags & FASTT_F_CP_PIN) | (pow2 ? 2 : 0);
+  int key = (int)(flags & FASTT_F_CP_PIN) | (pow2 ? 2 : 0) | (flags & FASTT_F_POLICY_INSERT ? 4 : 0);
   StreamCache &S = g->streams[key];
   *out = &S;
   if (S.valid) return FASTT_OK;
@@ -1093,6 +1113,7 @@ void fastt_free_graph(fastt_graph *g) {
     cudaFree(g->slot_result);
     cudaFree(g->slot_index);
     cudaFree(g->slab);
+    cudaFree(g->gap);
     cudaFree(g->wbest);
     cudaFree(g->best_dev);
     cudaFree(g->counters);
@@ -1191,7 +1212,6 @@ fastt_status fastt_schedule_batch(const fastt_graph *gc_, const fastt_candidate 
   fastt_graph *g = (fastt_graph *)gc_;
   if (!g || n < 0 || (n > 0 && (!cands || !makespan || !status))) return fail(FASTT_EINVAL, "bad argument");
   const uint32_t flags = flags_of(opts);
-  if (flags & FASTT_F_POLICY_INSERT) return fail(FASTT_EUNSUP, "FASTT_F_POLICY_INSERT is not implemented yet");
   if (n == 0) return FASTT_OK;
   std::lock_guard<std::mutex> lk(g->mu);
   Dev guard(g->dev);
@@ -1289,7 +1309,6 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
   fastt_graph *g = (fastt_graph *)gc_;
   if (!g || !gen || !best) return fail(FASTT_EINVAL, "NULL argument");
   const uint32_t flags = flags_of(opts);
-  if (flags & FASTT_F_POLICY_INSERT) return fail(FASTT_EUNSUP, "FASTT_F_POLICY_INSERT is not implemented yet");
   std::lock_guard<std::mutex> lk(g->mu);
   Dev guard(g->dev);
   cudaStream_t st = stream_of(opts);
@@ -1297,7 +1316,7 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
   TRY(ensure_stream(g, flags, gen->n_pow2_only, st, &S));
   TRY(check_gen(g, *S, gen, first, n, stride));
   Base &B = g->base;
-  TRY(ensure_sim(g, B, n));
+  TRY(ensure_sim(g, B, n, flags));
   const int64_t nwarps = (int64_t)g->sim_grid * (g->sim_block / 32) * g->sim_cpw;  // candidate slots
   {
     std::vector<int64_t> init(2 * nwarps);
@@ -1421,9 +1440,8 @@ fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, 
                                 fastt_split_result *out) {
   fastt_graph *g = (fastt_graph *)gc_;
   if (!g || !out) return fail(FASTT_EINVAL, "NULL argument");
-  const uint32_t flags = flags_of(opts) & FASTT_F_CP_PIN;
+  const uint32_t flags = flags_of(opts) & (FASTT_F_CP_PIN | FASTT_F_POLICY_INSERT);
   const bool best_mode = (flags_of(opts) & FASTT_F_SPLIT_BEST) != 0;
-  if (flags_of(opts) & FASTT_F_POLICY_INSERT) return fail(FASTT_EUNSUP, "FASTT_F_POLICY_INSERT is not implemented yet");
   memset(out, 0, sizeof *out);
   std::lock_guard<std::mutex> lk(g->mu);
   Dev guard(g->dev);

@@ -365,8 +365,9 @@ __device__ __noinline__ void cp_rounds_g(const PrepGraph *pg, int np, const uint
 // Several candidates per warp: lane group g (GP = 2^GSH lanes, GP >= G) owns
 // one candidate; lane d of the group is device d.  The main loop keeps the
 // warp converged (groups that finished idle) so every shuffle/vote is a
-// full-warp instruction.  T: time type; MEM: track per-device memory.
-template <typename T, int GSH, bool MEM>
+// full-warp instruction.  T: time type; MEM: track per-device memory;
+// INS: insertion policy (R1i) -- lane d keeps device d's idle slots.
+template <typename T, int GSH, bool MEM, bool INS>
 __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
   typedef typename Slab<T>::W W;
   constexpr int GP = 1 << GSH;   // lanes per candidate (>= G)
@@ -400,6 +401,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
   const bool cp_on = (a.flags & 1u) != 0;
   const bool cap_chk = MEM && a.cap_check != 0;
   const bool fastcomm = sizeof(T) == 4 && K == 1;
+  GapRec<T> *const gpool = INS ? (GapRec<T> *)a.gap + cslot * a.gap_stride : nullptr;
   if (d == 0) {
     s_best[lead][0] = a.track_best ? a.wbest[2 * cslot] : I64MAX;
     s_best[lead][1] = a.track_best ? a.wbest[2 * cslot + 1] : -1;
@@ -520,7 +522,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
     // starts from the recorded BASE state at t0 (exact)
     int32_t t0 = 0;
     bool share = false;
-    if (run && !MEM && !want_out && a.snap_mode == 2 && a.mode != 2) {
+    if (run && !MEM && !INS && !want_out && a.snap_mode == 2 && a.mode != 2) {
       t0 = n;
       for (int k = 0; k < np; k++) {
         const int32_t dq = (int32_t)__ldg(a.snap_dq + pp[k]);
@@ -542,6 +544,9 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
     }
     uint32_t top = 0;
     T avail = 0, makespan = 0;
+    // INSERT: this lane's device's idle slots before `avail` (a list sorted
+    // by start, head/tail record), and the group's record count
+    uint32_t ghead = NONE, gtail = NONE, galloc = 0;
     if (run && share) {
       avail = d < G ? __ldg((const T *)a.snap_avail + (size_t)t0 * G + d) : (T)0;
       makespan = __ldg((const T *)a.snap_ms + t0);
@@ -673,7 +678,8 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       }
       const uint32_t sdeg = ((uint32_t)d < nsucc) ? Slab<T>::indeg(slab0, SLOT(s0)) : 1u;
       // EST = max(avail[d], max_pred FT + c(pred -> i on d))   (R1, R6)
-      T est = avail;
+      // (INSERT: first the data-ready time r, then the idle-slot search)
+      T est = INS ? (T)0 : avail;
 #pragma unroll
       for (int k = 0; k < 4; k++) {
         T cm;
@@ -698,6 +704,30 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
             est = term > est ? term : est;
           }
         }
+      }
+      // INSERT (R1i): the first idle slot [ga, gb) before avail
+      // with max(ga, r) + w <= gb, else the open-ended slot at avail
+      uint32_t gk = NONE, gprev = NONE, gnx = NONE;
+      T ga = 0, gbb = 0;
+      if (INS && live && d < G && est < avail) {
+        uint32_t prev = NONE;
+        T t = avail;
+        for (uint32_t k = ghead; k != NONE;) {
+          const GapRec<T> e = gpool[k];
+          const T tt = e.a > est ? e.a : est;
+          if (tt + cst <= e.b) {
+            gk = k;
+            gprev = prev;
+            gnx = e.next;
+            ga = e.a;
+            gbb = e.b;
+            t = tt;
+            break;
+          }
+          prev = k;
+          k = e.next;
+        }
+        est = t;
       }
       const T eft = est + cst;
 
@@ -762,8 +792,50 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
         }
       }
       tstep++;
+      if (INS) {
+        // the chosen device's lane updates its idle slots
+        bool alloc = false;
+        if (go && d == dsel) {
+          if (gk != NONE) {
+            const bool left = est > ga, right = est + cst < gbb;
+            if (left && right) {
+              GapRec<T> ne;
+              ne.a = est + cst;
+              ne.b = gbb;
+              ne.next = gnx;
+              gpool[galloc] = ne;
+              gpool[gk].b = est;
+              gpool[gk].next = galloc;
+              if (gtail == gk) gtail = galloc;
+              alloc = true;
+            } else if (left) {
+              gpool[gk].b = est;
+            } else if (right) {
+              gpool[gk].a = est + cst;
+            } else {
+              if (gprev == NONE) ghead = gnx;
+              else gpool[gprev].next = gnx;
+              if (gtail == gk) gtail = gprev;
+            }
+          } else {
+            if (est > avail) {
+              GapRec<T> ne;
+              ne.a = avail;
+              ne.b = est;
+              ne.next = NONE;
+              gpool[galloc] = ne;
+              if (gtail == NONE) ghead = galloc;
+              else gpool[gtail].next = galloc;
+              gtail = galloc;
+              alloc = true;
+            }
+            avail = mn;
+          }
+        }
+        if (__ballot_sync(FULL, alloc) & gm) galloc++;
+      }
       if (go && d == dsel) {
-        avail = mn;
+        if (!INS) avail = mn;
         if (MEM) {
           used += mem;
           if (forced >= 0 && !pert) reserved -= mem;
@@ -856,24 +928,28 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
   }
 }
 
-template <typename T, bool MEM>
+template <typename T, bool MEM, bool INS>
 static const void *sim_fn_t(int gshift) {
   switch (gshift) {
-    case 0: return (const void *)k_sim<T, 0, MEM>;
-    case 1: return (const void *)k_sim<T, 1, MEM>;
-    case 2: return (const void *)k_sim<T, 2, MEM>;
-    case 3: return (const void *)k_sim<T, 3, MEM>;
-    case 4: return (const void *)k_sim<T, 4, MEM>;
-    default: return (const void *)k_sim<T, 5, MEM>;
+    case 0: return (const void *)k_sim<T, 0, MEM, INS>;
+    case 1: return (const void *)k_sim<T, 1, MEM, INS>;
+    case 2: return (const void *)k_sim<T, 2, MEM, INS>;
+    case 3: return (const void *)k_sim<T, 3, MEM, INS>;
+    case 4: return (const void *)k_sim<T, 4, MEM, INS>;
+    default: return (const void *)k_sim<T, 5, MEM, INS>;
   }
 }
-static const void *sim_fn(int tbits, int gshift, bool mem) {
-  if (tbits == 32) return mem ? sim_fn_t<uint32_t, true>(gshift) : sim_fn_t<uint32_t, false>(gshift);
-  return mem ? sim_fn_t<uint64_t, true>(gshift) : sim_fn_t<uint64_t, false>(gshift);
+template <typename T>
+static const void *sim_fn_m(int gshift, bool mem, bool ins) {
+  if (ins) return mem ? sim_fn_t<T, true, true>(gshift) : sim_fn_t<T, false, true>(gshift);
+  return mem ? sim_fn_t<T, true, false>(gshift) : sim_fn_t<T, false, false>(gshift);
+}
+static const void *sim_fn(int tbits, int gshift, bool mem, bool ins = false) {
+  return tbits == 32 ? sim_fn_m<uint32_t>(gshift, mem, ins) : sim_fn_m<uint64_t>(gshift, mem, ins);
 }
 
 void launch_sim(const SimArgs &a, int tbits, int grid, int block, size_t smem, cudaStream_t st) {
-  const void *f = sim_fn(tbits, a.gshift, a.need_mem != 0);
+  const void *f = sim_fn(tbits, a.gshift, a.need_mem != 0, a.ins != 0);
   SimArgs aa = a;
   void *args[] = {&aa};
   cudaLaunchKernel(f, dim3(grid), dim3(block), args, smem, st);
@@ -888,8 +964,9 @@ int sim_occupancy(int tbits, int gshift, int block, size_t smem) {
   return nb;
 }
 cudaError_t sim_set_smem(int tbits, int gshift, size_t smem) {
-  for (int mem = 0; mem < 2; mem++) {
-    cudaError_t e = cudaFuncSetAttribute(sim_fn(tbits, gshift, mem), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  for (int v = 0; v < 4; v++) {
+    cudaError_t e = cudaFuncSetAttribute(sim_fn(tbits, gshift, v & 1, v >> 1),
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
   }
   return cudaSuccess;

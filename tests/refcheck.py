@@ -7,7 +7,8 @@ the paper's definitions as brute force / verification routines.
   * an APPEND evaluator of a fixed (placement, order) (R1, R6),
   * brute force over all placements x all topological orders,
   * schedule invariants,
-  * a greedy-step replay checker.
+  * a greedy-step replay checker, APPEND or INSERT (R1i, EST by
+    brute force over time).
 """
 from __future__ import annotations
 
@@ -193,10 +194,37 @@ def check_invariants(g: G, res, pin=None):
             assert place[i] == d
 
 
-def check_greedy_steps(g: G, res, rank, cp_dev=None):
+def est_insert(ops, r, w):
+    """INSERT (R1i) by brute force over time.  ops = [(ST, FT)] of
+    the ops already on the device (zero-length included).  t is feasible iff
+    t is at or after the end of every op (the open-ended slot), or the op
+    [t, t+w] conflicts with none of them (w > 0: no overlap with any [s, f),
+    a zero-length op p counting as an obstacle when t < p < t+w; w = 0: t not
+    strictly inside any op) and, for w = 0, the device is idle just before or
+    just after t (t touches an idle slot of positive length; zero-length ops
+    at t do not count).  The earliest feasible t is r or the end of some op."""
+    last = max([f for (_, f) in ops] + [0])
+    for t in sorted({r} | {f for (_, f) in ops if f >= r}):
+        if t >= last:
+            return t
+        if w > 0:
+            if not any(s < t + w and t < f for (s, f) in ops):
+                return t
+            continue
+        if any(s < t < f for (s, f) in ops):
+            continue
+        left_idle = t > 0 and not any(s < t <= f for (s, f) in ops)
+        right_idle = not any(s <= t < f for (s, f) in ops)
+        if left_idle or right_idle:
+            return t
+    raise AssertionError("unreachable: the open-ended slot always fits")
+
+
+def check_greedy_steps(g: G, res, rank, cp_dev=None, insert=False):
     """every dequeued op is the max-(rank, -id) ready op and every
     free op sits on a device of minimum EFT (ties: lowest id) among the
-    memory-feasible ones, given the partial schedule."""
+    memory-feasible ones, given the partial schedule.  insert=True: EST by
+    est_insert (busy intervals of the ops placed so far) instead of APPEND."""
     V = g.V
     deq = [x for x in res["dequeue"][:V].tolist() if x >= 0]
     place = res["placement"][:V].tolist()
@@ -209,6 +237,12 @@ def check_greedy_steps(g: G, res, rank, cp_dev=None):
         for i, d in cp_dev.items():
             reserved[d] += g.mem[i]
     FT = {}
+    busy = [[] for _ in range(g.G)]
+
+    def est_on(i, d):
+        r = max([0 if insert else avail[d]] + [FT[p] + g.comm(b, place[p], d) for (p, b) in g.pred[i]])
+        return est_insert(busy[d], r, g.cost[i][d]) if insert else r
+
     for i in deq:
         ready = [j for j in range(V) if j not in done and all(p in done for (p, _) in g.pred[j])]
         best = max(ready, key=lambda j: (rank[j], -j))
@@ -216,19 +250,20 @@ def check_greedy_steps(g: G, res, rank, cp_dev=None):
         if cp_dev and i in cp_dev:
             d = cp_dev[i]
             reserved[d] -= g.mem[i]
-            est = max([avail[d]] + [FT[p] + g.comm(b, place[p], d) for (p, b) in g.pred[i]])
+            est = est_on(i, d)
         else:
             effs = []
             for d in range(g.G):
                 if used[d] + reserved[d] + g.mem[i] > g.cap[d]:
                     continue
-                est = max([avail[d]] + [FT[p] + g.comm(b, place[p], d) for (p, b) in g.pred[i]])
+                est = est_on(i, d)
                 effs.append((est + g.cost[i][d], d, est))
             eft, d, est = min(effs)
             assert place[i] == d, "device of minimum EFT (lowest id on ties)"
         assert start[i] == est
         FT[i] = est + g.cost[i][d]
         avail[d] = FT[i]
+        busy[d].append((est, FT[i]))
         used[d] += g.mem[i]
         done.add(i)
     assert len(done) == V

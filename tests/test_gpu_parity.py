@@ -370,3 +370,75 @@ def test_prefix_sharing_configs(name):
     for k in list(range(0, len(c), step)) + [0, len(c) - 1]:
         assert int(r["makespan"][k]) == og.schedule(c[k], flags=F.F_CP_PIN, outputs=False)["makespan"], (name, k)
     assert gg.sweep_best(gen, 0, ns + n, flags=F.F_CP_PIN) == g0.sweep_best(gen, 0, ns + n, flags=F.F_CP_PIN)
+
+
+# ------------------------------------------------ INSERT policy (R1i, NEXT N1)
+
+INS = F.F_POLICY_INSERT
+
+
+def test_a3_insert_golden_on_gpu():
+    a3 = json.load(open(os.path.join(GOLD, "a3_append_vs_insert.json")))
+    g = F.Graph(synth.append_vs_insert())
+    c = np.array([F.make_candidate(F.KIND_PIN, pins=[(1, 1)])])
+    r = g.schedule_batch(c, flags=F.F_CP_PIN | INS, placement=True, start=True)
+    assert int(r["makespan"][0]) == a3["insert"]["makespan"]
+    assert r["placement"][0][:3].tolist() == a3["insert"]["placement"]
+    assert r["start"][0][:3].tolist() == a3["insert"]["start"]
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_insert_fuzz_random_dags(seed):
+    desc = synth.random_dag(seed + 3000)
+    rng = np.random.default_rng(seed + 7)
+    cands = random_cands(desc, rng, 24)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    for flags in (INS, INS | F.F_CP_PIN):
+        compare(desc, cands, flags, gg=gg, og=og)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_insert_zero_cost_heavy(seed):
+    """Many zero-cost ops: zero-length slots and ops splitting idle slots."""
+    desc = synth.random_dag(seed + 3100, V=120, G=3, zero_frac=0.5, caps="none")
+    rng = np.random.default_rng(seed)
+    compare(desc, random_cands(desc, rng, 16), INS | F.F_CP_PIN)
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C4", "C5"])
+def test_insert_configs_sampled(name):
+    desc = synth.config(name)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    pow2 = name == "C4"
+    flags = F.F_CP_PIN | INS
+    gen = F.gen_params(seed=0xFA57, n_pow2_only=pow2)
+    n_split = gg.stream_info(gen, flags=flags)
+    assert n_split == og.stream_info(flags=flags, pow2_only=pow2)[0]
+    idx = [0] + list(range(1, min(n_split, 2) + 1)) + [n_split + 1 + 7919 * k for k in range(3 if name == "C5" else 8)]
+    cands = np.concatenate([gg.generate_candidates(gen, i, 1, flags=flags) for i in idx])
+    ocands = np.concatenate([og.generate(0xFA57, i, 1, flags=flags, pow2_only=pow2) for i in idx])
+    assert cands.tobytes() == ocands.tobytes()
+    compare(desc, cands, flags, gg=gg, og=og, outputs=(name != "C5"))
+
+
+@pytest.mark.parametrize("name", ["C1", "C4"])
+def test_insert_sweep(name):
+    desc = synth.config(name)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    pow2 = name == "C4"
+    flags = F.F_CP_PIN | INS
+    gen = F.gen_params(seed=21, n_pow2_only=pow2)
+    n = 300
+    assert gg.sweep_best(gen, 0, n, flags=flags) == tuple(
+        (lambda o: (o["makespan"], o["index"]))(og.sweep(21, 0, n, flags=flags, pow2_only=pow2)))
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_insert_split_search(seed):
+    desc = synth.random_dag(seed + 950, V=50, G=4, caps="none", max_in=2)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    for best in (False, True):
+        a = gg.split_search(flags=INS | F.F_CP_PIN, best_improvement=best)
+        b = og.split_search(flags=INS | F.F_CP_PIN, best_improvement=best)
+        assert a["sp"] == b["sp"] and a["makespan"] == b["makespan"]
+        assert (a["placement"] == b["placement"]).all() and (a["start"] == b["start"]).all()

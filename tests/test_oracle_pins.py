@@ -87,9 +87,19 @@ def test_a3_append_golden():
     assert r["start"][:3].tolist() == gd["append"]["start"]
 
 
+def test_a3_insert_golden():
+    gd = gold("a3_append_vs_insert.json")
+    g = O.OracleGraph(synth.append_vs_insert())
+    c = O.make_cand(O.KIND_PIN, pins=[(1, 1)])
+    r = g.schedule(c, flags=O.F_CP_PIN | O.F_POLICY_INSERT)
+    assert r["makespan"] == gd["insert"]["makespan"]
+    assert r["placement"][:3].tolist() == gd["insert"]["placement"]
+    assert r["start"][:3].tolist() == gd["insert"]["start"]
+
+
 # -------------------------------------------------------- closed forms (P3)
 
-@pytest.mark.parametrize("flags", [0, O.F_CP_PIN])
+@pytest.mark.parametrize("flags", [0, O.F_CP_PIN, O.F_POLICY_INSERT, O.F_CP_PIN | O.F_POLICY_INSERT])
 def test_single_device_is_sum_of_costs(flags):
     for seed in range(20):
         d = synth.random_dag(seed, G=1, caps="none")
@@ -176,6 +186,22 @@ def test_small_dag_vs_brute_force(k):
     RC.check_greedy_steps(rg, g.schedule(flags=0), RC.rank_by_paths(rg))
 
 
+@pytest.mark.parametrize("k", range(len(SMALL)))
+def test_small_dag_insert_vs_brute_force(k):
+    """INSERT (R1i): the schedule is valid (invariants), never beats the
+    optimum over all placements x orders, and every step is the brute-force
+    greedy choice (EST by exhaustive search over time, refcheck.est_insert)."""
+    d, rg = SMALL[k]
+    g = O.OracleGraph(d)
+    opt = RC.brute_force_opt(rg)
+    for flags in (O.F_POLICY_INSERT, O.F_POLICY_INSERT | O.F_CP_PIN):
+        r = g.schedule(flags=flags)
+        assert r["status"] == O.CAND_OK
+        assert opt <= r["makespan"]
+        RC.check_invariants(rg, r)
+    RC.check_greedy_steps(rg, g.schedule(flags=O.F_POLICY_INSERT), RC.rank_by_paths(rg), insert=True)
+
+
 @pytest.mark.parametrize("k", range(0, len(SMALL), 3))
 def test_small_dag_pinned_ranks(k):
     d, rg = SMALL[k]
@@ -239,6 +265,11 @@ def test_random_dag_invariants_and_greedy_replay(seed):
     r = g.schedule(flags=0)
     if r["status"] == O.CAND_OK:
         RC.check_greedy_steps(rg, r, g.rank()[: d.n_ops].tolist())
+    # INSERT policy (R1i): same checks, EST by brute force over time
+    r = g.schedule(flags=O.F_POLICY_INSERT)
+    if r["status"] == O.CAND_OK:
+        RC.check_invariants(rg, r)
+        RC.check_greedy_steps(rg, r, g.rank()[: d.n_ops].tolist(), insert=True)
     if d.n_devices > 1 and d.n_ops > 0:
         for _ in range(3):
             npin = int(rng.integers(1, min(4, d.n_ops) + 1))
