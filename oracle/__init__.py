@@ -26,10 +26,12 @@ KIND_BASE, KIND_PIN, KIND_SPLIT = 0, 1, 2
 DIM_BATCH, DIM_CHANNEL = 0, 1
 F_CP_PIN = 1
 F_POLICY_INSERT = 2
+F_MEM_LIVE = 64
+GEN_POW2, GEN_SUBSETS = 1, 2
 
 CAND_DTYPE = np.dtype(
     [("kind", "u1"), ("n_pins", "u1"), ("split_dim", "u1"), ("split_n", "u1"),
-     ("split_op", "<i4"), ("pin_op", "<i4", (4,)), ("pin_dev", "u1", (4,)), ("pad", "u1", (4,))]
+     ("split_op", "<i4"), ("pin_op", "<i4", (4,)), ("pin_dev", "u1", (4,)), ("dev_mask", "<u4")]
 )
 assert CAND_DTYPE.itemsize == 32
 
@@ -62,11 +64,11 @@ def lib():
         _lib.fastt_ref_num_edges.restype = i64
         _lib.fastt_ref_num_edges.argtypes = [P]
         _lib.fastt_ref_schedule.restype = i32
-        _lib.fastt_ref_schedule.argtypes = [P, i32, i32, P, P, i32, i32, i32, u32, P, P, P, P, P, P, P, P]
+        _lib.fastt_ref_schedule.argtypes = [P, i32, i32, P, P, i32, i32, i32, u32, u32, P, P, P, P, P, P, P, P]
         _lib.fastt_ref_split_export.restype = i64
         _lib.fastt_ref_split_export.argtypes = [P, i32, i32, i32, P, P, P, P, P, P, P, P, P]
         _lib.fastt_ref_rank.restype = i32
-        _lib.fastt_ref_rank.argtypes = [P, i32, i32, P, P, i32, i32, i32, P]
+        _lib.fastt_ref_rank.argtypes = [P, i32, i32, P, P, i32, i32, i32, u32, P]
         _lib.fastt_ref_split_search.restype = i32
         _lib.fastt_ref_split_search.argtypes = [P, u32, i32, i32, P, P, P, P, i32, P, P, P, P, P, P]
         _lib.fastt_ref_split_search_bi.restype = i32
@@ -146,15 +148,16 @@ class OracleGraph:
     @staticmethod
     def _cand_args(cand):
         if cand is None:
-            return KIND_BASE, 0, None, None, -1, 0, 0
+            return KIND_BASE, 0, None, None, -1, 0, 0, 0
         c = cand
         pin_op = np.ascontiguousarray(np.asarray(c["pin_op"], dtype=np.int32).reshape(4))
         pin_dev = np.ascontiguousarray(np.asarray(c["pin_dev"], dtype=np.uint8).reshape(4))
-        return int(c["kind"]), int(c["n_pins"]), pin_op, pin_dev, int(c["split_op"]), int(c["split_dim"]), int(c["split_n"])
+        return (int(c["kind"]), int(c["n_pins"]), pin_op, pin_dev, int(c["split_op"]), int(c["split_dim"]),
+                int(c["split_n"]), int(c["dev_mask"]))
 
     def schedule(self, cand=None, flags=0, outputs=True):
         """One candidate through DPOS.  Returns a dict."""
-        kind, npins, po, pd, so, sd, sn = self._cand_args(cand)
+        kind, npins, po, pd, so, sd, sn, dm = self._cand_args(cand)
         ms = np.zeros(1, np.int64)
         st = np.zeros(1, np.uint8)
         peak = np.zeros(self.G, np.int64)
@@ -164,7 +167,7 @@ class OracleGraph:
         start = np.zeros(vm, np.int64) if outputs else None
         rank = np.zeros(vm, np.int64) if outputs else None
         deq = np.zeros(vm, np.int32) if outputs else None
-        rc = lib().fastt_ref_schedule(self.h, kind, npins, _p(po), _p(pd), so, sd, sn, flags, _p(ms), _p(peak),
+        rc = lib().fastt_ref_schedule(self.h, kind, npins, _p(po), _p(pd), so, sd, sn, dm, flags, _p(ms), _p(peak),
                                       _p(st), _p(place), _p(order), _p(start), _p(rank), _p(deq))
         if rc != 0:
             raise OracleError(rc)
@@ -174,9 +177,9 @@ class OracleGraph:
         return out
 
     def rank(self, cand=None):
-        kind, npins, po, pd, so, sd, sn = self._cand_args(cand)
+        kind, npins, po, pd, so, sd, sn, dm = self._cand_args(cand)
         r = np.zeros(self.v_max, np.int64)
-        rc = lib().fastt_ref_rank(self.h, kind, npins, _p(po), _p(pd), so, sd, sn, _p(r))
+        rc = lib().fastt_ref_rank(self.h, kind, npins, _p(po), _p(pd), so, sd, sn, dm, _p(r))
         if rc != 0:
             raise OracleError(rc)
         return r
@@ -233,25 +236,31 @@ class OracleGraph:
                 "placement": place[:nf], "order": order[:nf], "start": start[:nf], "makespan": int(ms[0]),
                 "status": int(st[0])}
 
-    def stream_info(self, flags=0, pow2_only=False):
+    @staticmethod
+    def _gen_opts(pow2_only, subsets):
+        return (GEN_POW2 if pow2_only else 0) | (GEN_SUBSETS if subsets else 0)
+
+    def stream_info(self, flags=0, pow2_only=False, subsets=False):
         ns = np.zeros(1, np.int64)
         bp = np.zeros(max(self.V, 1), np.uint8)
-        lib().fastt_ref_stream_info(self.h, flags, int(bool(pow2_only)), _p(ns), _p(bp))
+        lib().fastt_ref_stream_info(self.h, flags, self._gen_opts(pow2_only, subsets), _p(ns), _p(bp))
         return int(ns[0]), bp[: self.V]
 
-    def generate(self, seed, first, n, kmin=1, kmax=4, flags=0, pow2_only=False):
+    def generate(self, seed, first, n, kmin=1, kmax=4, flags=0, pow2_only=False, subsets=False):
         out = np.zeros(n, CAND_DTYPE)
-        rc = lib().fastt_ref_generate(self.h, flags, seed, kmin, kmax, int(bool(pow2_only)), first, n, _p(out))
+        rc = lib().fastt_ref_generate(self.h, flags, seed, kmin, kmax, self._gen_opts(pow2_only, subsets), first, n,
+                                      _p(out))
         if rc != 0:
             raise OracleError(rc)
         return out
 
-    def sweep(self, seed, first, n, stride=1, kmin=1, kmax=4, flags=0, pow2_only=False, per_candidate=False):
+    def sweep(self, seed, first, n, stride=1, kmin=1, kmax=4, flags=0, pow2_only=False, per_candidate=False,
+              subsets=False):
         bm = np.zeros(1, np.int64)
         bi = np.zeros(1, np.int64)
         mss = np.zeros(n, np.int64) if per_candidate else None
-        rc = lib().fastt_ref_sweep(self.h, flags, seed, kmin, kmax, int(bool(pow2_only)), first, n, stride, _p(bm),
-                                   _p(bi), _p(mss))
+        rc = lib().fastt_ref_sweep(self.h, flags, seed, kmin, kmax, self._gen_opts(pow2_only, subsets), first, n,
+                                   stride, _p(bm), _p(bi), _p(mss))
         if rc != 0:
             raise OracleError(rc)
         res = {"makespan": int(bm[0]), "index": int(bi[0])}
@@ -260,8 +269,9 @@ class OracleGraph:
         return res
 
 
-def make_cand(kind=KIND_BASE, pins=(), split=None):
-    """Build one candidate record: pins = [(op, dev), ...]; split = (op, dim, n)."""
+def make_cand(kind=KIND_BASE, pins=(), split=None, dev_mask=0):
+    """Build one candidate record: pins = [(op, dev), ...]; split = (op, dim, n);
+    dev_mask = the candidate's device subset (R25, 0 = all devices)."""
     c = np.zeros(1, CAND_DTYPE)[0]
     c["kind"] = kind
     c["split_op"] = -1
@@ -272,4 +282,5 @@ def make_cand(kind=KIND_BASE, pins=(), split=None):
     c["n_pins"] = len(pins)
     if split is not None:
         c["split_op"], c["split_dim"], c["split_n"] = split
+    c["dev_mask"] = dev_mask
     return c

@@ -45,6 +45,7 @@
 
 #define FO_F_CP_PIN 1u
 #define FO_F_POLICY_INSERT 2u
+#define FO_F_MEM_LIVE 64u /* liveness-based memory (NEXT N3, R24) */
 
 #define FO_INF INT64_MAX
 #define FO_MAXG 32
@@ -402,22 +403,27 @@ static void fo_result_infeasible(fo_result *r, int32_t V, int32_t G, uint8_t sta
 
 /* w_i: "the maximal execution time of operation o_i (over different devices
  * that it could be assigned to run)", allowed set per R5. */
-static int64_t fo_w(const fo_graph *g, const int32_t *pin, int32_t i) {
+static int64_t fo_w(const fo_graph *g, const int32_t *pin, uint32_t dset, int32_t i) {
   if (pin && pin[i] >= 0) return g->cost[(int64_t)i * g->G + pin[i]];
   int64_t mx = 0;
-  for (int d = 0; d < g->G; d++) if (g->cost[(int64_t)i * g->G + d] > mx) mx = g->cost[(int64_t)i * g->G + d];
+  for (int d = 0; d < g->G; d++) {
+    if (!((dset >> d) & 1u)) continue; /* R25: only the candidate's devices */
+    if (g->cost[(int64_t)i * g->G + d] > mx) mx = g->cost[(int64_t)i * g->G + d];
+  }
   return mx;
 }
 
 /* c_ij: "the maximal transmission time of the tensor from o_i to o_j (over
  * different device pairs that they can be located on)", R5:
  * pairs with s != t only; 0 if there is no such pair. */
-static int64_t fo_c(const fo_graph *g, const int32_t *pin, int32_t i, int32_t j, int64_t bytes) {
+static int64_t fo_c(const fo_graph *g, const int32_t *pin, uint32_t dset, int32_t i, int32_t j, int64_t bytes) {
   int64_t mx = 0;
   for (int s = 0; s < g->G; s++) {
     if (pin && pin[i] >= 0 && s != pin[i]) continue;
+    if (!(pin && pin[i] >= 0) && !((dset >> s) & 1u)) continue;
     for (int t = 0; t < g->G; t++) {
       if (pin && pin[j] >= 0 && t != pin[j]) continue;
+      if (!(pin && pin[j] >= 0) && !((dset >> t) & 1u)) continue;
       if (s == t) continue;
       int64_t c = fo_comm(g, bytes, s, t);
       if (c > mx) mx = c;
@@ -428,7 +434,7 @@ static int64_t fo_c(const fo_graph *g, const int32_t *pin, int32_t i, int32_t j,
 
 /* rank_u(o_i) = w_i + max_{o_j in succ(o_i)} (c_ij + rank_u(o_j)),
  * rank_u(o_exit) = w_exit, evaluated in reverse topological order. */
-static void fo_rank(const fo_graph *g, const int32_t *pin, int64_t *rank) {
+static void fo_rank(const fo_graph *g, const int32_t *pin, uint32_t dset, int64_t *rank) {
   int32_t V = g->V;
   int32_t *topo = malloc(sizeof(int32_t) * ((size_t)V + 1));
   int32_t n = fo_topo(g, topo);
@@ -438,10 +444,10 @@ static void fo_rank(const fo_graph *g, const int32_t *pin, int64_t *rank) {
     int64_t best = 0;
     for (int32_t e = g->succ_off[i]; e < g->succ_off[i + 1]; e++) {
       int32_t j = g->succ_dst[e];
-      int64_t v = fo_c(g, pin, i, j, g->succ_bytes[e]) + rank[j];
+      int64_t v = fo_c(g, pin, dset, i, j, g->succ_bytes[e]) + rank[j];
       if (v > best) best = v;
     }
-    rank[i] = fo_w(g, pin, i) + best;
+    rank[i] = fo_w(g, pin, dset, i) + best;
   }
   free(topo);
 }
@@ -494,13 +500,19 @@ static int64_t fo_idle_slot(const int64_t *s, const int64_t *f, int32_t n, int64
   return a > r ? a : r;
 }
 
+/* The full device set D of P:322-323 as a bit mask. */
+static uint32_t fo_all_devices(int G) { return G >= 32 ? 0xFFFFFFFFu : ((1u << G) - 1u); }
+
 /* DPOS (Alg. 1) for one candidate: graph g (already split if the
- * candidate splits), perturbation pins pin[] (-1 = free), flags.
+ * candidate splits), perturbation pins pin[] (-1 = free), the candidate's
+ * device subset dset (R25: "FastT may not use all the input
+ * devices, and can choose a subset"; fo_all_devices = all), flags.
  * Ranks are written to rank[] (V entries). */
-static void fo_dpos(const fo_graph *g, const int32_t *pin, uint32_t flags, int64_t *rank, fo_result *r) {
+static void fo_dpos(const fo_graph *g, const int32_t *pin, uint32_t dset, uint32_t flags, int64_t *rank,
+                    fo_result *r) {
   int32_t V = g->V, G = g->G;
   /* Alg. 1 line 3-4: w, c and rank_u */
-  fo_rank(g, pin, rank);
+  fo_rank(g, pin, dset, rank);
   /* Alg. 1 lines 4-5: SET_CP and the critical-path devices d_cp (P:600-609,
    * P:678-682, R9) */
   int32_t *cpdev = malloc(sizeof(int32_t) * ((size_t)V + 1));
@@ -515,7 +527,7 @@ static void fo_dpos(const fo_graph *g, const int32_t *pin, uint32_t flags, int64
     for (int32_t q = 0; q < ncp; q++)
       if (!(pin && pin[cp[q]] >= 0)) fr[nf++] = cp[q];
     int devs[FO_MAXG];
-    for (int d = 0; d < G; d++) devs[d] = 1;
+    for (int d = 0; d < G; d++) devs[d] = (dset >> d) & 1u;
     int32_t k = 0;
     while (k < nf) {
       int any_dev = 0;
@@ -563,8 +575,15 @@ static void fo_dpos(const fo_graph *g, const int32_t *pin, uint32_t flags, int64
     bs = malloc(sizeof(int64_t) * ((size_t)V * G + 1));
     bf = malloc(sizeof(int64_t) * ((size_t)V * G + 1));
   }
+  /* liveness memory (NEXT N3, R24): an op's parameters stay on its device;
+   * its output activation (mem - param) is held from the step the op is
+   * dequeued until the step its last consumer is dequeued.  rem[i] counts
+   * the consumers of op i not dequeued yet. */
+  const int live = (flags & FO_F_MEM_LIVE) != 0;
+  int32_t *rem = malloc(sizeof(int32_t) * ((size_t)V + 1));
   for (int d = 0; d < G; d++) r->peak[d] = 0;
   for (int32_t i = 0; i < V; i++) {
+    rem[i] = g->succ_off[i + 1] - g->succ_off[i];
     indeg[i] = g->pred_off[i + 1] - g->pred_off[i];
     r->place[i] = 0xFF; r->start[i] = -1; r->finish[i] = -1; r->order[i] = -1; r->dq[i] = -1; r->deq[i] = -1;
     if (g->alive[i] && indeg[i] == 0) ready[nready++] = i;
@@ -612,6 +631,7 @@ static void fo_dpos(const fo_graph *g, const int32_t *pin, uint32_t flags, int64
       /* Alg. 1 lines 12-19: EFT = +inf if memory exceeds capacity; argmin EFT */
       int64_t best = FO_INF;
       for (int d = 0; d < G; d++) {
+        if (!((dset >> d) & 1u)) continue; /* R25: a device outside the candidate's subset */
         if (used[d] + reserved[d] + mi > g->cap[d]) continue;
         int64_t est;
         FO_EST(d, est);
@@ -643,6 +663,17 @@ static void fo_dpos(const fo_graph *g, const int32_t *pin, uint32_t flags, int64
       nb[dsel]++;
     }
     used[dsel] += mi;
+    if (live) {
+      /* peak = the largest live total seen at any step (R24) */
+      if (used[dsel] > r->peak[dsel]) r->peak[dsel] = used[dsel];
+      /* free each input whose last consumer this op is, then this op's own
+       * output if nothing consumes it */
+      for (int32_t e = g->pred_off[i]; e < g->pred_off[i + 1]; e++) {
+        int32_t m = g->pred_src[e];
+        if (--rem[m] == 0) used[r->place[m]] -= g->mem[m] - g->param[m];
+      }
+      if (rem[i] == 0) used[dsel] -= mi - g->param[i];
+    }
     r->dq[i] = seq;
     r->deq[seq] = i;
     seq++;
@@ -668,20 +699,26 @@ static void fo_dpos(const fo_graph *g, const int32_t *pin, uint32_t flags, int64
   /* Alg. 1 line 24 (R16): FT(o_exit) = max FT; peak memory per device (R8) */
   r->makespan = makespan;
   r->status = FO_CAND_OK;
-  for (int d = 0; d < G; d++) r->peak[d] = used[d];
+  if (!live)
+    for (int d = 0; d < G; d++) r->peak[d] = used[d];
 done:
-  free(cpdev); free(indeg); free(ready);
+  free(cpdev); free(indeg); free(ready); free(rem);
   free(bs); free(bf);
 }
 
 /* ----------------------------------------------------- candidate handling */
 
-/* Validate a candidate and produce (graph to schedule, pin array).
+/* Validate a candidate and produce (graph to schedule, pin array, device
+ * set).  dev_mask = 0 means every device; otherwise it must be a subset of
+ * the G devices and hold every pinned device (R25).
  * Returns FO_CAND_OK or FO_CAND_BADSPEC. *gs is g itself or a new split view. */
 static int fo_prepare(const fo_graph *g, int kind, int npins, const int32_t *pin_op, const uint8_t *pin_dev,
-                      int32_t split_op, int split_dim, int split_n, fo_graph **gs, int32_t **pin_out) {
+                      int32_t split_op, int split_dim, int split_n, uint32_t dev_mask, fo_graph **gs,
+                      int32_t **pin_out, uint32_t *dset) {
   *gs = (fo_graph *)g;
   *pin_out = NULL;
+  *dset = dev_mask ? dev_mask : fo_all_devices(g->G);
+  if (dev_mask & ~fo_all_devices(g->G)) return FO_CAND_BADSPEC;
   if (kind == FO_KIND_BASE) return FO_CAND_OK;
   if (kind == FO_KIND_PIN) {
     if (npins < 1 || npins > FO_MAXPINS) return FO_CAND_BADSPEC;
@@ -689,7 +726,10 @@ static int fo_prepare(const fo_graph *g, int kind, int npins, const int32_t *pin
     for (int32_t i = 0; i < g->V; i++) pin[i] = -1;
     for (int q = 0; q < npins; q++) {
       int32_t o = pin_op[q];
-      if (o < 0 || o >= g->V || !g->alive[o] || pin_dev[q] >= g->G || pin[o] >= 0) { free(pin); return FO_CAND_BADSPEC; }
+      if (o < 0 || o >= g->V || !g->alive[o] || pin_dev[q] >= g->G || pin[o] >= 0 || !((*dset >> pin_dev[q]) & 1u)) {
+        free(pin);
+        return FO_CAND_BADSPEC;
+      }
       pin[o] = pin_dev[q];
     }
     *pin_out = pin;
@@ -720,13 +760,14 @@ int32_t fastt_ref_v_max(const fo_graph *g) {
  * candidate's graph are 0xFF / -1).  Any output pointer may be NULL. */
 int32_t fastt_ref_schedule(const fo_graph *g, int32_t kind, int32_t npins, const int32_t *pin_op,
                            const uint8_t *pin_dev, int32_t split_op, int32_t split_dim, int32_t split_n,
-                           uint32_t flags, int64_t *makespan, int64_t *peak, uint8_t *status,
+                           uint32_t dev_mask, uint32_t flags, int64_t *makespan, int64_t *peak, uint8_t *status,
                            uint8_t *placement, int32_t *order, int64_t *start, int64_t *rank_out,
                            int32_t *deq_out) {
   int32_t vmax = fastt_ref_v_max(g), G = g->G;
   fo_graph *gs;
   int32_t *pin;
-  int st = fo_prepare(g, kind, npins, pin_op, pin_dev, split_op, split_dim, split_n, &gs, &pin);
+  uint32_t dset;
+  int st = fo_prepare(g, kind, npins, pin_op, pin_dev, split_op, split_dim, split_n, dev_mask, &gs, &pin, &dset);
   if (placement) memset(placement, 0xFF, (size_t)vmax);
   for (int32_t i = 0; i < vmax; i++) {
     if (order) order[i] = -1;
@@ -743,7 +784,7 @@ int32_t fastt_ref_schedule(const fo_graph *g, int32_t kind, int32_t npins, const
   fo_result r;
   fo_result_alloc(&r, gs->V, G);
   int64_t *rank = malloc(sizeof(int64_t) * ((size_t)gs->V + 1));
-  fo_dpos(gs, pin, flags, rank, &r);
+  fo_dpos(gs, pin, dset, flags, rank, &r);
   *makespan = r.makespan;
   *status = r.status;
   if (peak) for (int d = 0; d < G; d++) peak[d] = r.peak[d];
@@ -827,7 +868,7 @@ int32_t fastt_ref_split_search(const fo_graph *g0, uint32_t flags, int32_t pow2_
   fo_result_alloc(&best_r, g0->V, G);
   int64_t *rank = malloc(sizeof(int64_t) * ((size_t)g0->V + 1));
   /* Alg. 2 line 3 */
-  fo_dpos(cur, NULL, flags, rank, &best_r);
+  fo_dpos(cur, NULL, fo_all_devices(cur->G), flags, rank, &best_r);
   free(rank);
   *sp_n = 0;
   if (best_r.status != FO_CAND_OK) {
@@ -857,7 +898,7 @@ int32_t fastt_ref_split_search(const fo_graph *g0, uint32_t flags, int32_t pow2_
         fo_result r;
         fo_result_alloc(&r, sv->V, G);
         int64_t *rk = malloc(sizeof(int64_t) * ((size_t)sv->V + 1));
-        fo_dpos(sv, NULL, flags, rk, &r);
+        fo_dpos(sv, NULL, fo_all_devices(sv->G), flags, rk, &r);
         free(rk);
         if (r.status == FO_CAND_OK && r.makespan < bft) {
           if (bg) { fo_graph_free(bg); fo_result_free(&br); }
@@ -911,7 +952,7 @@ int32_t fastt_ref_split_search_bi(const fo_graph *g0, uint32_t flags, int32_t po
   fo_result best_r;
   fo_result_alloc(&best_r, g0->V, G);
   int64_t *rank = malloc(sizeof(int64_t) * ((size_t)g0->V + 1));
-  fo_dpos(cur, NULL, flags, rank, &best_r);
+  fo_dpos(cur, NULL, fo_all_devices(cur->G), flags, rank, &best_r);
   free(rank);
   *sp_n = 0;
   if (best_r.status != FO_CAND_OK) {
@@ -943,7 +984,7 @@ int32_t fastt_ref_split_search_bi(const fo_graph *g0, uint32_t flags, int32_t po
           fo_result r;
           fo_result_alloc(&r, sv->V, G);
           int64_t *rk = malloc(sizeof(int64_t) * ((size_t)sv->V + 1));
-          fo_dpos(sv, NULL, flags, rk, &r);
+          fo_dpos(sv, NULL, fo_all_devices(sv->G), flags, rk, &r);
           free(rk);
           if (r.status == FO_CAND_OK && r.makespan < bft) {
             if (bg) { fo_graph_free(bg); fo_result_free(&br); }
@@ -991,7 +1032,7 @@ typedef struct {
   int32_t split_op;
   int32_t pin_op[4];
   uint8_t pin_dev[4];
-  uint8_t pad[4];
+  uint32_t dev_mask; /* R25: device subset, 0 = all */
 } fo_cand; /* 32 bytes */
 
 static uint64_t fo_splitmix64(uint64_t *s) {
@@ -1012,18 +1053,24 @@ typedef struct {
   int64_t n_split;
   int32_t *live;
   int32_t n_live;
+  int64_t n_subset; /* G-1 prefix-subset candidates when enabled (R25), else 0 */
 } fo_stream;
 
 static void fo_stream_free(fo_stream *s) { free(s->base_place); free(s->split_op); free(s->split_dim); free(s->split_n); free(s->live); }
 
+/* gen_opts bits of the stream calls */
+#define FO_GEN_POW2 1    /* split counts {2,4,8,..} only (R14) */
+#define FO_GEN_SUBSETS 2 /* a block of device-subset candidates after the SPLITs (R25) */
+
 /* One DPOS run on the base graph gives the base placement and, through
  * Alg. 2 lines 4-5, the ordered split-eligible CP ops (R21). */
-static void fo_stream_init(const fo_graph *g, uint32_t flags, int pow2_only, fo_stream *s) {
+static void fo_stream_init(const fo_graph *g, uint32_t flags, int gen_opts, fo_stream *s) {
+  int pow2_only = gen_opts & FO_GEN_POW2;
   int32_t V = g->V, G = g->G;
   fo_result r;
   fo_result_alloc(&r, V, G);
   int64_t *rank = malloc(sizeof(int64_t) * ((size_t)V + 1));
-  fo_dpos(g, NULL, flags, rank, &r);
+  fo_dpos(g, NULL, fo_all_devices(g->G), flags, rank, &r);
   free(rank);
   s->base_place = malloc((size_t)V + 1);
   for (int32_t i = 0; i < V; i++) s->base_place[i] = r.status == FO_CAND_OK ? r.place[i] : 0;
@@ -1048,6 +1095,7 @@ static void fo_stream_init(const fo_graph *g, uint32_t flags, int pow2_only, fo_
   s->live = malloc(sizeof(int32_t) * ((size_t)V + 1));
   s->n_live = 0;
   for (int32_t i = 0; i < V; i++) if (g->alive[i]) s->live[s->n_live++] = i;
+  s->n_subset = (gen_opts & FO_GEN_SUBSETS) ? G - 1 : 0;
   free(list);
   fo_result_free(&r);
 }
@@ -1063,6 +1111,13 @@ static void fo_stream_cand(const fo_graph *g, const fo_stream *s, uint64_t seed,
     out->split_op = s->split_op[c - 1];
     out->split_dim = s->split_dim[c - 1];
     out->split_n = s->split_n[c - 1];
+    return;
+  }
+  if (c <= s->n_split + s->n_subset) {
+    /* R25: BASE on the first k devices, k = 1 .. G-1 */
+    int k = (int)(c - s->n_split);
+    out->kind = FO_KIND_BASE;
+    out->dev_mask = (1u << k) - 1u;
     return;
   }
   out->kind = FO_KIND_PIN;
@@ -1090,14 +1145,14 @@ static void fo_stream_cand(const fo_graph *g, const fo_stream *s, uint64_t seed,
 static int fo_stream_check(const fo_graph *g, const fo_stream *s, int kmin, int kmax, int64_t first, int64_t n,
                            int64_t stride) {
   if (kmin < 1 || kmax > 4 || kmin > kmax || first < 0 || n < 0 || stride < 1) return FO_EINVAL;
-  if (n > 0 && (g->G == 1 || s->n_live == 0) && first + (n - 1) * stride > s->n_split) return FO_EINVAL;
+  if (n > 0 && (g->G == 1 || s->n_live == 0) && first + (n - 1) * stride > s->n_split + s->n_subset) return FO_EINVAL;
   return FO_OK;
 }
 
-int32_t fastt_ref_stream_info(const fo_graph *g, uint32_t flags, int32_t pow2_only, int64_t *n_split,
+int32_t fastt_ref_stream_info(const fo_graph *g, uint32_t flags, int32_t gen_opts, int64_t *n_split,
                               uint8_t *base_place) {
   fo_stream s;
-  fo_stream_init(g, flags, pow2_only, &s);
+  fo_stream_init(g, flags, gen_opts, &s);
   *n_split = s.n_split;
   if (base_place) memcpy(base_place, s.base_place, (size_t)g->V);
   fo_stream_free(&s);
@@ -1105,9 +1160,9 @@ int32_t fastt_ref_stream_info(const fo_graph *g, uint32_t flags, int32_t pow2_on
 }
 
 int32_t fastt_ref_generate(const fo_graph *g, uint32_t flags, uint64_t seed, int32_t kmin, int32_t kmax,
-                           int32_t pow2_only, int64_t first, int64_t n, void *out) {
+                           int32_t gen_opts, int64_t first, int64_t n, void *out) {
   fo_stream s;
-  fo_stream_init(g, flags, pow2_only, &s);
+  fo_stream_init(g, flags, gen_opts, &s);
   int rc = fo_stream_check(g, &s, kmin, kmax, first, n, 1);
   if (rc == FO_OK)
     for (int64_t q = 0; q < n; q++) fo_stream_cand(g, &s, seed, kmin, kmax, first + q, (fo_cand *)out + q);
@@ -1118,10 +1173,10 @@ int32_t fastt_ref_generate(const fo_graph *g, uint32_t flags, uint64_t seed, int
 /* Sweep: evaluate candidates c = first + q*stride (q < n); best = smallest
  * makespan, then smallest index (R3).  Per-candidate makespans optional. */
 int32_t fastt_ref_sweep(const fo_graph *g, uint32_t flags, uint64_t seed, int32_t kmin, int32_t kmax,
-                        int32_t pow2_only, int64_t first, int64_t n, int64_t stride, int64_t *best_makespan,
+                        int32_t gen_opts, int64_t first, int64_t n, int64_t stride, int64_t *best_makespan,
                         int64_t *best_index, int64_t *makespans) {
   fo_stream s;
-  fo_stream_init(g, flags, pow2_only, &s);
+  fo_stream_init(g, flags, gen_opts, &s);
   int rc = fo_stream_check(g, &s, kmin, kmax, first, n, stride);
   *best_makespan = FO_INF;
   *best_index = -1;
@@ -1133,7 +1188,7 @@ int32_t fastt_ref_sweep(const fo_graph *g, uint32_t flags, uint64_t seed, int32_
       int64_t ms;
       uint8_t stt;
       fastt_ref_schedule(g, cd.kind, cd.n_pins, cd.pin_op, cd.pin_dev, cd.split_op, cd.split_dim, cd.split_n,
-                         flags, &ms, NULL, &stt, NULL, NULL, NULL, NULL, NULL);
+                         cd.dev_mask, flags, &ms, NULL, &stt, NULL, NULL, NULL, NULL, NULL);
       if (makespans) makespans[q] = ms;
       if (ms < *best_makespan || (ms == *best_makespan && ms != FO_INF && c < *best_index)) {
         *best_makespan = ms;
@@ -1147,15 +1202,17 @@ int32_t fastt_ref_sweep(const fo_graph *g, uint32_t flags, uint64_t seed, int32_
 
 /* Upward ranks of a candidate's graph (base when kind == BASE). */
 int32_t fastt_ref_rank(const fo_graph *g, int32_t kind, int32_t npins, const int32_t *pin_op, const uint8_t *pin_dev,
-                       int32_t split_op, int32_t split_dim, int32_t split_n, int64_t *rank_out) {
+                       int32_t split_op, int32_t split_dim, int32_t split_n, uint32_t dev_mask, int64_t *rank_out) {
   int32_t vmax = fastt_ref_v_max(g);
   fo_graph *gs;
   int32_t *pin;
+  uint32_t dset;
   for (int32_t i = 0; i < vmax; i++) rank_out[i] = -1;
-  if (fo_prepare(g, kind, npins, pin_op, pin_dev, split_op, split_dim, split_n, &gs, &pin) != FO_CAND_OK)
+  if (fo_prepare(g, kind, npins, pin_op, pin_dev, split_op, split_dim, split_n, dev_mask, &gs, &pin, &dset) !=
+      FO_CAND_OK)
     return FO_EINVAL;
   int64_t *rank = malloc(sizeof(int64_t) * ((size_t)gs->V + 1));
-  fo_rank(gs, pin, rank);
+  fo_rank(gs, pin, dset, rank);
   for (int32_t i = 0; i < gs->V; i++) rank_out[i] = gs->alive[i] ? rank[i] : -1;
   free(rank);
   free(pin);
@@ -1167,7 +1224,7 @@ int32_t fastt_ref_rank(const fo_graph *g, int32_t kind, int32_t npins, const int
 int32_t fastt_ref_cp(const fo_graph *g, int32_t *cp_out) {
   int64_t *rank = malloc(sizeof(int64_t) * ((size_t)g->V + 1));
   int32_t *cp = malloc(sizeof(int32_t) * ((size_t)g->V + 1));
-  fo_rank(g, NULL, rank);
+  fo_rank(g, NULL, fo_all_devices(g->G), rank);
   int32_t n = fo_critical_path(g, rank, cp);
   if (cp_out) memcpy(cp_out, cp, sizeof(int32_t) * (size_t)n);
   free(rank); free(cp);
@@ -1183,7 +1240,8 @@ int64_t fastt_ref_split_export(const fo_graph *g, int32_t op, int32_t dim, int32
   fo_graph *gs;
   int32_t *pin;
   uint8_t dummy = 0;
-  if (fo_prepare(g, FO_KIND_SPLIT, 0, NULL, &dummy, op, dim, n, &gs, &pin) != FO_CAND_OK) return FO_EINVAL;
+  uint32_t dset;
+  if (fo_prepare(g, FO_KIND_SPLIT, 0, NULL, &dummy, op, dim, n, 0, &gs, &pin, &dset) != FO_CAND_OK) return FO_EINVAL;
   *V_out = gs->V;
   for (int32_t i = 0; i < gs->V; i++) {
     for (int d = 0; d < gs->G; d++) cost[(int64_t)i * gs->G + d] = gs->cost[(int64_t)i * gs->G + d];

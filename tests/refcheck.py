@@ -8,7 +8,9 @@ the paper's definitions as brute force / verification routines.
   * brute force over all placements x all topological orders,
   * schedule invariants,
   * a greedy-step replay checker, APPEND or INSERT (R1i, EST by
-    brute force over time).
+    brute force over time), static or liveness memory (R24), device subsets
+    (R25),
+  * liveness peaks by their definition (R24).
 """
 from __future__ import annotations
 
@@ -37,6 +39,7 @@ class G:
             l.sort()
         self.cost = desc.cost.tolist()
         self.mem = desc.mem.tolist()
+        self.param = desc.param.tolist()
         self.cap = desc.cap.tolist()
         self.lc = desc.link_class.tolist()
         self.alpha = desc.alpha.tolist()
@@ -48,37 +51,42 @@ class G:
         k = self.lc[s][t]
         return self.alpha[k] + -(-(b * self.beta[k]) // 1_000_000)
 
-    def w(self, i, pin=None):
+    def w(self, i, pin=None, dset=None):
         if pin and i in pin:
             return self.cost[i][pin[i]]
-        return max(self.cost[i])
+        return max(self.cost[i][d] for d in range(self.G) if dset is None or d in dset)
 
-    def c(self, i, j, b, pin=None):
+    def c(self, i, j, b, pin=None, dset=None):
         best = 0
         for s in range(self.G):
             if pin and i in pin and s != pin[i]:
                 continue
+            if not (pin and i in pin) and dset is not None and s not in dset:
+                continue
             for t in range(self.G):
                 if pin and j in pin and t != pin[j]:
+                    continue
+                if not (pin and j in pin) and dset is not None and t not in dset:
                     continue
                 if s != t:
                     best = max(best, self.comm(b, s, t))
         return best
 
 
-def rank_by_paths(g: G, pin=None):
+def rank_by_paths(g: G, pin=None, dset=None):
     """rank_u(i) = max over all paths i -> sink of sum(w) + sum(c), by explicit
-    enumeration of paths (exponential; small graphs only)."""
+    enumeration of paths (exponential; small graphs only).  dset: the
+    candidate's device subset (R25) as the allowed set of unpinned ops."""
     out = []
     for i in range(g.V):
         best = -1
-        stack = [(i, g.w(i, pin))]
+        stack = [(i, g.w(i, pin, dset))]
         while stack:
             u, acc = stack.pop()
             if not g.succ[u]:
                 best = max(best, acc)
             for (v, b) in g.succ[u]:
-                stack.append((v, acc + g.c(u, v, b, pin) + g.w(v, pin)))
+                stack.append((v, acc + g.c(u, v, b, pin, dset) + g.w(v, pin, dset)))
         out.append(best)
     return out
 
@@ -123,9 +131,10 @@ def topo_orders(g: G, limit=None):
     return res
 
 
-def brute_force_opt(g: G, zero_comm=False):
+def brute_force_opt(g: G, zero_comm=False, dset=None):
     """Optimum of the APPEND schedule space: all placements x all
-    topological orders (every left-shifted schedule is one of these)."""
+    topological orders (every left-shifted schedule is one of these);
+    dset restricts the placements to a device subset (R25)."""
     orders = topo_orders(g)
     best = INF
     saved = (g.alpha, g.beta)
@@ -133,7 +142,7 @@ def brute_force_opt(g: G, zero_comm=False):
         g.alpha = [0] * len(g.alpha)
         g.beta = [0] * len(g.beta)
     try:
-        for place in itertools.product(range(g.G), repeat=g.V):
+        for place in itertools.product([d for d in range(g.G) if dset is None or d in dset], repeat=g.V):
             for o in orders:
                 best = min(best, evaluate(g, place, o)[2])
     finally:
@@ -220,15 +229,57 @@ def est_insert(ops, r, w):
     raise AssertionError("unreachable: the open-ended slot always fits")
 
 
-def check_greedy_steps(g: G, res, rank, cp_dev=None, insert=False):
+def live_usage(g: G, done, place, d):
+    """Liveness memory (R24) by its definition, before the next step: the
+    parameters of every op already dequeued on d, plus the output
+    (mem - param) of every such op that still has a consumer not dequeued."""
+    tot = 0
+    for j in done:
+        if place[j] != d:
+            continue
+        tot += g.param[j]
+        if any(c not in done for (c, _) in g.succ[j]):
+            tot += g.mem[j] - g.param[j]
+    return tot
+
+
+def live_peaks(g: G, res):
+    """R24 peak per device by definition: the largest, over the steps t of the
+    dequeue sequence, of the memory held on the device while step t's op is
+    placed: parameters of every op dequeued at or before t, outputs of ops
+    dequeued at or before t whose last consumer is dequeued at t or later,
+    and the output of step t's op itself."""
+    V = g.V
+    deq = [x for x in res["dequeue"][:V].tolist() if x >= 0]
+    place = res["placement"][:V].tolist()
+    dq = {op: t for t, op in enumerate(deq)}
+    peak = [0] * g.G
+    for t, i in enumerate(deq):
+        d = place[i]
+        tot = 0
+        for j in deq[: t + 1]:
+            if place[j] != d:
+                continue
+            tot += g.param[j]
+            last = max([dq[c] for (c, _) in g.succ[j]] or [dq[j]])
+            if j == i or last >= t:
+                tot += g.mem[j] - g.param[j]
+        peak[d] = max(peak[d], tot)
+    return peak
+
+
+def check_greedy_steps(g: G, res, rank, cp_dev=None, insert=False, live=False, dset=None):
     """every dequeued op is the max-(rank, -id) ready op and every
     free op sits on a device of minimum EFT (ties: lowest id) among the
     memory-feasible ones, given the partial schedule.  insert=True: EST by
-    est_insert (busy intervals of the ops placed so far) instead of APPEND."""
+    est_insert (busy intervals of the ops placed so far) instead of APPEND.
+    live=True: memory feasibility with the liveness usage of R24 (by
+    definition, live_usage).  dset: the candidate's device subset (R25)."""
     V = g.V
     deq = [x for x in res["dequeue"][:V].tolist() if x >= 0]
     place = res["placement"][:V].tolist()
     start = res["start"][:V].tolist()
+    devs = [d for d in range(g.G) if dset is None or d in dset]
     done = set()
     avail = [0] * g.G
     used = [0] * g.G
@@ -253,8 +304,9 @@ def check_greedy_steps(g: G, res, rank, cp_dev=None, insert=False):
             est = est_on(i, d)
         else:
             effs = []
-            for d in range(g.G):
-                if used[d] + reserved[d] + g.mem[i] > g.cap[d]:
+            for d in devs:
+                u = live_usage(g, done, place, d) if live else used[d]
+                if u + reserved[d] + g.mem[i] > g.cap[d]:
                     continue
                 est = est_on(i, d)
                 effs.append((est + g.cost[i][d], d, est))
