@@ -77,7 +77,11 @@ enum {
   FASTT_F_OUT_DEVICE = 1u << 2,    /* output pointers are device pointers */
   FASTT_F_IN_DEVICE = 1u << 3,     /* candidate input pointer is a device pointer */
   FASTT_F_TIMING = 1u << 4,        /* record CUDA events around the kernels of this call (fastt_last_timing) */
-  FASTT_F_SPLIT_BEST = 1u << 5     /* fastt_split_search: best-improvement rounds */
+  FASTT_F_SPLIT_BEST = 1u << 5,    /* fastt_split_search: best-improvement rounds */
+  FASTT_F_MEM_LIVE = 1u << 6       /* liveness memory (reading R24): an op's parameters stay on
+                                      its device; its output (mem - param) is held from the step it is dequeued
+                                      until the step its last consumer is dequeued.  The feasibility test of
+                                      Alg. 1 line 13 uses that live total; peak_mem = its maximum */
 };
 
 /* The problem input of P:321-328.  Edges are a CSR by source: the edges of
@@ -108,13 +112,20 @@ typedef struct {
  *          (a "placement perturbation"); pinned ops use w = cost on that
  *          device and c over the allowed device pairs (R5).
  *   SPLIT: SplitOperation(graph, split_op, split_dim, split_n), 2 <= n <= G,
- *          split_op must have split_mask bit split_dim (R13, R14). */
+ *          split_op must have split_mask bit split_dim (R13, R14).
+ *   dev_mask (any kind, reading R25): "FastT may not use all
+ *          the input devices, and can choose a subset".  0 = all
+ *          G devices; otherwise bit d set = device d may be used.  The
+ *          unpinned ops' allowed set (w, c of R5), the CP devices (R9) and
+ *          the EFT argmin (Alg. 1 line 12) range over the subset; every
+ *          pin_dev must be in it and no bit >= G may be set (else BADSPEC).
+ *          Devices outside the subset report peak_mem 0. */
 typedef struct {
   uint8_t kind, n_pins, split_dim, split_n;
   int32_t split_op;
   int32_t pin_op[4];
   uint8_t pin_dev[4];
-  uint8_t _pad[4];
+  uint32_t dev_mask;
 } fastt_candidate;
 
 /* The seeded candidate stream of a sweep (R21):
@@ -127,12 +138,17 @@ typedef struct {
  *   probing past ops already chosen) and device (base_place + 1 +
  *   x_{2+2k} mod (G-1)) mod G.  base_place comes from one DPOS run of the
  *   BASE candidate under the same flags (0 for every op if that run is
- *   infeasible).  With G == 1 the stream ends after the SPLIT block. */
+ *   infeasible).  With subset_prefixes = 1 a block of G-1 device-subset
+ *   candidates follows the SPLIT block (R25): index n_split + k, k = 1..G-1,
+ *   is BASE with dev_mask = (1 << k) - 1 (the first k devices); the PIN
+ *   block then starts at n_split + G.  With G == 1 the stream ends after
+ *   the SPLIT (and subset) block. */
 typedef struct {
   uint64_t seed;
   uint8_t pin_k_min, pin_k_max; /* 1 <= min <= max <= 4 */
   uint8_t n_pow2_only;          /* split counts {2,4,8,..} only (C4) */
-  uint8_t _pad[5];
+  uint8_t subset_prefixes;      /* 0/1: include the device-subset block (R25) */
+  uint8_t _pad[4];
 } fastt_gen_params;
 
 typedef struct {
@@ -166,7 +182,7 @@ fastt_status fastt_rank(const fastt_graph *g, const fastt_candidate *cand, const
 
 /* DPOS of n candidates (S2-S7).  makespan[n] (INT64_MAX if not OK),
  * status[n]; optional (NULL to skip): peak_mem[n*G] (sum of mem per device,
- * -1 if not OK), placement[n*v_max] (device per op id), order[n*v_max]
+ * -1 if not OK; with FASTT_F_MEM_LIVE the live peak of R24), placement[n*v_max] (device per op id), order[n*v_max]
  * (op ids sorted by (start, dequeue sequence), R17, -1 padded),
  * start_ns[n*v_max]. */
 fastt_status fastt_schedule_batch(const fastt_graph *g, const fastt_candidate *cands, int64_t n,

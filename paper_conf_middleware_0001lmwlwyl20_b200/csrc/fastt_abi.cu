@@ -106,7 +106,7 @@ static RawGraph raw_struct(char *b, const RawLayout &L, int32_t V, int32_t nl, i
 
 struct PrepLayout {
   int64_t ncap = 0, ecap = 0;
-  size_t o[19] = {0};
+  size_t o[20] = {0};
   size_t total = 0;
 };
 
@@ -114,7 +114,7 @@ static PrepLayout prep_layout(int64_t ncap, int64_t ecap, int G, int K, int tbyt
   PrepLayout L;
   L.ncap = ncap;
   L.ecap = ecap;
-  size_t sz[19] = {(size_t)ncap * CARD_WORDS * 4,        // card
+  size_t sz[20] = {(size_t)ncap * CARD_WORDS * 4,        // card
                    (size_t)ncap * G * tbytes,           // costp
                    (size_t)ecap * 4,                    // pe_src
                    (size_t)(ecap + 64) * K * tbytes,    // pe_comm (+ padding for speculative reads)
@@ -129,9 +129,10 @@ static PrepLayout prep_layout(int64_t ncap, int64_t ecap, int G, int K, int tbyt
                    (size_t)(ncap + 1) * G * 8,          // pcost
                    (size_t)ncap * 8, (size_t)ncap * 8,  // keys
                    (size_t)ncap * 4, (size_t)ncap * 4,  // vals
-                   33 * 4};                             // srcsumm
+                   33 * 4,                              // srcsumm
+                   (size_t)ncap * 8};                   // act
   size_t off = 0;
-  for (int k = 0; k < 19; k++) {
+  for (int k = 0; k < 20; k++) {
     L.o[k] = off;
     off += al16(sz[k]);
   }
@@ -162,6 +163,7 @@ static PrepGraph prep_struct(char *b, const PrepLayout &L, int tbits) {
   P.val0 = (uint32_t *)(b + L.o[16]);
   P.val1 = (uint32_t *)(b + L.o[17]);
   P.srcsumm = (uint32_t *)(b + L.o[18]);
+  P.act = (int64_t *)(b + L.o[19]);
   return P;
 }
 
@@ -233,7 +235,7 @@ struct fastt_graph {
   uint8_t *split_mask_dev = nullptr;
   Base base;
   std::vector<uint8_t> split_mask_h;
-  StreamCache streams[8];
+  StreamCache streams[16];
   // arena (per base layout)
   size_t arena_raw_total = 0, arena_prep_total = 0;
   int arena_slots = 0;
@@ -499,6 +501,11 @@ static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
   for (int d = 0; d < g->G; d++)
     if (g->gch.cap[d] != I64MAX) a.cap_check = 1;
   a.need_mem = a.cap_check;
+  a.fastcomm = B.tbits == 32 && g->K == 1;
+  if (flags & FASTT_F_MEM_LIVE) {
+    a.live_mem = 1;
+    a.need_mem = 1;
+  }
   if (flags & FASTT_F_POLICY_INSERT) {
     a.ins = 1;
     a.gap = g->gap;
@@ -631,7 +638,8 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
                                cudaStream_t st, DevOut o) {
   if (n <= 0) return FASTT_OK;
   TRY(ensure_sim(g, B, n, flags));
-  const bool sharing = g->share && !o.peak && !o.place && n >= 64 && !(flags & FASTT_F_POLICY_INSERT);
+  const bool sharing =
+      g->share && !o.peak && !o.place && n >= 64 && !(flags & (FASTT_F_POLICY_INSERT | FASTT_F_MEM_LIVE));
   if (sharing) TRY(ensure_snapshot(g, B, flags, st));  // before the work counters are reset
   if (o.place) CK(cudaMemsetAsync(o.place, 0xFF, (size_t)n * o.vmax, st));
   if (o.start) {
@@ -761,7 +769,8 @@ static fastt_status split_list(fastt_graph *g, Base &B, const uint8_t *d_place, 
 }
 
 static fastt_status ensure_stream(fastt_graph *g, uint32_t flags, int pow2, cudaStream_t st, StreamCache **out) {
-  int key = (int)(flags & FASTT_F_CP_PIN) | (pow2 ? 2 : 0) | (flags & FASTT_F_POLICY_INSERT ? 4 : 0);
+  int key = (int)(flags & FASTT_F_CP_PIN) | (pow2 ? 2 : 0) | (flags & FASTT_F_POLICY_INSERT ? 4 : 0) |
+            (flags & FASTT_F_MEM_LIVE ? 8 : 0);
   StreamCache &S = g->streams[key];
   *out = &S;
   if (S.valid) return FASTT_OK;
@@ -841,6 +850,7 @@ static StreamState stream_state(const fastt_graph *g, const StreamCache &S, cons
   s.kmin = gp->pin_k_min;
   s.kmax = gp->pin_k_max;
   s.G = g->G;
+  s.n_subset = gp->subset_prefixes ? g->G - 1 : 0;
   return s;
 }
 
@@ -850,7 +860,9 @@ static fastt_status check_gen(const fastt_graph *g, const StreamCache &S, const 
   if (gp->pin_k_min < 1 || gp->pin_k_max > 4 || gp->pin_k_min > gp->pin_k_max)
     return fail(FASTT_EINVAL, "need 1 <= pin_k_min <= pin_k_max <= 4");
   if (first < 0 || n < 0 || stride < 1) return fail(FASTT_EINVAL, "need first >= 0, n >= 0, stride >= 1");
-  if (n > 0 && (g->G == 1 || S.n_live == 0) && first + (n - 1) * stride > S.n_split)
+  if (gp->subset_prefixes > 1) return fail(FASTT_EINVAL, "subset_prefixes must be 0 or 1");
+  if (n > 0 && (g->G == 1 || S.n_live == 0) &&
+      first + (n - 1) * stride > S.n_split + (gp->subset_prefixes ? g->G - 1 : 0))
     return fail(FASTT_EINVAL, "the stream has no PIN candidates (G == 1 or no ops)");
   return FASTT_OK;
 }
@@ -1163,7 +1175,10 @@ fastt_status fastt_rank(const fastt_graph *gc_, const fastt_candidate *cand, con
   Base &B = g->base;
   const int64_t vm = g->v_max;
   std::vector<uint64_t> r(B.rl.vcap, ~0ull);
-  if (!cand || cand->kind == FASTT_KIND_BASE) {
+  const uint32_t all = all_devices(g->G);
+  if (cand && (cand->dev_mask & ~all)) return fail(FASTT_EINVAL, "dev_mask names a device >= G");
+  const uint32_t dset = cand && cand->dev_mask ? cand->dev_mask : all;
+  if (!cand || (cand->kind == FASTT_KIND_BASE && dset == all)) {
     if (B.V) CK(cudaMemcpy(r.data(), prep_struct(B.prep_block, B.pl, B.tbits).rank, 8 * (size_t)B.V,
                            cudaMemcpyDeviceToHost));
   } else {
@@ -1173,14 +1188,15 @@ fastt_status fastt_rank(const fastt_graph *gc_, const fastt_candidate *cand, con
     if (c.kind == FASTT_KIND_PIN) {
       if (c.n_pins < 1 || c.n_pins > 4) bad = true;
       for (int k = 0; k < c.n_pins && !bad; k++) {
-        if (c.pin_op[k] < 0 || c.pin_op[k] >= B.V || c.pin_dev[k] >= g->G) bad = true;
+        if (c.pin_op[k] < 0 || c.pin_op[k] >= B.V || c.pin_dev[k] >= g->G || !((dset >> c.pin_dev[k]) & 1u))
+          bad = true;
         for (int k2 = 0; k2 < k; k2++) bad |= c.pin_op[k2] == c.pin_op[k];
       }
     } else if (c.kind == FASTT_KIND_SPLIT) {
       if (c.split_op < 0 || c.split_op >= B.V || c.split_dim > 1 ||
           !(g->split_mask_h[c.split_op] & (1u << c.split_dim)) || c.split_n < 2 || c.split_n > g->G)
         bad = true;
-    } else {
+    } else if (c.kind != FASTT_KIND_BASE) {
       bad = true;
     }
     if (bad) return fail(FASTT_EINVAL, "invalid candidate");
@@ -1440,7 +1456,7 @@ fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, 
                                 fastt_split_result *out) {
   fastt_graph *g = (fastt_graph *)gc_;
   if (!g || !out) return fail(FASTT_EINVAL, "NULL argument");
-  const uint32_t flags = flags_of(opts) & (FASTT_F_CP_PIN | FASTT_F_POLICY_INSERT);
+  const uint32_t flags = flags_of(opts) & (FASTT_F_CP_PIN | FASTT_F_POLICY_INSERT | FASTT_F_MEM_LIVE);
   const bool best_mode = (flags_of(opts) & FASTT_F_SPLIT_BEST) != 0;
   memset(out, 0, sizeof *out);
   std::lock_guard<std::mutex> lk(g->mu);

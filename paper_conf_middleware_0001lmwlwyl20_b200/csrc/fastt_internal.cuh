@@ -98,6 +98,7 @@ struct PrepGraph {
   uint32_t *cp;     // critical path (positions)
   int64_t *pmem;    // cp prefix sums of mem, cp_len+1
   int64_t *pcost;   // cp prefix sums of cost, (cp_len+1)*G
+  int64_t *act;     // n: output bytes mem - param per position (liveness memory, R24)
   // scratch for the sort / scans
   uint64_t *key0, *key1;
   uint32_t *val0, *val1;
@@ -109,7 +110,7 @@ struct Cand {
   int32_t split_op;
   int32_t pin_op[4];
   uint8_t pin_dev[4];
-  uint8_t pad[4];
+  uint32_t dev_mask;  // device subset (R25), 0 = all
 };
 static_assert(sizeof(Cand) == 32, "candidate record is 32 bytes");
 
@@ -119,6 +120,7 @@ struct StreamState {
   int32_t *live;        // n_live uids
   int32_t n_live;
   int64_t n_split;
+  int32_t n_subset;     // device-subset block after the SPLITs (R25): G-1 or 0
   int32_t *split_op;    // n_split
   uint8_t *split_dim, *split_n;
   uint64_t seed;
@@ -130,6 +132,7 @@ __host__ __device__ inline int64_t comm_class(const GraphConst &c, int64_t bytes
   int64_t num = bytes * c.beta[k];
   return c.alpha[k] + (num + 999999) / 1000000;
 }
+__host__ __device__ inline uint32_t all_devices(int G) { return G >= 32 ? 0xFFFFFFFFu : ((1u << G) - 1u); }
 __host__ __device__ inline int64_t ceil_div64(int64_t a, int64_t b) { return (a + b - 1) / b; }
 __host__ __device__ inline int64_t part_bytes(int64_t b, int n, int k) { return b / n + (k < b % n ? 1 : 0); }
 
@@ -187,6 +190,8 @@ struct SimArgs {
   int32_t gshift;        // ceil(log2(G)): lanes per predecessor group = 1 << gshift
   int32_t track_best;
   int32_t need_mem;      // track per-device memory (caps present or peak output)
+  int32_t live_mem;      // liveness memory (R24, FASTT_F_MEM_LIVE); implies need_mem
+  int32_t fastcomm;      // uint32 time and one link class: comm values inline in the cards
   int32_t cap_check;     // some device has a finite memory cap (R8)
   // BASE-schedule prefix sharing: 1 = record the snapshot (one BASE run),
   // 2 = start eligible PIN candidates from it at their first pinned op

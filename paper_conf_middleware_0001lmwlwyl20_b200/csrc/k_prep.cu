@@ -202,12 +202,25 @@ void launch_patch_split(const RawGraph *base, RawGraph *raws, const GraphConst *
 
 // ----------------------------------------------------------------- ranks
 
-// c_ij of P:544-547 with the allowed sets of R5
-__device__ __forceinline__ int64_t c_allowed(const GraphConst &gc, int64_t bytes, int su, int tv) {
+// link classes over the device pairs (s, t), s in S, t in T, s != t
+__device__ __forceinline__ uint32_t class_mask(const GraphConst &gc, uint32_t S, uint32_t T) {
+  uint32_t m = 0;
+  for (uint32_t a = S; a; a &= a - 1) {
+    const int s = __ffs(a) - 1;
+    for (uint32_t b = T & ~(1u << s); b; b &= b - 1) m |= 1u << gc.link_class[s * gc.G + (__ffs(b) - 1)];
+  }
+  return m;
+}
+
+// c_ij of P:544-547 with the allowed sets of R5: a pinned endpoint's device,
+// else the candidate's device set dset (R25; offm = class_mask(dset, dset))
+__device__ __forceinline__ int64_t c_allowed(const GraphConst &gc, int64_t bytes, int su, int tv, uint32_t dset,
+                                             uint32_t offm) {
+  const bool full = dset == all_devices(gc.G);
   uint32_t mask;
-  if (su < 0 && tv < 0) mask = gc.offdiag_mask;
-  else if (su >= 0 && tv < 0) mask = gc.row_mask[su];
-  else if (su < 0) mask = gc.col_mask[tv];
+  if (su < 0 && tv < 0) mask = offm;
+  else if (su >= 0 && tv < 0) mask = full ? gc.row_mask[su] : class_mask(gc, 1u << su, dset);
+  else if (su < 0) mask = full ? gc.col_mask[tv] : class_mask(gc, dset, 1u << tv);
   else {
     if (su == tv) return 0;
     return comm_class(gc, bytes, gc.link_class[su * gc.G + tv]);
@@ -233,7 +246,8 @@ __device__ __forceinline__ int pin_of(int32_t u, const int32_t *po, const int32_
 // rank of one op u evaluated by one lane: w_u over the allowed
 // devices + max over successors of (c_uv + rank_v)
 __device__ __forceinline__ void rank_one(const RawGraph &R, const GraphConst &gc, uint64_t *rank, int32_t u,
-                                         const int32_t *po, const int32_t *pd, int np) {
+                                         const int32_t *po, const int32_t *pd, int np, uint32_t dset,
+                                         uint32_t offm) {
   const int G = gc.G;
   const int pu = pin_of(u, po, pd, np);
   int64_t w = 0;
@@ -241,13 +255,14 @@ __device__ __forceinline__ void rank_one(const RawGraph &R, const GraphConst &gc
   else
     for (int d = 0; d < G; d++) {
       const int64_t c = R.cost[(int64_t)u * G + d];
-      w = c > w ? c : w;
+      w = ((dset >> d) & 1u) && c > w ? c : w;
     }
   const uint32_t off = R.succ_off[u], cnt_s = R.succ_cnt[u];
   uint64_t best = 0;
   for (uint32_t j = 0; j < cnt_s; j++) {
     const int32_t s = R.succ_dst[off + j];
-    const uint64_t v = (uint64_t)c_allowed(gc, R.succ_bytes[off + j], pu, pin_of(s, po, pd, np)) + rank[s];
+    const uint64_t v =
+        (uint64_t)c_allowed(gc, R.succ_bytes[off + j], pu, pin_of(s, po, pd, np), dset, offm) + rank[s];
     best = v > best ? v : best;
   }
   rank[u] = (uint64_t)w + best;
@@ -266,14 +281,17 @@ __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *g
   const GraphConst &gc = *gcp;
   int32_t po[MAXPINS], pd[MAXPINS];
   int np = 0;
+  uint32_t dset = all_devices(gc.G);
   if (cands) {
     Cand c = cands[slot];
     if (c.kind == 1) {
       np = c.n_pins;
       for (int k = 0; k < MAXPINS; k++) { po[k] = c.pin_op[k]; pd[k] = c.pin_dev[k]; }
     }
+    if (c.dev_mask) dset = c.dev_mask;  // R25
   }
   for (int k = np; k < MAXPINS; k++) { po[k] = -1; pd[k] = -1; }
+  const uint32_t offm = dset == all_devices(gc.G) ? gc.offdiag_mask : class_mask(gc, dset, dset);
   uint64_t *rank = P.rank;
   for (int32_t u = lane; u < R.V; u += 32) rank[u] = ~0ull;
   __syncwarp();
@@ -296,7 +314,7 @@ __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *g
       const int32_t extra = (phase == 1 && split && lev == ho) ? R.ov_n : 0;
       for (int32_t q = lane; q < cnt + extra; q += 32) {
         int32_t u = q < cnt ? (list ? list[q] : lo + q) : R.ov_base + R.ov_P + (q - cnt);
-        if (R.alive[u]) rank_one(R, gc, rank, u, po, pd, np);
+        if (R.alive[u]) rank_one(R, gc, rank, u, po, pd, np, dset, offm);
       }
       __syncwarp();
     }
@@ -546,6 +564,7 @@ __global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, Prep
       c[CW_MEMHI] = (uint32_t)(m >> 32);
       c[CW_UID] = u;
       c[CW_FLAGS] = 0;
+      P.act[p] = R.mem[u] - R.param[u];
       P.npred[p] = np_;
       if (np_ == 0) atomicOr(&P.srcbits[p >> 5], 1u << (p & 31));
     }

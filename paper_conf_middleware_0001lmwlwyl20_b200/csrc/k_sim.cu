@@ -54,6 +54,10 @@ template <> struct Slab<uint32_t> {
     ft = (uint32_t)w;
     plc = (uint32_t)(w >> 32) & 0xFF;
   }
+  __device__ static void decode(const W &w, uint32_t &ft, uint32_t &plc) {
+    ft = (uint32_t)w;
+    plc = (uint32_t)(w >> 32) & 0xFF;
+  }
   __device__ static uint32_t indeg(const W *s, uint32_t p) {
     return (*((const uint32_t *)(s + p) + 1)) >> 8;
   }
@@ -62,6 +66,9 @@ template <> struct Slab<uint32_t> {
     s[p] = ((unsigned long long)plc << 32) | ft;
   }
   __device__ static void make(W &w, uint32_t ft, uint32_t plc) { w = ((unsigned long long)plc << 32) | ft; }
+  // liveness (R24): a scheduled op keeps its unreleased-consumer count in the indegree field
+  __device__ static uint32_t hiword(const W *s, uint32_t p) { return *((const uint32_t *)(s + p) + 1); }
+  __device__ static void set_hiword(W *s, uint32_t p, uint32_t v) { *((uint32_t *)(s + p) + 1) = v; }
 };
 template <> struct Slab<uint64_t> {
   typedef ulonglong2 W;
@@ -73,6 +80,10 @@ template <> struct Slab<uint64_t> {
   }
   __device__ static void load(const W *s, uint32_t p, uint64_t &ft, uint32_t &plc) {
     W w = s[p];
+    ft = w.x;
+    plc = (uint32_t)w.y & 0xFF;
+  }
+  __device__ static void decode(const W &w, uint64_t &ft, uint32_t &plc) {
     ft = w.x;
     plc = (uint32_t)w.y & 0xFF;
   }
@@ -90,6 +101,8 @@ template <> struct Slab<uint64_t> {
     w.x = ft;
     w.y = plc;
   }
+  __device__ static uint32_t hiword(const W *s, uint32_t p) { return *((const uint32_t *)(s + p) + 2); }
+  __device__ static void set_hiword(W *s, uint32_t p, uint32_t v) { *((uint32_t *)(s + p) + 2) = v; }
 };
 
 __device__ __forceinline__ uint64_t splitmix64(uint64_t &s) {
@@ -133,13 +146,18 @@ __device__ __forceinline__ void prefetch_l2(const void *p) { asm volatile("prefe
 __device__ Cand stream_cand(const StreamState &S, int64_t c) {
   Cand o;
   o.kind = 0; o.n_pins = 0; o.split_dim = 0; o.split_n = 0; o.split_op = -1;
-  for (int k = 0; k < 4; k++) { o.pin_op[k] = -1; o.pin_dev[k] = 0; o.pad[k] = 0; }
+  for (int k = 0; k < 4; k++) { o.pin_op[k] = -1; o.pin_dev[k] = 0; }
+  o.dev_mask = 0;
   if (c == 0) return o;
   if (c <= S.n_split) {
     o.kind = 2;
     o.split_op = S.split_op[c - 1];
     o.split_dim = S.split_dim[c - 1];
     o.split_n = S.split_n[c - 1];
+    return o;
+  }
+  if (c <= S.n_split + S.n_subset) {  // R25: BASE on the first k devices
+    o.dev_mask = (1u << (int)(c - S.n_split)) - 1u;
     return o;
   }
   o.kind = 1;
@@ -257,8 +275,8 @@ __device__ __noinline__ bool pin_changes_ranks(const PrepGraph *pg, const GraphC
 // receives round r.
 template <typename T>
 __device__ __noinline__ void cp_rounds_g(const PrepGraph *pg, int np, const uint32_t *pp, unsigned gm, int gb, int d,
-                                         int G, int64_t cap_d, uint32_t &r_lo, uint32_t &r_hi, int &r_dev,
-                                         int &nrounds, uint32_t *pcp, int64_t &reserved) {
+                                         int G, int64_t cap_d, uint32_t dset, uint32_t &r_lo, uint32_t &r_hi,
+                                         int &r_dev, int &nrounds, uint32_t *pcp, int64_t &reserved) {
   const uint32_t *card = pg->card;
   const T *costp = (const T *)pg->costp;
   const int32_t L = pg->cp_len;
@@ -316,7 +334,7 @@ __device__ __noinline__ void cp_rounds_g(const PrepGraph *pg, int np, const uint
       if (j < m && (int32_t)pcs[j] < re) v -= pcd[j];
     return v;
   };
-  uint32_t devs = G == 32 ? FULL : ((1u << G) - 1);
+  uint32_t devs = dset;  // the candidate's devices (R25)
   int32_t k = 0;
   while (k < Lf && devs) {
     int32_t t = 0;
@@ -367,7 +385,9 @@ __device__ __noinline__ void cp_rounds_g(const PrepGraph *pg, int np, const uint
 // warp converged (groups that finished idle) so every shuffle/vote is a
 // full-warp instruction.  T: time type; MEM: track per-device memory;
 // INS: insertion policy (R1i) -- lane d keeps device d's idle slots.
-template <typename T, int GSH, bool MEM, bool INS>
+// FC: uint32 time and one link class -- predecessor comm values come from
+// the op's card (no per-edge comm loads).
+template <typename T, int GSH, bool MEM, bool INS, bool FC>
 __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
   typedef typename Slab<T>::W W;
   constexpr int GP = 1 << GSH;   // lanes per candidate (>= G)
@@ -400,7 +420,9 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
   const int64_t cap_d = d < G ? gc.cap[d] : 0;
   const bool cp_on = (a.flags & 1u) != 0;
   const bool cap_chk = MEM && a.cap_check != 0;
-  const bool fastcomm = sizeof(T) == 4 && K == 1;
+  const bool lmem = MEM && a.live_mem != 0;  // liveness memory (R24)
+  constexpr bool fastcomm = FC;
+  static_assert(!FC || sizeof(T) == 4, "card comm values are uint32");
   GapRec<T> *const gpool = INS ? (GapRec<T> *)a.gap + cslot * a.gap_stride : nullptr;
   if (d == 0) {
     s_best[lead][0] = a.track_best ? a.wbest[2 * cslot] : I64MAX;
@@ -448,9 +470,14 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
     int np = 0;
     uint8_t st = 0;
     bool defer = false;
+    const uint32_t all = all_devices(G);
+    const uint32_t dset = (active && c.dev_mask) ? c.dev_mask : all;  // R25
     if (active) {
       if (a.mode != 2) {
-        if (c.kind == 0) {
+        if (c.dev_mask & ~all) st = 2;
+        else if (dset != all) defer = true;  // ranks over the subset: preparation pipeline
+        if (st) {
+        } else if (c.kind == 0) {
         } else if (c.kind == 1) {
           np = c.n_pins;
           if (np < 1 || np > MAXPINS) st = 2;
@@ -458,7 +485,8 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
             bool bad = false;
             for (int k = 0; k < np; k++) {
               int32_t o = c.pin_op[k];
-              if (o < 0 || o >= Vraw || posm[o] == NONE || c.pin_dev[k] >= G) bad = true;
+              if (o < 0 || o >= Vraw || posm[o] == NONE || c.pin_dev[k] >= G || !((dset >> c.pin_dev[k]) & 1u))
+                bad = true;
               for (int k2 = 0; k2 < k; k2++) bad |= c.pin_op[k2] == o;
             }
             if (bad) st = 2;
@@ -476,7 +504,10 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
         np = c.kind == 1 ? c.n_pins : 0;
       }
     }
-    if (st) np = 0;
+    if (st) {
+      np = 0;
+      defer = false;
+    }
     // the candidate's pins as group-uniform arrays (positions, packed devices)
     uint32_t pp[MAXPINS] = {NONE, NONE, NONE, NONE};
     uint32_t pdv = 0;
@@ -505,12 +536,12 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
     const bool run = active && !defer && st == 0;
 
     // ------------------------------------------------------ prologue
-    int64_t used = 0, reserved = 0;
+    int64_t used = 0, reserved = 0, peakv = 0;
     uint32_t r_lo = 0, r_hi = 0;
     int r_dev = -1, nrounds = 0;
     uint32_t pcp[MAXPINS] = {NONE, NONE, NONE, NONE};
     if (run && cp_on && pg->cp_len > 0)
-      cp_rounds_g<T>(pg, np, pp, gm, gb, d, G, cap_d, r_lo, r_hi, r_dev, nrounds, pcp, reserved);
+      cp_rounds_g<T>(pg, np, pp, gm, gb, d, G, cap_d, dset, r_lo, r_hi, r_dev, nrounds, pcp, reserved);
     if (d == 0) {
       s_res[lead] = res_idx;
       s_sidx[lead] = sidx;
@@ -613,6 +644,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       my_dev = d < 4 ? (int)((pdv >> (8 * d)) & 0xFF) : 0;
     }
     __syncwarp();
+    const bool dev_ok = d < G && ((dset >> d) & 1u);  // this lane's device may be used (R25)
     const bool any_pins = __any_sync(FULL, np > 0);
     const bool any_cp = __any_sync(FULL, nrounds > 0);
     const bool any_out = __any_sync(FULL, want_out);
@@ -670,13 +702,22 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       const uint32_t cmi[4] = {hc.x, hc.y, hc.z, hc.w};
       T ft[4];
       uint32_t pl[4];
+      // all four records and the successor's indegree are loaded
+      // unconditionally (unused card slots hold position 0), so the loads
+      // issue back to back instead of one dependent round trip each
+      W rw[4];
+#pragma unroll
+      for (int k = 0; k < 4; k++) rw[k] = slab0[SLOT(src[k])];
+      const uint32_t sdeg_raw = Slab<T>::indeg(slab0, SLOT(s0));
 #pragma unroll
       for (int k = 0; k < 4; k++) {
-        ft[k] = 0;
-        pl[k] = (uint32_t)d;
-        if ((uint32_t)k < npred) Slab<T>::load(slab0, SLOT(src[k]), ft[k], pl[k]);
+        T f;
+        uint32_t p;
+        Slab<T>::decode(rw[k], f, p);
+        ft[k] = (uint32_t)k < npred ? f : (T)0;
+        pl[k] = (uint32_t)k < npred ? p : (uint32_t)d;
       }
-      const uint32_t sdeg = ((uint32_t)d < nsucc) ? Slab<T>::indeg(slab0, SLOT(s0)) : 1u;
+      const uint32_t sdeg = ((uint32_t)d < nsucc) ? sdeg_raw : 1u;
       // EST = max(avail[d], max_pred FT + c(pred -> i on d))   (R1, R6)
       // (INSERT: first the data-ready time r, then the idle-slot search)
       T est = INS ? (T)0 : avail;
@@ -764,7 +805,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       }
       int64_t mem = 0;
       if (MEM) mem = (int64_t)(((uint64_t)__ldg(cd + CW_MEMHI) << 32) | __ldg(cd + CW_MEMLO));
-      bool feas = live && d < G && (forced < 0 || d == forced);
+      bool feas = live && dev_ok && (forced < 0 || d == forced);
       if (cap_chk && (forced < 0 || pert)) feas = feas && (used + reserved + mem <= cap_d);
       // argmin EFT over feasible devices, ties -> lowest device (Alg. 1 l.12-19, R3, R8)
       const T key = feas ? eft : TT<T>::MAXV;
@@ -839,10 +880,41 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
         if (MEM) {
           used += mem;
           if (forced >= 0 && !pert) reserved -= mem;
+          if (lmem) peakv = used > peakv ? used : peakv;
         }
       }
+      if (lmem) {
+        // R24: this op was the last unreleased consumer of an input -> free
+        // that input's output bytes on its device; a sink frees its own
+        uint32_t hw[4];
+#pragma unroll
+        for (int k = 0; k < 4; k++) hw[k] = (go && (uint32_t)k < npred) ? Slab<T>::hiword(slab0, SLOT(src[k])) : 256u;
+        __syncwarp();
+#pragma unroll
+        for (int k = 0; k < 4; k++)
+          if (go && (uint32_t)k < npred) {
+            if (d == 0) Slab<T>::set_hiword(slab0, SLOT(src[k]), hw[k] - 256u);
+            if ((hw[k] >> 8) == 1u && (uint32_t)d == pl[k]) used -= __ldg(pg->act + src[k]);
+          }
+        if (__any_sync(FULL, go && npred > 4u)) {
+          for (uint32_t k = 4; __any_sync(FULL, go && k < npred); k++) {
+            uint32_t sp = 0, w = 256u;
+            if (go && k < npred) {
+              sp = __ldg(pg->pe_src + h0.y + k);
+              w = Slab<T>::hiword(slab0, SLOT(sp));
+            }
+            __syncwarp();
+            if (go && k < npred) {
+              if (d == 0) Slab<T>::set_hiword(slab0, SLOT(sp), w - 256u);
+              if ((w >> 8) == 1u && (uint32_t)d == (w & 0xFFu)) used -= __ldg(pg->act + sp);
+            }
+          }
+        }
+        if (go && nsucc == 0 && d == dsel) used -= __ldg(pg->act + i);
+      }
       if (go) makespan = mn > makespan ? mn : makespan;
-      if (go && d == 0) Slab<T>::sched(slab0, SLOT(i), mn, (uint32_t)dsel);
+      // (the indegree field of a scheduled op holds its consumer count under R24)
+      if (go && d == 0) Slab<T>::sched(slab0, SLOT(i), mn, (uint32_t)dsel | (lmem ? nsucc << 8 : 0u));
       if (any_out) {
         const T stt = __shfl_sync(FULL, est, gb + dsel);
         if (go && want_out && d == 0) {
@@ -904,7 +976,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
           a.out.makespan[ri] = ms64;
           a.out.status[ri] = infeas ? 1 : 0;
         }
-        if (a.out.peak && d < G) a.out.peak[ri * G + d] = infeas ? -1 : used;
+        if (a.out.peak && d < G) a.out.peak[ri * G + d] = infeas ? -1 : (lmem ? peakv : used);
         if (infeas && a.out.place != nullptr) {
           const int64_t o2 = ri * (int64_t)a.out.vmax;
           for (int32_t u = d; u < a.out.vmax; u += GP) {
@@ -928,28 +1000,29 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
   }
 }
 
-template <typename T, bool MEM, bool INS>
+template <typename T, bool MEM, bool INS, bool FC>
 static const void *sim_fn_t(int gshift) {
   switch (gshift) {
-    case 0: return (const void *)k_sim<T, 0, MEM, INS>;
-    case 1: return (const void *)k_sim<T, 1, MEM, INS>;
-    case 2: return (const void *)k_sim<T, 2, MEM, INS>;
-    case 3: return (const void *)k_sim<T, 3, MEM, INS>;
-    case 4: return (const void *)k_sim<T, 4, MEM, INS>;
-    default: return (const void *)k_sim<T, 5, MEM, INS>;
+    case 0: return (const void *)k_sim<T, 0, MEM, INS, FC>;
+    case 1: return (const void *)k_sim<T, 1, MEM, INS, FC>;
+    case 2: return (const void *)k_sim<T, 2, MEM, INS, FC>;
+    case 3: return (const void *)k_sim<T, 3, MEM, INS, FC>;
+    case 4: return (const void *)k_sim<T, 4, MEM, INS, FC>;
+    default: return (const void *)k_sim<T, 5, MEM, INS, FC>;
   }
 }
-template <typename T>
+template <typename T, bool FC>
 static const void *sim_fn_m(int gshift, bool mem, bool ins) {
-  if (ins) return mem ? sim_fn_t<T, true, true>(gshift) : sim_fn_t<T, false, true>(gshift);
-  return mem ? sim_fn_t<T, true, false>(gshift) : sim_fn_t<T, false, false>(gshift);
+  if (ins) return mem ? sim_fn_t<T, true, true, FC>(gshift) : sim_fn_t<T, false, true, FC>(gshift);
+  return mem ? sim_fn_t<T, true, false, FC>(gshift) : sim_fn_t<T, false, false, FC>(gshift);
 }
-static const void *sim_fn(int tbits, int gshift, bool mem, bool ins = false) {
-  return tbits == 32 ? sim_fn_m<uint32_t>(gshift, mem, ins) : sim_fn_m<uint64_t>(gshift, mem, ins);
+static const void *sim_fn(int tbits, int gshift, bool mem, bool ins = false, bool fc = false) {
+  if (tbits != 32) return sim_fn_m<uint64_t, false>(gshift, mem, ins);
+  return fc ? sim_fn_m<uint32_t, true>(gshift, mem, ins) : sim_fn_m<uint32_t, false>(gshift, mem, ins);
 }
 
 void launch_sim(const SimArgs &a, int tbits, int grid, int block, size_t smem, cudaStream_t st) {
-  const void *f = sim_fn(tbits, a.gshift, a.need_mem != 0, a.ins != 0);
+  const void *f = sim_fn(tbits, a.gshift, a.need_mem != 0, a.ins != 0, a.fastcomm != 0);
   SimArgs aa = a;
   void *args[] = {&aa};
   cudaLaunchKernel(f, dim3(grid), dim3(block), args, smem, st);
@@ -957,15 +1030,15 @@ void launch_sim(const SimArgs &a, int tbits, int grid, int block, size_t smem, c
 
 int sim_occupancy(int tbits, int gshift, int block, size_t smem) {
   int nb = 1 << 30, x = 0;
-  for (int mem = 0; mem < 2; mem++) {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, sim_fn(tbits, gshift, mem), block, smem);
+  for (int v = 0; v < 4; v++) {
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, sim_fn(tbits, gshift, v & 1, false, v >> 1), block, smem);
     nb = x < nb ? x : nb;
   }
   return nb;
 }
 cudaError_t sim_set_smem(int tbits, int gshift, size_t smem) {
-  for (int v = 0; v < 4; v++) {
-    cudaError_t e = cudaFuncSetAttribute(sim_fn(tbits, gshift, v & 1, v >> 1),
+  for (int v = 0; v < 8; v++) {
+    cudaError_t e = cudaFuncSetAttribute(sim_fn(tbits, gshift, v & 1, (v >> 1) & 1, v >> 2),
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
   }

@@ -26,7 +26,7 @@ INT64_MAX = np.iinfo(np.int64).max
 
 CANDIDATE_DTYPE = np.dtype(
     [("kind", "u1"), ("n_pins", "u1"), ("split_dim", "u1"), ("split_n", "u1"),
-     ("split_op", "<i4"), ("pin_op", "<i4", (4,)), ("pin_dev", "u1", (4,)), ("_pad", "u1", (4,))]
+     ("split_op", "<i4"), ("pin_op", "<i4", (4,)), ("pin_dev", "u1", (4,)), ("dev_mask", "<u4")]
 )
 assert CANDIDATE_DTYPE.itemsize == 32
 
@@ -43,7 +43,7 @@ class fastt_graph_desc(C.Structure):
 
 class fastt_gen_params(C.Structure):
     _fields_ = [("seed", C.c_uint64), ("pin_k_min", C.c_uint8), ("pin_k_max", C.c_uint8),
-                ("n_pow2_only", C.c_uint8), ("_pad", C.c_uint8 * 5)]
+                ("n_pow2_only", C.c_uint8), ("subset_prefixes", C.c_uint8), ("_pad", C.c_uint8 * 4)]
 
 
 class fastt_opts(C.Structure):
@@ -67,6 +67,7 @@ SYMBOLS = ["fastt_load_graph", "fastt_free_graph", "fastt_graph_info", "fastt_ra
            "fastt_free_split_result", "fastt_last_timing", "fastt_last_error", "fastt_version"]
 F_TIMING = 16
 F_SPLIT_BEST = 32
+F_MEM_LIVE = 64
 
 _lib = None
 
@@ -142,16 +143,17 @@ def _opts(flags=0, stream=None):
     return o
 
 
-def gen_params(seed, pin_k_min=1, pin_k_max=4, n_pow2_only=False):
+def gen_params(seed, pin_k_min=1, pin_k_max=4, n_pow2_only=False, subset_prefixes=False):
     g = fastt_gen_params()
     g.seed = int(seed) & 0xFFFFFFFFFFFFFFFF
     g.pin_k_min = pin_k_min
     g.pin_k_max = pin_k_max
     g.n_pow2_only = 1 if n_pow2_only else 0
+    g.subset_prefixes = 1 if subset_prefixes else 0
     return g
 
 
-def make_candidate(kind=KIND_BASE, pins=(), split=None):
+def make_candidate(kind=KIND_BASE, pins=(), split=None, dev_mask=0):
     c = np.zeros(1, CANDIDATE_DTYPE)[0]
     c["kind"] = kind
     c["split_op"] = -1
@@ -162,6 +164,7 @@ def make_candidate(kind=KIND_BASE, pins=(), split=None):
     c["n_pins"] = len(pins)
     if split is not None:
         c["split_op"], c["split_dim"], c["split_n"] = split
+    c["dev_mask"] = dev_mask
     return c
 
 
