@@ -251,6 +251,7 @@ struct fastt_graph {
   void *slab = nullptr;
   void *gap = nullptr;  // INSERT idle-slot pools, one per candidate slot (lazy)
   int64_t gap_stride = 0;
+  int ins_grid = 0;
   int64_t *wbest = nullptr, *best_dev = nullptr;
   unsigned long long *counters = nullptr;  // [0] work counter, [1] deferred count
   int64_t *defer_q = nullptr;
@@ -457,15 +458,23 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     g->sim_ncap = ncap;
   }
   if ((flags & FASTT_F_POLICY_INSERT) && !g->gap) {
-    // INSERT: at most one idle-slot record per placed op per candidate
-    const int64_t nslot = (int64_t)g->sim_grid * (g->sim_block / 32) * g->sim_cpw;
+    // INSERT: per candidate slot and device an array of at most (ops on
+    // the device + 1) idle slots; the resident INSERT grid is capped so the
+    // arrays take at most a third of the free device memory
     g->gap_stride = g->sim_ncap + 1;
-    const size_t rec = B.tbits == 32 ? sizeof(GapRec<uint32_t>) : sizeof(GapRec<uint64_t>);
-    if (cudaMalloc(&g->gap, (size_t)nslot * g->gap_stride * rec) != cudaSuccess) {
+    const size_t rec = B.tbits == 32 ? sizeof(GapSlot<uint32_t>) : sizeof(GapSlot<uint64_t>);
+    const size_t per_block = (size_t)(g->sim_block / 32) * g->sim_cpw * g->G * g->gap_stride * rec;
+    size_t fr = 0, tot = 0;
+    CK(cudaMemGetInfo(&fr, &tot));
+    int64_t ig = std::min<int64_t>(g->sim_grid, (int64_t)(fr / 3 / per_block));
+    if (ig > g->sms) ig -= ig % g->sms;
+    if (ig < 1) return fail(FASTT_ENOMEM, "INSERT idle-slot arrays (%zu bytes per block)", per_block);
+    if (cudaMalloc(&g->gap, (size_t)ig * per_block) != cudaSuccess) {
       cudaGetLastError();
       g->gap = nullptr;
-      return fail(FASTT_ENOMEM, "INSERT idle-slot pools (%lld slots)", (long long)nslot);
+      return fail(FASTT_ENOMEM, "INSERT idle-slot arrays (%lld blocks)", (long long)ig);
     }
+    g->ins_grid = (int)ig;
   }
   if (!g->counters) {
     CK(cudaMalloc(&g->counters, 2 * sizeof(unsigned long long)));
@@ -510,6 +519,7 @@ static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
     a.ins = 1;
     a.gap = g->gap;
     a.gap_stride = g->gap_stride;
+    a.ins_grid = g->ins_grid;
   }
   return a;
 }

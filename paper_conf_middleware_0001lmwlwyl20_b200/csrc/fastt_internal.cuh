@@ -202,17 +202,18 @@ struct SimArgs {
   void *snap_ms;           // [n+1] T: makespan before step t
   void *snap_rec;          // [n] final slab records of the BASE schedule
   int32_t *snap_rounds;    // [4] base CP rounds: count, dev0, lo0, hi0 (written when recording)
-  // INSERT policy (R1i, NEXT N1): per candidate slot a pool of idle-slot
-  // records (GapRec<T>), linked per device; gap_stride records per slot
+  // INSERT policy (R1i, NEXT N1): idle-slot arrays (GapSlot<T>) per
+  // candidate slot and device, sorted by start,
+  // gap_stride entries each; INSERT launches use at most ins_grid blocks
   int32_t ins;
   void *gap;
   int64_t gap_stride;
+  int32_t ins_grid;
 };
 
-// one idle slot [a, b) of a device under INSERT, linked by `next` (record index)
-template <typename T> struct alignas(16) GapRec {
+// one idle slot [a, b) of a device under INSERT
+template <typename T> struct GapSlot {
   T a, b;
-  uint32_t next;
 };
 
 void launch_sim(const SimArgs &a, int tbits, int grid, int block, size_t smem, cudaStream_t st);

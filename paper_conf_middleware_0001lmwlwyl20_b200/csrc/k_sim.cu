@@ -423,7 +423,9 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
   const bool lmem = MEM && a.live_mem != 0;  // liveness memory (R24)
   constexpr bool fastcomm = FC;
   static_assert(!FC || sizeof(T) == 4, "card comm values are uint32");
-  GapRec<T> *const gpool = INS ? (GapRec<T> *)a.gap + cslot * a.gap_stride : nullptr;
+  // INSERT: lane d's array of device d's idle slots (sorted by start)
+  GapSlot<T> *const gsl =
+      INS ? (GapSlot<T> *)a.gap + ((size_t)cslot * G + (size_t)(d < G ? d : 0)) * (size_t)a.gap_stride : nullptr;
   if (d == 0) {
     s_best[lead][0] = a.track_best ? a.wbest[2 * cslot] : I64MAX;
     s_best[lead][1] = a.track_best ? a.wbest[2 * cslot + 1] : -1;
@@ -575,9 +577,8 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
     }
     uint32_t top = 0;
     T avail = 0, makespan = 0;
-    // INSERT: this lane's device's idle slots before `avail` (a list sorted
-    // by start, head/tail record), and the group's record count
-    uint32_t ghead = NONE, gtail = NONE, galloc = 0;
+    // INSERT: the number of idle slots before `avail` on this lane's device
+    uint32_t gn = 0;
     if (run && share) {
       avail = d < G ? __ldg((const T *)a.snap_avail + (size_t)t0 * G + d) : (T)0;
       makespan = __ldg((const T *)a.snap_ms + t0);
@@ -748,25 +749,28 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       }
       // INSERT (R1i): the first idle slot [ga, gb) before avail
       // with max(ga, r) + w <= gb, else the open-ended slot at avail
-      uint32_t gk = NONE, gprev = NONE, gnx = NONE;
+      // (the slots are disjoint and sorted, so no slot ending before r can
+      // fit: a binary search finds the first with b >= r, then a short scan)
+      uint32_t gk = NONE;
       T ga = 0, gbb = 0;
       if (INS && live && d < G && est < avail) {
-        uint32_t prev = NONE;
+        uint32_t lo = 0, hi = gn;
+        while (lo < hi) {
+          const uint32_t mid = (lo + hi) >> 1;
+          if (gsl[mid].b < est) lo = mid + 1;
+          else hi = mid;
+        }
         T t = avail;
-        for (uint32_t k = ghead; k != NONE;) {
-          const GapRec<T> e = gpool[k];
+        for (uint32_t k = lo; k < gn; k++) {
+          const GapSlot<T> e = gsl[k];
           const T tt = e.a > est ? e.a : est;
           if (tt + cst <= e.b) {
             gk = k;
-            gprev = prev;
-            gnx = e.next;
             ga = e.a;
             gbb = e.b;
             t = tt;
             break;
           }
-          prev = k;
-          k = e.next;
         }
         est = t;
       }
@@ -834,46 +838,39 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       }
       tstep++;
       if (INS) {
-        // the chosen device's lane updates its idle slots
-        bool alloc = false;
+        // the chosen device's lane updates its idle slots: the slot the op
+        // went into shrinks, splits in two (the tail of the array shifts
+        // up one) or disappears (the tail shifts down); an op appended
+        // after a data wait leaves a new slot [avail, ST)
         if (go && d == dsel) {
           if (gk != NONE) {
             const bool left = est > ga, right = est + cst < gbb;
             if (left && right) {
-              GapRec<T> ne;
+              for (uint32_t k = gn; k > gk + 1; k--) gsl[k] = gsl[k - 1];
+              GapSlot<T> ne;
               ne.a = est + cst;
               ne.b = gbb;
-              ne.next = gnx;
-              gpool[galloc] = ne;
-              gpool[gk].b = est;
-              gpool[gk].next = galloc;
-              if (gtail == gk) gtail = galloc;
-              alloc = true;
+              gsl[gk + 1] = ne;
+              gsl[gk].b = est;
+              gn++;
             } else if (left) {
-              gpool[gk].b = est;
+              gsl[gk].b = est;
             } else if (right) {
-              gpool[gk].a = est + cst;
+              gsl[gk].a = est + cst;
             } else {
-              if (gprev == NONE) ghead = gnx;
-              else gpool[gprev].next = gnx;
-              if (gtail == gk) gtail = gprev;
+              for (uint32_t k = gk; k + 1 < gn; k++) gsl[k] = gsl[k + 1];
+              gn--;
             }
           } else {
             if (est > avail) {
-              GapRec<T> ne;
+              GapSlot<T> ne;
               ne.a = avail;
               ne.b = est;
-              ne.next = NONE;
-              gpool[galloc] = ne;
-              if (gtail == NONE) ghead = galloc;
-              else gpool[gtail].next = galloc;
-              gtail = galloc;
-              alloc = true;
+              gsl[gn++] = ne;
             }
             avail = mn;
           }
         }
-        if (__ballot_sync(FULL, alloc) & gm) galloc++;
       }
       if (go && d == dsel) {
         if (!INS) avail = mn;
@@ -1022,6 +1019,7 @@ static const void *sim_fn(int tbits, int gshift, bool mem, bool ins = false, boo
 }
 
 void launch_sim(const SimArgs &a, int tbits, int grid, int block, size_t smem, cudaStream_t st) {
+  if (a.ins && grid > a.ins_grid) grid = a.ins_grid;  // INSERT slot arrays exist for ins_grid blocks
   const void *f = sim_fn(tbits, a.gshift, a.need_mem != 0, a.ins != 0, a.fastcomm != 0);
   SimArgs aa = a;
   void *args[] = {&aa};
