@@ -241,6 +241,38 @@ typedef struct {
 } fastt_timing;
 fastt_status fastt_last_timing(const fastt_graph *g, fastt_timing *out);
 
+/* Communication cost-model fit ("we gather
+ * tensors across the same source-destination device pairs into one group.
+ * For each group, we use linear regression to obtain a linear model: tensor
+ * size vs. transfer time"; reading R26).  Sample k is a transfer of
+ * bytes[k] bytes from device src_dev[k] to dst_dev[k] (!= src) that took
+ * time_ns[k].  For every ordered pair (s, t) the least-squares line
+ * time = alpha + beta * bytes with alpha >= 0 and beta >= 0 is fitted in
+ * exact integer arithmetic and reported as the nearest integers (halves up)
+ * in the units of the model R10: alpha_ns[s*G+t] in ns,
+ * beta_fs_per_byte[s*G+t] in fs/byte.  A pair with no sample gets 0, 0
+ * (unknown costs are 0); a pair whose samples all have one size
+ * gets beta = 0 and alpha = the mean time.  count[s*G+t] (NULL to skip) is
+ * the number of samples of the pair; the diagonal is 0.
+ * Envelope: 1 <= G <= 32, n_samples < 2^24, bytes and time in [0, 2^40)
+ * (EINVAL otherwise).  Runs on cuda_device: one pass over the samples
+ * (exact 64/128-bit moment sums per pair) and one thread per pair for the
+ * constrained normal equations.  Inputs are host memory unless
+ * FASTT_F_IN_DEVICE, outputs host memory unless FASTT_F_OUT_DEVICE. */
+fastt_status fastt_fit_comm(int32_t n_devices, int64_t n_samples, const uint8_t *src_dev, const uint8_t *dst_dev,
+                            const int64_t *bytes, const int64_t *time_ns, int cuda_device, const fastt_opts *opts,
+                            int64_t *alpha_ns, int64_t *beta_fs_per_byte, int64_t *count);
+
+/* The link model of fastt_graph_desc from per-pair parameters (host only):
+ * pairs with identical (alpha, beta) share a link class; classes are
+ * numbered in row-major order of first appearance over the off-diagonal
+ * pairs; the diagonal gets class 0.  Outputs: link_class[G*G],
+ * *n_link_classes, link_alpha_ns[16], link_beta_fs_per_byte[16].
+ * EUNSUP if more than 16 distinct pairs' parameters exist (K <= 16). */
+fastt_status fastt_link_model(int32_t n_devices, const int64_t *alpha_ns, const int64_t *beta_fs_per_byte,
+                              uint8_t *link_class, int32_t *n_link_classes, int64_t *link_alpha_ns,
+                              int64_t *link_beta_fs_per_byte);
+
 const char *fastt_last_error(void); /* thread-local; valid until the next call on this thread */
 const char *fastt_version(void);
 

@@ -6,7 +6,7 @@ import subprocess
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
-SRCS = [os.path.join(HERE, "csrc", f) for f in ("fastt_abi.cu", "k_prep.cu", "k_sim.cu")]
+SRCS = [os.path.join(HERE, "csrc", f) for f in ("fastt_abi.cu", "k_prep.cu", "k_sim.cu", "k_fit.cu")]
 DEPS = SRCS + [os.path.join(HERE, "csrc", "fastt_internal.cuh"), os.path.join(ROOT, "include", "fastt.h")]
 OUT = os.path.join(HERE, "libfastt.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

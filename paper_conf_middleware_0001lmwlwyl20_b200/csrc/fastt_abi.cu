@@ -1713,6 +1713,95 @@ fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, 
   return FASTT_OK;
 }
 
+// ------------------------------------------------- comm-model fit (N4)
+
+fastt_status fastt_fit_comm(int32_t G, int64_t n, const uint8_t *src, const uint8_t *dst, const int64_t *bytes,
+                            const int64_t *tns, int cuda_device, const fastt_opts *opts, int64_t *alpha,
+                            int64_t *beta, int64_t *count) {
+  if (G < 1 || G > MAXG) return fail(FASTT_EINVAL, "n_devices must be in 1..%d", MAXG);
+  if (n < 0 || n >= (1ll << 24)) return fail(FASTT_EINVAL, "n_samples must be in [0, 2^24)");
+  if (!alpha || !beta || (n > 0 && (!src || !dst || !bytes || !tns))) return fail(FASTT_EINVAL, "NULL argument");
+  const uint32_t flags = flags_of(opts);
+  cudaStream_t st = stream_of(opts);
+  Dev guard(cuda_device);
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cuda_device);
+  const int P = G * G;
+  const bool in_dev = (flags & FASTT_F_IN_DEVICE) != 0, out_dev = (flags & FASTT_F_OUT_DEVICE) != 0;
+  // one scratch block: [sums][err][alpha][beta][count][src][dst][bytes][time]
+  const size_t o_err = al16(fit_sums_bytes(G)), o_a = o_err + 16, o_b = o_a + al16(8 * P), o_c = o_b + al16(8 * P),
+               o_s = o_c + al16(8 * P), o_d = o_s + (in_dev ? 0 : al16(n)), o_by = o_d + (in_dev ? 0 : al16(n)),
+               o_t = o_by + (in_dev ? 0 : al16(8 * n)), tot = o_t + (in_dev ? 0 : al16(8 * n)) + 16;
+  char *buf = nullptr;
+  CK(cudaMalloc(&buf, tot));
+  struct Free {
+    char *p;
+    ~Free() { cudaFree(p); }
+  } fr{buf};
+  const uint8_t *d_src = src, *d_dst = dst;
+  const int64_t *d_by = bytes, *d_t = tns;
+  if (!in_dev && n > 0) {
+    CK(cudaMemcpyAsync(buf + o_s, src, n, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(buf + o_d, dst, n, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(buf + o_by, bytes, 8 * n, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(buf + o_t, tns, 8 * n, cudaMemcpyHostToDevice, st));
+    d_src = (const uint8_t *)(buf + o_s);
+    d_dst = (const uint8_t *)(buf + o_d);
+    d_by = (const int64_t *)(buf + o_by);
+    d_t = (const int64_t *)(buf + o_t);
+  }
+  int64_t *ra = out_dev ? alpha : (int64_t *)(buf + o_a), *rb = out_dev ? beta : (int64_t *)(buf + o_b);
+  int64_t *rc = count ? (out_dev ? count : (int64_t *)(buf + o_c)) : nullptr;
+  launch_fit(G, n, d_src, d_dst, d_by, d_t, buf, (unsigned *)(buf + o_err), ra, rb, rc, sms, st);
+  CK(cudaGetLastError());
+  unsigned err = 0;
+  CK(cudaMemcpyAsync(&err, buf + o_err, 4, cudaMemcpyDeviceToHost, st));
+  if (!out_dev) {
+    CK(cudaMemcpyAsync(alpha, ra, 8 * P, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(beta, rb, 8 * P, cudaMemcpyDeviceToHost, st));
+    if (count) CK(cudaMemcpyAsync(count, rc, 8 * P, cudaMemcpyDeviceToHost, st));
+  }
+  CK(cudaStreamSynchronize(st));
+  if (err) return fail(FASTT_EINVAL, "a sample has a bad device pair or bytes/time outside [0, 2^40)");
+  return FASTT_OK;
+}
+
+fastt_status fastt_link_model(int32_t G, const int64_t *alpha, const int64_t *beta, uint8_t *link_class,
+                              int32_t *n_classes, int64_t *link_alpha, int64_t *link_beta) {
+  if (G < 1 || G > MAXG) return fail(FASTT_EINVAL, "n_devices must be in 1..%d", MAXG);
+  if (!alpha || !beta || !link_class || !n_classes || !link_alpha || !link_beta) return fail(FASTT_EINVAL, "NULL argument");
+  int K = 0;
+  int64_t ka[MAXK], kb[MAXK];
+  for (int s = 0; s < G; s++)
+    for (int t = 0; t < G; t++) {
+      const int64_t a = alpha[s * G + t], b = beta[s * G + t];
+      if (s == t) {
+        link_class[s * G + t] = 0;
+        continue;
+      }
+      if (a < 0 || b < 0) return fail(FASTT_EINVAL, "negative link parameters");
+      int k = 0;
+      while (k < K && !(ka[k] == a && kb[k] == b)) k++;
+      if (k == K) {
+        if (K == MAXK) return fail(FASTT_EUNSUP, "more than %d distinct link parameter pairs", MAXK);
+        ka[K] = a;
+        kb[K] = b;
+        K++;
+      }
+      link_class[s * G + t] = (uint8_t)k;
+    }
+  if (K == 0) {  // G == 1: one (unused) class
+    ka[0] = kb[0] = 0;
+    K = 1;
+  }
+  *n_classes = K;
+  for (int k = 0; k < K; k++) {
+    link_alpha[k] = ka[k];
+    link_beta[k] = kb[k];
+  }
+  return FASTT_OK;
+}
+
 fastt_status fastt_last_timing(const fastt_graph *g, fastt_timing *out) {
   if (!g || !out) return fail(FASTT_EINVAL, "NULL argument");
   *out = g->last;

@@ -234,6 +234,9 @@ void launch_t0_sort(int from_stream, const StreamState &S, int64_t first, int64_
 void launch_gather_sorted(const Cand *src, const int64_t *sidx, const int64_t *sres, const int64_t *qs, int64_t n,
                           Cand *dst, int64_t *didx, int64_t *dres, cudaStream_t st);
 int sim_occupancy(int tbits, int gshift, int block, size_t smem);
+void launch_fit(int G, int64_t n, const uint8_t *src, const uint8_t *dst, const int64_t *bytes, const int64_t *tns,
+                void *sums, unsigned *err, int64_t *alpha, int64_t *beta, int64_t *count, int sms, cudaStream_t st);
+size_t fit_sums_bytes(int G);
 cudaError_t sim_set_smem(int tbits, int gshift, size_t smem);
 void launch_fill_i64(int64_t *p, int64_t n, int64_t v, cudaStream_t st);
 

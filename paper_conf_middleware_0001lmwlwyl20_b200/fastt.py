@@ -64,7 +64,8 @@ class fastt_timing(C.Structure):
 
 SYMBOLS = ["fastt_load_graph", "fastt_free_graph", "fastt_graph_info", "fastt_rank", "fastt_schedule_batch",
            "fastt_stream_info", "fastt_generate_candidates", "fastt_sweep_best", "fastt_split_search",
-           "fastt_free_split_result", "fastt_last_timing", "fastt_last_error", "fastt_version"]
+           "fastt_free_split_result", "fastt_last_timing", "fastt_last_error", "fastt_version",
+           "fastt_fit_comm", "fastt_link_model"]
 F_TIMING = 16
 F_SPLIT_BEST = 32
 F_MEM_LIVE = 64
@@ -103,6 +104,10 @@ def lib():
     L.fastt_last_timing.argtypes = [P, C.POINTER(fastt_timing)]
     L.fastt_last_error.restype = C.c_char_p
     L.fastt_version.restype = C.c_char_p
+    L.fastt_fit_comm.restype = i32
+    L.fastt_fit_comm.argtypes = [i32, i64, P, P, P, P, C.c_int, C.POINTER(fastt_opts), P, P, P]
+    L.fastt_link_model.restype = i32
+    L.fastt_link_model.argtypes = [i32, P, P, P, P, P, P]
     _lib = L
     return L
 
@@ -313,6 +318,41 @@ class Graph:
         finally:
             lib().fastt_free_split_result(C.byref(r))
         return res
+
+
+def fit_comm(n_devices, src, dst, nbytes, time_ns, device=0, stream=None):
+    """fastt_fit_comm: per ordered device pair the non-negative least-squares
+    line time = alpha + beta * bytes (R26).  Returns (alpha_ns, beta_fs, count)
+    as G x G int64 arrays."""
+    G = int(n_devices)
+    src = np.ascontiguousarray(np.asarray(src, np.uint8))
+    dst = np.ascontiguousarray(np.asarray(dst, np.uint8))
+    nb = np.ascontiguousarray(np.asarray(nbytes, np.int64))
+    tn = np.ascontiguousarray(np.asarray(time_ns, np.int64))
+    n = len(src)
+    if not (len(dst) == len(nb) == len(tn) == n):
+        raise ValueError("sample arrays differ in length")
+    a = np.zeros(G * G, np.int64)
+    b = np.zeros(G * G, np.int64)
+    c = np.zeros(G * G, np.int64)
+    o = _opts(0, stream)
+    _check(lib().fastt_fit_comm(G, n, _ptr(src), _ptr(dst), _ptr(nb), _ptr(tn), int(device), C.byref(o), _ptr(a),
+                                _ptr(b), _ptr(c)))
+    return a.reshape(G, G), b.reshape(G, G), c.reshape(G, G)
+
+
+def link_model(alpha_ns, beta_fs):
+    """fastt_link_model: per-pair parameters -> (link_class[G][G], alpha[K], beta[K])."""
+    a = np.ascontiguousarray(np.asarray(alpha_ns, np.int64))
+    b = np.ascontiguousarray(np.asarray(beta_fs, np.int64))
+    G = a.shape[0]
+    lc = np.zeros((G, G), np.uint8)
+    k = np.zeros(1, np.int32)
+    ka = np.zeros(16, np.int64)
+    kb = np.zeros(16, np.int64)
+    _check(lib().fastt_link_model(G, _ptr(a), _ptr(b), _ptr(lc), _ptr(k), _ptr(ka), _ptr(kb)))
+    K = int(k[0])
+    return lc, ka[:K].copy(), kb[:K].copy()
 
 
 def load_graph(desc, device=0):
