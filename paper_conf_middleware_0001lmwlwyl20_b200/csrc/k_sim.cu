@@ -114,9 +114,6 @@ __device__ __forceinline__ uint64_t splitmix64(uint64_t &s) {
 }
 
 
-#ifndef SIM_PEEK
-#define SIM_PEEK 0
-#endif
 #ifndef SIM_ASM_SMEM
 #define SIM_ASM_SMEM 0
 #endif
@@ -140,7 +137,6 @@ __device__ __forceinline__ uint32_t lds32(uint32_t a) { return *sptr(a); }
 __device__ __forceinline__ void sts32(uint32_t a, uint32_t v) { *sptr(a) = v; }
 __device__ __forceinline__ void red_or_s(uint32_t a, uint32_t v) { atomicOr(sptr(a), v); }
 #endif
-__device__ __forceinline__ void prefetch_l2(const void *p) { asm volatile("prefetch.global.L2 [%0];" ::"l"(p)); }
 
 // R21: the c-th candidate of the sweep stream
 __device__ Cand stream_cand(const StreamState &S, int64_t c) {
@@ -678,18 +674,6 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       if (fastcomm) hc = __ldg((const uint4 *)(cd + CW_PCOMM));
       const T cst = __ldg(costp + (size_t)i * G + (d < G ? d : 0));
       const uint32_t s0 = __ldg(cd + CW_SUCC + (d < S_IN ? d : 0));
-      // peek the next ready op (88% of pops on C5 are the op that was
-      // already next): its card now, its predecessor records prefetched
-      // into L2 at the end of this step
-      uint32_t jn = NONE;
-      if (SIM_PEEK && nlw) jn = ((uint32_t)w << 5) + (__ffs(nlw) - 1);
-      else if (SIM_PEEK && nm) {
-        const int w2 = (s << 5) + __ffs(nm) - 1;
-        const uint32_t l2 = lds32(la + 4u * w2);
-        jn = ((uint32_t)w2 << 5) + (__ffs(l2) - 1);
-      }
-      uint4 hn = make_uint4(0, 0, 0, 0);
-      if (SIM_PEEK && live && jn != NONE) hn = __ldg((const uint4 *)(card + (size_t)jn * CARD_WORDS + CARD_HDR));
       __syncwarp();
       if (live && d == 0) {
         sts32(la + 4u * w, nlw);
@@ -950,13 +934,6 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
 #pragma unroll
       for (int o = GP >> 1; o >= 1; o >>= 1) bits |= __shfl_xor_sync(FULL, bits, o);
       top |= bits;
-      // prefetch the peeked op's predecessor records (lane k of the group takes pred k)
-      if (SIM_PEEK && go && jn != NONE) {
-        const uint32_t npn = hn.x;  // hn = words 8..11 of the peeked card: its predecessor positions
-        (void)npn;
-        const uint32_t ps = d == 0 ? hn.x : d == 1 ? hn.y : d == 2 ? hn.z : hn.w;
-        if (d < 4) prefetch_l2(slab0 + SLOT(ps));
-      }
       __syncwarp();
     }
 
