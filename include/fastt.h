@@ -238,6 +238,8 @@ typedef struct {
   int64_t candidates;   /* candidates evaluated */
   int64_t deferred;     /* of which went through the preparation pipeline */
   float ms_sim, ms_prep, ms_total;
+  int32_t topo;         /* 1: the main simulation ran the position-order kernel (the graph's priority
+                           order is topological, so the dequeue order is the position order) */
 } fastt_timing;
 fastt_status fastt_last_timing(const fastt_graph *g, fastt_timing *out);
 

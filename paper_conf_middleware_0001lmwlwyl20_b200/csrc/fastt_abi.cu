@@ -181,6 +181,7 @@ struct Base {
   char *prep_block = nullptr;
   PrepGraph *pg_dev = nullptr;
   int tbits = 64, key_bits = 64;
+  int topo = 0;  // the prepared priority order is topological (k_sim's TOPO path)
   unsigned long long bound = 0, maxextra = 0;
   // recorded BASE schedule for prefix sharing, per CP-pin flag value
   struct Snap {
@@ -246,6 +247,9 @@ struct fastt_graph {
   int64_t *slot_result = nullptr, *slot_index = nullptr;
   // simulation workspace
   int sms = 148, sim_block = SIM_BLOCK, sim_grid = 0, sim_tbits = 0, sim_cpw = 1, sim_bm_stride = 0;
+  int sim_grid_topo = 0;  // resident blocks of the TOPO variant (no shared-memory ready set)
+  bool use_topo = true;   // FASTT_NO_TOPO=1 forces the ready-set path (A/B parity)
+  int last_topo = 0;      // the last main launch ran the TOPO variant
   int64_t sim_ncap = 0;
   size_t sim_smem = 0;
   void *slab = nullptr;
@@ -292,6 +296,7 @@ static fastt_status timing_end(fastt_graph *g, uint32_t flags, cudaStream_t st, 
   g->last.launches = g->launches;
   g->last.candidates = cands;
   g->last.deferred = deferred;
+  g->last.topo = g->last_topo;
   if (!(flags & FASTT_F_TIMING)) return FASTT_OK;
   CK(cudaEventRecord(g->ev[3], st));
   CK(cudaEventSynchronize(g->ev[3]));
@@ -371,6 +376,7 @@ static fastt_status prepare_base(fastt_graph *g, Base &B, cudaStream_t st) {
   CK(cudaStreamSynchronize(st));
   B.n = P.n;
   B.cp_len = P.cp_len;
+  B.topo = P.topo;
   return FASTT_OK;
 }
 
@@ -444,13 +450,14 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     while (stride % 32 != 8) stride++;  // candidates of one warp start on different banks
     size_t smem = (size_t)(g->sim_block / 32) * cpw * stride * 4;
     if (smem > 48 * 1024) CK(sim_set_smem(B.tbits, gsh, smem));
-    int per_sm = sim_occupancy(B.tbits, gsh, g->sim_block, smem);
+    int per_sm = sim_occupancy(B.tbits, gsh, g->sim_block, smem, false);
     if (per_sm < 1) return fail(FASTT_EUNSUP, "simulation kernel does not fit on an SM (smem %zu)", smem);
     g->sim_grid = g->sms * per_sm;
+    g->sim_grid_topo = g->sms * std::max(1, sim_occupancy(B.tbits, gsh, g->sim_block, 0, true));
     g->sim_smem = smem;
     g->sim_cpw = cpw;
     g->sim_bm_stride = stride;
-    int64_t nslot = (int64_t)g->sim_grid * (g->sim_block / 32) * cpw;
+    int64_t nslot = (int64_t)std::max(g->sim_grid, g->sim_grid_topo) * (g->sim_block / 32) * cpw;
     size_t rec = B.tbits == 32 ? 8 : 16;
     CK(cudaMalloc(&g->slab, (size_t)nslot * ncap * rec));
     CK(cudaMalloc(&g->wbest, sizeof(int64_t) * 2 * nslot));
@@ -466,7 +473,7 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     const size_t per_block = (size_t)(g->sim_block / 32) * g->sim_cpw * g->G * g->gap_stride * rec;
     size_t fr = 0, tot = 0;
     CK(cudaMemGetInfo(&fr, &tot));
-    int64_t ig = std::min<int64_t>(g->sim_grid, (int64_t)(fr / 3 / per_block));
+    int64_t ig = std::min<int64_t>(std::max(g->sim_grid, g->sim_grid_topo), (int64_t)(fr / 3 / per_block));
     if (ig > g->sms) ig -= ig % g->sms;
     if (ig < 1) return fail(FASTT_ENOMEM, "INSERT idle-slot arrays (%zu bytes per block)", per_block);
     if (cudaMalloc(&g->gap, (size_t)ig * per_block) != cudaSuccess) {
@@ -487,6 +494,26 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     g->defer_cap = cap;
   }
   return FASTT_OK;
+}
+
+// The launch shape of a base-graph simulation: the TOPO variant (no ready
+// set, no shared memory, more resident blocks) when the base's priority order
+// is topological, else the ready-set variant.  Slot launches (mode 2) use
+// the ready-set variant (slots may differ).
+static void main_shape(fastt_graph *g, const Base &B, SimArgs &a, int &grid, size_t &smem) {
+  g->last_topo = g->use_topo && B.topo && a.mode != 2;
+  if (g->last_topo) {
+    a.topo = 1;
+    grid = g->sim_grid_topo;
+    smem = 0;
+  } else {
+    a.topo = 0;
+    grid = g->sim_grid;
+    smem = g->sim_smem;
+  }
+}
+static int max_slots(const fastt_graph *g) {
+  return std::max(g->sim_grid, g->sim_grid_topo) * (g->sim_block / 32) * g->sim_cpw;
 }
 
 static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
@@ -585,7 +612,12 @@ static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cud
   a.snap_ms = S.ms;
   a.snap_rec = S.rec;
   a.snap_rounds = S.rounds;
-  launch_sim(a, B.tbits, 1, g->sim_block, g->sim_smem, st);
+  {
+    int grid;
+    size_t smem;
+    main_shape(g, B, a, grid, smem);
+    launch_sim(a, B.tbits, 1, g->sim_block, smem, st);
+  }
   g->launches += NL_SIM;
   CK(cudaGetLastError());
   int32_t rd[4];
@@ -686,7 +718,12 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
     a.slot_index = g->srt_i;
     a.slot_result = g->srt_res;
   }
-  launch_sim(a, B.tbits, g->sim_grid, g->sim_block, g->sim_smem, st);
+  {
+    int grid;
+    size_t smem;
+    main_shape(g, B, a, grid, smem);
+    launch_sim(a, B.tbits, grid, g->sim_block, smem, st);
+  }
   g->launches += NL_SIM;
   CK(cudaGetLastError());
   timing_mark(g, flags, 1, st);
@@ -706,6 +743,7 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
       SimArgs b = a;
       b.slots = g->slot_pgs_dev;
       b.mode = 2;
+      b.topo = 0;
       b.cands = g->slot_cands;
       b.slot_result = g->slot_result;
       b.slot_index = nullptr;
@@ -1050,6 +1088,8 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
   {
     const char *e = getenv("FASTT_NO_SHARE");
     g->share = !(e && e[0] == '1');
+    e = getenv("FASTT_NO_TOPO");
+    g->use_topo = !(e && e[0] == '1');
   }
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || cuda_device < 0 || cuda_device >= ndev) {
@@ -1343,7 +1383,7 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
   TRY(check_gen(g, *S, gen, first, n, stride));
   Base &B = g->base;
   TRY(ensure_sim(g, B, n, flags));
-  const int64_t nwarps = (int64_t)g->sim_grid * (g->sim_block / 32) * g->sim_cpw;  // candidate slots
+  const int64_t nwarps = max_slots(g);  // candidate slots
   {
     std::vector<int64_t> init(2 * nwarps);
     for (int64_t w = 0; w < nwarps; w++) {
@@ -1376,7 +1416,12 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
       a.slot_index = g->srt_i;
       a.slot_result = nullptr;
     }
-    launch_sim(a, B.tbits, g->sim_grid, g->sim_block, g->sim_smem, st);
+    {
+      int grid;
+      size_t smem;
+      main_shape(g, B, a, grid, smem);
+      launch_sim(a, B.tbits, grid, g->sim_block, smem, st);
+    }
     g->launches += NL_SIM;
     CK(cudaGetLastError());
     timing_mark(g, flags, 1, st);
@@ -1395,6 +1440,7 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
         SimArgs b = a;
         b.slots = g->slot_pgs_dev;
         b.mode = 2;
+        b.topo = 0;
         b.cands = g->slot_cands;
         b.slot_result = nullptr;
         b.slot_index = g->slot_index;

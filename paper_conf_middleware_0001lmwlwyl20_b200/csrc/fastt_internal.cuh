@@ -23,6 +23,9 @@
 #ifndef SIM_MINB
 #define SIM_MINB 5
 #endif
+#ifndef SIM_MINB_TOPO
+#define SIM_MINB_TOPO 7
+#endif
 
 namespace fastt {
 
@@ -83,6 +86,7 @@ struct PrepGraph {
   int64_t E;        // live edges
   int32_t cp_len;   // written by the CP kernel
   int32_t tbits;    // 32 or 64
+  int32_t topo;     // 1 iff every edge goes from a lower to a higher position (set by the card kernels)
   uint32_t *card;   // n * CARD_WORDS
   void *costp;      // n * G of T
   uint32_t *pe_src; // E: predecessor position, grouped by consumer position
@@ -192,6 +196,7 @@ struct SimArgs {
   int32_t need_mem;      // track per-device memory (caps present or peak output)
   int32_t live_mem;      // liveness memory (R24, FASTT_F_MEM_LIVE); implies need_mem
   int32_t fastcomm;      // uint32 time and one link class: comm values inline in the cards
+  int32_t topo;          // the graph's priority order is topological: dequeue order = position order
   int32_t cap_check;     // some device has a finite memory cap (R8)
   // BASE-schedule prefix sharing: 1 = record the snapshot (one BASE run),
   // 2 = start eligible PIN candidates from it at their first pinned op
@@ -233,7 +238,7 @@ void launch_t0_sort(int from_stream, const StreamState &S, int64_t first, int64_
                     cudaStream_t st);
 void launch_gather_sorted(const Cand *src, const int64_t *sidx, const int64_t *sres, const int64_t *qs, int64_t n,
                           Cand *dst, int64_t *didx, int64_t *dres, cudaStream_t st);
-int sim_occupancy(int tbits, int gshift, int block, size_t smem);
+int sim_occupancy(int tbits, int gshift, int block, size_t smem, bool topo);
 void launch_fit(int G, int64_t n, const uint8_t *src, const uint8_t *dst, const int64_t *bytes, const int64_t *tns,
                 void *sums, unsigned *err, int64_t *alpha, int64_t *beta, int64_t *count, int sms, cudaStream_t st);
 size_t fit_sums_bytes(int G);

@@ -545,6 +545,7 @@ __global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, Prep
   const int32_t n = P.n;
   uint32_t runp = 0, runs = 0;
   for (int32_t w = threadIdx.x; w < (n + 31) / 32; w += blockDim.x) P.srcbits[w] = 0;
+  if (threadIdx.x == 0) P.topo = 1;  // cleared by k_cards_edges on a backward edge
   __syncthreads();
   for (int32_t t0 = 0; t0 < n; t0 += blockDim.x) {
     int32_t p = t0 + threadIdx.x;
@@ -612,6 +613,7 @@ __global__ void k_cards_edges(const RawGraph *raws, PrepGraph *pgs, const GraphC
       int64_t b = R.pred_bytes[po + j];
       uint32_t sp = P.pos[s];
       P.pe_src[pb + j] = sp;
+      if (sp >= (uint32_t)p) P.topo = 0;  // the priority order is not topological
       for (int k = 0; k < K; k++) pec[(int64_t)(pb + j) * K + k] = (T)comm_class(gc, b, k);
       if (j < P_IN) {
         c[CARD_HDR + j] = sp;

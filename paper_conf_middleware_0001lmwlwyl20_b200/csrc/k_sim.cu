@@ -383,8 +383,15 @@ __device__ __noinline__ void cp_rounds_g(const PrepGraph *pg, int np, const uint
 // INS: insertion policy (R1i) -- lane d keeps device d's idle slots.
 // FC: uint32 time and one link class -- predecessor comm values come from
 // the op's card (no per-edge comm loads).
-template <typename T, int GSH, bool MEM, bool INS, bool FC>
-__global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
+// TOPO: the priority order of the prepared graph is a topological order
+// (PrepGraph::topo), so the dequeue order is the position order: the
+// highest-priority op not yet dequeued has all its predecessors at higher
+// priority, hence already dequeued, hence it is ready and it is the one
+// popped (by induction every step pops the next position).  No ready set,
+// no indegrees, no successor release; with prefix sharing the records of
+// positions before t0 are read from the recorded BASE schedule in place.
+template <typename T, int GSH, bool MEM, bool INS, bool FC, bool TOPO>
+__global__ void __launch_bounds__(SIM_BLOCK, TOPO ? SIM_MINB_TOPO : SIM_MINB) k_sim(SimArgs a) {
   typedef typename Slab<T>::W W;
   constexpr int GP = 1 << GSH;   // lanes per candidate (>= G)
   constexpr int CPW = 32 >> GSH; // candidates per warp
@@ -578,7 +585,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
     if (run && share) {
       avail = d < G ? __ldg((const T *)a.snap_avail + (size_t)t0 * G + d) : (T)0;
       makespan = __ldg((const T *)a.snap_ms + t0);
-      if (t0 < n) {
+      if (!TOPO && t0 < n) {
         const int32_t nwords = (n + 31) >> 5;
         for (int32_t w = d; w < nwords; w += GP) leaf[w] = 0;
         __syncwarp(gm);
@@ -619,7 +626,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
         for (int o = GP >> 1; o >= 1; o >>= 1) tb |= __shfl_xor_sync(gm, tb, o);
         top = tb;
       }
-    } else if (run) {
+    } else if (run && !TOPO) {
       const int32_t nwords = (n + 31) >> 5;
       for (int32_t w = d; w < nwords; w += GP) leaf[w] = __ldg(pg->srcbits + w);
       for (int32_t s = d; s < 32; s += GP) summ[s] = __ldg(pg->srcsumm + s);
@@ -647,23 +654,42 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
     const bool any_out = __any_sync(FULL, want_out);
     const int64_t ob = want_out ? res_idx * (int64_t)a.out.vmax : 0;
     const bool snap_rec_on = a.snap_mode == 1;
+    // step counter; under TOPO also the position processed (each group from its t0)
     int32_t tstep = 0;
+    if (TOPO) {
+      int32_t lo = run ? t0 : 0x7FFFFFFF;
+#pragma unroll
+      for (int o = 16; o >= 1; o >>= 1) {
+        const int32_t x = __shfl_xor_sync(FULL, lo, o);
+        lo = x < lo ? x : lo;
+      }
+      tstep = lo;
+    }
 
     // ---------------------------------------------------------- main loop
     int32_t seq = 0;
     bool infeas = false;
     const uint32_t la = leaf_sa, sa = summ_sa;  // shared-memory byte addresses
-    while (__any_sync(FULL, top != 0)) {
-      const bool live = top != 0;
-      // pop: highest priority = lowest position = lowest set bit
-      const int s = live ? __ffs(top) - 1 : 0;
-      const uint32_t m = lds32(sa + 4u * s);
-      const int b = m ? __ffs(m) - 1 : 0;
-      const int w = (s << 5) + b;
-      const uint32_t lw = lds32(la + 4u * w);
-      const uint32_t i = live ? ((uint32_t)w << 5) + (__ffs(lw) - 1) : 0u;
-      const uint32_t nlw = lw & (lw - 1);
-      const uint32_t nm = nlw ? m : (m & (m - 1));
+    while (TOPO ? __any_sync(FULL, run && !infeas && tstep < n) : __any_sync(FULL, top != 0)) {
+      bool live;
+      uint32_t i;
+      int s = 0, w = 0;
+      uint32_t nlw = 0, nm = 0;
+      if constexpr (TOPO) {
+        live = run && !infeas && tstep >= t0 && tstep < n;
+        i = live ? (uint32_t)tstep : 0u;
+      } else {
+        live = top != 0;
+        // pop: highest priority = lowest position = lowest set bit
+        s = live ? __ffs(top) - 1 : 0;
+        const uint32_t m = lds32(sa + 4u * s);
+        const int b = m ? __ffs(m) - 1 : 0;
+        w = (s << 5) + b;
+        const uint32_t lw = lds32(la + 4u * w);
+        i = live ? ((uint32_t)w << 5) + (__ffs(lw) - 1) : 0u;
+        nlw = lw & (lw - 1);
+        nm = nlw ? m : (m & (m - 1));
+      }
 
       // round 1 (all from the op's card line): header, predecessor
       // positions and comm, this lane's successor, cost on this lane's device
@@ -673,13 +699,15 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       uint4 hc = make_uint4(0, 0, 0, 0);
       if (fastcomm) hc = __ldg((const uint4 *)(cd + CW_PCOMM));
       const T cst = __ldg(costp + (size_t)i * G + (d < G ? d : 0));
-      const uint32_t s0 = __ldg(cd + CW_SUCC + (d < S_IN ? d : 0));
+      const uint32_t s0 = TOPO ? 0u : __ldg(cd + CW_SUCC + (d < S_IN ? d : 0));
       __syncwarp();
-      if (live && d == 0) {
-        sts32(la + 4u * w, nlw);
-        sts32(sa + 4u * s, nm);
+      if constexpr (!TOPO) {
+        if (live && d == 0) {
+          sts32(la + 4u * w, nlw);
+          sts32(sa + 4u * s, nm);
+        }
+        if (live && !nm) top &= top - 1;
       }
-      if (live && !nm) top &= top - 1;
       const uint32_t npred = live ? (h0.x & 0xFFFF) : 0u;
       const uint32_t nsucc = live ? (h0.x >> 16) : 0u;
       // round 2: predecessor records, successor indegree
@@ -692,8 +720,12 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       // issue back to back instead of one dependent round trip each
       W rw[4];
 #pragma unroll
-      for (int k = 0; k < 4; k++) rw[k] = slab0[SLOT(src[k])];
-      const uint32_t sdeg_raw = Slab<T>::indeg(slab0, SLOT(s0));
+      for (int k = 0; k < 4; k++) {
+        // TOPO + sharing: positions before t0 hold the BASE records (read in place)
+        const W *ad = (TOPO && share && (int32_t)src[k] < t0) ? (const W *)a.snap_rec + src[k] : slab0 + SLOT(src[k]);
+        rw[k] = *ad;
+      }
+      const uint32_t sdeg_raw = TOPO ? 1u : Slab<T>::indeg(slab0, SLOT(s0));
 #pragma unroll
       for (int k = 0; k < 4; k++) {
         T f;
@@ -722,7 +754,9 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
           if (k < npred) {
             T f;
             uint32_t p;
-            Slab<T>::load(slab0, SLOT(__ldg(pe_src + h0.y + k)), f, p);
+            const uint32_t q = __ldg(pe_src + h0.y + k);
+            const W wq = (TOPO && share && (int32_t)q < t0) ? ((const W *)a.snap_rec)[q] : slab0[SLOT(q)];
+            Slab<T>::decode(wq, f, p);
             T cm = 0;
             if (p != (uint32_t)d && d < G)
               cm = K == 1 ? __ldg(pe_comm + h0.y + k) : __ldg(pe_comm + (size_t)(h0.y + k) * K + gc.link_class[p * G + d]);
@@ -806,7 +840,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
       const unsigned fm = __ballot_sync(FULL, feas && key == mn) & gm;
       if (live && !fm) {
         infeas = true;
-        top = 0;
+        if (!TOPO) top = 0;
       }
       const bool go = live && fm != 0;
       const int dsel = fm ? __ffs(fm) - 1 - gb : 0;
@@ -906,6 +940,10 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
         }
         seq++;
       }
+      if constexpr (TOPO) {
+        __syncwarp();
+        continue;
+      }
       // release successors into the ready bitmap
       uint32_t bits = 0;
       if (go && (uint32_t)d < nsucc) {
@@ -974,46 +1012,51 @@ __global__ void __launch_bounds__(SIM_BLOCK, SIM_MINB) k_sim(SimArgs a) {
   }
 }
 
-template <typename T, bool MEM, bool INS, bool FC>
+template <typename T, bool MEM, bool INS, bool FC, bool TOPO>
 static const void *sim_fn_t(int gshift) {
   switch (gshift) {
-    case 0: return (const void *)k_sim<T, 0, MEM, INS, FC>;
-    case 1: return (const void *)k_sim<T, 1, MEM, INS, FC>;
-    case 2: return (const void *)k_sim<T, 2, MEM, INS, FC>;
-    case 3: return (const void *)k_sim<T, 3, MEM, INS, FC>;
-    case 4: return (const void *)k_sim<T, 4, MEM, INS, FC>;
-    default: return (const void *)k_sim<T, 5, MEM, INS, FC>;
+    case 0: return (const void *)k_sim<T, 0, MEM, INS, FC, TOPO>;
+    case 1: return (const void *)k_sim<T, 1, MEM, INS, FC, TOPO>;
+    case 2: return (const void *)k_sim<T, 2, MEM, INS, FC, TOPO>;
+    case 3: return (const void *)k_sim<T, 3, MEM, INS, FC, TOPO>;
+    case 4: return (const void *)k_sim<T, 4, MEM, INS, FC, TOPO>;
+    default: return (const void *)k_sim<T, 5, MEM, INS, FC, TOPO>;
   }
 }
-template <typename T, bool FC>
+template <typename T, bool FC, bool TOPO>
 static const void *sim_fn_m(int gshift, bool mem, bool ins) {
-  if (ins) return mem ? sim_fn_t<T, true, true, FC>(gshift) : sim_fn_t<T, false, true, FC>(gshift);
-  return mem ? sim_fn_t<T, true, false, FC>(gshift) : sim_fn_t<T, false, false, FC>(gshift);
+  if (ins) return mem ? sim_fn_t<T, true, true, FC, TOPO>(gshift) : sim_fn_t<T, false, true, FC, TOPO>(gshift);
+  return mem ? sim_fn_t<T, true, false, FC, TOPO>(gshift) : sim_fn_t<T, false, false, FC, TOPO>(gshift);
 }
-static const void *sim_fn(int tbits, int gshift, bool mem, bool ins = false, bool fc = false) {
-  if (tbits != 32) return sim_fn_m<uint64_t, false>(gshift, mem, ins);
-  return fc ? sim_fn_m<uint32_t, true>(gshift, mem, ins) : sim_fn_m<uint32_t, false>(gshift, mem, ins);
+template <bool TOPO>
+static const void *sim_fn_k(int tbits, int gshift, bool mem, bool ins, bool fc) {
+  if (tbits != 32) return sim_fn_m<uint64_t, false, TOPO>(gshift, mem, ins);
+  return fc ? sim_fn_m<uint32_t, true, TOPO>(gshift, mem, ins) : sim_fn_m<uint32_t, false, TOPO>(gshift, mem, ins);
+}
+static const void *sim_fn(int tbits, int gshift, bool mem, bool ins = false, bool fc = false, bool topo = false) {
+  return topo ? sim_fn_k<true>(tbits, gshift, mem, ins, fc) : sim_fn_k<false>(tbits, gshift, mem, ins, fc);
 }
 
 void launch_sim(const SimArgs &a, int tbits, int grid, int block, size_t smem, cudaStream_t st) {
   if (a.ins && grid > a.ins_grid) grid = a.ins_grid;  // INSERT slot arrays exist for ins_grid blocks
-  const void *f = sim_fn(tbits, a.gshift, a.need_mem != 0, a.ins != 0, a.fastcomm != 0);
+  const void *f = sim_fn(tbits, a.gshift, a.need_mem != 0, a.ins != 0, a.fastcomm != 0, a.topo != 0);
   SimArgs aa = a;
   void *args[] = {&aa};
   cudaLaunchKernel(f, dim3(grid), dim3(block), args, smem, st);
 }
 
-int sim_occupancy(int tbits, int gshift, int block, size_t smem) {
+int sim_occupancy(int tbits, int gshift, int block, size_t smem, bool topo) {
   int nb = 1 << 30, x = 0;
-  for (int v = 0; v < 4; v++) {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, sim_fn(tbits, gshift, v & 1, false, v >> 1), block, smem);
+  for (int v = 0; v < 8; v++) {
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, sim_fn(tbits, gshift, v & 1, (v >> 2) & 1, (v >> 1) & 1, topo),
+                                                  block, smem);
     nb = x < nb ? x : nb;
   }
   return nb;
 }
 cudaError_t sim_set_smem(int tbits, int gshift, size_t smem) {
   for (int v = 0; v < 8; v++) {
-    cudaError_t e = cudaFuncSetAttribute(sim_fn(tbits, gshift, v & 1, (v >> 1) & 1, v >> 2),
+    cudaError_t e = cudaFuncSetAttribute(sim_fn(tbits, gshift, v & 1, (v >> 1) & 1, v >> 2, false),
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
   }

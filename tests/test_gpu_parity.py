@@ -442,3 +442,56 @@ def test_insert_split_search(seed):
         b = og.split_search(flags=INS | F.F_CP_PIN, best_improvement=best)
         assert a["sp"] == b["sp"] and a["makespan"] == b["makespan"]
         assert (a["placement"] == b["placement"]).all() and (a["start"] == b["start"]).all()
+
+
+# ------------------------------------------------- TOPO path (dequeue = position order)
+
+def _graph(desc, no_topo):
+    old = os.environ.get("FASTT_NO_TOPO")
+    os.environ["FASTT_NO_TOPO"] = "1" if no_topo else "0"
+    try:
+        return F.Graph(desc)
+    finally:
+        if old is None:
+            del os.environ["FASTT_NO_TOPO"]
+        else:
+            os.environ["FASTT_NO_TOPO"] = old
+
+
+@pytest.mark.parametrize("name", ["C2", "C3", "C4", "C5"])
+def test_topo_path_used_and_equal_to_ready_set_path(name):
+    """The paper-shaped configs have c_ij > 0 on every edge (alpha > 0), so
+    ranks fall strictly along edges and the priority order is topological:
+    the sweep runs the TOPO kernel.  Its per-candidate results equal the
+    ready-set kernel's (FASTT_NO_TOPO=1) and the oracle's on a sample."""
+    desc = synth.config(name)
+    pow2 = name == "C4"
+    gen = F.gen_params(seed=0xFA57, n_pow2_only=pow2)
+    a, b = _graph(desc, False), _graph(desc, True)
+    ns = a.stream_info(gen, flags=F.F_CP_PIN)
+    n = 3000 if name == "C5" else 6000
+    first = ns + 1
+    ca = a.generate_candidates(gen, first, n, flags=F.F_CP_PIN)
+    ra = a.schedule_batch(ca, flags=F.F_CP_PIN, peak=False)
+    assert a.last_timing()["topo"] == 1
+    rb = b.schedule_batch(ca, flags=F.F_CP_PIN, peak=False)
+    assert b.last_timing()["topo"] == 0
+    assert (ra["makespan"] == rb["makespan"]).all() and (ra["status"] == rb["status"]).all()
+    assert a.sweep_best(gen, 0, ns + 1 + n, flags=F.F_CP_PIN) == b.sweep_best(gen, 0, ns + 1 + n, flags=F.F_CP_PIN)
+    og = O.OracleGraph(desc)
+    for k in range(0, n, n // 12):
+        assert int(ra["makespan"][k]) == og.schedule(ca[k], flags=O.F_CP_PIN)["makespan"]
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_topo_vs_ready_set_random(seed):
+    """Random DAGs (some with alpha = 0 classes and zero costs, where the
+    priority order is not topological and the ready-set kernel must run):
+    both paths agree with the oracle on every output."""
+    desc = synth.random_dag(seed + 6000)
+    rng = np.random.default_rng(seed)
+    cands = random_cands(desc, rng, 30)
+    og = O.OracleGraph(desc)
+    for g in (_graph(desc, False), _graph(desc, True)):
+        for flags in (0, F.F_CP_PIN):
+            compare(desc, cands, flags, gg=g, og=og)
