@@ -238,8 +238,10 @@ typedef struct {
   int64_t candidates;   /* candidates evaluated */
   int64_t deferred;     /* of which went through the preparation pipeline */
   float ms_sim, ms_prep, ms_total;
-  int32_t topo;         /* 1: the main simulation ran the position-order kernel (the graph's priority
-                           order is topological, so the dequeue order is the position order) */
+  int32_t topo;         /* 1 or 2: the main simulation ran a position-order kernel (the graph's priority
+                           order is topological, so the dequeue order is the position order):
+                           1 = one lane group per candidate (k_sim), 2 = one lane per candidate
+                           (k_sim_lane: makespan-only evaluation without memory tracking) */
 } fastt_timing;
 fastt_status fastt_last_timing(const fastt_graph *g, fastt_timing *out);
 

@@ -10,14 +10,14 @@ from concurrent.futures import ThreadPoolExecutor
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
-SRCS = [os.path.join(HERE, "csrc", f) for f in ("fastt_abi.cu", "k_prep.cu", "k_sim.cu", "k_fit.cu")]
-DEPS = SRCS + [os.path.join(HERE, "csrc", "fastt_internal.cuh"), os.path.join(ROOT, "include", "fastt.h")]
+SRCS = [os.path.join(HERE, "csrc", f) for f in ("fastt_abi.cu", "k_prep.cu", "k_sim.cu", "k_sim_lane.cu", "k_fit.cu")]
+DEPS = SRCS + [os.path.join(HERE, "csrc", "fastt_internal.cuh"), os.path.join(HERE, "csrc", "sim_common.cuh"), os.path.join(ROOT, "include", "fastt.h")]
 OUT = os.path.join(HERE, "libfastt.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 CFLAGS = ARCH + ["-lineinfo", "-O3", "-std=c++17", "-Xcompiler", "-fPIC", "-I" + os.path.join(ROOT, "include")]
 # launch-shape overrides for tuning experiments (defaults live in fastt_internal.cuh)
-CFLAGS += ["-D%s=%s" % (k, os.environ[k]) for k in ("SIM_MINB", "SIM_MINB_TOPO", "SIM_BLOCK") if os.environ.get(k)]
+CFLAGS += ["-D%s=%s" % (k, os.environ[k]) for k in ("SIM_MINB", "SIM_MINB_TOPO", "SIM_BLOCK", "LANE_MINB", "LANE_BLOCK") if os.environ.get(k)]
 FLAGS = CFLAGS + ["-shared"]  # (single-command form, kept for tools)
 
 

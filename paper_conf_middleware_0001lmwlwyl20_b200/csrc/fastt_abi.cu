@@ -249,7 +249,9 @@ struct fastt_graph {
   int sms = 148, sim_block = SIM_BLOCK, sim_grid = 0, sim_tbits = 0, sim_cpw = 1, sim_bm_stride = 0;
   int sim_grid_topo = 0;  // resident blocks of the TOPO variant (no shared-memory ready set)
   bool use_topo = true;   // FASTT_NO_TOPO=1 forces the ready-set path (A/B parity)
-  int last_topo = 0;      // the last main launch ran the TOPO variant
+  int sim_grid_lane = 0;  // resident blocks of the lane-per-candidate position-order kernel
+  bool use_lane = true;   // FASTT_NO_LANE=1 keeps position-order launches on the group kernel (A/B parity)
+  int last_topo = 0;      // the last main launch: 0 ready-set kernel, 1 group position-order, 2 lane position-order
   int64_t sim_ncap = 0;
   size_t sim_smem = 0;
   void *slab = nullptr;
@@ -454,10 +456,12 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     if (per_sm < 1) return fail(FASTT_EUNSUP, "simulation kernel does not fit on an SM (smem %zu)", smem);
     g->sim_grid = g->sms * per_sm;
     g->sim_grid_topo = g->sms * std::max(1, sim_occupancy(B.tbits, gsh, g->sim_block, 0, true));
+    g->sim_grid_lane = g->sms * std::max(1, lane_occupancy(B.tbits, gsh));
     g->sim_smem = smem;
     g->sim_cpw = cpw;
     g->sim_bm_stride = stride;
     int64_t nslot = (int64_t)std::max(g->sim_grid, g->sim_grid_topo) * (g->sim_block / 32) * cpw;
+    nslot = std::max<int64_t>(nslot, (int64_t)g->sim_grid_lane * LANE_BLOCK);  // one column per lane
     size_t rec = B.tbits == 32 ? 8 : 16;
     CK(cudaMalloc(&g->slab, (size_t)nslot * ncap * rec));
     CK(cudaMalloc(&g->wbest, sizeof(int64_t) * 2 * nslot));
@@ -501,8 +505,17 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
 // is topological, else the ready-set variant.  Slot launches (mode 2) use
 // the ready-set variant (slots may differ).
 static void main_shape(fastt_graph *g, const Base &B, SimArgs &a, int &grid, size_t &smem) {
-  g->last_topo = g->use_topo && B.topo && a.mode != 2;
-  if (g->last_topo) {
+  const bool topo = g->use_topo && B.topo && a.mode != 2;
+  // the lane kernel covers makespan-only evaluation without memory tracking
+  const bool lane = topo && g->use_lane && !a.need_mem && !a.ins && !a.out.place && !a.out.start && !a.out.deq &&
+                    !a.out.peak && a.snap_mode != 1;
+  g->last_topo = lane ? 2 : topo ? 1 : 0;
+  a.lane = lane;
+  if (lane) {
+    a.topo = 1;
+    grid = g->sim_grid_lane;
+    smem = 0;
+  } else if (topo) {
     a.topo = 1;
     grid = g->sim_grid_topo;
     smem = 0;
@@ -513,7 +526,8 @@ static void main_shape(fastt_graph *g, const Base &B, SimArgs &a, int &grid, siz
   }
 }
 static int max_slots(const fastt_graph *g) {
-  return std::max(g->sim_grid, g->sim_grid_topo) * (g->sim_block / 32) * g->sim_cpw;
+  return std::max(std::max(g->sim_grid, g->sim_grid_topo) * (g->sim_block / 32) * g->sim_cpw,
+                  g->sim_grid_lane * (LANE_BLOCK / 32));
 }
 
 static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
@@ -533,6 +547,7 @@ static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
   a.leaf_words = (int32_t)((g->sim_ncap + 31) / 32);
   a.bm_stride = g->sim_bm_stride;
   a.G = g->G;
+  a.gc_K = g->K;
   while ((1 << a.gshift) < g->G) a.gshift++;
   for (int d = 0; d < g->G; d++)
     if (g->gch.cap[d] != I64MAX) a.cap_check = 1;
@@ -744,6 +759,7 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
       b.slots = g->slot_pgs_dev;
       b.mode = 2;
       b.topo = 0;
+      b.lane = 0;
       b.cands = g->slot_cands;
       b.slot_result = g->slot_result;
       b.slot_index = nullptr;
@@ -1090,6 +1106,8 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     g->share = !(e && e[0] == '1');
     e = getenv("FASTT_NO_TOPO");
     g->use_topo = !(e && e[0] == '1');
+    e = getenv("FASTT_NO_LANE");
+    g->use_lane = !(e && e[0] == '1');
   }
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || cuda_device < 0 || cuda_device >= ndev) {
@@ -1441,6 +1459,7 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
         b.slots = g->slot_pgs_dev;
         b.mode = 2;
         b.topo = 0;
+        b.lane = 0;
         b.cands = g->slot_cands;
         b.slot_result = nullptr;
         b.slot_index = g->slot_index;

@@ -26,6 +26,13 @@
 #ifndef SIM_MINB_TOPO
 #define SIM_MINB_TOPO 7
 #endif
+// lane-per-candidate position-order kernel (k_sim_lane.cu)
+#ifndef LANE_BLOCK
+#define LANE_BLOCK 128
+#endif
+#ifndef LANE_MINB
+#define LANE_MINB 4
+#endif
 
 namespace fastt {
 
@@ -197,6 +204,8 @@ struct SimArgs {
   int32_t live_mem;      // liveness memory (R24, FASTT_F_MEM_LIVE); implies need_mem
   int32_t fastcomm;      // uint32 time and one link class: comm values inline in the cards
   int32_t topo;          // the graph's priority order is topological: dequeue order = position order
+  int32_t lane;          // run the lane-per-candidate position-order kernel (k_sim_lane)
+  int32_t gc_K;          // link classes (host copy of GraphConst::K)
   int32_t cap_check;     // some device has a finite memory cap (R8)
   // BASE-schedule prefix sharing: 1 = record the snapshot (one BASE run),
   // 2 = start eligible PIN candidates from it at their first pinned op
@@ -239,6 +248,8 @@ void launch_t0_sort(int from_stream, const StreamState &S, int64_t first, int64_
 void launch_gather_sorted(const Cand *src, const int64_t *sidx, const int64_t *sres, const int64_t *qs, int64_t n,
                           Cand *dst, int64_t *didx, int64_t *dres, cudaStream_t st);
 int sim_occupancy(int tbits, int gshift, int block, size_t smem, bool topo);
+void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st);
+int lane_occupancy(int tbits, int gshift);
 void launch_fit(int G, int64_t n, const uint8_t *src, const uint8_t *dst, const int64_t *bytes, const int64_t *tns,
                 void *sums, unsigned *err, int64_t *alpha, int64_t *beta, int64_t *count, int sms, cudaStream_t st);
 size_t fit_sums_bytes(int G);

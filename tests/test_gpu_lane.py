@@ -1,0 +1,166 @@
+"""GPU parity of the lane-per-candidate position-order kernel (k_sim_lane.cu):
+bit-exact against the CPU oracle and against the group-per-candidate kernels
+(FASTT_NO_LANE=1 / FASTT_NO_TOPO=1 A/B), on graphs whose priority order is
+topological (all op costs > 0, so rank_u strictly decreases along edges, R2).
+
+Coverage: device counts 1..32 (every lane-group width), one and several link
+classes (the single-class arrival shortcut and the per-pair path), 32- and
+64-bit time, hetero costs (CP devices that move when CP ops are pinned, so
+prefix sharing is refused), sweeps against the group kernel."""
+import dataclasses
+import os
+
+import numpy as np
+import pytest
+
+import oracle as O
+from paper_conf_middleware_0001lmwlwyl20_b200 import synth
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("no CUDA device", allow_module_level=True)
+
+from paper_conf_middleware_0001lmwlwyl20_b200 import build as B  # noqa: E402
+
+B.build()
+from paper_conf_middleware_0001lmwlwyl20_b200 import fastt as F  # noqa: E402
+
+LANE, GROUP = 2, 1
+
+
+def _graph_env(desc, **env):
+    old = {k: os.environ.get(k) for k in env}
+    os.environ.update(env)
+    try:
+        return F.Graph(desc)
+    finally:
+        for k, v in old.items():
+            if v is None:
+                del os.environ[k]
+            else:
+                os.environ[k] = v
+
+
+def topo_dag(seed, V, G, K=1, homogeneous=False, scale=1):
+    """random DAG with every op cost > 0 (topological priority order)"""
+    d = synth.random_dag(seed, V=V, G=G, K=K, zero_frac=0.0, caps="none", homogeneous=homogeneous)
+    cost = np.maximum(d.cost, 1) * scale
+    return dataclasses.replace(d, cost=cost)
+
+
+def pin_cands(desc, rng, n, kmax=4):
+    V, G = desc.n_ops, desc.n_devices
+    out = np.zeros(n, F.CANDIDATE_DTYPE)
+    for k in range(n):
+        if k == 0 or V == 0:
+            out[k] = F.make_candidate()
+            continue
+        npin = int(rng.integers(1, min(kmax, V) + 1))
+        ops = rng.choice(V, npin, replace=False)
+        out[k] = F.make_candidate(F.KIND_PIN, pins=[(int(o), int(rng.integers(0, G))) for o in ops])
+    return out
+
+
+def check(desc, cands, flags, expect_kernel=LANE, oracle_every=1):
+    gl = F.Graph(desc)
+    gg = _graph_env(desc, FASTT_NO_LANE="1")
+    r = gl.schedule_batch(cands, flags=flags, peak=False)
+    assert gl.last_timing()["topo"] == expect_kernel
+    r0 = gg.schedule_batch(cands, flags=flags, peak=False)
+    assert gg.last_timing()["topo"] in (0, GROUP)
+    assert (r["makespan"] == r0["makespan"]).all() and (r["status"] == r0["status"]).all()
+    og = O.OracleGraph(desc)
+    for k in range(0, len(cands), oracle_every):
+        o = og.schedule(cands[k], flags=flags, outputs=False)
+        assert int(r["makespan"][k]) == o["makespan"] and int(r["status"][k]) == o["status"], (desc.name, k, flags)
+    return r
+
+
+@pytest.mark.parametrize("G", [1, 2, 3, 4, 5, 8, 13, 16, 32])
+def test_lane_device_counts(G):
+    desc = topo_dag(4000 + G, V=150, G=G, K=1, homogeneous=bool(G % 2))
+    cands = pin_cands(desc, np.random.default_rng(G), 160)
+    for flags in (0, F.F_CP_PIN):
+        check(desc, cands, flags)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_lane_link_classes(seed):
+    """several link classes: per (pred, device) comm terms (CM = 2)"""
+    desc = topo_dag(4100 + seed, V=120, G=int(3 + seed % 6), K=3)
+    cands = pin_cands(desc, np.random.default_rng(seed), 128)
+    check(desc, cands, F.F_CP_PIN)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_lane_64bit_time(seed):
+    desc = topo_dag(4200 + seed, V=100, G=int(2 + 2 * seed), K=1 + seed % 2, scale=50_000_000)
+    assert F.Graph(desc).time_bits == 64
+    cands = pin_cands(desc, np.random.default_rng(seed), 96)
+    check(desc, cands, F.F_CP_PIN)
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_cp_pins_refuse_sharing(seed):
+    """Hetero costs: pinning critical-path ops moves the CP device (R9), so
+    those candidates cannot start from the recorded BASE prefix; every CP op
+    pinned to every device, both position-order kernels against the oracle."""
+    desc = topo_dag(4300 + seed, V=80, G=3 + seed % 3, K=1)
+    og = O.OracleGraph(desc)
+    base = og.schedule(F.make_candidate(), flags=F.F_CP_PIN)
+    cands = [F.make_candidate()]
+    for o in range(desc.n_ops):
+        for dv in range(desc.n_devices):
+            cands.append(F.make_candidate(F.KIND_PIN, pins=[(o, dv)]))
+    cands = np.array(cands)
+    r = check(desc, cands, F.F_CP_PIN)
+    assert int(r["makespan"][0]) == base["makespan"]
+    # the group position-order kernel on the same list (t0 of refused candidates)
+    gg = _graph_env(desc, FASTT_NO_LANE="1")
+    r1 = gg.schedule_batch(cands, flags=F.F_CP_PIN, peak=False)
+    assert gg.last_timing()["topo"] == GROUP
+    assert (r1["makespan"] == r["makespan"]).all()
+
+
+@pytest.mark.parametrize("name", ["C2", "C5"])
+def test_lane_sweep_configs(name):
+    desc = synth.config(name)
+    gl, gg = F.Graph(desc), _graph_env(desc, FASTT_NO_LANE="1")
+    gen = F.gen_params(seed=0xFA57)
+    ns = gl.stream_info(gen, flags=F.F_CP_PIN)
+    n = ns + 3000
+    b1 = gl.sweep_best(gen, 0, n, flags=F.F_CP_PIN)
+    assert gl.last_timing()["topo"] == LANE
+    b0 = gg.sweep_best(gen, 0, n, flags=F.F_CP_PIN)
+    assert b1 == b0
+    c = gl.generate_candidates(gen, ns + 1, 700, flags=F.F_CP_PIN)
+    r = gl.schedule_batch(c, flags=F.F_CP_PIN, peak=False)
+    assert gl.last_timing()["topo"] == LANE
+    r0 = gg.schedule_batch(c, flags=F.F_CP_PIN, peak=False)
+    assert (r["makespan"] == r0["makespan"]).all()
+    og = O.OracleGraph(desc)
+    for k in range(0, len(c), 233):
+        assert int(r["makespan"][k]) == og.schedule(c[k], flags=F.F_CP_PIN, outputs=False)["makespan"], (name, k)
+
+
+def test_lane_small_batches_no_sharing():
+    """fewer than 64 candidates: no snapshot, every candidate from step 0"""
+    desc = topo_dag(4400, V=200, G=8, K=1)
+    cands = pin_cands(desc, np.random.default_rng(1), 40)
+    check(desc, cands, F.F_CP_PIN)
+    check(desc, cands, 0)
+
+
+def test_lane_ragged_and_invalid():
+    """a batch that is not a multiple of 32, bad specs and splits mixed in"""
+    desc = topo_dag(4500, V=90, G=4, K=1)
+    desc = dataclasses.replace(desc, split_mask=np.full(desc.n_ops, 3, np.uint8))
+    rng = np.random.default_rng(2)
+    cands = list(pin_cands(desc, rng, 101))
+    cands[7] = F.make_candidate(F.KIND_PIN, pins=[(3, desc.n_devices)])         # device out of range
+    cands[40] = F.make_candidate(F.KIND_SPLIT, split=(10, 0, 2))                 # deferred (prep pipeline)
+    cands[41] = F.make_candidate(F.KIND_PIN, pins=[(5, 1), (5, 2)])              # duplicate op
+    cands[77] = F.make_candidate(dev_mask=0b0011)                                # device subset (deferred)
+    check(desc, np.array(cands), F.F_CP_PIN)
