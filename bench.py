@@ -51,6 +51,14 @@ def b_alg(V, E, G):
     return V * (8 * G + 45) + 29 * E
 
 
+def b_alg_lane(V, E, G):
+    """Touched-once bytes per candidate when 32 candidates share each read of
+    the graph (k_sim_lane: one warp = 32 candidates at the same position):
+    B_state + B_graph / 32 with SURVEY 8(d)'s B_state = 21V + 13E and
+    B_graph = V(8G + 24) + 16E."""
+    return 21 * V + 13 * E + (V * (8 * G + 24) + 16 * E) / 32.0
+
+
 def peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -269,7 +277,9 @@ def main():
     sim_ms = statistics.mean(x["ms_sim"] for x in tms)
     fast = statistics.mean(x["candidates"] - x["deferred"] for x in tms)
     prep_ms = statistics.mean(x["ms_prep"] for x in tms)
-    achieved = b_alg(V, E, G) * fast / (sim_ms / 1000.0) / 1e9
+    lane = tms[-1].get("topo", 0) == 2
+    bpc = b_alg_lane(V, E, G) if lane else b_alg(V, E, G)
+    achieved = bpc * fast / (sim_ms / 1000.0) / 1e9
     peak, peak_src = peaks()
     traffic = None
     try:
@@ -331,8 +341,11 @@ def main():
                        "parallelism": "candidates sharded c = rank mod N; NCCL all_reduce(MIN) argmin"},
             "best": {"makespan_ns": best[0], "index": best[1]},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                         "traffic": traffic, "kernel": "k_sim<uint32_t> (sweep launch)", "peak_source": peak_src,
-                         "bytes_per_candidate": b_alg(V, E, G), "candidates_per_launch": fast,
+                         "traffic": traffic,
+                         "kernel": ("k_sim_lane" if lane else "k_sim") + "<uint32_t> (sweep launch)",
+                         "peak_source": peak_src,
+                         "bytes_per_candidate": bpc, "bytes_per_candidate_survey": b_alg(V, E, G),
+                         "candidates_per_launch": fast,
                          "launch_ms": sim_ms, "prep_ms_per_step": prep_ms,
                          "note": "latency-bound sequential list scheduling; frac is of the measured copy bandwidth"},
             "cpu_baseline": cpu,

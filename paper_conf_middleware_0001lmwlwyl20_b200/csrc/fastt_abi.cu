@@ -679,6 +679,28 @@ static fastt_status ensure_sort_buf(fastt_graph *g, int64_t n) {
   return FASTT_OK;
 }
 
+// Simulation of nc prepared slots (mode 2).  Slots whose priority order is
+// topological (the flag the card kernels write into each slot's PrepGraph)
+// run the position-order variant, the others the ready-set variant: two
+// launches, each skipping the other kind of slot.
+static void launch_slots(fastt_graph *g, SimArgs b, int tbits, int nc, cudaStream_t st) {
+  b.mode = 2;
+  b.lane = 0;
+  const int per_block = (g->sim_block / 32) * g->sim_cpw;
+  if (g->use_topo) {
+    b.topo = 1;
+    b.slot_filter = 1;
+    launch_sim(b, tbits, (int)std::min<int64_t>(g->sim_grid_topo, nc / per_block + 1), g->sim_block, 0, st);
+    cudaMemsetAsync(g->counters, 0, sizeof(unsigned long long), st);
+    b.slot_filter = 2;
+  } else {
+    b.slot_filter = 0;
+  }
+  b.topo = 0;
+  launch_sim(b, tbits, (int)std::min<int64_t>(g->sim_grid, nc / per_block + 1), g->sim_block, g->sim_smem, st);
+  g->launches += g->use_topo ? 1 : 0;
+}
+
 struct DevOut {
   int64_t *makespan = nullptr;
   uint8_t *status = nullptr;
@@ -757,15 +779,11 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
       CK(cudaMemsetAsync(g->counters, 0, sizeof(unsigned long long), st));
       SimArgs b = a;
       b.slots = g->slot_pgs_dev;
-      b.mode = 2;
-      b.topo = 0;
-      b.lane = 0;
       b.cands = g->slot_cands;
       b.slot_result = g->slot_result;
       b.slot_index = nullptr;
       b.n = nc;
-      launch_sim(b, B.tbits, std::min<int64_t>(g->sim_grid, nc / ((g->sim_block / 32) * g->sim_cpw) + 1), g->sim_block,
-                 g->sim_smem, st);
+      launch_slots(g, b, B.tbits, nc, st);
       CK(cudaGetLastError());
     }
   }
@@ -1457,14 +1475,11 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
         CK(cudaMemsetAsync(g->counters, 0, sizeof(unsigned long long), st));
         SimArgs b = a;
         b.slots = g->slot_pgs_dev;
-        b.mode = 2;
-        b.topo = 0;
-        b.lane = 0;
         b.cands = g->slot_cands;
         b.slot_result = nullptr;
         b.slot_index = g->slot_index;
         b.n = nc;
-        launch_sim(b, B.tbits, g->sim_grid, g->sim_block, g->sim_smem, st);
+        launch_slots(g, b, B.tbits, nc, st);
         CK(cudaGetLastError());
       }
     }

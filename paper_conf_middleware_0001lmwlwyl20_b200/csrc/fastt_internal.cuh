@@ -206,6 +206,7 @@ struct SimArgs {
   int32_t topo;          // the graph's priority order is topological: dequeue order = position order
   int32_t lane;          // run the lane-per-candidate position-order kernel (k_sim_lane)
   int32_t gc_K;          // link classes (host copy of GraphConst::K)
+  int32_t slot_filter;   // mode 2: 0 all slots, 1 only slots with a topological order, 2 only the others
   int32_t cap_check;     // some device has a finite memory cap (R8)
   // BASE-schedule prefix sharing: 1 = record the snapshot (one BASE run),
   // 2 = start eligible PIN candidates from it at their first pinned op

@@ -252,7 +252,7 @@ __global__ void __launch_bounds__(SIM_BLOCK, TOPO ? SIM_MINB_TOPO : SIM_MINB) k_
     q0 = __shfl_sync(FULL, q0, 0);
     if ((int64_t)q0 >= a.n) break;
     const int64_t q = (int64_t)q0 + grp;
-    const bool active = q < a.n;
+    bool active = q < a.n;
     Cand c;
     c.kind = 0; c.n_pins = 0; c.split_op = -1;
     const PrepGraph *pg = a.base;
@@ -273,6 +273,8 @@ __global__ void __launch_bounds__(SIM_BLOCK, TOPO ? SIM_MINB_TOPO : SIM_MINB) k_
         pg = a.slots + q;
         res_idx = a.slot_result ? a.slot_result[q] : -1;
         sidx = a.slot_index ? a.slot_index[q] : q;
+        // two launches over the slots: position-order (1) / ready-set (2)
+        if (a.slot_filter && (pg->topo != 0) != (a.slot_filter == 1)) active = false;
       }
     }
     const uint32_t *__restrict__ card = pg->card;

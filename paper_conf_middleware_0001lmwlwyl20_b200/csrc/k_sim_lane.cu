@@ -38,8 +38,72 @@
 
 namespace fastt {
 
+// pipeline depth: records of positions at distance <= D-1 are read from the
+// shared-memory ring of the last D records; older ones are staged by
+// cp.async D-1 steps ahead (SLAB records are 8 B for 32-bit time, 16 B else)
+#ifndef LANE_D
+#define LANE_D 8
+#endif
+template <typename T> struct LaneDepth { static constexpr int D = sizeof(T) == 4 ? LANE_D : LANE_D / 2; };
+// staged card of one position: header (words 0-3), predecessor positions
+// (words 8-11), the inline predecessors' comm values (4 x T), then the cost
+// row padded to 16 B
+template <typename T> __host__ __device__ constexpr int card_cost_off() { return 32 + 4 * (int)sizeof(T); }
+template <typename T, int GP> __host__ __device__ constexpr int card_slot_bytes() {
+  return card_cost_off<T>() + (int)((GP * sizeof(T) + 15) / 16) * 16;
+}
+template <typename T, int GP> __host__ __device__ constexpr size_t lane_smem_per_warp() {
+  // ring D x 32 + stage D x 4 x 32 records, then 2D staged cards
+  return (size_t)LaneDepth<T>::D * 5 * 32 * (sizeof(T) == 4 ? 8 : 16) +
+         (size_t)2 * LaneDepth<T>::D * card_slot_bytes<T, GP>();
+}
+
+template <int BYTES> __device__ __forceinline__ void cp_async(uint32_t saddr, const void *g);
+template <> __device__ __forceinline__ void cp_async<4>(uint32_t saddr, const void *g) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(saddr), "l"(g) : "memory");
+}
+template <> __device__ __forceinline__ void cp_async<8>(uint32_t saddr, const void *g) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(saddr), "l"(g) : "memory");
+}
+template <> __device__ __forceinline__ void cp_async<16>(uint32_t saddr, const void *g) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(saddr), "l"(g) : "memory");
+}
+// predicated form: the copy is issued iff p
+template <int BYTES> __device__ __forceinline__ void cp_async_if(bool p, uint32_t saddr, const void *g);
+#define FASTT_CP_ASYNC_IF(BYTES, CACHE)                                                                    \
+  template <> __device__ __forceinline__ void cp_async_if<BYTES>(bool p, uint32_t saddr, const void *g) {  \
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t@q cp.async." CACHE                       \
+                 ".shared.global [%0], [%1], " #BYTES ";\n}\n" ::"r"(saddr),                                \
+                 "l"(g), "r"((int)p)                                                                        \
+                 : "memory");                                                                               \
+  }
+FASTT_CP_ASYNC_IF(4, "ca")
+FASTT_CP_ASYNC_IF(8, "ca")
+FASTT_CP_ASYNC_IF(16, "cg")
+#undef FASTT_CP_ASYNC_IF
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N> __device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+
 template <typename T> struct RowLd;
 template <> struct RowLd<uint32_t> {
+  template <int GP>
+  __device__ static void load_s(const uint32_t *row, int G, uint32_t (&c)[GP]) {  // shared memory, 16-B aligned
+    if (GP >= 4) {
+#pragma unroll
+      for (int j = 0; j < GP / 4; j++) {
+        const uint4 x = ((const uint4 *)row)[j];
+        c[4 * j] = x.x;
+        c[4 * j + 1] = x.y;
+        c[4 * j + 2] = x.z;
+        c[4 * j + 3] = x.w;
+      }
+    } else {
+#pragma unroll
+      for (int d = 0; d < GP; d++) c[d] = row[d];
+    }
+  }
   template <int GP>
   __device__ static void load(const uint32_t *row, int G, uint32_t (&c)[GP]) {
     if (GP >= 4 && G == GP) {
@@ -59,6 +123,19 @@ template <> struct RowLd<uint32_t> {
 };
 template <> struct RowLd<uint64_t> {
   template <int GP>
+  __device__ static void load_s(const uint64_t *row, int G, uint64_t (&c)[GP]) {
+    if (GP >= 2) {
+#pragma unroll
+      for (int j = 0; j < GP / 2; j++) {
+        const ulonglong2 x = ((const ulonglong2 *)row)[j];
+        c[2 * j] = x.x;
+        c[2 * j + 1] = x.y;
+      }
+    } else {
+      c[0] = row[0];
+    }
+  }
+  template <int GP>
   __device__ static void load(const uint64_t *row, int G, uint64_t (&c)[GP]) {
     if (GP >= 2 && G == GP) {
 #pragma unroll
@@ -77,7 +154,8 @@ template <> struct RowLd<uint64_t> {
 // CM: 0 = uint32 time and one link class, comm values inline in the card;
 //     1 = one link class, comm per edge from pe_comm;
 //     2 = several link classes (per (pred, device) comm).
-template <typename T, int GSH, int CM>
+// EX: G == GP (no per-device range checks).
+template <typename T, int GSH, int CM, bool EX>
 __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   typedef typename Slab<T>::W W;
   constexpr int GP = 1 << GSH;
@@ -86,6 +164,28 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   const int64_t gwarp = (int64_t)blockIdx.x * (LANE_BLOCK / 32) + (threadIdx.x >> 5);
   // this lane's slab column: record of position p at col[p * 32]
   W *const col = (W *)a.slab + (size_t)gwarp * (size_t)a.slab_stride * 32 + lane;
+  // shared memory of this warp: ring[D][32] (records of the last D positions)
+  // and stage[D][4][32] (inline predecessors' records prefetched by cp.async)
+  constexpr int D = LaneDepth<T>::D, P = D - 1;
+  extern __shared__ __align__(16) unsigned char lsm[];
+  unsigned char *const wsm = lsm + (threadIdx.x >> 5) * lane_smem_per_warp<T, GP>();
+  W *const ring = (W *)wsm + lane;
+  W *const stage = ring + D * 32;
+  const uint32_t stage_sa = (uint32_t)__cvta_generic_to_shared(stage);
+  // 2D staged cards (warp-shared): the card of position u is copied at step
+  // u - 2P and read at steps u - P (record prefetch) and u (compute)
+  constexpr int CS = card_slot_bytes<T, GP>();
+  const unsigned char *const cards = wsm + (size_t)D * 5 * 32 * sizeof(W);
+  const uint32_t cards_sa = (uint32_t)__cvta_generic_to_shared(cards);
+  constexpr int CO = card_cost_off<T>();
+  const bool row16 = (a.G * (int)sizeof(T)) % 16 == 0;
+  // this lane's 16-B chunk of a card copy: lane 0 header (words 0-3), lane 1
+  // predecessor positions (8-11), lane 2 comm (12-15, CM 0), lanes 3.. the
+  // cost row (when its length is a multiple of 16 B, else element-wise)
+  const bool cc_cost = lane >= 3;
+  const uint32_t cc_src = lane == 0 ? 0u : lane == 1 ? 4u * CARD_HDR : lane == 2 ? 4u * CW_PCOMM : 16u * (lane - 3);
+  const uint32_t cc_dst = lane < 3 ? 16u * lane : (uint32_t)CO + 16u * (lane - 3);
+  const bool cc_on = lane < 2 || (lane == 2 && CM == 0) || (lane >= 3 && lane - 3 < a.G * (int)sizeof(T) / 16);
   const GraphConst &gc = *a.gc;
   const int G = a.G;
   const int K = gc.K;
@@ -244,29 +344,102 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       lo = x < lo ? x : lo;
     }
 
+    // the next pinned position at or after the current step (NONE: none left)
+    uint32_t nxt = NONE;
+#pragma unroll
+    for (int k = 0; k < MAXPINS; k++)
+      if (pp[k] >= (uint32_t)lo && pp[k] < nxt) nxt = pp[k];
     // ---------------------------------------------------------- main loop
+    // Software pipeline over positions (all cp.async copies are predicated,
+    // so the step is branch-free for every lane):
+    //   step u - 2P : the card of u (header, predecessor positions, comm,
+    //                 cost row) is copied into cards[u % 2D] by lanes 0..;
+    //   step u - P  : the inline predecessors of u at distance > P (and
+    //                 BASE-prefix records, s < t0) are copied into
+    //                 stage[u % D]; one commit group per step;
+    //   step u      : the others were written at most P steps earlier and
+    //                 are read from the ring of the last D records.
+    // A staged record was stored at least one step before its copy is issued
+    // (same thread, program order).  A stage or card slot is overwritten only
+    // after the step that read it has consumed the values.
+    // (t0 = 0 unless the candidate shares the BASE prefix, so "s < t0" alone
+    // selects the BASE record; a record is staged iff s < max(t0, u - P))
+    auto copy_card = [&](int32_t u) {
+      const uint32_t dst = cards_sa + (uint32_t)((u & (2 * D - 1)) * CS) + cc_dst;
+      const char *srcp = cc_cost ? (const char *)(costp + (size_t)u * G) + cc_src
+                                 : (const char *)(card + (size_t)u * CARD_WORDS) + cc_src;
+      if (row16) cp_async_if<16>(cc_on && u < n, dst, srcp);
+      else {
+        cp_async_if<16>(cc_on && !cc_cost && u < n, dst, srcp);
+        for (int j = lane; j < G; j += 32)
+          cp_async_if<sizeof(T)>(u < n, cards_sa + (uint32_t)((u & (2 * D - 1)) * CS + CO + j * sizeof(T)),
+                                 costp + (size_t)u * G + j);
+      }
+    };
+    auto prefetch = [&](int32_t u) {  // records of step u (its card is staged)
+      const unsigned char *cu = cards + (u & (2 * D - 1)) * CS;
+      const uint4 hu = *(const uint4 *)cu;
+      const uint32_t npu = u < n ? (hu.x & 0xFFFF) : 0u;
+      if (CM == 1)  // the inline predecessors' comm values (warp-uniform card)
+        cp_async_if<sizeof(T)>((uint32_t)lane < npu && lane < 4,
+                               cards_sa + (uint32_t)((u & (2 * D - 1)) * CS + 32 + (lane & 3) * sizeof(T)),
+                               pe_comm + hu.y + (lane & 3));
+      const uint4 su = *(const uint4 *)(cu + 16);
+      const uint32_t ss[4] = {su.x, su.y, su.z, su.w};
+      const uint32_t sl = stage_sa + (uint32_t)((u & (D - 1)) * 4 * 32 * sizeof(W));
+      const bool on = run && u >= t0;
+      const int32_t thr = t0 > u - P ? t0 : u - P;
+#pragma unroll
+      for (int k = 0; k < 4; k++) {
+        const W *gp = (int32_t)ss[k] < t0 ? snap + ss[k] : col + (size_t)ss[k] * 32;
+        cp_async_if<sizeof(W)>(on && (uint32_t)k < npu && (int32_t)ss[k] < thr, sl + (uint32_t)(k * 32 * sizeof(W)), gp);
+      }
+    };
+    // record of position s < t outside the inline slots (extra predecessors)
+    auto rec_at = [&](uint32_t s, int32_t t) -> W {
+      if ((int32_t)s < t0) return snap[s];
+      if ((int32_t)s + P >= t) return ring[(s & (D - 1)) * 32];
+      return col[(size_t)s * 32];
+    };
+    // prologue: cards of lo .. lo+2P-1 (synchronously), records of lo .. lo+P-1
+    for (int32_t u = lo; u < lo + 2 * P; u++) copy_card(u);
+    cp_async_commit();
+    cp_async_wait<0>();
+    __syncwarp();
+    for (int32_t u = lo; u < lo + P; u++) {
+      prefetch(u);
+      cp_async_commit();
+    }
     for (int32_t t = lo; t < n; t++) {
       const bool live = run && t >= t0;
-      const uint32_t *cd = card + (size_t)t * CARD_WORDS;
-      const uint4 h0 = __ldg((const uint4 *)cd);
-      const uint4 hs = __ldg((const uint4 *)(cd + CARD_HDR));
+      cp_async_wait<P - 1>();  // the group of step t - P: records of t, card of t + P
+      __syncwarp();            // (cards were copied by other lanes)
+      const unsigned char *cs = cards + (t & (2 * D - 1)) * CS;
+      const uint4 h0 = *(const uint4 *)cs;
+      const uint4 hs = *(const uint4 *)(cs + 16);
       uint4 hc = make_uint4(0, 0, 0, 0);
-      if (CM == 0) hc = __ldg((const uint4 *)(cd + CW_PCOMM));
+      if (CM == 0) hc = *(const uint4 *)(cs + 32);
+      const T *cm1 = (const T *)(cs + 32);  // CM 1: staged comm values
       T cst[GP];
-      RowLd<T>::template load<GP>(costp + (size_t)t * G, G, cst);
+      RowLd<T>::template load_s<GP>((const T *)(cs + CO), G, cst);
       const uint32_t npred = h0.x & 0xFFFF;
       const uint32_t src[4] = {hs.x, hs.y, hs.z, hs.w};
-      // predecessor records (unused card slots hold position 0: valid address)
+      // predecessor records: staged or from the ring (unused slots: garbage, masked)
       W rw[4];
+      const W *stg = stage + (t & (D - 1)) * 4 * 32;
+      const int32_t thr = t0 > t - P ? t0 : t - P;
 #pragma unroll
-      for (int k = 0; k < 4; k++) rw[k] = (share && (int32_t)src[k] < t0) ? snap[src[k]] : col[(size_t)src[k] * 32];
+      for (int k = 0; k < 4; k++) rw[k] = *((int32_t)src[k] < thr ? stg + k * 32 : ring + (src[k] & (D - 1)) * 32);
+      prefetch(t + P);
+      copy_card(t + 2 * P);
+      cp_async_commit();
       T f[4];
       uint32_t p[4];
 #pragma unroll
       for (int k = 0; k < 4; k++) {
         T ft;
         uint32_t pl;
-        Slab<T>::decode(rw[k], ft, pl);
+        Slab<T>::decode_clean(rw[k], ft, pl);
         f[k] = (uint32_t)k < npred ? ft : (T)0;
         p[k] = (uint32_t)k < npred ? pl : 0xFFu;
       }
@@ -274,27 +447,30 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       T M = 0, E = 0;
       uint32_t pa = 0xFFu;
       if (CM != 2) {
+        // M = max over preds of FT + c, pa = the device of a pred attaining it,
+        // E = the arrival on pa (its co-located preds contribute FT only)
         T R[4];
 #pragma unroll
         for (int k = 0; k < 4; k++) {
           T cm;
           if (CM == 0) cm = (T)(k == 0 ? hc.x : k == 1 ? hc.y : k == 2 ? hc.z : hc.w);
-          else cm = (uint32_t)k < npred ? __ldg(pe_comm + h0.y + k) : (T)0;
+          else cm = cm1[k];
           R[k] = (uint32_t)k < npred ? f[k] + cm : (T)0;
         }
+        M = R[0];
+        pa = p[0];
 #pragma unroll
-        for (int k = 0; k < 4; k++)
-          if ((uint32_t)k < npred && (pa == 0xFFu || R[k] > M)) {
+        for (int k = 1; k < 4; k++)
+          if (R[k] > M) {
             M = R[k];
             pa = p[k];
           }
         if (npred > 4u) {  // (warp-uniform)
           for (uint32_t k = 4; k < npred; k++) {
-            const uint32_t qs = __ldg(pe_src + h0.y + k);
-            const W w = (share && (int32_t)qs < t0) ? snap[qs] : col[(size_t)qs * 32];
+            const W w = rec_at(__ldg(pe_src + h0.y + k), t);
             T ft;
             uint32_t pl;
-            Slab<T>::decode(w, ft, pl);
+            Slab<T>::decode_clean(w, ft, pl);
             const T r = ft + __ldg(pe_comm + h0.y + k);
             if (r > M) {
               M = r;
@@ -309,20 +485,21 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
         }
         if (npred > 4u) {
           for (uint32_t k = 4; k < npred; k++) {
-            const uint32_t qs = __ldg(pe_src + h0.y + k);
-            const W w = (share && (int32_t)qs < t0) ? snap[qs] : col[(size_t)qs * 32];
+            const W w = rec_at(__ldg(pe_src + h0.y + k), t);
             T ft;
             uint32_t pl;
-            Slab<T>::decode(w, ft, pl);
+            Slab<T>::decode_clean(w, ft, pl);
             const T v = pl == pa ? ft : ft + __ldg(pe_comm + h0.y + k);
             E = v > E ? v : E;
           }
         }
       } else {
+        // (only live lanes: a waiting lane's records are not yet valid, and
+        // here a placement indexes the link-class table)
 #pragma unroll
         for (int d = 0; d < GP; d++) {
           T v = 0;
-          if (d < G) {
+          if (live && d < G) {
 #pragma unroll
             for (int k = 0; k < 4; k++)
               if ((uint32_t)k < npred) {
@@ -332,11 +509,10 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
                 v = term > v ? term : v;
               }
             for (uint32_t k = 4; k < npred; k++) {
-              const uint32_t qs = __ldg(pe_src + h0.y + k);
-              const W w = (share && (int32_t)qs < t0) ? snap[qs] : col[(size_t)qs * 32];
+              const W w = rec_at(__ldg(pe_src + h0.y + k), t);
               T ft;
               uint32_t pl;
-              Slab<T>::decode(w, ft, pl);
+              Slab<T>::decode_clean(w, ft, pl);
               const T term =
                   pl == (uint32_t)d ? ft : ft + __ldg(pe_comm + (size_t)(h0.y + k) * K + gc.link_class[pl * G + d]);
               v = term > v ? term : v;
@@ -345,25 +521,41 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
           arrd[d] = v;
         }
       }
-      // device forced by a perturbation pin (hard) or a CP pin (Alg. 1 l.9-10)
-      int forced = -1;
-#pragma unroll
-      for (int k = 0; k < MAXPINS; k++)
-        if (pp[k] == (uint32_t)t) forced = (int)((pdv >> (8 * k)) & 0xFFu);
-      if (forced < 0 && r_dev >= 0 && h0.w != NONE) forced = r_dev;
-      // argmin EFT, ties -> lowest device (Alg. 1 lines 12-19, R3)
-      T best = 0;
-      int bd = -1;
+      // EFT per device; argmin with ties to the lowest device
+      // (Alg. 1 lines 12-19, R3); devices >= G are never chosen
+      T eft[GP];
 #pragma unroll
       for (int d = 0; d < GP; d++) {
-        if (d < G) {
-          const T arr = CM == 2 ? arrd[d] : ((uint32_t)d == pa ? E : M);
-          const T est = avail[d] > arr ? avail[d] : arr;
-          const T eft = est + cst[d];
-          if ((forced < 0 || forced == d) && (bd < 0 || eft < best)) {
-            best = eft;
-            bd = d;
+        const T arr = CM == 2 ? arrd[d] : ((uint32_t)d == pa ? E : M);
+        const T est = avail[d] > arr ? avail[d] : arr;
+        eft[d] = (EX || d < G) ? est + cst[d] : TT<T>::MAXV;
+      }
+      T best = eft[0];
+      int bd = 0;
+#pragma unroll
+      for (int d = 1; d < GP; d++)
+        if (eft[d] < best) {
+          best = eft[d];
+          bd = d;
+        }
+      // device forced by a perturbation pin (hard) or a CP pin (Alg. 1
+      // l.9-10): rare steps -- the next pinned position, or a CP op
+      if (__any_sync(FULL, (uint32_t)t == nxt || (h0.w != NONE && r_dev >= 0))) {
+        int forced = -1;
+        if ((uint32_t)t == nxt) {
+          nxt = NONE;
+#pragma unroll
+          for (int k = 0; k < MAXPINS; k++) {
+            if (pp[k] == (uint32_t)t) forced = (int)((pdv >> (8 * k)) & 0xFFu);
+            else if (pp[k] > (uint32_t)t && pp[k] < nxt) nxt = pp[k];
           }
+        }
+        if (forced < 0 && r_dev >= 0 && h0.w != NONE) forced = r_dev;
+        if (forced >= 0) {
+#pragma unroll
+          for (int d = 0; d < GP; d++)
+            if (d == forced) best = eft[d];
+          bd = forced;
         }
       }
       if (live) {
@@ -374,8 +566,10 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
         W w;
         Slab<T>::make(w, best, (uint32_t)bd);
         col[(size_t)t * 32] = w;
+        ring[(t & (D - 1)) * 32] = w;
       }
     }
+    cp_async_wait<0>();  // (no copy may land in the stage after this candidate)
 
     // ------------------------------------------------------------ epilogue
     if (run) {
@@ -408,23 +602,40 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   }
 }
 
-template <typename T, int CM>
+template <typename T, int CM, bool EX>
 static const void *lane_fn_t(int gshift) {
   switch (gshift) {
-    case 0: return (const void *)k_sim_lane<T, 0, CM>;
-    case 1: return (const void *)k_sim_lane<T, 1, CM>;
-    case 2: return (const void *)k_sim_lane<T, 2, CM>;
-    case 3: return (const void *)k_sim_lane<T, 3, CM>;
-    case 4: return (const void *)k_sim_lane<T, 4, CM>;
-    default: return (const void *)k_sim_lane<T, 5, CM>;
+    case 0: return (const void *)k_sim_lane<T, 0, CM, EX>;
+    case 1: return (const void *)k_sim_lane<T, 1, CM, EX>;
+    case 2: return (const void *)k_sim_lane<T, 2, CM, EX>;
+    case 3: return (const void *)k_sim_lane<T, 3, CM, EX>;
+    case 4: return (const void *)k_sim_lane<T, 4, CM, EX>;
+    default: return (const void *)k_sim_lane<T, 5, CM, EX>;
   }
 }
-static const void *lane_fn(int tbits, int gshift, int cm) {
+template <bool EX> static const void *lane_fn_x(int tbits, int gshift, int cm) {
   if (tbits == 32) {
-    if (cm == 0) return lane_fn_t<uint32_t, 0>(gshift);
-    return cm == 1 ? lane_fn_t<uint32_t, 1>(gshift) : lane_fn_t<uint32_t, 2>(gshift);
+    if (cm == 0) return lane_fn_t<uint32_t, 0, EX>(gshift);
+    return cm == 1 ? lane_fn_t<uint32_t, 1, EX>(gshift) : lane_fn_t<uint32_t, 2, EX>(gshift);
   }
-  return cm == 2 ? lane_fn_t<uint64_t, 2>(gshift) : lane_fn_t<uint64_t, 1>(gshift);
+  return cm == 2 ? lane_fn_t<uint64_t, 2, EX>(gshift) : lane_fn_t<uint64_t, 1, EX>(gshift);
+}
+static const void *lane_fn(int tbits, int gshift, int cm, bool exact) {
+  return exact ? lane_fn_x<true>(tbits, gshift, cm) : lane_fn_x<false>(tbits, gshift, cm);
+}
+
+template <typename T> static size_t lane_smem_t(int gshift) {
+  switch (gshift) {
+    case 0: return lane_smem_per_warp<T, 1>();
+    case 1: return lane_smem_per_warp<T, 2>();
+    case 2: return lane_smem_per_warp<T, 4>();
+    case 3: return lane_smem_per_warp<T, 8>();
+    case 4: return lane_smem_per_warp<T, 16>();
+    default: return lane_smem_per_warp<T, 32>();
+  }
+}
+size_t lane_smem(int tbits, int gshift) {
+  return (LANE_BLOCK / 32) * (tbits == 32 ? lane_smem_t<uint32_t>(gshift) : lane_smem_t<uint64_t>(gshift));
 }
 
 int lane_comm_mode(const SimArgs &a, int tbits) {
@@ -433,16 +644,18 @@ int lane_comm_mode(const SimArgs &a, int tbits) {
 }
 
 void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
-  const void *f = lane_fn(tbits, a.gshift, lane_comm_mode(a, tbits));
+  const void *f = lane_fn(tbits, a.gshift, lane_comm_mode(a, tbits), a.G == (1 << a.gshift));
   SimArgs aa = a;
   void *args[] = {&aa};
-  cudaLaunchKernel(f, dim3(grid), dim3(LANE_BLOCK), args, 0, st);
+  cudaLaunchKernel(f, dim3(grid), dim3(LANE_BLOCK), args, lane_smem(tbits, a.gshift), st);
 }
 
 int lane_occupancy(int tbits, int gshift) {
   int nb = 1 << 30, x = 0;
-  for (int cm = (tbits == 32 ? 0 : 1); cm < 3; cm++) {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, lane_fn(tbits, gshift, cm), LANE_BLOCK, 0);
+  for (int v = (tbits == 32 ? 0 : 2); v < 6; v++) {
+    const void *f = lane_fn(tbits, gshift, v >> 1, v & 1);
+    cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lane_smem(tbits, gshift));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, f, LANE_BLOCK, lane_smem(tbits, gshift));
     nb = x < nb ? x : nb;
   }
   return nb;

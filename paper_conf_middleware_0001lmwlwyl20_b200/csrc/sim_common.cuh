@@ -38,6 +38,11 @@ template <> struct Slab<uint32_t> {
     ft = (uint32_t)w;
     plc = (uint32_t)(w >> 32) & 0xFF;
   }
+  // a record written by make() / sched() without indegree bits
+  __device__ static void decode_clean(const W &w, uint32_t &ft, uint32_t &plc) {
+    ft = (uint32_t)w;
+    plc = (uint32_t)(w >> 32);
+  }
   __device__ static uint32_t indeg(const W *s, uint32_t p) {
     return (*((const uint32_t *)(s + p) + 1)) >> 8;
   }
@@ -66,6 +71,10 @@ template <> struct Slab<uint64_t> {
   __device__ static void decode(const W &w, uint64_t &ft, uint32_t &plc) {
     ft = w.x;
     plc = (uint32_t)w.y & 0xFF;
+  }
+  __device__ static void decode_clean(const W &w, uint64_t &ft, uint32_t &plc) {
+    ft = w.x;
+    plc = (uint32_t)w.y;
   }
   __device__ static uint32_t indeg(const W *s, uint32_t p) {
     return (*((const uint32_t *)(s + p) + 2)) >> 8;
