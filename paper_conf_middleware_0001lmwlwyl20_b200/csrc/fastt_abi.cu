@@ -280,7 +280,7 @@ struct fastt_graph {
 };
 
 // kernels each launcher issues (for the launch count of fastt_last_timing)
-enum { NL_SIM = 1, NL_PREP = 8, NL_ARGMIN = 1, NL_GATHER = 1, NL_CANDGEN = 1, NL_ORDER = 1, NL_FILL = 1 };
+enum { NL_SIM = 1, NL_PREP = 9, NL_ARGMIN = 1, NL_GATHER = 1, NL_CANDGEN = 1, NL_ORDER = 1, NL_FILL = 1 };
 
 static fastt_status timing_begin(fastt_graph *g, uint32_t flags, cudaStream_t st) {
   g->launches = 0;
@@ -371,8 +371,8 @@ static fastt_status prepare_base(fastt_graph *g, Base &B, cudaStream_t st) {
   CK(cudaMemcpyAsync(B.pg_dev, &P, sizeof P, cudaMemcpyHostToDevice, st));
   launch_rank(B.raw_dev, B.pg_dev, g->gc_dev, nullptr, 1, g->G, st);
   launch_sort(B.pg_dev, B.raw_dev, 1, B.key_bits, B.n_live, st);
-  launch_cards(B.raw_dev, B.pg_dev, g->gc_dev, 1, B.n_live, g->G, g->K, B.tbits, st);
-  launch_cp(B.pg_dev, 1, g->G, B.tbits, st);
+  launch_cards(B.raw_dev, B.pg_dev, g->gc_dev, 1, B.n_live, g->G, g->K, B.tbits, st, true);
+  launch_cp(B.raw_dev, B.pg_dev, 1, g->G, B.tbits, st);
   CK(cudaGetLastError());
   CK(cudaMemcpyAsync(&P, B.pg_dev, sizeof P, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
@@ -577,8 +577,10 @@ static fastt_status run_prep(fastt_graph *g, const Base &B, int nslots, cudaStre
   launch_patch_split(B.raw_dev, g->slot_raws_dev, g->gc_dev, g->slot_cands, nslots, st);
   launch_rank(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, g->slot_cands, nslots, g->G, st);
   launch_sort(g->slot_pgs_dev, g->slot_raws_dev, nslots, B.key_bits, (int)B.rl.vcap, st);
-  launch_cards(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, nslots, (int)B.rl.vcap, g->G, g->K, B.tbits, st);
-  launch_cp(g->slot_pgs_dev, nslots, g->G, B.tbits, st);
+  // (successor lists only for slots the ready-set kernel will run: see launch_slots)
+  launch_cards(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, nslots, (int)B.rl.vcap, g->G, g->K, B.tbits, st,
+               !g->use_topo);
+  launch_cp(g->slot_raws_dev, g->slot_pgs_dev, nslots, g->G, B.tbits, st);
   CK(cudaGetLastError());
   return FASTT_OK;
 }

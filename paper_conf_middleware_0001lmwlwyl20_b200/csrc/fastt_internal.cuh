@@ -155,8 +155,8 @@ void launch_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, con
 void launch_heights(RawGraph *raw_dev, int32_t *scratch, int64_t vcap, cudaStream_t st);
 void launch_sort(PrepGraph *pgs, const RawGraph *raws, int nslots, int key_bits, int max_n, cudaStream_t st);
 void launch_cards(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, int nslots, int max_n, int G, int K,
-                  int tbits, cudaStream_t st);
-void launch_cp(PrepGraph *pgs, int nslots, int G, int tbits, cudaStream_t st);
+                  int tbits, cudaStream_t st, bool succ_all);
+void launch_cp(const RawGraph *raws, PrepGraph *pgs, int nslots, int G, int tbits, cudaStream_t st);
 void launch_copy_block(const void *src, void *dst, int64_t slot_stride_bytes, int64_t bytes, const Cand *cands,
                        int nslots, cudaStream_t st);
 void launch_patch_split(const RawGraph *base, RawGraph *raws, const GraphConst *gc, const Cand *cands, int nslots,

@@ -7,6 +7,7 @@
 //   k_cp          : critical path (R7) and its prefix sums for the CP devices
 //   k_bound       : the schedule bound that selects 32-bit time (R18)
 //   k_splitlist   : Alg. 2 lines 4-5: placement-aware CP, split-eligible, sorted (R15)
+#include <algorithm>
 #include "fastt_internal.cuh"
 
 namespace fastt {
@@ -588,38 +589,70 @@ __global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, Prep
   }
 }
 
-// One warp per position: edge arrays, inline card entries and the cost row.
+// One thread per position: the cost row, the predecessor edge arrays and
+// the inline predecessor entries of the card (words 8-15); clears P.topo on
+// an edge that does not go from a lower to a higher position.
 template <typename T>
-__global__ void k_cards_edges(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gcp, int max_n) {
-  const int lane = threadIdx.x & 31;
-  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+__global__ void k_cards_pred(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gcp) {
   const int slot = blockIdx.y;
   const RawGraph &R = raws[slot];
   PrepGraph &P = pgs[slot];
   const GraphConst &gc = *gcp;
   const int G = gc.G, K = gc.K;
   const int32_t n = P.n;
+  T *costp = (T *)P.costp;
+  T *pec = (T *)P.pe_comm;
+  bool back = false;
+  for (int32_t p = blockIdx.x * blockDim.x + threadIdx.x; p < n; p += gridDim.x * blockDim.x) {
+    uint32_t *c = P.card + (int64_t)p * CARD_WORDS;
+    const uint32_t u = P.uid[p];
+    const uint2 dp = *(const uint2 *)c;  // CW_DEG, CW_PBASE (k_cards_hdr)
+    const uint32_t np_ = dp.x & 0xFFFF, pb = dp.y;
+    for (int d = 0; d < G; d++) costp[(int64_t)p * G + d] = (T)R.cost[(int64_t)u * G + d];
+    const uint32_t po = R.pred_off[u];
+    uint32_t inl[P_IN] = {0, 0, 0, 0}, icm[P_IN] = {0, 0, 0, 0};  // unused slots hold position 0
+#pragma unroll
+    for (int j = 0; j < P_IN; j++)
+      if ((uint32_t)j < np_) {
+        const int32_t s = R.pred_src[po + j];
+        const int64_t b = R.pred_bytes[po + j];
+        const uint32_t sp = P.pos[s];
+        P.pe_src[pb + j] = sp;
+        back |= sp >= (uint32_t)p;
+        for (int k = 0; k < K; k++) pec[(int64_t)(pb + j) * K + k] = (T)comm_class(gc, b, k);
+        inl[j] = sp;
+        icm[j] = (uint32_t)comm_class(gc, b, 0);  // used only for uint32 time, one class
+      }
+    for (uint32_t j = P_IN; j < np_; j++) {
+      const int32_t s = R.pred_src[po + j];
+      const int64_t b = R.pred_bytes[po + j];
+      const uint32_t sp = P.pos[s];
+      P.pe_src[pb + j] = sp;
+      back |= sp >= (uint32_t)p;
+      for (int k = 0; k < K; k++) pec[(int64_t)(pb + j) * K + k] = (T)comm_class(gc, b, k);
+    }
+    *(uint4 *)(c + CARD_HDR) = make_uint4(inl[0], inl[1], inl[2], inl[3]);
+    *(uint4 *)(c + CW_PCOMM) = make_uint4(icm[0], icm[1], icm[2], icm[3]);
+  }
+  if (__syncthreads_or(back) && threadIdx.x == 0) P.topo = 0;  // the priority order is not topological
+}
+
+// One warp per position: successor edge arrays and inline successor entries
+// (words 16-31).  Only the ready-set simulator and the PIN classification
+// read them, so slots whose order is topological are skipped unless `all`.
+__global__ void k_cards_succ(const RawGraph *raws, PrepGraph *pgs, int all) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int slot = blockIdx.y;
+  const RawGraph &R = raws[slot];
+  PrepGraph &P = pgs[slot];
+  if (!all && P.topo) return;
+  const int32_t n = P.n;
   for (int64_t p = gw; p < n; p += ((int64_t)gridDim.x * blockDim.x) >> 5) {
     uint32_t *c = P.card + p * CARD_WORDS;
-    uint32_t u = P.uid[p];
-    uint32_t np_ = c[CW_DEG] & 0xFFFF, ns_ = c[CW_DEG] >> 16;
-    uint32_t pb = c[CW_PBASE], sb = c[CW_SBASE];
-    T *costp = (T *)P.costp;
-    T *pec = (T *)P.pe_comm;
-    if (lane < G) costp[p * G + lane] = (T)R.cost[(int64_t)u * G + lane];
-    uint32_t po = R.pred_off[u], so = R.succ_off[u];
-    for (uint32_t j = lane; j < np_; j += 32) {
-      int32_t s = R.pred_src[po + j];
-      int64_t b = R.pred_bytes[po + j];
-      uint32_t sp = P.pos[s];
-      P.pe_src[pb + j] = sp;
-      if (sp >= (uint32_t)p) P.topo = 0;  // the priority order is not topological
-      for (int k = 0; k < K; k++) pec[(int64_t)(pb + j) * K + k] = (T)comm_class(gc, b, k);
-      if (j < P_IN) {
-        c[CARD_HDR + j] = sp;
-        c[CW_PCOMM + j] = (uint32_t)comm_class(gc, b, 0);  // used only for uint32 time, one class
-      }
-    }
+    const uint32_t u = P.uid[p];
+    const uint32_t ns_ = c[CW_DEG] >> 16, sb = c[CW_SBASE];
+    const uint32_t so = R.succ_off[u];
     for (uint32_t j = lane; j < ns_; j += 32) {
       int32_t d = R.succ_dst[so + j];
       uint32_t dp = P.pos[d];
@@ -631,25 +664,21 @@ __global__ void k_cards_edges(const RawGraph *raws, PrepGraph *pgs, const GraphC
       if (j < S_IN) c[CW_SUCC + j] = dp;
     }
     // unused inline slots hold position 0 so the simulator may load them speculatively
-    if (lane >= np_ && lane < P_IN) {
-      c[CARD_HDR + lane] = 0;
-      c[CW_PCOMM + lane] = 0;
-    }
     if (lane >= ns_ && lane < S_IN) c[CW_SUCC + lane] = 0;
   }
-  (void)max_n;
 }
 
 void launch_cards(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, int nslots, int max_n, int G, int K,
-                  int tbits, cudaStream_t st) {
+                  int tbits, cudaStream_t st, bool succ_all) {
   (void)G; (void)K;
   k_cards_hdr<<<nslots, SORT_T, 0, st>>>(raws, pgs);
+  dim3 gp((unsigned)std::max(1, std::min((max_n + 255) / 256, 1024)), nslots);
+  if (tbits == 32) k_cards_pred<uint32_t><<<gp, 256, 0, st>>>(raws, pgs, gc);
+  else k_cards_pred<uint64_t><<<gp, 256, 0, st>>>(raws, pgs, gc);
   int blocks = (max_n * 32 + 255) / 256;
   if (blocks > 2048) blocks = 2048;
   if (blocks < 1) blocks = 1;
-  dim3 grid(blocks, nslots);
-  if (tbits == 32) k_cards_edges<uint32_t><<<grid, 256, 0, st>>>(raws, pgs, gc, max_n);
-  else k_cards_edges<uint64_t><<<grid, 256, 0, st>>>(raws, pgs, gc, max_n);
+  k_cards_succ<<<dim3(blocks, nslots), 256, 0, st>>>(raws, pgs, succ_all ? 1 : 0);
 }
 
 // -------------------------------------------------------------------- CP
@@ -658,10 +687,11 @@ void launch_cards(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, in
 // op, then repeatedly the successor of highest priority (= lowest position) --
 // and its prefix sums of memory and per-device cost (for R9).
 template <typename T>
-__global__ void k_cp(PrepGraph *pgs, int nslots, int G) {
+__global__ void k_cp(const RawGraph *raws, PrepGraph *pgs, int nslots, int G) {
   const int lane = threadIdx.x & 31;
   const int slot = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (slot >= nslots) return;
+  const RawGraph &R = raws[slot];
   PrepGraph &P = pgs[slot];
   const int32_t n = P.n;
   const T *costp = (const T *)P.costp;
@@ -698,10 +728,12 @@ __global__ void k_cp(PrepGraph *pgs, int nslots, int G) {
     len++;
     if (lane == 0) P.pmem[len] = accm;
     if (lane < G) P.pcost[(int64_t)len * G + lane] = accc;
-    uint32_t ns_ = deg >> 16, sb = c[CW_SBASE];
+    // successors from the raw lists (the card's successor part is built
+    // only where the ready-set simulator needs it)
+    const uint32_t ns_ = deg >> 16, so = R.succ_off[c[CW_UID]];
     uint32_t best = NONE;
     for (uint32_t j = lane; j < ns_; j += 32) {
-      uint32_t d = j < S_IN ? c[CW_SUCC + j] : P.se_dst[sb + j];
+      const uint32_t d = P.pos[R.succ_dst[so + j]];
       best = d < best ? d : best;
     }
     best = warp_min_u32(best);
@@ -710,10 +742,10 @@ __global__ void k_cp(PrepGraph *pgs, int nslots, int G) {
   if (lane == 0) P.cp_len = len;
 }
 
-void launch_cp(PrepGraph *pgs, int nslots, int G, int tbits, cudaStream_t st) {
+void launch_cp(const RawGraph *raws, PrepGraph *pgs, int nslots, int G, int tbits, cudaStream_t st) {
   int blocks = (nslots + 3) / 4;
-  if (tbits == 32) k_cp<uint32_t><<<blocks, 128, 0, st>>>(pgs, nslots, G);
-  else k_cp<uint64_t><<<blocks, 128, 0, st>>>(pgs, nslots, G);
+  if (tbits == 32) k_cp<uint32_t><<<blocks, 128, 0, st>>>(raws, pgs, nslots, G);
+  else k_cp<uint64_t><<<blocks, 128, 0, st>>>(raws, pgs, nslots, G);
 }
 
 // ----------------------------------------------------------------- bound
