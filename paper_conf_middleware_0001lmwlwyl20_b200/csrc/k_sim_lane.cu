@@ -29,8 +29,9 @@
 //             total cost of the free CP ops (equal counts, exact compare).
 //   sharing : a candidate whose schedule provably equals the BASE schedule
 //             before its first pinned op (k_sim.cu) starts at that
-//             step t0 from the recorded BASE avail/makespan; records of
-//             positions before t0 are read from the BASE record in place.
+//             step t0; the warp starts at the smallest t0 of its lanes
+//             from the recorded BASE avail/makespan, and records of
+//             positions before that step are read from the BASE record.
 // Memory caps, liveness memory, INSERT, per-op outputs, SPLIT and
 // rank-changing candidates stay on k_sim (group-per-candidate kernel).
 #include "fastt_internal.cuh"
@@ -326,22 +327,26 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
         }
       }
     }
-    T avail[GP];
-    T ms = 0;
-#pragma unroll
-    for (int d = 0; d < GP; d++) avail[d] = 0;
-    if (share) {
-      const T *sa = (const T *)a.snap_avail + (size_t)t0 * G;
-#pragma unroll
-      for (int d = 0; d < GP; d++)
-        if (d < G) avail[d] = __ldg(sa + d);
-      ms = __ldg((const T *)a.snap_ms + t0);
-    }
+    // The warp starts at lo = the smallest t0 of its candidates (0 if one of
+    // them does not share): a sharing candidate started from the recorded
+    // BASE state at any step <= its t0 makes the BASE decisions up to t0, so
+    // all lanes may start at lo; positions before lo hold BASE records.
     int32_t lo = run ? t0 : n;
 #pragma unroll
     for (int o = 16; o >= 1; o >>= 1) {
       const int32_t x = __shfl_xor_sync(FULL, lo, o);
       lo = x < lo ? x : lo;
+    }
+    T avail[GP];
+    T ms = 0;
+#pragma unroll
+    for (int d = 0; d < GP; d++) avail[d] = 0;
+    if (run && lo > 0) {  // (lo > 0 implies every running lane shares)
+      const T *sa = (const T *)a.snap_avail + (size_t)lo * G;
+#pragma unroll
+      for (int d = 0; d < GP; d++)
+        if (d < G) avail[d] = __ldg(sa + d);
+      ms = __ldg((const T *)a.snap_ms + lo);
     }
 
     // the next pinned position at or after the current step (NONE: none left)
@@ -355,15 +360,14 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     //   step u - 2P : the card of u (header, predecessor positions, comm,
     //                 cost row) is copied into cards[u % 2D] by lanes 0..;
     //   step u - P  : the inline predecessors of u at distance > P (and
-    //                 BASE-prefix records, s < t0) are copied into
+    //                 BASE records, s < lo) are copied into
     //                 stage[u % D]; one commit group per step;
     //   step u      : the others were written at most P steps earlier and
     //                 are read from the ring of the last D records.
     // A staged record was stored at least one step before its copy is issued
     // (same thread, program order).  A stage or card slot is overwritten only
     // after the step that read it has consumed the values.
-    // (t0 = 0 unless the candidate shares the BASE prefix, so "s < t0" alone
-    // selects the BASE record; a record is staged iff s < max(t0, u - P))
+    // (a record is staged iff s < max(lo, u - P); s < lo: the BASE record)
     auto copy_card = [&](int32_t u) {
       const uint32_t dst = cards_sa + (uint32_t)((u & (2 * D - 1)) * CS) + cc_dst;
       const char *srcp = cc_cost ? (const char *)(costp + (size_t)u * G) + cc_src
@@ -387,17 +391,17 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       const uint4 su = *(const uint4 *)(cu + 16);
       const uint32_t ss[4] = {su.x, su.y, su.z, su.w};
       const uint32_t sl = stage_sa + (uint32_t)((u & (D - 1)) * 4 * 32 * sizeof(W));
-      const bool on = run && u >= t0;
-      const int32_t thr = t0 > u - P ? t0 : u - P;
+      const bool on = run;
+      const int32_t thr = lo > u - P ? lo : u - P;
 #pragma unroll
       for (int k = 0; k < 4; k++) {
-        const W *gp = (int32_t)ss[k] < t0 ? snap + ss[k] : col + (size_t)ss[k] * 32;
+        const W *gp = (int32_t)ss[k] < lo ? snap + ss[k] : col + (size_t)ss[k] * 32;
         cp_async_if<sizeof(W)>(on && (uint32_t)k < npu && (int32_t)ss[k] < thr, sl + (uint32_t)(k * 32 * sizeof(W)), gp);
       }
     };
     // record of position s < t outside the inline slots (extra predecessors)
     auto rec_at = [&](uint32_t s, int32_t t) -> W {
-      if ((int32_t)s < t0) return snap[s];
+      if ((int32_t)s < lo) return snap[s];
       if ((int32_t)s + P >= t) return ring[(s & (D - 1)) * 32];
       return col[(size_t)s * 32];
     };
@@ -411,7 +415,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       cp_async_commit();
     }
     for (int32_t t = lo; t < n; t++) {
-      const bool live = run && t >= t0;
+      const bool live = run;
       cp_async_wait<P - 1>();  // the group of step t - P: records of t, card of t + P
       __syncwarp();            // (cards were copied by other lanes)
       const unsigned char *cs = cards + (t & (2 * D - 1)) * CS;
@@ -427,7 +431,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       // predecessor records: staged or from the ring (unused slots: garbage, masked)
       W rw[4];
       const W *stg = stage + (t & (D - 1)) * 4 * 32;
-      const int32_t thr = t0 > t - P ? t0 : t - P;
+      const int32_t thr = lo > t - P ? lo : t - P;
 #pragma unroll
       for (int k = 0; k < 4; k++) rw[k] = *((int32_t)src[k] < thr ? stg + k * 32 : ring + (src[k] & (D - 1)) * 32);
       prefetch(t + P);
