@@ -687,15 +687,26 @@ static fastt_status ensure_sort_buf(fastt_graph *g, int64_t n) {
 // launches, each skipping the other kind of slot.
 static void launch_slots(fastt_graph *g, SimArgs b, int tbits, int nc, cudaStream_t st) {
   b.mode = 2;
-  b.lane = 0;
   const int per_block = (g->sim_block / 32) * g->sim_cpw;
-  if (g->use_topo) {
+  if (g->use_topo && b.lane) {
+    // makespan-only evaluation without memory tracking: the multi-graph lane
+    // kernel (one slot per lane, one warp per block) for topological slots
+    b.lane = 2;
+    b.topo = 1;
+    b.slot_filter = 1;
+    launch_sim(b, tbits, (nc + 31) / 32, 32, 0, st);
+    cudaMemsetAsync(b.counter, 0, sizeof(unsigned long long), st);
+    b.lane = 0;
+    b.slot_filter = 2;
+  } else if (g->use_topo) {
+    b.lane = 0;
     b.topo = 1;
     b.slot_filter = 1;
     launch_sim(b, tbits, (int)std::min<int64_t>(g->sim_grid_topo, nc / per_block + 1), g->sim_block, 0, st);
-    cudaMemsetAsync(g->counters, 0, sizeof(unsigned long long), st);
+    cudaMemsetAsync(b.counter, 0, sizeof(unsigned long long), st);
     b.slot_filter = 2;
   } else {
+    b.lane = 0;
     b.slot_filter = 0;
   }
   b.topo = 0;

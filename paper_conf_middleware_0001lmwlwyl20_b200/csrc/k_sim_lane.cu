@@ -53,10 +53,11 @@ template <typename T> __host__ __device__ constexpr int card_cost_off() { return
 template <typename T, int GP> __host__ __device__ constexpr int card_slot_bytes() {
   return card_cost_off<T>() + (int)((GP * sizeof(T) + 15) / 16) * 16;
 }
-template <typename T, int GP> __host__ __device__ constexpr size_t lane_smem_per_warp() {
-  // ring D x 32 + stage D x 4 x 32 records, then 2D staged cards
+template <typename T, int GP, bool MG> __host__ __device__ constexpr size_t lane_smem_per_warp() {
+  // ring D x 32 + stage D x 4 x 32 records, then 2D staged cards (per lane
+  // in the multi-graph variant)
   return (size_t)LaneDepth<T>::D * 5 * 32 * (sizeof(T) == 4 ? 8 : 16) +
-         (size_t)2 * LaneDepth<T>::D * card_slot_bytes<T, GP>();
+         (size_t)(MG ? 32 : 1) * 2 * LaneDepth<T>::D * card_slot_bytes<T, GP>();
 }
 
 template <int BYTES> __device__ __forceinline__ void cp_async(uint32_t saddr, const void *g);
@@ -156,27 +157,30 @@ template <> struct RowLd<uint64_t> {
 //     1 = one link class, comm per edge from pe_comm;
 //     2 = several link classes (per (pred, device) comm).
 // EX: G == GP (no per-device range checks).
-template <typename T, int GSH, int CM, bool EX>
+// MG: multi-graph -- lane l simulates prepared slot q0 + l (mode 2: SPLIT and
+//     rank-changing candidates, each with its own priority order, so cards
+//     are staged per lane); launched with one warp per block.
+template <typename T, int GSH, int CM, bool EX, bool MG>
 __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   typedef typename Slab<T>::W W;
   constexpr int GP = 1 << GSH;
   static_assert(CM != 0 || sizeof(T) == 4, "card comm values are uint32");
   const int lane = threadIdx.x & 31;
-  const int64_t gwarp = (int64_t)blockIdx.x * (LANE_BLOCK / 32) + (threadIdx.x >> 5);
+  const int64_t gwarp = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
   // this lane's slab column: record of position p at col[p * 32]
   W *const col = (W *)a.slab + (size_t)gwarp * (size_t)a.slab_stride * 32 + lane;
   // shared memory of this warp: ring[D][32] (records of the last D positions)
   // and stage[D][4][32] (inline predecessors' records prefetched by cp.async)
   constexpr int D = LaneDepth<T>::D, P = D - 1;
   extern __shared__ __align__(16) unsigned char lsm[];
-  unsigned char *const wsm = lsm + (threadIdx.x >> 5) * lane_smem_per_warp<T, GP>();
+  unsigned char *const wsm = lsm + (threadIdx.x >> 5) * lane_smem_per_warp<T, GP, MG>();
   W *const ring = (W *)wsm + lane;
   W *const stage = ring + D * 32;
   const uint32_t stage_sa = (uint32_t)__cvta_generic_to_shared(stage);
   // 2D staged cards (warp-shared): the card of position u is copied at step
   // u - 2P and read at steps u - P (record prefetch) and u (compute)
   constexpr int CS = card_slot_bytes<T, GP>();
-  const unsigned char *const cards = wsm + (size_t)D * 5 * 32 * sizeof(W);
+  const unsigned char *const cards = wsm + (size_t)D * 5 * 32 * sizeof(W) + (MG ? (size_t)lane * 2 * D * CS : 0);
   const uint32_t cards_sa = (uint32_t)__cvta_generic_to_shared(cards);
   constexpr int CO = card_cost_off<T>();
   const bool row16 = (a.G * (int)sizeof(T)) % 16 == 0;
@@ -190,13 +194,14 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   const GraphConst &gc = *a.gc;
   const int G = a.G;
   const int K = gc.K;
-  const PrepGraph *pg = a.base;
-  const uint32_t *__restrict__ card = pg->card;
-  const T *__restrict__ costp = (const T *)pg->costp;
-  const T *__restrict__ pe_comm = (const T *)pg->pe_comm;
-  const uint32_t *__restrict__ pe_src = pg->pe_src;
-  const uint32_t *__restrict__ posm = pg->pos;
-  const int32_t n = pg->n, Vraw = pg->V, cpl = pg->cp_len;
+  // the graph (per candidate in the multi-graph variant)
+  const PrepGraph *pg = MG ? a.slots : a.base;
+  const uint32_t *card = pg->card;
+  const T *costp = (const T *)pg->costp;
+  const T *pe_comm = (const T *)pg->pe_comm;
+  const uint32_t *pe_src = pg->pe_src;
+  const uint32_t *posm = pg->pos;
+  int32_t n = pg->n, Vraw = pg->V, cpl = pg->cp_len;
   const W *__restrict__ snap = (const W *)a.snap_rec;
   const bool cp_on = (a.flags & 1u) != 0;
   const uint32_t all = all_devices(G);
@@ -208,14 +213,31 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     q0 = __shfl_sync(FULL, q0, 0);
     if ((int64_t)q0 >= a.n) break;
     const int64_t q = (int64_t)q0 + lane;
-    const bool active = q < a.n;
+    bool active = q < a.n;
     Cand c;
     c.kind = 0;
     c.n_pins = 0;
     c.split_op = -1;
     c.dev_mask = 0;
     int64_t res_idx = -1, sidx = q;
-    if (active) {
+    if (MG) {
+      pg = a.slots + (active ? q : (int64_t)q0);
+      card = pg->card;
+      costp = (const T *)pg->costp;
+      pe_comm = (const T *)pg->pe_comm;
+      pe_src = pg->pe_src;
+      posm = pg->pos;
+      n = pg->n;
+      Vraw = pg->V;
+      cpl = pg->cp_len;
+      if (active) {
+        c = a.cands[q];
+        res_idx = a.slot_result ? a.slot_result[q] : -1;
+        sidx = a.slot_index ? a.slot_index[q] : q;
+        if (a.slot_filter == 1 && !pg->topo) active = false;  // (the ready-set launch takes it)
+      }
+      if (!active) n = 0;
+    } else if (active) {
       if (a.mode == 0) {
         sidx = a.first + q * a.stride;
         c = stream_cand(a.stream, sidx);
@@ -233,7 +255,9 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     int np = 0;
     uint8_t st = 0;
     bool defer = false;
-    if (active) {
+    if (MG) {
+      np = (active && c.kind == 1) ? c.n_pins : 0;  // (validated by the main launch)
+    } else if (active) {
       if (c.dev_mask & ~all) st = 2;
       else if (c.dev_mask && c.dev_mask != all) defer = true;  // device subset (R25): own ranks
       if (st) {
@@ -274,7 +298,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
         pdv |= (uint32_t)c.pin_dev[k] << (8 * k);
       }
     // pins that change w or c (R5) need the candidate's own ranks
-    if (active && !defer)
+    if (!MG && active && !defer)
       for (int k = 0; k < np && !defer; k++)
         defer = pin_changes_ranks<T>(pg, gc, c, np, pp[k], c.pin_dev[k], G, K);
     if (active && defer) {
@@ -292,6 +316,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     // round over the free CP ops (perturbation-pinned CP ops excluded)
     int r_dev = -1;
     int m = 0;
+    const uint32_t dmask = (MG && c.dev_mask) ? c.dev_mask : all;  // the candidate's devices (R25)
     if (run && cp_on && cpl > 0) {
       uint32_t pc[MAXPINS];
 #pragma unroll
@@ -302,6 +327,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       if (cpl - m > 0) {
         int64_t bs = 0;
         for (int d = 0; d < G; d++) {
+          if (MG && !((dmask >> d) & 1u)) continue;
           int64_t s = pg->pcost[(int64_t)cpl * G + d];
 #pragma unroll
           for (int k = 0; k < MAXPINS; k++)
@@ -317,7 +343,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     // no caps => the BASE schedule up to the first pinned op's step t0
     int32_t t0 = 0;
     bool share = false;
-    if (run && a.snap_mode == 2) {
+    if (!MG && run && a.snap_mode == 2) {
       share = m == 0 || (a.snap_round_dev >= 0 && r_dev == a.snap_round_dev);
       if (share) {
         t0 = n;
@@ -332,11 +358,15 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     // BASE state at any step <= its t0 makes the BASE decisions up to t0, so
     // all lanes may start at lo; positions before lo hold BASE records.
     int32_t lo = run ? t0 : n;
+    int32_t nmax = run ? n : 0;  // steps of the warp (MG: the longest slot)
 #pragma unroll
     for (int o = 16; o >= 1; o >>= 1) {
       const int32_t x = __shfl_xor_sync(FULL, lo, o);
       lo = x < lo ? x : lo;
+      const int32_t y = __shfl_xor_sync(FULL, nmax, o);
+      nmax = y > nmax ? y : nmax;
     }
+    if (MG) lo = 0;
     T avail[GP];
     T ms = 0;
 #pragma unroll
@@ -369,6 +399,22 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     // after the step that read it has consumed the values.
     // (a record is staged iff s < max(lo, u - P); s < lo: the BASE record)
     auto copy_card = [&](int32_t u) {
+      if (MG) {  // this lane's own card: header, predecessors, comm, cost row
+        if (u < n) {
+          const uint32_t dst = cards_sa + (uint32_t)((u & (2 * D - 1)) * CS);
+          const char *cu = (const char *)(card + (size_t)u * CARD_WORDS);
+          const char *row = (const char *)(costp + (size_t)u * G);
+          cp_async<16>(dst, cu);
+          cp_async<16>(dst + 16, cu + 4 * CARD_HDR);
+          if (CM == 0) cp_async<16>(dst + 32, cu + 4 * CW_PCOMM);
+          if (row16) {
+            for (int j = 0; j < G * (int)sizeof(T) / 16; j++) cp_async<16>(dst + CO + 16 * j, row + 16 * j);
+          } else {
+            for (int j = 0; j < G; j++) cp_async<sizeof(T)>(dst + CO + j * sizeof(T), row + j * sizeof(T));
+          }
+        }
+        return;
+      }
       const uint32_t dst = cards_sa + (uint32_t)((u & (2 * D - 1)) * CS) + cc_dst;
       const char *srcp = cc_cost ? (const char *)(costp + (size_t)u * G) + cc_src
                                  : (const char *)(card + (size_t)u * CARD_WORDS) + cc_src;
@@ -384,10 +430,13 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       const unsigned char *cu = cards + (u & (2 * D - 1)) * CS;
       const uint4 hu = *(const uint4 *)cu;
       const uint32_t npu = u < n ? (hu.x & 0xFFFF) : 0u;
-      if (CM == 1)  // the inline predecessors' comm values (warp-uniform card)
+      if (CM == 1 && !MG)  // the inline predecessors' comm values (warp-uniform card)
         cp_async_if<sizeof(T)>((uint32_t)lane < npu && lane < 4,
                                cards_sa + (uint32_t)((u & (2 * D - 1)) * CS + 32 + (lane & 3) * sizeof(T)),
                                pe_comm + hu.y + (lane & 3));
+      if (CM == 1 && MG)  // (this lane's card)
+        for (uint32_t k = 0; k < npu && k < 4; k++)
+          cp_async<sizeof(T)>(cards_sa + (uint32_t)((u & (2 * D - 1)) * CS + 32 + k * sizeof(T)), pe_comm + hu.y + k);
       const uint4 su = *(const uint4 *)(cu + 16);
       const uint32_t ss[4] = {su.x, su.y, su.z, su.w};
       const uint32_t sl = stage_sa + (uint32_t)((u & (D - 1)) * 4 * 32 * sizeof(W));
@@ -414,8 +463,8 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       prefetch(u);
       cp_async_commit();
     }
-    for (int32_t t = lo; t < n; t++) {
-      const bool live = run;
+    for (int32_t t = lo; t < nmax; t++) {
+      const bool live = run && (!MG || t < n);
       cp_async_wait<P - 1>();  // the group of step t - P: records of t, card of t + P
       __syncwarp();            // (cards were copied by other lanes)
       const unsigned char *cs = cards + (t & (2 * D - 1)) * CS;
@@ -426,7 +475,8 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       const T *cm1 = (const T *)(cs + 32);  // CM 1: staged comm values
       T cst[GP];
       RowLd<T>::template load_s<GP>((const T *)(cs + CO), G, cst);
-      const uint32_t npred = h0.x & 0xFFFF;
+      // (MG: a lane past its slot's last position reads a stale card)
+      const uint32_t npred = (!MG || live) ? (h0.x & 0xFFFF) : 0u;
       const uint32_t src[4] = {hs.x, hs.y, hs.z, hs.w};
       // predecessor records: staged or from the ring (unused slots: garbage, masked)
       W rw[4];
@@ -532,7 +582,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       for (int d = 0; d < GP; d++) {
         const T arr = CM == 2 ? arrd[d] : ((uint32_t)d == pa ? E : M);
         const T est = avail[d] > arr ? avail[d] : arr;
-        eft[d] = (EX || d < G) ? est + cst[d] : TT<T>::MAXV;
+        eft[d] = ((EX || d < G) && (!MG || ((dmask >> d) & 1u))) ? est + cst[d] : TT<T>::MAXV;
       }
       T best = eft[0];
       int bd = 0;
@@ -606,40 +656,44 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   }
 }
 
-template <typename T, int CM, bool EX>
+template <typename T, int CM, bool EX, bool MG>
 static const void *lane_fn_t(int gshift) {
   switch (gshift) {
-    case 0: return (const void *)k_sim_lane<T, 0, CM, EX>;
-    case 1: return (const void *)k_sim_lane<T, 1, CM, EX>;
-    case 2: return (const void *)k_sim_lane<T, 2, CM, EX>;
-    case 3: return (const void *)k_sim_lane<T, 3, CM, EX>;
-    case 4: return (const void *)k_sim_lane<T, 4, CM, EX>;
-    default: return (const void *)k_sim_lane<T, 5, CM, EX>;
+    case 0: return (const void *)k_sim_lane<T, 0, CM, EX, MG>;
+    case 1: return (const void *)k_sim_lane<T, 1, CM, EX, MG>;
+    case 2: return (const void *)k_sim_lane<T, 2, CM, EX, MG>;
+    case 3: return (const void *)k_sim_lane<T, 3, CM, EX, MG>;
+    case 4: return (const void *)k_sim_lane<T, 4, CM, EX, MG>;
+    default: return (const void *)k_sim_lane<T, 5, CM, EX, MG>;
   }
 }
-template <bool EX> static const void *lane_fn_x(int tbits, int gshift, int cm) {
+template <bool EX, bool MG> static const void *lane_fn_x(int tbits, int gshift, int cm) {
   if (tbits == 32) {
-    if (cm == 0) return lane_fn_t<uint32_t, 0, EX>(gshift);
-    return cm == 1 ? lane_fn_t<uint32_t, 1, EX>(gshift) : lane_fn_t<uint32_t, 2, EX>(gshift);
+    if (cm == 0) return lane_fn_t<uint32_t, 0, EX, MG>(gshift);
+    return cm == 1 ? lane_fn_t<uint32_t, 1, EX, MG>(gshift) : lane_fn_t<uint32_t, 2, EX, MG>(gshift);
   }
-  return cm == 2 ? lane_fn_t<uint64_t, 2, EX>(gshift) : lane_fn_t<uint64_t, 1, EX>(gshift);
+  return cm == 2 ? lane_fn_t<uint64_t, 2, EX, MG>(gshift) : lane_fn_t<uint64_t, 1, EX, MG>(gshift);
 }
-static const void *lane_fn(int tbits, int gshift, int cm, bool exact) {
-  return exact ? lane_fn_x<true>(tbits, gshift, cm) : lane_fn_x<false>(tbits, gshift, cm);
+static const void *lane_fn(int tbits, int gshift, int cm, bool exact, bool mg) {
+  if (mg) return exact ? lane_fn_x<true, true>(tbits, gshift, cm) : lane_fn_x<false, true>(tbits, gshift, cm);
+  return exact ? lane_fn_x<true, false>(tbits, gshift, cm) : lane_fn_x<false, false>(tbits, gshift, cm);
 }
 
-template <typename T> static size_t lane_smem_t(int gshift) {
+template <typename T, bool MG> static size_t lane_smem_t(int gshift) {
   switch (gshift) {
-    case 0: return lane_smem_per_warp<T, 1>();
-    case 1: return lane_smem_per_warp<T, 2>();
-    case 2: return lane_smem_per_warp<T, 4>();
-    case 3: return lane_smem_per_warp<T, 8>();
-    case 4: return lane_smem_per_warp<T, 16>();
-    default: return lane_smem_per_warp<T, 32>();
+    case 0: return lane_smem_per_warp<T, 1, MG>();
+    case 1: return lane_smem_per_warp<T, 2, MG>();
+    case 2: return lane_smem_per_warp<T, 4, MG>();
+    case 3: return lane_smem_per_warp<T, 8, MG>();
+    case 4: return lane_smem_per_warp<T, 16, MG>();
+    default: return lane_smem_per_warp<T, 32, MG>();
   }
 }
-size_t lane_smem(int tbits, int gshift) {
-  return (LANE_BLOCK / 32) * (tbits == 32 ? lane_smem_t<uint32_t>(gshift) : lane_smem_t<uint64_t>(gshift));
+// dynamic shared memory of a block: LANE_BLOCK threads, or one warp (MG)
+size_t lane_smem(int tbits, int gshift, bool mg) {
+  if (mg) return tbits == 32 ? lane_smem_t<uint32_t, true>(gshift) : lane_smem_t<uint64_t, true>(gshift);
+  return (LANE_BLOCK / 32) *
+         (tbits == 32 ? lane_smem_t<uint32_t, false>(gshift) : lane_smem_t<uint64_t, false>(gshift));
 }
 
 int lane_comm_mode(const SimArgs &a, int tbits) {
@@ -647,19 +701,24 @@ int lane_comm_mode(const SimArgs &a, int tbits) {
   return a.gc_K == 1 ? 1 : 2;
 }
 
+// a.lane: 1 = candidates of the base graph (LANE_BLOCK threads per block),
+// 2 = prepared slots, one per lane (one warp per block; grid = warps)
 void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
-  const void *f = lane_fn(tbits, a.gshift, lane_comm_mode(a, tbits), a.G == (1 << a.gshift));
+  const bool mg = a.lane == 2;
+  const void *f = lane_fn(tbits, a.gshift, lane_comm_mode(a, tbits), a.G == (1 << a.gshift), mg);
+  const size_t sm = lane_smem(tbits, a.gshift, mg);
+  if (mg) cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
   SimArgs aa = a;
   void *args[] = {&aa};
-  cudaLaunchKernel(f, dim3(grid), dim3(LANE_BLOCK), args, lane_smem(tbits, a.gshift), st);
+  cudaLaunchKernel(f, dim3(grid), dim3(mg ? 32 : LANE_BLOCK), args, sm, st);
 }
 
 int lane_occupancy(int tbits, int gshift) {
   int nb = 1 << 30, x = 0;
   for (int v = (tbits == 32 ? 0 : 2); v < 6; v++) {
-    const void *f = lane_fn(tbits, gshift, v >> 1, v & 1);
-    cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lane_smem(tbits, gshift));
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, f, LANE_BLOCK, lane_smem(tbits, gshift));
+    const void *f = lane_fn(tbits, gshift, v >> 1, v & 1, false);
+    cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lane_smem(tbits, gshift, false));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, f, LANE_BLOCK, lane_smem(tbits, gshift, false));
     nb = x < nb ? x : nb;
   }
   return nb;
