@@ -13,9 +13,11 @@ one NCCL all_reduce(MIN) pair picks the winner (weak scaling).
           launching stream, max over ranks), inputs resident in HBM
   e2e     the same metric through fastt_schedule_batch with HOST (pinned)
           candidate and result buffers, copies inside the timed region
-  roofline  dominant kernel = the simulation kernel k_sim: algorithmic bytes
-          B_alg = V*(8G+45) + 29E per candidate x candidates of
-          the launch / its CUDA-event duration, vs MEASURED_PEAKS hbm_gbs
+  roofline  dominant kernel = the simulation kernel k_sim_lane (sweep launch),
+          bound "alu": algorithmic int32 ops V(8G+2) + 7E per candidate x
+          candidates of the launch / its CUDA-event duration, vs 148 SMs x
+          128 int32 lanes/clk x max SM clock; the touched-once
+          HBM figure (B_state + B_graph/32) rides along under roofline.hbm
   cpu_baseline  the plain C oracle on a bounded strided sample of the same
           stream, all host cores (one oracle call per candidate per thread)
 
@@ -57,6 +59,31 @@ def b_alg_lane(V, E, G):
     B_state + B_graph / 32 with SURVEY 8(d)'s B_state = 21V + 13E and
     B_graph = V(8G + 24) + 16E."""
     return 21 * V + 13 * E + (V * (8 * G + 24) + 16 * E) / 32.0
+
+
+def alu_ops_lane(V, E, G):
+    """Algorithmic int32 ALU operations of one candidate's DPOS evaluation on
+    the lane kernel's (exact, single-link-class) EST form (DESIGN.md section
+    5, "ALU roofline"): per predecessor edge 7 (arrival FT + c, running max,
+    argmax device, co-located select, E max), per op-step and device 8
+    (arrival select, max with avail, + cost, argmin compare + 2 selects,
+    avail update), + 2 per op-step (makespan max, record pack); V' = V op-steps
+    per PIN candidate, counted in full even where the BASE prefix is reused."""
+    return V * (8 * G + 2) + 7 * E
+
+
+def alu_peak_tops():
+    """int32 lanes/s: 148 SMs x 4 SMSPs x (alu pipe + fma pipe, 16 lanes/clk
+    each: rt_SMSP = 2 cycles per warp instruction, B300_MICROARCH.md "Pipe
+    rates") x the max SM clock of MEASURED_PEAKS.json."""
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            mhz = float(json.load(f)["sm_max_mhz"])
+        src = "derived: 148 SMs x 128 int32 lanes/clk (alu+fma pipes) x sm_max_mhz of MEASURED_PEAKS.json"
+    except Exception:
+        mhz = 1965.0
+        src = "derived: 148 SMs x 128 int32 lanes/clk (alu+fma pipes) x 1965 MHz (fallback clock)"
+    return 148 * 4 * 2 * 16 * mhz * 1e6 / 1e12, src
 
 
 def peaks():
@@ -279,7 +306,7 @@ def main():
     prep_ms = statistics.mean(x["ms_prep"] for x in tms)
     lane = tms[-1].get("topo", 0) == 2
     bpc = b_alg_lane(V, E, G) if lane else b_alg(V, E, G)
-    achieved = bpc * fast / (sim_ms / 1000.0) / 1e9
+    hbm_gbs = bpc * fast / (sim_ms / 1000.0) / 1e9
     peak, peak_src = peaks()
     traffic = None
     try:
@@ -288,6 +315,23 @@ def main():
         traffic = tj["dram_bytes_per_candidate"] * fast
     except Exception:
         traffic = None
+    if lane:
+        # ncu (profiles/r01d_ncu_k_sim_lane_full.json): alu pipe 80 % busy,
+        # DRAM 21 % of peak -> the kernel is bound by integer ALU issue
+        opc = alu_ops_lane(V, E, G)
+        achieved = opc * fast / (sim_ms / 1000.0) / 1e12
+        apeak, apeak_src = alu_peak_tops()
+        roof = {"bound": "alu", "achieved": achieved, "peak": apeak, "unit": "Tops/s (int32)",
+                "frac": achieved / apeak, "traffic": traffic, "peak_source": apeak_src,
+                "ops_per_candidate": opc,
+                "hbm": {"achieved_gbs_touched_once": hbm_gbs, "peak_gbs": peak, "peak_source": peak_src,
+                        "bytes_per_candidate_touched_once": bpc,
+                        "dram_gbs_ncu": (traffic / (sim_ms / 1000.0) / 1e9) if traffic else None}}
+    else:
+        roof = {"bound": "hbm", "achieved": hbm_gbs, "peak": peak, "unit": "GB/s", "frac": hbm_gbs / peak,
+                "traffic": traffic, "peak_source": peak_src, "bytes_per_candidate": bpc}
+    roof.update({"kernel": ("k_sim_lane" if lane else "k_sim") + "<uint32_t> (sweep launch)",
+                 "candidates_per_launch": fast, "launch_ms": sim_ms, "prep_ms_per_step": prep_ms})
     launches = sum(x["launches"] for x in tms)
 
     # end to end through the public API with host buffers
@@ -340,14 +384,7 @@ def main():
                        "l2": "per-warp state slabs (>1 GB) exceed L2; a 256 MB buffer is written between steps",
                        "parallelism": "candidates sharded c = rank mod N; NCCL all_reduce(MIN) argmin"},
             "best": {"makespan_ns": best[0], "index": best[1]},
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                         "traffic": traffic,
-                         "kernel": ("k_sim_lane" if lane else "k_sim") + "<uint32_t> (sweep launch)",
-                         "peak_source": peak_src,
-                         "bytes_per_candidate": bpc, "bytes_per_candidate_survey": b_alg(V, E, G),
-                         "candidates_per_launch": fast,
-                         "launch_ms": sim_ms, "prep_ms_per_step": prep_ms,
-                         "note": "latency-bound sequential list scheduling; frac is of the measured copy bandwidth"},
+            "roofline": roof,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": launches,
