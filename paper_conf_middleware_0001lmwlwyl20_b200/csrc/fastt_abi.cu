@@ -183,6 +183,9 @@ struct Base {
   int tbits = 64, key_bits = 64;
   int topo = 0;  // the prepared priority order is topological (k_sim's TOPO path)
   unsigned long long bound = 0, maxextra = 0;
+  // packed device keys of the lane kernel (32-bit time, one link class)
+  uint32_t *costk = nullptr;
+  uint32_t pk_lim = 0;
   // recorded BASE schedule for prefix sharing, per CP-pin flag value
   struct Snap {
     bool valid = false;
@@ -197,6 +200,9 @@ struct Base {
     cudaFree(raw_dev);
     cudaFree(prep_block);
     cudaFree(pg_dev);
+    cudaFree(costk);
+    costk = nullptr;
+    pk_lim = 0;
     for (auto &x : snap) {
       cudaFree(x.buf);
       x = Snap();
@@ -250,6 +256,8 @@ struct fastt_graph {
   int sim_grid_topo = 0;  // resident blocks of the TOPO variant (no shared-memory ready set)
   bool use_topo = true;   // FASTT_NO_TOPO=1 forces the ready-set path (A/B parity)
   int sim_grid_lane = 0;  // resident blocks of the lane-per-candidate position-order kernel
+  bool use_pk = true;      // FASTT_NO_PK=1: the lane kernel without packed device keys (A/B parity)
+  uint32_t pk_lim_cap = 0xFFFFFFFFu;  // FASTT_PK_LIM=<ns>: lower the deferral bound (tests of the deferral path)
   bool use_lane = true;   // FASTT_NO_LANE=1 keeps position-order launches on the group kernel (A/B parity)
   int last_topo = 0;      // the last main launch: 0 ready-set kernel, 1 group position-order, 2 lane position-order
   int64_t sim_ncap = 0;
@@ -379,6 +387,22 @@ static fastt_status prepare_base(fastt_graph *g, Base &B, cudaStream_t st) {
   B.n = P.n;
   B.cp_len = P.cp_len;
   B.topo = P.topo;
+  // packed keys (k_sim_lane PK): the bound below which no key wraps
+  if (g->use_pk && B.tbits == 32 && g->K == 1 && B.n > 0) {
+    int gsh = 0;
+    while ((1 << gsh) < g->G) gsh++;
+    CK(cudaMalloc(&B.costk, sizeof(uint32_t) * (size_t)B.n * g->G));
+    unsigned long long *d_m = nullptr, hm[2];
+    CK(cudaMalloc(&d_m, 16));
+    CK(cudaMemsetAsync(d_m, 0, 16, st));
+    launch_pack_costs(B.pg_dev, B.n, g->G, gsh, P.E, B.costk, d_m, st);
+    CK(cudaGetLastError());
+    CK(cudaMemcpyAsync(hm, d_m, 16, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    cudaFree(d_m);
+    const long long lim = (1ll << (32 - gsh)) - (long long)hm[0] - (long long)hm[1];
+    B.pk_lim = lim > 0 ? (uint32_t)std::min<long long>(lim, (long long)g->pk_lim_cap) : 0u;
+  }
   return FASTT_OK;
 }
 
@@ -553,6 +577,8 @@ static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
     if (g->gch.cap[d] != I64MAX) a.cap_check = 1;
   a.need_mem = a.cap_check;
   a.fastcomm = B.tbits == 32 && g->K == 1;
+  a.costk = B.costk;
+  a.pk_lim = B.pk_lim;
   if (flags & FASTT_F_MEM_LIVE) {
     a.live_mem = 1;
     a.need_mem = 1;
@@ -1139,6 +1165,10 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     g->use_topo = !(e && e[0] == '1');
     e = getenv("FASTT_NO_LANE");
     g->use_lane = !(e && e[0] == '1');
+    e = getenv("FASTT_NO_PK");
+    g->use_pk = !(e && e[0] == '1');
+    e = getenv("FASTT_PK_LIM");
+    if (e && e[0]) g->pk_lim_cap = (uint32_t)std::max(1ll, std::min(0xFFFFFFFFll, atoll(e)));
   }
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || cuda_device < 0 || cuda_device >= ndev) {

@@ -224,6 +224,11 @@ struct SimArgs {
   void *gap;
   int64_t gap_stride;
   int32_t ins_grid;
+  // packed device keys of the lane kernel (k_sim_lane PK): cost rows
+  // (cost << gshift) | d of the base graph, and the makespan at or above
+  // which a candidate is deferred (0 = packed keys off)
+  const uint32_t *costk;
+  uint32_t pk_lim;
 };
 
 // one idle slot [a, b) of a device under INSERT
@@ -251,6 +256,10 @@ void launch_gather_sorted(const Cand *src, const int64_t *sidx, const int64_t *s
 int sim_occupancy(int tbits, int gshift, int block, size_t smem, bool topo);
 void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st);
 int lane_occupancy(int tbits, int gshift);
+// costk[p][d] = (cost[p][d] << gshift) | d over n positions; mx[0] = max
+// cost, mx[1] = max edge comm (one link class) of the prepared graph
+void launch_pack_costs(const PrepGraph *pg_dev, int32_t n, int G, int gshift, int64_t E, uint32_t *costk,
+                       unsigned long long *mx, cudaStream_t st);
 void launch_fit(int G, int64_t n, const uint8_t *src, const uint8_t *dst, const int64_t *bytes, const int64_t *tns,
                 void *sums, unsigned *err, int64_t *alpha, int64_t *beta, int64_t *count, int sms, cudaStream_t st);
 size_t fit_sums_bytes(int G);

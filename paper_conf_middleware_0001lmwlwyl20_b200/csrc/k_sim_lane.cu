@@ -53,11 +53,19 @@ template <typename T> __host__ __device__ constexpr int card_cost_off() { return
 template <typename T, int GP> __host__ __device__ constexpr int card_slot_bytes() {
   return card_cost_off<T>() + (int)((GP * sizeof(T) + 15) / 16) * 16;
 }
+// MG: per-lane card regions are 2D slots + 16 B apart, so the 8 lanes of a
+// 128-bit shared-memory phase hit distinct bank quads (a 2D x CS stride is a
+// multiple of 128 B: every lane's card load would fall in the same banks)
+template <typename T, int GP> __host__ __device__ constexpr int mg_lane_stride() {
+  return 2 * LaneDepth<T>::D * card_slot_bytes<T, GP>() + 16;
+}
 template <typename T, int GP, bool MG> __host__ __device__ constexpr size_t lane_smem_per_warp() {
   // ring D x 32 + stage D x 4 x 32 records, then 2D staged cards (per lane
-  // in the multi-graph variant)
+  // in the multi-graph variant), then (base-graph launches) the packed-key
+  // avail rows [32 lanes][GP] of the PK variant
   return (size_t)LaneDepth<T>::D * 5 * 32 * (sizeof(T) == 4 ? 8 : 16) +
-         (size_t)(MG ? 32 : 1) * 2 * LaneDepth<T>::D * card_slot_bytes<T, GP>();
+         (MG ? (size_t)32 * mg_lane_stride<T, GP>() : (size_t)2 * LaneDepth<T>::D * card_slot_bytes<T, GP>()) +
+         (size_t)(MG ? 0 : 32 * GP * 4);
 }
 
 template <int BYTES> __device__ __forceinline__ void cp_async(uint32_t saddr, const void *g);
@@ -160,10 +168,22 @@ template <> struct RowLd<uint64_t> {
 // MG: multi-graph -- lane l simulates prepared slot q0 + l (mode 2: SPLIT and
 //     rank-changing candidates, each with its own priority order, so cards
 //     are staged per lane); launched with one warp per block.
-template <typename T, int GSH, int CM, bool EX, bool MG>
+// PK: packed device keys (32-bit time, one link class, base graph): the EFT
+//     of device d is carried as the key (EFT << GSH) | d, so the argmin with
+//     ties to the lowest device (Alg. 1 lines 12-19, R3) is a plain unsigned
+//     min (3-input VIMNMX3), the cost row is pre-packed (costk = cost << GSH
+//     | d), avail[d] << GSH lives in a per-lane shared-memory row so the
+//     chosen device's update and the arrival on the predecessor device pa
+//     (R6) are one indexed store / load instead of a select per device.
+//     Exact while every key fits 32 bits: EFT <= makespan + max comm + max
+//     cost at every step, so a candidate whose final makespan reaches
+//     pk_lim = 2^(32-GSH) - max cost - max comm is deferred and re-run by the
+//     preparation pipeline (unpacked kernels).
+template <typename T, int GSH, int CM, bool EX, bool MG, bool PK>
 __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   typedef typename Slab<T>::W W;
   constexpr int GP = 1 << GSH;
+  static_assert(!PK || (sizeof(T) == 4 && CM != 2 && !MG), "packed keys: 32-bit time, one link class, base graph");
   static_assert(CM != 0 || sizeof(T) == 4, "card comm values are uint32");
   const int lane = threadIdx.x & 31;
   const int64_t gwarp = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
@@ -180,8 +200,14 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   // 2D staged cards (warp-shared): the card of position u is copied at step
   // u - 2P and read at steps u - P (record prefetch) and u (compute)
   constexpr int CS = card_slot_bytes<T, GP>();
-  const unsigned char *const cards = wsm + (size_t)D * 5 * 32 * sizeof(W) + (MG ? (size_t)lane * 2 * D * CS : 0);
+  const unsigned char *const cards = wsm + (size_t)D * 5 * 32 * sizeof(W) + (MG ? (size_t)lane * mg_lane_stride<T, GP>() : 0);
   const uint32_t cards_sa = (uint32_t)__cvta_generic_to_shared(cards);
+  // PK: avail[d] << GSH of every lane, after the warp's cards, as device
+  // pairs [d / 2][32 lanes][2] (a pair per lane is one 64-bit access; the
+  // indexed access of device d by all lanes is 2-way conflicted at most)
+  uint32_t *const avk = (uint32_t *)(wsm + (size_t)D * 5 * 32 * sizeof(W) + (size_t)2 * D * card_slot_bytes<T, GP>()) +
+                        (GP >= 2 ? 2 * lane : lane);
+  auto avk_at = [&](uint32_t d) -> uint32_t & { return GP >= 2 ? avk[(d >> 1) * 64 + (d & 1)] : avk[0]; };
   constexpr int CO = card_cost_off<T>();
   const bool row16 = (a.G * (int)sizeof(T)) % 16 == 0;
   // this lane's 16-B chunk of a card copy: lane 0 header (words 0-3), lane 1
@@ -198,6 +224,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   const PrepGraph *pg = MG ? a.slots : a.base;
   const uint32_t *card = pg->card;
   const T *costp = (const T *)pg->costp;
+  const T *costsrc = PK ? (const T *)a.costk : costp;  // the cost rows staged with the cards
   const T *pe_comm = (const T *)pg->pe_comm;
   const uint32_t *pe_src = pg->pe_src;
   const uint32_t *posm = pg->pos;
@@ -378,6 +405,10 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
         if (d < G) avail[d] = __ldg(sa + d);
       ms = __ldg((const T *)a.snap_ms + lo);
     }
+    if (PK) {
+#pragma unroll
+      for (int d = 0; d < GP; d++) avk_at(d) = (uint32_t)avail[d] << GSH;
+    }
 
     // the next pinned position at or after the current step (NONE: none left)
     uint32_t nxt = NONE;
@@ -416,14 +447,14 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
         return;
       }
       const uint32_t dst = cards_sa + (uint32_t)((u & (2 * D - 1)) * CS) + cc_dst;
-      const char *srcp = cc_cost ? (const char *)(costp + (size_t)u * G) + cc_src
+      const char *srcp = cc_cost ? (const char *)(costsrc + (size_t)u * G) + cc_src
                                  : (const char *)(card + (size_t)u * CARD_WORDS) + cc_src;
       if (row16) cp_async_if<16>(cc_on && u < n, dst, srcp);
       else {
         cp_async_if<16>(cc_on && !cc_cost && u < n, dst, srcp);
         for (int j = lane; j < G; j += 32)
           cp_async_if<sizeof(T)>(u < n, cards_sa + (uint32_t)((u & (2 * D - 1)) * CS + CO + j * sizeof(T)),
-                                 costp + (size_t)u * G + j);
+                                 costsrc + (size_t)u * G + j);
       }
     };
     auto prefetch = [&](int32_t u) {  // records of step u (its card is staged)
@@ -575,6 +606,64 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
           arrd[d] = v;
         }
       }
+      if (PK) {
+        // keys (EFT << GSH) | d: EST = max(avail[d], arrival),
+        // arrival M on every device but pa, E on pa (R6); min key = EFT
+        // argmin with ties to the lowest device (Alg. 1 lines 12-19, R3)
+        const uint32_t Mk = (uint32_t)M << GSH, Ek = (uint32_t)E << GSH;
+        uint32_t av[GP];
+        if (GP >= 2) {
+#pragma unroll
+          for (int j = 0; j < GP / 2; j++) {
+            const uint2 x = *(const uint2 *)(avk + j * 64);
+            av[2 * j] = x.x;
+            av[2 * j + 1] = x.y;
+          }
+        } else {
+          av[0] = avk[0];
+        }
+        const uint32_t pq = pa & (uint32_t)(GP - 1);
+        const uint32_t ap = avk_at(pq), cpa = ((const uint32_t *)(cs + CO))[pq];
+        uint32_t kpa = (ap > Ek ? ap : Ek) + cpa;
+        if (!EX && pq >= (uint32_t)G) kpa = 0xFFFFFFFFu;
+        uint32_t key[GP];
+#pragma unroll
+        for (int d = 0; d < GP; d++)
+          key[d] = (EX || d < G) ? (av[d] > Mk ? av[d] : Mk) + (uint32_t)cst[d] : 0xFFFFFFFFu;
+        uint32_t bk = kpa;
+#pragma unroll
+        for (int d = 0; d < GP; d++) bk = key[d] < bk ? key[d] : bk;
+        // device forced by a perturbation pin (hard) or a CP pin (Alg. 1
+        // l.9-10): rare steps
+        if (__any_sync(FULL, (uint32_t)t == nxt || (h0.w != NONE && r_dev >= 0))) {
+          int forced = -1;
+          if ((uint32_t)t == nxt) {
+            nxt = NONE;
+#pragma unroll
+            for (int k = 0; k < MAXPINS; k++) {
+              if (pp[k] == (uint32_t)t) forced = (int)((pdv >> (8 * k)) & 0xFFu);
+              else if (pp[k] > (uint32_t)t && pp[k] < nxt) nxt = pp[k];
+            }
+          }
+          if (forced < 0 && r_dev >= 0 && h0.w != NONE) forced = r_dev;
+          if (forced >= 0) {
+#pragma unroll
+            for (int d = 0; d < GP; d++)
+              if (d == forced) bk = key[d];
+            if ((uint32_t)forced == pq && kpa < bk) bk = kpa;
+          }
+        }
+        if (live) {
+          const uint32_t bkc = bk & ~(uint32_t)(GP - 1);
+          avk_at(bk & (uint32_t)(GP - 1)) = bkc;
+          const T best = (T)(bkc >> GSH);
+          ms = best > ms ? best : ms;
+          W w;
+          Slab<T>::make(w, best, bk & (uint32_t)(GP - 1));
+          col[(size_t)t * 32] = w;
+          ring[(t & (D - 1)) * 32] = w;
+        }
+      } else {
       // EFT per device; argmin with ties to the lowest device
       // (Alg. 1 lines 12-19, R3); devices >= G are never chosen
       T eft[GP];
@@ -622,11 +711,15 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
         col[(size_t)t * 32] = w;
         ring[(t & (D - 1)) * 32] = w;
       }
+      }  // !PK
     }
     cp_async_wait<0>();  // (no copy may land in the stage after this candidate)
 
     // ------------------------------------------------------------ epilogue
-    if (run) {
+    if (PK && run && (uint32_t)ms >= a.pk_lim) {  // a key may have wrapped: re-run unpacked
+      const unsigned long long k = atomicAdd(a.ndefer, 1ull);
+      a.defer_q[k] = q;
+    } else if (run) {
       if (res_idx >= 0) {
         a.out.makespan[res_idx] = (int64_t)ms;
         a.out.status[res_idx] = 0;
@@ -656,27 +749,29 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   }
 }
 
-template <typename T, int CM, bool EX, bool MG>
+template <typename T, int CM, bool EX, bool MG, bool PK = false>
 static const void *lane_fn_t(int gshift) {
   switch (gshift) {
-    case 0: return (const void *)k_sim_lane<T, 0, CM, EX, MG>;
-    case 1: return (const void *)k_sim_lane<T, 1, CM, EX, MG>;
-    case 2: return (const void *)k_sim_lane<T, 2, CM, EX, MG>;
-    case 3: return (const void *)k_sim_lane<T, 3, CM, EX, MG>;
-    case 4: return (const void *)k_sim_lane<T, 4, CM, EX, MG>;
-    default: return (const void *)k_sim_lane<T, 5, CM, EX, MG>;
+    case 0: return (const void *)k_sim_lane<T, 0, CM, EX, MG, PK>;
+    case 1: return (const void *)k_sim_lane<T, 1, CM, EX, MG, PK>;
+    case 2: return (const void *)k_sim_lane<T, 2, CM, EX, MG, PK>;
+    case 3: return (const void *)k_sim_lane<T, 3, CM, EX, MG, PK>;
+    case 4: return (const void *)k_sim_lane<T, 4, CM, EX, MG, PK>;
+    default: return (const void *)k_sim_lane<T, 5, CM, EX, MG, PK>;
   }
 }
-template <bool EX, bool MG> static const void *lane_fn_x(int tbits, int gshift, int cm) {
+template <bool EX, bool MG> static const void *lane_fn_x(int tbits, int gshift, int cm, bool pk) {
   if (tbits == 32) {
+    if (!MG && pk && cm != 2)
+      return cm == 0 ? lane_fn_t<uint32_t, 0, EX, false, true>(gshift) : lane_fn_t<uint32_t, 1, EX, false, true>(gshift);
     if (cm == 0) return lane_fn_t<uint32_t, 0, EX, MG>(gshift);
     return cm == 1 ? lane_fn_t<uint32_t, 1, EX, MG>(gshift) : lane_fn_t<uint32_t, 2, EX, MG>(gshift);
   }
   return cm == 2 ? lane_fn_t<uint64_t, 2, EX, MG>(gshift) : lane_fn_t<uint64_t, 1, EX, MG>(gshift);
 }
-static const void *lane_fn(int tbits, int gshift, int cm, bool exact, bool mg) {
-  if (mg) return exact ? lane_fn_x<true, true>(tbits, gshift, cm) : lane_fn_x<false, true>(tbits, gshift, cm);
-  return exact ? lane_fn_x<true, false>(tbits, gshift, cm) : lane_fn_x<false, false>(tbits, gshift, cm);
+static const void *lane_fn(int tbits, int gshift, int cm, bool exact, bool mg, bool pk) {
+  if (mg) return exact ? lane_fn_x<true, true>(tbits, gshift, cm, false) : lane_fn_x<false, true>(tbits, gshift, cm, false);
+  return exact ? lane_fn_x<true, false>(tbits, gshift, cm, pk) : lane_fn_x<false, false>(tbits, gshift, cm, pk);
 }
 
 template <typename T, bool MG> static size_t lane_smem_t(int gshift) {
@@ -696,6 +791,28 @@ size_t lane_smem(int tbits, int gshift, bool mg) {
          (tbits == 32 ? lane_smem_t<uint32_t, false>(gshift) : lane_smem_t<uint64_t, false>(gshift));
 }
 
+__global__ void k_pack_costs(const PrepGraph *pgp, int32_t n, int G, int gshift, int64_t E, uint32_t *costk,
+                             unsigned long long *mx) {
+  const PrepGraph &P = *pgp;
+  const uint32_t *c = (const uint32_t *)P.costp;
+  const uint32_t *pc = (const uint32_t *)P.pe_comm;
+  uint32_t mc = 0, mm = 0;
+  const int64_t NG = (int64_t)n * G;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < NG; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t v = c[i];
+    mc = v > mc ? v : mc;
+    costk[i] = (v << gshift) | (uint32_t)(i % G);
+  }
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < E; i += (int64_t)gridDim.x * blockDim.x)
+    mm = pc[i] > mm ? pc[i] : mm;
+  atomicMax(mx, (unsigned long long)mc);
+  atomicMax(mx + 1, (unsigned long long)mm);
+}
+void launch_pack_costs(const PrepGraph *pg_dev, int32_t n, int G, int gshift, int64_t E, uint32_t *costk,
+                       unsigned long long *mx, cudaStream_t st) {
+  k_pack_costs<<<148, 256, 0, st>>>(pg_dev, n, G, gshift, E, costk, mx);
+}
+
 int lane_comm_mode(const SimArgs &a, int tbits) {
   if (a.fastcomm && tbits == 32) return 0;
   return a.gc_K == 1 ? 1 : 2;
@@ -705,7 +822,9 @@ int lane_comm_mode(const SimArgs &a, int tbits) {
 // 2 = prepared slots, one per lane (one warp per block; grid = warps)
 void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
   const bool mg = a.lane == 2;
-  const void *f = lane_fn(tbits, a.gshift, lane_comm_mode(a, tbits), a.G == (1 << a.gshift), mg);
+  const int cm = lane_comm_mode(a, tbits);
+  const bool pk = !mg && tbits == 32 && cm != 2 && a.costk != nullptr && a.pk_lim > 0;
+  const void *f = lane_fn(tbits, a.gshift, cm, a.G == (1 << a.gshift), mg, pk);
   const size_t sm = lane_smem(tbits, a.gshift, mg);
   if (mg) cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
   SimArgs aa = a;
@@ -715,8 +834,9 @@ void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
 
 int lane_occupancy(int tbits, int gshift) {
   int nb = 1 << 30, x = 0;
-  for (int v = (tbits == 32 ? 0 : 2); v < 6; v++) {
-    const void *f = lane_fn(tbits, gshift, v >> 1, v & 1, false);
+  for (int v = (tbits == 32 ? 0 : 2); v < (tbits == 32 ? 10 : 6); v++) {
+    const void *f = v < 6 ? lane_fn(tbits, gshift, v >> 1, v & 1, false, false)
+                          : lane_fn(tbits, gshift, (v - 6) >> 1, v & 1, false, true);
     cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lane_smem(tbits, gshift, false));
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, f, LANE_BLOCK, lane_smem(tbits, gshift, false));
     nb = x < nb ? x : nb;

@@ -164,3 +164,66 @@ def test_lane_ragged_and_invalid():
     cands[41] = F.make_candidate(F.KIND_PIN, pins=[(5, 1), (5, 2)])              # duplicate op
     cands[77] = F.make_candidate(dev_mask=0b0011)                                # device subset (deferred)
     check(desc, np.array(cands), F.F_CP_PIN)
+
+
+# ------------------------------------------- packed device keys (PK variant)
+
+@pytest.mark.parametrize("G", [1, 2, 3, 5, 8, 16, 32])
+def test_pk_ab_device_counts(G):
+    """the packed-key lane kernel (default for 32-bit time, one link class)
+    against the unpacked lane kernel (FASTT_NO_PK=1) and the oracle"""
+    desc = topo_dag(4600 + G, V=140, G=G, K=1, homogeneous=bool(G % 2))
+    cands = pin_cands(desc, np.random.default_rng(100 + G), 200)
+    gp = F.Graph(desc)
+    gu = _graph_env(desc, FASTT_NO_PK="1")
+    for flags in (0, F.F_CP_PIN):
+        r = check(desc, cands, flags)
+        r0 = gu.schedule_batch(cands, flags=flags, peak=False)
+        assert gu.last_timing()["topo"] == LANE
+        assert (r["makespan"] == r0["makespan"]).all()
+        if G > 1:  # (G = 1: the stream has no PIN candidates)
+            assert gp.sweep_best(F.gen_params(seed=G), 0, 3000, flags=flags) == \
+                gu.sweep_best(F.gen_params(seed=G), 0, 3000, flags=flags)
+
+
+@pytest.mark.parametrize("lim_q", [0.0, 0.3, 0.7])
+def test_pk_deferral_path(lim_q):
+    """candidates whose makespan reaches the packed-key bound are deferred to
+    the preparation pipeline and re-run unpacked: FASTT_PK_LIM lowers the bound
+    to a quantile of the makespans so part (or all) of a batch takes that path"""
+    desc = topo_dag(4700, V=180, G=8, K=1)
+    cands = pin_cands(desc, np.random.default_rng(7), 256)
+    ms = F.Graph(desc).schedule_batch(cands, flags=F.F_CP_PIN, peak=False)["makespan"]
+    lim = max(1, int(np.quantile(ms, lim_q)))
+    gl = _graph_env(desc, FASTT_PK_LIM=str(lim))
+    r = gl.schedule_batch(cands, flags=F.F_CP_PIN, peak=False)
+    t = gl.last_timing()
+    assert t["topo"] == LANE and t["deferred"] >= int((ms >= lim).sum()) > 0
+    assert (r["makespan"] == ms).all()
+    og = O.OracleGraph(desc)
+    for k in range(0, len(cands), 5):
+        assert int(r["makespan"][k]) == og.schedule(cands[k], flags=F.F_CP_PIN, outputs=False)["makespan"]
+    # the sweep: deferred candidates still compete for the argmin
+    gen = F.gen_params(seed=3)
+    assert gl.sweep_best(gen, 0, 2000, flags=F.F_CP_PIN) == F.Graph(desc).sweep_best(gen, 0, 2000, flags=F.F_CP_PIN)
+
+
+def test_pk_large_makespans():
+    """makespans above 2^29 ns with 32-bit time at G = 8: the natural
+    packed-key bound defers them (no key may wrap), results stay exact"""
+    d0 = topo_dag(4800, V=120, G=8, K=1)
+    V = d0.n_ops
+    # a chain through all ops on top of the random edges: makespan ~ sum of costs
+    src = np.concatenate([np.asarray(d0.src), np.arange(V - 1)]).astype(np.asarray(d0.src).dtype)
+    dst = np.concatenate([np.asarray(d0.dst), np.arange(1, V)]).astype(np.asarray(d0.dst).dtype)
+    nb = np.concatenate([np.asarray(d0.bytes), np.full(V - 1, 1024)]).astype(np.asarray(d0.bytes).dtype)
+    ep = np.concatenate([np.asarray(d0.eparam), np.zeros(V - 1)]).astype(np.asarray(d0.eparam).dtype)
+    scale = max(1, int(1.5e9 / float(d0.cost.reshape(V, -1).max(axis=1).sum())))
+    desc = dataclasses.replace(d0, src=src, dst=dst, bytes=nb, eparam=ep, cost=d0.cost * scale)
+    g = F.Graph(desc)
+    assert g.time_bits == 32
+    cands = pin_cands(desc, np.random.default_rng(9), 96)
+    r = check(desc, cands, F.F_CP_PIN)
+    assert int(r["makespan"].max()) >= (1 << 29)
+    g.schedule_batch(cands, flags=F.F_CP_PIN, peak=False)
+    assert g.last_timing()["deferred"] >= int((r["makespan"] >= (1 << 29)).sum()) > 0
