@@ -429,6 +429,12 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     // (same thread, program order).  A stage or card slot is overwritten only
     // after the step that read it has consumed the values.
     // (a record is staged iff s < max(lo, u - P); s < lo: the BASE record)
+    // this lane's source row of a card copy: base + u * stride (card words or
+    // the cost row), one 64-bit multiply-add per copy instead of a select of
+    // two address computations
+    const char *const cc_base =
+        cc_cost ? (const char *)costsrc + cc_src : (const char *)card + cc_src;
+    const uint32_t cc_stride = cc_cost ? (uint32_t)(G * sizeof(T)) : (uint32_t)(CARD_WORDS * 4);
     auto copy_card = [&](int32_t u) {
       if (MG) {  // this lane's own card: header, predecessors, comm, cost row
         if (u < n) {
@@ -447,8 +453,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
         return;
       }
       const uint32_t dst = cards_sa + (uint32_t)((u & (2 * D - 1)) * CS) + cc_dst;
-      const char *srcp = cc_cost ? (const char *)(costsrc + (size_t)u * G) + cc_src
-                                 : (const char *)(card + (size_t)u * CARD_WORDS) + cc_src;
+      const char *srcp = cc_base + (size_t)(uint32_t)u * cc_stride;
       if (row16) cp_async_if<16>(cc_on && u < n, dst, srcp);
       else {
         cp_async_if<16>(cc_on && !cc_cost && u < n, dst, srcp);
