@@ -256,6 +256,7 @@ struct fastt_graph {
   int sim_grid_topo = 0;  // resident blocks of the TOPO variant (no shared-memory ready set)
   bool use_topo = true;   // FASTT_NO_TOPO=1 forces the ready-set path (A/B parity)
   int sim_grid_lane = 0;  // resident blocks of the lane-per-candidate position-order kernel
+  bool use_rank_reuse = true;  // FASTT_NO_RANK_REUSE=1: SPLIT slots recompute every rank (A/B parity)
   bool use_pk = true;      // FASTT_NO_PK=1: the lane kernel without packed device keys (A/B parity)
   uint32_t pk_lim_cap = 0xFFFFFFFFu;  // FASTT_PK_LIM=<ns>: lower the deferral bound (tests of the deferral path)
   bool use_lane = true;   // FASTT_NO_LANE=1 keeps position-order launches on the group kernel (A/B parity)
@@ -601,7 +602,8 @@ static fastt_status run_prep(fastt_graph *g, const Base &B, int nslots, cudaStre
   launch_copy_block(B.raw_block, g->arena, (int64_t)(g->arena_raw_total + g->arena_prep_total), (int64_t)B.rl.total,
                     g->slot_cands, nslots, st);
   launch_patch_split(B.raw_dev, g->slot_raws_dev, g->gc_dev, g->slot_cands, nslots, st);
-  launch_rank(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, g->slot_cands, nslots, g->G, st);
+  launch_rank(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, g->slot_cands, nslots, g->G, st,
+              g->use_rank_reuse ? prep_struct(B.prep_block, B.pl, B.tbits).rank : nullptr);
   launch_sort(g->slot_pgs_dev, g->slot_raws_dev, nslots, B.key_bits, (int)B.rl.vcap, st);
   // (successor lists only for slots the ready-set kernel will run: see launch_slots)
   launch_cards(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, nslots, (int)B.rl.vcap, g->G, g->K, B.tbits, st,
@@ -1165,6 +1167,8 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     g->use_topo = !(e && e[0] == '1');
     e = getenv("FASTT_NO_LANE");
     g->use_lane = !(e && e[0] == '1');
+    e = getenv("FASTT_NO_RANK_REUSE");
+    g->use_rank_reuse = !(e && e[0] == '1');
     e = getenv("FASTT_NO_PK");
     g->use_pk = !(e && e[0] == '1');
     e = getenv("FASTT_PK_LIM");

@@ -150,8 +150,11 @@ __host__ __device__ inline int64_t part_bytes(int64_t b, int n, int k) { return 
 // ------------------------------------------------------------ launchers
 // (defined in k_prep.cu / k_sim.cu; all asynchronous on `st`)
 
+// base_rank (optional): rank_u of the base graph by uid; a SPLIT slot on all
+// devices then copies the ranks below the split op's height instead of
+// recomputing them (they have no path to the split op)
 void launch_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, const Cand *cands, int nslots,
-                 int G, cudaStream_t st);
+                 int G, cudaStream_t st, const uint64_t *base_rank = nullptr);
 void launch_heights(RawGraph *raw_dev, int32_t *scratch, int64_t vcap, cudaStream_t st);
 void launch_sort(PrepGraph *pgs, const RawGraph *raws, int nslots, int key_bits, int max_n, cudaStream_t st);
 void launch_cards(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, int nslots, int max_n, int G, int K,

@@ -273,7 +273,8 @@ __device__ __forceinline__ void rank_one(const RawGraph &R, const GraphConst &gc
 // successor of an op sits on a lower level); the ops of a level are
 // independent, one lane each.  A split slot inserts its concat nodes before
 // level h(o), its sub-ops with level h(o) and its split nodes after it.
-__global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gcp, const Cand *cands, int nslots) {
+__global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gcp, const Cand *cands, int nslots,
+                       const uint64_t *base_rank) {
   const int lane = threadIdx.x & 31;
   const int slot = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (slot >= nslots) return;
@@ -298,7 +299,19 @@ __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *g
   __syncwarp();
   const bool split = R.ov_P >= 0;
   const int32_t ho = split ? R.height[R.ov_o] : -1;
-  for (int32_t lev = 0; lev <= R.H; lev++) {
+  int32_t lev0 = 0;
+  if (split && base_rank && cands && cands[slot].kind == 2 && cands[slot].dev_mask == 0) {
+    // an op below the split op's height has no path to it: its descendants,
+    // their costs and edges are the base graph's, and so is its rank_u
+    const int32_t hi = R.lvl_off[ho];
+    for (int32_t q = lane; q < hi; q += 32) {
+      const int32_t u = R.lvl_ops[q];
+      if (R.alive[u]) rank[u] = base_rank[u];
+    }
+    __syncwarp();
+    lev0 = ho;
+  }
+  for (int32_t lev = lev0; lev <= R.H; lev++) {
     for (int phase = 0; phase < 3; phase++) {
       // phase 0: concat nodes (label 4h(o)-2), 1: the level (+ sub-ops at h(o)), 2: split nodes (4h(o)+2)
       int32_t lo, cnt;
@@ -323,11 +336,11 @@ __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *g
 }
 
 void launch_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, const Cand *cands, int nslots, int G,
-                 cudaStream_t st) {
+                 cudaStream_t st, const uint64_t *base_rank) {
   (void)G;
   int warps_per_block = 4;
   int blocks = (nslots + warps_per_block - 1) / warps_per_block;
-  k_rank<<<blocks, warps_per_block * 32, 0, st>>>(raws, pgs, gc, cands, nslots);
+  k_rank<<<blocks, warps_per_block * 32, 0, st>>>(raws, pgs, gc, cands, nslots, base_rank);
 }
 
 __device__ uint32_t cta_exscan(uint32_t v, uint32_t *total, uint32_t *s_w);
@@ -677,6 +690,9 @@ void launch_cards(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, in
   else k_cards_pred<uint64_t><<<gp, 256, 0, st>>>(raws, pgs, gc);
   int blocks = (max_n * 32 + 255) / 256;
   if (blocks > 2048) blocks = 2048;
+  // (only the rare non-topological slots do work unless succ_all: a full-width
+  // grid per slot cost ~3.5 ms per 4k-slot wave in empty blocks alone)
+  if (!succ_all && nslots > 1 && blocks > 32) blocks = 32;
   if (blocks < 1) blocks = 1;
   k_cards_succ<<<dim3(blocks, nslots), 256, 0, st>>>(raws, pgs, succ_all ? 1 : 0);
 }

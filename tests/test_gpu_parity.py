@@ -496,3 +496,28 @@ def test_topo_vs_ready_set_random(seed):
     for g in (_graph(desc, False), _graph(desc, True)):
         for flags in (0, F.F_CP_PIN):
             compare(desc, cands, flags, gg=g, og=og)
+
+
+# ------------------------------------------ SPLIT slots reuse the base ranks
+
+@pytest.mark.parametrize("name", ["C2", "C3", "C5"])
+def test_split_rank_reuse_ab(name):
+    """SPLIT slots copy the base ranks below the split op's height (no path to
+    the split op): every split candidate of the stream against the slots that
+    recompute all ranks (FASTT_NO_RANK_REUSE=1), a sample against the oracle"""
+    desc = synth.config(name)
+    gg = F.Graph(desc)
+    os.environ["FASTT_NO_RANK_REUSE"] = "1"
+    try:
+        g0 = F.Graph(desc)
+    finally:
+        del os.environ["FASTT_NO_RANK_REUSE"]
+    gen = F.gen_params(seed=0xFA57)
+    ns = gg.stream_info(gen, flags=F.F_CP_PIN)
+    c = gg.generate_candidates(gen, 1, min(ns, 600), flags=F.F_CP_PIN)
+    a = gg.schedule_batch(c, flags=F.F_CP_PIN, peak=False)
+    b = g0.schedule_batch(c, flags=F.F_CP_PIN, peak=False)
+    assert (a["makespan"] == b["makespan"]).all() and (a["status"] == b["status"]).all()
+    og = O.OracleGraph(desc)
+    for k in range(0, len(c), max(1, len(c) // 6)):
+        assert int(a["makespan"][k]) == og.schedule(c[k], flags=O.F_CP_PIN, outputs=False)["makespan"], (name, k)
