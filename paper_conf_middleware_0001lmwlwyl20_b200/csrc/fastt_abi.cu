@@ -256,6 +256,12 @@ struct fastt_graph {
   int sim_grid_topo = 0;  // resident blocks of the TOPO variant (no shared-memory ready set)
   bool use_topo = true;   // FASTT_NO_TOPO=1 forces the ready-set path (A/B parity)
   int sim_grid_lane = 0;  // resident blocks of the lane-per-candidate position-order kernel
+  // device staging buffers of fastt_schedule_batch (host candidates in,
+  // makespan/status out), kept across calls and grown on demand
+  struct IoBuf {
+    void *p = nullptr;
+    size_t cap = 0;
+  } io[3];
   bool use_rank_reuse = true;  // FASTT_NO_RANK_REUSE=1: SPLIT slots recompute every rank (A/B parity)
   bool use_pk = true;      // FASTT_NO_PK=1: the lane kernel without packed device keys (A/B parity)
   uint32_t pk_lim_cap = 0xFFFFFFFFu;  // FASTT_PK_LIM=<ns>: lower the deferral bound (tests of the deferral path)
@@ -1268,6 +1274,7 @@ void fastt_free_graph(fastt_graph *g) {
     cudaFree(g->scratch_list);
     cudaFree(g->scratch_n);
     cudaFree(g->sort_buf);
+    for (auto &b : g->io) cudaFree(b.p);
     for (auto &e : g->ev)
       if (e) cudaEventDestroy(e);
   }
@@ -1285,6 +1292,18 @@ fastt_status fastt_graph_info(const fastt_graph *g, int32_t *n_ops, int32_t *v_m
 }
 
 // host or device candidates -> device array
+static void *io_buf(fastt_graph *g, int k, size_t bytes) {
+  auto &b = g->io[k];
+  if (b.cap < bytes) {
+    cudaFree(b.p);
+    b.p = nullptr;
+    b.cap = 0;
+    if (cudaMalloc(&b.p, bytes) != cudaSuccess) return nullptr;
+    b.cap = bytes;
+  }
+  return b.p;
+}
+
 static fastt_status upload_cands(const fastt_candidate *cands, int64_t n, uint32_t flags, Cand **d, bool *owned,
                                  cudaStream_t st) {
   *owned = false;
@@ -1369,8 +1388,14 @@ fastt_status fastt_schedule_batch(const fastt_graph *gc_, const fastt_candidate 
   const int64_t vm = g->v_max;
   const bool outdev = (flags & FASTT_F_OUT_DEVICE) != 0;
   Cand *d_c;
-  bool own_c;
-  TRY(upload_cands(cands, n, flags, &d_c, &own_c, st));
+  bool own_c = false;
+  if (flags & FASTT_F_IN_DEVICE) {
+    d_c = (Cand *)cands;
+  } else {
+    d_c = (Cand *)io_buf(g, 0, sizeof(Cand) * (size_t)(n + 1));
+    if (!d_c) return fail(FASTT_ENOMEM, "candidate staging buffer");
+    CK(cudaMemcpyAsync(d_c, cands, sizeof(Cand) * n, cudaMemcpyHostToDevice, st));
+  }
   DevOut o;
   o.vmax = vm;
   std::vector<void *> tmp;
@@ -1382,8 +1407,8 @@ fastt_status fastt_schedule_batch(const fastt_graph *gc_, const fastt_candidate 
     tmp.push_back(p);
     return p;
   };
-  o.makespan = (int64_t *)dalloc(makespan, 8 * (size_t)n, true);
-  o.status = (uint8_t *)dalloc(status, (size_t)n, true);
+  o.makespan = (int64_t *)(outdev ? dalloc(makespan, 8 * (size_t)n, true) : io_buf(g, 1, 8 * (size_t)n));
+  o.status = (uint8_t *)(outdev ? dalloc(status, (size_t)n, true) : io_buf(g, 2, (size_t)n));
   o.peak = (int64_t *)dalloc(peak_mem, 8 * (size_t)n * g->G, peak_mem != nullptr);
   const bool want_sched = placement || order || start_ns;
   o.place = (uint8_t *)dalloc(placement, (size_t)n * vm, want_sched);
@@ -1397,10 +1422,12 @@ fastt_status fastt_schedule_batch(const fastt_graph *gc_, const fastt_candidate 
   unsigned long long nd0 = 0;
   if (rc == FASTT_OK) rc = timing_begin(g, flags, st);
   if (rc == FASTT_OK) rc = eval_batch(g, B, d_c, n, flags, st, o);
-  if (rc == FASTT_OK) cudaMemcpy(&nd0, g->counters + 1, sizeof nd0, cudaMemcpyDeviceToHost);
+  if (rc == FASTT_OK && (cudaMemcpyAsync(&nd0, g->counters + 1, sizeof nd0, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+                         cudaStreamSynchronize(st) != cudaSuccess))
+    rc = fail(FASTT_ECUDA, "deferred count");
   if (rc == FASTT_OK && !outdev) {
     auto back = [&](void *h, void *dd, size_t bytes) {
-      if (h && dd && cudaMemcpy(h, dd, bytes, cudaMemcpyDeviceToHost) != cudaSuccess)
+      if (h && dd && cudaMemcpyAsync(h, dd, bytes, cudaMemcpyDeviceToHost, st) != cudaSuccess)
         rc = fail(FASTT_ECUDA, "download");
     };
     back(makespan, o.makespan, 8 * (size_t)n);
@@ -1411,6 +1438,7 @@ fastt_status fastt_schedule_batch(const fastt_graph *gc_, const fastt_candidate 
     back(order, o.order, 4 * (size_t)n * vm);
   }
   if (rc == FASTT_OK) rc = timing_end(g, flags, st, n, (int64_t)nd0);
+  if (cudaStreamSynchronize(st) != cudaSuccess && rc == FASTT_OK) rc = fail(FASTT_ECUDA, "synchronize");
   for (void *p : tmp) cudaFree(p);
   if (own_c) cudaFree(d_c);
   return rc;

@@ -4,7 +4,7 @@
 #   3. one `ncu --set full` capture of the main k_sim_lane sweep launch.
 # usage: tools/profile_round.sh <tag>
 set -u
-tag=${1:-r01}
+tag=${1:-r01f}
 mkdir -p gpurun_out
 python bench.py > gpurun_out/${tag}_bench.json 2> gpurun_out/${tag}_bench.err
 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/${tag}_launches.csv \
