@@ -451,6 +451,37 @@ __device__ uint32_t cta_exscan(uint32_t v, uint32_t *total, uint32_t *s_w) {
   return r;
 }
 
+// cta_exscan on a 64-bit word: two independent 32-bit counters scanned in
+// one pass (half the barriers), valid while each half's CTA total stays
+// below 2^32 (no carry crosses into the high half).
+__device__ uint64_t cta_exscan64(uint64_t v, uint64_t *total, uint64_t *s_w) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  uint64_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint64_t y = __shfl_up_sync(FULL, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) s_w[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    uint64_t t = lane < nw ? s_w[lane] : 0;
+    uint64_t tt = t;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      uint64_t y = __shfl_up_sync(FULL, tt, o);
+      if (lane >= o) tt += y;
+    }
+    if (lane < nw) s_w[lane] = tt - t;
+    if (lane == 31) s_w[32] = tt;
+  }
+  __syncthreads();
+  uint64_t r = s_w[w] + x - v;
+  *total = s_w[32];
+  __syncthreads();
+  return r;
+}
+
 // One CTA per slot: order live ops by (rank desc, uid asc) with a stable LSD
 // radix sort of key = (2^key_bits - 1 - rank) over values initially in uid order.
 __global__ void __launch_bounds__(SORT_T) k_sort(PrepGraph *pgs, const RawGraph *raws, int key_bits) {
@@ -555,7 +586,7 @@ void launch_sort(PrepGraph *pgs, const RawGraph *raws, int nslots, int key_bits,
 __global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, PrepGraph *pgs) {
   const RawGraph &R = raws[blockIdx.x];
   PrepGraph &P = pgs[blockIdx.x];
-  __shared__ uint32_t s_w[33];
+  __shared__ uint64_t s_w[33];
   const int32_t n = P.n;
   uint32_t runp = 0, runs = 0;
   for (int32_t w = threadIdx.x; w < (n + 31) / 32; w += blockDim.x) P.srcbits[w] = 0;
@@ -565,9 +596,12 @@ __global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, Prep
     int32_t p = t0 + threadIdx.x;
     uint32_t u = p < n ? P.uid[p] : 0;
     uint32_t np_ = p < n ? R.pred_cnt[u] : 0, ns_ = p < n ? R.succ_cnt[u] : 0;
-    uint32_t totp, tots;
-    uint32_t bp = cta_exscan(np_, &totp, s_w);
-    uint32_t bs = cta_exscan(ns_, &tots, s_w);
+    // both degree scans in one pass: degrees < 2^16 (CW_DEG), so a chunk's
+    // half-totals stay below 2^26
+    uint64_t tot2;
+    const uint64_t b2 = cta_exscan64((uint64_t)np_ | ((uint64_t)ns_ << 32), &tot2, s_w);
+    const uint32_t bp = (uint32_t)b2, bs = (uint32_t)(b2 >> 32);
+    const uint32_t totp = (uint32_t)tot2, tots = (uint32_t)(tot2 >> 32);
     if (p < n) {
       uint32_t *c = P.card + (int64_t)p * CARD_WORDS;
       c[CW_DEG] = np_ | (ns_ << 16);
