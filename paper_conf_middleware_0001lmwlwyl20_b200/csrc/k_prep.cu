@@ -278,7 +278,9 @@ __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *g
   const int lane = threadIdx.x & 31;
   const int slot = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (slot >= nslots) return;
-  const RawGraph &R = raws[slot];
+  // by value: the rank stores cannot alias the descriptor, so its pointers
+  // stay in registers instead of being re-loaded after every store
+  const RawGraph R = raws[slot];
   PrepGraph &P = pgs[slot];
   const GraphConst &gc = *gcp;
   int32_t po[MAXPINS], pd[MAXPINS];
@@ -584,7 +586,7 @@ void launch_sort(PrepGraph *pgs, const RawGraph *raws, int nslots, int key_bits,
 
 // One CTA per slot: degree scans in position order + card headers.
 __global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, PrepGraph *pgs) {
-  const RawGraph &R = raws[blockIdx.x];
+  const RawGraph R = raws[blockIdx.x];  // (by value: see k_rank)
   PrepGraph &P = pgs[blockIdx.x];
   __shared__ uint64_t s_w[33];
   const int32_t n = P.n;
@@ -642,7 +644,7 @@ __global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, Prep
 template <typename T>
 __global__ void k_cards_pred(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gcp) {
   const int slot = blockIdx.y;
-  const RawGraph &R = raws[slot];
+  const RawGraph R = raws[slot];  // (by value: see k_rank)
   PrepGraph &P = pgs[slot];
   const GraphConst &gc = *gcp;
   const int G = gc.G, K = gc.K;
@@ -691,7 +693,7 @@ __global__ void k_cards_succ(const RawGraph *raws, PrepGraph *pgs, int all) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int slot = blockIdx.y;
-  const RawGraph &R = raws[slot];
+  const RawGraph R = raws[slot];  // (by value: see k_rank)
   PrepGraph &P = pgs[slot];
   if (!all && P.topo) return;
   const int32_t n = P.n;
@@ -741,7 +743,7 @@ __global__ void k_cp(const RawGraph *raws, PrepGraph *pgs, int nslots, int G) {
   const int lane = threadIdx.x & 31;
   const int slot = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (slot >= nslots) return;
-  const RawGraph &R = raws[slot];
+  const RawGraph R = raws[slot];  // (by value: see k_rank)
   PrepGraph &P = pgs[slot];
   const int32_t n = P.n;
   const T *costp = (const T *)P.costp;

@@ -13,6 +13,6 @@ ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-fil
 ncu --set full --clock-control none --import-source on -k regex:k_sim_lane -c 1 -o gpurun_out/${tag}_k_sim_lane -f \
     python tools/ncu_sim.py 300000 > gpurun_out/${tag}_ncu_full.log 2>&1
 # the preparation pipeline's heaviest kernels (split candidates)
-ncu --set full --clock-control none --import-source on -k regex:"k_cards_edges|k_sim<" -c 4 -o gpurun_out/${tag}_prep -f \
+ncu --set full --clock-control none --import-source on -k regex:"k_rank|k_sort|k_cards_hdr|k_cards_pred|k_cp" -c 5 -o gpurun_out/${tag}_prep -f \
     python bench.py --steps 1 --warmup 1 --candidates 20000 --no-e2e --no-cpu > gpurun_out/${tag}_ncu_prep.log 2>&1
 ls -la gpurun_out
