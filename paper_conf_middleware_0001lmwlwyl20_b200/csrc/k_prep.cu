@@ -764,28 +764,34 @@ __global__ void k_cp(const RawGraph *raws, PrepGraph *pgs, int nslots, int G) {
     }
   }
   int64_t accm = 0, accc = 0;
-  if (lane == 0) P.pmem[0] = 0;
-  if (lane < G) P.pcost[lane] = 0;
+  // the walk's arrays in registers: its stores would otherwise force the
+  // PrepGraph pointers to be re-loaded on every step of the chain
+  uint32_t *const card = P.card, *const cpl = P.cp;
+  const uint32_t *const pos = P.pos;
+  int64_t *const pmem = P.pmem, *const pcost = P.pcost;
+  if (lane == 0) pmem[0] = 0;
+  if (lane < G) pcost[lane] = 0;
   int32_t len = 0;
   while (cur != NONE) {
-    const uint32_t *c = P.card + (int64_t)cur * CARD_WORDS;
+    const uint32_t *c = card + (int64_t)cur * CARD_WORDS;
     uint32_t deg = c[CW_DEG];
     int64_t m = (int64_t)(((uint64_t)c[CW_MEMHI] << 32) | c[CW_MEMLO]);
+    const uint32_t uid = c[CW_UID];
     if (lane == 0) {
-      P.cp[len] = cur;
-      P.card[(int64_t)cur * CARD_WORDS + CW_CPIDX] = (uint32_t)len;
+      cpl[len] = cur;
+      card[(int64_t)cur * CARD_WORDS + CW_CPIDX] = (uint32_t)len;
     }
     accm += m;
     if (lane < G) accc += (int64_t)costp[(int64_t)cur * G + lane];
     len++;
-    if (lane == 0) P.pmem[len] = accm;
-    if (lane < G) P.pcost[(int64_t)len * G + lane] = accc;
+    if (lane == 0) pmem[len] = accm;
+    if (lane < G) pcost[(int64_t)len * G + lane] = accc;
     // successors from the raw lists (the card's successor part is built
     // only where the ready-set simulator needs it)
-    const uint32_t ns_ = deg >> 16, so = R.succ_off[c[CW_UID]];
+    const uint32_t ns_ = deg >> 16, so = R.succ_off[uid];
     uint32_t best = NONE;
     for (uint32_t j = lane; j < ns_; j += 32) {
-      const uint32_t d = P.pos[R.succ_dst[so + j]];
+      const uint32_t d = pos[R.succ_dst[so + j]];
       best = d < best ? d : best;
     }
     best = warp_min_u32(best);
