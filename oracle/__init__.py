@@ -19,6 +19,11 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "fastt_oracle.c")
 _LIB = os.path.join(_HERE, "liboracle_fastt.so")
+# tools/oracle_mutants.py points this at a mutated copy of the source (built
+# into /tmp) to show that the pins catch each mutation
+if os.environ.get("FASTT_ORACLE_SRC"):
+    _SRC = os.path.abspath(os.environ["FASTT_ORACLE_SRC"])
+    _LIB = "/tmp/liboracle_%s.so" % os.path.basename(_SRC).replace(".c", "")
 
 INF = np.iinfo(np.int64).max
 CAND_OK, CAND_INFEASIBLE, CAND_BADSPEC = 0, 1, 2

@@ -109,6 +109,7 @@ static int fo_build_adjacency(fo_graph *g, fo_edge *ed, int64_t ne) {
   for (int64_t e = 0; e < ne; e++) {
     if (ed[e].s == ed[e].d) return FO_ECYCLE;
     if (m > 0 && ed[m - 1].s == ed[e].s && ed[m - 1].d == ed[e].d) {
+      if (ed[m - 1].b > INT64_MAX / 4 - ed[e].b) return FO_ERANGE; /* merged bytes stay far inside int64 */
       ed[m - 1].b += ed[e].b;
       ed[m - 1].p |= ed[e].p;
     } else {
@@ -242,6 +243,9 @@ int32_t fastt_ref_load(int32_t n_ops, int64_t n_edges, int32_t n_devices, const 
   for (int64_t e = 0; e < g->E; e++)
     for (int k = 0; k < g->K; k++)
       if (g->beta[k] && g->succ_bytes[e] > (INT64_MAX / 4) / g->beta[k]) { fo_graph_free(g); return FO_ERANGE; }
+  /* ... and so must the split/concat node cost bytes * copy_fs (R13) */
+  for (int64_t e = 0; e < g->E; e++)
+    if (g->copy_fs && g->succ_bytes[e] > (INT64_MAX / 4) / g->copy_fs) { fo_graph_free(g); return FO_ERANGE; }
   int32_t *topo = malloc(sizeof(int32_t) * ((size_t)V + 1));
   int32_t n = fo_topo(g, topo);
   free(topo);

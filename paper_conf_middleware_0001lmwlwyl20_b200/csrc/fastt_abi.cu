@@ -1061,6 +1061,9 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     for (int k = 0; k < K; k++)
       if (d->link_beta_fs_per_byte[k] && x.b > (INT64_MAX / 4) / d->link_beta_fs_per_byte[k])
         return fail(FASTT_ERANGE, "bytes * beta overflows int64");
+  for (auto &x : ed)
+    if (d->split_copy_fs_per_byte && x.b > (INT64_MAX / 4) / d->split_copy_fs_per_byte)
+      return fail(FASTT_ERANGE, "bytes * split_copy_fs_per_byte overflows int64");
   std::vector<uint32_t> so(V), sc(V, 0), po(V), pc(V, 0);
   std::vector<int32_t> sdst(Em), psrc(Em);
   std::vector<int64_t> sb(Em), pb(Em);

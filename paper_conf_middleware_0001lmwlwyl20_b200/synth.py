@@ -109,6 +109,25 @@ def append_vs_insert():
                    link=(0, 1_000_000))
 
 
+def stop_rule_chain():
+    """tests/golden/alg2_stop_rule.json: P(1) -> X(100) -> Q(1) -> Y(60) -> R(1),
+    X and Y batch-splittable; bytes 1000, 1000, 0, 0; G=2; one link class
+    alpha=0, beta=1e6 fs/B (comm = bytes ns)."""
+    G = 2
+    cost = np.repeat(np.array([1, 100, 1, 60, 1], np.int64)[:, None], G, axis=1)
+    return _finish("stop_rule_chain", G, [0, 1, 2, 3], [1, 2, 3, 4], [1000, 1000, 0, 0], [0] * 4, cost, [0] * 5,
+                   [0] * 5, [0, DIM_BATCH_BIT, 0, DIM_BATCH_BIT, 0], link=(0, 1_000_000))
+
+
+def r9_average_pair():
+    """tests/golden/r9_exact_average.json: A -> B (5 bytes); costs A (3, 3),
+    B (4, 100); mem 10 each; caps (20, 10); G=2; comm = bytes ns."""
+    G = 2
+    cost = np.array([[3, 3], [4, 100]], np.int64)
+    return _finish("r9_average_pair", G, [0], [1], [5], [0], cost, [10, 10], [0, 0], [0, 0], cap=[20, 10],
+                   link=(0, 1_000_000))
+
+
 # ------------------------------------------------------------ random fuzz
 
 def random_dag(seed, V=None, G=None, K=None, p_edge=None, zero_frac=None, caps="random", homogeneous=None,

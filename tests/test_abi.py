@@ -75,6 +75,14 @@ def test_load_validation_errors(F):
     with pytest.raises(F.FasttError) as e:
         F.Graph(d)
     assert e.value.code == F.ERANGE
+    # bytes * split_copy_fs_per_byte (R13 split/concat node cost) must stay in int64
+    d = _mk(2, 2, [(0, 1)], np.ones((2, 2)))
+    d.bytes = np.array([1 << 40], np.int64)
+    d.beta = np.array([0], np.int64)
+    d.copy_fs = 1 << 22
+    with pytest.raises(F.FasttError) as e:
+        F.Graph(d)
+    assert e.value.code == F.ERANGE
 
 
 def test_no_cpu_fallback_without_device(F):

@@ -1,0 +1,241 @@
+"""Round-2 pins of the oracle's OS-DPOS loop (Alg. 2), critical-path device
+rule (R9), CP-pinned schedules and the sweep stream (R21) against things
+other than itself.  CPU only.
+
+* Hand-derived goldens (tests/golden/alg2_stop_rule.json,
+  tests/golden/r9_exact_average.json) on which Alg. 2's stop rule
+  (line 12), its descending sort (line 5) and R9's exact
+  average each change the answer.
+* An independent Python re-implementation (tests/pyref.py: heap ready set,
+  Fraction averages, dict split rewriting) compared with the oracle on
+  random DAGs: DPOS with pins / caps / CP pinning, OS-DPOS, and the stream.
+* The greedy-step replay (refcheck.check_greedy_steps) of CP-pinned
+  schedules with the CP devices re-derived by pyref.cp_devices.
+
+The mutation runs these were designed against are reproducible with
+tools/oracle_mutants.py.
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import oracle as O
+import pyref as PR
+import refcheck as RC
+from paper_conf_middleware_0001lmwlwyl20_b200 import synth
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def gold(name):
+    with open(os.path.join(GOLD, name)) as f:
+        return json.load(f)
+
+
+# ------------------------------------------------------------- goldens
+
+def test_alg2_stop_rule_golden():
+    gd = gold("alg2_stop_rule.json")
+    d = synth.stop_rule_chain()
+    g = O.OracleGraph(d)
+    for flags in (0, O.F_CP_PIN):
+        assert g.schedule(flags=flags)["makespan"] == gd["base_makespan"]
+        assert g.schedule(O.make_cand(O.KIND_SPLIT, split=(1, 0, 2)), flags=flags)["makespan"] == gd["split_X_makespan"]
+        assert g.schedule(O.make_cand(O.KIND_SPLIT, split=(3, 0, 2)), flags=flags)["makespan"] == gd["split_Y_makespan"]
+        ss = g.split_search(flags=flags)
+        assert [list(x) for x in ss["sp"]] == gd["split_search"]["sp"]
+        assert ss["makespan"] == gd["split_search"]["makespan"]
+        bi = g.split_search(flags=flags, best_improvement=True)
+        assert [list(x) for x in bi["sp"]] == gd["split_search_best_improvement"]["sp"]
+        assert bi["makespan"] == gd["split_search_best_improvement"]["makespan"]
+        # the stream's SPLIT block is the sorted list x dims x n (R21)
+        n_split, _ = g.stream_info(flags=flags)
+        cs = g.generate(seed=1, first=1, n=n_split, flags=flags)
+        assert [[int(c["split_op"]), int(c["split_dim"]), int(c["split_n"])] for c in cs] == gd["stream_split_block"]
+    # the independent implementation agrees, including the counterfactual
+    pg = PR.PG.from_desc(d)
+    assert PR.split_list(pg, PR.dpos(pg)["place"]) == gd["split_list"]
+    assert PR.split_search(pg)["sp"] == [tuple(x) for x in gd["split_search"]["sp"]]
+
+
+def test_r9_exact_average_golden():
+    gd = gold("r9_exact_average.json")
+    g = O.OracleGraph(synth.r9_average_pair())
+    r = g.schedule(flags=O.F_CP_PIN)
+    for k in ("makespan",):
+        assert r[k] == gd["cp_pin"][k]
+    assert r["placement"][:2].tolist() == gd["cp_pin"]["placement"]
+    assert r["start"][:2].tolist() == gd["cp_pin"]["start"]
+    assert r["peak_mem"].tolist() == gd["cp_pin"]["peak_mem"]
+    r = g.schedule(flags=0)
+    assert r["makespan"] == gd["pure_eft"]["makespan"]
+    assert r["placement"][:2].tolist() == gd["pure_eft"]["placement"]
+    assert r["start"][:2].tolist() == gd["pure_eft"]["start"]
+    assert r["peak_mem"].tolist() == gd["pure_eft"]["peak_mem"]
+    pg = PR.PG.from_desc(synth.r9_average_pair())
+    assert PR.cp_devices(pg, PR.ranks(pg)) == {0: 1, 1: 0}
+
+
+# ------------------------------------------- independent implementation
+
+def _dags(n, lo, hi, seed0, **kw):
+    out = []
+    for s in range(n):
+        rng = np.random.default_rng(seed0 + s)
+        out.append(synth.random_dag(seed0 + s, V=int(rng.integers(lo, hi + 1)), **kw))
+    return out
+
+
+# one link class / homogeneous costs make "a later op improves after an
+# earlier one failed" common enough that the stop rule (Alg. 2 line 12)
+# changes the answer on several of these (seeds 7100, 7110, 7111, 7201, 7209)
+ALG2_DAGS = (_dags(24, 20, 40, 7100, G=4, caps="none", max_in=2, K=1)
+             + _dags(12, 20, 40, 7200, G=3, caps="none", max_in=3, homogeneous=True)
+             + _dags(8, 20, 40, 7300, caps="none", max_in=3))
+
+
+@pytest.mark.parametrize("k", range(len(ALG2_DAGS)))
+def test_split_search_matches_independent(k):
+    """Alg. 2 end to end: SP list, final makespan, placement and
+    start times of every live op equal the independent implementation's."""
+    d = ALG2_DAGS[k]
+    g = O.OracleGraph(d)
+    pg = PR.PG.from_desc(d)
+    for flags, cp in ((0, False), (O.F_CP_PIN, True)):
+        for pow2 in ((False, True) if d.n_devices > 2 else (False,)):
+            ss = g.split_search(flags=flags, pow2_only=pow2)
+            ps = PR.split_search(pg, cp_pin=cp, pow2_only=pow2)
+            assert [tuple(x) for x in ss["sp"]] == ps["sp"]
+            assert ss["makespan"] == ps["makespan"]
+            if ps["status"] == 0:
+                assert ss["n_ops_final"] == ps["n_ops_final"]
+                for i, dv in ps["place"].items():
+                    assert ss["placement"][i] == dv and ss["start"][i] == ps["start"][i]
+
+
+# + the round-1 seeds on which the variant differs from Alg. 2 or splits >= 2 ops
+BI_DAGS = [ALG2_DAGS[k] for k in range(0, len(ALG2_DAGS), 2)] + \
+    [synth.random_dag(s, V=40, G=4, caps="none", max_in=2) for s in (4, 13, 21, 32, 34, 39, 116, 122, 214, 1, 3)]
+
+
+@pytest.mark.parametrize("k", range(len(BI_DAGS)))
+def test_split_search_best_matches_independent(k):
+    """Best-improvement variant (R23, NEXT N2): every round, not only the
+    first, equals the independent implementation (SP list, makespan,
+    placement, start)."""
+    d = BI_DAGS[k]
+    g = O.OracleGraph(d)
+    pg = PR.PG.from_desc(d)
+    for flags, cp in ((0, False), (O.F_CP_PIN, True)):
+        ss = g.split_search(flags=flags, best_improvement=True)
+        ps = PR.split_search_best(pg, cp_pin=cp)
+        assert [tuple(x) for x in ss["sp"]] == ps["sp"]
+        assert ss["makespan"] == ps["makespan"]
+        if ps["status"] == 0:
+            for i, dv in ps["place"].items():
+                assert ss["placement"][i] == dv and ss["start"][i] == ps["start"][i]
+
+
+DPOS_DAGS = _dags(40, 2, 80, 7500)
+
+
+@pytest.mark.parametrize("k", range(len(DPOS_DAGS)))
+def test_dpos_matches_independent(k):
+    """DPOS (Alg. 1) with random caps (some infeasible), perturbation pins,
+    CP pinning on and off, single splits and device subsets: makespan,
+    status, placement, start, peak memory equal the independent
+    implementation's."""
+    d = DPOS_DAGS[k]
+    g = O.OracleGraph(d)
+    pg = PR.PG.from_desc(d)
+    rng = np.random.default_rng(k)
+    cands = [(None, None, None)]
+    if d.n_devices > 1:
+        for _ in range(4):
+            npin = int(rng.integers(1, min(4, d.n_ops) + 1))
+            ops = rng.choice(d.n_ops, npin, replace=False).tolist()
+            cands.append(([(o, int(rng.integers(0, d.n_devices))) for o in ops], None, None))
+        m = int(rng.integers(1, (1 << d.n_devices) - 1))
+        cands.append((None, None, m))
+    sps = [i for i in range(d.n_ops) if d.split_mask[i]]
+    for op in sps[:3]:
+        dim = 0 if d.split_mask[op] & 1 else 1
+        if d.n_devices >= 2:
+            cands.append((None, (op, dim, int(rng.integers(2, d.n_devices + 1))), None))
+    for pins, split, mask in cands:
+        if pins:
+            c = O.make_cand(O.KIND_PIN, pins=pins)
+        elif split:
+            c = O.make_cand(O.KIND_SPLIT, split=split)
+        else:
+            c = O.make_cand(O.KIND_BASE, dev_mask=mask or 0)
+        gg = PR.split_view(pg, *split) if split else pg
+        dset = None if not mask else {x for x in range(d.n_devices) if mask >> x & 1}
+        for flags, cp in ((0, False), (O.F_CP_PIN, True)):
+            r = g.schedule(c, flags=flags)
+            p = PR.dpos(gg, pin=dict(pins) if pins else None, dset=dset, cp_pin=cp)
+            assert r["makespan"] == p["makespan"] and r["status"] == p["status"]
+            if p["status"] == 0:
+                for i, dv in p["place"].items():
+                    assert r["placement"][i] == dv and r["start"][i] == p["start"][i]
+                assert r["order"][: len(p["order"])].tolist() == p["order"]
+                peak = [0] * d.n_devices
+                for i, dv in p["place"].items():
+                    peak[dv] += gg.mem[i]
+                assert r["peak_mem"].tolist() == peak
+
+
+@pytest.mark.parametrize("k", range(0, len(DPOS_DAGS), 2))
+def test_greedy_replay_cp_pinned(k):
+    """SURVEY P6 for CP_PIN schedules: every pop is the max-(rank, -id) ready
+    op, CP ops sit on the R9 devices re-derived by pyref.cp_devices (with
+    their memory reserved up front), every other op on its minimum-EFT
+    feasible device."""
+    d = DPOS_DAGS[k]
+    g = O.OracleGraph(d)
+    r = g.schedule(flags=O.F_CP_PIN)
+    if r["status"] != O.CAND_OK:
+        return
+    pg = PR.PG.from_desc(d)
+    rk = PR.ranks(pg)
+    cpd = PR.cp_devices(pg, rk)
+    for i, dv in cpd.items():
+        assert r["placement"][i] == dv
+    RC.check_greedy_steps(RC.G(d), r, [rk[i] for i in range(d.n_ops)], cp_dev=cpd)
+
+
+STREAM_CASES = [("C1", {}), ("C1", {"kmin": 2, "kmax": 3}), ("C1", {"subsets": True})] + \
+    [("rand%d" % s, {"pow2_only": bool(s % 2), "subsets": s % 3 == 0}) for s in range(8)]
+
+
+@pytest.mark.parametrize("name,kw", STREAM_CASES)
+def test_stream_matches_independent(name, kw):
+    """R21: the oracle's candidate stream equals the independent splitmix64
+    stream byte for byte (BASE, SPLIT block, subset block, PIN block)."""
+    if name == "C1":
+        d = synth.config("C1")
+    else:
+        s = int(name[4:])
+        d = synth.random_dag(7900 + s, V=30 + 5 * s, G=2 + s % 7, caps="none")
+    g = O.OracleGraph(d)
+    pg = PR.PG.from_desc(d)
+    kmin, kmax = kw.get("kmin", 1), kw.get("kmax", 4)
+    pow2, subs = kw.get("pow2_only", False), kw.get("subsets", False)
+    seed = 0xFA57 + len(name)
+    n_split, _ = g.stream_info(flags=O.F_CP_PIN, pow2_only=pow2, subsets=subs)
+    n = n_split + (d.n_devices - 1 if subs else 0) + 300
+    got = g.generate(seed=seed, first=0, n=n, kmin=kmin, kmax=kmax, flags=O.F_CP_PIN, pow2_only=pow2, subsets=subs)
+    want = PR.stream(pg, seed, 0, n, kmin, kmax, cp_pin=True, pow2_only=pow2, subsets=subs)
+    exp = np.zeros(n, O.CAND_DTYPE)
+    for q, (kind, npin, dim, sn, sop, po, pd, dm) in enumerate(want):
+        exp[q]["kind"], exp[q]["n_pins"], exp[q]["split_dim"], exp[q]["split_n"] = kind, npin, dim, sn
+        exp[q]["split_op"], exp[q]["pin_op"], exp[q]["pin_dev"], exp[q]["dev_mask"] = sop, po, pd, dm
+    assert got.tobytes() == exp.tobytes()
+    # index-addressable far into the stream
+    far = g.generate(seed=seed, first=987_654, n=5, kmin=kmin, kmax=kmax, flags=O.F_CP_PIN, pow2_only=pow2,
+                     subsets=subs)
+    fw = PR.stream(pg, seed, 987_654, 5, kmin, kmax, cp_pin=True, pow2_only=pow2, subsets=subs)
+    assert [list(c["pin_op"]) for c in far] == [x[5] for x in fw]
+    assert [list(c["pin_dev"]) for c in far] == [x[6] for x in fw]

@@ -452,6 +452,13 @@ def test_load_errors_and_empty_graph():
     with pytest.raises(O.OracleError) as e:
         O.OracleGraph(mk(2, 2, [(0, 1, 1)], [1, -1]))
     assert e.value.code == -1
+    # bytes * split_copy_fs_per_byte (R13) and merged parallel-edge bytes (R11) must stay in int64
+    with pytest.raises(O.OracleError) as e:
+        O.OracleGraph(mk(2, 2, [(0, 1, 1 << 40)], [1, 1], link=(0, 0), copy_fs=1 << 22))
+    assert e.value.code == -5
+    with pytest.raises(O.OracleError) as e:
+        O.OracleGraph(mk(2, 2, [(0, 1, 1 << 61), (0, 1, 1 << 61)], [1, 1], link=(0, 0)))
+    assert e.value.code == -5
     r = O.OracleGraph(mk(0, 2, [], np.zeros((0, 2), np.int64))).schedule(flags=O.F_CP_PIN)
     assert r["makespan"] == 0 and r["status"] == O.CAND_OK
 
