@@ -86,6 +86,17 @@ def alu_peak_tops():
     return 148 * 4 * 2 * 16 * mhz * 1e6 / 1e12, src
 
 
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for ln in f:
+                if ln.startswith("model name"):
+                    return ln.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return None
+
+
 def peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -172,23 +183,24 @@ def oracle_rate(desc, S, budget_s, threads=None):
         step = max(1, S // M)
         idx = list(range(0, S, step))[:M]
         cands = np.concatenate([og.generate(GEN_SEED, i, 1, flags=O.F_CP_PIN) for i in idx])
-        _ORACLE_SAMPLE[key] = (og, cores, step, cands)
-    og, cores, step, cands = _ORACLE_SAMPLE[key]
-    chunks = [cands[k::cores] for k in range(cores)]
+        _ORACLE_SAMPLE[key] = (og, cores, step, cands, idx)
+    og, cores, step, cands, idx = _ORACLE_SAMPLE[key]
+    chunks = [list(range(k, len(cands), cores)) for k in range(cores)]
 
     def work(ch):
-        best = (O.INF, -1)
-        for c in ch:
-            r = og.schedule(c, flags=O.F_CP_PIN, outputs=False)
-            best = min(best, (r["makespan"], 0))
-        return len(ch)
+        out = []
+        for j in ch:
+            r = og.schedule(cands[j], flags=O.F_CP_PIN, outputs=False)
+            out.append((idx[j], r["makespan"], r["status"]))
+        return out
 
     t0 = time.time()
     with ThreadPoolExecutor(cores) as ex:
-        done = sum(ex.map(work, chunks))
+        res = [x for part in ex.map(work, chunks) for x in part]
     el = time.time() - t0
+    done = len(res)
     sample = "%d candidates (every %d-th index of the %d-candidate stream window, BASE/SPLIT/PIN mix)" % (done, step, S)
-    return done / el, cores, sample, el
+    return done / el, cores, sample, el, res
 
 
 def run_reference(args, rank, world):
@@ -198,7 +210,7 @@ def run_reference(args, rank, world):
     S = args.candidates
     times = []
     for k in range(args.warmup + args.steps):
-        rate, cores, sample, el = oracle_rate(desc, S, args.ref_budget)
+        rate, cores, sample, el, _ = oracle_rate(desc, S, args.ref_budget)
         if k >= args.warmup:
             times.append((rate, el, cores, sample))
     rate = statistics.mean(t[0] for t in times)
@@ -377,9 +389,29 @@ def main():
                "api": "fastt_schedule_batch (host pinned buffers)", "argmin_local_index": i}
 
     cpu = None
+    parity = None
     if rank == 0 and world == 1 and not args.no_cpu:
-        rate, cores, sample, _ = oracle_rate(desc, S, args.cpu_budget)
-        cpu = {"value": rate, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample}
+        rate, cores, sample, _, ores = oracle_rate(desc, S, args.cpu_budget)
+        cpu = {"value": rate, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample,
+               "single_thread_value": rate / cores if cores else None, "cpu_model": cpu_model(),
+               "oracle_build": "gcc -O2 (oracle/__init__.py), one thread per candidate"}
+        # parity at full size: the oracle's sample against the GPU's
+        # per-candidate results for the same stream indices (e2e vector when
+        # it ran, else one fastt_schedule_batch over the sampled candidates)
+        oidx = np.array([r[0] for r in ores], np.int64)
+        if e2e is not None:
+            gms, gst = outn["makespan"][oidx], outn["status"][oidx]
+            src = "e2e fastt_schedule_batch vector"
+        else:
+            sc = np.concatenate([g.generate_candidates(gen, int(i), 1, flags=FLAGS_CP) for i in oidx])
+            rr = g.schedule_batch(sc, flags=FLAGS_CP, stream=st, peak=False)
+            gms, gst = rr["makespan"], rr["status"]
+            src = "fastt_schedule_batch over the sampled candidates"
+        mism = [int(i) for i, m, s_, a, b in zip(oidx, gms, gst, [r[1] for r in ores], [r[2] for r in ores])
+                if int(m) != int(a) or int(s_) != int(b)]
+        parity = {"checked": len(ores), "mismatches": len(mism), "first_mismatch": mism[0] if mism else None,
+                  "against": "oracle (plain C, one thread per candidate)", "gpu_side": src,
+                  "indices": "every %d-th stream index of [0, %d)" % (int(oidx[1] - oidx[0]) if len(oidx) > 1 else 1, S)}
 
     if rank == 0:
         line = {
@@ -395,6 +427,7 @@ def main():
             "best": {"makespan_ns": best[0], "index": best[1]},
             "roofline": roof,
             "cpu_baseline": cpu,
+            "parity": parity,
             "e2e": e2e,
             "gpu_launches": launches,
             "clocks": clk.summary(),

@@ -384,9 +384,10 @@ def _dense(tb, x, din, dout, rows, act=None):
 
 
 def bert_large(G=8, R=4, seed=0xFA57_0004, layers=24, hid=1024, heads=16, seq=64, batch=16, ffn=4096,
-               link=LINK_PAPER, hetero_ppm=0, iter_s=0.19):
+               link=LINK_PAPER, hetero_ppm=0, iter_s=0.19, cap_frac=None):
     """C5: BERT-large training DAG (~20k ops), seq 64, batch 16
-    (P:930), Sigma cost per replica ~0.19 s."""
+    (P:930), Sigma cost per replica ~0.19 s.  cap_frac (test
+    variants only): per-device caps = cap_frac x ceil(Sigma mem / G)."""
     rng = np.random.default_rng(seed)
     tb = _TB()
     rows = batch * seq // R if R > 1 else batch * seq
@@ -442,7 +443,7 @@ def bert_large(G=8, R=4, seed=0xFA57_0004, layers=24, hid=1024, heads=16, seq=64
     lbl = tb.op("Data", [], rows * 4)
     tb.op("Loss", [logits, lbl], 4)
     return _replicate_training(tb, R, G, rng, "C5_bert_large", int(iter_s * 1e9), link=link, hetero_ppm=hetero_ppm,
-                               seed=seed)
+                               cap_frac=cap_frac, seed=seed)
 
 
 def _conv(tb, x, cin, cout, k, hw_out, bs, stride_w=1.0, bn=True, relu=True):

@@ -201,7 +201,9 @@ def test_c4_tight_caps_infeasible():
     ns = gg.stream_info(gen, flags=F.F_CP_PIN)
     c = gg.generate_candidates(gen, 0, ns + 60, flags=F.F_CP_PIN)
     res = compare(desc, c, F.F_CP_PIN, gg=gg, og=og, outputs=False)
-    assert (res["status"] == 1).any() or True
+    n_inf = sum(1 for x in c if og.schedule(x, flags=O.F_CP_PIN, outputs=False)["status"] == 1)
+    assert n_inf > 0, "1.05x caps should make some candidates infeasible"
+    assert int((res["status"] == 1).sum()) == n_inf
 
 
 # ------------------------------------------------------------- sweep + argmin
