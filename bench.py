@@ -411,7 +411,7 @@ def main():
                 if int(m) != int(a) or int(s_) != int(b)]
         parity = {"checked": len(ores), "mismatches": len(mism), "first_mismatch": mism[0] if mism else None,
                   "against": "oracle (plain C, one thread per candidate)", "gpu_side": src,
-                  "indices": "every %d-th stream index of [0, %d)" % (int(oidx[1] - oidx[0]) if len(oidx) > 1 else 1, S)}
+                  "indices": "every %d-th stream index of [0, %d)" % (int(np.diff(np.sort(oidx))[0]) if len(oidx) > 1 else 1, S)}
 
     if rank == 0:
         line = {

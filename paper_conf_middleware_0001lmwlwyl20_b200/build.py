@@ -1,6 +1,8 @@
 """Build libfastt.so in-tree with nvcc for sm_100a (no JIT, no torch extension).
 Each translation unit compiles to an object in parallel (relocatable device
-code is not needed: no kernel calls across files), then one link."""
+code is not needed: no kernel calls across files), then one link.  The two
+simulation kernels' template instances are split by device-count width GSH:
+k_sim_inst.cu and k_sim_lane_inst.cu are compiled once per GSH = 0..5."""
 from __future__ import annotations
 
 import os
@@ -10,8 +12,14 @@ from concurrent.futures import ThreadPoolExecutor
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
-SRCS = [os.path.join(HERE, "csrc", f) for f in ("fastt_abi.cu", "k_prep.cu", "k_sim.cu", "k_sim_lane.cu", "k_fit.cu")]
-DEPS = SRCS + [os.path.join(HERE, "csrc", "fastt_internal.cuh"), os.path.join(HERE, "csrc", "sim_common.cuh"), os.path.join(ROOT, "include", "fastt.h")]
+_C = os.path.join(HERE, "csrc")
+SRCS = [os.path.join(_C, f) for f in ("fastt_abi.cu", "k_prep.cu", "k_sim.cu", "k_sim_lane.cu", "k_fit.cu",
+                                      "k_sim_inst.cu", "k_sim_lane_inst.cu")]
+# (source, extra flags): one object per unit
+UNITS = [(s, []) for s in SRCS[:5]] + [(os.path.join(_C, f), ["-DFASTT_GSH=%d" % g])
+                                         for g in range(6) for f in ("k_sim_lane_inst.cu", "k_sim_inst.cu")]
+DEPS = SRCS + [os.path.join(_C, f) for f in ("fastt_internal.cuh", "sim_common.cuh", "k_sim_body.cuh",
+                                             "k_sim_lane_body.cuh")] + [os.path.join(ROOT, "include", "fastt.h")]
 OUT = os.path.join(HERE, "libfastt.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -25,15 +33,15 @@ def build(force: bool = False, verbose: bool = False, out: str = OUT) -> str:
     if not force and os.path.exists(out) and all(os.path.getmtime(out) >= os.path.getmtime(d) for d in DEPS):
         return out
     with tempfile.TemporaryDirectory(prefix="fastt_build_") as td:
-        objs = [os.path.join(td, os.path.basename(s) + ".o") for s in SRCS]
+        objs = [os.path.join(td, "%02d_%s.o" % (k, os.path.basename(u[0]))) for k, u in enumerate(UNITS)]
 
         def cc(pair):
-            src, obj = pair
-            cmd = [NVCC] + CFLAGS + (["-Xptxas", "-v"] if verbose else []) + ["-c", src, "-o", obj]
+            (src, extra), obj = pair
+            cmd = [NVCC] + CFLAGS + extra + (["-Xptxas", "-v"] if verbose else []) + ["-c", src, "-o", obj]
             subprocess.check_call(cmd)
 
-        with ThreadPoolExecutor(max_workers=len(SRCS)) as ex:
-            list(ex.map(cc, zip(SRCS, objs)))
+        with ThreadPoolExecutor(max_workers=min(len(UNITS), os.cpu_count() or 4)) as ex:
+            list(ex.map(cc, zip(UNITS, objs)))
         tmp = out + ".tmp%d" % os.getpid()
         subprocess.check_call([NVCC] + ARCH + ["-shared", "-o", tmp] + objs)
         os.replace(tmp, out)

@@ -240,6 +240,18 @@ template <typename T> struct GapSlot {
 };
 
 void launch_sim(const SimArgs &a, int tbits, int grid, int block, size_t smem, cudaStream_t st);
+// per-GSH kernel getters (k_sim_inst.cu / k_sim_lane_inst.cu, compiled once
+// per lane-group width so the template instances build in parallel)
+#define FASTT_CAT2(a, b) a##b
+#define FASTT_CAT(a, b) FASTT_CAT2(a, b)
+#define FASTT_DECL_SIM_FN(N) const void *sim_fn_g##N(int tbits, bool mem, bool ins, bool fc, bool topo);
+FASTT_DECL_SIM_FN(0) FASTT_DECL_SIM_FN(1) FASTT_DECL_SIM_FN(2) FASTT_DECL_SIM_FN(3) FASTT_DECL_SIM_FN(4)
+FASTT_DECL_SIM_FN(5)
+#undef FASTT_DECL_SIM_FN
+#define FASTT_DECL_LANE_FN(N) const void *lane_fn_g##N(int tbits, int cm, bool exact, bool mg, bool pk);
+FASTT_DECL_LANE_FN(0) FASTT_DECL_LANE_FN(1) FASTT_DECL_LANE_FN(2) FASTT_DECL_LANE_FN(3) FASTT_DECL_LANE_FN(4)
+FASTT_DECL_LANE_FN(5)
+#undef FASTT_DECL_LANE_FN
 void launch_argmin(const int64_t *wbest, int64_t nwarps, int64_t *best_dev, cudaStream_t st);
 void launch_order_chunk(const int32_t *deq, const int64_t *start, int32_t *order, const int64_t *results, int64_t n,
                         int64_t vmax, int key_bits, uint64_t *k0, uint64_t *k1, uint32_t *v0, uint32_t *v1,

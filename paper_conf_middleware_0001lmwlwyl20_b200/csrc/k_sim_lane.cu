@@ -34,749 +34,22 @@
 //             positions before that step are read from the BASE record.
 // Memory caps, liveness memory, INSERT, per-op outputs, SPLIT and
 // rank-changing candidates stay on k_sim (group-per-candidate kernel).
-#include "fastt_internal.cuh"
-#include "sim_common.cuh"
+//
+// The kernel itself is in k_sim_lane_body.cuh (instances: k_sim_lane_inst.cu).
+#include "k_sim_lane_body.cuh"
 
 namespace fastt {
 
-// pipeline depth: records of positions at distance <= D-1 are read from the
-// shared-memory ring of the last D records; older ones are staged by
-// cp.async D-1 steps ahead (SLAB records are 8 B for 32-bit time, 16 B else)
-#ifndef LANE_D
-#define LANE_D 8
-#endif
-template <typename T> struct LaneDepth { static constexpr int D = sizeof(T) == 4 ? LANE_D : LANE_D / 2; };
-// staged card of one position: header (words 0-3), predecessor positions
-// (words 8-11), the inline predecessors' comm values (4 x T), then the cost
-// row padded to 16 B
-template <typename T> __host__ __device__ constexpr int card_cost_off() { return 32 + 4 * (int)sizeof(T); }
-template <typename T, int GP> __host__ __device__ constexpr int card_slot_bytes() {
-  return card_cost_off<T>() + (int)((GP * sizeof(T) + 15) / 16) * 16;
-}
-// MG: per-lane card regions are 2D slots + 16 B apart, so the 8 lanes of a
-// 128-bit shared-memory phase hit distinct bank quads (a 2D x CS stride is a
-// multiple of 128 B: every lane's card load would fall in the same banks)
-template <typename T, int GP> __host__ __device__ constexpr int mg_lane_stride() {
-  return 2 * LaneDepth<T>::D * card_slot_bytes<T, GP>() + 16;
-}
-template <typename T, int GP, bool MG> __host__ __device__ constexpr size_t lane_smem_per_warp() {
-  // ring D x 32 + stage D x 4 x 32 records, then 2D staged cards (per lane
-  // in the multi-graph variant), then (base-graph launches) the packed-key
-  // avail rows [32 lanes][GP] of the PK variant
-  return (size_t)LaneDepth<T>::D * 5 * 32 * (sizeof(T) == 4 ? 8 : 16) +
-         (MG ? (size_t)32 * mg_lane_stride<T, GP>() : (size_t)2 * LaneDepth<T>::D * card_slot_bytes<T, GP>()) +
-         (size_t)(MG ? 0 : 32 * GP * 4);
-}
-
-template <int BYTES> __device__ __forceinline__ void cp_async(uint32_t saddr, const void *g);
-template <> __device__ __forceinline__ void cp_async<4>(uint32_t saddr, const void *g) {
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(saddr), "l"(g) : "memory");
-}
-template <> __device__ __forceinline__ void cp_async<8>(uint32_t saddr, const void *g) {
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(saddr), "l"(g) : "memory");
-}
-template <> __device__ __forceinline__ void cp_async<16>(uint32_t saddr, const void *g) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(saddr), "l"(g) : "memory");
-}
-// predicated form: the copy is issued iff p
-template <int BYTES> __device__ __forceinline__ void cp_async_if(bool p, uint32_t saddr, const void *g);
-#define FASTT_CP_ASYNC_IF(BYTES, CACHE)                                                                    \
-  template <> __device__ __forceinline__ void cp_async_if<BYTES>(bool p, uint32_t saddr, const void *g) {  \
-    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t@q cp.async." CACHE                       \
-                 ".shared.global [%0], [%1], " #BYTES ";\n}\n" ::"r"(saddr),                                \
-                 "l"(g), "r"((int)p)                                                                        \
-                 : "memory");                                                                               \
-  }
-FASTT_CP_ASYNC_IF(4, "ca")
-FASTT_CP_ASYNC_IF(8, "ca")
-FASTT_CP_ASYNC_IF(16, "cg")
-#undef FASTT_CP_ASYNC_IF
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N> __device__ __forceinline__ void cp_async_wait() {
-  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
-}
-
-template <typename T> struct RowLd;
-template <> struct RowLd<uint32_t> {
-  template <int GP>
-  __device__ static void load_s(const uint32_t *row, int G, uint32_t (&c)[GP]) {  // shared memory, 16-B aligned
-    if (GP >= 4) {
-#pragma unroll
-      for (int j = 0; j < GP / 4; j++) {
-        const uint4 x = ((const uint4 *)row)[j];
-        c[4 * j] = x.x;
-        c[4 * j + 1] = x.y;
-        c[4 * j + 2] = x.z;
-        c[4 * j + 3] = x.w;
-      }
-    } else {
-#pragma unroll
-      for (int d = 0; d < GP; d++) c[d] = row[d];
-    }
-  }
-  template <int GP>
-  __device__ static void load(const uint32_t *row, int G, uint32_t (&c)[GP]) {
-    if (GP >= 4 && G == GP) {
-#pragma unroll
-      for (int j = 0; j < GP / 4; j++) {
-        const uint4 x = __ldg((const uint4 *)row + j);
-        c[4 * j] = x.x;
-        c[4 * j + 1] = x.y;
-        c[4 * j + 2] = x.z;
-        c[4 * j + 3] = x.w;
-      }
-    } else {
-#pragma unroll
-      for (int d = 0; d < GP; d++) c[d] = d < G ? __ldg(row + d) : 0u;
-    }
-  }
-};
-template <> struct RowLd<uint64_t> {
-  template <int GP>
-  __device__ static void load_s(const uint64_t *row, int G, uint64_t (&c)[GP]) {
-    if (GP >= 2) {
-#pragma unroll
-      for (int j = 0; j < GP / 2; j++) {
-        const ulonglong2 x = ((const ulonglong2 *)row)[j];
-        c[2 * j] = x.x;
-        c[2 * j + 1] = x.y;
-      }
-    } else {
-      c[0] = row[0];
-    }
-  }
-  template <int GP>
-  __device__ static void load(const uint64_t *row, int G, uint64_t (&c)[GP]) {
-    if (GP >= 2 && G == GP) {
-#pragma unroll
-      for (int j = 0; j < GP / 2; j++) {
-        const ulonglong2 x = __ldg((const ulonglong2 *)row + j);
-        c[2 * j] = x.x;
-        c[2 * j + 1] = x.y;
-      }
-    } else {
-#pragma unroll
-      for (int d = 0; d < GP; d++) c[d] = d < G ? __ldg(row + d) : 0ull;
-    }
-  }
-};
-
-// CM: 0 = uint32 time and one link class, comm values inline in the card;
-//     1 = one link class, comm per edge from pe_comm;
-//     2 = several link classes (per (pred, device) comm).
-// EX: G == GP (no per-device range checks).
-// MG: multi-graph -- lane l simulates prepared slot q0 + l (mode 2: SPLIT and
-//     rank-changing candidates, each with its own priority order, so cards
-//     are staged per lane); launched with one warp per block.
-// PK: packed device keys (32-bit time, one link class, base graph): the EFT
-//     of device d is carried as the key (EFT << GSH) | d, so the argmin with
-//     ties to the lowest device (Alg. 1 lines 12-19, R3) is a plain unsigned
-//     min (3-input VIMNMX3), the cost row is pre-packed (costk = cost << GSH
-//     | d), avail[d] << GSH lives in a per-lane shared-memory row so the
-//     chosen device's update and the arrival on the predecessor device pa
-//     (R6) are one indexed store / load instead of a select per device.
-//     Exact while every key fits 32 bits: EFT <= makespan + max comm + max
-//     cost at every step, so a candidate whose final makespan reaches
-//     pk_lim = 2^(32-GSH) - max cost - max comm is deferred and re-run by the
-//     preparation pipeline (unpacked kernels).
-template <typename T, int GSH, int CM, bool EX, bool MG, bool PK>
-__global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
-  typedef typename Slab<T>::W W;
-  constexpr int GP = 1 << GSH;
-  static_assert(!PK || (sizeof(T) == 4 && CM != 2 && !MG), "packed keys: 32-bit time, one link class, base graph");
-  static_assert(CM != 0 || sizeof(T) == 4, "card comm values are uint32");
-  const int lane = threadIdx.x & 31;
-  const int64_t gwarp = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
-  // this lane's slab column: record of position p at col[p * 32]
-  W *const col = (W *)a.slab + (size_t)gwarp * (size_t)a.slab_stride * 32 + lane;
-  // shared memory of this warp: ring[D][32] (records of the last D positions)
-  // and stage[D][4][32] (inline predecessors' records prefetched by cp.async)
-  constexpr int D = LaneDepth<T>::D, P = D - 1;
-  extern __shared__ __align__(16) unsigned char lsm[];
-  unsigned char *const wsm = lsm + (threadIdx.x >> 5) * lane_smem_per_warp<T, GP, MG>();
-  W *const ring = (W *)wsm + lane;
-  W *const stage = ring + D * 32;
-  const uint32_t stage_sa = (uint32_t)__cvta_generic_to_shared(stage);
-  // 2D staged cards (warp-shared): the card of position u is copied at step
-  // u - 2P and read at steps u - P (record prefetch) and u (compute)
-  constexpr int CS = card_slot_bytes<T, GP>();
-  const unsigned char *const cards = wsm + (size_t)D * 5 * 32 * sizeof(W) + (MG ? (size_t)lane * mg_lane_stride<T, GP>() : 0);
-  const uint32_t cards_sa = (uint32_t)__cvta_generic_to_shared(cards);
-  // PK: avail[d] << GSH of every lane, after the warp's cards, as device
-  // pairs [d / 2][32 lanes][2] (a pair per lane is one 64-bit access; the
-  // indexed access of device d by all lanes is 2-way conflicted at most)
-  uint32_t *const avk = (uint32_t *)(wsm + (size_t)D * 5 * 32 * sizeof(W) + (size_t)2 * D * card_slot_bytes<T, GP>()) +
-                        (GP >= 2 ? 2 * lane : lane);
-  auto avk_at = [&](uint32_t d) -> uint32_t & { return GP >= 2 ? avk[(d >> 1) * 64 + (d & 1)] : avk[0]; };
-  constexpr int CO = card_cost_off<T>();
-  const bool row16 = (a.G * (int)sizeof(T)) % 16 == 0;
-  // this lane's 16-B chunk of a card copy: lane 0 header (words 0-3), lane 1
-  // predecessor positions (8-11), lane 2 comm (12-15, CM 0), lanes 3.. the
-  // cost row (when its length is a multiple of 16 B, else element-wise)
-  const bool cc_cost = lane >= 3;
-  const uint32_t cc_src = lane == 0 ? 0u : lane == 1 ? 4u * CARD_HDR : lane == 2 ? 4u * CW_PCOMM : 16u * (lane - 3);
-  const uint32_t cc_dst = lane < 3 ? 16u * lane : (uint32_t)CO + 16u * (lane - 3);
-  const bool cc_on = lane < 2 || (lane == 2 && CM == 0) || (lane >= 3 && lane - 3 < a.G * (int)sizeof(T) / 16);
-  const GraphConst &gc = *a.gc;
-  const int G = a.G;
-  const int K = gc.K;
-  // the graph (per candidate in the multi-graph variant)
-  const PrepGraph *pg = MG ? a.slots : a.base;
-  const uint32_t *card = pg->card;
-  const T *costp = (const T *)pg->costp;
-  const T *costsrc = PK ? (const T *)a.costk : costp;  // the cost rows staged with the cards
-  const T *pe_comm = (const T *)pg->pe_comm;
-  const uint32_t *pe_src = pg->pe_src;
-  const uint32_t *posm = pg->pos;
-  int32_t n = pg->n, Vraw = pg->V, cpl = pg->cp_len;
-  const W *__restrict__ snap = (const W *)a.snap_rec;
-  const bool cp_on = (a.flags & 1u) != 0;
-  const uint32_t all = all_devices(G);
-  int64_t bms = I64MAX, bidx = -1;  // this lane's best (makespan, stream index) for the sweep argmin
-
-  for (;;) {
-    unsigned long long q0 = 0;
-    if (lane == 0) q0 = atomicAdd(a.counter, 32ull);
-    q0 = __shfl_sync(FULL, q0, 0);
-    if ((int64_t)q0 >= a.n) break;
-    const int64_t q = (int64_t)q0 + lane;
-    bool active = q < a.n;
-    Cand c;
-    c.kind = 0;
-    c.n_pins = 0;
-    c.split_op = -1;
-    c.dev_mask = 0;
-    int64_t res_idx = -1, sidx = q;
-    if (MG) {
-      pg = a.slots + (active ? q : (int64_t)q0);
-      card = pg->card;
-      costp = (const T *)pg->costp;
-      pe_comm = (const T *)pg->pe_comm;
-      pe_src = pg->pe_src;
-      posm = pg->pos;
-      n = pg->n;
-      Vraw = pg->V;
-      cpl = pg->cp_len;
-      if (active) {
-        c = a.cands[q];
-        res_idx = a.slot_result ? a.slot_result[q] : -1;
-        sidx = a.slot_index ? a.slot_index[q] : q;
-        if (a.slot_filter == 1 && !pg->topo) active = false;  // (the ready-set launch takes it)
-      }
-      if (!active) n = 0;
-    } else if (active) {
-      if (a.mode == 0) {
-        sidx = a.first + q * a.stride;
-        c = stream_cand(a.stream, sidx);
-      } else if (a.mode == 1) {
-        c = a.cands[q];
-        res_idx = q;
-      } else {  // mode 3: list ordered by BASE-prefix start step
-        c = a.cands[q];
-        res_idx = a.slot_result ? a.slot_result[q] : -1;
-        sidx = a.slot_index[q];
-      }
-    }
-
-    // ---------------------------------------------------------- validate
-    int np = 0;
-    uint8_t st = 0;
-    bool defer = false;
-    if (MG) {
-      np = (active && c.kind == 1) ? c.n_pins : 0;  // (validated by the main launch)
-    } else if (active) {
-      if (c.dev_mask & ~all) st = 2;
-      else if (c.dev_mask && c.dev_mask != all) defer = true;  // device subset (R25): own ranks
-      if (st) {
-      } else if (c.kind == 0) {
-      } else if (c.kind == 1) {
-        np = c.n_pins;
-        if (np < 1 || np > MAXPINS) st = 2;
-        else {
-          const uint32_t dset = c.dev_mask ? c.dev_mask : all;
-          bool bad = false;
-          for (int k = 0; k < np; k++) {
-            const int32_t o = c.pin_op[k];
-            if (o < 0 || o >= Vraw || posm[o] == NONE || c.pin_dev[k] >= G || !((dset >> c.pin_dev[k]) & 1u))
-              bad = true;
-            for (int k2 = 0; k2 < k; k2++) bad |= c.pin_op[k2] == o;
-          }
-          if (bad) st = 2;
-        }
-      } else if (c.kind == 2) {
-        const int32_t o = c.split_op;
-        if (o < 0 || o >= Vraw || posm[o] == NONE || c.split_dim > 1 || !(a.split_mask[o] & (1u << c.split_dim)) ||
-            c.split_n < 2 || c.split_n > G)
-          st = 2;
-        else defer = true;
-      } else {
-        st = 2;
-      }
-    }
-    if (st) {
-      np = 0;
-      defer = false;
-    }
-    uint32_t pp[MAXPINS] = {NONE, NONE, NONE, NONE};
-    uint32_t pdv = 0;
-    if (active && !defer)
-      for (int k = 0; k < np; k++) {
-        pp[k] = posm[c.pin_op[k]];
-        pdv |= (uint32_t)c.pin_dev[k] << (8 * k);
-      }
-    // pins that change w or c (R5) need the candidate's own ranks
-    if (!MG && active && !defer)
-      for (int k = 0; k < np && !defer; k++)
-        defer = pin_changes_ranks<T>(pg, gc, c, np, pp[k], c.pin_dev[k], G, K);
-    if (active && defer) {
-      const unsigned long long k = atomicAdd(a.ndefer, 1ull);
-      a.defer_q[k] = q;
-    }
-    if (active && !defer && st && res_idx >= 0) {
-      a.out.makespan[res_idx] = I64MAX;
-      a.out.status[res_idx] = st;
-    }
-    const bool run = active && !defer && st == 0;
-
-    // ------------------------------------------------------ prologue
-    // CP devices (Alg. 1 line 5, R9) without memory caps: one
-    // round over the free CP ops (perturbation-pinned CP ops excluded)
-    int r_dev = -1;
-    int m = 0;
-    const uint32_t dmask = (MG && c.dev_mask) ? c.dev_mask : all;  // the candidate's devices (R25)
-    if (run && cp_on && cpl > 0) {
-      uint32_t pc[MAXPINS];
-#pragma unroll
-      for (int k = 0; k < MAXPINS; k++) {
-        pc[k] = k < np ? __ldg(card + (size_t)pp[k] * CARD_WORDS + CW_CPIDX) : NONE;
-        m += pc[k] != NONE;
-      }
-      if (cpl - m > 0) {
-        int64_t bs = 0;
-        for (int d = 0; d < G; d++) {
-          if (MG && !((dmask >> d) & 1u)) continue;
-          int64_t s = pg->pcost[(int64_t)cpl * G + d];
-#pragma unroll
-          for (int k = 0; k < MAXPINS; k++)
-            if (pc[k] != NONE) s -= (int64_t)costp[(size_t)pp[k] * G + d];
-          if (r_dev < 0 || s < bs) {
-            bs = s;
-            r_dev = d;
-          }
-        }
-      }
-    }
-    // BASE-prefix sharing: same ranks, same CP devices for the free CP ops,
-    // no caps => the BASE schedule up to the first pinned op's step t0
-    int32_t t0 = 0;
-    bool share = false;
-    if (!MG && run && a.snap_mode == 2) {
-      share = m == 0 || (a.snap_round_dev >= 0 && r_dev == a.snap_round_dev);
-      if (share) {
-        t0 = n;
-        for (int k = 0; k < np; k++) {
-          const int32_t dq = (int32_t)__ldg(a.snap_dq + pp[k]);
-          t0 = dq < t0 ? dq : t0;
-        }
-      }
-    }
-    // The warp starts at lo = the smallest t0 of its candidates (0 if one of
-    // them does not share): a sharing candidate started from the recorded
-    // BASE state at any step <= its t0 makes the BASE decisions up to t0, so
-    // all lanes may start at lo; positions before lo hold BASE records.
-    int32_t lo = run ? t0 : n;
-    int32_t nmax = run ? n : 0;  // steps of the warp (MG: the longest slot)
-#pragma unroll
-    for (int o = 16; o >= 1; o >>= 1) {
-      const int32_t x = __shfl_xor_sync(FULL, lo, o);
-      lo = x < lo ? x : lo;
-      const int32_t y = __shfl_xor_sync(FULL, nmax, o);
-      nmax = y > nmax ? y : nmax;
-    }
-    if (MG) lo = 0;
-    T avail[GP];
-    T ms = 0;
-#pragma unroll
-    for (int d = 0; d < GP; d++) avail[d] = 0;
-    if (run && lo > 0) {  // (lo > 0 implies every running lane shares)
-      const T *sa = (const T *)a.snap_avail + (size_t)lo * G;
-#pragma unroll
-      for (int d = 0; d < GP; d++)
-        if (d < G) avail[d] = __ldg(sa + d);
-      ms = __ldg((const T *)a.snap_ms + lo);
-    }
-    if (PK) {
-#pragma unroll
-      for (int d = 0; d < GP; d++) avk_at(d) = (uint32_t)avail[d] << GSH;
-    }
-
-    // the next pinned position at or after the current step (NONE: none left)
-    uint32_t nxt = NONE;
-#pragma unroll
-    for (int k = 0; k < MAXPINS; k++)
-      if (pp[k] >= (uint32_t)lo && pp[k] < nxt) nxt = pp[k];
-    // ---------------------------------------------------------- main loop
-    // Software pipeline over positions (all cp.async copies are predicated,
-    // so the step is branch-free for every lane):
-    //   step u - 2P : the card of u (header, predecessor positions, comm,
-    //                 cost row) is copied into cards[u % 2D] by lanes 0..;
-    //   step u - P  : the inline predecessors of u at distance > P (and
-    //                 BASE records, s < lo) are copied into
-    //                 stage[u % D]; one commit group per step;
-    //   step u      : the others were written at most P steps earlier and
-    //                 are read from the ring of the last D records.
-    // A staged record was stored at least one step before its copy is issued
-    // (same thread, program order).  A stage or card slot is overwritten only
-    // after the step that read it has consumed the values.
-    // (a record is staged iff s < max(lo, u - P); s < lo: the BASE record)
-    // this lane's source row of a card copy: base + u * stride (card words or
-    // the cost row), one 64-bit multiply-add per copy instead of a select of
-    // two address computations
-    const char *const cc_base =
-        cc_cost ? (const char *)costsrc + cc_src : (const char *)card + cc_src;
-    const uint32_t cc_stride = cc_cost ? (uint32_t)(G * sizeof(T)) : (uint32_t)(CARD_WORDS * 4);
-    auto copy_card = [&](int32_t u) {
-      if (MG) {  // this lane's own card: header, predecessors, comm, cost row
-        if (u < n) {
-          const uint32_t dst = cards_sa + (uint32_t)((u & (2 * D - 1)) * CS);
-          const char *cu = (const char *)(card + (size_t)u * CARD_WORDS);
-          const char *row = (const char *)(costp + (size_t)u * G);
-          cp_async<16>(dst, cu);
-          cp_async<16>(dst + 16, cu + 4 * CARD_HDR);
-          if (CM == 0) cp_async<16>(dst + 32, cu + 4 * CW_PCOMM);
-          if (row16) {
-            for (int j = 0; j < G * (int)sizeof(T) / 16; j++) cp_async<16>(dst + CO + 16 * j, row + 16 * j);
-          } else {
-            for (int j = 0; j < G; j++) cp_async<sizeof(T)>(dst + CO + j * sizeof(T), row + j * sizeof(T));
-          }
-        }
-        return;
-      }
-      const uint32_t dst = cards_sa + (uint32_t)((u & (2 * D - 1)) * CS) + cc_dst;
-      const char *srcp = cc_base + (size_t)(uint32_t)u * cc_stride;
-      if (row16) cp_async_if<16>(cc_on && u < n, dst, srcp);
-      else {
-        cp_async_if<16>(cc_on && !cc_cost && u < n, dst, srcp);
-        for (int j = lane; j < G; j += 32)
-          cp_async_if<sizeof(T)>(u < n, cards_sa + (uint32_t)((u & (2 * D - 1)) * CS + CO + j * sizeof(T)),
-                                 costsrc + (size_t)u * G + j);
-      }
-    };
-    auto prefetch = [&](int32_t u) {  // records of step u (its card is staged)
-      const unsigned char *cu = cards + (u & (2 * D - 1)) * CS;
-      const uint4 hu = *(const uint4 *)cu;
-      const uint32_t npu = u < n ? (hu.x & 0xFFFF) : 0u;
-      if (CM == 1 && !MG)  // the inline predecessors' comm values (warp-uniform card)
-        cp_async_if<sizeof(T)>((uint32_t)lane < npu && lane < 4,
-                               cards_sa + (uint32_t)((u & (2 * D - 1)) * CS + 32 + (lane & 3) * sizeof(T)),
-                               pe_comm + hu.y + (lane & 3));
-      if (CM == 1 && MG)  // (this lane's card)
-        for (uint32_t k = 0; k < npu && k < 4; k++)
-          cp_async<sizeof(T)>(cards_sa + (uint32_t)((u & (2 * D - 1)) * CS + 32 + k * sizeof(T)), pe_comm + hu.y + k);
-      const uint4 su = *(const uint4 *)(cu + 16);
-      const uint32_t ss[4] = {su.x, su.y, su.z, su.w};
-      const uint32_t sl = stage_sa + (uint32_t)((u & (D - 1)) * 4 * 32 * sizeof(W));
-      const bool on = run;
-      const int32_t thr = lo > u - P ? lo : u - P;
-#pragma unroll
-      for (int k = 0; k < 4; k++) {
-        const W *gp = (int32_t)ss[k] < lo ? snap + ss[k] : col + (size_t)ss[k] * 32;
-        cp_async_if<sizeof(W)>(on && (uint32_t)k < npu && (int32_t)ss[k] < thr, sl + (uint32_t)(k * 32 * sizeof(W)), gp);
-      }
-    };
-    // record of position s < t outside the inline slots (extra predecessors)
-    auto rec_at = [&](uint32_t s, int32_t t) -> W {
-      if ((int32_t)s < lo) return snap[s];
-      if ((int32_t)s + P >= t) return ring[(s & (D - 1)) * 32];
-      return col[(size_t)s * 32];
-    };
-    // prologue: cards of lo .. lo+2P-1 (synchronously), records of lo .. lo+P-1
-    for (int32_t u = lo; u < lo + 2 * P; u++) copy_card(u);
-    cp_async_commit();
-    cp_async_wait<0>();
-    __syncwarp();
-    for (int32_t u = lo; u < lo + P; u++) {
-      prefetch(u);
-      cp_async_commit();
-    }
-    for (int32_t t = lo; t < nmax; t++) {
-      const bool live = run && (!MG || t < n);
-      cp_async_wait<P - 1>();  // the group of step t - P: records of t, card of t + P
-      __syncwarp();            // (cards were copied by other lanes)
-      const unsigned char *cs = cards + (t & (2 * D - 1)) * CS;
-      const uint4 h0 = *(const uint4 *)cs;
-      const uint4 hs = *(const uint4 *)(cs + 16);
-      uint4 hc = make_uint4(0, 0, 0, 0);
-      if (CM == 0) hc = *(const uint4 *)(cs + 32);
-      const T *cm1 = (const T *)(cs + 32);  // CM 1: staged comm values
-      T cst[GP];
-      RowLd<T>::template load_s<GP>((const T *)(cs + CO), G, cst);
-      // (MG: a lane past its slot's last position reads a stale card)
-      const uint32_t npred = (!MG || live) ? (h0.x & 0xFFFF) : 0u;
-      const uint32_t src[4] = {hs.x, hs.y, hs.z, hs.w};
-      // predecessor records: staged or from the ring (unused slots: garbage, masked)
-      W rw[4];
-      const W *stg = stage + (t & (D - 1)) * 4 * 32;
-      const int32_t thr = lo > t - P ? lo : t - P;
-#pragma unroll
-      for (int k = 0; k < 4; k++) rw[k] = *((int32_t)src[k] < thr ? stg + k * 32 : ring + (src[k] & (D - 1)) * 32);
-      prefetch(t + P);
-      copy_card(t + 2 * P);
-      cp_async_commit();
-      T f[4];
-      uint32_t p[4];
-#pragma unroll
-      for (int k = 0; k < 4; k++) {
-        T ft;
-        uint32_t pl;
-        Slab<T>::decode_clean(rw[k], ft, pl);
-        f[k] = (uint32_t)k < npred ? ft : (T)0;
-        p[k] = (uint32_t)k < npred ? pl : 0xFFu;
-      }
-      T arrd[GP];  // CM 2: arrival per device
-      T M = 0, E = 0;
-      uint32_t pa = 0xFFu;
-      if (CM != 2) {
-        // M = max over preds of FT + c, pa = the device of a pred attaining it,
-        // E = the arrival on pa (its co-located preds contribute FT only)
-        T R[4];
-#pragma unroll
-        for (int k = 0; k < 4; k++) {
-          T cm;
-          if (CM == 0) cm = (T)(k == 0 ? hc.x : k == 1 ? hc.y : k == 2 ? hc.z : hc.w);
-          else cm = cm1[k];
-          R[k] = (uint32_t)k < npred ? f[k] + cm : (T)0;
-        }
-        M = R[0];
-        pa = p[0];
-#pragma unroll
-        for (int k = 1; k < 4; k++)
-          if (R[k] > M) {
-            M = R[k];
-            pa = p[k];
-          }
-        if (npred > 4u) {  // (warp-uniform)
-          for (uint32_t k = 4; k < npred; k++) {
-            const W w = rec_at(__ldg(pe_src + h0.y + k), t);
-            T ft;
-            uint32_t pl;
-            Slab<T>::decode_clean(w, ft, pl);
-            const T r = ft + __ldg(pe_comm + h0.y + k);
-            if (r > M) {
-              M = r;
-              pa = pl;
-            }
-          }
-        }
-#pragma unroll
-        for (int k = 0; k < 4; k++) {
-          const T v = p[k] == pa ? f[k] : R[k];
-          E = v > E ? v : E;
-        }
-        if (npred > 4u) {
-          for (uint32_t k = 4; k < npred; k++) {
-            const W w = rec_at(__ldg(pe_src + h0.y + k), t);
-            T ft;
-            uint32_t pl;
-            Slab<T>::decode_clean(w, ft, pl);
-            const T v = pl == pa ? ft : ft + __ldg(pe_comm + h0.y + k);
-            E = v > E ? v : E;
-          }
-        }
-      } else {
-        // (only live lanes: a waiting lane's records are not yet valid, and
-        // here a placement indexes the link-class table)
-#pragma unroll
-        for (int d = 0; d < GP; d++) {
-          T v = 0;
-          if (live && d < G) {
-#pragma unroll
-            for (int k = 0; k < 4; k++)
-              if ((uint32_t)k < npred) {
-                const T term = p[k] == (uint32_t)d
-                                   ? f[k]
-                                   : f[k] + __ldg(pe_comm + (size_t)(h0.y + k) * K + gc.link_class[p[k] * G + d]);
-                v = term > v ? term : v;
-              }
-            for (uint32_t k = 4; k < npred; k++) {
-              const W w = rec_at(__ldg(pe_src + h0.y + k), t);
-              T ft;
-              uint32_t pl;
-              Slab<T>::decode_clean(w, ft, pl);
-              const T term =
-                  pl == (uint32_t)d ? ft : ft + __ldg(pe_comm + (size_t)(h0.y + k) * K + gc.link_class[pl * G + d]);
-              v = term > v ? term : v;
-            }
-          }
-          arrd[d] = v;
-        }
-      }
-      if (PK) {
-        // keys (EFT << GSH) | d: EST = max(avail[d], arrival),
-        // arrival M on every device but pa, E on pa (R6); min key = EFT
-        // argmin with ties to the lowest device (Alg. 1 lines 12-19, R3)
-        const uint32_t Mk = (uint32_t)M << GSH, Ek = (uint32_t)E << GSH;
-        uint32_t av[GP];
-        if (GP >= 2) {
-#pragma unroll
-          for (int j = 0; j < GP / 2; j++) {
-            const uint2 x = *(const uint2 *)(avk + j * 64);
-            av[2 * j] = x.x;
-            av[2 * j + 1] = x.y;
-          }
-        } else {
-          av[0] = avk[0];
-        }
-        const uint32_t pq = pa & (uint32_t)(GP - 1);
-        const uint32_t ap = avk_at(pq), cpa = ((const uint32_t *)(cs + CO))[pq];
-        uint32_t kpa = (ap > Ek ? ap : Ek) + cpa;
-        if (!EX && pq >= (uint32_t)G) kpa = 0xFFFFFFFFu;
-        uint32_t key[GP];
-#pragma unroll
-        for (int d = 0; d < GP; d++)
-          key[d] = (EX || d < G) ? (av[d] > Mk ? av[d] : Mk) + (uint32_t)cst[d] : 0xFFFFFFFFu;
-        uint32_t bk = kpa;
-#pragma unroll
-        for (int d = 0; d < GP; d++) bk = key[d] < bk ? key[d] : bk;
-        // device forced by a perturbation pin (hard) or a CP pin (Alg. 1
-        // l.9-10): rare steps
-        if (__any_sync(FULL, (uint32_t)t == nxt || (h0.w != NONE && r_dev >= 0))) {
-          int forced = -1;
-          if ((uint32_t)t == nxt) {
-            nxt = NONE;
-#pragma unroll
-            for (int k = 0; k < MAXPINS; k++) {
-              if (pp[k] == (uint32_t)t) forced = (int)((pdv >> (8 * k)) & 0xFFu);
-              else if (pp[k] > (uint32_t)t && pp[k] < nxt) nxt = pp[k];
-            }
-          }
-          if (forced < 0 && r_dev >= 0 && h0.w != NONE) forced = r_dev;
-          if (forced >= 0) {
-#pragma unroll
-            for (int d = 0; d < GP; d++)
-              if (d == forced) bk = key[d];
-            if ((uint32_t)forced == pq && kpa < bk) bk = kpa;
-          }
-        }
-        if (live) {
-          const uint32_t bkc = bk & ~(uint32_t)(GP - 1);
-          avk_at(bk & (uint32_t)(GP - 1)) = bkc;
-          const T best = (T)(bkc >> GSH);
-          ms = best > ms ? best : ms;
-          W w;
-          Slab<T>::make(w, best, bk & (uint32_t)(GP - 1));
-          col[(size_t)t * 32] = w;
-          ring[(t & (D - 1)) * 32] = w;
-        }
-      } else {
-      // EFT per device; argmin with ties to the lowest device
-      // (Alg. 1 lines 12-19, R3); devices >= G are never chosen
-      T eft[GP];
-#pragma unroll
-      for (int d = 0; d < GP; d++) {
-        const T arr = CM == 2 ? arrd[d] : ((uint32_t)d == pa ? E : M);
-        const T est = avail[d] > arr ? avail[d] : arr;
-        eft[d] = ((EX || d < G) && (!MG || ((dmask >> d) & 1u))) ? est + cst[d] : TT<T>::MAXV;
-      }
-      T best = eft[0];
-      int bd = 0;
-#pragma unroll
-      for (int d = 1; d < GP; d++)
-        if (eft[d] < best) {
-          best = eft[d];
-          bd = d;
-        }
-      // device forced by a perturbation pin (hard) or a CP pin (Alg. 1
-      // l.9-10): rare steps -- the next pinned position, or a CP op
-      if (__any_sync(FULL, (uint32_t)t == nxt || (h0.w != NONE && r_dev >= 0))) {
-        int forced = -1;
-        if ((uint32_t)t == nxt) {
-          nxt = NONE;
-#pragma unroll
-          for (int k = 0; k < MAXPINS; k++) {
-            if (pp[k] == (uint32_t)t) forced = (int)((pdv >> (8 * k)) & 0xFFu);
-            else if (pp[k] > (uint32_t)t && pp[k] < nxt) nxt = pp[k];
-          }
-        }
-        if (forced < 0 && r_dev >= 0 && h0.w != NONE) forced = r_dev;
-        if (forced >= 0) {
-#pragma unroll
-          for (int d = 0; d < GP; d++)
-            if (d == forced) best = eft[d];
-          bd = forced;
-        }
-      }
-      if (live) {
-#pragma unroll
-        for (int d = 0; d < GP; d++)
-          if (d == bd) avail[d] = best;
-        ms = best > ms ? best : ms;
-        W w;
-        Slab<T>::make(w, best, (uint32_t)bd);
-        col[(size_t)t * 32] = w;
-        ring[(t & (D - 1)) * 32] = w;
-      }
-      }  // !PK
-    }
-    cp_async_wait<0>();  // (no copy may land in the stage after this candidate)
-
-    // ------------------------------------------------------------ epilogue
-    if (PK && run && (uint32_t)ms >= a.pk_lim) {  // a key may have wrapped: re-run unpacked
-      const unsigned long long k = atomicAdd(a.ndefer, 1ull);
-      a.defer_q[k] = q;
-    } else if (run) {
-      if (res_idx >= 0) {
-        a.out.makespan[res_idx] = (int64_t)ms;
-        a.out.status[res_idx] = 0;
-      }
-      if ((int64_t)ms < bms || ((int64_t)ms == bms && sidx < bidx)) {
-        bms = (int64_t)ms;
-        bidx = sidx;
-      }
-    }
-  }
-  if (a.track_best) {
-#pragma unroll
-    for (int o = 16; o >= 1; o >>= 1) {
-      const int64_t m2 = __shfl_xor_sync(FULL, bms, o), i2 = __shfl_xor_sync(FULL, bidx, o);
-      if (i2 >= 0 && (bidx < 0 || m2 < bms || (m2 == bms && i2 < bidx))) {
-        bms = m2;
-        bidx = i2;
-      }
-    }
-    if (lane == 0 && bidx >= 0) {
-      const int64_t m0 = a.wbest[2 * gwarp], i0 = a.wbest[2 * gwarp + 1];
-      if (i0 < 0 || bms < m0 || (bms == m0 && bidx < i0)) {
-        a.wbest[2 * gwarp] = bms;
-        a.wbest[2 * gwarp + 1] = bidx;
-      }
-    }
-  }
-}
-
-template <typename T, int CM, bool EX, bool MG, bool PK = false>
-static const void *lane_fn_t(int gshift) {
-  switch (gshift) {
-    case 0: return (const void *)k_sim_lane<T, 0, CM, EX, MG, PK>;
-    case 1: return (const void *)k_sim_lane<T, 1, CM, EX, MG, PK>;
-    case 2: return (const void *)k_sim_lane<T, 2, CM, EX, MG, PK>;
-    case 3: return (const void *)k_sim_lane<T, 3, CM, EX, MG, PK>;
-    case 4: return (const void *)k_sim_lane<T, 4, CM, EX, MG, PK>;
-    default: return (const void *)k_sim_lane<T, 5, CM, EX, MG, PK>;
-  }
-}
-template <bool EX, bool MG> static const void *lane_fn_x(int tbits, int gshift, int cm, bool pk) {
-  if (tbits == 32) {
-    if (!MG && pk && cm != 2)
-      return cm == 0 ? lane_fn_t<uint32_t, 0, EX, false, true>(gshift) : lane_fn_t<uint32_t, 1, EX, false, true>(gshift);
-    if (cm == 0) return lane_fn_t<uint32_t, 0, EX, MG>(gshift);
-    return cm == 1 ? lane_fn_t<uint32_t, 1, EX, MG>(gshift) : lane_fn_t<uint32_t, 2, EX, MG>(gshift);
-  }
-  return cm == 2 ? lane_fn_t<uint64_t, 2, EX, MG>(gshift) : lane_fn_t<uint64_t, 1, EX, MG>(gshift);
-}
+// kernel getters of the per-GSH instance objects (k_sim_lane_inst.cu)
 static const void *lane_fn(int tbits, int gshift, int cm, bool exact, bool mg, bool pk) {
-  if (mg) return exact ? lane_fn_x<true, true>(tbits, gshift, cm, false) : lane_fn_x<false, true>(tbits, gshift, cm, false);
-  return exact ? lane_fn_x<true, false>(tbits, gshift, cm, pk) : lane_fn_x<false, false>(tbits, gshift, cm, pk);
+  switch (gshift) {
+    case 0: return lane_fn_g0(tbits, cm, exact, mg, pk);
+    case 1: return lane_fn_g1(tbits, cm, exact, mg, pk);
+    case 2: return lane_fn_g2(tbits, cm, exact, mg, pk);
+    case 3: return lane_fn_g3(tbits, cm, exact, mg, pk);
+    case 4: return lane_fn_g4(tbits, cm, exact, mg, pk);
+    default: return lane_fn_g5(tbits, cm, exact, mg, pk);
+  }
 }
 
 template <typename T, bool MG> static size_t lane_smem_t(int gshift) {
