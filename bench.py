@@ -236,6 +236,7 @@ def main():
     ap.add_argument("--ref-budget", type=float, default=8.0, help="seconds per reference step")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-configs", action="store_true", help="skip the C1-C4 per-config sweeps")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3) if args.impl == "fastt" else args.warmup
 
@@ -361,10 +362,11 @@ def main():
         cands = np.ascontiguousarray(g.generate_candidates(gen, 0, world * S, flags=FLAGS_CP)[rank::world])
         n = len(cands)
         hc = torch.from_numpy(cands.view(np.uint8).reshape(-1, 32).copy()).pin_memory()
-        # a search needs each candidate's makespan and status (per-device peak
-        # memory is optional in the API and not requested here)
+        # each candidate's makespan, status and per-device peak memory (the
+        # outputs north_star names for the simulation)
         out = {"makespan": torch.empty(n, dtype=torch.int64).pin_memory(),
-               "status": torch.empty(n, dtype=torch.uint8).pin_memory()}
+               "status": torch.empty(n, dtype=torch.uint8).pin_memory(),
+               "peak_mem": torch.empty((n, G), dtype=torch.int64).pin_memory()}
         hcn = hc.numpy().view(F.CANDIDATE_DTYPE).reshape(-1)
         outn = {k: v.numpy() for k, v in out.items()}
         for _ in range(2):
@@ -385,8 +387,38 @@ def main():
             allreduce(t2, dist.ReduceOp.MAX)
         e2e_ms = float(t2.item()) / args.steps
         e2e = {"value": world * n / (e2e_ms / 1000.0), "unit": UNIT, "h2d_bytes_per_step": int(32 * n),
-               "d2h_bytes_per_step": int(n * (8 + 1)), "ms_per_step": e2e_ms,
-               "api": "fastt_schedule_batch (host pinned buffers)", "argmin_local_index": i}
+               "d2h_bytes_per_step": int(n * (8 + 1 + 8 * G)), "ms_per_step": e2e_ms,
+               "api": "fastt_schedule_batch (host pinned buffers; makespan, status, per-device peak memory)",
+               "argmin_local_index": i, "kernel": "k_sim_lane" if g.last_timing()["topo"] == 2 else "k_sim"}
+
+    # the other paper-shaped configs: one sweep each,
+    # device-timed (not part of the step), candidates/s and DAG-ops/s
+    configs = None
+    if not args.no_configs:
+        configs = {}
+        for name, ncand in (("C1", 1_000_000), ("C2", 300_000), ("C3", 200_000), ("C4", 300_000)):
+            d2 = synth.config(name)
+            g2 = F.Graph(d2, device=local)
+            gen2 = F.gen_params(seed=GEN_SEED, pin_k_min=1, pin_k_max=4, n_pow2_only=(name == "C4"))
+            g2.stream_info(gen2, flags=FLAGS_CP, stream=st)
+            for _ in range(2):
+                g2.sweep_best(gen2, rank, ncand, stride=world, flags=FLAGS_CP, stream=st)
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(st)
+            for _ in range(2):
+                g2.sweep_best(gen2, rank, ncand, stride=world, flags=FLAGS_CP, stream=st)
+            e1.record(st)
+            torch.cuda.synchronize()
+            ms2 = e0.elapsed_time(e1) / 2
+            tm2 = g2.last_timing()
+            cps = ncand / (ms2 / 1000.0)
+            configs[name] = {"V": d2.n_ops, "E": d2.n_edges, "G": d2.n_devices, "candidates": ncand,
+                             "time_bits": g2.time_bits, "caps": bool((d2.cap < synth.INT64_MAX).any()),
+                             "candidates_per_s": cps, "ops_per_s": cps * d2.n_ops, "ms_per_sweep": ms2,
+                             "kernel": "k_sim_lane" if tm2["topo"] == 2 else "k_sim",
+                             "deferred_to_prep": tm2["deferred"]}
+            del g2
 
     cpu = None
     parity = None
@@ -425,6 +457,8 @@ def main():
                        "l2": "per-warp state slabs (>1 GB) exceed L2; a 256 MB buffer is written between steps",
                        "parallelism": "candidates sharded c = rank mod N; NCCL all_reduce(MIN) argmin"},
             "best": {"makespan_ns": best[0], "index": best[1]},
+            "ops_per_s": value * V,
+            "configs": configs,
             "roofline": roof,
             "cpu_baseline": cpu,
             "parity": parity,

@@ -2,7 +2,8 @@
 Each translation unit compiles to an object in parallel (relocatable device
 code is not needed: no kernel calls across files), then one link.  The two
 simulation kernels' template instances are split by device-count width GSH:
-k_sim_inst.cu and k_sim_lane_inst.cu are compiled once per GSH = 0..5."""
+k_sim_inst.cu is compiled once per GSH = 0..5, k_sim_lane_inst.cu once per
+(GSH, memory mode MM = 0..2)."""
 from __future__ import annotations
 
 import os
@@ -16,8 +17,10 @@ _C = os.path.join(HERE, "csrc")
 SRCS = [os.path.join(_C, f) for f in ("fastt_abi.cu", "k_prep.cu", "k_sim.cu", "k_sim_lane.cu", "k_fit.cu",
                                       "k_sim_inst.cu", "k_sim_lane_inst.cu")]
 # (source, extra flags): one object per unit
-UNITS = [(s, []) for s in SRCS[:5]] + [(os.path.join(_C, f), ["-DFASTT_GSH=%d" % g])
-                                         for g in range(6) for f in ("k_sim_lane_inst.cu", "k_sim_inst.cu")]
+UNITS = ([(os.path.join(_C, "k_sim_lane_inst.cu"), ["-DFASTT_GSH=%d" % g, "-DFASTT_MM=%d" % m])
+          for g in (5, 4, 3, 2, 1, 0) for m in range(3)] +
+         [(os.path.join(_C, "k_sim_inst.cu"), ["-DFASTT_GSH=%d" % g]) for g in (5, 4, 3, 2, 1, 0)] +
+         [(s, []) for s in SRCS[:5]])
 DEPS = SRCS + [os.path.join(_C, f) for f in ("fastt_internal.cuh", "sim_common.cuh", "k_sim_body.cuh",
                                              "k_sim_lane_body.cuh")] + [os.path.join(ROOT, "include", "fastt.h")]
 OUT = os.path.join(HERE, "libfastt.so")

@@ -190,9 +190,9 @@ struct Base {
   struct Snap {
     bool valid = false;
     int round_dev = -1;
-    char *buf = nullptr;  // dq | avail | ms | rec | rounds
+    char *buf = nullptr;  // dq | avail | ms | rec | rounds | used | used + reserved
     uint32_t *dq = nullptr;
-    void *avail = nullptr, *ms = nullptr, *rec = nullptr;
+    void *avail = nullptr, *ms = nullptr, *rec = nullptr, *used = nullptr, *ur = nullptr;
     int32_t *rounds = nullptr;
   } snap[2];
   void release() {
@@ -255,7 +255,7 @@ struct fastt_graph {
   int sms = 148, sim_block = SIM_BLOCK, sim_grid = 0, sim_tbits = 0, sim_cpw = 1, sim_bm_stride = 0;
   int sim_grid_topo = 0;  // resident blocks of the TOPO variant (no shared-memory ready set)
   bool use_topo = true;   // FASTT_NO_TOPO=1 forces the ready-set path (A/B parity)
-  int sim_grid_lane = 0;  // resident blocks of the lane-per-candidate position-order kernel
+  int sim_grid_lane[3] = {0, 0, 0};  // resident blocks of the lane-per-candidate kernel per memory mode
   // device staging buffers of fastt_schedule_batch (host candidates in,
   // makespan/status out), kept across calls and grown on demand
   struct IoBuf {
@@ -487,12 +487,13 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     if (per_sm < 1) return fail(FASTT_EUNSUP, "simulation kernel does not fit on an SM (smem %zu)", smem);
     g->sim_grid = g->sms * per_sm;
     g->sim_grid_topo = g->sms * std::max(1, sim_occupancy(B.tbits, gsh, g->sim_block, 0, true));
-    g->sim_grid_lane = g->sms * std::max(1, lane_occupancy(B.tbits, gsh));
+    for (int mm = 0; mm < 3; mm++) g->sim_grid_lane[mm] = g->sms * std::max(1, lane_occupancy(B.tbits, gsh, mm));
     g->sim_smem = smem;
     g->sim_cpw = cpw;
     g->sim_bm_stride = stride;
     int64_t nslot = (int64_t)std::max(g->sim_grid, g->sim_grid_topo) * (g->sim_block / 32) * cpw;
-    nslot = std::max<int64_t>(nslot, (int64_t)g->sim_grid_lane * LANE_BLOCK);  // one column per lane
+    for (int mm = 0; mm < 3; mm++)
+      nslot = std::max<int64_t>(nslot, (int64_t)g->sim_grid_lane[mm] * LANE_BLOCK);  // one column per lane
     size_t rec = B.tbits == 32 ? 8 : 16;
     CK(cudaMalloc(&g->slab, (size_t)nslot * ncap * rec));
     CK(cudaMalloc(&g->wbest, sizeof(int64_t) * 2 * nslot));
@@ -537,14 +538,16 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
 // the ready-set variant (slots may differ).
 static void main_shape(fastt_graph *g, const Base &B, SimArgs &a, int &grid, size_t &smem) {
   const bool topo = g->use_topo && B.topo && a.mode != 2;
-  // the lane kernel covers makespan-only evaluation without memory tracking
-  const bool lane = topo && g->use_lane && !a.need_mem && !a.ins && !a.out.place && !a.out.start && !a.out.deq &&
-                    !a.out.peak && a.snap_mode != 1;
+  // the lane kernel covers makespan (+ per-device peak, + memory caps)
+  // without per-op outputs, liveness memory or INSERT
+  const bool lane = topo && g->use_lane && !a.live_mem && !a.ins && !a.out.place && !a.out.start && !a.out.deq &&
+                    a.snap_mode != 1;
   g->last_topo = lane ? 2 : topo ? 1 : 0;
   a.lane = lane;
+  a.lane_mm = a.cap_check ? 2 : (a.out.peak ? 1 : 0);
   if (lane) {
     a.topo = 1;
-    grid = g->sim_grid_lane;
+    grid = g->sim_grid_lane[a.lane_mm];
     smem = 0;
   } else if (topo) {
     a.topo = 1;
@@ -557,8 +560,9 @@ static void main_shape(fastt_graph *g, const Base &B, SimArgs &a, int &grid, siz
   }
 }
 static int max_slots(const fastt_graph *g) {
-  return std::max(std::max(g->sim_grid, g->sim_grid_topo) * (g->sim_block / 32) * g->sim_cpw,
-                  g->sim_grid_lane * (LANE_BLOCK / 32));
+  int gl = 0;
+  for (int mm = 0; mm < 3; mm++) gl = std::max(gl, g->sim_grid_lane[mm]);
+  return std::max(std::max(g->sim_grid, g->sim_grid_topo) * (g->sim_block / 32) * g->sim_cpw, gl * (LANE_BLOCK / 32));
 }
 
 static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
@@ -625,18 +629,18 @@ static fastt_status run_prep(fastt_graph *g, const Base &B, int nslots, cudaStre
 static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cudaStream_t st) {
   Base::Snap &S = B.snap[flags & FASTT_F_CP_PIN ? 1 : 0];
   if (S.valid || (flags & FASTT_F_POLICY_INSERT)) return FASTT_OK;  // (no sharing under INSERT)
-  for (int d = 0; d < g->G; d++)
-    if (g->gch.cap[d] != I64MAX) return FASTT_OK;  // sharing needs unlimited memory
   const size_t tb = B.tbits / 8, n = (size_t)B.pl.ncap;
   const size_t o_dq = 0, o_av = al16(4 * n), o_ms = o_av + al16(tb * (n + 1) * g->G),
                o_rec = o_ms + al16(tb * (n + 1)), o_rd = o_rec + al16((B.tbits == 32 ? 8 : 16) * n),
-               tot = o_rd + 64;
+               o_us = o_rd + 64, o_ur = o_us + al16(8 * (n + 1) * g->G), tot = o_ur + al16(8 * (n + 1) * g->G);
   CK(cudaMalloc(&S.buf, tot));
   S.dq = (uint32_t *)(S.buf + o_dq);
   S.avail = S.buf + o_av;
   S.ms = S.buf + o_ms;
   S.rec = S.buf + o_rec;
   S.rounds = (int32_t *)(S.buf + o_rd);
+  S.used = S.buf + o_us;
+  S.ur = S.buf + o_ur;
   CK(cudaMemsetAsync(S.rounds, 0, 16, st));
   Cand c;
   memset(&c, 0, sizeof c);
@@ -663,6 +667,9 @@ static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cud
   a.snap_ms = S.ms;
   a.snap_rec = S.rec;
   a.snap_rounds = S.rounds;
+  a.snap_used = S.used;  // (memory tracked in the recording run: peak / caps of the lane kernel)
+  a.snap_ur = S.ur;
+  a.need_mem = 1;
   {
     int grid;
     size_t smem;
@@ -679,7 +686,7 @@ static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cud
   cudaFree(d_c);
   cudaFree(d_ms);
   cudaFree(d_st);
-  if (hst != FASTT_CAND_OK) return FASTT_OK;  // (cannot happen without caps)
+  if (hst != FASTT_CAND_OK) return FASTT_OK;  // an infeasible BASE (caps): no sharing
   S.round_dev = (rd[0] == 1 && rd[2] == 0 && rd[3] == B.cp_len) ? rd[1] : -1;
   S.valid = true;
   return FASTT_OK;
@@ -688,8 +695,10 @@ static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cud
 // enable prefix sharing on a launch when the snapshot exists
 static void use_snapshot(const Base &B, uint32_t flags, SimArgs &a) {
   const Base::Snap &S = B.snap[flags & FASTT_F_CP_PIN ? 1 : 0];
-  if (!S.valid || a.need_mem || a.out.place || a.ins) return;
+  if (!S.valid || a.live_mem || a.out.place || a.ins) return;
   a.snap_mode = 2;
+  a.snap_used = S.used;
+  a.snap_ur = S.ur;
   a.snap_round_dev = S.round_dev;
   a.snap_dq = S.dq;
   a.snap_avail = S.avail;
@@ -765,7 +774,7 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
   if (n <= 0) return FASTT_OK;
   TRY(ensure_sim(g, B, n, flags));
   const bool sharing =
-      g->share && !o.peak && !o.place && n >= 64 && !(flags & (FASTT_F_POLICY_INSERT | FASTT_F_MEM_LIVE));
+      g->share && !o.place && n >= 64 && !(flags & (FASTT_F_POLICY_INSERT | FASTT_F_MEM_LIVE));
   if (sharing) TRY(ensure_snapshot(g, B, flags, st));  // before the work counters are reset
   if (o.place) CK(cudaMemsetAsync(o.place, 0xFF, (size_t)n * o.vmax, st));
   if (o.start) {

@@ -232,6 +232,12 @@ struct SimArgs {
   // which a candidate is deferred (0 = packed keys off)
   const uint32_t *costk;
   uint32_t pk_lim;
+  // memory mode of the lane kernel: 0 none, 1 per-device peak, 2 finite caps
+  int32_t lane_mm;
+  // BASE snapshot memory before step t ([(n+1)*G] int64, recorded with the
+  // snapshot): used[d], and used[d] + reserved[d]
+  void *snap_used;
+  void *snap_ur;
 };
 
 // one idle slot [a, b) of a device under INSERT
@@ -248,9 +254,11 @@ void launch_sim(const SimArgs &a, int tbits, int grid, int block, size_t smem, c
 FASTT_DECL_SIM_FN(0) FASTT_DECL_SIM_FN(1) FASTT_DECL_SIM_FN(2) FASTT_DECL_SIM_FN(3) FASTT_DECL_SIM_FN(4)
 FASTT_DECL_SIM_FN(5)
 #undef FASTT_DECL_SIM_FN
-#define FASTT_DECL_LANE_FN(N) const void *lane_fn_g##N(int tbits, int cm, bool exact, bool mg, bool pk);
-FASTT_DECL_LANE_FN(0) FASTT_DECL_LANE_FN(1) FASTT_DECL_LANE_FN(2) FASTT_DECL_LANE_FN(3) FASTT_DECL_LANE_FN(4)
-FASTT_DECL_LANE_FN(5)
+#define FASTT_DECL_LANE_FN(N, M) const void *lane_fn_g##N##_m##M(int tbits, int cm, bool exact, bool mg, bool pk);
+#define FASTT_DECL_LANE_FN3(N) FASTT_DECL_LANE_FN(N, 0) FASTT_DECL_LANE_FN(N, 1) FASTT_DECL_LANE_FN(N, 2)
+FASTT_DECL_LANE_FN3(0) FASTT_DECL_LANE_FN3(1) FASTT_DECL_LANE_FN3(2) FASTT_DECL_LANE_FN3(3) FASTT_DECL_LANE_FN3(4)
+FASTT_DECL_LANE_FN3(5)
+#undef FASTT_DECL_LANE_FN3
 #undef FASTT_DECL_LANE_FN
 void launch_argmin(const int64_t *wbest, int64_t nwarps, int64_t *best_dev, cudaStream_t st);
 void launch_order_chunk(const int32_t *deq, const int64_t *start, int32_t *order, const int64_t *results, int64_t n,
@@ -270,7 +278,7 @@ void launch_gather_sorted(const Cand *src, const int64_t *sidx, const int64_t *s
                           Cand *dst, int64_t *didx, int64_t *dres, cudaStream_t st);
 int sim_occupancy(int tbits, int gshift, int block, size_t smem, bool topo);
 void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st);
-int lane_occupancy(int tbits, int gshift);
+int lane_occupancy(int tbits, int gshift, int mm);
 // costk[p][d] = (cost[p][d] << gshift) | d over n positions; mx[0] = max
 // cost, mx[1] = max edge comm (one link class) of the prepared graph
 void launch_pack_costs(const PrepGraph *pg_dev, int32_t n, int G, int gshift, int64_t E, uint32_t *costk,

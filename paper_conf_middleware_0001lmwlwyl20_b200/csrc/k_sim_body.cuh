@@ -620,6 +620,10 @@ __global__ void __launch_bounds__(SIM_BLOCK, TOPO ? SIM_MINB_TOPO : SIM_MINB) k_
       const int dsel = fm ? __ffs(fm) - 1 - gb : 0;
       if (snap_rec_on && go) {
         if (d < G) ((T *)a.snap_avail)[(size_t)tstep * G + d] = avail;
+        if (MEM && a.snap_used && d < G) {  // memory before the step (lane kernel MM 1 / MM 2)
+          ((int64_t *)a.snap_used)[(size_t)tstep * G + d] = used;
+          ((int64_t *)a.snap_ur)[(size_t)tstep * G + d] = used + reserved;
+        }
         if (d == 0) {
           ((T *)a.snap_ms)[tstep] = makespan;
           a.snap_dq[i] = (uint32_t)tstep;
@@ -752,6 +756,10 @@ __global__ void __launch_bounds__(SIM_BLOCK, TOPO ? SIM_MINB_TOPO : SIM_MINB) k_
     // ------------------------------------------------------------ epilogue
     if (snap_rec_on && run && !infeas) {
       if (d < G) ((T *)a.snap_avail)[(size_t)tstep * G + d] = avail;
+      if (MEM && a.snap_used && d < G) {
+        ((int64_t *)a.snap_used)[(size_t)tstep * G + d] = used;
+        ((int64_t *)a.snap_ur)[(size_t)tstep * G + d] = used + reserved;
+      }
       if (d == 0) ((T *)a.snap_ms)[tstep] = makespan;
     }
     if (run) {

@@ -40,33 +40,46 @@
 
 namespace fastt {
 
-// kernel getters of the per-GSH instance objects (k_sim_lane_inst.cu)
-static const void *lane_fn(int tbits, int gshift, int cm, bool exact, bool mg, bool pk) {
+// kernel getters of the per-(GSH, MM) instance objects (k_sim_lane_inst.cu)
+#define FASTT_LANE_CASE(N)                                                        \
+  case N:                                                                         \
+    return mm == 0 ? lane_fn_g##N##_m0(tbits, cm, exact, mg, pk)                  \
+                   : mm == 1 ? lane_fn_g##N##_m1(tbits, cm, exact, mg, pk)        \
+                             : lane_fn_g##N##_m2(tbits, cm, exact, mg, pk);
+static const void *lane_fn(int tbits, int gshift, int cm, bool exact, bool mg, bool pk, int mm) {
   switch (gshift) {
-    case 0: return lane_fn_g0(tbits, cm, exact, mg, pk);
-    case 1: return lane_fn_g1(tbits, cm, exact, mg, pk);
-    case 2: return lane_fn_g2(tbits, cm, exact, mg, pk);
-    case 3: return lane_fn_g3(tbits, cm, exact, mg, pk);
-    case 4: return lane_fn_g4(tbits, cm, exact, mg, pk);
-    default: return lane_fn_g5(tbits, cm, exact, mg, pk);
+    FASTT_LANE_CASE(0)
+    FASTT_LANE_CASE(1)
+    FASTT_LANE_CASE(2)
+    FASTT_LANE_CASE(3)
+    FASTT_LANE_CASE(4)
+    default:
+      FASTT_LANE_CASE(5)
   }
 }
+#undef FASTT_LANE_CASE
 
-template <typename T, bool MG> static size_t lane_smem_t(int gshift) {
+template <typename T, bool MG, int MM> static size_t lane_smem_t(int gshift) {
   switch (gshift) {
-    case 0: return lane_smem_per_warp<T, 1, MG>();
-    case 1: return lane_smem_per_warp<T, 2, MG>();
-    case 2: return lane_smem_per_warp<T, 4, MG>();
-    case 3: return lane_smem_per_warp<T, 8, MG>();
-    case 4: return lane_smem_per_warp<T, 16, MG>();
-    default: return lane_smem_per_warp<T, 32, MG>();
+    case 0: return lane_smem_per_warp<T, 1, MG, MM>();
+    case 1: return lane_smem_per_warp<T, 2, MG, MM>();
+    case 2: return lane_smem_per_warp<T, 4, MG, MM>();
+    case 3: return lane_smem_per_warp<T, 8, MG, MM>();
+    case 4: return lane_smem_per_warp<T, 16, MG, MM>();
+    default: return lane_smem_per_warp<T, 32, MG, MM>();
   }
+}
+template <bool MG> static size_t lane_smem_w(int tbits, int gshift, int mm) {
+  if (tbits == 32)
+    return mm == 0 ? lane_smem_t<uint32_t, MG, 0>(gshift)
+                   : mm == 1 ? lane_smem_t<uint32_t, MG, 1>(gshift) : lane_smem_t<uint32_t, MG, 2>(gshift);
+  return mm == 0 ? lane_smem_t<uint64_t, MG, 0>(gshift)
+                 : mm == 1 ? lane_smem_t<uint64_t, MG, 1>(gshift) : lane_smem_t<uint64_t, MG, 2>(gshift);
 }
 // dynamic shared memory of a block: LANE_BLOCK threads, or one warp (MG)
-size_t lane_smem(int tbits, int gshift, bool mg) {
-  if (mg) return tbits == 32 ? lane_smem_t<uint32_t, true>(gshift) : lane_smem_t<uint64_t, true>(gshift);
-  return (LANE_BLOCK / 32) *
-         (tbits == 32 ? lane_smem_t<uint32_t, false>(gshift) : lane_smem_t<uint64_t, false>(gshift));
+size_t lane_smem(int tbits, int gshift, bool mg, int mm) {
+  if (mg) return lane_smem_w<true>(tbits, gshift, mm);
+  return (LANE_BLOCK / 32) * lane_smem_w<false>(tbits, gshift, mm);
 }
 
 __global__ void k_pack_costs(const PrepGraph *pgp, int32_t n, int G, int gshift, int64_t E, uint32_t *costk,
@@ -102,21 +115,25 @@ void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
   const bool mg = a.lane == 2;
   const int cm = lane_comm_mode(a, tbits);
   const bool pk = !mg && tbits == 32 && cm != 2 && a.costk != nullptr && a.pk_lim > 0;
-  const void *f = lane_fn(tbits, a.gshift, cm, a.G == (1 << a.gshift), mg, pk);
-  const size_t sm = lane_smem(tbits, a.gshift, mg);
+  const void *f = lane_fn(tbits, a.gshift, cm, a.G == (1 << a.gshift), mg, pk, a.lane_mm);
+  const size_t sm = lane_smem(tbits, a.gshift, mg, a.lane_mm);
   if (mg) cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
   SimArgs aa = a;
   void *args[] = {&aa};
   cudaLaunchKernel(f, dim3(grid), dim3(mg ? 32 : LANE_BLOCK), args, sm, st);
 }
 
-int lane_occupancy(int tbits, int gshift) {
+// resident blocks per SM of the base-graph launch of memory mode mm (the
+// minimum over its comm / exactness / packed-key variants); sets their
+// dynamic shared memory limit
+int lane_occupancy(int tbits, int gshift, int mm) {
   int nb = 1 << 30, x = 0;
+  const size_t sm = lane_smem(tbits, gshift, false, mm);
   for (int v = (tbits == 32 ? 0 : 2); v < (tbits == 32 ? 10 : 6); v++) {
-    const void *f = v < 6 ? lane_fn(tbits, gshift, v >> 1, v & 1, false, false)
-                          : lane_fn(tbits, gshift, (v - 6) >> 1, v & 1, false, true);
-    cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lane_smem(tbits, gshift, false));
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, f, LANE_BLOCK, lane_smem(tbits, gshift, false));
+    const void *f = v < 6 ? lane_fn(tbits, gshift, v >> 1, v & 1, false, false, mm)
+                          : lane_fn(tbits, gshift, (v - 6) >> 1, v & 1, false, true, mm);
+    cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, f, LANE_BLOCK, sm);
     nb = x < nb ? x : nb;
   }
   return nb;

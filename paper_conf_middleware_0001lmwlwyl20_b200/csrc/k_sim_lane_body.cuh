@@ -17,25 +17,36 @@ namespace fastt {
 #endif
 template <typename T> struct LaneDepth { static constexpr int D = sizeof(T) == 4 ? LANE_D : LANE_D / 2; };
 // staged card of one position: header (words 0-3), predecessor positions
-// (words 8-11), the inline predecessors' comm values (4 x T), then the cost
-// row padded to 16 B
-template <typename T> __host__ __device__ constexpr int card_cost_off() { return 32 + 4 * (int)sizeof(T); }
-template <typename T, int GP> __host__ __device__ constexpr int card_slot_bytes() {
-  return card_cost_off<T>() + (int)((GP * sizeof(T) + 15) / 16) * 16;
+// (words 8-11), the inline predecessors' comm values (4 x T), with memory
+// tracking (MM > 0) header words 4-7 (mem lo/hi), then the cost row padded
+// to 16 B
+template <typename T> __host__ __device__ constexpr int card_hdr1_off() { return 32 + 4 * (int)sizeof(T); }
+template <typename T, int MM> __host__ __device__ constexpr int card_cost_off() {
+  return card_hdr1_off<T>() + (MM ? 16 : 0);
+}
+template <typename T, int GP, int MM> __host__ __device__ constexpr int card_slot_bytes() {
+  return card_cost_off<T, MM>() + (int)((GP * sizeof(T) + 15) / 16) * 16;
 }
 // MG: per-lane card regions are 2D slots + 16 B apart, so the 8 lanes of a
 // 128-bit shared-memory phase hit distinct bank quads (a 2D x CS stride is a
 // multiple of 128 B: every lane's card load would fall in the same banks)
-template <typename T, int GP> __host__ __device__ constexpr int mg_lane_stride() {
-  return 2 * LaneDepth<T>::D * card_slot_bytes<T, GP>() + 16;
+template <typename T, int GP, int MM> __host__ __device__ constexpr int mg_lane_stride() {
+  return 2 * LaneDepth<T>::D * card_slot_bytes<T, GP, MM>() + 16;
 }
-template <typename T, int GP, bool MG> __host__ __device__ constexpr size_t lane_smem_per_warp() {
+// offset of the memory-tracking area in a warp's shared memory
+template <typename T, int GP, bool MG, int MM> __host__ __device__ constexpr size_t lane_mm_off() {
+  return (size_t)LaneDepth<T>::D * 5 * 32 * (sizeof(T) == 4 ? 8 : 16) +
+         (MG ? (size_t)32 * mg_lane_stride<T, GP, MM>() : (size_t)2 * LaneDepth<T>::D * card_slot_bytes<T, GP, MM>()) +
+         (size_t)(MG ? 0 : 32 * GP * 4);
+}
+template <typename T, int GP, bool MG, int MM> __host__ __device__ constexpr size_t lane_smem_per_warp() {
   // ring D x 32 + stage D x 4 x 32 records, then 2D staged cards (per lane
   // in the multi-graph variant), then (base-graph launches) the packed-key
-  // avail rows [32 lanes][GP] of the PK variant
-  return (size_t)LaneDepth<T>::D * 5 * 32 * (sizeof(T) == 4 ? 8 : 16) +
-         (MG ? (size_t)32 * mg_lane_stride<T, GP>() : (size_t)2 * LaneDepth<T>::D * card_slot_bytes<T, GP>()) +
-         (size_t)(MG ? 0 : 32 * GP * 4);
+  // avail rows [32 lanes][GP] of the PK variant, then the memory state:
+  // MM 1 used[d] (int64 [GP][32]); MM 2 slack[d] = cap - used - reserved
+  // (int64 [GP][32]), its clamped 32-bit copy (quads [GP/4][32][4]) and the
+  // CP rounds ([GP][32] u32)
+  return lane_mm_off<T, GP, MG, MM>() + (MM >= 1 ? (size_t)32 * GP * 8 : 0) + (MM == 2 ? (size_t)32 * GP * 8 : 0);
 }
 
 template <int BYTES> __device__ __forceinline__ void cp_async(uint32_t saddr, const void *g);
@@ -131,6 +142,101 @@ template <> struct RowLd<uint64_t> {
   }
 };
 
+// CP devices under memory caps (Alg. 1 line 5, R9),
+// one candidate per lane: repeatedly give the device with the smallest exact
+// average cost (cross-multiplied, ties lowest id) the longest prefix of the
+// remaining free CP ops that fits its cap, reserve that memory up front
+// (slack[d] -= the prefix's mem), and drop the device; perturbation-pinned CP
+// ops are excluded (free-index space).  Round r is stored as rnd[r * 32] =
+// (raw CP index just past its last op) | device << 24; returns the count.
+template <typename T>
+__device__ __noinline__ int cp_rounds_lane(const PrepGraph *pg, const GraphConst &gc, int G, uint32_t dset, int np,
+                                           const uint32_t *pp, const uint32_t *pc, uint32_t *rnd, int64_t *mv) {
+  const T *costp = (const T *)pg->costp;
+  const uint32_t *card = pg->card;
+  const int32_t L = pg->cp_len;
+  uint32_t pcs[MAXPINS], pps[MAXPINS];
+  int64_t pms[MAXPINS];
+  int m = 0;
+  for (int k = 0; k < np; k++) {
+    if (pc[k] == NONE) continue;
+    const uint32_t *ci = card + (size_t)pp[k] * CARD_WORDS;
+    const int64_t mk = (int64_t)(((uint64_t)ci[CW_MEMHI] << 32) | ci[CW_MEMLO]);
+    int j = m++;
+    while (j > 0 && pcs[j - 1] > pc[k]) {
+      pcs[j] = pcs[j - 1];
+      pps[j] = pps[j - 1];
+      pms[j] = pms[j - 1];
+      j--;
+    }
+    pcs[j] = pc[k];
+    pps[j] = pp[k];
+    pms[j] = mk;
+  }
+  auto raw_end = [&](int32_t f) -> int32_t {  // raw CP index just past the f-th free op (f >= 1)
+    int32_t r = f - 1;
+    for (int j = 0; j < m; j++)
+      if ((int32_t)pcs[j] <= r) r++;
+    return r + 1;
+  };
+  auto fp_mem = [&](int32_t f) -> int64_t {
+    if (f <= 0) return 0;
+    const int32_t re = raw_end(f);
+    int64_t v = pg->pmem[re];
+    for (int j = 0; j < m; j++)
+      if ((int32_t)pcs[j] < re) v -= pms[j];
+    return v;
+  };
+  auto fp_cost = [&](int32_t f, int d) -> int64_t {
+    if (f <= 0) return 0;
+    const int32_t re = raw_end(f);
+    int64_t v = pg->pcost[(int64_t)re * G + d];
+    for (int j = 0; j < m; j++)
+      if ((int32_t)pcs[j] < re) v -= (int64_t)costp[(size_t)pps[j] * G + d];
+    return v;
+  };
+  const int32_t Lf = L - m;
+  uint32_t devs = dset;
+  int32_t k = 0;
+  int nr = 0;
+  while (k < Lf && devs) {
+    const int64_t bm = fp_mem(k), rest = fp_mem(Lf) - bm;
+    int best = -1;
+    int32_t tb = 0;
+    int64_t Sb = 0;
+    for (int d = 0; d < G; d++) {
+      if (!((devs >> d) & 1u)) continue;
+      const int64_t cap = gc.cap[d];
+      int32_t t;
+      if (rest <= cap) {
+        t = Lf - k;
+      } else {  // fp(k + lo) - bm <= cap < fp(k + hi) - bm
+        int32_t lo = 0, hi = Lf - k;
+        while (hi - lo > 1) {
+          const int32_t mid = (lo + hi) >> 1;
+          if (fp_mem(k + mid) - bm <= cap) lo = mid;
+          else hi = mid;
+        }
+        t = lo;
+      }
+      if (t <= 0) continue;
+      const int64_t S = fp_cost(k + t, d) - fp_cost(k, d);
+      if (best < 0 || lt_cross((uint64_t)S, (uint64_t)tb, (uint64_t)Sb, (uint64_t)t)) {
+        best = d;
+        tb = t;
+        Sb = S;
+      }
+    }
+    if (best < 0) break;
+    mv[best * 32] -= fp_mem(k + tb) - bm;
+    rnd[nr * 32] = (uint32_t)raw_end(k + tb) | ((uint32_t)best << 24);
+    devs &= ~(1u << best);
+    k += tb;
+    nr++;
+  }
+  return nr;
+}
+
 // CM: 0 = uint32 time and one link class, comm values inline in the card;
 //     1 = one link class, comm per edge from pe_comm;
 //     2 = several link classes (per (pred, device) comm).
@@ -149,7 +255,12 @@ template <> struct RowLd<uint64_t> {
 //     cost at every step, so a candidate whose final makespan reaches
 //     pk_lim = 2^(32-GSH) - max cost - max comm is deferred and re-run by the
 //     preparation pipeline (unpacked kernels).
-template <typename T, int GSH, int CM, bool EX, bool MG, bool PK>
+// MM: memory (Alg. 1 line 13, R8): 0 none; 1 per-device peak only (no caps:
+//     used[d] += mem of every op placed on d); 2 finite caps -- lane-local CP
+//     rounds (R9, memory reserved up front), slack[d] = cap - used - reserved
+//     per lane, a device is feasible iff mem_i <= slack[d] (a CP-pinned op
+//     draws on its reservation), no feasible device => INFEASIBLE.
+template <typename T, int GSH, int CM, bool EX, bool MG, bool PK, int MM>
 __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   typedef typename Slab<T>::W W;
   constexpr int GP = 1 << GSH;
@@ -163,30 +274,47 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   // and stage[D][4][32] (inline predecessors' records prefetched by cp.async)
   constexpr int D = LaneDepth<T>::D, P = D - 1;
   extern __shared__ __align__(16) unsigned char lsm[];
-  unsigned char *const wsm = lsm + (threadIdx.x >> 5) * lane_smem_per_warp<T, GP, MG>();
+  unsigned char *const wsm = lsm + (threadIdx.x >> 5) * lane_smem_per_warp<T, GP, MG, MM>();
   W *const ring = (W *)wsm + lane;
   W *const stage = ring + D * 32;
   const uint32_t stage_sa = (uint32_t)__cvta_generic_to_shared(stage);
   // 2D staged cards (warp-shared): the card of position u is copied at step
   // u - 2P and read at steps u - P (record prefetch) and u (compute)
-  constexpr int CS = card_slot_bytes<T, GP>();
-  const unsigned char *const cards = wsm + (size_t)D * 5 * 32 * sizeof(W) + (MG ? (size_t)lane * mg_lane_stride<T, GP>() : 0);
+  constexpr int CS = card_slot_bytes<T, GP, MM>();
+  const unsigned char *const cards = wsm + (size_t)D * 5 * 32 * sizeof(W) + (MG ? (size_t)lane * mg_lane_stride<T, GP, MM>() : 0);
   const uint32_t cards_sa = (uint32_t)__cvta_generic_to_shared(cards);
   // PK: avail[d] << GSH of every lane, after the warp's cards, as device
   // pairs [d / 2][32 lanes][2] (a pair per lane is one 64-bit access; the
   // indexed access of device d by all lanes is 2-way conflicted at most)
-  uint32_t *const avk = (uint32_t *)(wsm + (size_t)D * 5 * 32 * sizeof(W) + (size_t)2 * D * card_slot_bytes<T, GP>()) +
+  uint32_t *const avk = (uint32_t *)(wsm + (size_t)D * 5 * 32 * sizeof(W) + (size_t)2 * D * CS) +
                         (GP >= 2 ? 2 * lane : lane);
   auto avk_at = [&](uint32_t d) -> uint32_t & { return GP >= 2 ? avk[(d >> 1) * 64 + (d & 1)] : avk[0]; };
-  constexpr int CO = card_cost_off<T>();
+  // memory state (MM): mv[d * 32] = used[d] (MM 1) or slack[d] (MM 2), int64;
+  // MM 2: s32 = min(slack, 2^32 - 1) as quads [d / 4][32 lanes][4] (one
+  // 128-bit load per 4 devices), rnd[r * 32] = CP round r: raw CP index just
+  // past the round | device << 24
+  int64_t *const mv = (int64_t *)(wsm + lane_mm_off<T, GP, MG, MM>()) + lane;
+  uint32_t *const s32b = (uint32_t *)(wsm + lane_mm_off<T, GP, MG, MM>() + (size_t)32 * GP * 8) + (GP >= 4 ? 4 * lane : lane);
+  uint32_t *const rnd = (uint32_t *)(wsm + lane_mm_off<T, GP, MG, MM>() + (size_t)32 * GP * 12) + lane;
+  auto s32_at = [&](uint32_t d) -> uint32_t & { return GP >= 4 ? s32b[(d >> 2) * 128 + (d & 3)] : s32b[d * 32]; };
+  auto clamp32 = [](int64_t v) -> uint32_t { return v >= (int64_t)0xFFFFFFFFll ? 0xFFFFFFFFu : (uint32_t)v; };
+  constexpr int CO = card_cost_off<T, MM>();
+  constexpr int HO = card_hdr1_off<T>();
   const bool row16 = (a.G * (int)sizeof(T)) % 16 == 0;
   // this lane's 16-B chunk of a card copy: lane 0 header (words 0-3), lane 1
-  // predecessor positions (8-11), lane 2 comm (12-15, CM 0), lanes 3.. the
-  // cost row (when its length is a multiple of 16 B, else element-wise)
-  const bool cc_cost = lane >= 3;
-  const uint32_t cc_src = lane == 0 ? 0u : lane == 1 ? 4u * CARD_HDR : lane == 2 ? 4u * CW_PCOMM : 16u * (lane - 3);
-  const uint32_t cc_dst = lane < 3 ? 16u * lane : (uint32_t)CO + 16u * (lane - 3);
-  const bool cc_on = lane < 2 || (lane == 2 && CM == 0) || (lane >= 3 && lane - 3 < a.G * (int)sizeof(T) / 16);
+  // predecessor positions (8-11), lane 2 comm (12-15, CM 0), lane 3 header
+  // words 4-7 (MM), lanes C0.. the cost row (when its length is a multiple
+  // of 16 B, else element-wise)
+  constexpr int C0 = MM ? 4 : 3;
+  const bool cc_cost = lane >= C0;
+  const uint32_t cc_src = lane == 0   ? 0u
+                          : lane == 1 ? 4u * CARD_HDR
+                          : lane == 2 ? 4u * CW_PCOMM
+                          : (MM && lane == 3) ? 16u
+                                              : 16u * (lane - C0);
+  const uint32_t cc_dst = lane < 3 ? 16u * lane : (MM && lane == 3) ? (uint32_t)HO : (uint32_t)CO + 16u * (lane - C0);
+  const bool cc_on = lane < 2 || (lane == 2 && CM == 0) || (MM && lane == 3) ||
+                     (lane >= C0 && lane - C0 < a.G * (int)sizeof(T) / 16);
   const GraphConst &gc = *a.gc;
   const int G = a.G;
   const int K = gc.K;
@@ -305,6 +433,8 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     if (active && !defer && st && res_idx >= 0) {
       a.out.makespan[res_idx] = I64MAX;
       a.out.status[res_idx] = st;
+      if (MM && a.out.peak)
+        for (int d = 0; d < G; d++) a.out.peak[res_idx * G + d] = -1;
     }
     const bool run = active && !defer && st == 0;
 
@@ -313,7 +443,15 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     // round over the free CP ops (perturbation-pinned CP ops excluded)
     int r_dev = -1;
     int m = 0;
+    // MM 2: CP rounds (count, cursor, raw end and device of the current one)
+    int nr = 0, rc = 0, rdv = -1;
+    uint32_t rhi = 0;
+    bool dead = false;  // MM 2: no feasible device at some step (R8)
     const uint32_t dmask = (MG && c.dev_mask) ? c.dev_mask : all;  // the candidate's devices (R25)
+    if (MM && run) {
+#pragma unroll
+      for (int d = 0; d < GP; d++) mv[d * 32] = (MM == 2 && d < G) ? gc.cap[d] : 0;
+    }
     if (run && cp_on && cpl > 0) {
       uint32_t pc[MAXPINS];
 #pragma unroll
@@ -321,7 +459,13 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
         pc[k] = k < np ? __ldg(card + (size_t)pp[k] * CARD_WORDS + CW_CPIDX) : NONE;
         m += pc[k] != NONE;
       }
-      if (cpl - m > 0) {
+      if (MM == 2) {
+        nr = cp_rounds_lane<T>(pg, gc, G, dmask, np, pp, pc, rnd, mv);
+        if (nr > 0) {
+          rhi = rnd[0] & 0xFFFFFFu;
+          rdv = (int)(rnd[0] >> 24);
+        }
+      } else if (cpl - m > 0) {
         int64_t bs = 0;
         for (int d = 0; d < G; d++) {
           if (MG && !((dmask >> d) & 1u)) continue;
@@ -340,8 +484,9 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     // no caps => the BASE schedule up to the first pinned op's step t0
     int32_t t0 = 0;
     bool share = false;
-    if (!MG && run && a.snap_mode == 2) {
-      share = m == 0 || (a.snap_round_dev >= 0 && r_dev == a.snap_round_dev);
+    if (!MG && run && a.snap_mode == 2 && (!MM || a.snap_used)) {
+      // (caps: the same free CP list gives the base's rounds and reservations)
+      share = m == 0 || (MM != 2 && a.snap_round_dev >= 0 && r_dev == a.snap_round_dev);
       if (share) {
         t0 = n;
         for (int k = 0; k < np; k++) {
@@ -374,6 +519,15 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       for (int d = 0; d < GP; d++)
         if (d < G) avail[d] = __ldg(sa + d);
       ms = __ldg((const T *)a.snap_ms + lo);
+      // memory before step lo: used (MM 1), cap - used - reserved (MM 2)
+      if (MM == 1)
+        for (int d = 0; d < G; d++) mv[d * 32] = __ldg((const int64_t *)a.snap_used + (size_t)lo * G + d);
+      if (MM == 2)
+        for (int d = 0; d < G; d++) mv[d * 32] = gc.cap[d] - __ldg((const int64_t *)a.snap_ur + (size_t)lo * G + d);
+    }
+    if (MM == 2 && run) {
+#pragma unroll
+      for (int d = 0; d < GP; d++) s32_at(d) = clamp32(mv[d * 32]);
     }
     if (PK) {
 #pragma unroll
@@ -414,6 +568,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
           cp_async<16>(dst, cu);
           cp_async<16>(dst + 16, cu + 4 * CARD_HDR);
           if (CM == 0) cp_async<16>(dst + 32, cu + 4 * CW_PCOMM);
+          if (MM) cp_async<16>(dst + HO, cu + 16);
           if (row16) {
             for (int j = 0; j < G * (int)sizeof(T) / 16; j++) cp_async<16>(dst + CO + 16 * j, row + 16 * j);
           } else {
@@ -470,7 +625,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       cp_async_commit();
     }
     for (int32_t t = lo; t < nmax; t++) {
-      const bool live = run && (!MG || t < n);
+      const bool live = run && !dead && (!MG || t < n);
       cp_async_wait<P - 1>();  // the group of step t - P: records of t, card of t + P
       __syncwarp();            // (cards were copied by other lanes)
       const unsigned char *cs = cards + (t & (2 * D - 1)) * CS;
@@ -481,6 +636,15 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       const T *cm1 = (const T *)(cs + 32);  // CM 1: staged comm values
       T cst[GP];
       RowLd<T>::template load_s<GP>((const T *)(cs + CO), G, cst);
+      // the op's memory (card words 4-5, MM)
+      uint32_t memlo = 0, memhi = 0;
+      if (MM) {
+        const uint2 mw = *(const uint2 *)(cs + HO);
+        memlo = mw.x;
+        memhi = mw.y;
+      }
+      const int64_t mem64 = (int64_t)(((uint64_t)memhi << 32) | memlo);
+      bool cpf = false;  // the device is forced by a CP round (its memory is reserved)
       // (MG: a lane past its slot's last position reads a stale card)
       const uint32_t npred = (!MG || live) ? (h0.x & 0xFFFF) : 0u;
       const uint32_t src[4] = {hs.x, hs.y, hs.z, hs.w};
@@ -581,6 +745,39 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
           arrd[d] = v;
         }
       }
+      // the device forced by a perturbation pin (hard) or a CP round (Alg. 1
+      // l.9-10, R9; cpf: memory reserved up front) -- rare steps: the next
+      // pinned position, or a CP op while the lane has a CP device
+      const bool cp_any = MM == 2 ? rc < nr : r_dev >= 0;
+      auto forced_dev = [&]() -> int {
+        int forced = -1;
+        if ((uint32_t)t == nxt) {
+          nxt = NONE;
+#pragma unroll
+          for (int k = 0; k < MAXPINS; k++) {
+            if (pp[k] == (uint32_t)t) forced = (int)((pdv >> (8 * k)) & 0xFFu);
+            else if (pp[k] > (uint32_t)t && pp[k] < nxt) nxt = pp[k];
+          }
+        }
+        if (forced < 0 && h0.w != NONE) {
+          if (MM == 2) {
+            // CP ops come in CP order (positions are topological): advance
+            // to the round holding raw CP index h0.w
+            while (rc < nr && h0.w >= rhi) {
+              rc++;
+              if (rc < nr) {
+                rhi = rnd[rc * 32] & 0xFFFFFFu;
+                rdv = (int)(rnd[rc * 32] >> 24);
+              }
+            }
+            if (rc < nr) forced = rdv;
+          } else if (r_dev >= 0) {
+            forced = r_dev;
+          }
+          cpf = forced >= 0;
+        }
+        return forced;
+      };
       if (PK) {
         // keys (EFT << GSH) | d: EST = max(avail[d], arrival),
         // arrival M on every device but pa, E on pa (R6); min key = EFT
@@ -605,30 +802,63 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
 #pragma unroll
         for (int d = 0; d < GP; d++)
           key[d] = (EX || d < G) ? (av[d] > Mk ? av[d] : Mk) + (uint32_t)cst[d] : 0xFFFFFFFFu;
-        uint32_t bk = kpa;
+        // MM 2: a device is feasible iff mem_i <= slack[d] (Alg. 1 line 13,
+        // R8); infeasible keys become ~0 (the 32-bit slack copy decides when
+        // the op's memory is below 2^32, exactly: slack >= 2^32 clamps to
+        // 2^32 - 1 >= mem)
+        uint32_t fk[GP], fkpa = kpa;
 #pragma unroll
-        for (int d = 0; d < GP; d++) bk = key[d] < bk ? key[d] : bk;
-        // device forced by a perturbation pin (hard) or a CP pin (Alg. 1
-        // l.9-10): rare steps
-        if (__any_sync(FULL, (uint32_t)t == nxt || (h0.w != NONE && r_dev >= 0))) {
-          int forced = -1;
-          if ((uint32_t)t == nxt) {
-            nxt = NONE;
-#pragma unroll
-            for (int k = 0; k < MAXPINS; k++) {
-              if (pp[k] == (uint32_t)t) forced = (int)((pdv >> (8 * k)) & 0xFFu);
-              else if (pp[k] > (uint32_t)t && pp[k] < nxt) nxt = pp[k];
-            }
-          }
-          if (forced < 0 && r_dev >= 0 && h0.w != NONE) forced = r_dev;
-          if (forced >= 0) {
+        for (int d = 0; d < GP; d++) fk[d] = key[d];
+        if (MM == 2) {
+          if (memhi != 0) {  // (warp-uniform)
 #pragma unroll
             for (int d = 0; d < GP; d++)
-              if (d == forced) bk = key[d];
-            if ((uint32_t)forced == pq && kpa < bk) bk = kpa;
+              if (mv[d * 32] < mem64) fk[d] = 0xFFFFFFFFu;
+            if (mv[pq * 32] < mem64) fkpa = 0xFFFFFFFFu;
+          } else {
+            uint32_t sv[GP];
+            if (GP >= 4) {
+#pragma unroll
+              for (int j = 0; j < GP / 4; j++) {
+                const uint4 x = *(const uint4 *)(s32b + j * 128);
+                sv[4 * j] = x.x;
+                sv[4 * j + 1] = x.y;
+                sv[4 * j + 2] = x.z;
+                sv[4 * j + 3] = x.w;
+              }
+            } else {
+#pragma unroll
+              for (int d = 0; d < GP; d++) sv[d] = s32b[d * 32];
+            }
+#pragma unroll
+            for (int d = 0; d < GP; d++)
+              if (sv[d] < memlo) fk[d] = 0xFFFFFFFFu;
+            if (s32_at(pq) < memlo) fkpa = 0xFFFFFFFFu;
           }
         }
-        if (live) {
+        uint32_t bk = fkpa;
+#pragma unroll
+        for (int d = 0; d < GP; d++) bk = fk[d] < bk ? fk[d] : bk;
+        if (__any_sync(FULL, (uint32_t)t == nxt || (h0.w != NONE && cp_any))) {
+          const int forced = forced_dev();
+          if (forced >= 0) {  // (a CP round's device draws on its reservation)
+#pragma unroll
+            for (int d = 0; d < GP; d++)
+              if (d == forced) bk = cpf ? key[d] : fk[d];
+            const uint32_t kp = cpf ? kpa : fkpa;
+            if ((uint32_t)forced == pq && kp < bk) bk = kp;
+          }
+        }
+        const bool go = live && (MM != 2 || bk != 0xFFFFFFFFu);
+        if (MM == 2 && live && !go) dead = true;  // no feasible device: INFEASIBLE
+        if (go) {
+          const uint32_t dc = bk & (uint32_t)(GP - 1);
+          if (MM == 1) mv[dc * 32] += mem64;
+          if (MM == 2 && !cpf) {
+            const int64_t v = mv[dc * 32] - mem64;
+            mv[dc * 32] = v;
+            s32_at(dc) = clamp32(v);
+          }
           const uint32_t bkc = bk & ~(uint32_t)(GP - 1);
           avk_at(bk & (uint32_t)(GP - 1)) = bkc;
           const T best = (T)(bkc >> GSH);
@@ -648,35 +878,40 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
         const T est = avail[d] > arr ? avail[d] : arr;
         eft[d] = ((EX || d < G) && (!MG || ((dmask >> d) & 1u))) ? est + cst[d] : TT<T>::MAXV;
       }
-      T best = eft[0];
+      // MM 2: memory-feasible devices only (Alg. 1 line 13, R8)
+      T feft[GP];
+#pragma unroll
+      for (int d = 0; d < GP; d++) {
+        bool fe = true;
+        if (MM == 2) fe = memhi != 0 ? mv[d * 32] >= mem64 : s32_at(d) >= memlo;
+        feft[d] = fe ? eft[d] : TT<T>::MAXV;
+      }
+      T best = feft[0];
       int bd = 0;
 #pragma unroll
       for (int d = 1; d < GP; d++)
-        if (eft[d] < best) {
-          best = eft[d];
+        if (feft[d] < best) {
+          best = feft[d];
           bd = d;
         }
-      // device forced by a perturbation pin (hard) or a CP pin (Alg. 1
-      // l.9-10): rare steps -- the next pinned position, or a CP op
-      if (__any_sync(FULL, (uint32_t)t == nxt || (h0.w != NONE && r_dev >= 0))) {
-        int forced = -1;
-        if ((uint32_t)t == nxt) {
-          nxt = NONE;
-#pragma unroll
-          for (int k = 0; k < MAXPINS; k++) {
-            if (pp[k] == (uint32_t)t) forced = (int)((pdv >> (8 * k)) & 0xFFu);
-            else if (pp[k] > (uint32_t)t && pp[k] < nxt) nxt = pp[k];
-          }
-        }
-        if (forced < 0 && r_dev >= 0 && h0.w != NONE) forced = r_dev;
-        if (forced >= 0) {
+      if (__any_sync(FULL, (uint32_t)t == nxt || (h0.w != NONE && cp_any))) {
+        const int forced = forced_dev();
+        if (forced >= 0) {  // (a CP round's device draws on its reservation)
 #pragma unroll
           for (int d = 0; d < GP; d++)
-            if (d == forced) best = eft[d];
+            if (d == forced) best = cpf ? eft[d] : feft[d];
           bd = forced;
         }
       }
-      if (live) {
+      const bool go = live && (MM != 2 || best != TT<T>::MAXV);
+      if (MM == 2 && live && !go) dead = true;  // no feasible device: INFEASIBLE
+      if (go) {
+        if (MM == 1) mv[bd * 32] += mem64;
+        if (MM == 2 && !cpf) {
+          const int64_t v = mv[bd * 32] - mem64;
+          mv[bd * 32] = v;
+          s32_at(bd) = clamp32(v);
+        }
 #pragma unroll
         for (int d = 0; d < GP; d++)
           if (d == bd) avail[d] = best;
@@ -696,10 +931,15 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       a.defer_q[k] = q;
     } else if (run) {
       if (res_idx >= 0) {
-        a.out.makespan[res_idx] = (int64_t)ms;
-        a.out.status[res_idx] = 0;
+        a.out.makespan[res_idx] = dead ? I64MAX : (int64_t)ms;
+        a.out.status[res_idx] = dead ? 1 : 0;
+        // per-device peak (R8: the final static total; reservations are all
+        // drawn by then), -1 when infeasible
+        if (MM && a.out.peak)
+          for (int d = 0; d < G; d++)
+            a.out.peak[res_idx * G + d] = dead ? -1 : (MM == 1 ? mv[d * 32] : gc.cap[d] - mv[d * 32]);
       }
-      if ((int64_t)ms < bms || ((int64_t)ms == bms && sidx < bidx)) {
+      if (!dead && ((int64_t)ms < bms || ((int64_t)ms == bms && sidx < bidx))) {
         bms = (int64_t)ms;
         bidx = sidx;
       }

@@ -43,9 +43,9 @@ def _graph_env(desc, **env):
                 os.environ[k] = v
 
 
-def topo_dag(seed, V, G, K=1, homogeneous=False, scale=1):
+def topo_dag(seed, V, G, K=1, homogeneous=False, scale=1, caps="none"):
     """random DAG with every op cost > 0 (topological priority order)"""
-    d = synth.random_dag(seed, V=V, G=G, K=K, zero_frac=0.0, caps="none", homogeneous=homogeneous)
+    d = synth.random_dag(seed, V=V, G=G, K=K, zero_frac=0.0, caps=caps, homogeneous=homogeneous)
     cost = np.maximum(d.cost, 1) * scale
     return dataclasses.replace(d, cost=cost)
 
@@ -63,18 +63,22 @@ def pin_cands(desc, rng, n, kmax=4):
     return out
 
 
-def check(desc, cands, flags, expect_kernel=LANE, oracle_every=1):
+def check(desc, cands, flags, expect_kernel=LANE, oracle_every=1, peak=False):
     gl = F.Graph(desc)
     gg = _graph_env(desc, FASTT_NO_LANE="1")
-    r = gl.schedule_batch(cands, flags=flags, peak=False)
+    r = gl.schedule_batch(cands, flags=flags, peak=peak)
     assert gl.last_timing()["topo"] == expect_kernel
-    r0 = gg.schedule_batch(cands, flags=flags, peak=False)
+    r0 = gg.schedule_batch(cands, flags=flags, peak=peak)
     assert gg.last_timing()["topo"] in (0, GROUP)
     assert (r["makespan"] == r0["makespan"]).all() and (r["status"] == r0["status"]).all()
+    if peak:
+        assert (r["peak_mem"] == r0["peak_mem"]).all()
     og = O.OracleGraph(desc)
     for k in range(0, len(cands), oracle_every):
         o = og.schedule(cands[k], flags=flags, outputs=False)
         assert int(r["makespan"][k]) == o["makespan"] and int(r["status"][k]) == o["status"], (desc.name, k, flags)
+        if peak:
+            assert (r["peak_mem"][k] == o["peak_mem"]).all(), (desc.name, k, flags)
     return r
 
 
@@ -227,3 +231,73 @@ def test_pk_large_makespans():
     assert int(r["makespan"].max()) >= (1 << 29)
     g.schedule_batch(cands, flags=F.F_CP_PIN, peak=False)
     assert g.last_timing()["deferred"] >= int((r["makespan"] >= (1 << 29)).sum()) > 0
+
+
+# ------------------------------------------- memory on the lane kernel (MM)
+
+@pytest.mark.parametrize("G", [1, 2, 3, 5, 8, 13, 32])
+def test_lane_peak_memory(G):
+    """per-device peak memory (R8: the static total per device) requested
+    without caps: the lane kernel's MM 1 variant, against the group kernel
+    and the oracle, with and without prefix sharing"""
+    desc = topo_dag(5000 + G, V=150, G=G, K=1 + G % 2, homogeneous=bool(G % 2))
+    cands = pin_cands(desc, np.random.default_rng(G), 160)
+    for flags in (0, F.F_CP_PIN):
+        check(desc, cands, flags, peak=True)
+    gn = _graph_env(desc, FASTT_NO_SHARE="1")
+    r0 = gn.schedule_batch(cands, flags=F.F_CP_PIN, peak=True)
+    r1 = F.Graph(desc).schedule_batch(cands, flags=F.F_CP_PIN, peak=True)
+    assert (r0["peak_mem"] == r1["peak_mem"]).all() and (r0["makespan"] == r1["makespan"]).all()
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_lane_memory_caps(seed):
+    """finite per-device caps (Alg. 1 line 13, R8, R9: multi-round CP devices
+    with reservations, infeasible candidates): the lane kernel's MM 2 variant
+    on 32- and 64-bit time, one and several link classes"""
+    G = [2, 3, 4, 5, 8, 16][seed % 6]
+    desc = topo_dag(5100 + seed, V=130, G=G, K=1 + (seed % 3 == 2) * 2, caps="random",
+                    scale=(50_000_000 if seed % 4 == 3 else 1))
+    cands = pin_cands(desc, np.random.default_rng(seed), 192)
+    for flags in (0, F.F_CP_PIN):
+        r = check(desc, cands, flags, peak=True)
+        r2 = F.Graph(desc).schedule_batch(cands, flags=flags, peak=False)
+        assert (r2["makespan"] == r["makespan"]).all() and (r2["status"] == r["status"]).all()
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_lane_caps_tight_and_sweep(seed):
+    """caps just above the average load (many infeasible candidates, CP
+    rounds that span several devices), the sweep argmin and prefix sharing
+    (A/B against FASTT_NO_SHARE=1 and the group kernel)"""
+    d0 = topo_dag(5200 + seed, V=160, G=4 + seed % 5, K=1)
+    cap = np.full(d0.n_devices, int(d0.mem.sum() * (1.1 + 0.1 * (seed % 3)) / d0.n_devices), np.int64)
+    desc = dataclasses.replace(d0, cap=cap)
+    cands = pin_cands(desc, np.random.default_rng(seed), 200)
+    r = check(desc, cands, F.F_CP_PIN, peak=True)
+    gn = _graph_env(desc, FASTT_NO_SHARE="1")
+    r0 = gn.schedule_batch(cands, flags=F.F_CP_PIN, peak=True)
+    assert (r0["makespan"] == r["makespan"]).all() and (r0["peak_mem"] == r["peak_mem"]).all()
+    gen = F.gen_params(seed=seed)
+    gl, gg = F.Graph(desc), _graph_env(desc, FASTT_NO_LANE="1")
+    b1 = gl.sweep_best(gen, 0, 2500, flags=F.F_CP_PIN)
+    assert gl.last_timing()["topo"] == LANE
+    assert b1 == gg.sweep_best(gen, 0, 2500, flags=F.F_CP_PIN)
+
+
+def test_lane_memory_configs():
+    """C4 (VGG-19, caps, 64-bit time) and C5 (peak requested) stay on the
+    lane kernel; sampled against the oracle"""
+    for name, peak in (("C4", True), ("C5", True)):
+        desc = synth.config(name)
+        gl = F.Graph(desc)
+        gen = F.gen_params(seed=0xFA57, n_pow2_only=name == "C4")
+        ns = gl.stream_info(gen, flags=F.F_CP_PIN)
+        c = gl.generate_candidates(gen, ns + 1, 600, flags=F.F_CP_PIN)
+        r = gl.schedule_batch(c, flags=F.F_CP_PIN, peak=peak)
+        assert gl.last_timing()["topo"] == LANE, name
+        og = O.OracleGraph(desc)
+        for k in range(0, len(c), 50):
+            o = og.schedule(c[k], flags=F.F_CP_PIN, outputs=False)
+            assert (int(r["makespan"][k]), int(r["status"][k])) == (o["makespan"], o["status"]), (name, k)
+            assert (r["peak_mem"][k] == o["peak_mem"]).all(), (name, k)
