@@ -14,10 +14,12 @@ one NCCL all_reduce(MIN) pair picks the winner (weak scaling).
   e2e     the same metric through fastt_schedule_batch with HOST (pinned)
           candidate and result buffers, copies inside the timed region
   roofline  dominant kernel = the simulation kernel k_sim_lane (sweep launch),
-          bound "alu": algorithmic int32 ops V(8G+2) + 7E per candidate x
-          candidates of the launch / its CUDA-event duration, vs 148 SMs x
-          128 int32 lanes/clk x max SM clock; the touched-once
-          HBM figure (B_state + B_graph/32) rides along under roofline.hbm
+          bound "alu": algorithmic ALU-pipe ops per op-step (2.5G + 6E/V + 5)
+          x op-steps executed in the launch (device counter) / its CUDA-event
+          duration, vs the ALU pipe's lane-instruction rate measured in the
+          same run (tools/alu_peak.cu); the committed ncu capture's issue /
+          pipe / L1 / DRAM fractions ride along under roofline.ncu and the
+          touched-once HBM figure under roofline.hbm
   cpu_baseline  the plain C oracle on a bounded strided sample of the same
           stream, all host cores (one oracle call per candidate per thread)
 
@@ -61,29 +63,45 @@ def b_alg_lane(V, E, G):
     return 21 * V + 13 * E + (V * (8 * G + 24) + 16 * E) / 32.0
 
 
-def alu_ops_lane(V, E, G):
-    """Algorithmic int32 ALU operations of one candidate's DPOS evaluation on
-    the lane kernel's (exact, single-link-class) EST form (DESIGN.md section
-    5, "ALU roofline"): per predecessor edge 7 (arrival FT + c, running max,
-    argmax device, co-located select, E max), per op-step and device 8
-    (arrival select, max with avail, + cost, argmin compare + 2 selects,
-    avail update), + 2 per op-step (makespan max, record pack); V' = V op-steps
-    per PIN candidate, counted in full even where the BASE prefix is reused."""
-    return V * (8 * G + 2) + 7 * E
+def alu_ops_step(V, E, G):
+    """Algorithmic integer ALU-pipe instructions of one DPOS op-step on the
+    lane kernel's exact single-link-class EST form (DESIGN.md section 5,
+    "Roofline"), the minimal instruction count of the method per step: per
+    device 2.5 (key = max(avail, arrival) + cost; its share of a 3-input min
+    tree), per predecessor edge 6 (arrival FT + c, running max with argmax
+    device, co-located test, select, E max), 5 fixed (arrival on the argmax
+    device, makespan, avail update, record).  Executed op-steps are counted
+    on the device (fastt_timing.lane_steps: prefix-shared steps excluded)."""
+    return 2.5 * G + 6.0 * E / max(V, 1) + 5.0
 
 
-def alu_peak_tops():
-    """int32 lanes/s: 148 SMs x 4 SMSPs x (alu pipe + fma pipe, 16 lanes/clk
-    each: rt_SMSP = 2 cycles per warp instruction, B300_MICROARCH.md "Pipe
-    rates") x the max SM clock of MEASURED_PEAKS.json."""
+def alu_peak_measured():
+    """The integer ALU pipe's measured lane-instruction rate on this GPU
+    (tools/alu_peak.cu, run here, now): VIMNMX + LOP3 chains, 16 warps/SM."""
+    from paper_conf_middleware_0001lmwlwyl20_b200 import build as B
     try:
-        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
-            mhz = float(json.load(f)["sm_max_mhz"])
-        src = "derived: 148 SMs x 128 int32 lanes/clk (alu+fma pipes) x sm_max_mhz of MEASURED_PEAKS.json"
+        exe = B.build_alu_peak()
+        out = subprocess.run([exe], capture_output=True, text=True, timeout=120).stdout.strip().splitlines()[-1]
+        j = json.loads(out)
+        return float(j["alu_pipe_tops"]), "measured: tools/alu_peak.cu (VIMNMX+LOP3 chains, 16 warps/SM) in this run", j
+    except Exception as e:  # (fallback: the guide's unit counts and the max clock)
+        try:
+            with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+                mhz = float(json.load(f)["sm_max_mhz"])
+        except Exception:
+            mhz = 1965.0
+        return 148 * 4 * 16 * mhz * 1e6 / 1e12, "derived (microbenchmark failed: %s): 148 SMs x 64 ALU lanes/clk x %.0f MHz" % (
+            str(e)[:80], mhz), None
+
+
+def ncu_current():
+    """pipe / issue / DRAM fractions of the committed ncu capture of the main
+    sweep launch (profiles/ncu_k_sim_lane_current.json)"""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_k_sim_lane_current.json")) as f:
+            return json.load(f)
     except Exception:
-        mhz = 1965.0
-        src = "derived: 148 SMs x 128 int32 lanes/clk (alu+fma pipes) x 1965 MHz (fallback clock)"
-    return 148 * 4 * 2 * 16 * mhz * 1e6 / 1e12, src
+        return None
 
 
 def cpu_model():
@@ -278,6 +296,7 @@ def main():
     S = args.candidates
     st = torch.cuda.current_stream()
     n_split = g.stream_info(gen, flags=FLAGS_CP, stream=st)
+    apeak, apeak_src, apeak_json = alu_peak_measured() if rank == 0 else (None, None, None)
     flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device="cuda")  # > 126 MB L2
     best_dev = torch.zeros(2, dtype=torch.int64, device="cuda")
 
@@ -321,31 +340,30 @@ def main():
     value = world * S / (ms_step / 1000.0)
     best = tuple(int(x) for x in best_dev.cpu().tolist())
 
-    # roofline of the dominant kernel (k_sim, main sweep launch)
+    # roofline of the dominant kernel (k_sim_lane, the main sweep launch)
     V, E, G = g.V, int(desc.n_edges), desc.n_devices
     sim_ms = statistics.mean(x["ms_sim"] for x in tms)
     fast = statistics.mean(x["candidates"] - x["deferred"] for x in tms)
     prep_ms = statistics.mean(x["ms_prep"] for x in tms)
+    lane_steps = statistics.mean(x["lane_steps"] for x in tms)
+    warp_steps = statistics.mean(x["warp_steps"] for x in tms)
     lane = tms[-1].get("topo", 0) == 2
     bpc = b_alg_lane(V, E, G) if lane else b_alg(V, E, G)
     hbm_gbs = bpc * fast / (sim_ms / 1000.0) / 1e9
     peak, peak_src = peaks()
+    nc = ncu_current()
     traffic = None
-    try:
-        with open(os.path.join(ROOT, "profiles", "ncu_sim_traffic.json")) as f:
-            tj = json.load(f)
-        traffic = tj["dram_bytes_per_candidate"] * fast
-    except Exception:
-        traffic = None
+    if nc and nc.get("dram_bytes_per_candidate"):
+        traffic = nc["dram_bytes_per_candidate"] * fast
     if lane:
-        # ncu (profiles/r01d_ncu_k_sim_lane_full.json): alu pipe 80 % busy,
-        # DRAM 21 % of peak -> the kernel is bound by integer ALU issue
-        opc = alu_ops_lane(V, E, G)
-        achieved = opc * fast / (sim_ms / 1000.0) / 1e12
-        apeak, apeak_src = alu_peak_tops()
-        roof = {"bound": "alu", "achieved": achieved, "peak": apeak, "unit": "Tops/s (int32)",
-                "frac": achieved / apeak, "traffic": traffic, "peak_source": apeak_src,
-                "ops_per_candidate": opc,
+        ops = alu_ops_step(V, E, G)
+        achieved = ops * lane_steps / (sim_ms / 1000.0) / 1e12 if lane_steps else 0.0
+        roof = {"bound": "alu", "achieved": achieved, "peak": apeak, "unit": "T int32 ALU-pipe ops/s",
+                "frac": achieved / apeak if apeak else None, "traffic": traffic, "peak_source": apeak_src,
+                "alu_ops_per_op_step": ops, "op_steps_executed_per_launch": lane_steps,
+                "op_steps_per_candidate": lane_steps / fast if fast else None,
+                "warp_steps_per_launch": warp_steps, "alu_peak_run": apeak_json,
+                "ncu": nc,
                 "hbm": {"achieved_gbs_touched_once": hbm_gbs, "peak_gbs": peak, "peak_source": peak_src,
                         "bytes_per_candidate_touched_once": bpc,
                         "dram_gbs_ncu": (traffic / (sim_ms / 1000.0) / 1e9) if traffic else None}}

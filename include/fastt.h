@@ -241,7 +241,11 @@ typedef struct {
   int32_t topo;         /* 1 or 2: the main simulation ran a position-order kernel (the graph's priority
                            order is topological, so the dequeue order is the position order):
                            1 = one lane group per candidate (k_sim), 2 = one lane per candidate
-                           (k_sim_lane: makespan-only evaluation without memory tracking) */
+                           (k_sim_lane: makespan, per-device peak memory, memory caps) */
+  int32_t _pad;
+  int64_t warp_steps;   /* k_sim_lane main launch: op-steps executed per warp, summed (every lane of a
+                           warp executes the warp's steps; prefix-shared steps are not executed) */
+  int64_t lane_steps;   /* of which the steps of running candidates (each from its warp's start step) */
 } fastt_timing;
 fastt_status fastt_last_timing(const fastt_graph *g, fastt_timing *out);
 

@@ -51,6 +51,19 @@ def build(force: bool = False, verbose: bool = False, out: str = OUT) -> str:
     return out
 
 
+ALU_PEAK_SRC = os.path.join(ROOT, "tools", "alu_peak.cu")
+ALU_PEAK = os.path.join(HERE, "alu_peak")
+
+
+def build_alu_peak(force: bool = False) -> str:
+    """the int32 pipe microbenchmark bench.py runs for its roofline peak"""
+    if force or not os.path.exists(ALU_PEAK) or os.path.getmtime(ALU_PEAK) < os.path.getmtime(ALU_PEAK_SRC):
+        tmp = ALU_PEAK + ".tmp%d" % os.getpid()
+        subprocess.check_call([NVCC] + ARCH + ["-O3", "-o", tmp, ALU_PEAK_SRC])
+        os.replace(tmp, ALU_PEAK)
+    return ALU_PEAK
+
+
 if __name__ == "__main__":
     import sys
     print(build(force="-f" in sys.argv, verbose="-v" in sys.argv))

@@ -274,7 +274,7 @@ struct fastt_graph {
   int64_t gap_stride = 0;
   int ins_grid = 0;
   int64_t *wbest = nullptr, *best_dev = nullptr;
-  unsigned long long *counters = nullptr;  // [0] work counter, [1] deferred count
+  unsigned long long *counters = nullptr;  // [0] work counter, [1] deferred count, [2..3] k_sim_lane step counts
   int64_t *defer_q = nullptr;
   int64_t defer_cap = 0;
   // misc scratch
@@ -301,6 +301,7 @@ static fastt_status timing_begin(fastt_graph *g, uint32_t flags, cudaStream_t st
   g->launches = 0;
   memset(&g->last, 0, sizeof g->last);
   if (!(flags & FASTT_F_TIMING)) return FASTT_OK;
+  if (g->counters) CK(cudaMemsetAsync(g->counters + 2, 0, 2 * sizeof(unsigned long long), st));
   for (auto &e : g->ev)
     if (!e) CK(cudaEventCreate(&e));
   CK(cudaEventRecord(g->ev[0], st));
@@ -317,6 +318,12 @@ static fastt_status timing_end(fastt_graph *g, uint32_t flags, cudaStream_t st, 
   if (!(flags & FASTT_F_TIMING)) return FASTT_OK;
   CK(cudaEventRecord(g->ev[3], st));
   CK(cudaEventSynchronize(g->ev[3]));
+  if (g->counters) {
+    unsigned long long ws[2] = {0, 0};
+    CK(cudaMemcpy(ws, g->counters + 2, sizeof ws, cudaMemcpyDeviceToHost));
+    g->last.warp_steps = (int64_t)ws[0];
+    g->last.lane_steps = (int64_t)ws[1];
+  }
   float a = 0, b = 0, c = 0;
   CK(cudaEventElapsedTime(&a, g->ev[0], g->ev[1]));
   CK(cudaEventElapsedTime(&b, g->ev[1], g->ev[2]));
@@ -520,7 +527,8 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     g->ins_grid = (int)ig;
   }
   if (!g->counters) {
-    CK(cudaMalloc(&g->counters, 2 * sizeof(unsigned long long)));
+    CK(cudaMalloc(&g->counters, 4 * sizeof(unsigned long long)));
+    CK(cudaMemset(g->counters, 0, 4 * sizeof(unsigned long long)));
     CK(cudaMalloc(&g->best_dev, 2 * sizeof(int64_t)));
   }
   if (g->defer_cap < defer_need) {
@@ -575,6 +583,7 @@ static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
   a.split_mask = B.raw_block ? raw_struct(B.raw_block, B.rl, 0, 0, 0).split_mask : nullptr;
   a.counter = g->counters;
   a.ndefer = g->counters + 1;
+  a.stat = g->counters + 2;
   a.defer_q = g->defer_q;
   a.wbest = g->wbest;
   a.slab = g->slab;
@@ -730,6 +739,7 @@ static fastt_status ensure_sort_buf(fastt_graph *g, int64_t n) {
 // launches, each skipping the other kind of slot.
 static void launch_slots(fastt_graph *g, SimArgs b, int tbits, int nc, cudaStream_t st) {
   b.mode = 2;
+  b.stat = nullptr;  // (the step counts are the main launch's)
   const int per_block = (g->sim_block / 32) * g->sim_cpw;
   if (g->use_topo && b.lane) {
     // makespan-only evaluation without memory tracking: the multi-graph lane

@@ -153,17 +153,22 @@ __host__ __device__ inline int64_t part_bytes(int64_t b, int n, int k) { return 
 // base_rank (optional): rank_u of the base graph by uid; a SPLIT slot on all
 // devices then copies the ranks below the split op's height instead of
 // recomputing them (they have no path to the split op)
+// nact (all prep launchers, nullable): device count of the active slots; the
+// grid covers nslots, slots at or past *nact exit at once (a preparation
+// wave sized on the device, without a host round trip)
 void launch_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, const Cand *cands, int nslots,
-                 int G, cudaStream_t st, const uint64_t *base_rank = nullptr);
+                 int G, cudaStream_t st, const uint64_t *base_rank = nullptr, const uint32_t *nact = nullptr);
 void launch_heights(RawGraph *raw_dev, int32_t *scratch, int64_t vcap, cudaStream_t st);
-void launch_sort(PrepGraph *pgs, const RawGraph *raws, int nslots, int key_bits, int max_n, cudaStream_t st);
+void launch_sort(PrepGraph *pgs, const RawGraph *raws, int nslots, int key_bits, int max_n, cudaStream_t st,
+                 const uint32_t *nact = nullptr);
 void launch_cards(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, int nslots, int max_n, int G, int K,
-                  int tbits, cudaStream_t st, bool succ_all);
-void launch_cp(const RawGraph *raws, PrepGraph *pgs, int nslots, int G, int tbits, cudaStream_t st);
+                  int tbits, cudaStream_t st, bool succ_all, const uint32_t *nact = nullptr);
+void launch_cp(const RawGraph *raws, PrepGraph *pgs, int nslots, int G, int tbits, cudaStream_t st,
+               const uint32_t *nact = nullptr);
 void launch_copy_block(const void *src, void *dst, int64_t slot_stride_bytes, int64_t bytes, const Cand *cands,
-                       int nslots, cudaStream_t st);
+                       int nslots, cudaStream_t st, const uint32_t *nact = nullptr);
 void launch_patch_split(const RawGraph *base, RawGraph *raws, const GraphConst *gc, const Cand *cands, int nslots,
-                        cudaStream_t st);
+                        cudaStream_t st, const uint32_t *nact = nullptr);
 void launch_bound(const RawGraph *raw, const GraphConst *gc, int G, unsigned long long *out /* [2] */,
                   cudaStream_t st);
 void launch_splitlist(const RawGraph *raw, const GraphConst *gc, const uint8_t *place, int32_t *list,
@@ -238,6 +243,14 @@ struct SimArgs {
   // snapshot): used[d], and used[d] + reserved[d]
   void *snap_used;
   void *snap_ur;
+  // the list was classified by launch_t0_sort (deferred candidates sorted to
+  // its tail): the kernel skips its own rank-change test and processes the
+  // first *n_dev entries (n_dev nullable: a.n)
+  int32_t preclassified;
+  const uint32_t *n_dev;
+  // k_sim_lane instrumentation (nullable): [0] += steps per warp batch,
+  // [1] += steps of the batch's running lanes
+  unsigned long long *stat;
 };
 
 // one idle slot [a, b) of a device under INSERT
@@ -270,10 +283,22 @@ void launch_candgen_idx(const StreamState &s, int64_t first, int64_t stride, con
 void launch_slot_setup(const Cand *cands, const RawGraph *tmpl, const RawGraph *base, RawGraph *raws, int nslots,
                        cudaStream_t st);
 void launch_gather_cands(const Cand *src, const int64_t *idx, int64_t n, Cand *dst, int64_t *res, cudaStream_t st);
+// Bucket-sort the candidates by BASE-prefix start step.  With `classify`
+// (base PrepGraph pg, time bits tbits), candidates that need their own
+// prepared graph (cand_classify) go to one extra bucket at the tail and
+// *n_main receives the count of the others.
+struct T0Classify {
+  int on;
+  int tbits;
+  const PrepGraph *pg;
+  const GraphConst *gc;
+  const uint8_t *split_mask;
+  uint32_t *n_main;
+};
 void launch_t0_sort(int from_stream, const StreamState &S, int64_t first, int64_t stride, const Cand *list, int64_t n,
                     const uint32_t *pos, const uint32_t *snap_dq, int32_t nops, int32_t vraw, int G, Cand *tmp_c,
                     int64_t *tmp_i, uint32_t *key, uint32_t *hist, Cand *out_c, int64_t *out_i, int64_t *out_res,
-                    cudaStream_t st);
+                    cudaStream_t st, T0Classify cl = T0Classify{0, 0, nullptr, nullptr, nullptr, nullptr});
 void launch_gather_sorted(const Cand *src, const int64_t *sidx, const int64_t *sres, const int64_t *qs, int64_t n,
                           Cand *dst, int64_t *didx, int64_t *dres, cudaStream_t st);
 int sim_occupancy(int tbits, int gshift, int block, size_t smem, bool topo);

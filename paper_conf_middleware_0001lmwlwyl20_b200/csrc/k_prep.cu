@@ -27,9 +27,10 @@ __device__ __forceinline__ uint32_t warp_min_u32(uint32_t v) { return __reduce_m
 // ---------------------------------------------------------------- materialize
 
 // Bulk copy of the base raw block into every SPLIT slot (same layout, contiguous).
+// (nact: device count of active slots, nullable -- slots at or past it exit)
 __global__ void k_copy_block(const uint4 *src, uint4 *dst_base, int64_t slot_stride_words, int64_t words,
-                             const Cand *cands) {
-  if (cands[blockIdx.y].kind != 2) return;
+                             const Cand *cands, const uint32_t *nact) {
+  if ((nact && blockIdx.y >= *nact) || cands[blockIdx.y].kind != 2) return;
   uint4 *dst = dst_base + (int64_t)blockIdx.y * slot_stride_words;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += (int64_t)gridDim.x * blockDim.x)
     dst[i] = src[i];
@@ -56,8 +57,9 @@ __device__ void list_replace(int32_t *ids, int64_t *bytes, uint8_t *prm, uint32_
 __device__ __forceinline__ bool edge_cut(int dim, int p) { return dim == 0 ? !p : (bool)p; }
 
 // One CTA per slot: apply SplitOperation to the slot's copy of the base graph.
-__global__ void k_patch_split(const RawGraph *base_p, RawGraph *raws, const GraphConst *gc, const Cand *cands) {
-  if (cands[blockIdx.x].kind != 2) return;  // non-split slots alias the base graph: never write them
+__global__ void k_patch_split(const RawGraph *base_p, RawGraph *raws, const GraphConst *gc, const Cand *cands,
+                              const uint32_t *nact) {
+  if ((nact && blockIdx.x >= *nact) || cands[blockIdx.x].kind != 2) return;  // non-split slots alias the base graph: never write them
   const RawGraph &B = *base_p;
   RawGraph &R = raws[blockIdx.x];
   const Cand c = cands[blockIdx.x];
@@ -191,14 +193,14 @@ __global__ void k_patch_split(const RawGraph *base_p, RawGraph *raws, const Grap
 
 // host-visible entry points used by the ABI (declared in the .cpp)
 void launch_copy_block(const void *src, void *dst, int64_t slot_stride_bytes, int64_t bytes, const Cand *cands,
-                       int nslots, cudaStream_t st) {
+                       int nslots, cudaStream_t st, const uint32_t *nact) {
   int64_t words = (bytes + 15) / 16;
   dim3 grid((unsigned)((words + 255) / 256 > 1024 ? 1024 : (words + 255) / 256), (unsigned)nslots);
-  k_copy_block<<<grid, 256, 0, st>>>((const uint4 *)src, (uint4 *)dst, slot_stride_bytes / 16, words, cands);
+  k_copy_block<<<grid, 256, 0, st>>>((const uint4 *)src, (uint4 *)dst, slot_stride_bytes / 16, words, cands, nact);
 }
 void launch_patch_split(const RawGraph *base, RawGraph *raws, const GraphConst *gc, const Cand *cands, int nslots,
-                        cudaStream_t st) {
-  k_patch_split<<<nslots, 256, 0, st>>>(base, raws, gc, cands);
+                        cudaStream_t st, const uint32_t *nact) {
+  k_patch_split<<<nslots, 256, 0, st>>>(base, raws, gc, cands, nact);
 }
 
 // ----------------------------------------------------------------- ranks
@@ -274,10 +276,10 @@ __device__ __forceinline__ void rank_one(const RawGraph &R, const GraphConst &gc
 // independent, one lane each.  A split slot inserts its concat nodes before
 // level h(o), its sub-ops with level h(o) and its split nodes after it.
 __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gcp, const Cand *cands, int nslots,
-                       const uint64_t *base_rank) {
+                       const uint64_t *base_rank, const uint32_t *nact) {
   const int lane = threadIdx.x & 31;
   const int slot = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (slot >= nslots) return;
+  if (slot >= nslots || (nact && (uint32_t)slot >= *nact)) return;
   // by value: the rank stores cannot alias the descriptor, so its pointers
   // stay in registers instead of being re-loaded after every store
   const RawGraph R = raws[slot];
@@ -338,11 +340,11 @@ __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *g
 }
 
 void launch_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, const Cand *cands, int nslots, int G,
-                 cudaStream_t st, const uint64_t *base_rank) {
+                 cudaStream_t st, const uint64_t *base_rank, const uint32_t *nact) {
   (void)G;
   int warps_per_block = 4;
   int blocks = (nslots + warps_per_block - 1) / warps_per_block;
-  k_rank<<<blocks, warps_per_block * 32, 0, st>>>(raws, pgs, gc, cands, nslots, base_rank);
+  k_rank<<<blocks, warps_per_block * 32, 0, st>>>(raws, pgs, gc, cands, nslots, base_rank, nact);
 }
 
 __device__ uint32_t cta_exscan(uint32_t v, uint32_t *total, uint32_t *s_w);
@@ -486,7 +488,9 @@ __device__ uint64_t cta_exscan64(uint64_t v, uint64_t *total, uint64_t *s_w) {
 
 // One CTA per slot: order live ops by (rank desc, uid asc) with a stable LSD
 // radix sort of key = (2^key_bits - 1 - rank) over values initially in uid order.
-__global__ void __launch_bounds__(SORT_T) k_sort(PrepGraph *pgs, const RawGraph *raws, int key_bits) {
+__global__ void __launch_bounds__(SORT_T) k_sort(PrepGraph *pgs, const RawGraph *raws, int key_bits,
+                                                 const uint32_t *nact) {
+  if (nact && blockIdx.x >= *nact) return;
   PrepGraph &P = pgs[blockIdx.x];
   const RawGraph &R = raws[blockIdx.x];
   __shared__ uint32_t s_w[33];
@@ -577,15 +581,17 @@ __global__ void __launch_bounds__(SORT_T) k_sort(PrepGraph *pgs, const RawGraph 
   }
 }
 
-void launch_sort(PrepGraph *pgs, const RawGraph *raws, int nslots, int key_bits, int max_n, cudaStream_t st) {
+void launch_sort(PrepGraph *pgs, const RawGraph *raws, int nslots, int key_bits, int max_n, cudaStream_t st,
+                 const uint32_t *nact) {
   (void)max_n;
-  k_sort<<<nslots, SORT_T, 0, st>>>(pgs, raws, key_bits);
+  k_sort<<<nslots, SORT_T, 0, st>>>(pgs, raws, key_bits, nact);
 }
 
 // ----------------------------------------------------------------- cards
 
 // One CTA per slot: degree scans in position order + card headers.
-__global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, PrepGraph *pgs) {
+__global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, PrepGraph *pgs, const uint32_t *nact) {
+  if (nact && blockIdx.x >= *nact) return;
   const RawGraph R = raws[blockIdx.x];  // (by value: see k_rank)
   PrepGraph &P = pgs[blockIdx.x];
   __shared__ uint64_t s_w[33];
@@ -642,8 +648,9 @@ __global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, Prep
 // the inline predecessor entries of the card (words 8-15); clears P.topo on
 // an edge that does not go from a lower to a higher position.
 template <typename T>
-__global__ void k_cards_pred(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gcp) {
+__global__ void k_cards_pred(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gcp, const uint32_t *nact) {
   const int slot = blockIdx.y;
+  if (nact && (uint32_t)slot >= *nact) return;
   const RawGraph R = raws[slot];  // (by value: see k_rank)
   PrepGraph &P = pgs[slot];
   const GraphConst &gc = *gcp;
@@ -689,10 +696,11 @@ __global__ void k_cards_pred(const RawGraph *raws, PrepGraph *pgs, const GraphCo
 // One warp per position: successor edge arrays and inline successor entries
 // (words 16-31).  Only the ready-set simulator and the PIN classification
 // read them, so slots whose order is topological are skipped unless `all`.
-__global__ void k_cards_succ(const RawGraph *raws, PrepGraph *pgs, int all) {
+__global__ void k_cards_succ(const RawGraph *raws, PrepGraph *pgs, int all, const uint32_t *nact) {
   const int lane = threadIdx.x & 31;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int slot = blockIdx.y;
+  if (nact && (uint32_t)slot >= *nact) return;
   const RawGraph R = raws[slot];  // (by value: see k_rank)
   PrepGraph &P = pgs[slot];
   if (!all && P.topo) return;
@@ -718,19 +726,19 @@ __global__ void k_cards_succ(const RawGraph *raws, PrepGraph *pgs, int all) {
 }
 
 void launch_cards(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, int nslots, int max_n, int G, int K,
-                  int tbits, cudaStream_t st, bool succ_all) {
+                  int tbits, cudaStream_t st, bool succ_all, const uint32_t *nact) {
   (void)G; (void)K;
-  k_cards_hdr<<<nslots, SORT_T, 0, st>>>(raws, pgs);
+  k_cards_hdr<<<nslots, SORT_T, 0, st>>>(raws, pgs, nact);
   dim3 gp((unsigned)std::max(1, std::min((max_n + 255) / 256, 1024)), nslots);
-  if (tbits == 32) k_cards_pred<uint32_t><<<gp, 256, 0, st>>>(raws, pgs, gc);
-  else k_cards_pred<uint64_t><<<gp, 256, 0, st>>>(raws, pgs, gc);
+  if (tbits == 32) k_cards_pred<uint32_t><<<gp, 256, 0, st>>>(raws, pgs, gc, nact);
+  else k_cards_pred<uint64_t><<<gp, 256, 0, st>>>(raws, pgs, gc, nact);
   int blocks = (max_n * 32 + 255) / 256;
   if (blocks > 2048) blocks = 2048;
   // (only the rare non-topological slots do work unless succ_all: a full-width
   // grid per slot cost ~3.5 ms per 4k-slot wave in empty blocks alone)
   if (!succ_all && nslots > 1 && blocks > 32) blocks = 32;
   if (blocks < 1) blocks = 1;
-  k_cards_succ<<<dim3(blocks, nslots), 256, 0, st>>>(raws, pgs, succ_all ? 1 : 0);
+  k_cards_succ<<<dim3(blocks, nslots), 256, 0, st>>>(raws, pgs, succ_all ? 1 : 0, nact);
 }
 
 // -------------------------------------------------------------------- CP
@@ -739,10 +747,10 @@ void launch_cards(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, in
 // op, then repeatedly the successor of highest priority (= lowest position) --
 // and its prefix sums of memory and per-device cost (for R9).
 template <typename T>
-__global__ void k_cp(const RawGraph *raws, PrepGraph *pgs, int nslots, int G) {
+__global__ void k_cp(const RawGraph *raws, PrepGraph *pgs, int nslots, int G, const uint32_t *nact) {
   const int lane = threadIdx.x & 31;
   const int slot = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (slot >= nslots) return;
+  if (slot >= nslots || (nact && (uint32_t)slot >= *nact)) return;
   const RawGraph R = raws[slot];  // (by value: see k_rank)
   PrepGraph &P = pgs[slot];
   const int32_t n = P.n;
@@ -800,10 +808,11 @@ __global__ void k_cp(const RawGraph *raws, PrepGraph *pgs, int nslots, int G) {
   if (lane == 0) P.cp_len = len;
 }
 
-void launch_cp(const RawGraph *raws, PrepGraph *pgs, int nslots, int G, int tbits, cudaStream_t st) {
+void launch_cp(const RawGraph *raws, PrepGraph *pgs, int nslots, int G, int tbits, cudaStream_t st,
+               const uint32_t *nact) {
   int blocks = (nslots + 3) / 4;
-  if (tbits == 32) k_cp<uint32_t><<<blocks, 128, 0, st>>>(raws, pgs, nslots, G);
-  else k_cp<uint64_t><<<blocks, 128, 0, st>>>(raws, pgs, nslots, G);
+  if (tbits == 32) k_cp<uint32_t><<<blocks, 128, 0, st>>>(raws, pgs, nslots, G, nact);
+  else k_cp<uint64_t><<<blocks, 128, 0, st>>>(raws, pgs, nslots, G, nact);
 }
 
 // ----------------------------------------------------------------- bound

@@ -97,9 +97,10 @@ cudaError_t sim_set_smem(int tbits, int gshift, size_t smem) {
 // Key of a candidate for prefix sharing: the BASE dequeue step of its first
 // pinned op (n for BASE, 0 otherwise).  Candidates are bucket-sorted by it so
 // the lane groups of a warp start at similar steps.
+template <typename T>
 __global__ void k_t0_keys(int from_stream, StreamState S, int64_t first, int64_t stride, const Cand *list, int64_t n,
                           const uint32_t *pos, const uint32_t *snap_dq, int32_t nops, int32_t vraw, int G, Cand *out,
-                          int64_t *oidx, uint32_t *key) {
+                          int64_t *oidx, uint32_t *key, T0Classify cl, uint32_t defer_key) {
   for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x) {
     Cand c;
     int64_t ix;
@@ -124,6 +125,10 @@ __global__ void k_t0_keys(int from_stream, StreamState S, int64_t first, int64_t
         k = t < k ? t : k;
       }
     }
+    if (cl.on) {
+      uint8_t st;
+      if (cand_classify<T>(c, cl.pg, *cl.gc, cl.split_mask, G, true, st)) k = defer_key;
+    }
     out[q] = c;
     oidx[q] = ix;
     key[q] = k;
@@ -135,8 +140,9 @@ __global__ void k_bucket_hist(const uint32_t *key, int64_t n, int shift, uint32_
     atomicAdd(&hist[key[q] >> shift], 1u);
 }
 
-// exclusive scan of nb <= 1024 bucket counts, in place (one block of 1024)
-__global__ void k_bucket_scan(uint32_t *hist, int nb) {
+// exclusive scan of nb <= 1024 bucket counts, in place (one block of 1024);
+// nlast (nullable) receives the offset of bucket nb - 1
+__global__ void k_bucket_scan(uint32_t *hist, int nb, uint32_t *nlast) {
   __shared__ uint32_t sw[33];
   const int t = threadIdx.x, lane = t & 31, w = t >> 5;
   uint32_t v = t < nb ? hist[t] : 0, x = v;
@@ -156,6 +162,7 @@ __global__ void k_bucket_scan(uint32_t *hist, int nb) {
   }
   __syncthreads();
   if (t < nb) hist[t] = sw[w] + x - v;
+  if (nlast && t == nb - 1) *nlast = sw[w] + x - v;
 }
 
 __global__ void k_bucket_scatter(const uint32_t *key, const Cand *in, const int64_t *iidx, int64_t n, int shift,
@@ -174,17 +181,24 @@ __global__ void k_bucket_scatter(const uint32_t *key, const Cand *in, const int6
 void launch_t0_sort(int from_stream, const StreamState &S, int64_t first, int64_t stride, const Cand *list, int64_t n,
                     const uint32_t *pos, const uint32_t *snap_dq, int32_t nops, int32_t vraw, int G, Cand *tmp_c,
                     int64_t *tmp_i, uint32_t *key, uint32_t *hist, Cand *out_c, int64_t *out_i, int64_t *out_res,
-                    cudaStream_t st) {
+                    cudaStream_t st, T0Classify cl) {
   if (n <= 0) return;
   int shift = 0;
   while ((nops >> shift) >= 1023) shift++;
-  const int nb = (nops >> shift) + 1;
+  int nb = (nops >> shift) + 1;
+  // classified lists: one more bucket (index nb) at the tail for the deferred
+  const uint32_t defer_key = (uint32_t)nb << shift;
+  if (cl.on) nb++;
   const int blocks = (int)((n + 255) / 256 < 2048 ? (n + 255) / 256 : 2048);
-  k_t0_keys<<<blocks, 256, 0, st>>>(from_stream, S, first, stride, list, n, pos, snap_dq, nops, vraw, G, tmp_c, tmp_i,
-                                    key);
+  if (cl.tbits == 64)
+    k_t0_keys<uint64_t><<<blocks, 256, 0, st>>>(from_stream, S, first, stride, list, n, pos, snap_dq, nops, vraw, G,
+                                                tmp_c, tmp_i, key, cl, defer_key);
+  else
+    k_t0_keys<uint32_t><<<blocks, 256, 0, st>>>(from_stream, S, first, stride, list, n, pos, snap_dq, nops, vraw, G,
+                                                tmp_c, tmp_i, key, cl, defer_key);
   cudaMemsetAsync(hist, 0, sizeof(uint32_t) * 1024, st);
   k_bucket_hist<<<blocks, 256, 0, st>>>(key, n, shift, hist);
-  k_bucket_scan<<<1, 1024, 0, st>>>(hist, nb);
+  k_bucket_scan<<<1, 1024, 0, st>>>(hist, nb, cl.on ? cl.n_main : nullptr);
   k_bucket_scatter<<<blocks, 256, 0, st>>>(key, tmp_c, tmp_i, n, shift, nb, hist, out_c, out_i, out_res);
 }
 

@@ -206,13 +206,16 @@ __global__ void __launch_bounds__(SIM_BLOCK, TOPO ? SIM_MINB_TOPO : SIM_MINB) k_
   }
   __syncwarp();
 
+  // work items: a.n, or the device count of a list classified / gathered on
+  // the device (n_dev)
+  const int64_t nlim = a.n_dev ? ((int64_t)*a.n_dev < a.n ? (int64_t)*a.n_dev : a.n) : a.n;
   for (;;) {
     unsigned long long q0 = 0;
     if (lane == 0) q0 = atomicAdd(a.counter, (unsigned long long)CPW);
     q0 = __shfl_sync(FULL, q0, 0);
-    if ((int64_t)q0 >= a.n) break;
+    if ((int64_t)q0 >= nlim) break;
     const int64_t q = (int64_t)q0 + grp;
-    bool active = q < a.n;
+    bool active = q < nlim;
     Cand c;
     c.kind = 0; c.n_pins = 0; c.split_op = -1;
     const PrepGraph *pg = a.base;

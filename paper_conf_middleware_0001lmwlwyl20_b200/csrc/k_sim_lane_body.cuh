@@ -332,13 +332,16 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   const uint32_t all = all_devices(G);
   int64_t bms = I64MAX, bidx = -1;  // this lane's best (makespan, stream index) for the sweep argmin
 
+  // work items: a.n, or the device count of a list classified / gathered on
+  // the device (n_dev)
+  const int64_t nlim = a.n_dev ? ((int64_t)*a.n_dev < a.n ? (int64_t)*a.n_dev : a.n) : a.n;
   for (;;) {
     unsigned long long q0 = 0;
     if (lane == 0) q0 = atomicAdd(a.counter, 32ull);
     q0 = __shfl_sync(FULL, q0, 0);
-    if ((int64_t)q0 >= a.n) break;
+    if ((int64_t)q0 >= nlim) break;
     const int64_t q = (int64_t)q0 + lane;
-    bool active = q < a.n;
+    bool active = q < nlim;
     Cand c;
     c.kind = 0;
     c.n_pins = 0;
@@ -381,39 +384,11 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     uint8_t st = 0;
     bool defer = false;
     if (MG) {
-      np = (active && c.kind == 1) ? c.n_pins : 0;  // (validated by the main launch)
+      np = (active && c.kind == 1) ? c.n_pins : 0;  // (validated by the classification)
     } else if (active) {
-      if (c.dev_mask & ~all) st = 2;
-      else if (c.dev_mask && c.dev_mask != all) defer = true;  // device subset (R25): own ranks
-      if (st) {
-      } else if (c.kind == 0) {
-      } else if (c.kind == 1) {
-        np = c.n_pins;
-        if (np < 1 || np > MAXPINS) st = 2;
-        else {
-          const uint32_t dset = c.dev_mask ? c.dev_mask : all;
-          bool bad = false;
-          for (int k = 0; k < np; k++) {
-            const int32_t o = c.pin_op[k];
-            if (o < 0 || o >= Vraw || posm[o] == NONE || c.pin_dev[k] >= G || !((dset >> c.pin_dev[k]) & 1u))
-              bad = true;
-            for (int k2 = 0; k2 < k; k2++) bad |= c.pin_op[k2] == o;
-          }
-          if (bad) st = 2;
-        }
-      } else if (c.kind == 2) {
-        const int32_t o = c.split_op;
-        if (o < 0 || o >= Vraw || posm[o] == NONE || c.split_dim > 1 || !(a.split_mask[o] & (1u << c.split_dim)) ||
-            c.split_n < 2 || c.split_n > G)
-          st = 2;
-        else defer = true;
-      } else {
-        st = 2;
-      }
-    }
-    if (st) {
-      np = 0;
-      defer = false;
+      // (a pre-classified list holds no candidate that needs its own graph)
+      defer = cand_classify<T>(c, pg, gc, a.split_mask, G, !a.preclassified, st);
+      np = (st == 0 && c.kind == 1) ? c.n_pins : 0;
     }
     uint32_t pp[MAXPINS] = {NONE, NONE, NONE, NONE};
     uint32_t pdv = 0;
@@ -422,10 +397,6 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
         pp[k] = posm[c.pin_op[k]];
         pdv |= (uint32_t)c.pin_dev[k] << (8 * k);
       }
-    // pins that change w or c (R5) need the candidate's own ranks
-    if (!MG && active && !defer)
-      for (int k = 0; k < np && !defer; k++)
-        defer = pin_changes_ranks<T>(pg, gc, c, np, pp[k], c.pin_dev[k], G, K);
     if (active && defer) {
       const unsigned long long k = atomicAdd(a.ndefer, 1ull);
       a.defer_q[k] = q;
@@ -509,6 +480,13 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       nmax = y > nmax ? y : nmax;
     }
     if (MG) lo = 0;
+    if (a.stat) {  // executed op-steps (the roofline's work count)
+      const uint32_t ls = __reduce_add_sync(FULL, run ? (uint32_t)(n - lo) : 0u);
+      if (lane == 0 && nmax > lo) {
+        atomicAdd(a.stat, (unsigned long long)(nmax - lo));
+        atomicAdd(a.stat + 1, (unsigned long long)ls);
+      }
+    }
     T avail[GP];
     T ms = 0;
 #pragma unroll

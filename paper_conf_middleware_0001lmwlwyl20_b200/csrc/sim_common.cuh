@@ -208,4 +208,61 @@ static __device__ __noinline__ bool pin_changes_ranks(const PrepGraph *pg, const
   return changed;
 }
 
+// Validation and classification of a candidate on the base graph (SURVEY
+// 8(a) S2-S5): st = 2 for a bad specification (BADSPEC: pins out of range,
+// on dead ops, on devices outside the candidate's subset or repeated; a split
+// of an op or dim that is not splittable, n outside 2..G; an unknown kind),
+// else 0.  Returns true iff a valid candidate needs its own prepared graph
+// (the preparation pipeline): a SPLIT (SplitOperation, Alg. 2 lines 16-30),
+// a proper device subset (R25: ranks over the subset), or -- when rank_test
+// -- pins that change w or c under R5's allowed sets.  The single definition
+// used by the pre-classification pass and the lane kernel's prologue.
+template <typename T>
+__device__ __forceinline__ bool cand_classify(const Cand &c, const PrepGraph *pg, const GraphConst &gc,
+                                              const uint8_t *split_mask, int G, bool rank_test, uint8_t &st) {
+  const uint32_t all = all_devices(G);
+  const uint32_t *posm = pg->pos;
+  const int32_t Vraw = pg->V;
+  st = 0;
+  bool defer = false;
+  if (c.dev_mask & ~all) {
+    st = 2;
+    return false;
+  }
+  if (c.dev_mask && c.dev_mask != all) defer = true;  // device subset (R25): own ranks
+  if (c.kind == 0) {
+  } else if (c.kind == 1) {
+    const int np = c.n_pins;
+    if (np < 1 || np > MAXPINS) {
+      st = 2;
+      return false;
+    }
+    const uint32_t dset = c.dev_mask ? c.dev_mask : all;
+    for (int k = 0; k < np; k++) {
+      const int32_t o = c.pin_op[k];
+      bool bad = o < 0 || o >= Vraw || posm[o] == NONE || c.pin_dev[k] >= G || !((dset >> c.pin_dev[k]) & 1u);
+      for (int k2 = 0; k2 < k; k2++) bad |= c.pin_op[k2] == o;
+      if (bad) {
+        st = 2;
+        return false;
+      }
+    }
+    if (!defer && rank_test)
+      for (int k = 0; k < np && !defer; k++)
+        defer = pin_changes_ranks<T>(pg, gc, c, np, posm[c.pin_op[k]], c.pin_dev[k], G, gc.K);
+  } else if (c.kind == 2) {
+    const int32_t o = c.split_op;
+    if (o < 0 || o >= Vraw || posm[o] == NONE || c.split_dim > 1 || !(split_mask[o] & (1u << c.split_dim)) ||
+        c.split_n < 2 || c.split_n > G) {
+      st = 2;
+      return false;
+    }
+    defer = true;
+  } else {
+    st = 2;
+    return false;
+  }
+  return defer;
+}
+
 }  // namespace fastt

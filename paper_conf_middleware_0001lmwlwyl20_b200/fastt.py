@@ -59,7 +59,8 @@ class fastt_split_result(C.Structure):
 
 class fastt_timing(C.Structure):
     _fields_ = [("launches", C.c_int64), ("candidates", C.c_int64), ("deferred", C.c_int64),
-                ("ms_sim", C.c_float), ("ms_prep", C.c_float), ("ms_total", C.c_float), ("topo", C.c_int32)]
+                ("ms_sim", C.c_float), ("ms_prep", C.c_float), ("ms_total", C.c_float), ("topo", C.c_int32),
+                ("_pad", C.c_int32), ("warp_steps", C.c_int64), ("lane_steps", C.c_int64)]
 
 
 SYMBOLS = ["fastt_load_graph", "fastt_free_graph", "fastt_graph_info", "fastt_rank", "fastt_schedule_batch",
@@ -302,7 +303,7 @@ class Graph:
         _check(lib().fastt_last_timing(self.h, C.byref(t)))
         return {"launches": int(t.launches), "candidates": int(t.candidates), "deferred": int(t.deferred),
                 "ms_sim": float(t.ms_sim), "ms_prep": float(t.ms_prep), "ms_total": float(t.ms_total),
-                "topo": int(t.topo)}
+                "topo": int(t.topo), "warp_steps": int(t.warp_steps), "lane_steps": int(t.lane_steps)}
 
     def split_search(self, flags=0, n_pow2_only=False, stream=None, best_improvement=False):
         r = fastt_split_result()

@@ -10,6 +10,10 @@ KEYS = ['Kernel Name', 'Grid Size', 'Block Size', 'gpu__time_duration.sum', 'dra
         'dram__throughput.avg.pct_of_peak_sustained_elapsed', 'lts__throughput.avg.pct_of_peak_sustained_elapsed',
         'sm__cycles_elapsed.avg.per_second', 'launch__sm_count', 'local_load_bytes', 'smsp__sass_inst_executed_op_local_ld.sum']
 STALL = 'smsp__average_warps_issue_stalled_'
+# pipe utilisation and L1 wavefront columns (the roofline fractions bench.py reports)
+PATTERNS = ('inst_executed_pipe_alu', 'inst_executed_pipe_fma', 'inst_executed_pipe_lsu', 'inst_executed_pipe_uniform',
+            'pipe_alu_cycles_active', 'pipe_fma_cycles_active', 'pipe_lsu', 'l1tex__data_pipe_lsu_wavefronts',
+            'l1tex__lsu_writeback', 'dram__bytes.sum', 'issue_active', 'pipe_shared_cycles_active')
 def main(rep):
     out = subprocess.run(['ncu', '-i', rep, '--page', 'raw', '--csv'], capture_output=True, text=True).stdout
     r = list(csv.reader(out.splitlines()))
@@ -18,6 +22,7 @@ def main(rep):
     for row in r[2:]:
         d = dict(zip(h, row)); u = dict(zip(h, units))
         s = {k: (d.get(k), u.get(k)) for k in KEYS if k in d}
+        s.update({k: (d.get(k), u.get(k)) for k in h if any(p in k for p in PATTERNS) and d.get(k) not in ('', None)})
         st = {k[len(STALL):].replace('_per_issue_active.ratio', ''): d[k] for k in h if k.startswith(STALL) and k.endswith('_per_issue_active.ratio')}
         st = dict(sorted(((k, float(v)) for k, v in st.items() if v not in ('', None)), key=lambda x: -x[1])[:10])
         s['top_stalls_per_issue'] = st
