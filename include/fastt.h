@@ -271,6 +271,21 @@ fastt_status fastt_fit_comm(int32_t n_devices, int64_t n_samples, const uint8_t 
                             const int64_t *bytes, const int64_t *time_ns, int cuda_device, const fastt_opts *opts,
                             int64_t *alpha_ns, int64_t *beta_fs_per_byte, int64_t *count);
 
+/* Computation cost model ("The
+ * computation cost model provides the execution time of a (sub-)operation on
+ * a device, using the operation's name and device as the key"
+ * unknown costs are 0).  Sample k says op[k] ran on dev[k] for time_ns[k];
+ * cost_ns[o*G+d] = the mean of the (o, d) samples as the nearest integer ns
+ * (halves up), 0 where there is none -- the cost_ns table of
+ * fastt_graph_desc.  Envelope: 1 <= G <= 32, n_ops >= 1, n_samples < 2^24,
+ * op in [0, n_ops), dev < G, time in [0, 2^40) (EINVAL otherwise).  Runs on
+ * cuda_device (integer sums and counts per entry, order-independent, then
+ * one thread per entry); host memory unless FASTT_F_IN_DEVICE /
+ * FASTT_F_OUT_DEVICE. */
+fastt_status fastt_cost_table(int32_t n_ops, int32_t n_devices, int64_t n_samples, const int32_t *op,
+                              const uint8_t *dev, const int64_t *time_ns, int cuda_device, const fastt_opts *opts,
+                              int64_t *cost_ns);
+
 /* The link model of fastt_graph_desc from per-pair parameters (host only):
  * pairs with identical (alpha, beta) share a link class; classes are
  * numbered in row-major order of first appearance over the off-diagonal

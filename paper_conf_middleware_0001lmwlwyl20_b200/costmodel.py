@@ -7,21 +7,28 @@ operation's name and device as the key.  The communication cost model provides
 the tensor transfer time between adjacent operations assigned to two different
 devices, according to tensor size and device pair", with a linear
 regression per device pair.  The B200 analogue reads a Chrome
-trace as exported by ``torch.profiler`` (``prof.export_chrome_trace``):
+trace as exported by ``torch.profiler`` (``prof.export_chrome_trace``, the
+Kineto format; ``tests/golden/trace_b200_mlp2.json`` is a trimmed capture
+from a B200, ``tools/capture_trace.py``):
 
-* complete events (``"ph": "X"``) of category ``kernel`` / ``cpu_op`` /
-  ``gpu_op`` whose ``name`` is a graph op name give computation samples,
-  keyed by (name, ``args["device"]``); ``dur`` is in microseconds;
-* events of category ``gpu_memcpy`` with ``args["bytes"]``,
-  ``args["src_device"]`` and ``args["dst_device"]`` (or ``args["device"]``
-  as the source) give transfer samples.
+* computation samples: complete events (``"ph": "X"``) whose ``name`` is a
+  graph op name -- the GPU-side spans of ``record_function(op_name)``
+  (category ``gpu_user_annotation``, one per annotated op execution on the
+  device in ``args["device"]``), or ``kernel`` / ``cpu_op`` / ``gpu_op``
+  events named after graph ops; ``dur`` is in microseconds;
+* transfer samples: ``gpu_memcpy`` events with ``args["bytes"]``.  The
+  device pair comes from ``args["src_device"]`` / ``args["dst_device"]`` when
+  present (peer copies), else from the copy kind in the name: ``HtoD`` is
+  host -> ``args["device"]``, ``DtoH`` the reverse, with the host mapped to
+  device index ``host_device`` (transfers over the host link are skipped when
+  it is None); same-device copies are not transfers.
 
 ``cost_table`` averages the computation samples into the int64-ns table of
-``fastt_graph_desc`` (unknown entries are 0); ``fit_link_model``
-fits the transfer samples on the GPU (``fastt_fit_comm``, reading R26) and
-groups the pairs into link classes (``fastt_link_model``).  Everything here is
-argument marshalling around the C-ABI; the arithmetic of the fit runs in
-``k_fit.cu``.
+``fastt_graph_desc`` on the GPU (``fastt_cost_table``: unknown entries are 0,
+P:472-477); ``fit_link_model`` fits the transfer samples on the GPU
+(``fastt_fit_comm``, reading R26) and groups the pairs into link classes
+(``fastt_link_model``).  Everything here is trace parsing and argument
+marshalling around the C-ABI; the arithmetic runs in ``k_fit.cu``.
 """
 from __future__ import annotations
 
@@ -32,7 +39,7 @@ import numpy as np
 
 from . import fastt as F
 
-_COMPUTE_CATS = ("kernel", "cpu_op", "gpu_op", "operator")
+_COMPUTE_CATS = ("gpu_user_annotation", "kernel", "cpu_op", "gpu_op", "operator")
 
 
 def load_trace(path_or_obj):
@@ -65,41 +72,56 @@ def compute_samples(events, op_index):
     return out
 
 
-def comm_samples(events):
-    """(src device, dst device, bytes, ns) for every device-to-device copy."""
+def _copy_pair(e, host_device):
+    """(src, dst) devices of a gpu_memcpy event, None if not a transfer"""
+    a = e.get("args") or {}
+    if "src_device" in a and "dst_device" in a:
+        return int(a["src_device"]), int(a["dst_device"])
+    name = e.get("name", "")
+    dev = a.get("device")
+    if dev is None:
+        return None
+    if "HtoD" in name:
+        return (None if host_device is None else (int(host_device), int(dev)))
+    if "DtoH" in name:
+        return (None if host_device is None else (int(dev), int(host_device)))
+    if "dst_device" in a:
+        return int(dev), int(a["dst_device"])
+    return None  # DtoD / DtoH without a host index / memset: no device pair
+
+
+def comm_samples(events, host_device=None):
+    """(src device, dst device, bytes, ns) for every copy between two devices
+    (the host counts as device host_device when given)."""
     out = []
     for e in events:
-        if e.get("ph") != "X" or e.get("cat") != "gpu_memcpy":
+        if e.get("ph") != "X" or e.get("cat") != "gpu_memcpy" or "dur" not in e:
             continue
-        a = e.get("args") or {}
-        s = a.get("src_device", a.get("device"))
-        d = a.get("dst_device")
-        b = a.get("bytes")
-        if s is None or d is None or b is None or int(s) == int(d) or "dur" not in e:
+        b = (e.get("args") or {}).get("bytes")
+        pr = _copy_pair(e, host_device)
+        if pr is None or b is None or pr[0] == pr[1]:
             continue
-        out.append((int(s), int(d), int(b), _ns(e["dur"])))
+        out.append((pr[0], pr[1], int(b), _ns(e["dur"])))
     return out
 
 
-def cost_table(events, op_index, n_ops, n_devices):
+def cost_table(events, op_index, n_ops, n_devices, device=0):
     """cost_ns[op][device] = mean of the op's samples on the device (nearest
-    integer ns, halves up); 0 where no sample exists."""
-    acc = {}
-    for op, dev, t in compute_samples(events, op_index):
-        if 0 <= op < n_ops and 0 <= dev < n_devices:
-            s = acc.setdefault((op, dev), [0, 0])
-            s[0] += t
-            s[1] += 1
-    cost = np.zeros((n_ops, n_devices), np.int64)
-    for (op, dev), (tot, cnt) in acc.items():
-        cost[op, dev] = (2 * tot + cnt) // (2 * cnt)
-    return cost
+    integer ns, halves up); 0 where no sample exists.  The
+    averaging runs in the library (fastt_cost_table)."""
+    smp = [(op, dev, t) for op, dev, t in compute_samples(events, op_index) if 0 <= op < n_ops and 0 <= dev < n_devices]
+    if smp:
+        op, dv, t = (np.asarray(x) for x in zip(*smp))
+    else:
+        op = dv = t = np.zeros(0, np.int64)
+    return F.cost_table(n_ops, n_devices, op, dv, t, device=device)
 
 
-def fit_link_model(events, n_devices, device=0):
+def fit_link_model(events, n_devices, device=0, host_device=None):
     """Transfer samples -> per-pair fit on the GPU -> link classes.
-    Returns dict(link_class, alpha, beta, pair_alpha, pair_beta, count)."""
-    smp = comm_samples(events)
+    Returns dict(link_class, alpha, beta, pair_alpha, pair_beta, count).
+    With host_device, n_devices counts the host as one more device."""
+    smp = comm_samples(events, host_device)
     if smp:
         s, d, b, t = (np.asarray(x) for x in zip(*smp))
     else:

@@ -184,14 +184,15 @@ struct Base {
   int topo = 0;  // the prepared priority order is topological (k_sim's TOPO path)
   unsigned long long bound = 0, maxextra = 0;
   // packed device keys of the lane kernel (32-bit time, one link class)
-  uint32_t *costk = nullptr;
+  uint32_t *costk = nullptr;  // [n][G] cost << gshift | d, then commk [n][4] (inline comm << gshift)
+  uint32_t *commk = nullptr;
   uint32_t pk_lim = 0;
   // recorded BASE schedule for prefix sharing, per CP-pin flag value
   struct Snap {
     bool valid = false;
     int round_dev = -1;
-    char *buf = nullptr;  // dq | avail | ms | rec | rounds | used | used + reserved
-    uint32_t *dq = nullptr;
+    char *buf = nullptr;  // dq | avail | ms | rec | rounds | used | used + reserved | keys
+    uint32_t *dq = nullptr, *key = nullptr;  // key: the records as packed keys FT << gshift | place (PK)
     void *avail = nullptr, *ms = nullptr, *rec = nullptr, *used = nullptr, *ur = nullptr;
     int32_t *rounds = nullptr;
   } snap[2];
@@ -202,6 +203,7 @@ struct Base {
     cudaFree(pg_dev);
     cudaFree(costk);
     costk = nullptr;
+    commk = nullptr;
     pk_lim = 0;
     for (auto &x : snap) {
       cudaFree(x.buf);
@@ -255,7 +257,8 @@ struct fastt_graph {
   int sms = 148, sim_block = SIM_BLOCK, sim_grid = 0, sim_tbits = 0, sim_cpw = 1, sim_bm_stride = 0;
   int sim_grid_topo = 0;  // resident blocks of the TOPO variant (no shared-memory ready set)
   bool use_topo = true;   // FASTT_NO_TOPO=1 forces the ready-set path (A/B parity)
-  int sim_grid_lane[3] = {0, 0, 0};  // resident blocks of the lane-per-candidate kernel per memory mode
+  // resident blocks of the lane-per-candidate kernel per memory mode and packed keys
+  int sim_grid_lane[3][2] = {{0, 0}, {0, 0}, {0, 0}};
   // device staging buffers of fastt_schedule_batch (host candidates in,
   // makespan/status out), kept across calls and grown on demand
   struct IoBuf {
@@ -405,11 +408,13 @@ static fastt_status prepare_base(fastt_graph *g, Base &B, cudaStream_t st) {
   if (g->use_pk && B.tbits == 32 && g->K == 1 && B.n > 0) {
     int gsh = 0;
     while ((1 << gsh) < g->G) gsh++;
-    CK(cudaMalloc(&B.costk, sizeof(uint32_t) * (size_t)B.n * g->G));
+    const size_t nck = ((size_t)B.n * g->G + 3) & ~(size_t)3;  // (commk 16-B aligned)
+    CK(cudaMalloc(&B.costk, sizeof(uint32_t) * (nck + 4 * (size_t)B.n)));
+    B.commk = B.costk + nck;
     unsigned long long *d_m = nullptr, hm[2];
     CK(cudaMalloc(&d_m, 16));
     CK(cudaMemsetAsync(d_m, 0, 16, st));
-    launch_pack_costs(B.pg_dev, B.n, g->G, gsh, P.E, B.costk, d_m, st);
+    launch_pack_costs(B.pg_dev, B.n, g->G, gsh, P.E, B.costk, B.commk, d_m, st);
     CK(cudaGetLastError());
     CK(cudaMemcpyAsync(hm, d_m, 16, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -494,13 +499,16 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     if (per_sm < 1) return fail(FASTT_EUNSUP, "simulation kernel does not fit on an SM (smem %zu)", smem);
     g->sim_grid = g->sms * per_sm;
     g->sim_grid_topo = g->sms * std::max(1, sim_occupancy(B.tbits, gsh, g->sim_block, 0, true));
-    for (int mm = 0; mm < 3; mm++) g->sim_grid_lane[mm] = g->sms * std::max(1, lane_occupancy(B.tbits, gsh, mm));
+    for (int mm = 0; mm < 3; mm++)
+      for (int pk = 0; pk < 2; pk++)
+        g->sim_grid_lane[mm][pk] = g->sms * std::max(1, lane_occupancy(B.tbits, gsh, mm, pk != 0));
     g->sim_smem = smem;
     g->sim_cpw = cpw;
     g->sim_bm_stride = stride;
     int64_t nslot = (int64_t)std::max(g->sim_grid, g->sim_grid_topo) * (g->sim_block / 32) * cpw;
     for (int mm = 0; mm < 3; mm++)
-      nslot = std::max<int64_t>(nslot, (int64_t)g->sim_grid_lane[mm] * LANE_BLOCK);  // one column per lane
+      for (int pk = 0; pk < 2; pk++)
+        nslot = std::max<int64_t>(nslot, (int64_t)g->sim_grid_lane[mm][pk] * LANE_BLOCK);  // one column per lane
     size_t rec = B.tbits == 32 ? 8 : 16;
     CK(cudaMalloc(&g->slab, (size_t)nslot * ncap * rec));
     CK(cudaMalloc(&g->wbest, sizeof(int64_t) * 2 * nslot));
@@ -555,7 +563,9 @@ static void main_shape(fastt_graph *g, const Base &B, SimArgs &a, int &grid, siz
   a.lane_mm = a.cap_check ? 2 : (a.out.peak ? 1 : 0);
   if (lane) {
     a.topo = 1;
-    grid = g->sim_grid_lane[a.lane_mm];
+    // (the packed-key variant: 32-bit time, one link class, keys prepared)
+    const bool pk = B.tbits == 32 && g->K == 1 && a.costk != nullptr && a.pk_lim > 0;
+    grid = g->sim_grid_lane[a.lane_mm][pk ? 1 : 0];
     smem = 0;
   } else if (topo) {
     a.topo = 1;
@@ -569,7 +579,7 @@ static void main_shape(fastt_graph *g, const Base &B, SimArgs &a, int &grid, siz
 }
 static int max_slots(const fastt_graph *g) {
   int gl = 0;
-  for (int mm = 0; mm < 3; mm++) gl = std::max(gl, g->sim_grid_lane[mm]);
+  for (int mm = 0; mm < 3; mm++) gl = std::max(gl, std::max(g->sim_grid_lane[mm][0], g->sim_grid_lane[mm][1]));
   return std::max(std::max(g->sim_grid, g->sim_grid_topo) * (g->sim_block / 32) * g->sim_cpw, gl * (LANE_BLOCK / 32));
 }
 
@@ -598,6 +608,7 @@ static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
   a.need_mem = a.cap_check;
   a.fastcomm = B.tbits == 32 && g->K == 1;
   a.costk = B.costk;
+  a.commk = B.commk;
   a.pk_lim = B.pk_lim;
   if (flags & FASTT_F_MEM_LIVE) {
     a.live_mem = 1;
@@ -641,7 +652,8 @@ static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cud
   const size_t tb = B.tbits / 8, n = (size_t)B.pl.ncap;
   const size_t o_dq = 0, o_av = al16(4 * n), o_ms = o_av + al16(tb * (n + 1) * g->G),
                o_rec = o_ms + al16(tb * (n + 1)), o_rd = o_rec + al16((B.tbits == 32 ? 8 : 16) * n),
-               o_us = o_rd + 64, o_ur = o_us + al16(8 * (n + 1) * g->G), tot = o_ur + al16(8 * (n + 1) * g->G);
+               o_us = o_rd + 64, o_ur = o_us + al16(8 * (n + 1) * g->G), o_k = o_ur + al16(8 * (n + 1) * g->G),
+               tot = o_k + al16(4 * n);
   CK(cudaMalloc(&S.buf, tot));
   S.dq = (uint32_t *)(S.buf + o_dq);
   S.avail = S.buf + o_av;
@@ -650,6 +662,7 @@ static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cud
   S.rounds = (int32_t *)(S.buf + o_rd);
   S.used = S.buf + o_us;
   S.ur = S.buf + o_ur;
+  S.key = (uint32_t *)(S.buf + o_k);
   CK(cudaMemsetAsync(S.rounds, 0, 16, st));
   Cand c;
   memset(&c, 0, sizeof c);
@@ -696,6 +709,10 @@ static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cud
   cudaFree(d_ms);
   cudaFree(d_st);
   if (hst != FASTT_CAND_OK) return FASTT_OK;  // an infeasible BASE (caps): no sharing
+  if (B.tbits == 32) {
+    launch_snap_keys(S.rec, B.n, gshift_of(g->G), S.key, st);
+    CK(cudaGetLastError());
+  }
   S.round_dev = (rd[0] == 1 && rd[2] == 0 && rd[3] == B.cp_len) ? rd[1] : -1;
   S.valid = true;
   return FASTT_OK;
@@ -708,6 +725,7 @@ static void use_snapshot(const Base &B, uint32_t flags, SimArgs &a) {
   a.snap_mode = 2;
   a.snap_used = S.used;
   a.snap_ur = S.ur;
+  a.snap_key = S.key;
   a.snap_round_dev = S.round_dev;
   a.snap_dq = S.dq;
   a.snap_avail = S.avail;
@@ -1891,6 +1909,53 @@ fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, 
 }
 
 // ------------------------------------------------- comm-model fit (N4)
+
+fastt_status fastt_cost_table(int32_t V, int32_t G, int64_t n, const int32_t *op, const uint8_t *dev,
+                              const int64_t *tns, int cuda_device, const fastt_opts *opts, int64_t *cost) {
+  if (G < 1 || G > MAXG) return fail(FASTT_EINVAL, "n_devices must be in 1..%d", MAXG);
+  if (V < 1) return fail(FASTT_EINVAL, "n_ops must be >= 1");
+  if (n < 0 || n >= (1ll << 24)) return fail(FASTT_EINVAL, "n_samples must be in [0, 2^24)");
+  if (!cost || (n > 0 && (!op || !dev || !tns))) return fail(FASTT_EINVAL, "NULL argument");
+  const uint32_t flags = flags_of(opts);
+  cudaStream_t st = stream_of(opts);
+  Dev guard(cuda_device);
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cuda_device);
+  const bool in_dev = (flags & FASTT_F_IN_DEVICE) != 0, out_dev = (flags & FASTT_F_OUT_DEVICE) != 0;
+  const size_t ne = (size_t)V * G;
+  // one scratch block: [sum | count][err][cost][op][dev][time]
+  const size_t o_err = al16(16 * ne), o_c = o_err + 16, o_op = o_c + al16(8 * ne),
+               o_dv = o_op + (in_dev ? 0 : al16(4 * n)), o_t = o_dv + (in_dev ? 0 : al16(n)),
+               tot = o_t + (in_dev ? 0 : al16(8 * n)) + 16;
+  char *buf = nullptr;
+  CK(cudaMalloc(&buf, tot));
+  struct Free {
+    char *p;
+    ~Free() { cudaFree(p); }
+  } fr{buf};
+  const int32_t *d_op = op;
+  const uint8_t *d_dv = dev;
+  const int64_t *d_t = tns;
+  if (!in_dev && n > 0) {
+    CK(cudaMemcpyAsync(buf + o_op, op, 4 * n, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(buf + o_dv, dev, n, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(buf + o_t, tns, 8 * n, cudaMemcpyHostToDevice, st));
+    d_op = (const int32_t *)(buf + o_op);
+    d_dv = (const uint8_t *)(buf + o_dv);
+    d_t = (const int64_t *)(buf + o_t);
+  }
+  unsigned *d_err = (unsigned *)(buf + o_err);
+  CK(cudaMemsetAsync(d_err, 0, 4, st));
+  int64_t *d_cost = out_dev ? cost : (int64_t *)(buf + o_c);
+  launch_cost_table(V, G, n, d_op, d_dv, d_t, buf, d_err, d_cost, sms, st);
+  CK(cudaGetLastError());
+  unsigned herr = 0;
+  CK(cudaMemcpyAsync(&herr, d_err, 4, cudaMemcpyDeviceToHost, st));
+  if (!out_dev) CK(cudaMemcpyAsync(cost, d_cost, 8 * ne, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  if (herr) return fail(FASTT_EINVAL, "a sample is outside the envelope (op, device or time range)");
+  return FASTT_OK;
+}
 
 fastt_status fastt_fit_comm(int32_t G, int64_t n, const uint8_t *src, const uint8_t *dst, const int64_t *bytes,
                             const int64_t *tns, int cuda_device, const fastt_opts *opts, int64_t *alpha,

@@ -236,6 +236,7 @@ struct SimArgs {
   // (cost << gshift) | d of the base graph, and the makespan at or above
   // which a candidate is deferred (0 = packed keys off)
   const uint32_t *costk;
+  const uint32_t *commk;  // [n][4] inline predecessors' comm << gshift (PK, one class)
   uint32_t pk_lim;
   // memory mode of the lane kernel: 0 none, 1 per-device peak, 2 finite caps
   int32_t lane_mm;
@@ -243,6 +244,7 @@ struct SimArgs {
   // snapshot): used[d], and used[d] + reserved[d]
   void *snap_used;
   void *snap_ur;
+  const uint32_t *snap_key;  // [n] BASE records as packed keys (PK records)
   // the list was classified by launch_t0_sort (deferred candidates sorted to
   // its tail): the kernel skips its own rank-change test and processes the
   // first *n_dev entries (n_dev nullable: a.n)
@@ -303,14 +305,19 @@ void launch_gather_sorted(const Cand *src, const int64_t *sidx, const int64_t *s
                           Cand *dst, int64_t *didx, int64_t *dres, cudaStream_t st);
 int sim_occupancy(int tbits, int gshift, int block, size_t smem, bool topo);
 void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st);
-int lane_occupancy(int tbits, int gshift, int mm);
+int lane_occupancy(int tbits, int gshift, int mm, bool pk);
 // costk[p][d] = (cost[p][d] << gshift) | d over n positions; mx[0] = max
 // cost, mx[1] = max edge comm (one link class) of the prepared graph
 void launch_pack_costs(const PrepGraph *pg_dev, int32_t n, int G, int gshift, int64_t E, uint32_t *costk,
-                       unsigned long long *mx, cudaStream_t st);
+                       uint32_t *commk, unsigned long long *mx, cudaStream_t st);
+// BASE records (uint32 time: FT | place << 32) -> packed keys FT << gshift | place
+void launch_snap_keys(const void *rec, int32_t n, int gshift, uint32_t *key, cudaStream_t st);
 void launch_fit(int G, int64_t n, const uint8_t *src, const uint8_t *dst, const int64_t *bytes, const int64_t *tns,
                 void *sums, unsigned *err, int64_t *alpha, int64_t *beta, int64_t *count, int sms, cudaStream_t st);
 size_t fit_sums_bytes(int G);
+// computation cost table (N4): scratch = 16 * n_ops * G bytes
+void launch_cost_table(int32_t V, int G, int64_t n, const int32_t *op, const uint8_t *dev, const int64_t *tns,
+                       void *scratch, unsigned *err, int64_t *cost, int sms, cudaStream_t st);
 cudaError_t sim_set_smem(int tbits, int gshift, size_t smem);
 void launch_fill_i64(int64_t *p, int64_t n, int64_t v, cudaStream_t st);
 

@@ -20,6 +20,8 @@
 // time in [0, 2^40), fewer than 2^24 samples, so Sb, St < 2^64 and
 // Sbb, Sbt < 2^104; every intermediate of the solve fits 256 bits and both
 // results fit 64 bits.
+#include <algorithm>
+
 #include "fastt_internal.cuh"
 
 namespace fastt {
@@ -159,5 +161,43 @@ void launch_fit(int G, int64_t n, const uint8_t *src, const uint8_t *dst, const 
   k_fit_solve<<<(P + 127) / 128, 128, 0, st>>>(G, (const FitSums *)sums, alpha, beta, count);
 }
 size_t fit_sums_bytes(int G) { return sizeof(FitSums) * (size_t)G * G; }
+
+// ------------------------------------------------ computation cost table
+// "execution time of a (sub-)operation on a device, using the operation's
+// name and device as the key": per (op, device) entry the sum and
+// count of its samples (64-bit integer atomics: exact, order-independent),
+// then the mean rounded to the nearest ns, halves up: q + (2r >= cnt).
+__global__ void k_cost_sums(int32_t V, int G, int64_t n, const int32_t *op, const uint8_t *dev, const int64_t *tns,
+                            u64 *sum, u64 *cnt, unsigned *err) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t o = op[i];
+    const int d = dev[i];
+    const int64_t t = tns[i];
+    if (o < 0 || o >= V || d >= G || t < 0 || t >= (1ll << 40)) {
+      atomicOr(err, 1u);
+      continue;
+    }
+    const int64_t e = (int64_t)o * G + d;
+    atomicAdd(&sum[e], (u64)t);
+    atomicAdd(&cnt[e], 1ull);
+  }
+}
+__global__ void k_cost_final(int64_t ne, const u64 *sum, const u64 *cnt, int64_t *cost) {
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < ne; e += (int64_t)gridDim.x * blockDim.x) {
+    const u64 c = cnt[e], s = sum[e];
+    cost[e] = c ? (int64_t)(s / c + (2 * (s % c) >= c ? 1 : 0)) : 0;  // (unknown: 0)
+  }
+}
+void launch_cost_table(int32_t V, int G, int64_t n, const int32_t *op, const uint8_t *dev, const int64_t *tns,
+                       void *scratch, unsigned *err, int64_t *cost, int sms, cudaStream_t st) {
+  const int64_t ne = (int64_t)V * G;
+  u64 *sum = (u64 *)scratch, *cnt = sum + ne;
+  cudaMemsetAsync(scratch, 0, sizeof(u64) * 2 * ne, st);
+  if (n > 0) {
+    const int blocks = (int)std::min<int64_t>((n + 255) / 256, (int64_t)sms * 8);
+    k_cost_sums<<<blocks, 256, 0, st>>>(V, G, n, op, dev, tns, sum, cnt, err);
+  }
+  k_cost_final<<<(int)std::min<int64_t>((ne + 255) / 256, (int64_t)sms * 8), 256, 0, st>>>(ne, sum, cnt, cost);
+}
 
 }  // namespace fastt

@@ -59,31 +59,32 @@ static const void *lane_fn(int tbits, int gshift, int cm, bool exact, bool mg, b
 }
 #undef FASTT_LANE_CASE
 
-template <typename T, bool MG, int MM> static size_t lane_smem_t(int gshift) {
+template <typename T, bool MG, int MM, bool PK> static size_t lane_smem_t(int gshift) {
   switch (gshift) {
-    case 0: return lane_smem_per_warp<T, 1, MG, MM>();
-    case 1: return lane_smem_per_warp<T, 2, MG, MM>();
-    case 2: return lane_smem_per_warp<T, 4, MG, MM>();
-    case 3: return lane_smem_per_warp<T, 8, MG, MM>();
-    case 4: return lane_smem_per_warp<T, 16, MG, MM>();
-    default: return lane_smem_per_warp<T, 32, MG, MM>();
+    case 0: return lane_smem_per_warp<T, 1, MG, MM, PK>();
+    case 1: return lane_smem_per_warp<T, 2, MG, MM, PK>();
+    case 2: return lane_smem_per_warp<T, 4, MG, MM, PK>();
+    case 3: return lane_smem_per_warp<T, 8, MG, MM, PK>();
+    case 4: return lane_smem_per_warp<T, 16, MG, MM, PK>();
+    default: return lane_smem_per_warp<T, 32, MG, MM, PK>();
   }
 }
-template <bool MG> static size_t lane_smem_w(int tbits, int gshift, int mm) {
+template <bool MG, bool PK> static size_t lane_smem_w(int tbits, int gshift, int mm) {
   if (tbits == 32)
-    return mm == 0 ? lane_smem_t<uint32_t, MG, 0>(gshift)
-                   : mm == 1 ? lane_smem_t<uint32_t, MG, 1>(gshift) : lane_smem_t<uint32_t, MG, 2>(gshift);
-  return mm == 0 ? lane_smem_t<uint64_t, MG, 0>(gshift)
-                 : mm == 1 ? lane_smem_t<uint64_t, MG, 1>(gshift) : lane_smem_t<uint64_t, MG, 2>(gshift);
+    return mm == 0 ? lane_smem_t<uint32_t, MG, 0, PK>(gshift)
+                   : mm == 1 ? lane_smem_t<uint32_t, MG, 1, PK>(gshift) : lane_smem_t<uint32_t, MG, 2, PK>(gshift);
+  return mm == 0 ? lane_smem_t<uint64_t, MG, 0, false>(gshift)
+                 : mm == 1 ? lane_smem_t<uint64_t, MG, 1, false>(gshift) : lane_smem_t<uint64_t, MG, 2, false>(gshift);
 }
-// dynamic shared memory of a block: LANE_BLOCK threads, or one warp (MG)
-size_t lane_smem(int tbits, int gshift, bool mg, int mm) {
-  if (mg) return lane_smem_w<true>(tbits, gshift, mm);
-  return (LANE_BLOCK / 32) * lane_smem_w<false>(tbits, gshift, mm);
+// dynamic shared memory of a block: LANE_BLOCK threads, or one warp (MG);
+// pk: the packed-key variant (4-byte records)
+size_t lane_smem(int tbits, int gshift, bool mg, int mm, bool pk) {
+  if (mg) return lane_smem_w<true, false>(tbits, gshift, mm);
+  return (LANE_BLOCK / 32) * (pk ? lane_smem_w<false, true>(tbits, gshift, mm) : lane_smem_w<false, false>(tbits, gshift, mm));
 }
 
 __global__ void k_pack_costs(const PrepGraph *pgp, int32_t n, int G, int gshift, int64_t E, uint32_t *costk,
-                             unsigned long long *mx) {
+                             uint32_t *commk, unsigned long long *mx) {
   const PrepGraph &P = *pgp;
   const uint32_t *c = (const uint32_t *)P.costp;
   const uint32_t *pc = (const uint32_t *)P.pe_comm;
@@ -96,12 +97,26 @@ __global__ void k_pack_costs(const PrepGraph *pgp, int32_t n, int G, int gshift,
   }
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < E; i += (int64_t)gridDim.x * blockDim.x)
     mm = pc[i] > mm ? pc[i] : mm;
+  // the cards' inline comm values (words 12-15, 0 in unused slots), pre-shifted
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < 4 * (int64_t)n;
+       i += (int64_t)gridDim.x * blockDim.x)
+    commk[i] = P.card[(i >> 2) * CARD_WORDS + CW_PCOMM + (i & 3)] << gshift;
   atomicMax(mx, (unsigned long long)mc);
   atomicMax(mx + 1, (unsigned long long)mm);
 }
 void launch_pack_costs(const PrepGraph *pg_dev, int32_t n, int G, int gshift, int64_t E, uint32_t *costk,
-                       unsigned long long *mx, cudaStream_t st) {
-  k_pack_costs<<<148, 256, 0, st>>>(pg_dev, n, G, gshift, E, costk, mx);
+                       uint32_t *commk, unsigned long long *mx, cudaStream_t st) {
+  k_pack_costs<<<148, 256, 0, st>>>(pg_dev, n, G, gshift, E, costk, commk, mx);
+}
+
+__global__ void k_snap_keys(const unsigned long long *rec, int32_t n, int gshift, uint32_t *key) {
+  for (int32_t p = blockIdx.x * blockDim.x + threadIdx.x; p < n; p += gridDim.x * blockDim.x) {
+    const unsigned long long w = rec[p];
+    key[p] = ((uint32_t)w << gshift) | (uint32_t)(w >> 32);
+  }
+}
+void launch_snap_keys(const void *rec, int32_t n, int gshift, uint32_t *key, cudaStream_t st) {
+  if (n > 0) k_snap_keys<<<(n + 255) / 256, 256, 0, st>>>((const unsigned long long *)rec, n, gshift, key);
 }
 
 int lane_comm_mode(const SimArgs &a, int tbits) {
@@ -116,22 +131,23 @@ void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
   const int cm = lane_comm_mode(a, tbits);
   const bool pk = !mg && tbits == 32 && cm != 2 && a.costk != nullptr && a.pk_lim > 0;
   const void *f = lane_fn(tbits, a.gshift, cm, a.G == (1 << a.gshift), mg, pk, a.lane_mm);
-  const size_t sm = lane_smem(tbits, a.gshift, mg, a.lane_mm);
+  const size_t sm = lane_smem(tbits, a.gshift, mg, a.lane_mm, pk);
   if (mg) cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
   SimArgs aa = a;
   void *args[] = {&aa};
   cudaLaunchKernel(f, dim3(grid), dim3(mg ? 32 : LANE_BLOCK), args, sm, st);
 }
 
-// resident blocks per SM of the base-graph launch of memory mode mm (the
-// minimum over its comm / exactness / packed-key variants); sets their
+// resident blocks per SM of the base-graph launch of memory mode mm and
+// packed keys pk (the minimum over the comm / exactness variants); sets their
 // dynamic shared memory limit
-int lane_occupancy(int tbits, int gshift, int mm) {
+int lane_occupancy(int tbits, int gshift, int mm, bool pk) {
   int nb = 1 << 30, x = 0;
-  const size_t sm = lane_smem(tbits, gshift, false, mm);
-  for (int v = (tbits == 32 ? 0 : 2); v < (tbits == 32 ? 10 : 6); v++) {
-    const void *f = v < 6 ? lane_fn(tbits, gshift, v >> 1, v & 1, false, false, mm)
-                          : lane_fn(tbits, gshift, (v - 6) >> 1, v & 1, false, true, mm);
+  if (pk && tbits != 32) return 0;
+  const size_t sm = lane_smem(tbits, gshift, false, mm, pk);
+  for (int v = (tbits == 32 ? 0 : 2); v < (tbits == 32 ? 6 : 6); v++) {
+    if (pk && (v >> 1) == 2) continue;  // (packed keys need one link class)
+    const void *f = lane_fn(tbits, gshift, v >> 1, v & 1, false, pk, mm);
     cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, f, LANE_BLOCK, sm);
     nb = x < nb ? x : nb;

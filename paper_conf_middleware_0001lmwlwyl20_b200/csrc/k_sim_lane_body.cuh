@@ -33,20 +33,26 @@ template <typename T, int GP, int MM> __host__ __device__ constexpr int card_slo
 template <typename T, int GP, int MM> __host__ __device__ constexpr int mg_lane_stride() {
   return 2 * LaneDepth<T>::D * card_slot_bytes<T, GP, MM>() + 16;
 }
+// bytes of one slab record: FT | place (8 B for 32-bit time, 16 B else), or
+// under packed keys the key FT << GSH | place itself (4 B)
+template <typename T, bool PK> __host__ __device__ constexpr int lane_rec_bytes() {
+  return PK ? 4 : (sizeof(T) == 4 ? 8 : 16);
+}
 // offset of the memory-tracking area in a warp's shared memory
-template <typename T, int GP, bool MG, int MM> __host__ __device__ constexpr size_t lane_mm_off() {
-  return (size_t)LaneDepth<T>::D * 5 * 32 * (sizeof(T) == 4 ? 8 : 16) +
+template <typename T, int GP, bool MG, int MM, bool PK = false> __host__ __device__ constexpr size_t lane_mm_off() {
+  return (size_t)LaneDepth<T>::D * 5 * 32 * lane_rec_bytes<T, PK>() +
          (MG ? (size_t)32 * mg_lane_stride<T, GP, MM>() : (size_t)2 * LaneDepth<T>::D * card_slot_bytes<T, GP, MM>()) +
          (size_t)(MG ? 0 : 32 * GP * 4);
 }
-template <typename T, int GP, bool MG, int MM> __host__ __device__ constexpr size_t lane_smem_per_warp() {
+template <typename T, int GP, bool MG, int MM, bool PK = false>
+__host__ __device__ constexpr size_t lane_smem_per_warp() {
   // ring D x 32 + stage D x 4 x 32 records, then 2D staged cards (per lane
   // in the multi-graph variant), then (base-graph launches) the packed-key
   // avail rows [32 lanes][GP] of the PK variant, then the memory state:
   // MM 1 used[d] (int64 [GP][32]); MM 2 slack[d] = cap - used - reserved
   // (int64 [GP][32]), its clamped 32-bit copy (quads [GP/4][32][4]) and the
   // CP rounds ([GP][32] u32)
-  return lane_mm_off<T, GP, MG, MM>() + (MM >= 1 ? (size_t)32 * GP * 8 : 0) + (MM == 2 ? (size_t)32 * GP * 8 : 0);
+  return lane_mm_off<T, GP, MG, MM, PK>() + (MM >= 1 ? (size_t)32 * GP * 8 : 0) + (MM == 2 ? (size_t)32 * GP * 8 : 0);
 }
 
 template <int BYTES> __device__ __forceinline__ void cp_async(uint32_t saddr, const void *g);
@@ -262,7 +268,8 @@ __device__ __noinline__ int cp_rounds_lane(const PrepGraph *pg, const GraphConst
 //     draws on its reservation), no feasible device => INFEASIBLE.
 template <typename T, int GSH, int CM, bool EX, bool MG, bool PK, int MM>
 __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
-  typedef typename Slab<T>::W W;
+  // slab / ring / stage record: FT | place, or the packed key (PK)
+  typedef typename std::conditional<PK, uint32_t, typename Slab<T>::W>::type W;
   constexpr int GP = 1 << GSH;
   static_assert(!PK || (sizeof(T) == 4 && CM != 2 && !MG), "packed keys: 32-bit time, one link class, base graph");
   static_assert(CM != 0 || sizeof(T) == 4, "card comm values are uint32");
@@ -274,7 +281,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   // and stage[D][4][32] (inline predecessors' records prefetched by cp.async)
   constexpr int D = LaneDepth<T>::D, P = D - 1;
   extern __shared__ __align__(16) unsigned char lsm[];
-  unsigned char *const wsm = lsm + (threadIdx.x >> 5) * lane_smem_per_warp<T, GP, MG, MM>();
+  unsigned char *const wsm = lsm + (threadIdx.x >> 5) * lane_smem_per_warp<T, GP, MG, MM, PK>();
   W *const ring = (W *)wsm + lane;
   W *const stage = ring + D * 32;
   const uint32_t stage_sa = (uint32_t)__cvta_generic_to_shared(stage);
@@ -293,9 +300,9 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   // MM 2: s32 = min(slack, 2^32 - 1) as quads [d / 4][32 lanes][4] (one
   // 128-bit load per 4 devices), rnd[r * 32] = CP round r: raw CP index just
   // past the round | device << 24
-  int64_t *const mv = (int64_t *)(wsm + lane_mm_off<T, GP, MG, MM>()) + lane;
-  uint32_t *const s32b = (uint32_t *)(wsm + lane_mm_off<T, GP, MG, MM>() + (size_t)32 * GP * 8) + (GP >= 4 ? 4 * lane : lane);
-  uint32_t *const rnd = (uint32_t *)(wsm + lane_mm_off<T, GP, MG, MM>() + (size_t)32 * GP * 12) + lane;
+  int64_t *const mv = (int64_t *)(wsm + lane_mm_off<T, GP, MG, MM, PK>()) + lane;
+  uint32_t *const s32b = (uint32_t *)(wsm + lane_mm_off<T, GP, MG, MM, PK>() + (size_t)32 * GP * 8) + (GP >= 4 ? 4 * lane : lane);
+  uint32_t *const rnd = (uint32_t *)(wsm + lane_mm_off<T, GP, MG, MM, PK>() + (size_t)32 * GP * 12) + lane;
   auto s32_at = [&](uint32_t d) -> uint32_t & { return GP >= 4 ? s32b[(d >> 2) * 128 + (d & 3)] : s32b[d * 32]; };
   auto clamp32 = [](int64_t v) -> uint32_t { return v >= (int64_t)0xFFFFFFFFll ? 0xFFFFFFFFu : (uint32_t)v; };
   constexpr int CO = card_cost_off<T, MM>();
@@ -327,7 +334,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
   const uint32_t *pe_src = pg->pe_src;
   const uint32_t *posm = pg->pos;
   int32_t n = pg->n, Vraw = pg->V, cpl = pg->cp_len;
-  const W *__restrict__ snap = (const W *)a.snap_rec;
+  const W *__restrict__ snap = PK ? (const W *)a.snap_key : (const W *)a.snap_rec;
   const bool cp_on = (a.flags & 1u) != 0;
   const uint32_t all = all_devices(G);
   int64_t bms = I64MAX, bidx = -1;  // this lane's best (makespan, stream index) for the sweep argmin
@@ -534,9 +541,12 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     // this lane's source row of a card copy: base + u * stride (card words or
     // the cost row), one 64-bit multiply-add per copy instead of a select of
     // two address computations
-    const char *const cc_base =
-        cc_cost ? (const char *)costsrc + cc_src : (const char *)card + cc_src;
-    const uint32_t cc_stride = cc_cost ? (uint32_t)(G * sizeof(T)) : (uint32_t)(CARD_WORDS * 4);
+    // (PK: lane 2 copies the pre-shifted comm values comm << GSH of commk)
+    const bool cc_ck = PK && CM == 0 && lane == 2;
+    const char *const cc_base = cc_cost ? (const char *)costsrc + cc_src
+                                : cc_ck ? (const char *)a.commk
+                                        : (const char *)card + cc_src;
+    const uint32_t cc_stride = cc_cost ? (uint32_t)(G * sizeof(T)) : cc_ck ? 16u : (uint32_t)(CARD_WORDS * 4);
     auto copy_card = [&](int32_t u) {
       if (MG) {  // this lane's own card: header, predecessors, comm, cost row
         if (u < n) {
@@ -637,18 +647,52 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       cp_async_commit();
       T f[4];
       uint32_t p[4];
-#pragma unroll
-      for (int k = 0; k < 4; k++) {
-        T ft;
-        uint32_t pl;
-        Slab<T>::decode_clean(rw[k], ft, pl);
-        f[k] = (uint32_t)k < npred ? ft : (T)0;
-        p[k] = (uint32_t)k < npred ? pl : 0xFFu;
-      }
       T arrd[GP];  // CM 2: arrival per device
       T M = 0, E = 0;
       uint32_t pa = 0xFFu;
-      if (CM != 2) {
+      // PK: the arrival terms in key space.  A record is the key FT << GSH |
+      // place, so R_k = key_k + (c_k << GSH) orders by FT + c and carries the
+      // place of predecessor k in its low bits: Mkey = max R_k gives M << GSH
+      // and pa (any argmax is exact, see above); the co-located test is
+      // ((key_k ^ Mkey) & (GP - 1)) == 0.  Unused slots count as key 0.
+      uint32_t Mk = 0, Ek = 0, pqk = 0;
+      if constexpr (PK) {
+        constexpr uint32_t gmk = GP - 1;
+        const uint32_t hcw[4] = {hc.x, hc.y, hc.z, hc.w};  // (commk: already << GSH)
+        uint32_t rkm[4], R[4];
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+          const bool u = (uint32_t)k < npred;
+          rkm[k] = u ? (uint32_t)rw[k] : 0u;
+          const uint32_t ck = CM == 0 ? hcw[k] : (u ? (uint32_t)cm1[k] << GSH : 0u);
+          R[k] = rkm[k] + ck;
+        }
+        uint32_t Mkey = max(max(R[0], R[1]), max(R[2], R[3]));
+        if (npred > 4u)  // (warp-uniform)
+          for (uint32_t k = 4; k < npred; k++)
+            Mkey = max(Mkey, (uint32_t)rec_at(__ldg(pe_src + h0.y + k), t) + ((uint32_t)__ldg(pe_comm + h0.y + k) << GSH));
+        uint32_t Ekey = 0;
+#pragma unroll
+        for (int k = 0; k < 4; k++) Ekey = max(Ekey, ((rkm[k] ^ Mkey) & gmk) == 0u ? rkm[k] : R[k]);
+        if (npred > 4u)
+          for (uint32_t k = 4; k < npred; k++) {
+            const uint32_t rk = (uint32_t)rec_at(__ldg(pe_src + h0.y + k), t);
+            Ekey = max(Ekey, ((rk ^ Mkey) & gmk) == 0u ? rk : rk + ((uint32_t)__ldg(pe_comm + h0.y + k) << GSH));
+          }
+        Mk = Mkey & ~gmk;
+        Ek = Ekey & ~gmk;
+        pqk = Mkey & gmk;
+      } else {
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+          T ft;
+          uint32_t pl;
+          Slab<T>::decode_clean(rw[k], ft, pl);
+          f[k] = (uint32_t)k < npred ? ft : (T)0;
+          p[k] = (uint32_t)k < npred ? pl : 0xFFu;
+        }
+      }
+      if (!PK && CM != 2) {
         // M = max over preds of FT + c, pa = the device of a pred attaining it,
         // E = the arrival on pa (its co-located preds contribute FT only)
         T R[4];
@@ -695,7 +739,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
             E = v > E ? v : E;
           }
         }
-      } else {
+      } else if (!PK) {
         // (only live lanes: a waiting lane's records are not yet valid, and
         // here a placement indexes the link-class table)
 #pragma unroll
@@ -756,11 +800,10 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
         }
         return forced;
       };
-      if (PK) {
+      if constexpr (PK) {
         // keys (EFT << GSH) | d: EST = max(avail[d], arrival),
         // arrival M on every device but pa, E on pa (R6); min key = EFT
         // argmin with ties to the lowest device (Alg. 1 lines 12-19, R3)
-        const uint32_t Mk = (uint32_t)M << GSH, Ek = (uint32_t)E << GSH;
         uint32_t av[GP];
         if (GP >= 2) {
 #pragma unroll
@@ -772,7 +815,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
         } else {
           av[0] = avk[0];
         }
-        const uint32_t pq = pa & (uint32_t)(GP - 1);
+        const uint32_t pq = pqk;
         const uint32_t ap = avk_at(pq), cpa = ((const uint32_t *)(cs + CO))[pq];
         uint32_t kpa = (ap > Ek ? ap : Ek) + cpa;
         if (!EX && pq >= (uint32_t)G) kpa = 0xFFFFFFFFu;
@@ -841,10 +884,9 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
           avk_at(bk & (uint32_t)(GP - 1)) = bkc;
           const T best = (T)(bkc >> GSH);
           ms = best > ms ? best : ms;
-          W w;
-          Slab<T>::make(w, best, bk & (uint32_t)(GP - 1));
-          col[(size_t)t * 32] = w;
-          ring[(t & (D - 1)) * 32] = w;
+          // the record is the key itself: FT << GSH | device
+          col[(size_t)t * 32] = bk;
+          ring[(t & (D - 1)) * 32] = bk;
         }
       } else {
       // EFT per device; argmin with ties to the lowest device

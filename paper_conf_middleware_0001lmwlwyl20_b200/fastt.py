@@ -66,7 +66,7 @@ class fastt_timing(C.Structure):
 SYMBOLS = ["fastt_load_graph", "fastt_free_graph", "fastt_graph_info", "fastt_rank", "fastt_schedule_batch",
            "fastt_stream_info", "fastt_generate_candidates", "fastt_sweep_best", "fastt_split_search",
            "fastt_free_split_result", "fastt_last_timing", "fastt_last_error", "fastt_version",
-           "fastt_fit_comm", "fastt_link_model"]
+           "fastt_fit_comm", "fastt_link_model", "fastt_cost_table"]
 F_TIMING = 16
 F_SPLIT_BEST = 32
 F_MEM_LIVE = 64
@@ -109,6 +109,8 @@ def lib():
     L.fastt_fit_comm.argtypes = [i32, i64, P, P, P, P, C.c_int, C.POINTER(fastt_opts), P, P, P]
     L.fastt_link_model.restype = i32
     L.fastt_link_model.argtypes = [i32, P, P, P, P, P, P]
+    L.fastt_cost_table.restype = i32
+    L.fastt_cost_table.argtypes = [i32, i32, i64, P, P, P, C.c_int, C.POINTER(fastt_opts), P]
     _lib = L
     return L
 
@@ -341,6 +343,22 @@ def fit_comm(n_devices, src, dst, nbytes, time_ns, device=0, stream=None):
     _check(lib().fastt_fit_comm(G, n, _ptr(src), _ptr(dst), _ptr(nb), _ptr(tn), int(device), C.byref(o), _ptr(a),
                                 _ptr(b), _ptr(c)))
     return a.reshape(G, G), b.reshape(G, G), c.reshape(G, G)
+
+
+def cost_table(n_ops, n_devices, op, dev, time_ns, device=0, stream=None):
+    """fastt_cost_table: per (op, device) the mean sample time, nearest ns
+    (halves up), 0 where no sample exists."""
+    V, G = int(n_ops), int(n_devices)
+    op = np.ascontiguousarray(np.asarray(op, np.int32))
+    dv = np.ascontiguousarray(np.asarray(dev, np.uint8))
+    tn = np.ascontiguousarray(np.asarray(time_ns, np.int64))
+    n = len(op)
+    if not (len(dv) == len(tn) == n):
+        raise ValueError("sample arrays differ in length")
+    out = np.zeros(V * G, np.int64)
+    o = _opts(0, stream)
+    _check(lib().fastt_cost_table(V, G, n, _ptr(op), _ptr(dv), _ptr(tn), int(device), C.byref(o), _ptr(out)))
+    return out.reshape(V, G)
 
 
 def link_model(alpha_ns, beta_fs):

@@ -106,3 +106,64 @@ def test_fitted_model_schedules_like_the_oracle():
         r = og.schedule(cand, flags=O.F_CP_PIN)
         assert int(res["makespan"][k]) == r["makespan"]
         assert (res["placement"][k] == r["placement"]).all() and (res["start"][k] == r["start"]).all()
+
+
+# ------------------------------------------------ computation cost table (N4)
+
+@pytest.mark.parametrize("seed", range(6))
+def test_cost_table_matches_oracle(seed):
+    """fastt_cost_table (GPU integer sums) equals the exact-rational mean of
+    every (op, device) group, halves up; groups without a sample are 0"""
+    rng = np.random.default_rng(seed)
+    V, G = int(rng.integers(1, 300)), int(rng.integers(1, 33))
+    n = int(rng.integers(0, 20_000))
+    op = rng.integers(0, V, n)
+    dv = rng.integers(0, G, n)
+    t = rng.integers(0, 1 << (10 + 5 * (seed % 7)), n)
+    if seed == 5:
+        t[:] = (1 << 40) - 1  # the envelope's edge: sums near 2^64
+    got = F.cost_table(V, G, op, dv, t)
+    assert got.tolist() == CF.cost_table(V, G, zip(op, dv, t))
+
+
+def test_cost_table_rounding_and_envelope():
+    got = F.cost_table(2, 2, [0, 0, 1], [1, 1, 0], [1, 2, 7])  # mean 1.5 -> 2
+    assert got.tolist() == [[0, 2], [7, 0]]
+    for bad in (([2], [0], [1]), ([0], [2], [1]), ([0], [0], [-1]), ([0], [0], [1 << 40]), ([-1], [0], [1])):
+        with pytest.raises(F.FasttError) as e:
+            F.cost_table(2, 2, *bad)
+        assert e.value.code == F.EINVAL
+
+
+def test_trace_cost_table_hand_trace():
+    import json
+    from test_costmodel import trace as hand_trace
+    ev = CM.load_trace(json.dumps(hand_trace()))
+    cost = CM.cost_table(ev, {"matmul": 0, "relu": 1, "softmax": 2}, 3, 2)
+    # mean 11250 ns on device 0; 1.5 ns rounds half up to 2; unknown entries 0 (P:472-477)
+    assert cost.tolist() == [[11250, 11000], [0, 2], [0, 0]]
+
+
+def test_committed_b200_trace_to_cost_model():
+    """the trimmed torch.profiler capture from a B200: GPU cost table and host
+    link fit equal the oracle's exact computations on the same samples"""
+    import json
+    import os
+    path = os.path.join(os.path.dirname(__file__), "golden", "trace_b200_mlp2.json")
+    if not os.path.exists(path):
+        pytest.skip("trace not captured yet")
+    obj = json.load(open(path))
+    ev = CM.load_trace(obj)
+    names = obj["fastt_op_names"]
+    idx = {n: i for i, n in enumerate(names)}
+    cost = CM.cost_table(ev, idx, len(names), 1)
+    assert cost.tolist() == CF.cost_table(len(names), 1, CM.compute_samples(ev, idx))
+    assert (cost[:, 0] > 0).all()
+    m = CM.fit_link_model(ev, 2, host_device=1)
+    smp = CM.comm_samples(ev, host_device=1)
+    for s, d in ((0, 1), (1, 0)):
+        grp = [(b, t) for s_, d_, b, t in smp if (s_, d_) == (s, d)]
+        a_q, b_q = CF.nnls_line([b for b, _ in grp], [t for _, t in grp])
+        a_ref, b_ref = CF.round_half_up(a_q), CF.round_half_up(b_q * 10**6)
+        assert (int(m["pair_alpha"][s][d]), int(m["pair_beta"][s][d])) == (a_ref, b_ref)
+        assert b_ref > 0  # bytes cost time over the host link
