@@ -58,6 +58,17 @@ def _ns(dur_us):
     return int((q.numerator * 2 + q.denominator) // (2 * q.denominator))
 
 
+def _device(e):
+    """the device of an event: args.device, else (device-side Kineto events,
+    whose pid is the GPU index) pid"""
+    a = e.get("args") or {}
+    if a.get("device") is not None:
+        return a["device"]
+    if str(e.get("cat", "")).startswith("gpu_") or e.get("cat") == "kernel":
+        return e.get("pid")
+    return None
+
+
 def compute_samples(events, op_index):
     """(op id, device, ns) for every compute event whose name is a graph op."""
     out = []
@@ -65,7 +76,7 @@ def compute_samples(events, op_index):
         if e.get("ph") != "X" or e.get("cat") not in _COMPUTE_CATS:
             continue
         op = op_index.get(e.get("name"))
-        dev = (e.get("args") or {}).get("device")
+        dev = _device(e)
         if op is None or dev is None or "dur" not in e:
             continue
         out.append((int(op), int(dev), _ns(e["dur"])))
@@ -78,7 +89,7 @@ def _copy_pair(e, host_device):
     if "src_device" in a and "dst_device" in a:
         return int(a["src_device"]), int(a["dst_device"])
     name = e.get("name", "")
-    dev = a.get("device")
+    dev = _device(e)
     if dev is None:
         return None
     if "HtoD" in name:

@@ -4,10 +4,11 @@ the C1 MLP training graph's ops (synth.config("C1")) are executed as torch
 CUDA ops, each under record_function("<op id>:<op type>") so the trace
 carries one GPU-side span per op execution, plus host<->device copies of
 several sizes (the only device pair one GPU has).  The trace is trimmed to
-the events the cost model reads and written to tests/golden/trace_b200_mlp2.json
-(or argv[1]); the untrimmed export goes to gpurun_out/.
+the events the cost model reads and written to tests/golden/trace_b200_mlp2.json;
+the untrimmed export goes to gpurun_out/.
 
-usage (on the box): python tools/capture_trace.py [out.json]
+usage (on the box): python tools/capture_trace.py
+       (here)         python tools/capture_trace.py --trim gpurun_out/trace_b200_mlp2_full.json "<gpu, torch>"
 """
 import json
 import os
@@ -20,7 +21,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 from paper_conf_middleware_0001lmwlwyl20_b200 import synth  # noqa: E402
 
-OUT = sys.argv[1] if len(sys.argv) > 1 else os.path.join(ROOT, "tests", "golden", "trace_b200_mlp2.json")
+OUT = os.path.join(ROOT, "tests", "golden", "trace_b200_mlp2.json")
 
 
 def main():
@@ -60,6 +61,13 @@ def main():
     os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
     full = os.path.join(ROOT, "gpurun_out", "trace_b200_mlp2_full.json")
     prof.export_chrome_trace(full)
+    trim(full, names, OUT, "%s, torch %s" % (torch.cuda.get_device_name(0), torch.__version__))
+
+
+def trim(full, names, out, where):
+    """keep the events the cost model reads: the GPU-side record_function
+    spans of the graph ops and the memcpy events (Kineto puts the GPU index
+    of device-side events in pid; args.device where it exists)"""
     tr = json.load(open(full))
     keep = []
     cats = {}
@@ -70,19 +78,23 @@ def main():
         c = e.get("cat")
         a = e.get("args") or {}
         if c == "gpu_user_annotation" and e.get("name") in names:
-            keep.append({"ph": "X", "cat": c, "name": e["name"], "ts": e.get("ts"), "dur": e["dur"],
-                         "args": {"device": a.get("device")}})
+            keep.append({"ph": "X", "cat": c, "name": e["name"], "pid": e.get("pid"), "ts": e.get("ts"), "dur": e["dur"],
+                         "args": {k: a[k] for k in ("device",) if k in a}})
         elif c == "gpu_memcpy":
-            keep.append({"ph": "X", "cat": c, "name": e["name"], "ts": e.get("ts"), "dur": e["dur"],
+            keep.append({"ph": "X", "cat": c, "name": e["name"], "pid": e.get("pid"), "ts": e.get("ts"), "dur": e["dur"],
                          "args": {k: a[k] for k in ("device", "bytes", "src_device", "dst_device") if k in a}})
-    res = {"fastt_note": "torch.profiler (Kineto) trace captured by tools/capture_trace.py on %s, torch %s; "
-                         "trimmed to gpu_user_annotation spans of the C1 ops and gpu_memcpy events"
-                         % (torch.cuda.get_device_name(0), torch.__version__),
+    res = {"fastt_note": "torch.profiler (Kineto) trace captured by tools/capture_trace.py on %s; trimmed to the "
+                         "gpu_user_annotation spans of the C1 ops and the gpu_memcpy events" % where,
            "fastt_op_names": names, "fastt_event_categories": cats, "traceEvents": keep}
-    with open(OUT, "w") as f:
+    with open(out, "w") as f:
         json.dump(res, f, indent=0)
     print("kept %d of %d events; categories %s" % (len(keep), sum(cats.values()), cats))
 
 
 if __name__ == "__main__":
-    main()
+    if len(sys.argv) > 2 and sys.argv[1] == "--trim":  # re-trim an untrimmed export: --trim full.json [where]
+        d = synth.config("C1")
+        trim(sys.argv[2], ["%d:%s" % (i, d.op_type[i]) for i in range(d.n_ops)], OUT,
+             sys.argv[3] if len(sys.argv) > 3 else "NVIDIA B200")
+    else:
+        main()
