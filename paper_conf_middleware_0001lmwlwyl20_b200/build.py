@@ -15,14 +15,15 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 _C = os.path.join(HERE, "csrc")
 SRCS = [os.path.join(_C, f) for f in ("fastt_abi.cu", "k_prep.cu", "k_sim.cu", "k_sim_lane.cu", "k_fit.cu",
-                                      "k_sim_inst.cu", "k_sim_lane_inst.cu")]
+                                      "k_sim_inst.cu", "k_sim_lane_inst.cu", "k_lane_pk_inst.cu")]
 # (source, extra flags): one object per unit
 UNITS = ([(os.path.join(_C, "k_sim_lane_inst.cu"), ["-DFASTT_GSH=%d" % g, "-DFASTT_MM=%d" % m])
           for g in (5, 4, 3, 2, 1, 0) for m in range(3)] +
          [(os.path.join(_C, "k_sim_inst.cu"), ["-DFASTT_GSH=%d" % g]) for g in (5, 4, 3, 2, 1, 0)] +
+         [(os.path.join(_C, "k_lane_pk_inst.cu"), ["-DFASTT_GSH=%d" % g]) for g in (5, 4, 3, 2, 1, 0)] +
          [(s, []) for s in SRCS[:5]])
 DEPS = SRCS + [os.path.join(_C, f) for f in ("fastt_internal.cuh", "sim_common.cuh", "k_sim_body.cuh",
-                                             "k_sim_lane_body.cuh")] + [os.path.join(ROOT, "include", "fastt.h")]
+                                             "k_sim_lane_body.cuh", "k_lane_pk.cuh")] + [os.path.join(ROOT, "include", "fastt.h")]
 OUT = os.path.join(HERE, "libfastt.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

@@ -186,6 +186,7 @@ struct Base {
   // packed device keys of the lane kernel (32-bit time, one link class)
   uint32_t *costk = nullptr;  // [n][G] cost << gshift | d, then commk [n][4] (inline comm << gshift)
   uint32_t *commk = nullptr;
+  uint32_t *pkc = nullptr;  // compact PK cards of k_lane_pk (same allocation)
   uint32_t pk_lim = 0;
   // recorded BASE schedule for prefix sharing, per CP-pin flag value
   struct Snap {
@@ -204,6 +205,7 @@ struct Base {
     cudaFree(costk);
     costk = nullptr;
     commk = nullptr;
+    pkc = nullptr;
     pk_lim = 0;
     for (auto &x : snap) {
       cudaFree(x.buf);
@@ -267,6 +269,7 @@ struct fastt_graph {
   } io[3];
   bool use_rank_reuse = true;  // FASTT_NO_RANK_REUSE=1: SPLIT slots recompute every rank (A/B parity)
   bool use_pk = true;      // FASTT_NO_PK=1: the lane kernel without packed device keys (A/B parity)
+  bool use_pk_tma = true;  // FASTT_NO_PK_TMA=1: packed keys on k_sim_lane instead of k_lane_pk (A/B parity)
   uint32_t pk_lim_cap = 0xFFFFFFFFu;  // FASTT_PK_LIM=<ns>: lower the deferral bound (tests of the deferral path)
   bool use_lane = true;   // FASTT_NO_LANE=1 keeps position-order launches on the group kernel (A/B parity)
   int last_topo = 0;      // the last main launch: 0 ready-set kernel, 1 group position-order, 2 lane position-order
@@ -408,13 +411,15 @@ static fastt_status prepare_base(fastt_graph *g, Base &B, cudaStream_t st) {
   if (g->use_pk && B.tbits == 32 && g->K == 1 && B.n > 0) {
     int gsh = 0;
     while ((1 << gsh) < g->G) gsh++;
-    const size_t nck = ((size_t)B.n * g->G + 3) & ~(size_t)3;  // (commk 16-B aligned)
-    CK(cudaMalloc(&B.costk, sizeof(uint32_t) * (nck + 4 * (size_t)B.n)));
+    const size_t nck = ((size_t)B.n * g->G + 3) & ~(size_t)3;  // (commk, pkc 16-B aligned)
+    const size_t pkw = (size_t)pk_card_words_host(gsh);
+    CK(cudaMalloc(&B.costk, sizeof(uint32_t) * (nck + 4 * (size_t)B.n + pkw * (size_t)B.n)));
     B.commk = B.costk + nck;
+    B.pkc = B.commk + 4 * (size_t)B.n;
     unsigned long long *d_m = nullptr, hm[2];
     CK(cudaMalloc(&d_m, 16));
     CK(cudaMemsetAsync(d_m, 0, 16, st));
-    launch_pack_costs(B.pg_dev, B.n, g->G, gsh, P.E, B.costk, B.commk, d_m, st);
+    launch_pack_costs(B.pg_dev, B.n, g->G, gsh, P.E, B.costk, B.commk, B.pkc, d_m, st);
     CK(cudaGetLastError());
     CK(cudaMemcpyAsync(hm, d_m, 16, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -609,6 +614,7 @@ static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
   a.fastcomm = B.tbits == 32 && g->K == 1;
   a.costk = B.costk;
   a.commk = B.commk;
+  a.pkc = g->use_pk_tma ? B.pkc : nullptr;
   a.pk_lim = B.pk_lim;
   if (flags & FASTT_F_MEM_LIVE) {
     a.live_mem = 1;
@@ -1217,6 +1223,8 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     g->use_rank_reuse = !(e && e[0] == '1');
     e = getenv("FASTT_NO_PK");
     g->use_pk = !(e && e[0] == '1');
+    e = getenv("FASTT_NO_PK_TMA");
+    g->use_pk_tma = !(e && e[0] == '1');
     e = getenv("FASTT_PK_LIM");
     if (e && e[0]) g->pk_lim_cap = (uint32_t)std::max(1ll, std::min(0xFFFFFFFFll, atoll(e)));
   }

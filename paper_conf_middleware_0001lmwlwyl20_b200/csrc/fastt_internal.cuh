@@ -237,6 +237,7 @@ struct SimArgs {
   // which a candidate is deferred (0 = packed keys off)
   const uint32_t *costk;
   const uint32_t *commk;  // [n][4] inline predecessors' comm << gshift (PK, one class)
+  const uint32_t *pkc;    // [n][pk_card_words] compact PK cards (k_lane_pk.cuh)
   uint32_t pk_lim;
   // memory mode of the lane kernel: 0 none, 1 per-device peak, 2 finite caps
   int32_t lane_mm;
@@ -270,6 +271,9 @@ FASTT_DECL_SIM_FN(0) FASTT_DECL_SIM_FN(1) FASTT_DECL_SIM_FN(2) FASTT_DECL_SIM_FN
 FASTT_DECL_SIM_FN(5)
 #undef FASTT_DECL_SIM_FN
 #define FASTT_DECL_LANE_FN(N, M) const void *lane_fn_g##N##_m##M(int tbits, int cm, bool exact, bool mg, bool pk);
+#define FASTT_DECL_PK_FN(N) const void *lane_pk_fn_g##N(int mm, bool exact);
+FASTT_DECL_PK_FN(0) FASTT_DECL_PK_FN(1) FASTT_DECL_PK_FN(2) FASTT_DECL_PK_FN(3) FASTT_DECL_PK_FN(4) FASTT_DECL_PK_FN(5)
+#undef FASTT_DECL_PK_FN
 #define FASTT_DECL_LANE_FN3(N) FASTT_DECL_LANE_FN(N, 0) FASTT_DECL_LANE_FN(N, 1) FASTT_DECL_LANE_FN(N, 2)
 FASTT_DECL_LANE_FN3(0) FASTT_DECL_LANE_FN3(1) FASTT_DECL_LANE_FN3(2) FASTT_DECL_LANE_FN3(3) FASTT_DECL_LANE_FN3(4)
 FASTT_DECL_LANE_FN3(5)
@@ -309,7 +313,9 @@ int lane_occupancy(int tbits, int gshift, int mm, bool pk);
 // costk[p][d] = (cost[p][d] << gshift) | d over n positions; mx[0] = max
 // cost, mx[1] = max edge comm (one link class) of the prepared graph
 void launch_pack_costs(const PrepGraph *pg_dev, int32_t n, int G, int gshift, int64_t E, uint32_t *costk,
-                       uint32_t *commk, unsigned long long *mx, cudaStream_t st);
+                       uint32_t *commk, uint32_t *pkc, unsigned long long *mx, cudaStream_t st);
+// words of one compact PK card (k_lane_pk.cuh)
+int pk_card_words_host(int gshift);
 // BASE records (uint32 time: FT | place << 32) -> packed keys FT << gshift | place
 void launch_snap_keys(const void *rec, int32_t n, int gshift, uint32_t *key, cudaStream_t st);
 void launch_fit(int G, int64_t n, const uint8_t *src, const uint8_t *dst, const int64_t *bytes, const int64_t *tns,

@@ -37,6 +37,7 @@
 //
 // The kernel itself is in k_sim_lane_body.cuh (instances: k_sim_lane_inst.cu).
 #include "k_sim_lane_body.cuh"
+#include "k_lane_pk.cuh"
 
 namespace fastt {
 
@@ -84,7 +85,7 @@ size_t lane_smem(int tbits, int gshift, bool mg, int mm, bool pk) {
 }
 
 __global__ void k_pack_costs(const PrepGraph *pgp, int32_t n, int G, int gshift, int64_t E, uint32_t *costk,
-                             uint32_t *commk, unsigned long long *mx) {
+                             uint32_t *commk, uint32_t *pkc, int pkw, unsigned long long *mx) {
   const PrepGraph &P = *pgp;
   const uint32_t *c = (const uint32_t *)P.costp;
   const uint32_t *pc = (const uint32_t *)P.pe_comm;
@@ -101,12 +102,31 @@ __global__ void k_pack_costs(const PrepGraph *pgp, int32_t n, int G, int gshift,
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < 4 * (int64_t)n;
        i += (int64_t)gridDim.x * blockDim.x)
     commk[i] = P.card[(i >> 2) * CARD_WORDS + CW_PCOMM + (i & 3)] << gshift;
+  // compact PK cards (k_lane_pk.cuh): deg, pbase, cpidx, 0 | 4 predecessor
+  // positions | their comm << gshift | mem lo, hi, 0, 0 | packed cost row
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < (int64_t)pkw * n;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t p = i / pkw;
+    const int w = (int)(i % pkw);
+    const uint32_t *cd = P.card + p * CARD_WORDS;
+    uint32_t v = 0;
+    if (w == 0) v = cd[CW_DEG];
+    else if (w == 1) v = cd[CW_PBASE];
+    else if (w == 2) v = cd[CW_CPIDX];
+    else if (w >= 4 && w < 8) v = cd[CARD_HDR + (w - 4)];
+    else if (w >= 8 && w < 12) v = cd[CW_PCOMM + (w - 8)] << gshift;
+    else if (w == 12) v = cd[CW_MEMLO];
+    else if (w == 13) v = cd[CW_MEMHI];
+    else if (w >= 16 && w - 16 < G) v = (c[p * G + (w - 16)] << gshift) | (uint32_t)(w - 16);
+    pkc[i] = v;
+  }
   atomicMax(mx, (unsigned long long)mc);
   atomicMax(mx + 1, (unsigned long long)mm);
 }
+int pk_card_words_host(int gshift) { return pk_card_words(1 << gshift); }
 void launch_pack_costs(const PrepGraph *pg_dev, int32_t n, int G, int gshift, int64_t E, uint32_t *costk,
-                       uint32_t *commk, unsigned long long *mx, cudaStream_t st) {
-  k_pack_costs<<<148, 256, 0, st>>>(pg_dev, n, G, gshift, E, costk, commk, mx);
+                       uint32_t *commk, uint32_t *pkc, unsigned long long *mx, cudaStream_t st) {
+  k_pack_costs<<<148, 256, 0, st>>>(pg_dev, n, G, gshift, E, costk, commk, pkc, pk_card_words(1 << gshift), mx);
 }
 
 __global__ void k_snap_keys(const unsigned long long *rec, int32_t n, int gshift, uint32_t *key) {
@@ -126,10 +146,45 @@ int lane_comm_mode(const SimArgs &a, int tbits) {
 
 // a.lane: 1 = candidates of the base graph (LANE_BLOCK threads per block),
 // 2 = prepared slots, one per lane (one warp per block; grid = warps)
+// the packed-key kernel k_lane_pk (k_lane_pk.cuh) and its shared memory
+static const void *lane_pk_fn(int gshift, int mm, bool exact) {
+  switch (gshift) {
+    case 0: return lane_pk_fn_g0(mm, exact);
+    case 1: return lane_pk_fn_g1(mm, exact);
+    case 2: return lane_pk_fn_g2(mm, exact);
+    case 3: return lane_pk_fn_g3(mm, exact);
+    case 4: return lane_pk_fn_g4(mm, exact);
+    default: return lane_pk_fn_g5(mm, exact);
+  }
+}
+template <int GP> static size_t pk_smem_w(int mm) {
+  return mm == 0 ? pk_smem_per_warp<GP, 0>() : mm == 1 ? pk_smem_per_warp<GP, 1>() : pk_smem_per_warp<GP, 2>();
+}
+static size_t lane_pk_smem(int gshift, int mm) {
+  size_t w;
+  switch (gshift) {
+    case 0: w = pk_smem_w<1>(mm); break;
+    case 1: w = pk_smem_w<2>(mm); break;
+    case 2: w = pk_smem_w<4>(mm); break;
+    case 3: w = pk_smem_w<8>(mm); break;
+    case 4: w = pk_smem_w<16>(mm); break;
+    default: w = pk_smem_w<32>(mm); break;
+  }
+  return (LANE_BLOCK / 32) * w;
+}
+
 void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
   const bool mg = a.lane == 2;
   const int cm = lane_comm_mode(a, tbits);
   const bool pk = !mg && tbits == 32 && cm != 2 && a.costk != nullptr && a.pk_lim > 0;
+  if (pk && a.pkc) {  // the base-graph sweep kernel: TMA-staged packed-key cards
+    const void *f = lane_pk_fn(a.gshift, a.lane_mm, a.G == (1 << a.gshift));
+    const size_t sm = lane_pk_smem(a.gshift, a.lane_mm);
+    SimArgs aa = a;
+    void *args[] = {&aa};
+    cudaLaunchKernel(f, dim3(grid), dim3(LANE_BLOCK), args, sm, st);
+    return;
+  }
   const void *f = lane_fn(tbits, a.gshift, cm, a.G == (1 << a.gshift), mg, pk, a.lane_mm);
   const size_t sm = lane_smem(tbits, a.gshift, mg, a.lane_mm, pk);
   if (mg) cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
@@ -144,6 +199,16 @@ void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
 int lane_occupancy(int tbits, int gshift, int mm, bool pk) {
   int nb = 1 << 30, x = 0;
   if (pk && tbits != 32) return 0;
+  if (pk) {  // k_lane_pk
+    const size_t sm = lane_pk_smem(gshift, mm);
+    for (int ex = 0; ex < 2; ex++) {
+      const void *f = lane_pk_fn(gshift, mm, ex != 0);
+      cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, f, LANE_BLOCK, sm);
+      nb = x < nb ? x : nb;
+    }
+    return nb;
+  }
   const size_t sm = lane_smem(tbits, gshift, false, mm, pk);
   for (int v = (tbits == 32 ? 0 : 2); v < (tbits == 32 ? 6 : 6); v++) {
     if (pk && (v >> 1) == 2) continue;  // (packed keys need one link class)
