@@ -7,23 +7,23 @@
 //   * every position has a compact 16-B aligned "PK card" (pkc, built once
 //     per base by k_pack_costs): header (in-degree, edge base, CP index),
 //     the 4 inline predecessor positions, their comm << GSH, the op's memory
-//     and the packed cost row (cost << GSH | d).  The card of position u is
-//     copied into the warp's shared memory by ONE cp.async.bulk (TMA bulk
-//     engine, SASS UBLKCP) issued by one lane at step u - 2P;
+//     and the packed cost row (cost << GSH | d).  The cards of 8 consecutive
+//     positions (a chunk) are copied into the warp's 32-card ring by ONE
+//     cp.async.bulk (TMA bulk engine, SASS UBLKCP) two chunks ahead, with
+//     completion on an mbarrier (expect_tx / complete_tx) waited once per
+//     chunk;
 //   * records are packed keys FT << GSH | device (4 B): a step's 32 records
 //     are one 128-B row of the warp's slab, so the up-to-4 far predecessor
 //     rows of a step are staged by ONE warp-wide 16-B cp.async (lane l copies
-//     chunk l & 7 of predecessor l >> 3); a predecessor before the warp's
-//     start step lo is the BASE record (the same for every lane): its 16-B
-//     chunk of the BASE key array is staged and word s & 3 read;
-//   * both kinds of copy complete on one mbarrier per pipeline slot: the
-//     card's bytes through expect_tx / complete_tx, the records through
-//     cp.async.mbarrier.arrive.noinc (one arrival per lane); a step waits
-//     on that barrier's phase -- no cp.async groups, no extra __syncwarp.
+//     chunk l & 7 of predecessor l >> 3) P steps ahead; a predecessor before
+//     the warp's start step lo is the BASE record (the same for every lane):
+//     its 16-B chunk of the BASE key array is staged and word s & 3 read.
+//     With the copies the issuing step writes the step's read plan (per
+//     predecessor: the shared-memory address of its record, per-lane or
+//     not), so the step itself reads each record with one add and one load.
 // The state record rows are written by this warp with plain stores and read
-// back by cp.async (the generic proxy), so no proxy fence is needed; only
-// the read-only cards go through the async proxy (written by an earlier
-// kernel).
+// back by cp.async (the generic proxy); only the read-only cards (written by
+// an earlier kernel) go through the async proxy.
 #pragma once
 #include "fastt_internal.cuh"
 #include "sim_common.cuh"
@@ -37,11 +37,13 @@ namespace fastt {
 __host__ __device__ constexpr int pk_card_words(int GP) { return 16 + ((GP + 3) / 4) * 4; }
 __host__ __device__ constexpr int pk_card_bytes(int GP) { return 4 * pk_card_words(GP); }
 
+constexpr int PK_CR = 32;  // card ring slots (4 chunks of 8)
 template <int GP, int MM> __host__ __device__ constexpr size_t pk_mm_off() {
-  // mbarriers [D] u64 | ring [D][32] u32 | stage [D][4][32] u32 | cards [2D]
-  // | avail keys [GP/2][32][2] u32 | memory state (as k_sim_lane)
-  return (size_t)LANE_D * 8 + (size_t)LANE_D * 32 * 4 + (size_t)LANE_D * 4 * 32 * 4 +
-         (size_t)2 * LANE_D * pk_card_bytes(GP) + (size_t)32 * GP * 4;
+  // card mbarriers [4] u64 (64 B) | ring [D][32] u32 | stage [D][4][32] u32 |
+  // read plans [D][8] u32 | cards [32] | avail keys [GP/2][32][2] u32 |
+  // memory state (as k_sim_lane)
+  return (size_t)64 + (size_t)LANE_D * 32 * 4 + (size_t)LANE_D * 4 * 32 * 4 + (size_t)LANE_D * 32 +
+         (size_t)PK_CR * pk_card_bytes(GP) + (size_t)32 * GP * 4;
 }
 template <int GP, int MM> __host__ __device__ constexpr size_t pk_smem_per_warp() {
   return pk_mm_off<GP, MM>() + (MM >= 1 ? (size_t)32 * GP * 8 : 0) + (MM == 2 ? (size_t)32 * GP * 8 : 0);
@@ -50,12 +52,10 @@ template <int GP, int MM> __host__ __device__ constexpr size_t pk_smem_per_warp(
 __device__ __forceinline__ void mbar_init(uint32_t a, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(a), "r"(count) : "memory");
 }
-__device__ __forceinline__ void mbar_expect_tx(uint32_t a, uint32_t bytes) {
-  asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(a), "r"(bytes) : "memory");
-}
-// arrive on the barrier when all prior cp.async of this thread complete
-__device__ __forceinline__ void mbar_cp_async_arrive(uint32_t a) {
-  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(a) : "memory");
+// arrive (the barrier's single expected arrival) and expect `bytes` of
+// asynchronous copies (complete_tx) before the phase completes
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint32_t a, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(a), "r"(bytes) : "memory");
 }
 __device__ __forceinline__ void mbar_wait(uint32_t a, uint32_t parity) {
   asm volatile(
@@ -95,13 +95,14 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_lane_pk(SimArgs a) {
   extern __shared__ __align__(16) unsigned char lsm[];
   unsigned char *const wsm = lsm + (threadIdx.x >> 5) * pk_smem_per_warp<GP, MM>();
   const uint32_t wsa = (uint32_t)__cvta_generic_to_shared(wsm);
-  const uint32_t mbar_sa = wsa;                                   // [D] u64
-  uint32_t *const ring = (uint32_t *)(wsm + D * 8) + lane;       // [D][32]
-  uint32_t *const stage = (uint32_t *)(wsm + D * 8 + D * 128);   // [D][4][32]
-  const uint32_t stage_sa = wsa + D * 8 + D * 128;
-  unsigned char *const cards = wsm + D * 8 + D * 128 + D * 512;  // [2D][CB]
-  const uint32_t cards_sa = stage_sa + D * 512;
-  uint32_t *const avk = (uint32_t *)(cards + 2 * D * CB) + (GP >= 2 ? 2 * lane : lane);
+  const uint32_t mbar_sa = wsa;                              // card barriers [4] u64
+  uint32_t *const ring = (uint32_t *)(wsm + 64) + lane;     // [D][32]
+  const uint32_t ring_sa = wsa + 64;
+  const uint32_t stage_sa = ring_sa + D * 128;              // [D][4][32]
+  uint32_t *const plan = (uint32_t *)(wsm + 64 + D * 640);  // [D][8]: per predecessor (address, lane mask)
+  unsigned char *const cards = wsm + 64 + D * 672;          // [PK_CR][CB]
+  const uint32_t cards_sa = wsa + 64 + D * 672;
+  uint32_t *const avk = (uint32_t *)(cards + PK_CR * CB) + (GP >= 2 ? 2 * lane : lane);
   auto avk_at = [&](uint32_t d) -> uint32_t & { return GP >= 2 ? avk[(d >> 1) * 64 + (d & 1)] : avk[0]; };
   int64_t *const mv = (int64_t *)(wsm + pk_mm_off<GP, MM>()) + lane;
   uint32_t *const s32b = (uint32_t *)(wsm + pk_mm_off<GP, MM>() + (size_t)32 * GP * 8) + (GP >= 4 ? 4 * lane : lane);
@@ -109,7 +110,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_lane_pk(SimArgs a) {
   auto s32_at = [&](uint32_t d) -> uint32_t & { return GP >= 4 ? s32b[(d >> 2) * 128 + (d & 3)] : s32b[d * 32]; };
   auto clamp32 = [](int64_t v) -> uint32_t { return v >= (int64_t)0xFFFFFFFFll ? 0xFFFFFFFFu : (uint32_t)v; };
   if (lane == 0)
-    for (int j = 0; j < D; j++) mbar_init(mbar_sa + 8 * j, 32);
+    for (int j = 0; j < 4; j++) mbar_init(mbar_sa + 8 * j, 1);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncwarp();
 
@@ -126,7 +127,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_lane_pk(SimArgs a) {
   const uint32_t *__restrict__ snap = a.snap_key;
   const bool cp_on = (a.flags & 1u) != 0;
   int64_t bms = I64MAX, bidx = -1;
-  uint32_t grp = 0;  // groups (pipeline slots) issued by this warp so far
+  uint32_t zc = 0;  // card chunks issued by this warp so far (barrier zc & 3, phase (zc >> 2) & 1)
   // this lane's part of a step's record staging: chunk (lane & 7) of inline
   // predecessor (lane >> 3)
   const int pk_k = lane >> 3, pk_c = lane & 7;
@@ -274,45 +275,60 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_lane_pk(SimArgs a) {
       if (pp[k] >= (uint32_t)lo && pp[k] < nxt) nxt = pp[k];
 
     // ------------------------------------------------------ pipeline
-    // group j of this candidate batch (issued at step lo + j - P; the
-    // prologue issues j < P) holds the staged records of step lo + j and the
-    // card of step lo + j + P; it completes on barrier (g0 + j) % D with
-    // phase parity ((g0 + j) / D) & 1.  A record of position s < t is staged
-    // iff s < max(lo, t - P) (older than the ring of the last D records).
-    const uint32_t g0 = grp;
-    auto issue = [&](int32_t u, bool with_card) {  // records of u, card of u + P
-      const uint32_t j = grp++;
-      const uint32_t mb = mbar_sa + 8 * (j & (D - 1));
-      const int32_t uc = u + P;
-      if (with_card && uc < n && lane == 0) {
-        mbar_expect_tx(mb, CB);
-        bulk_g2s(cards_sa + (uint32_t)((uc & (2 * D - 1)) * CB), pkc + (size_t)uc * (CB / 4), CB, mb);
+    // records: the far predecessor rows of step u are staged at step u - P
+    // (one commit group per step, waited P - 1 groups later: the group of
+    // step t is complete at step t); a record of position s < u is staged
+    // iff s < max(lo, u - P), else read from the ring of the last D records.
+    // cards: chunk c = positions [8c, 8c + 8) is copied by one bulk copy at
+    // step 8(c - 2) and waited at step 8c - P (its first card is read by the
+    // staging of step 8c); chunks up to j0 + 1 (j0 = ceil(lo / 8)) are copied
+    // directly here.
+    const int32_t jlo = lo >> 3, j0 = (lo + 7) >> 3;
+    const uint32_t z0 = zc;
+    uint32_t zw = zc;
+    const uint32_t lane4 = 4u * (uint32_t)lane;
+    {
+      const int32_t pend = min(n, 8 * (j0 + 2));
+      for (int32_t u = 8 * jlo; u < pend; u++) {
+        const uint32_t *src = pkc + (size_t)u * (CB / 4);
+        uint32_t *dst = (uint32_t *)(cards + (u & (PK_CR - 1)) * CB);
+        for (int w = lane; w < CB / 4; w += 32) dst[w] = __ldg(src + w);
       }
+    }
+    __syncwarp();
+    auto issue = [&](int32_t u) {  // records of step u and its read plan
       if (u < n) {
-        const uint32_t *cu = (const uint32_t *)(cards + (u & (2 * D - 1)) * CB);
+        const uint32_t slot = (uint32_t)u & (D - 1);
+        const uint32_t *cu = (const uint32_t *)(cards + (u & (PK_CR - 1)) * CB);
         const uint32_t npu = cu[0] & 0xFFFF;
         const uint32_t s = cu[4 + pk_k];
         const int32_t thr = lo > u - P ? lo : u - P;
+        const bool used = (uint32_t)pk_k < npu;
+        const bool staged = used && (int32_t)s < thr;
         const bool base_rec = (int32_t)s < lo;  // the BASE record: one 16-B chunk holds it
-        const bool on = (uint32_t)pk_k < npu && (int32_t)s < thr && (!base_rec || pk_c == 0);
         const uint32_t *src = base_rec ? snap + (s & ~3u) : col0 + (size_t)s * 32 + 4 * pk_c;
-        cp16_if(on, stage_sa + (uint32_t)(((u & (D - 1)) * 4 + pk_k) * 128 + 16 * pk_c), src);
+        const uint32_t row = stage_sa + (slot * 4 + (uint32_t)pk_k) * 128;
+        cp16_if(staged && (!base_rec || pk_c == 0), row + 16 * pk_c, src);
+        if (pk_c == 0) {  // the read plan: record address for lane 0, and the per-lane mask
+          const uint32_t ad = staged ? (base_rec ? row + 4 * (s & 3u) : row) : ring_sa + (s & (D - 1)) * 128;
+          const uint32_t mk = (staged && base_rec) ? 0u : 0xFFFFFFFFu;
+          *(uint2 *)(plan + slot * 8 + 2 * pk_k) = make_uint2(ad, mk);
+        }
       }
-      mbar_cp_async_arrive(mb);
+      cp_async_commit();
     };
-    auto wait_grp = [&](uint32_t j) { mbar_wait(mbar_sa + 8 * (j & (D - 1)), (j / D) & 1); };
-    // prologue: cards of lo .. lo + P - 1 copied directly, groups 0 .. P - 1
-    for (int32_t u = lo; u < lo + P && u < n; u++) {
-      const uint32_t *src = pkc + (size_t)u * (CB / 4);
-      uint32_t *dst = (uint32_t *)(cards + (u & (2 * D - 1)) * CB);
-      for (int w = lane; w < CB / 4; w += 32) dst[w] = __ldg(src + w);
-    }
-    __syncwarp();
-    for (int32_t u = lo; u < lo + P; u++) {
-      // (the card of u + P is copied by this group; the records of u need
-      // the card of u, copied above)
-      issue(u, true);
-    }
+    auto issue_chunk = [&](int32_t c) {  // cards [8c, 8c + 8) into the card ring
+      if (8 * c < n) {
+        const uint32_t z = zc++;
+        if (lane == 0) {
+          const uint32_t cnt = (uint32_t)min(8, n - 8 * c);
+          const uint32_t mb = mbar_sa + 8 * (z & 3);
+          mbar_arrive_expect_tx(mb, cnt * CB);
+          bulk_g2s(cards_sa + (uint32_t)(((8 * c) & (PK_CR - 1)) * CB), pkc + (size_t)(8 * c) * (CB / 4), cnt * CB, mb);
+        }
+      }
+    };
+    for (int32_t u = lo; u < lo + P; u++) issue(u);
     // a record of position s (extra predecessors beyond the card's 4)
     auto rec_at = [&](uint32_t s, int32_t t) -> uint32_t {
       if ((int32_t)s < lo) return __ldg(snap + s);
@@ -321,10 +337,19 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_lane_pk(SimArgs a) {
     };
     for (int32_t t = lo; t < nmax; t++) {
       const bool live = run && !dead;
-      wait_grp(g0 + (uint32_t)(t - lo));  // records of t, card of t + P
-      const uint32_t *cw = (const uint32_t *)(cards + (t & (2 * D - 1)) * CB);
+      if (((t + P) & 7) == 0) {  // the next chunk's first card is staged below
+        const int32_t c = (t + P) >> 3;
+        if (c >= j0 + 2 && 8 * c < n) {
+          const uint32_t z = z0 + (uint32_t)(c - (j0 + 2));
+          mbar_wait(mbar_sa + 8 * (z & 3), (z >> 2) & 1);
+          zw = z + 1;
+        }
+      }
+      if ((t & 7) == 0) issue_chunk((t >> 3) + 2);
+      cp_async_wait<P - 1>();  // the group of step t: its staged records
+      __syncwarp();            // (and the read plan other lanes wrote)
+      const uint32_t *cw = (const uint32_t *)(cards + (t & (PK_CR - 1)) * CB);
       const uint4 h0 = *(const uint4 *)cw;
-      const uint4 hs = *(const uint4 *)(cw + 4);
       const uint4 hc = *(const uint4 *)(cw + 8);  // comm << GSH (0 in unused slots)
       uint32_t cst[GP];
       RowLd<uint32_t>::template load_s<GP>(cw + 16, G, cst);
@@ -337,17 +362,17 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_lane_pk(SimArgs a) {
       const int64_t mem64 = (int64_t)(((uint64_t)memhi << 32) | memlo);
       bool cpf = false;
       const uint32_t npred = h0.x & 0xFFFF;
-      const uint32_t src[4] = {hs.x, hs.y, hs.z, hs.w};
-      const int32_t thr = lo > t - P ? lo : t - P;
       uint32_t rk[4];
+      {
+        const uint4 pa = *(const uint4 *)(plan + (t & (D - 1)) * 8);
+        const uint4 pb = *(const uint4 *)(plan + (t & (D - 1)) * 8 + 4);
+        const uint32_t ad[4] = {pa.x + (lane4 & pa.y), pa.z + (lane4 & pa.w), pb.x + (lane4 & pb.y),
+                                pb.z + (lane4 & pb.w)};
 #pragma unroll
-      for (int k = 0; k < 4; k++) {
-        const uint32_t s = src[k];
-        const uint32_t *stg = stage + ((t & (D - 1)) * 4 + k) * 32;
-        rk[k] = (int32_t)s < thr ? stg[(int32_t)s < lo ? (s & 3u) : (uint32_t)lane] : ring[(s & (D - 1)) * 32];
+        for (int k = 0; k < 4; k++) rk[k] = *(const uint32_t *)__cvta_shared_to_generic(ad[k]);
       }
-      __syncwarp();  // (every lane has read the stage slot and card slot the next issue may overwrite)
-      issue(t + P, true);
+      __syncwarp();  // (every lane has read the stage, plan and card slots the next issue may overwrite)
+      issue(t + P);
       // arrival terms in key space (k_sim_lane): R_k = key_k + (c_k << GSH)
       const uint32_t hcw[4] = {hc.x, hc.y, hc.z, hc.w};
       uint32_t rkm[4], R[4];
@@ -473,12 +498,9 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_lane_pk(SimArgs a) {
         ring[(t & (D - 1)) * 32] = bk;
       }
     }
-    // drain: the P groups issued past the last step (nothing may land in
-    // the stage or card slots after this batch)
-    {
-      const uint32_t done = (uint32_t)(nmax > lo ? nmax - lo : 0);
-      for (uint32_t j = done; j < done + (uint32_t)P; j++) wait_grp(g0 + j);
-    }
+    // drain: nothing may land in the stage or card slots after this batch
+    cp_async_wait<0>();
+    for (uint32_t z = zw; z < zc; z++) mbar_wait(mbar_sa + 8 * (z & 3), (z >> 2) & 1);
     __syncwarp();
 
     // ------------------------------------------------------------ epilogue
