@@ -297,6 +297,22 @@ struct fastt_graph {
   int64_t *srt_tmp_i = nullptr, *srt_i = nullptr, *srt_res = nullptr;
   uint32_t *srt_key = nullptr, *srt_hist = nullptr;
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+  // overlapped preparation: the deferred tail of a classified list is
+  // prepared and simulated on a high-priority stream while the main launch
+  // (non-persistent, on the call's stream) runs
+  bool use_overlap = true;  // FASTT_NO_OVERLAP=1 (A/B parity)
+  int lane_batches = 1;     // FASTT_LANE_BATCHES: batches per warp of the non-persistent main launch
+  cudaStream_t st_prep = nullptr;
+  cudaEvent_t ov_ev[4] = {nullptr, nullptr, nullptr, nullptr};  // classified, prep start, prep done, main done
+  void *slab_mg = nullptr;  // slab columns of the concurrent slot launches
+  int64_t slab_mg_cols = 0;
+  unsigned long long *counters2 = nullptr;  // work counter of the concurrent slot launches
+  uint32_t *ov_words = nullptr;             // [0] n_main (classified), [1] active preparation slots
+  uint32_t *slot_bm = nullptr;              // slab-slot bitmap of the non-persistent main launch
+  int32_t slot_bm_bits = 0;
+  int64_t wbest_cap = 0;        // wbest entries allocated
+  int64_t pin_defer_hint = 256; // rank-changing PINs seen by the last classified call
+  int64_t last_nd = -1;         // deferred candidates of the last eval_batch (overlapped path), else -1
   std::mutex mu;
 };
 
@@ -517,6 +533,7 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     size_t rec = B.tbits == 32 ? 8 : 16;
     CK(cudaMalloc(&g->slab, (size_t)nslot * ncap * rec));
     CK(cudaMalloc(&g->wbest, sizeof(int64_t) * 2 * nslot));
+    g->wbest_cap = nslot;
     g->sim_tbits = B.tbits;
     g->sim_ncap = ncap;
   }
@@ -632,19 +649,22 @@ static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
 // Preparation pipeline for nslots deferred candidates already in slot_cands
 // (SURVEY 8(a) S3 + S4 + S5 per candidate): materialise splits, ranks with
 // the candidate's allowed sets, priority sort, cards, critical path.
-static fastt_status run_prep(fastt_graph *g, const Base &B, int nslots, cudaStream_t st) {
+// (nact: the device count of active slots when the wave is sized on the
+// device -- the grids cover nslots, slots past *nact exit at once)
+static fastt_status run_prep(fastt_graph *g, const Base &B, int nslots, cudaStream_t st,
+                             const uint32_t *nact = nullptr) {
   g->launches += NL_PREP;
   launch_slot_setup(g->slot_cands, g->tmpl_dev, B.raw_dev, g->slot_raws_dev, nslots, st);
   launch_copy_block(B.raw_block, g->arena, (int64_t)(g->arena_raw_total + g->arena_prep_total), (int64_t)B.rl.total,
-                    g->slot_cands, nslots, st);
-  launch_patch_split(B.raw_dev, g->slot_raws_dev, g->gc_dev, g->slot_cands, nslots, st);
+                    g->slot_cands, nslots, st, nact);
+  launch_patch_split(B.raw_dev, g->slot_raws_dev, g->gc_dev, g->slot_cands, nslots, st, nact);
   launch_rank(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, g->slot_cands, nslots, g->G, st,
-              g->use_rank_reuse ? prep_struct(B.prep_block, B.pl, B.tbits).rank : nullptr);
-  launch_sort(g->slot_pgs_dev, g->slot_raws_dev, nslots, B.key_bits, (int)B.rl.vcap, st);
+              g->use_rank_reuse ? prep_struct(B.prep_block, B.pl, B.tbits).rank : nullptr, nact);
+  launch_sort(g->slot_pgs_dev, g->slot_raws_dev, nslots, B.key_bits, (int)B.rl.vcap, st, nact);
   // (successor lists only for slots the ready-set kernel will run: see launch_slots)
   launch_cards(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, nslots, (int)B.rl.vcap, g->G, g->K, B.tbits, st,
-               !g->use_topo);
-  launch_cp(g->slot_raws_dev, g->slot_pgs_dev, nslots, g->G, B.tbits, st);
+               !g->use_topo, nact);
+  launch_cp(g->slot_raws_dev, g->slot_pgs_dev, nslots, g->G, B.tbits, st, nact);
   CK(cudaGetLastError());
   return FASTT_OK;
 }
@@ -791,6 +811,157 @@ static void launch_slots(fastt_graph *g, SimArgs b, int tbits, int nc, cudaStrea
   g->launches += g->use_topo ? 1 : 0;
 }
 
+// ------------------------------------------------- overlapped evaluation
+// A start-step-sorted candidate list classified on the device (launch_t0_sort
+// with T0Classify: the candidates that need their own prepared graph sorted
+// to the tail, n_main = ov_words[0] the others) is evaluated by two
+// concurrent pipelines: the main lane launch over [0, n_main) on the call's
+// stream -- non-persistent (each warp takes lane_batches batches and a slab
+// slot), so its blocks retire while it runs -- and, on a high-priority
+// stream, the gather of the tail into the preparation arena, the
+// preparation kernels and the slot simulations (their own slab columns,
+// work counter and wbest entries after the main launch's).  The wave is
+// sized on the device (nact); a tail longer than the arena, and candidates
+// the main launch defers (packed-key bound), run after the join.
+
+static fastt_status ensure_overlap(fastt_graph *g, const Base &B, int cap, int wmain) {
+  if (!g->st_prep) {
+    int lo = 0, hi = 0;
+    CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+    CK(cudaStreamCreateWithPriority(&g->st_prep, cudaStreamNonBlocking, hi));
+    for (auto &e : g->ov_ev) CK(cudaEventCreate(&e));
+    CK(cudaMalloc(&g->counters2, 2 * sizeof(unsigned long long)));
+    CK(cudaMalloc(&g->ov_words, 16));
+    CK(cudaMemset(g->ov_words, 0, 16));
+  }
+  const int64_t cols = (int64_t)cap + 64;
+  const size_t rec = B.tbits == 32 ? 8 : 16;
+  if (!g->slab_mg || g->slab_mg_cols < cols) {
+    cudaFree(g->slab_mg);
+    g->slab_mg = nullptr;
+    CK(cudaMalloc(&g->slab_mg, (size_t)cols * (size_t)g->sim_ncap * rec));
+    g->slab_mg_cols = cols;
+  }
+  if (g->slot_bm_bits < wmain) {
+    cudaFree(g->slot_bm);
+    g->slot_bm = nullptr;
+    CK(cudaMalloc(&g->slot_bm, sizeof(uint32_t) * (size_t)((wmain + 31) / 32)));
+    g->slot_bm_bits = wmain;
+  }
+  if (g->wbest_cap < wmain + cols) {
+    cudaFree(g->wbest);
+    g->wbest = nullptr;
+    CK(cudaMalloc(&g->wbest, sizeof(int64_t) * 2 * (size_t)(wmain + cols)));
+    g->wbest_cap = wmain + cols;
+  }
+  return FASTT_OK;
+}
+
+// resident warps of the main lane launch (its slab slots and wbest entries)
+static int lane_warps(const fastt_graph *g, const SimArgs &a) { return g->sim_grid_lane[a.lane_mm][1] * (LANE_BLOCK / 32); }
+
+// the overlapped launches after the classified sort (a: the main launch's
+// arguments, mode 3 over g->srt_*); results: per-candidate outputs through
+// slot_result (schedule_batch) instead of per-warp bests (sweeps)
+static fastt_status run_overlapped(fastt_graph *g, Base &B, SimArgs a, int64_t n, uint32_t flags, cudaStream_t st,
+                                   bool results, int cap, int wmain) {
+  cudaStream_t sp = g->st_prep;
+  if (a.track_best) launch_init_best(g->wbest, (int64_t)wmain + cap + 64, st);
+  CK(cudaMemsetAsync(g->slot_bm, 0, sizeof(uint32_t) * (size_t)((wmain + 31) / 32), st));
+  CK(cudaMemsetAsync(g->counters2, 0, 2 * sizeof(unsigned long long), st));
+  CK(cudaEventRecord(g->ov_ev[0], st));
+  // preparation pipeline + slot simulations (high priority)
+  CK(cudaStreamWaitEvent(sp, g->ov_ev[0], 0));
+  if (flags & FASTT_F_TIMING) CK(cudaEventRecord(g->ov_ev[1], sp));
+  launch_gather_tail(g->srt_c, g->srt_i, results ? g->srt_res : nullptr, g->ov_words, n, 0, cap, g->slot_cands,
+                     g->slot_index, results ? g->slot_result : nullptr, g->ov_words + 1, sp);
+  g->launches += NL_GATHER;
+  TRY(run_prep(g, B, cap, sp, g->ov_words + 1));
+  SimArgs b = a;
+  b.slots = g->slot_pgs_dev;
+  b.cands = g->slot_cands;
+  b.slot_index = results ? nullptr : g->slot_index;
+  b.slot_result = results ? g->slot_result : nullptr;
+  b.n = cap;
+  b.n_dev = g->ov_words + 1;
+  b.counter = g->counters2;
+  b.ndefer = g->counters2 + 1;
+  b.wbest = g->wbest + 2 * (int64_t)wmain;
+  b.slab = g->slab_mg;
+  b.lane_batches = 0;
+  b.preclassified = 0;
+  b.stat = nullptr;
+  launch_slots(g, b, B.tbits, cap, sp);
+  g->launches += NL_SIM;
+  CK(cudaGetLastError());
+  CK(cudaEventRecord(g->ov_ev[2], sp));
+  // the main launch (the call's stream)
+  a.preclassified = 1;
+  a.n_dev = g->ov_words;
+  a.lane_batches = g->lane_batches;
+  a.slot_bm = g->slot_bm;
+  a.n_slab_slots = wmain;
+  const int64_t warps = (n + 31) / 32;
+  const int64_t blocks = (warps + (int64_t)g->lane_batches * (LANE_BLOCK / 32) - 1) /
+                         ((int64_t)g->lane_batches * (LANE_BLOCK / 32));
+  launch_sim(a, B.tbits, (int)std::max<int64_t>(1, std::min<int64_t>(blocks, 1 << 30)), LANE_BLOCK, 0, st);
+  g->launches += NL_SIM;
+  CK(cudaGetLastError());
+  timing_mark(g, flags, 1, st);
+  CK(cudaStreamWaitEvent(st, g->ov_ev[2], 0));
+  return FASTT_OK;
+}
+
+// after the join (host-synchronising): a tail longer than the arena and the
+// main launch's packed-key deferrals, sequentially on st
+static fastt_status finish_overlapped(fastt_graph *g, Base &B, SimArgs a, int64_t n, cudaStream_t st, bool results,
+                                      int cap, int wmain, unsigned long long *nd_total) {
+  uint32_t w[2] = {0, 0};
+  unsigned long long pkd = 0;
+  CK(cudaMemcpyAsync(w, g->ov_words, 8, cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(&pkd, g->counters + 1, sizeof pkd, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  const int64_t tail = n - (int64_t)w[0];
+  g->pin_defer_hint = tail;
+  *nd_total = (unsigned long long)tail + pkd;
+  SimArgs b = a;
+  b.slots = g->slot_pgs_dev;
+  b.cands = g->slot_cands;
+  b.slot_index = results ? nullptr : g->slot_index;
+  b.slot_result = results ? g->slot_result : nullptr;
+  b.wbest = g->wbest + 2 * (int64_t)wmain;
+  b.slab = g->slab_mg;
+  b.lane_batches = 0;
+  b.preclassified = 0;
+  b.stat = nullptr;
+  b.n_dev = nullptr;
+  for (int64_t off = cap; off < tail; off += cap) {  // the tail past the arena
+    const int nc = (int)std::min<int64_t>(cap, tail - off);
+    launch_gather_tail(g->srt_c, g->srt_i, results ? g->srt_res : nullptr, g->ov_words, n, off, cap, g->slot_cands,
+                       g->slot_index, results ? g->slot_result : nullptr, g->ov_words + 1, st);
+    g->launches += NL_GATHER + NL_SIM;
+    TRY(run_prep(g, B, nc, st));
+    CK(cudaMemsetAsync(g->counters2, 0, sizeof(unsigned long long), st));
+    b.counter = g->counters2;
+    b.n = nc;
+    launch_slots(g, b, B.tbits, nc, st);
+    CK(cudaGetLastError());
+  }
+  for (int64_t c0 = 0; c0 < (int64_t)pkd; c0 += cap) {  // packed-key deferrals of the main launch
+    const int nc = (int)std::min<int64_t>(cap, (int64_t)pkd - c0);
+    launch_gather_sorted(g->srt_c, g->srt_i, results ? g->srt_res : nullptr, g->defer_q + c0, nc, g->slot_cands,
+                         results ? nullptr : g->slot_index, results ? g->slot_result : nullptr, st);
+    g->launches += NL_GATHER + NL_SIM;
+    TRY(run_prep(g, B, nc, st));
+    CK(cudaMemsetAsync(g->counters2, 0, sizeof(unsigned long long), st));
+    b.counter = g->counters2;
+    b.n = nc;
+    launch_slots(g, b, B.tbits, nc, st);
+    CK(cudaGetLastError());
+  }
+  return FASTT_OK;
+}
+
 struct DevOut {
   int64_t *makespan = nullptr;
   uint8_t *status = nullptr;
@@ -831,6 +1002,53 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
   a.out.vmax = (int32_t)o.vmax;
   if (sharing) use_snapshot(B, flags, a);
   const bool sorted = a.snap_mode == 2;
+  // the overlapped path (see run_overlapped): packed-key lane kernel, no per-op outputs
+  bool ovl = false;
+  if (sorted && g->use_overlap && a.pkc && a.costk && a.pk_lim > 0 && !o.place && !o.start && !o.deq) {
+    SimArgs t = a;
+    int gr;
+    size_t sm;
+    main_shape(g, B, t, gr, sm);
+    ovl = t.lane == 1;
+  }
+  if (ovl) {
+    TRY(ensure_arena(g, B, st, std::max<int64_t>(256, std::min<int64_t>(g->pin_defer_hint, 8192))));
+    const int cap = g->arena_slots;
+    int wmain;
+    {
+      SimArgs t = a;
+      int gr;
+      size_t sm;
+      main_shape(g, B, t, gr, sm);
+      wmain = lane_warps(g, t);
+    }
+    TRY(ensure_overlap(g, B, cap, wmain));
+    TRY(ensure_sort_buf(g, n));
+    const PrepGraph P = prep_struct(B.prep_block, B.pl, B.tbits);
+    StreamState dummy;
+    memset(&dummy, 0, sizeof dummy);
+    T0Classify cl{1, B.tbits, B.pg_dev, g->gc_dev, a.split_mask, g->ov_words};
+    launch_t0_sort(0, dummy, 0, 1, d_cands, n, P.pos, a.snap_dq, B.n, B.V, g->G, g->srt_tmp_c, g->srt_tmp_i,
+                   g->srt_key, g->srt_hist, g->srt_c, g->srt_i, g->srt_res, st, cl);
+    g->launches += 4;
+    a.mode = 3;
+    a.cands = g->srt_c;
+    a.slot_index = g->srt_i;
+    a.slot_result = g->srt_res;
+    {
+      int gr;
+      size_t sm;
+      main_shape(g, B, a, gr, sm);
+    }
+    TRY(run_overlapped(g, B, a, n, flags, st, true, cap, wmain));
+    timing_mark(g, flags, 2, st);
+    unsigned long long ndo = 0;
+    TRY(finish_overlapped(g, B, a, n, st, true, cap, wmain, &ndo));
+    g->last_nd = (int64_t)ndo;
+    if (o.order) return fail(FASTT_EINVAL, "order output on the overlapped path");  // (excluded above)
+    CK(cudaStreamSynchronize(st));
+    return FASTT_OK;
+  }
   if (sorted) {
     // order the list by BASE-prefix start step (results keep their index)
     TRY(ensure_sort_buf(g, n));
@@ -1225,6 +1443,10 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     g->use_pk = !(e && e[0] == '1');
     e = getenv("FASTT_NO_PK_TMA");
     g->use_pk_tma = !(e && e[0] == '1');
+    e = getenv("FASTT_NO_OVERLAP");
+    g->use_overlap = !(e && e[0] == '1');
+    e = getenv("FASTT_LANE_BATCHES");
+    if (e && e[0]) g->lane_batches = std::max(1, atoi(e));
     e = getenv("FASTT_PK_LIM");
     if (e && e[0]) g->pk_lim_cap = (uint32_t)std::max(1ll, std::min(0xFFFFFFFFll, atoll(e)));
   }
@@ -1325,6 +1547,13 @@ void fastt_free_graph(fastt_graph *g) {
     for (auto &b : g->io) cudaFree(b.p);
     for (auto &e : g->ev)
       if (e) cudaEventDestroy(e);
+    for (auto &e : g->ov_ev)
+      if (e) cudaEventDestroy(e);
+    if (g->st_prep) cudaStreamDestroy(g->st_prep);
+    cudaFree(g->slab_mg);
+    cudaFree(g->counters2);
+    cudaFree(g->ov_words);
+    cudaFree(g->slot_bm);
   }
   delete g;
 }
@@ -1469,9 +1698,12 @@ fastt_status fastt_schedule_batch(const fastt_graph *gc_, const fastt_candidate 
     rc = fail(FASTT_ENOMEM, "device output buffers");
   unsigned long long nd0 = 0;
   if (rc == FASTT_OK) rc = timing_begin(g, flags, st);
+  g->last_nd = -1;
   if (rc == FASTT_OK) rc = eval_batch(g, B, d_c, n, flags, st, o);
-  if (rc == FASTT_OK && (cudaMemcpyAsync(&nd0, g->counters + 1, sizeof nd0, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
-                         cudaStreamSynchronize(st) != cudaSuccess))
+  if (rc == FASTT_OK && g->last_nd >= 0) nd0 = (unsigned long long)g->last_nd;  // (overlapped path)
+  else if (rc == FASTT_OK &&
+           (cudaMemcpyAsync(&nd0, g->counters + 1, sizeof nd0, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+            cudaStreamSynchronize(st) != cudaSuccess))
     rc = fail(FASTT_ECUDA, "deferred count");
   if (rc == FASTT_OK && !outdev) {
     auto back = [&](void *h, void *dd, size_t bytes) {
@@ -1542,28 +1774,74 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
   TRY(check_gen(g, *S, gen, first, n, stride));
   Base &B = g->base;
   TRY(ensure_sim(g, B, n, flags));
-  const int64_t nwarps = max_slots(g);  // candidate slots
-  {
-    std::vector<int64_t> init(2 * nwarps);
-    for (int64_t w = 0; w < nwarps; w++) {
-      init[2 * w] = I64MAX;
-      init[2 * w + 1] = -1;
-    }
-    CK(cudaMemcpyAsync(g->wbest, init.data(), 16 * nwarps, cudaMemcpyHostToDevice, st));
-  }
   if (g->share) TRY(ensure_snapshot(g, B, flags, st));
+  int64_t nwarps = max_slots(g);  // candidate slots (per-warp bests)
+  SimArgs a = sim_args(g, B, flags);
+  a.mode = 0;
+  a.stream = stream_state(g, *S, gen);
+  a.first = first;
+  a.n = n;
+  a.stride = stride;
+  a.track_best = 1;
+  if (g->share) use_snapshot(B, flags, a);
+  // the overlapped path: a sorted, classified list on the packed-key lane kernel
+  bool ovl = false;
+  if (n > 0 && g->use_overlap && a.snap_mode == 2 && a.pkc && a.costk && a.pk_lim > 0) {
+    SimArgs t = a;
+    int gr;
+    size_t sm;
+    main_shape(g, B, t, gr, sm);
+    ovl = t.lane == 1;
+  }
+  int cap = 0, wmain = 0;
+  if (ovl) {
+    // arena: the window's SPLIT and device-subset candidates plus the
+    // rank-changing PINs of the last call (a longer tail runs after the join)
+    const int64_t hi = a.stream.n_split + a.stream.n_subset;
+    int64_t nsp = 0;
+    if (hi >= 1 && first <= hi) {
+      const int64_t q_lo = first >= 1 ? 0 : (1 - first + stride - 1) / stride;
+      const int64_t q_hi = std::min<int64_t>(n - 1, (hi - first) / stride);
+      nsp = q_hi >= q_lo ? q_hi - q_lo + 1 : 0;
+    }
+    TRY(ensure_arena(g, B, st, std::max<int64_t>(nsp + 256, std::min<int64_t>(g->pin_defer_hint, 8192))));
+    cap = g->arena_slots;
+    {
+      SimArgs t = a;
+      int gr;
+      size_t sm;
+      main_shape(g, B, t, gr, sm);
+      wmain = lane_warps(g, t);
+    }
+    TRY(ensure_overlap(g, B, cap, wmain));
+    nwarps = (int64_t)wmain + cap + 64;
+  } else {
+    launch_init_best(g->wbest, nwarps, st);
+  }
   TRY(timing_begin(g, flags, st));
   unsigned long long nd = 0;
-  if (n > 0) {
+  if (n > 0 && ovl) {
     CK(cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), st));
-    SimArgs a = sim_args(g, B, flags);
-    a.mode = 0;
-    a.stream = stream_state(g, *S, gen);
-    a.first = first;
-    a.n = n;
-    a.stride = stride;
-    a.track_best = 1;
-    if (g->share) use_snapshot(B, flags, a);
+    TRY(ensure_sort_buf(g, n));
+    const PrepGraph P = prep_struct(B.prep_block, B.pl, B.tbits);
+    T0Classify cl{1, B.tbits, B.pg_dev, g->gc_dev, a.split_mask, g->ov_words};
+    launch_t0_sort(1, a.stream, first, stride, nullptr, n, P.pos, a.snap_dq, B.n, B.V, g->G, g->srt_tmp_c,
+                   g->srt_tmp_i, g->srt_key, g->srt_hist, g->srt_c, g->srt_i, nullptr, st, cl);
+    g->launches += 4;
+    a.mode = 3;
+    a.cands = g->srt_c;
+    a.slot_index = g->srt_i;
+    a.slot_result = nullptr;
+    {
+      int gr;
+      size_t sm;
+      main_shape(g, B, a, gr, sm);
+    }
+    TRY(run_overlapped(g, B, a, n, flags, st, false, cap, wmain));
+    timing_mark(g, flags, 2, st);
+    TRY(finish_overlapped(g, B, a, n, st, false, cap, wmain, &nd));
+  } else if (n > 0) {
+    CK(cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), st));
     if (a.snap_mode == 2) {
       TRY(ensure_sort_buf(g, n));
       const PrepGraph P = prep_struct(B.prep_block, B.pl, B.tbits);
@@ -1606,9 +1884,11 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
         CK(cudaGetLastError());
       }
     }
+    timing_mark(g, flags, 2, st);
+  } else {
+    timing_mark(g, flags, 1, st);
+    timing_mark(g, flags, 2, st);
   }
-  else timing_mark(g, flags, 1, st);
-  timing_mark(g, flags, 2, st);
   launch_argmin(g->wbest, nwarps, g->best_dev, st);
   g->launches += NL_ARGMIN;
   CK(cudaGetLastError());
@@ -1618,6 +1898,11 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
     CK(cudaMemcpyAsync(best, g->best_dev, 16, cudaMemcpyDeviceToHost, st));
   }
   TRY(timing_end(g, flags, st, n, (int64_t)nd));
+  if (ovl && (flags & FASTT_F_TIMING)) {  // the concurrent preparation stream's own duration
+    float mp = 0;
+    CK(cudaEventElapsedTime(&mp, g->ov_ev[1], g->ov_ev[2]));
+    g->last.ms_prep = mp;
+  }
   CK(cudaStreamSynchronize(st));
   return FASTT_OK;
 }

@@ -254,6 +254,14 @@ struct SimArgs {
   // k_sim_lane instrumentation (nullable): [0] += steps per warp batch,
   // [1] += steps of the batch's running lanes
   unsigned long long *stat;
+  // k_lane_pk non-persistent mode (lane_batches > 0): a warp takes at most
+  // lane_batches batches of 32 candidates, holding one of n_slab_slots slab
+  // columns (and wbest entries) acquired from the bitmap slot_bm for its
+  // lifetime, so the launch's blocks retire while it runs and a concurrent
+  // higher-priority stream (the preparation pipeline) gets SM resources
+  int32_t lane_batches;
+  int32_t n_slab_slots;
+  uint32_t *slot_bm;
 };
 
 // one idle slot [a, b) of a device under INSERT
@@ -305,6 +313,10 @@ void launch_t0_sort(int from_stream, const StreamState &S, int64_t first, int64_
                     const uint32_t *pos, const uint32_t *snap_dq, int32_t nops, int32_t vraw, int G, Cand *tmp_c,
                     int64_t *tmp_i, uint32_t *key, uint32_t *hist, Cand *out_c, int64_t *out_i, int64_t *out_res,
                     cudaStream_t st, T0Classify cl = T0Classify{0, 0, nullptr, nullptr, nullptr, nullptr});
+void launch_gather_tail(const Cand *src, const int64_t *sidx, const int64_t *sres, const uint32_t *n_main, int64_t n,
+                        int64_t off, int cap, Cand *dst, int64_t *didx, int64_t *dres, uint32_t *nslot,
+                        cudaStream_t st);
+void launch_init_best(int64_t *wb, int64_t nw, cudaStream_t st);
 void launch_gather_sorted(const Cand *src, const int64_t *sidx, const int64_t *sres, const int64_t *qs, int64_t n,
                           Cand *dst, int64_t *didx, int64_t *dres, cudaStream_t st);
 int sim_occupancy(int tbits, int gshift, int block, size_t smem, bool topo);

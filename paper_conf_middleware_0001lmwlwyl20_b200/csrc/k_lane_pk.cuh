@@ -87,7 +87,34 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_lane_pk(SimArgs a) {
   constexpr int CB = pk_card_bytes(GP);
   static_assert((D & (D - 1)) == 0 && CB % 16 == 0, "pipeline slots");
   const int lane = threadIdx.x & 31;
-  const int64_t gwarp = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  int64_t gwarp = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  if (a.lane_batches > 0) {
+    // non-persistent launch: the warp's slab column block and wbest entry
+    // are a slot taken from the bitmap for the warp's lifetime (at most
+    // n_slab_slots warps are resident, so one is always free)
+    uint32_t sl = 0;
+    if (lane == 0) {
+      const uint32_t nw = (uint32_t)(a.n_slab_slots + 31) >> 5;
+      for (uint32_t w = (uint32_t)(gwarp % nw);; w = w + 1 == nw ? 0 : w + 1) {
+        uint32_t v = a.slot_bm[w];
+        bool got = false;
+        while (~v) {
+          const uint32_t b = __ffs(~v) - 1;
+          if (w * 32 + b >= (uint32_t)a.n_slab_slots) break;
+          const uint32_t old = atomicOr(&a.slot_bm[w], 1u << b);
+          if (!(old & (1u << b))) {
+            sl = w * 32 + b;
+            got = true;
+            break;
+          }
+          v = old | (1u << b);
+        }
+        if (got) break;
+      }
+      __threadfence();  // (the previous holder's wbest entry is visible)
+    }
+    gwarp = __shfl_sync(FULL, (int)sl, 0);
+  }
   // this lane's slab column (record of position p at col[p * 32]); row p of
   // the warp (all 32 records) starts at col0 + p * 32
   uint32_t *const col = (uint32_t *)a.slab + (size_t)gwarp * (size_t)a.slab_stride * 32 + lane;
@@ -133,7 +160,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_lane_pk(SimArgs a) {
   const int pk_k = lane >> 3, pk_c = lane & 7;
 
   const int64_t nlim = a.n_dev ? ((int64_t)*a.n_dev < a.n ? (int64_t)*a.n_dev : a.n) : a.n;
-  for (;;) {
+  for (int32_t nb = 0; a.lane_batches <= 0 || nb < a.lane_batches; nb++) {
     unsigned long long q0 = 0;
     if (lane == 0) q0 = atomicAdd(a.counter, 32ull);
     q0 = __shfl_sync(FULL, q0, 0);
@@ -296,25 +323,25 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_lane_pk(SimArgs a) {
       }
     }
     __syncwarp();
+    // (branch-free: past the last position the card slot is stale, the
+    // copy is predicated off and the plan is never read)
     auto issue = [&](int32_t u) {  // records of step u and its read plan
-      if (u < n) {
-        const uint32_t slot = (uint32_t)u & (D - 1);
-        const uint32_t *cu = (const uint32_t *)(cards + (u & (PK_CR - 1)) * CB);
-        const uint32_t npu = cu[0] & 0xFFFF;
-        const uint32_t s = cu[4 + pk_k];
-        const int32_t thr = lo > u - P ? lo : u - P;
-        const bool used = (uint32_t)pk_k < npu;
-        const bool staged = used && (int32_t)s < thr;
-        const bool base_rec = (int32_t)s < lo;  // the BASE record: one 16-B chunk holds it
-        const uint32_t *src = base_rec ? snap + (s & ~3u) : col0 + (size_t)s * 32 + 4 * pk_c;
-        const uint32_t row = stage_sa + (slot * 4 + (uint32_t)pk_k) * 128;
-        cp16_if(staged && (!base_rec || pk_c == 0), row + 16 * pk_c, src);
-        if (pk_c == 0) {  // the read plan: record address for lane 0, and the per-lane mask
-          const uint32_t ad = staged ? (base_rec ? row + 4 * (s & 3u) : row) : ring_sa + (s & (D - 1)) * 128;
-          const uint32_t mk = (staged && base_rec) ? 0u : 0xFFFFFFFFu;
-          *(uint2 *)(plan + slot * 8 + 2 * pk_k) = make_uint2(ad, mk);
-        }
-      }
+      const uint32_t slot = (uint32_t)u & (D - 1);
+      const uint32_t *cu = (const uint32_t *)(cards + (u & (PK_CR - 1)) * CB);
+      const uint32_t npu = cu[0] & 0xFFFF;
+      const uint32_t s = cu[4 + pk_k];
+      const int32_t thr = lo > u - P ? lo : u - P;
+      const bool staged = u < n && (uint32_t)pk_k < npu && (int32_t)s < thr;
+      const bool base_rec = (int32_t)s < lo;  // the BASE record: one 16-B chunk holds it
+      const uint32_t *src = base_rec ? snap + (s & ~3u) : col0 + (size_t)s * 32 + 4 * pk_c;
+      const uint32_t row = stage_sa + (slot * 4 + (uint32_t)pk_k) * 128;
+      cp16_if(staged && (!base_rec || pk_c == 0), row + 16 * pk_c, src);
+      // the read plan of predecessor pk_k: its record's address for lane 0
+      // and the per-lane mask (the 8 lanes of a predecessor store the same
+      // pair: one broadcast store)
+      const uint32_t ad = staged ? (base_rec ? row + 4 * (s & 3u) : row) : ring_sa + (s & (D - 1)) * 128;
+      const uint32_t mk = (staged && base_rec) ? 0u : 0xFFFFFFFFu;
+      *(uint2 *)(plan + slot * 8 + 2 * pk_k) = make_uint2(ad, mk);
       cp_async_commit();
     };
     auto issue_chunk = [&](int32_t c) {  // cards [8c, 8c + 8) into the card ring
@@ -371,7 +398,8 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_lane_pk(SimArgs a) {
 #pragma unroll
         for (int k = 0; k < 4; k++) rk[k] = *(const uint32_t *)__cvta_shared_to_generic(ad[k]);
       }
-      __syncwarp();  // (every lane has read the stage, plan and card slots the next issue may overwrite)
+      // (the slots issue(t + P) overwrites were read at step t - 1, before
+      // every lane passed this step's __syncwarp)
       issue(t + P);
       // arrival terms in key space (k_sim_lane): R_k = key_k + (c_k << GSH)
       const uint32_t hcw[4] = {hc.x, hc.y, hc.z, hc.w};
@@ -536,6 +564,13 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_lane_pk(SimArgs a) {
         a.wbest[2 * gwarp] = bms;
         a.wbest[2 * gwarp + 1] = bidx;
       }
+    }
+  }
+  if (a.lane_batches > 0) {
+    __syncwarp();
+    if (lane == 0) {  // release the slot
+      __threadfence();
+      atomicAnd(&a.slot_bm[gwarp >> 5], ~(1u << (gwarp & 31)));
     }
   }
 }

@@ -202,6 +202,38 @@ void launch_t0_sort(int from_stream, const StreamState &S, int64_t first, int64_
   k_bucket_scatter<<<blocks, 256, 0, st>>>(key, tmp_c, tmp_i, n, shift, nb, hist, out_c, out_i, out_res);
 }
 
+// the deferred tail of a classified sorted list: entries [*n_main + off,
+// *n_main + off + cap) into the preparation slots; *nslot = their count
+__global__ void k_gather_tail(const Cand *src, const int64_t *sidx, const int64_t *sres, const uint32_t *n_main,
+                              int64_t n, int64_t off, int cap, Cand *dst, int64_t *didx, int64_t *dres, uint32_t *nslot) {
+  const int64_t base = (int64_t)*n_main + off;
+  int64_t cnt = n - base;
+  cnt = cnt < 0 ? 0 : (cnt > cap ? cap : cnt);
+  if (blockIdx.x == 0 && threadIdx.x == 0) *nslot = (uint32_t)cnt;
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < cnt; k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t q = base + k;
+    dst[k] = src[q];
+    if (didx) didx[k] = sidx[q];
+    if (dres) dres[k] = sres ? sres[q] : -1;
+  }
+}
+void launch_gather_tail(const Cand *src, const int64_t *sidx, const int64_t *sres, const uint32_t *n_main, int64_t n,
+                        int64_t off, int cap, Cand *dst, int64_t *didx, int64_t *dres, uint32_t *nslot,
+                        cudaStream_t st) {
+  const int blocks = (cap + 255) / 256 < 1024 ? (cap + 255) / 256 : 1024;
+  k_gather_tail<<<blocks > 0 ? blocks : 1, 256, 0, st>>>(src, sidx, sres, n_main, n, off, cap, dst, didx, dres, nslot);
+}
+// per-warp best pairs (makespan, index) := (INT64_MAX, -1)
+__global__ void k_init_best(int64_t *wb, int64_t nw) {
+  for (int64_t w = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; w < nw; w += (int64_t)gridDim.x * blockDim.x) {
+    wb[2 * w] = I64MAX;
+    wb[2 * w + 1] = -1;
+  }
+}
+void launch_init_best(int64_t *wb, int64_t nw, cudaStream_t st) {
+  if (nw > 0) k_init_best<<<(int)((nw + 255) / 256 < 1024 ? (nw + 255) / 256 : 1024), 256, 0, st>>>(wb, nw);
+}
+
 __global__ void k_gather_sorted(const Cand *src, const int64_t *sidx, const int64_t *sres, const int64_t *qs, int64_t n,
                                 Cand *dst, int64_t *didx, int64_t *dres) {
   int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
