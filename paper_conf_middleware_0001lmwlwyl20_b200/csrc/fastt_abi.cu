@@ -301,7 +301,8 @@ struct fastt_graph {
   // prepared and simulated on a high-priority stream while the main launch
   // (non-persistent, on the call's stream) runs
   bool use_overlap = true;  // FASTT_NO_OVERLAP=1 (A/B parity)
-  int lane_batches = 1;     // FASTT_LANE_BATCHES: batches per warp of the non-persistent main launch
+  int lane_batches = 1;     // FASTT_LANE_BATCHES: batches per warp of the non-persistent main launch (0: persistent)
+  int main_bps = 0;         // FASTT_MAIN_BPS: resident blocks per SM of a persistent overlapped main launch (0: all)
   cudaStream_t st_prep = nullptr;
   cudaEvent_t ov_ev[4] = {nullptr, nullptr, nullptr, nullptr};  // classified, prep start, prep done, main done
   void *slab_mg = nullptr;  // slab columns of the concurrent slot launches
@@ -901,9 +902,14 @@ static fastt_status run_overlapped(fastt_graph *g, Base &B, SimArgs a, int64_t n
   a.lane_batches = g->lane_batches;
   a.slot_bm = g->slot_bm;
   a.n_slab_slots = wmain;
-  const int64_t warps = (n + 31) / 32;
-  const int64_t blocks = (warps + (int64_t)g->lane_batches * (LANE_BLOCK / 32) - 1) /
-                         ((int64_t)g->lane_batches * (LANE_BLOCK / 32));
+  int64_t blocks;
+  if (g->lane_batches > 0) {
+    const int64_t warps = (n + 31) / 32;
+    blocks = (warps + (int64_t)g->lane_batches * (LANE_BLOCK / 32) - 1) / ((int64_t)g->lane_batches * (LANE_BLOCK / 32));
+  } else {  // persistent, optionally leaving block slots to the preparation stream
+    blocks = wmain / (LANE_BLOCK / 32);
+    if (g->main_bps > 0) blocks = std::min<int64_t>(blocks, (int64_t)g->sms * g->main_bps);
+  }
   launch_sim(a, B.tbits, (int)std::max<int64_t>(1, std::min<int64_t>(blocks, 1 << 30)), LANE_BLOCK, 0, st);
   g->launches += NL_SIM;
   CK(cudaGetLastError());
@@ -1446,7 +1452,9 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     e = getenv("FASTT_NO_OVERLAP");
     g->use_overlap = !(e && e[0] == '1');
     e = getenv("FASTT_LANE_BATCHES");
-    if (e && e[0]) g->lane_batches = std::max(1, atoi(e));
+    if (e && e[0]) g->lane_batches = std::max(0, atoi(e));
+    e = getenv("FASTT_MAIN_BPS");
+    if (e && e[0]) g->main_bps = std::max(0, atoi(e));
     e = getenv("FASTT_PK_LIM");
     if (e && e[0]) g->pk_lim_cap = (uint32_t)std::max(1ll, std::min(0xFFFFFFFFll, atoll(e)));
   }
