@@ -409,12 +409,14 @@ def main():
                "api": "fastt_schedule_batch (host pinned buffers; makespan, status, per-device peak memory)",
                "argmin_local_index": i, "kernel": "k_sim_lane" if g.last_timing()["topo"] == 2 else "k_sim"}
 
-    # the other paper-shaped configs: one sweep each,
+    # the other paper-shaped configs (SURVEY 8(d) C1-C4, and C5R8 = BERT-large
+    # x 8 replicas, 37,921 ops): one sweep each,
     # device-timed (not part of the step), candidates/s and DAG-ops/s
     configs = None
     if not args.no_configs:
         configs = {}
-        for name, ncand in (("C1", 1_000_000), ("C2", 300_000), ("C3", 200_000), ("C4", 300_000)):
+        for name, ncand in (("C1", 1_000_000), ("C2", 300_000), ("C3", 200_000), ("C4", 300_000),
+                            ("C5R8", 200_000)):
             d2 = synth.config(name)
             g2 = F.Graph(d2, device=local)
             gen2 = F.gen_params(seed=GEN_SEED, pin_k_min=1, pin_k_max=4, n_pow2_only=(name == "C4"))

@@ -280,7 +280,7 @@ struct fastt_graph {
   int64_t gap_stride = 0;
   int ins_grid = 0;
   int64_t *wbest = nullptr, *best_dev = nullptr;
-  unsigned long long *counters = nullptr;  // [0] work counter, [1] deferred count, [2..3] k_sim_lane step counts
+  unsigned long long *counters = nullptr;  // [0] work counter, [1] deferred count, [2..3] k_sim_lane step counts, [4] kernel error
   int64_t *defer_q = nullptr;
   int64_t defer_cap = 0;
   // misc scratch
@@ -333,7 +333,23 @@ static fastt_status timing_begin(fastt_graph *g, uint32_t flags, cudaStream_t st
 static void timing_mark(fastt_graph *g, uint32_t flags, int k, cudaStream_t st) {
   if (flags & FASTT_F_TIMING) cudaEventRecord(g->ev[k], st);
 }
+// a ready-set launch met a graph above READY_SET_MAX positions (k_sim sets
+// counters[4]): the call fails (reads and clears the flag; synchronises st)
+static fastt_status check_kernel_err(fastt_graph *g, cudaStream_t st) {
+  if (!g->counters) return FASTT_OK;
+  unsigned long long e = 0;
+  CK(cudaMemcpyAsync(&e, g->counters + 4, sizeof e, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  if (e) {
+    CK(cudaMemsetAsync(g->counters + 4, 0, sizeof e, st));
+    return fail(FASTT_EUNSUP, "a candidate's priority order is not topological and its graph has more than %d ops "
+                              "(the ready-set kernel's bitmap)", (int)READY_SET_MAX);
+  }
+  return FASTT_OK;
+}
+
 static fastt_status timing_end(fastt_graph *g, uint32_t flags, cudaStream_t st, int64_t cands, int64_t deferred) {
+  TRY(check_kernel_err(g, st));
   g->last.launches = g->launches;
   g->last.candidates = cands;
   g->last.deferred = deferred;
@@ -424,6 +440,11 @@ static fastt_status prepare_base(fastt_graph *g, Base &B, cudaStream_t st) {
   B.n = P.n;
   B.cp_len = P.cp_len;
   B.topo = P.topo;
+  if (B.rl.vcap > READY_SET_MAX && !B.topo)
+    return fail(FASTT_EUNSUP,
+                "a graph above %d ops needs a topological priority order (every edge with w_i + c_ij > 0, R2): "
+                "the ready-set kernel's bitmap covers %d positions",
+                READY_SET_MAX, READY_SET_MAX);
   // packed keys (k_sim_lane PK): the bound below which no key wraps
   if (g->use_pk && B.tbits == 32 && g->K == 1 && B.n > 0) {
     int gsh = 0;
@@ -512,7 +533,9 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     g->gap = nullptr;
     const int gsh = gshift_of(g->G);
     const int cpw = 32 >> gsh;
-    int leaf = (int)((ncap + 31) / 32);
+    // (the ready-set bitmap: the ready-set kernel runs on at most
+    // READY_SET_MAX positions, larger graphs are topological)
+    int leaf = (int)((std::min<int64_t>(ncap, READY_SET_MAX) + 31) / 32);
     int stride = leaf + 32;
     while (stride % 32 != 8) stride++;  // candidates of one warp start on different banks
     size_t smem = (size_t)(g->sim_block / 32) * cpw * stride * 4;
@@ -558,8 +581,8 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     g->ins_grid = (int)ig;
   }
   if (!g->counters) {
-    CK(cudaMalloc(&g->counters, 4 * sizeof(unsigned long long)));
-    CK(cudaMemset(g->counters, 0, 4 * sizeof(unsigned long long)));
+    CK(cudaMalloc(&g->counters, 5 * sizeof(unsigned long long)));
+    CK(cudaMemset(g->counters, 0, 5 * sizeof(unsigned long long)));
     CK(cudaMalloc(&g->best_dev, 2 * sizeof(int64_t)));
   }
   if (g->defer_cap < defer_need) {
@@ -617,6 +640,7 @@ static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
   a.counter = g->counters;
   a.ndefer = g->counters + 1;
   a.stat = g->counters + 2;
+  a.err = (unsigned *)(g->counters + 4);
   a.defer_q = g->defer_q;
   a.wbest = g->wbest;
   a.slab = g->slab;
@@ -1469,9 +1493,13 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
   g->sms = sms > 0 ? sms : 148;
   const int64_t vcap = (int64_t)V + overlay_v(g);
   const int64_t ecap = Em + overlay_e(g);
-  if (vcap > 32768) {
+  // positions are 24-bit in the lane kernels' CP rounds and the group
+  // kernel's records; the ready-set kernel's 3-level bitmap covers 32768
+  // positions, so larger graphs need a topological priority order (checked
+  // after the base is prepared)
+  if (vcap > MAX_VCAP) {
     delete g;
-    return fail(FASTT_EUNSUP, "graphs above 32768 ops (+ split overlay) are not supported yet (V=%d)", V);
+    return fail(FASTT_EUNSUP, "graphs above %d ops (+ split overlay) are not supported (V=%d)", MAX_VCAP, V);
   }
   Base &B = g->base;
   B.V = V;
@@ -1931,7 +1959,8 @@ static fastt_status materialize_base(fastt_graph *g, Base &from, const Cand &c, 
   to.n_live = from.n_live - 1 + (int32_t)(P + c.split_n + S);
   const int64_t newE = from.E + (int64_t)P + (int64_t)P * c.split_n * 2 + (int64_t)S * c.split_n * 2 + S + 16;
   to.rl = raw_layout((int64_t)to.V + overlay_v(g), newE + overlay_e(g), g->G);
-  if (to.rl.vcap > 32768) return fail(FASTT_EUNSUP, "split search grew the graph above 32768 ops");
+  if (to.rl.vcap > MAX_VCAP || (to.rl.vcap > READY_SET_MAX && !from.topo))
+    return fail(FASTT_EUNSUP, "split search grew the graph above %d ops", to.rl.vcap > MAX_VCAP ? MAX_VCAP : READY_SET_MAX);
   CK(cudaMalloc(&to.raw_block, to.rl.total));
   CK(cudaMalloc(&to.raw_dev, sizeof(RawGraph)));
   CK(cudaMemsetAsync(to.raw_block, 0, to.rl.total, st));
@@ -1977,7 +2006,9 @@ fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, 
   int64_t *d_ms, *d_start;
   uint8_t *d_st, *d_place;
   int32_t *d_deq, *d_order;
-  int64_t cap_v = 32768 + 64;
+  // per-op output buffers of a round: the graph grows by at most one split
+  // overlay per accepted split (checked before every round below)
+  int64_t cap_v = std::max<int64_t>(READY_SET_MAX + 64, 2 * cur->rl.vcap);
   CK(cudaMalloc(&d_c, sizeof(Cand) * maxc));
   CK(cudaMalloc(&d_ms, 8 * maxc));
   CK(cudaMalloc(&d_st, maxc));
@@ -2095,9 +2126,10 @@ fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, 
         if (rc == FASTT_OK && bi >= 0 && ms[bi] < ft_old) {
           // the winner's placement / order / start (one more evaluation with outputs)
           vm = cur->rl.vcap;
+          if (vm > cap_v) rc = fail(FASTT_EUNSUP, "split search grew the graph past its output buffers");
           o.vmax = vm;
           CK(cudaMemcpy(d_c, &cs[bi], sizeof(Cand), cudaMemcpyHostToDevice));
-          rc = eval_batch(g, *cur, d_c, 1, flags, st, o);
+          if (rc == FASTT_OK) rc = eval_batch(g, *cur, d_c, 1, flags, st, o);
           if (rc == FASTT_OK) {
             owned.emplace_back();
             Base &nb = owned.back();
@@ -2149,8 +2181,9 @@ fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, 
       if (cs.empty()) continue;
       CK(cudaMemcpy(d_c, cs.data(), sizeof(Cand) * cs.size(), cudaMemcpyHostToDevice));
       vm = cur->rl.vcap;
+      if (vm > cap_v) rc = fail(FASTT_EUNSUP, "split search grew the graph past its output buffers");
       o.vmax = vm;
-      rc = eval_batch(g, *cur, d_c, (int64_t)cs.size(), flags, st, o);
+      if (rc == FASTT_OK) rc = eval_batch(g, *cur, d_c, (int64_t)cs.size(), flags, st, o);
       if (rc != FASTT_OK) {
         cleanup();
         return rc;
@@ -2184,6 +2217,11 @@ fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, 
       CK(cudaMemcpy(border.data(), d_order + (size_t)bi * vm, 4 * vm, cudaMemcpyDeviceToHost));
       cur = &nb;
     }
+  }
+  rc = check_kernel_err(g, st);
+  if (rc != FASTT_OK) {
+    cleanup();
+    return rc;
   }
   out->status = s0;
   out->makespan = s0 == FASTT_CAND_OK ? ft_old : I64MAX;

@@ -49,6 +49,10 @@ constexpr int CW_PCOMM = CARD_HDR + P_IN;  // inline comm values
 constexpr int CW_SUCC = CW_PCOMM + P_IN;   // inline successor positions
 constexpr uint32_t NONE = 0xFFFFFFFFu;
 constexpr int64_t I64MAX = INT64_MAX;
+// graph size envelope: positions fit 24 bits (lane-kernel CP rounds, group
+// kernel records); the ready-set kernel's 3-level bitmap covers 32768
+constexpr int64_t MAX_VCAP = 1 << 23;
+constexpr int64_t READY_SET_MAX = 32768;
 
 // card header words
 enum { CW_DEG = 0, CW_PBASE = 1, CW_SBASE = 2, CW_CPIDX = 3, CW_MEMLO = 4, CW_MEMHI = 5, CW_UID = 6, CW_FLAGS = 7 };
@@ -262,6 +266,9 @@ struct SimArgs {
   int32_t lane_batches;
   int32_t n_slab_slots;
   uint32_t *slot_bm;
+  // set when a ready-set launch meets a graph above READY_SET_MAX positions
+  // (the call then fails with FASTT_EUNSUP)
+  unsigned *err;
 };
 
 // one idle slot [a, b) of a device under INSERT

@@ -240,6 +240,10 @@ __global__ void __launch_bounds__(SIM_BLOCK, TOPO ? SIM_MINB_TOPO : SIM_MINB) k_
         if (a.slot_filter && (pg->topo != 0) != (a.slot_filter == 1)) active = false;
       }
     }
+    if (!TOPO && active && pg->n > (int32_t)READY_SET_MAX) {  // (the bitmap covers READY_SET_MAX positions)
+      active = false;
+      if (a.err && d == 0) atomicOr(a.err, 1u);
+    }
     const uint32_t *__restrict__ card = pg->card;
     const T *__restrict__ costp = (const T *)pg->costp;
     const T *__restrict__ pe_comm = (const T *)pg->pe_comm;

@@ -595,6 +595,10 @@ CONFIGS = {
     "C3": inception_v3,
     "C4": vgg19,
     "C5": bert_large,
+    # C5 with the model replicated once per device (OS-DPOS starts
+    # from a data-parallel graph with one replica per GPU): ~38k ops, past the
+    # ready-set kernel's 32,768 positions (topological priority order)
+    "C5R8": lambda **kw: bert_large(**dict({"R": 8}, **kw)),
 }
 
 

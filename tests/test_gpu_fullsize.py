@@ -171,3 +171,48 @@ def test_c5_insert_sampled():
     for k, (m, s, pk) in enumerate(ref):
         assert (int(res["makespan"][k]), int(res["status"][k])) == (m, s), (k, idx[k])
         assert tuple(int(x) for x in res["peak_mem"][k]) == pk, (k, idx[k])
+
+
+def test_c5r8_above_ready_set_envelope():
+    """BERT-large x 8 replicas (37,921 ops): past the ready-set
+    kernel's 32,768 positions; its priority order is topological (alpha > 0 on
+    every edge), so the lane kernels evaluate it -- sampled against the
+    oracle (BASE, SPLITs, PINs), the sweep against the per-candidate vector"""
+    desc = synth.config("C5R8")
+    assert desc.n_ops > 32768
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    gen = F.gen_params(seed=SEED, pin_k_min=1, pin_k_max=4)
+    n_split = gg.stream_info(gen, flags=F.F_CP_PIN)
+    assert n_split == og.stream_info(flags=O.F_CP_PIN)[0]
+    idx = [0] + list(range(1, n_split + 1, max(1, n_split // 24))) + [n_split + 1 + 7919 * k for k in range(40)]
+    cands = np.concatenate([gg.generate_candidates(gen, i, 1, flags=F.F_CP_PIN) for i in idx])
+    res = gg.schedule_batch(cands, flags=F.F_CP_PIN, peak=True)
+    ref = _oracle_many(og, cands, range(len(cands)), peak=True)
+    for k, (m, s, pk) in enumerate(ref):
+        assert (int(res["makespan"][k]), int(res["status"][k])) == (m, s), (k, idx[k])
+        assert tuple(int(x) for x in res["peak_mem"][k]) == pk, (k, idx[k])
+    n = n_split + 3000
+    best = gg.sweep_best(gen, 0, n, flags=F.F_CP_PIN)
+    assert gg.last_timing()["topo"] == 2
+    allc = gg.generate_candidates(gen, 0, n, flags=F.F_CP_PIN)
+    ms = gg.schedule_batch(allc, flags=F.F_CP_PIN, peak=False)["makespan"].astype(np.int64)
+    k = int(np.lexsort((np.arange(n), ms))[0])
+    assert best == (int(ms[k]), k)
+
+
+def test_non_topological_graph_above_envelope_is_refused():
+    """a graph above 32,768 ops whose priority order is not topological (zero
+    costs on zero-alpha links, R2) would need the ready-set kernel: EUNSUP"""
+    import dataclasses
+    d = synth.config("C5R8")
+    V = d.n_ops
+    cost = d.cost.copy()
+    cost[::7] = 0  # zero-cost ops on free links: equal ranks along their edges ...
+    rev = lambda a: np.ascontiguousarray(a[::-1])  # ... and ids reversed, so the id tie-break goes against the edges
+    d = dataclasses.replace(d, cost=rev(cost), mem=rev(d.mem), param=rev(d.param), split_mask=rev(d.split_mask),
+                            src=(V - 1 - np.asarray(d.src)).astype(np.asarray(d.src).dtype),
+                            dst=(V - 1 - np.asarray(d.dst)).astype(np.asarray(d.dst).dtype),
+                            alpha=np.zeros_like(d.alpha), beta=np.zeros_like(d.beta), op_type=None)
+    with pytest.raises(F.FasttError) as e:
+        F.Graph(d)
+    assert e.value.code == F.EUNSUP
