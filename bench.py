@@ -96,9 +96,9 @@ def alu_peak_measured():
 
 def ncu_current():
     """pipe / issue / DRAM fractions of the committed ncu capture of the main
-    sweep launch (profiles/ncu_k_sim_lane_current.json)"""
+    sweep launch (profiles/ncu_sweep_kernel_current.json)"""
     try:
-        with open(os.path.join(ROOT, "profiles", "ncu_k_sim_lane_current.json")) as f:
+        with open(os.path.join(ROOT, "profiles", "ncu_sweep_kernel_current.json")) as f:
             return json.load(f)
     except Exception:
         return None
@@ -370,7 +370,8 @@ def main():
     else:
         roof = {"bound": "hbm", "achieved": hbm_gbs, "peak": peak, "unit": "GB/s", "frac": hbm_gbs / peak,
                 "traffic": traffic, "peak_source": peak_src, "bytes_per_candidate": bpc}
-    roof.update({"kernel": ("k_sim_lane" if lane else "k_sim") + "<uint32_t> (sweep launch)",
+    pk = lane and g.time_bits == 32 and int(len(desc.alpha)) == 1
+    roof.update({"kernel": ("k_lane_pk<GSH=3, EX, MM=0>" if pk else "k_sim_lane" if lane else "k_sim") + " (sweep launch)",
                  "candidates_per_launch": fast, "launch_ms": sim_ms, "prep_ms_per_step": prep_ms})
     launches = sum(x["launches"] for x in tms)
 
@@ -407,7 +408,9 @@ def main():
         e2e = {"value": world * n / (e2e_ms / 1000.0), "unit": UNIT, "h2d_bytes_per_step": int(32 * n),
                "d2h_bytes_per_step": int(n * (8 + 1 + 8 * G)), "ms_per_step": e2e_ms,
                "api": "fastt_schedule_batch (host pinned buffers; makespan, status, per-device peak memory)",
-               "argmin_local_index": i, "kernel": "k_sim_lane" if g.last_timing()["topo"] == 2 else "k_sim"}
+               "argmin_local_index": i,
+               "kernel": ("k_lane_pk<MM=1>" if g.time_bits == 32 and len(desc.alpha) == 1 else "k_sim_lane")
+               if g.last_timing()["topo"] == 2 else "k_sim"}
 
     # the other paper-shaped configs (SURVEY 8(d) C1-C4, and C5R8 = BERT-large
     # x 8 replicas, 37,921 ops): one sweep each,
@@ -436,7 +439,8 @@ def main():
             configs[name] = {"V": d2.n_ops, "E": d2.n_edges, "G": d2.n_devices, "candidates": ncand,
                              "time_bits": g2.time_bits, "caps": bool((d2.cap < synth.INT64_MAX).any()),
                              "candidates_per_s": cps, "ops_per_s": cps * d2.n_ops, "ms_per_sweep": ms2,
-                             "kernel": "k_sim_lane" if tm2["topo"] == 2 else "k_sim",
+                             "kernel": ("k_lane_pk" if g2.time_bits == 32 and len(d2.alpha) == 1 else "k_sim_lane")
+                             if tm2["topo"] == 2 else "k_sim",
                              "deferred_to_prep": tm2["deferred"]}
             del g2
 

@@ -1,5 +1,5 @@
 """Condense an ncu summary of the main sweep launch (tools/ncu_summary.py
-output) into profiles/ncu_k_sim_lane_current.json, the fractions bench.py
+output) into profiles/ncu_sweep_kernel_current.json, the fractions bench.py
 reports under roofline.ncu: issue, ALU pipe, L1/shared LSU wavefronts, DRAM,
 and the DRAM bytes per candidate (the roofline's `traffic`).
 usage: ncu_current.py <summary.json> <candidates in the captured launch> <tag>"""
@@ -44,6 +44,6 @@ out["dram_frac"] = out["dram_gbs"] / hbm
 out["dram_peak_gbs"] = hbm
 fr = {k: out[k] for k in ("issue_active_frac", "alu_pipe_frac", "lsu_wavefronts_frac", "dram_frac")}
 out["binding"] = max(fr, key=fr.get)
-with open(os.path.join(root, "profiles", "ncu_k_sim_lane_current.json"), "w") as f:
+with open(os.path.join(root, "profiles", "ncu_sweep_kernel_current.json"), "w") as f:
     json.dump(out, f, indent=1)
 print(json.dumps(out, indent=1))

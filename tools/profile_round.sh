@@ -15,11 +15,11 @@ nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o gpurun_out/alu_peak tools/al
     --clock-control none -c 5 --csv --log-file gpurun_out/${tag}_alu_peak_ncu.csv ./gpurun_out/alu_peak > /dev/null 2>&1
 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/${tag}_launches.csv \
     python bench.py --steps 1 --warmup 3 --candidates 200000 --no-e2e --no-cpu --no-configs > gpurun_out/${tag}_ncu_bench.log 2>&1
-# the main sweep launch: the lane-per-candidate kernel (k_sim_lane) over 300k PIN candidates
-ncu --set full --clock-control none --import-source on -k regex:k_sim_lane -c 1 -o gpurun_out/${tag}_k_sim_lane -f \
+# the main sweep launch: the packed-key lane kernel (k_lane_pk) over 300k PIN candidates
+ncu --set full --clock-control none --import-source on -k regex:k_lane_pk -c 1 -o gpurun_out/${tag}_k_lane_pk -f \
     python tools/ncu_sim.py 300000 > gpurun_out/${tag}_ncu_full.log 2>&1
-ncu -i gpurun_out/${tag}_k_sim_lane.ncu-rep --page raw --csv > gpurun_out/${tag}_k_sim_lane_raw.csv 2>/dev/null
-ncu -i gpurun_out/${tag}_k_sim_lane.ncu-rep --page source --csv --print-source sass > gpurun_out/${tag}_k_sim_lane_source.csv 2>/dev/null
+ncu -i gpurun_out/${tag}_k_lane_pk.ncu-rep --page raw --csv > gpurun_out/${tag}_k_lane_pk_raw.csv 2>/dev/null
+ncu -i gpurun_out/${tag}_k_lane_pk.ncu-rep --page source --csv --print-source sass > gpurun_out/${tag}_k_lane_pk_source.csv 2>/dev/null
 # the preparation pipeline's heaviest kernels (split candidates)
 ncu --set full --clock-control none --import-source on -k regex:"k_rank|k_sort|k_cards_hdr|k_cards_pred|k_cp" -c 5 -o gpurun_out/${tag}_prep -f \
     python bench.py --steps 1 --warmup 1 --candidates 20000 --no-e2e --no-cpu --no-configs > gpurun_out/${tag}_ncu_prep.log 2>&1
