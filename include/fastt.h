@@ -78,6 +78,10 @@ enum {
   FASTT_F_IN_DEVICE = 1u << 3,     /* candidate input pointer is a device pointer */
   FASTT_F_TIMING = 1u << 4,        /* record CUDA events around the kernels of this call (fastt_last_timing) */
   FASTT_F_SPLIT_BEST = 1u << 5,    /* fastt_split_search: best-improvement rounds */
+  FASTT_F_SPLIT_MULTI = 1u << 7,   /* fastt_split_search: best-improvement rounds with multi-split candidates
+                                      (reading R27): each round also evaluates C_j = the best
+                                      split of each of the j best-improving ops, applied in rank order
+                                      (j = 2..4), and accepts the best C_j (ties: fewer splits) */
   FASTT_F_MEM_LIVE = 1u << 6       /* liveness memory (reading R24): an op's parameters stay on
                                       its device; its output (mem - param) is held from the step it is dequeued
                                       until the step its last consumer is dequeued.  The feasibility test of

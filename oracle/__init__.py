@@ -32,6 +32,7 @@ DIM_BATCH, DIM_CHANNEL = 0, 1
 F_CP_PIN = 1
 F_POLICY_INSERT = 2
 F_MEM_LIVE = 64
+F_SPLIT_MULTI = 128  # best-improvement split search with multi-split candidates (R27)
 GEN_POW2, GEN_SUBSETS = 1, 2
 
 CAND_DTYPE = np.dtype(
@@ -215,7 +216,7 @@ class OracleGraph:
         n = lib().fastt_ref_cp(self.h, _p(cp))
         return cp[:n]
 
-    def split_search(self, flags=0, pow2_only=False, out_cap=None, best_improvement=False):
+    def split_search(self, flags=0, pow2_only=False, out_cap=None, best_improvement=False, multi=False):
         cap = out_cap or (self.V + 64 * (self.G + 64) + 1024)
         sp_n = np.zeros(1, np.int32)
         spc = 4096
@@ -228,15 +229,15 @@ class OracleGraph:
         start = np.zeros(cap, np.int64)
         ms = np.zeros(1, np.int64)
         st = np.zeros(1, np.uint8)
-        fn = lib().fastt_ref_split_search_bi if best_improvement else lib().fastt_ref_split_search
-        rc = fn(self.h, flags, int(bool(pow2_only)), spc, _p(sp_n), _p(sp_op), _p(sp_dim),
+        fn = lib().fastt_ref_split_search_bi if (best_improvement or multi) else lib().fastt_ref_split_search
+        rc = fn(self.h, flags | (F_SPLIT_MULTI if multi else 0), int(bool(pow2_only)), spc, _p(sp_n), _p(sp_op), _p(sp_dim),
                 _p(sp_cnt), cap, _p(nfin), _p(place), _p(order), _p(start), _p(ms), _p(st))
         if rc != 0:
             raise OracleError(rc)
         n = int(sp_n[0])
         nf = int(nfin[0])
         if nf > cap:
-            return self.split_search(flags, pow2_only, out_cap=nf + 16, best_improvement=best_improvement)
+            return self.split_search(flags, pow2_only, out_cap=nf + 16, best_improvement=best_improvement, multi=multi)
         return {"sp": [(int(sp_op[q]), int(sp_dim[q]), int(sp_cnt[q])) for q in range(n)], "n_ops_final": nf,
                 "placement": place[:nf], "order": order[:nf], "start": start[:nf], "makespan": int(ms[0]),
                 "status": int(st[0])}

@@ -946,7 +946,17 @@ int32_t fastt_ref_split_search(const fo_graph *g0, uint32_t flags, int32_t pow2_
  * n) of every not-yet-split op of the list on the current graph and accepts
  * the one with the smallest FT (ties: list order, dim asc, n asc) if it is
  * strictly better; stops when no split improves.  (A variant of Alg. 2,
- * the paper stops at the first op that does not improve.) */
+ * the paper stops at the first op that does not improve.)
+ *
+ * With FO_F_SPLIT_MULTI (reading R27, multi-split candidates): each op's
+ * best variant (smallest FT, ties dim asc, n asc) among those that improve;
+ * the improving ops ranked by (FT asc, list order); the candidates C_j =
+ * the best variants of the first j ranked ops applied in rank order (each
+ * SplitOperation on the graph the previous one produced; ops keep their ids,
+ * R13), j = 1 .. min(4, #improving); the round accepts the C_j of smallest
+ * FT (ties: smaller j) -- C_1 improves by construction -- and marks its ops
+ * split. */
+#define FO_F_SPLIT_MULTI (1u << 7)
 int32_t fastt_ref_split_search_bi(const fo_graph *g0, uint32_t flags, int32_t pow2_only, int32_t sp_cap,
                                   int32_t *sp_n, int32_t *sp_op, uint8_t *sp_dim, uint8_t *sp_cnt,
                                   int32_t out_cap, int32_t *n_ops_final, uint8_t *placement, int32_t *order,
@@ -970,7 +980,13 @@ int32_t fastt_ref_split_search_bi(const fo_graph *g0, uint32_t flags, int32_t po
   uint8_t *done = calloc((size_t)nl + 1, 1);
   int ns[FO_MAXG];
   int nns = fo_split_ns(G, pow2_only, ns);
+  const int multi = (flags & FO_F_SPLIT_MULTI) != 0;
+  flags &= ~FO_F_SPLIT_MULTI;
+  /* per list op: FT, dim and n of its best improving variant this round */
+  int64_t *oft = malloc(sizeof(int64_t) * ((size_t)nl + 1));
+  int *odim = malloc(sizeof(int) * ((size_t)nl + 1)), *on = malloc(sizeof(int) * ((size_t)nl + 1));
   for (;;) {
+    for (int32_t li = 0; li < nl; li++) oft[li] = FO_INF;
     int64_t bft = FO_INF;
     int32_t bli = -1;
     int bdim = -1, bn = -1;
@@ -990,6 +1006,11 @@ int32_t fastt_ref_split_search_bi(const fo_graph *g0, uint32_t flags, int32_t po
           int64_t *rk = malloc(sizeof(int64_t) * ((size_t)sv->V + 1));
           fo_dpos(sv, NULL, fo_all_devices(sv->G), flags, rk, &r);
           free(rk);
+          if (r.status == FO_CAND_OK && r.makespan < oft[li]) {
+            oft[li] = r.makespan;
+            odim[li] = dim;
+            on[li] = ns[q];
+          }
           if (r.status == FO_CAND_OK && r.makespan < bft) {
             if (bg) { fo_graph_free(bg); fo_result_free(&br); }
             bg = sv; br = r; bft = r.makespan; bli = li; bdim = dim; bn = ns[q];
@@ -1004,15 +1025,66 @@ int32_t fastt_ref_split_search_bi(const fo_graph *g0, uint32_t flags, int32_t po
       if (bg) { fo_graph_free(bg); fo_result_free(&br); }
       break;
     }
-    if (*sp_n < sp_cap) { sp_op[*sp_n] = list[bli]; sp_dim[*sp_n] = (uint8_t)bdim; sp_cnt[*sp_n] = (uint8_t)bn; }
-    (*sp_n)++;
-    done[bli] = 1;
+    /* the accepted candidate: C_1 (the single best split), or a multi-split C_j */
+    int32_t acc_li[4] = {bli, -1, -1, -1};
+    int nacc = 1;
+    if (multi) {
+      /* the improving ops ranked by (FT asc, list order asc); the first is bli
+         (the same order and tie rule as the single best) */
+      int32_t rk_li[4];
+      int nrk = 0;
+      for (int32_t li = 0; li < nl; li++) {
+        if (done[li] || oft[li] >= ft_old) continue;
+        int pos = nrk;
+        while (pos > 0 && oft[rk_li[pos - 1]] > oft[li]) pos--;
+        if (pos >= 4) continue;
+        for (int t = (nrk < 4 ? nrk : 3); t > pos; t--) rk_li[t] = rk_li[t - 1];
+        rk_li[pos] = li;
+        if (nrk < 4) nrk++;
+      }
+      /* C_j's graph: C_{j-1}'s graph with the j-th ranked op's best split */
+      fo_graph *cg[5] = {NULL, bg, NULL, NULL, NULL};
+      for (int j = 2; j <= nrk; j++) {
+        const int32_t li = rk_li[j - 1];
+        if (fo_split_view(cg[j - 1], list[li], odim[li], on[li], &cg[j]) != FO_OK) {
+          cg[j] = NULL;
+          break;
+        }
+        fo_result r;
+        fo_result_alloc(&r, cg[j]->V, G);
+        int64_t *rkj = malloc(sizeof(int64_t) * ((size_t)cg[j]->V + 1));
+        fo_dpos(cg[j], NULL, fo_all_devices(cg[j]->G), flags, rkj, &r);
+        free(rkj);
+        if (r.status == FO_CAND_OK && r.makespan < bft) {  /* (ties: the smaller j stays) */
+          fo_result_free(&br);
+          br = r;
+          bft = r.makespan;
+          nacc = j;
+        } else {
+          fo_result_free(&r);
+        }
+      }
+      for (int j = 1; j <= 4; j++)
+        if (cg[j] && j != nacc) fo_graph_free(cg[j]);
+      bg = cg[nacc];
+      for (int t = 0; t < nacc; t++) acc_li[t] = rk_li[t];
+    }
+    for (int t = 0; t < nacc; t++) {
+      const int32_t li = acc_li[t];
+      const int dim = multi ? odim[li] : bdim, n = multi ? on[li] : bn;
+      if (*sp_n < sp_cap) { sp_op[*sp_n] = list[li]; sp_dim[*sp_n] = (uint8_t)dim; sp_cnt[*sp_n] = (uint8_t)n; }
+      (*sp_n)++;
+      done[li] = 1;
+    }
     ft_old = bft;
     if (cur != g0) fo_graph_free(cur);
     cur = bg;
     fo_result_free(&best_r);
     best_r = br;
   }
+  free(oft);
+  free(odim);
+  free(on);
   *makespan = ft_old;
   *status = FO_CAND_OK;
   *n_ops_final = cur->V;

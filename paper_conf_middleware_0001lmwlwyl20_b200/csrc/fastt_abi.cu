@@ -1992,7 +1992,8 @@ fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, 
   fastt_graph *g = (fastt_graph *)gc_;
   if (!g || !out) return fail(FASTT_EINVAL, "NULL argument");
   const uint32_t flags = flags_of(opts) & (FASTT_F_CP_PIN | FASTT_F_POLICY_INSERT | FASTT_F_MEM_LIVE);
-  const bool best_mode = (flags_of(opts) & FASTT_F_SPLIT_BEST) != 0;
+  const bool multi_mode = (flags_of(opts) & FASTT_F_SPLIT_MULTI) != 0;
+  const bool best_mode = (flags_of(opts) & FASTT_F_SPLIT_BEST) != 0 || multi_mode;
   memset(out, 0, sizeof *out);
   std::lock_guard<std::mutex> lk(g->mu);
   Dev guard(g->dev);
@@ -2123,6 +2124,80 @@ fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, 
         int bi = -1;
         for (size_t q = 0; rc == FASTT_OK && q < cs.size(); q++)
           if (sts[q] == FASTT_CAND_OK && (bi < 0 || ms[q] < ms[bi])) bi = (int)q;
+        // R27 multi-split candidates: each op's best improving variant (the
+        // first minimum in (dim, n) order), the ops ranked by (makespan, list
+        // order), C_j = the first j ranked splits applied in rank order
+        // (materialised one after the other), the C_j of smallest makespan
+        // (ties: smaller j) is accepted -- C_1 is the single best (bi)
+        if (multi_mode && rc == FASTT_OK && bi >= 0 && ms[bi] < ft_old) {
+          std::vector<int> bestq(list.size(), -1), rk;
+          for (size_t q = 0; q < cs.size(); q++) {
+            const size_t li = li_of[q];
+            if (sts[q] == FASTT_CAND_OK && ms[q] < ft_old && (bestq[li] < 0 || ms[q] < ms[bestq[li]])) bestq[li] = (int)q;
+          }
+          for (size_t li = 0; li < list.size(); li++)
+            if (bestq[li] >= 0) rk.push_back(bestq[li]);
+          std::stable_sort(rk.begin(), rk.end(), [&](int x, int y) { return ms[x] < ms[y]; });  // (list order kept)
+          if (rk.size() > 4) rk.resize(4);
+          if (rk.size() >= 2) {
+            std::vector<Base *> chain(rk.size() + 1, nullptr);
+            std::vector<int64_t> ftj(rk.size() + 1, I64MAX);
+            chain[0] = cur;
+            ftj[1] = ms[rk[0]];
+            int bj = 1;
+            for (size_t j = 1; j <= rk.size() && rc == FASTT_OK; j++) {
+              owned.emplace_back();
+              chain[j] = &owned.back();
+              rc = materialize_base(g, *chain[j - 1], cs[rk[j - 1]], *chain[j], st);
+              if (rc != FASTT_OK || j == 1) continue;
+              DevOut jo;
+              jo.makespan = d_rms;
+              jo.status = d_rst;
+              jo.vmax = chain[j]->rl.vcap;
+              CK(cudaMemcpy(d_round, &base, sizeof base, cudaMemcpyHostToDevice));
+              rc = eval_batch(g, *chain[j], d_round, 1, flags, st, jo);
+              int64_t m = I64MAX;
+              uint8_t s1 = 1;
+              if (rc == FASTT_OK && (cudaMemcpy(&m, d_rms, 8, cudaMemcpyDeviceToHost) != cudaSuccess ||
+                                     cudaMemcpy(&s1, d_rst, 1, cudaMemcpyDeviceToHost) != cudaSuccess))
+                rc = fail(FASTT_ECUDA, "download a multi-split result");
+              if (rc == FASTT_OK && s1 == FASTT_CAND_OK) {
+                ftj[j] = m;
+                if (m < ftj[bj]) bj = (int)j;
+              }
+            }
+            if (rc == FASTT_OK && bj >= 2) {  // accept C_bj: outputs of its graph
+              for (size_t j = 1; j <= rk.size(); j++)  // (each base is a copy: the others can go)
+                if (j != (size_t)bj) chain[j]->release();
+              vm = chain[bj]->rl.vcap;
+              if (vm > cap_v) rc = fail(FASTT_EUNSUP, "split search grew the graph past its output buffers");
+              o.vmax = vm;
+              CK(cudaMemcpy(d_c, &base, sizeof base, cudaMemcpyHostToDevice));
+              if (rc == FASTT_OK) rc = eval_batch(g, *chain[bj], d_c, 1, flags, st, o);
+              if (rc == FASTT_OK) {
+                ft_old = ftj[bj];
+                for (int j = 1; j <= bj; j++) {
+                  const Cand &cj = cs[rk[j - 1]];
+                  done[li_of[rk[j - 1]]] = 1;
+                  sp_op.push_back(cj.split_op);
+                  sp_dim.push_back(cj.split_dim);
+                  sp_n.push_back(cj.split_n);
+                }
+                vfinal = chain[bj]->V;
+                bplace.resize(vm);
+                bstart.resize(vm);
+                border.resize(vm);
+                CK(cudaMemcpy(bplace.data(), d_place, vm, cudaMemcpyDeviceToHost));
+                CK(cudaMemcpy(bstart.data(), d_start, 8 * vm, cudaMemcpyDeviceToHost));
+                CK(cudaMemcpy(border.data(), d_order, 4 * vm, cudaMemcpyDeviceToHost));
+                cur = chain[bj];
+                continue;
+              }
+            } else if (rc == FASTT_OK) {  // C_1 wins: drop the chain beyond it (C_1 is re-made below)
+              for (size_t j = 1; j <= rk.size(); j++) chain[j]->release();
+            }
+          }
+        }
         if (rc == FASTT_OK && bi >= 0 && ms[bi] < ft_old) {
           // the winner's placement / order / start (one more evaluation with outputs)
           vm = cur->rl.vcap;

@@ -70,6 +70,7 @@ SYMBOLS = ["fastt_load_graph", "fastt_free_graph", "fastt_graph_info", "fastt_ra
 F_TIMING = 16
 F_SPLIT_BEST = 32
 F_MEM_LIVE = 64
+F_SPLIT_MULTI = 128
 
 _lib = None
 
@@ -307,9 +308,9 @@ class Graph:
                 "ms_sim": float(t.ms_sim), "ms_prep": float(t.ms_prep), "ms_total": float(t.ms_total),
                 "topo": int(t.topo), "warp_steps": int(t.warp_steps), "lane_steps": int(t.lane_steps)}
 
-    def split_search(self, flags=0, n_pow2_only=False, stream=None, best_improvement=False):
+    def split_search(self, flags=0, n_pow2_only=False, stream=None, best_improvement=False, multi=False):
         r = fastt_split_result()
-        o = _opts(flags | (F_SPLIT_BEST if best_improvement else 0), stream)
+        o = _opts(flags | (F_SPLIT_BEST if best_improvement else 0) | (F_SPLIT_MULTI if multi else 0), stream)
         _check(lib().fastt_split_search(self.h, C.byref(o), 1 if n_pow2_only else 0, C.byref(r)))
         try:
             n = r.n_splits

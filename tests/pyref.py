@@ -339,6 +339,53 @@ def split_search_best(g: PG, cp_pin=False, pow2_only=False):
             "n_ops_final": cur.V}
 
 
+def split_search_multi(g: PG, cp_pin=False, pow2_only=False):
+    """Reading R27 (NEXT N2 multi-split candidates, on top of R23): per round,
+    every op's best improving split (smallest makespan, ties dim, n); the
+    improving ops ranked by (makespan, list order); candidates C_j = the
+    first j ranked ops' best splits applied in rank order, j = 1..min(4, k);
+    accept the C_j of smallest makespan (ties: smaller j) -- written from the
+    definition: each C_j built from scratch from the round's graph."""
+    r = dpos(g, cp_pin=cp_pin)
+    if r["status"] != 0:
+        return {"sp": [], "makespan": INF, "status": r["status"]}
+    lst = split_list(g, r["place"])
+    cur, ft_old, best_r, sp, done, rounds = g, r["makespan"], r, [], set(), []
+    while True:
+        per_op = {}
+        for li, op in enumerate(lst):
+            if op in done or not any(cur.smask[op] & (1 << dim) for dim in (0, 1)):
+                continue
+            best = None
+            for dim in (0, 1):
+                if cur.smask[op] & (1 << dim):
+                    for n in split_counts(g.G, pow2_only):
+                        rr = dpos(split_view(cur, op, dim, n), cp_pin=cp_pin)
+                        if rr["status"] == 0 and (best is None or rr["makespan"] < best[0]):
+                            best = (rr["makespan"], dim, n)
+            if best is not None and best[0] < ft_old:
+                per_op[li] = best
+        if not per_op:
+            break
+        ranked = sorted(per_op, key=lambda li: (per_op[li][0], li))[:4]
+        choice = None
+        for j in range(1, len(ranked) + 1):
+            gj = cur
+            for li in ranked[:j]:
+                gj = split_view(gj, lst[li], per_op[li][1], per_op[li][2])
+            rr = dpos(gj, cp_pin=cp_pin)
+            if rr["status"] == 0 and (choice is None or rr["makespan"] < choice[0]):
+                choice = (rr["makespan"], j, gj, rr)
+        ms, j, gj, rr = choice
+        for li in ranked[:j]:
+            sp.append((lst[li], per_op[li][1], per_op[li][2]))
+            done.add(lst[li])
+        rounds.append(j)
+        cur, ft_old, best_r = gj, ms, rr
+    return {"sp": sp, "makespan": ft_old, "status": 0, "place": best_r["place"], "start": best_r["start"],
+            "n_ops_final": cur.V, "rounds": rounds}
+
+
 # ---------------------------------------------------- the sweep stream (R21)
 
 def splitmix64(state):

@@ -282,6 +282,37 @@ def test_split_search_best_configs(name):
     assert (a["placement"] == b["placement"]).all() and (a["order"] == b["order"]).all()
 
 
+# seeds whose multi-split search (R27) accepts a C_j with j >= 2 in some round
+# (tests/test_oracle_alg2.py BI_DAGS: random_dag(s, V=40, G=4, max_in=2))
+MULTI_SEEDS = [4, 13, 21, 32, 34, 39, 116, 122, 214, 1, 3] + list(range(8))
+
+
+@pytest.mark.parametrize("seed", MULTI_SEEDS)
+def test_split_search_multi_random(seed):
+    """NEXT N2 multi-split candidates (R27): the GPU's rounds (C_j
+    materialised split after split, DPOS of each) equal the oracle's SP list,
+    makespan and per-op outputs"""
+    desc = synth.random_dag(seed, V=40, G=4, caps="none", max_in=2)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    for flags in (0, F.F_CP_PIN):
+        a = gg.split_search(flags=flags, multi=True)
+        b = og.split_search(flags=flags, multi=True)
+        assert a["sp"] == b["sp"] and a["makespan"] == b["makespan"] and a["n_ops_final"] == b["n_ops_final"]
+        assert (a["placement"] == b["placement"]).all()
+        assert (a["start"] == b["start"]).all()
+        assert (a["order"] == b["order"]).all()
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C4"])
+def test_split_search_multi_configs(name):
+    desc = synth.config(name)
+    gg, og = F.Graph(desc), O.OracleGraph(desc)
+    a = gg.split_search(flags=F.F_CP_PIN, n_pow2_only=(name == "C4"), multi=True)
+    b = og.split_search(flags=O.F_CP_PIN, pow2_only=(name == "C4"), multi=True)
+    assert a["sp"] == b["sp"] and a["makespan"] == b["makespan"]
+    assert (a["placement"] == b["placement"]).all() and (a["order"] == b["order"]).all()
+
+
 @pytest.mark.parametrize("name", ["C3", "C5"])
 def test_split_search_best_large_properties(name):
     """C3/C5 best-improvement is minutes of oracle time, so check properties:

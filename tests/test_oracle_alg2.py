@@ -138,6 +138,42 @@ def test_split_search_best_matches_independent(k):
                 assert ss["placement"][i] == dv and ss["start"][i] == ps["start"][i]
 
 
+@pytest.mark.parametrize("k", range(len(BI_DAGS)))
+def test_split_search_multi_matches_independent(k):
+    """Multi-split candidates (R27, NEXT N2): every round's C_j -- the first
+    j ranked improving ops' best splits, applied in rank order -- equals the
+    independent implementation, which rebuilds each C_j from the round's graph
+    (the oracle grows C_j from C_{j-1}'s graph)."""
+    d = BI_DAGS[k]
+    g = O.OracleGraph(d)
+    pg = PR.PG.from_desc(d)
+    for flags, cp in ((0, False), (O.F_CP_PIN, True)):
+        ss = g.split_search(flags=flags, multi=True)
+        ps = PR.split_search_multi(pg, cp_pin=cp)
+        assert [tuple(x) for x in ss["sp"]] == ps["sp"]
+        assert ss["makespan"] == ps["makespan"]
+        if ps["status"] == 0:
+            assert ss["n_ops_final"] == ps["n_ops_final"]
+            for i, dv in ps["place"].items():
+                assert ss["placement"][i] == dv and ss["start"][i] == ps["start"][i]
+
+
+def test_split_search_multi_properties():
+    """R27 on the best-improvement DAGs: never worse than the initial DPOS,
+    and some rounds accept a multi-split candidate (>= 2 splits at once), so
+    the combination path of the oracle is exercised by the comparison above"""
+    multi_rounds = 0
+    for d in BI_DAGS:
+        g = O.OracleGraph(d)
+        base = g.schedule(O.make_cand(O.KIND_BASE), flags=0)["makespan"]
+        m = g.split_search(flags=0, multi=True)
+        assert m["makespan"] <= base
+        ps = PR.split_search_multi(PR.PG.from_desc(d))
+        assert sum(ps["rounds"]) == len(m["sp"])
+        multi_rounds += sum(1 for j in ps["rounds"] if j >= 2)
+    assert multi_rounds >= 1
+
+
 DPOS_DAGS = _dags(40, 2, 80, 7500)
 
 
