@@ -277,6 +277,11 @@ struct fastt_graph {
   size_t sim_smem = 0;
   void *slab = nullptr;
   void *gap = nullptr;  // INSERT idle-slot pools, one per candidate slot (lazy)
+  void *gap_lane = nullptr;  // INSERT idle-slot arrays of the lane kernel (lazy)
+  int32_t gap_cap = 0;       // idle slots per lane and device
+  int ins_lane_grid = 0;
+  bool use_lane_ins = true;  // FASTT_NO_LANE_INS=1 keeps INSERT on the group kernel (A/B parity)
+  int64_t ins_cap_env = 0;   // FASTT_INS_CAP=<slots>: lower the per-device capacity (tests of the deferral)
   int64_t gap_stride = 0;
   int ins_grid = 0;
   int64_t *wbest = nullptr, *best_dev = nullptr;
@@ -528,9 +533,12 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     cudaFree(g->slab);
     cudaFree(g->wbest);
     cudaFree(g->gap);
+    cudaFree(g->gap_lane);
     g->slab = nullptr;
     g->wbest = nullptr;
     g->gap = nullptr;
+    g->gap_lane = nullptr;
+    g->ins_lane_grid = 0;
     const int gsh = gshift_of(g->G);
     const int cpw = 32 >> gsh;
     // (the ready-set bitmap: the ready-set kernel runs on at most
@@ -580,6 +588,28 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     }
     g->ins_grid = (int)ig;
   }
+  if ((flags & FASTT_F_POLICY_INSERT) && !g->gap_lane && g->use_lane_ins) {
+    // INSERT on the lane kernel: per lane and device gap_cap idle slots (a
+    // device holding more is deferred to the group kernel), for as many
+    // resident blocks as a third of the free memory allows
+    const int G = g->G, GP = 1 << gshift_of(G);
+    int64_t cap = std::min<int64_t>(g->sim_ncap + 1, 2 * ((g->sim_ncap + G - 1) / G) + 256);
+    if (g->ins_cap_env > 0) cap = std::min<int64_t>(cap, g->ins_cap_env);
+    const size_t rec = B.tbits == 32 ? sizeof(GapSlot<uint32_t>) : sizeof(GapSlot<uint64_t>);
+    const size_t per_block = (size_t)LANE_BLOCK * GP * (size_t)cap * rec;
+    size_t fr = 0, tot = 0;
+    CK(cudaMemGetInfo(&fr, &tot));
+    int64_t ig = std::min<int64_t>(g->sim_grid_lane[0][0], (int64_t)(fr / 3 / per_block));
+    if (ig > g->sms) ig -= ig % g->sms;
+    if (ig >= 1 && cudaMalloc(&g->gap_lane, (size_t)ig * per_block) == cudaSuccess) {
+      g->gap_cap = (int32_t)cap;
+      g->ins_lane_grid = (int)ig;
+    } else {
+      cudaGetLastError();
+      g->gap_lane = nullptr;
+      g->ins_lane_grid = 0;  // (INSERT stays on the group kernel)
+    }
+  }
   if (!g->counters) {
     CK(cudaMalloc(&g->counters, 5 * sizeof(unsigned long long)));
     CK(cudaMemset(g->counters, 0, 5 * sizeof(unsigned long long)));
@@ -600,14 +630,20 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
 // the ready-set variant (slots may differ).
 static void main_shape(fastt_graph *g, const Base &B, SimArgs &a, int &grid, size_t &smem) {
   const bool topo = g->use_topo && B.topo && a.mode != 2;
-  // the lane kernel covers makespan (+ per-device peak, + memory caps)
-  // without per-op outputs, liveness memory or INSERT
-  const bool lane = topo && g->use_lane && !a.live_mem && !a.ins && !a.out.place && !a.out.start && !a.out.deq &&
+  // the lane kernel covers makespan (+ per-device peak, + memory caps, or
+  // INSERT without memory) without per-op outputs or liveness memory
+  const int mm = a.cap_check ? 2 : (a.out.peak ? 1 : 0);
+  const bool ins_ok = !a.ins || (mm == 0 && g->gap_lane != nullptr && g->ins_lane_grid > 0);
+  const bool lane = topo && g->use_lane && !a.live_mem && ins_ok && !a.out.place && !a.out.start && !a.out.deq &&
                     a.snap_mode != 1;
   g->last_topo = lane ? 2 : topo ? 1 : 0;
   a.lane = lane;
-  a.lane_mm = a.cap_check ? 2 : (a.out.peak ? 1 : 0);
-  if (lane) {
+  a.lane_mm = mm;
+  if (lane && a.ins) {
+    a.topo = 1;
+    grid = g->ins_lane_grid;
+    smem = 0;
+  } else if (lane) {
     a.topo = 1;
     // (the packed-key variant: 32-bit time, one link class, keys prepared)
     const bool pk = B.tbits == 32 && g->K == 1 && a.costk != nullptr && a.pk_lim > 0;
@@ -667,6 +703,8 @@ static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
     a.gap = g->gap;
     a.gap_stride = g->gap_stride;
     a.ins_grid = g->ins_grid;
+    a.gap_lane = g->gap_lane;
+    a.gap_cap = g->gap_cap;
   }
   return a;
 }
@@ -810,7 +848,7 @@ static void launch_slots(fastt_graph *g, SimArgs b, int tbits, int nc, cudaStrea
   b.mode = 2;
   b.stat = nullptr;  // (the step counts are the main launch's)
   const int per_block = (g->sim_block / 32) * g->sim_cpw;
-  if (g->use_topo && b.lane) {
+  if (g->use_topo && b.lane && !b.ins) {
     // makespan-only evaluation without memory tracking: the multi-graph lane
     // kernel (one slot per lane, one warp per block) for topological slots
     b.lane = 2;
@@ -1473,6 +1511,10 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     g->use_pk = !(e && e[0] == '1');
     e = getenv("FASTT_NO_PK_TMA");
     g->use_pk_tma = !(e && e[0] == '1');
+    e = getenv("FASTT_NO_LANE_INS");
+    g->use_lane_ins = !(e && e[0] == '1');
+    e = getenv("FASTT_INS_CAP");
+    if (e && e[0]) g->ins_cap_env = std::max(1ll, atoll(e));
     e = getenv("FASTT_NO_OVERLAP");
     g->use_overlap = !(e && e[0] == '1');
     e = getenv("FASTT_LANE_BATCHES");
@@ -1571,6 +1613,7 @@ void fastt_free_graph(fastt_graph *g) {
     cudaFree(g->slot_index);
     cudaFree(g->slab);
     cudaFree(g->gap);
+    cudaFree(g->gap_lane);
     cudaFree(g->wbest);
     cudaFree(g->best_dev);
     cudaFree(g->counters);

@@ -269,6 +269,9 @@ struct SimArgs {
   // set when a ready-set launch meets a graph above READY_SET_MAX positions
   // (the call then fails with FASTT_EUNSUP)
   unsigned *err;
+  // INSERT on the lane kernel: per lane and device gap_cap idle slots
+  void *gap_lane;
+  int32_t gap_cap;
 };
 
 // one idle slot [a, b) of a device under INSERT
@@ -286,7 +289,8 @@ FASTT_DECL_SIM_FN(0) FASTT_DECL_SIM_FN(1) FASTT_DECL_SIM_FN(2) FASTT_DECL_SIM_FN
 FASTT_DECL_SIM_FN(5)
 #undef FASTT_DECL_SIM_FN
 #define FASTT_DECL_LANE_FN(N, M) const void *lane_fn_g##N##_m##M(int tbits, int cm, bool exact, bool mg, bool pk);
-#define FASTT_DECL_PK_FN(N) const void *lane_pk_fn_g##N(int mm, bool exact);
+#define FASTT_DECL_PK_FN(N) const void *lane_pk_fn_g##N(int mm, bool exact); \
+  const void *lane_ins_fn_g##N(int tbits, int cm, bool exact);
 FASTT_DECL_PK_FN(0) FASTT_DECL_PK_FN(1) FASTT_DECL_PK_FN(2) FASTT_DECL_PK_FN(3) FASTT_DECL_PK_FN(4) FASTT_DECL_PK_FN(5)
 #undef FASTT_DECL_PK_FN
 #define FASTT_DECL_LANE_FN3(N) FASTT_DECL_LANE_FN(N, 0) FASTT_DECL_LANE_FN(N, 1) FASTT_DECL_LANE_FN(N, 2)

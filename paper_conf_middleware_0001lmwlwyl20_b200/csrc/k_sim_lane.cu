@@ -173,9 +173,29 @@ static size_t lane_pk_smem(int gshift, int mm) {
   return (LANE_BLOCK / 32) * w;
 }
 
+static const void *lane_ins_fn(int tbits, int gshift, int cm, bool exact) {
+  switch (gshift) {
+    case 0: return lane_ins_fn_g0(tbits, cm, exact);
+    case 1: return lane_ins_fn_g1(tbits, cm, exact);
+    case 2: return lane_ins_fn_g2(tbits, cm, exact);
+    case 3: return lane_ins_fn_g3(tbits, cm, exact);
+    case 4: return lane_ins_fn_g4(tbits, cm, exact);
+    default: return lane_ins_fn_g5(tbits, cm, exact);
+  }
+}
+
 void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
   const bool mg = a.lane == 2;
   const int cm = lane_comm_mode(a, tbits);
+  if (a.ins) {  // INSERT (R1i): the plain-key base-graph kernel with idle-slot arrays
+    const void *f = lane_ins_fn(tbits, a.gshift, cm, a.G == (1 << a.gshift));
+    const size_t sm = lane_smem(tbits, a.gshift, false, 0, false);
+    cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    SimArgs aa = a;
+    void *args[] = {&aa};
+    cudaLaunchKernel(f, dim3(grid), dim3(LANE_BLOCK), args, sm, st);
+    return;
+  }
   const bool pk = !mg && tbits == 32 && cm != 2 && a.costk != nullptr && a.pk_lim > 0;
   if (pk && a.pkc) {  // the base-graph sweep kernel: TMA-staged packed-key cards
     const void *f = lane_pk_fn(a.gshift, a.lane_mm, a.G == (1 << a.gshift));

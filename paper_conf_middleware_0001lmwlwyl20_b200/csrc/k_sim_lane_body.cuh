@@ -266,8 +266,17 @@ __device__ __noinline__ int cp_rounds_lane(const PrepGraph *pg, const GraphConst
 //     rounds (R9, memory reserved up front), slack[d] = cap - used - reserved
 //     per lane, a device is feasible iff mem_i <= slack[d] (a CP-pinned op
 //     draws on its reservation), no feasible device => INFEASIBLE.
-template <typename T, int GSH, int CM, bool EX, bool MG, bool PK, int MM>
+// INS: the insertion policy (R1i; NEXT N1) -- lane l keeps, per
+//     device, the device's positive-length idle slots as an array sorted by
+//     start in global memory (a.gap_lane, gap_cap slots per device); EST on
+//     d is the arrival when it is at or after avail[d], else the first slot
+//     [a, b) ending after the arrival r with max(a, r) + w <= b (binary
+//     search + short scan, as k_sim), else avail[d].  A lane whose device
+//     would need more than gap_cap slots is deferred to the group kernel.
+//     (base graph, no memory mode, no packed keys)
+template <typename T, int GSH, int CM, bool EX, bool MG, bool PK, int MM, bool INS = false>
 __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
+  static_assert(!INS || (!MG && !PK && MM == 0), "INSERT lanes: base graph, plain keys, no memory mode");
   // slab / ring / stage record: FT | place, or the packed key (PK)
   typedef typename std::conditional<PK, uint32_t, typename Slab<T>::W>::type W;
   constexpr int GP = 1 << GSH;
@@ -425,6 +434,13 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     int nr = 0, rc = 0, rdv = -1;
     uint32_t rhi = 0;
     bool dead = false;  // MM 2: no feasible device at some step (R8)
+    // INS: idle-slot counts per device, and an overflow flag (defer the lane)
+    uint32_t gn[GP];
+    bool ovf = false;
+#pragma unroll
+    for (int d = 0; d < GP; d++) gn[d] = 0;
+    GapSlot<T> *const gbase =
+        INS ? (GapSlot<T> *)a.gap_lane + ((size_t)gwarp * 32 + lane) * (size_t)GP * (size_t)a.gap_cap : nullptr;
     const uint32_t dmask = (MG && c.dev_mask) ? c.dev_mask : all;  // the candidate's devices (R25)
     if (MM && run) {
 #pragma unroll
@@ -892,10 +908,32 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
       // EFT per device; argmin with ties to the lowest device
       // (Alg. 1 lines 12-19, R3); devices >= G are never chosen
       T eft[GP];
+      uint32_t gk[GP];  // INS: the idle slot the op would go into on d (NONE: appended)
 #pragma unroll
       for (int d = 0; d < GP; d++) {
         const T arr = CM == 2 ? arrd[d] : ((uint32_t)d == pa ? E : M);
-        const T est = avail[d] > arr ? avail[d] : arr;
+        T est = avail[d] > arr ? avail[d] : arr;
+        gk[d] = NONE;
+        if (INS && live && (EX || d < G) && arr < avail[d] && gn[d] > 0) {
+          // R1i: the first idle slot [a, b) with max(a, r) + w <= b; slots
+          // are disjoint and sorted, none ending before r can fit
+          const GapSlot<T> *gl = gbase + (size_t)d * a.gap_cap;
+          uint32_t lo = 0, hi = gn[d];
+          while (lo < hi) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (gl[mid].b < arr) lo = mid + 1;
+            else hi = mid;
+          }
+          for (uint32_t k = lo; k < gn[d]; k++) {
+            const GapSlot<T> e = gl[k];
+            const T tt = e.a > arr ? e.a : arr;
+            if (tt + cst[d] <= e.b) {
+              gk[d] = k;
+              est = tt;
+              break;
+            }
+          }
+        }
         eft[d] = ((EX || d < G) && (!MG || ((dmask >> d) & 1u))) ? est + cst[d] : TT<T>::MAXV;
       }
       // MM 2: memory-feasible devices only (Alg. 1 line 13, R8)
@@ -932,9 +970,62 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
           mv[bd * 32] = v;
           s32_at(bd) = clamp32(v);
         }
+        bool appended = true;
+        if (INS) {
+          // the chosen device's idle slots: the slot the op went into shrinks,
+          // splits in two (tail shifted up) or disappears (tail shifted down);
+          // an op appended after a data wait leaves a new slot [avail, ST)
+          uint32_t k0 = NONE, n0 = 0;
+          T av0 = 0, w0 = 0;
+#pragma unroll
+          for (int d = 0; d < GP; d++)
+            if (d == bd) {
+              k0 = gk[d];
+              n0 = gn[d];
+              av0 = avail[d];
+              w0 = cst[d];
+            }
+          GapSlot<T> *gl = gbase + (size_t)bd * a.gap_cap;
+          const T st0 = best - w0;
+          if (k0 != NONE) {
+            const GapSlot<T> e = gl[k0];
+            const bool left = st0 > e.a, right = best < e.b;
+            if (left && right) {
+              if (n0 + 1 > (uint32_t)a.gap_cap) ovf = true;
+              else {
+                for (uint32_t k = n0; k > k0 + 1; k--) gl[k] = gl[k - 1];
+                GapSlot<T> ne;
+                ne.a = best;
+                ne.b = e.b;
+                gl[k0 + 1] = ne;
+                gl[k0].b = st0;
+                n0++;
+              }
+            } else if (left) {
+              gl[k0].b = st0;
+            } else if (right) {
+              gl[k0].a = best;
+            } else {
+              for (uint32_t k = k0; k + 1 < n0; k++) gl[k] = gl[k + 1];
+              n0--;
+            }
+          } else if (st0 > av0) {
+            if (n0 + 1 > (uint32_t)a.gap_cap) ovf = true;
+            else {
+              GapSlot<T> ne;
+              ne.a = av0;
+              ne.b = st0;
+              gl[n0++] = ne;
+            }
+          }
+#pragma unroll
+          for (int d = 0; d < GP; d++)
+            if (d == bd) gn[d] = n0;
+          appended = k0 == NONE;
+        }
 #pragma unroll
         for (int d = 0; d < GP; d++)
-          if (d == bd) avail[d] = best;
+          if (d == bd && appended) avail[d] = best;
         ms = best > ms ? best : ms;
         W w;
         Slab<T>::make(w, best, (uint32_t)bd);
@@ -946,7 +1037,9 @@ __global__ void __launch_bounds__(LANE_BLOCK, LANE_MINB) k_sim_lane(SimArgs a) {
     cp_async_wait<0>();  // (no copy may land in the stage after this candidate)
 
     // ------------------------------------------------------------ epilogue
-    if (PK && run && (uint32_t)ms >= a.pk_lim) {  // a key may have wrapped: re-run unpacked
+    if ((PK && run && (uint32_t)ms >= a.pk_lim) || (INS && run && ovf)) {
+      // a key may have wrapped / a device ran out of idle-slot capacity: re-run
+      // through the preparation pipeline on the group kernel
       const unsigned long long k = atomicAdd(a.ndefer, 1ull);
       a.defer_q[k] = q;
     } else if (run) {

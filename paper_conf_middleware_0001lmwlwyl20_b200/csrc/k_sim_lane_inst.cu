@@ -28,4 +28,19 @@ const void *FASTT_CAT(FASTT_CAT(FASTT_CAT(lane_fn_g, FASTT_GSH), _m), FASTT_MM)(
   return exact ? lane_fn_x<true, false>(tbits, cm, pk) : lane_fn_x<false, false>(tbits, cm, pk);
 }
 
+#if FASTT_MM == 0
+// INSERT (R1i) on the lane kernel: base graph, plain keys, no memory mode
+template <typename T, int CM, bool EX> static const void *lane_ins_t() {
+  return (const void *)k_sim_lane<T, FASTT_GSH, CM, EX, false, false, 0, true>;
+}
+template <bool EX> static const void *lane_ins_x(int tbits, int cm) {
+  if (tbits == 32)
+    return cm == 0 ? lane_ins_t<uint32_t, 0, EX>() : cm == 1 ? lane_ins_t<uint32_t, 1, EX>() : lane_ins_t<uint32_t, 2, EX>();
+  return cm == 2 ? lane_ins_t<uint64_t, 2, EX>() : lane_ins_t<uint64_t, 1, EX>();
+}
+const void *FASTT_CAT(lane_ins_fn_g, FASTT_GSH)(int tbits, int cm, bool exact) {
+  return exact ? lane_ins_x<true>(tbits, cm) : lane_ins_x<false>(tbits, cm);
+}
+#endif
+
 }  // namespace fastt

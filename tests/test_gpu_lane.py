@@ -301,3 +301,54 @@ def test_lane_memory_configs():
             o = og.schedule(c[k], flags=F.F_CP_PIN, outputs=False)
             assert (int(r["makespan"][k]), int(r["status"][k])) == (o["makespan"], o["status"]), (name, k)
             assert (r["peak_mem"][k] == o["peak_mem"]).all(), (name, k)
+
+
+# ------------------------------------------- INSERT on the lane kernel (R1i)
+
+INS = F.F_POLICY_INSERT
+
+
+@pytest.mark.parametrize("G", [1, 2, 3, 5, 8, 16])
+def test_lane_insert(G):
+    """INSERT (R1i) on the lane kernel: per-lane idle-slot
+    arrays, binary search + scan, slot split/shrink/removal -- against the
+    group kernel (FASTT_NO_LANE=1) and the oracle, with and without CP pins,
+    one and several link classes, 32- and 64-bit time"""
+    for K, scale in ((1, 1), (3, 1), (1, 50_000_000)):
+        desc = topo_dag(5300 + G + 7 * K, V=140, G=G, K=K, homogeneous=bool(G % 2), scale=scale)
+        cands = pin_cands(desc, np.random.default_rng(G + K), 128)
+        for flags in (INS, INS | F.F_CP_PIN):
+            check(desc, cands, flags)
+
+
+def test_lane_insert_capacity_deferral():
+    """a device needing more idle slots than the lane kernel's capacity
+    (FASTT_INS_CAP) defers the candidate to the group kernel: same results"""
+    desc = topo_dag(5400, V=200, G=4, K=1)
+    cands = pin_cands(desc, np.random.default_rng(3), 96)
+    ref = F.Graph(desc).schedule_batch(cands, flags=INS | F.F_CP_PIN, peak=False)
+    for cap in ("1", "3"):
+        g = _graph_env(desc, FASTT_INS_CAP=cap)
+        r = g.schedule_batch(cands, flags=INS | F.F_CP_PIN, peak=False)
+        assert g.last_timing()["topo"] == LANE and g.last_timing()["deferred"] > 0
+        assert (r["makespan"] == ref["makespan"]).all() and (r["status"] == ref["status"]).all()
+    og = O.OracleGraph(desc)
+    for k in range(0, len(cands), 7):
+        assert int(ref["makespan"][k]) == og.schedule(cands[k], flags=INS | F.F_CP_PIN, outputs=False)["makespan"]
+
+
+@pytest.mark.parametrize("name", ["C2", "C5"])
+def test_lane_insert_sweep_configs(name):
+    """the INSERT sweep on paper-shaped configs: lane kernel == group kernel,
+    winner == the oracle's makespan at that index"""
+    desc = synth.config(name)
+    gl, gg = F.Graph(desc), _graph_env(desc, FASTT_NO_LANE_INS="1")
+    flags = INS | F.F_CP_PIN
+    gen = F.gen_params(seed=0xFA57)
+    ns = gl.stream_info(gen, flags=flags)
+    n = ns + 1500
+    b1 = gl.sweep_best(gen, 0, n, flags=flags)
+    assert gl.last_timing()["topo"] == LANE
+    assert b1 == gg.sweep_best(gen, 0, n, flags=flags)
+    c = gl.generate_candidates(gen, b1[1], 1, flags=flags)
+    assert O.OracleGraph(desc).schedule(c[0], flags=flags, outputs=False)["makespan"] == b1[0]
