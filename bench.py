@@ -443,6 +443,23 @@ def main():
                              if tm2["topo"] == 2 else "k_sim",
                              "deferred_to_prep": tm2["deferred"]}
             del g2
+        # C5 under the paper's insertion policy (R1i): the same
+        # stream, 100k candidates (the group kernel, a lane per device)
+        nins = 100_000
+        fl_ins = FLAGS_CP | F.F_POLICY_INSERT
+        g.stream_info(gen, flags=fl_ins, stream=st)
+        g.sweep_best(gen, rank, nins, stride=world, flags=fl_ins, stream=st)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(st)
+        bi = g.sweep_best(gen, rank, nins, stride=world, flags=fl_ins, stream=st)
+        e1.record(st)
+        torch.cuda.synchronize()
+        ms_i = e0.elapsed_time(e1)
+        configs["C5_insert"] = {"V": V, "G": G, "candidates": nins, "policy": "INSERT (R1i)",
+                                "candidates_per_s": nins / (ms_i / 1000.0), "ops_per_s": nins / (ms_i / 1000.0) * V,
+                                "ms_per_sweep": ms_i, "best": list(bi),
+                                "kernel": "k_lane_ins" if g.last_timing()["topo"] == 2 else "k_sim<INS>"}
 
     cpu = None
     parity = None

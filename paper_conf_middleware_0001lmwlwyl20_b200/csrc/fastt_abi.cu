@@ -280,7 +280,11 @@ struct fastt_graph {
   void *gap_lane = nullptr;  // INSERT idle-slot arrays of the lane kernel (lazy)
   int32_t gap_cap = 0;       // idle slots per lane and device
   int ins_lane_grid = 0;
-  bool use_lane_ins = true;  // FASTT_NO_LANE_INS=1 keeps INSERT on the group kernel (A/B parity)
+  // FASTT_LANE_INS=1 runs INSERT on the lane kernel; off by default: on C5 it
+  // evaluates 53k candidates/s against the group kernel's 147k/s (one lane
+  // searches its G devices' idle slots one after the other, the group kernel
+  // searches them in parallel, a lane per device)
+  bool use_lane_ins = false;
   int64_t ins_cap_env = 0;   // FASTT_INS_CAP=<slots>: lower the per-device capacity (tests of the deferral)
   int64_t gap_stride = 0;
   int ins_grid = 0;
@@ -1511,8 +1515,8 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     g->use_pk = !(e && e[0] == '1');
     e = getenv("FASTT_NO_PK_TMA");
     g->use_pk_tma = !(e && e[0] == '1');
-    e = getenv("FASTT_NO_LANE_INS");
-    g->use_lane_ins = !(e && e[0] == '1');
+    e = getenv("FASTT_LANE_INS");
+    g->use_lane_ins = e && e[0] == '1';
     e = getenv("FASTT_INS_CAP");
     if (e && e[0]) g->ins_cap_env = std::max(1ll, atoll(e));
     e = getenv("FASTT_NO_OVERLAP");

@@ -64,7 +64,7 @@ def pin_cands(desc, rng, n, kmax=4):
 
 
 def check(desc, cands, flags, expect_kernel=LANE, oracle_every=1, peak=False):
-    gl = F.Graph(desc)
+    gl = _graph_env(desc, FASTT_LANE_INS="1") if flags & F.F_POLICY_INSERT else F.Graph(desc)
     gg = _graph_env(desc, FASTT_NO_LANE="1")
     r = gl.schedule_batch(cands, flags=flags, peak=peak)
     assert gl.last_timing()["topo"] == expect_kernel
@@ -310,10 +310,11 @@ INS = F.F_POLICY_INSERT
 
 @pytest.mark.parametrize("G", [1, 2, 3, 5, 8, 16])
 def test_lane_insert(G):
-    """INSERT (R1i) on the lane kernel: per-lane idle-slot
-    arrays, binary search + scan, slot split/shrink/removal -- against the
-    group kernel (FASTT_NO_LANE=1) and the oracle, with and without CP pins,
-    one and several link classes, 32- and 64-bit time"""
+    """INSERT (R1i) on the lane kernel (FASTT_LANE_INS=1: opt-in,
+    the group kernel is faster on C5): per-lane idle-slot arrays, binary
+    search + scan, slot split/shrink/removal -- against the group kernel
+    (FASTT_NO_LANE=1) and the oracle, with and without CP pins, one and
+    several link classes, 32- and 64-bit time"""
     for K, scale in ((1, 1), (3, 1), (1, 50_000_000)):
         desc = topo_dag(5300 + G + 7 * K, V=140, G=G, K=K, homogeneous=bool(G % 2), scale=scale)
         cands = pin_cands(desc, np.random.default_rng(G + K), 128)
@@ -328,7 +329,7 @@ def test_lane_insert_capacity_deferral():
     cands = pin_cands(desc, np.random.default_rng(3), 96)
     ref = F.Graph(desc).schedule_batch(cands, flags=INS | F.F_CP_PIN, peak=False)
     for cap in ("1", "3"):
-        g = _graph_env(desc, FASTT_INS_CAP=cap)
+        g = _graph_env(desc, FASTT_INS_CAP=cap, FASTT_LANE_INS="1")
         r = g.schedule_batch(cands, flags=INS | F.F_CP_PIN, peak=False)
         assert g.last_timing()["topo"] == LANE and g.last_timing()["deferred"] > 0
         assert (r["makespan"] == ref["makespan"]).all() and (r["status"] == ref["status"]).all()
@@ -342,7 +343,7 @@ def test_lane_insert_sweep_configs(name):
     """the INSERT sweep on paper-shaped configs: lane kernel == group kernel,
     winner == the oracle's makespan at that index"""
     desc = synth.config(name)
-    gl, gg = F.Graph(desc), _graph_env(desc, FASTT_NO_LANE_INS="1")
+    gl, gg = _graph_env(desc, FASTT_LANE_INS="1"), F.Graph(desc)
     flags = INS | F.F_CP_PIN
     gen = F.gen_params(seed=0xFA57)
     ns = gl.stream_info(gen, flags=flags)
