@@ -36,9 +36,26 @@
  *   - Errors: every call returns a status; nothing throws or aborts across
  *     the ABI.  On error fastt_last_error() (thread-local) explains why.
  *     Per-candidate infeasibility is a status value, not an error.
- *   - Synchronisation: work is issued on opts->cuda_stream (NULL = the
- *     legacy default stream of the graph's device) and every call returns
- *     after that stream has completed it (calls are blocking).
+ *   - Synchronisation ("calls are asynchronous on
+ *     cuda_stream; the caller synchronizes"): work is issued on
+ *     opts->cuda_stream (NULL = the legacy default stream of the graph's
+ *     device).  With FASTT_F_ASYNC, fastt_schedule_batch,
+ *     fastt_sweep_best and fastt_generate_candidates return once the work
+ *     is enqueued: nothing on their steady-state path waits for the device
+ *     (how many preparation rounds a batch needs is decided on the device,
+ *     by a CUDA-graph WHILE loop), and their outputs are valid once the
+ *     stream -- or fastt_sync -- has completed.  Inputs are consumed before
+ *     the call returns.  Host output buffers must then be page-locked for
+ *     the copies to be asynchronous; device buffers (FASTT_F_OUT_DEVICE /
+ *     FASTT_F_IN_DEVICE) always are.  The first call for a graph and flag
+ *     set (the BASE run, snapshot, stream and arena setup) and a call that
+ *     grows a workspace may block once.  Without FASTT_F_ASYNC a call
+ *     returns after the stream has completed it.  fastt_rank and
+ *     fastt_split_search are always blocking (their results come back
+ *     through host decisions: Alg. 2's accept/stop rule).  Calls on one
+ *     graph are ordered among themselves whatever stream they use (the
+ *     graph's scratch is shared); calls on different graphs are
+ *     independent and may overlap.
  *   - Determinism: every output is a pure function of (graph, candidates,
  *     flags, generator parameters); it is bit-identical to the CPU oracle.
  */
@@ -82,6 +99,7 @@ enum {
                                       (reading R27): each round also evaluates C_j = the best
                                       split of each of the j best-improving ops, applied in rank order
                                       (j = 2..4), and accepts the best C_j (ties: fewer splits) */
+  FASTT_F_ASYNC = 1u << 8,         /* return once enqueued on cuda_stream (see Synchronisation above) */
   FASTT_F_MEM_LIVE = 1u << 6       /* liveness memory (reading R24): an op's parameters stay on
                                       its device; its output (mem - param) is held from the step it is dequeued
                                       until the step its last consumer is dequeued.  The feasibility test of
@@ -252,6 +270,15 @@ typedef struct {
   int64_t lane_steps;   /* of which the steps of running candidates (each from its warp's start step) */
 } fastt_timing;
 fastt_status fastt_last_timing(const fastt_graph *g, fastt_timing *out);
+
+/* Completion of asynchronous calls (FASTT_F_ASYNC): waits until the work of
+ * every call issued on g so far has completed (on opts->cuda_stream and the
+ * graph's internal streams), then reports what a blocking call would have:
+ * FASTT_EUNSUP if a candidate met the envelope check done on the device (a
+ * non-topological priority order on a graph above 32,768 ops), FASTT_ECUDA
+ * if the device work failed.  Afterwards fastt_last_timing's `deferred`
+ * and `launches` describe the last asynchronous call. */
+fastt_status fastt_sync(const fastt_graph *g, const fastt_opts *opts);
 
 /* Communication cost-model fit ("we gather
  * tensors across the same source-destination device pairs into one group.

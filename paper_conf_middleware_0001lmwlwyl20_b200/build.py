@@ -8,7 +8,6 @@ from __future__ import annotations
 
 import os
 import subprocess
-import tempfile
 from concurrent.futures import ThreadPoolExecutor
 
 HERE = os.path.dirname(os.path.abspath(__file__))
@@ -33,22 +32,47 @@ CFLAGS += ["-D%s=%s" % (k, os.environ[k]) for k in ("SIM_MINB", "SIM_MINB_TOPO",
 FLAGS = CFLAGS + ["-shared"]  # (single-command form, kept for tools)
 
 
+OBJ_DIR = os.path.join(HERE, ".objs")  # per-unit objects kept between builds (git-ignored)
+_ABI_DEPS = [os.path.join(_C, "fastt_abi.cu"), os.path.join(_C, "fastt_internal.cuh"),
+             os.path.join(ROOT, "include", "fastt.h")]
+
+
+_HDRS = [d for d in DEPS if not d.endswith(".cu")]
+
+
+def _unit_deps(src):
+    # fastt_abi.cu includes only the ABI header and fastt_internal.cuh; every
+    # kernel unit is taken to depend on every header
+    return _ABI_DEPS if os.path.basename(src) == "fastt_abi.cu" else [src] + _HDRS
+
+
 def build(force: bool = False, verbose: bool = False, out: str = OUT) -> str:
     if not force and os.path.exists(out) and all(os.path.getmtime(out) >= os.path.getmtime(d) for d in DEPS):
         return out
-    with tempfile.TemporaryDirectory(prefix="fastt_build_") as td:
-        objs = [os.path.join(td, "%02d_%s.o" % (k, os.path.basename(u[0]))) for k, u in enumerate(UNITS)]
+    os.makedirs(OBJ_DIR, exist_ok=True)
+    objs = [os.path.join(OBJ_DIR, "%02d_%s_%s.o" % (k, os.path.basename(u[0]), "_".join(u[1]) or "x"))
+            for k, u in enumerate(UNITS)]
+    stamp = os.path.join(OBJ_DIR, "flags")
+    if not os.path.exists(stamp) or open(stamp).read() != " ".join(CFLAGS):
+        force = True
 
-        def cc(pair):
-            (src, extra), obj = pair
-            cmd = [NVCC] + CFLAGS + extra + (["-Xptxas", "-v"] if verbose else []) + ["-c", src, "-o", obj]
-            subprocess.check_call(cmd)
+    def cc(pair):
+        (src, extra), obj = pair
+        if not force and not verbose and os.path.exists(obj) and \
+                all(os.path.getmtime(obj) >= os.path.getmtime(d) for d in _unit_deps(src)):
+            return
+        tmpo = obj + ".tmp%d" % os.getpid()
+        cmd = [NVCC] + CFLAGS + extra + (["-Xptxas", "-v"] if verbose else []) + ["-c", src, "-o", tmpo]
+        subprocess.check_call(cmd)
+        os.replace(tmpo, obj)
 
-        with ThreadPoolExecutor(max_workers=min(len(UNITS), os.cpu_count() or 4)) as ex:
-            list(ex.map(cc, zip(UNITS, objs)))
-        tmp = out + ".tmp%d" % os.getpid()
-        subprocess.check_call([NVCC] + ARCH + ["-shared", "-o", tmp] + objs)
-        os.replace(tmp, out)
+    with ThreadPoolExecutor(max_workers=min(len(UNITS), os.cpu_count() or 4)) as ex:
+        list(ex.map(cc, zip(UNITS, objs)))
+    with open(stamp, "w") as f:
+        f.write(" ".join(CFLAGS))
+    tmp = out + ".tmp%d" % os.getpid()
+    subprocess.check_call([NVCC] + ARCH + ["-shared", "-o", tmp] + objs)
+    os.replace(tmp, out)
     return out
 
 

@@ -7,6 +7,7 @@
 #include "fastt_internal.cuh"
 
 #include <algorithm>
+#include <chrono>
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
@@ -322,9 +323,40 @@ struct fastt_graph {
   int32_t slot_bm_bits = 0;
   int64_t wbest_cap = 0;        // wbest entries allocated
   int64_t pin_defer_hint = 256; // rank-changing PINs seen by the last classified call
-  int64_t last_nd = -1;         // deferred candidates of the last eval_batch (overlapped path), else -1
+  // device-driven deferral loop (run_defer_loop): a cached CUDA graph with a
+  // WHILE node over the preparation rounds, rebuilt when its arguments change
+  DeferBlock *dblk = nullptr;
+  uint32_t *dwords = nullptr;      // zero words (n_main of a loop without a tail)
+  cudaStream_t st_cap = nullptr;   // capture stream of the loop graph
+  cudaGraphExec_t dl_exec = nullptr;
+  std::vector<char> dl_key;
+  cudaEvent_t dl_ev = nullptr;     // recorded after every launch of dl_exec
+  std::vector<std::pair<cudaGraphExec_t, cudaEvent_t>> dl_retired;  // destroyed once their event completed
+  int dl_round_launches = 0;       // kernels per loop round (fastt_last_timing)
+  DeferBlock *dl_sum = nullptr;    // pinned host copy of the last loop's block (hints, deferred counts)
+  cudaEvent_t dl_sum_ev = nullptr;
+  bool dl_sum_pending = false;
+  bool dl_ran = false;             // this call ran the loop
+  // call ordering: every call on this graph waits for the previous one (its
+  // internal scratch is shared), whatever stream either was issued on
+  cudaEvent_t done_ev = nullptr;
+  bool done_rec = false;
   std::mutex mu;
 };
+
+static void read_defer_summary(fastt_graph *g);
+static void reap_defer(fastt_graph *g, bool wait);
+
+// FASTT_HOST_TRACE=1: host wall-clock checkpoints of a call on stderr (where
+// a call waits for the device)
+static void host_trace(const char *what) {
+  static int on = -1;
+  if (on < 0) on = getenv("FASTT_HOST_TRACE") && atoi(getenv("FASTT_HOST_TRACE")) ? 1 : 0;
+  if (!on) return;
+  static auto t0 = std::chrono::steady_clock::now();
+  const double us = std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - t0).count();
+  fprintf(stderr, "[fastt host] %12.1f us  %s\n", us, what);
+}
 
 // kernels each launcher issues (for the launch count of fastt_last_timing)
 enum { NL_SIM = 1, NL_PREP = 9, NL_ARGMIN = 1, NL_GATHER = 1, NL_CANDGEN = 1, NL_ORDER = 1, NL_FILL = 1 };
@@ -357,11 +389,22 @@ static fastt_status check_kernel_err(fastt_graph *g, cudaStream_t st) {
   return FASTT_OK;
 }
 
-static fastt_status timing_end(fastt_graph *g, uint32_t flags, cudaStream_t st, int64_t cands, int64_t deferred) {
-  TRY(check_kernel_err(g, st));
+// the last deferral loop of this call, once its summary has landed (host
+// synchronised): deferred count and the loop's kernel launches
+static void defer_stats(fastt_graph *g) {
+  if (!g->dl_ran || g->dl_sum_pending) return;
+  const DeferBlock &d = *g->dl_sum;
+  const int64_t tail = d.do_tail && d.n_main >= 0 ? d.n - d.n_main : 0;
+  const int64_t past = d.n - d.tail_lo;  // the tail past the arena: loop rounds
+  const int64_t cap = d.cap > 0 ? d.cap : 1;
+  g->last.deferred = tail + d.n_defer;
+  g->last.launches += ((past + cap - 1) / cap + (d.n_defer + cap - 1) / cap) * g->dl_round_launches;
+}
+
+static fastt_status timing_end(fastt_graph *g, uint32_t flags, cudaStream_t st, int64_t cands) {
   g->last.launches = g->launches;
   g->last.candidates = cands;
-  g->last.deferred = deferred;
+  g->last.deferred = 0;
   g->last.topo = g->last_topo;
   if (!(flags & FASTT_F_TIMING)) return FASTT_OK;
   CK(cudaEventRecord(g->ev[3], st));
@@ -381,6 +424,42 @@ static fastt_status timing_end(fastt_graph *g, uint32_t flags, cudaStream_t st, 
   g->last.ms_total = c;
   return FASTT_OK;
 }
+
+// Every ABI call that issues work: call_begin orders it after the previous
+// call on this graph (any stream); call_end records the graph's completion
+// event and -- unless FASTT_F_ASYNC -- waits for the stream, reports a
+// kernel-side envelope error and fills the deferred statistics.
+static fastt_status call_begin(fastt_graph *g, cudaStream_t st) {
+  if (g->done_rec) CK(cudaStreamWaitEvent(st, g->done_ev, 0));
+  read_defer_summary(g);
+  g->dl_ran = false;
+  return FASTT_OK;
+}
+static fastt_status call_end(fastt_graph *g, uint32_t flags, cudaStream_t st, fastt_status rc) {
+  if (!g->done_ev && cudaEventCreateWithFlags(&g->done_ev, cudaEventDisableTiming) != cudaSuccess) g->done_ev = nullptr;
+  if (g->done_ev && cudaEventRecord(g->done_ev, st) == cudaSuccess) g->done_rec = true;
+  if (flags & FASTT_F_ASYNC) return rc;
+  if (cudaStreamSynchronize(st) != cudaSuccess && rc == FASTT_OK) rc = fail(FASTT_ECUDA, "synchronize");
+  if (rc == FASTT_OK) rc = check_kernel_err(g, st);
+  read_defer_summary(g);
+  defer_stats(g);
+  // retired loop graphs are destroyed here, never on an asynchronous path
+  // (cudaGraphExecDestroy waits for the device)
+  reap_defer(g, false);
+  return rc;
+}
+
+// the blocking calls (rank, split search, stream info): ordered after the
+// previous call on the graph; their completion recorded at scope exit
+struct CallGuard {
+  fastt_graph *g;
+  cudaStream_t st;
+  CallGuard(fastt_graph *g_, cudaStream_t st_) : g(g_), st(st_) { call_begin(g, st); }
+  ~CallGuard() {
+    if (!g->done_ev && cudaEventCreateWithFlags(&g->done_ev, cudaEventDisableTiming) != cudaSuccess) g->done_ev = nullptr;
+    if (g->done_ev && cudaEventRecord(g->done_ev, st) == cudaSuccess) g->done_rec = true;
+  }
+};
 
 static int64_t overlay_v(const fastt_graph *g) { return (int64_t)g->maxP + g->G + g->maxS + 1; }
 static int64_t overlay_e(const fastt_graph *g) {
@@ -878,6 +957,177 @@ static void launch_slots(fastt_graph *g, SimArgs b, int tbits, int nc, cudaStrea
   g->launches += g->use_topo ? 1 : 0;
 }
 
+// ------------------------------------------- device-driven deferral loop
+// The candidates a main launch hands to the preparation pipeline (the tail
+// of a classified list past the arena, the deferral queue) are evaluated in
+// rounds of at most `cap` slots: gather -> preparation -> slot simulations.
+// How many rounds run is only known on the device, so the rounds are the
+// body of a CUDA-graph WHILE node whose condition k_defer_begin /
+// k_defer_plan set (cudaGraphSetConditional): the call enqueues the loop and
+// never waits for a count (fastt.h: calls are asynchronous on cuda_stream).
+// The instantiated graph depends only on the graph's buffers and the slot
+// launches' arguments; per-call values (list length, sources) live in the
+// device block dblk, written by k_defer_setup.
+
+static fastt_status ensure_defer(fastt_graph *g) {
+  if (g->dblk) return FASTT_OK;
+  CK(cudaMalloc(&g->dblk, sizeof(DeferBlock)));
+  CK(cudaMemset(g->dblk, 0, sizeof(DeferBlock)));
+  CK(cudaMalloc(&g->dwords, 16));
+  CK(cudaMemset(g->dwords, 0, 16));
+  if (!g->counters2) CK(cudaMalloc(&g->counters2, 2 * sizeof(unsigned long long)));
+  CK(cudaStreamCreateWithFlags(&g->st_cap, cudaStreamNonBlocking));
+  CK(cudaEventCreateWithFlags(&g->dl_ev, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&g->dl_sum_ev, cudaEventDisableTiming));
+  CK(cudaMallocHost(&g->dl_sum, sizeof(DeferBlock)));
+  memset(g->dl_sum, 0, sizeof(DeferBlock));
+  return FASTT_OK;
+}
+
+// destroy retired loop graphs whose last launch has completed (all of them
+// when wait: the caller has synchronised the device); only from blocking
+// calls: cudaGraphExecDestroy waits for the device
+static void reap_defer(fastt_graph *g, bool wait) {
+  for (size_t k = 0; k < g->dl_retired.size();) {
+    auto &r = g->dl_retired[k];
+    if (wait || cudaEventQuery(r.second) == cudaSuccess) {
+      cudaGraphExecDestroy(r.first);
+      cudaEventDestroy(r.second);
+      g->dl_retired[k] = g->dl_retired.back();
+      g->dl_retired.pop_back();
+    } else {
+      k++;
+    }
+  }
+}
+
+// the last loop's summary (pinned copy) once its event completed: the arena
+// hint (rank-changing PINs of the last classified list)
+static void read_defer_summary(fastt_graph *g) {
+  if (!g->dl_sum_pending || cudaEventQuery(g->dl_sum_ev) != cudaSuccess) return;
+  g->dl_sum_pending = false;
+  if (g->dl_sum->do_tail && g->dl_sum->n_main >= 0) g->pin_defer_hint = g->dl_sum->n - g->dl_sum->n_main;
+}
+
+static fastt_status build_defer_graph(fastt_graph *g, Base &B, const SimArgs &b, int cap, bool results,
+                                      const uint32_t *n_main, const unsigned long long *ndefer,
+                                      cudaGraphExec_t *out) {
+  cudaStream_t cs = g->st_cap;
+  cudaGraph_t gr = nullptr, body = nullptr, tmp = nullptr;
+  CK(cudaGraphCreate(&gr, 0));
+  cudaGraphConditionalHandle h;
+  fastt_status rc = FASTT_OK;
+  auto ck = [&](cudaError_t e, const char *what) {
+    if (e != cudaSuccess && rc == FASTT_OK) rc = fail(FASTT_ECUDA, "%s: %s", what, cudaGetErrorString(e));
+  };
+  ck(cudaGraphConditionalHandleCreate(&h, gr, 0, 0), "conditional handle");
+  ck(cudaStreamBeginCaptureToGraph(cs, gr, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed), "capture");
+  launch_defer_begin(g->dblk, n_main, ndefer, h, cs);
+  cudaStreamCaptureStatus cst;
+  cudaGraph_t cg = nullptr;
+  const cudaGraphNode_t *deps = nullptr;
+  size_t nd = 0;
+  ck(cudaStreamGetCaptureInfo(cs, &cst, nullptr, &cg, &deps, &nd), "capture info");
+  cudaGraphNodeParams cp = {};
+  cp.type = cudaGraphNodeTypeConditional;
+  cp.conditional.handle = h;
+  cp.conditional.type = cudaGraphCondTypeWhile;
+  cp.conditional.size = 1;
+  cudaGraphNode_t cn = nullptr;
+  if (rc == FASTT_OK) ck(cudaGraphAddNode(&cn, cg, deps, nd, &cp), "WHILE node");
+  if (rc == FASTT_OK) ck(cudaStreamUpdateCaptureDependencies(cs, &cn, 1, cudaStreamSetCaptureDependencies), "deps");
+  ck(cudaStreamEndCapture(cs, &tmp), "end capture");
+  host_trace("loop build: WHILE node");
+  if (rc == FASTT_OK) {
+    body = cp.conditional.phGraph_out[0];
+    const int64_t l0 = g->launches;
+    ck(cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed), "body capture");
+    launch_defer_plan(g->dblk, h, cs);
+    launch_defer_gather(g->dblk, cap, g->srt_c, g->srt_i, results ? g->srt_res : nullptr, g->defer_q,
+                        g->slot_cands, g->slot_index, results ? g->slot_result : nullptr, cs);
+    fastt_status pr = run_prep(g, B, cap, cs, &g->dblk->nact);
+    if (pr != FASTT_OK && rc == FASTT_OK) rc = pr;
+    ck(cudaMemsetAsync(b.counter, 0, sizeof(unsigned long long), cs), "counter reset");
+    launch_slots(g, b, B.tbits, cap, cs);
+    g->launches += NL_SIM;
+    g->dl_round_launches = 2 + (int)(g->launches - l0);
+    g->launches = l0;
+    ck(cudaGetLastError(), "body launches");
+    ck(cudaStreamEndCapture(cs, &tmp), "end body capture");
+  }
+  host_trace("loop build: captured");
+  if (rc == FASTT_OK) ck(cudaGraphInstantiate(out, gr, 0), "instantiate the deferral loop");
+  host_trace("loop build: instantiated");
+  cudaGraphDestroy(gr);
+  return rc;
+}
+
+// Evaluate the deferred candidates of a finished main launch (b: the slot
+// launches' arguments; src: defer_q entries index the sorted list (0), the
+// candidate list cands (1) or the stream (2); do_tail: also the classified
+// tail past the arena, positions [*n_main + cap, n) of the sorted list).
+static fastt_status run_defer_loop(fastt_graph *g, Base &B, SimArgs b, int cap, int src, bool do_tail, int64_t n,
+                                   const Cand *cands, const StreamState *ss, int64_t first, int64_t stride,
+                                   bool results, const unsigned long long *ndefer, cudaStream_t st) {
+  TRY(ensure_defer(g));
+  const uint32_t *n_main = do_tail ? g->ov_words : g->dwords;
+  b.slots = g->slot_pgs_dev;
+  b.cands = g->slot_cands;
+  b.slot_index = results ? nullptr : g->slot_index;
+  b.slot_result = results ? g->slot_result : nullptr;
+  b.n = cap;
+  b.n_dev = &g->dblk->nact;
+  b.counter = g->counters2;
+  b.lane_batches = 0;
+  b.preclassified = 0;
+  b.stat = nullptr;
+  b.flags &= ~(uint32_t)(FASTT_F_ASYNC | FASTT_F_TIMING | FASTT_F_OUT_DEVICE | FASTT_F_IN_DEVICE);  // (host-side)
+  StreamState s0;
+  memset(&s0, 0, sizeof s0);
+  launch_defer_setup(g->dblk, n, cap, src, do_tail ? 1 : 0, results ? 1 : 0, cands, ss ? *ss : s0, first, stride, st);
+  // the loop graph's identity: the slot launches' arguments and every buffer
+  // the body touches
+  const void *ptrs[] = {g->arena,     g->slot_raws_dev, g->slot_pgs_dev, g->slot_cands, g->slot_index,
+                        g->slot_result, g->tmpl_dev,    B.raw_block,     B.raw_dev,     B.prep_block,
+                        B.pg_dev,     g->srt_c,         g->srt_i,        g->srt_res,    g->defer_q,
+                        n_main,       ndefer,           g->gc_dev};
+  const int ints[] = {cap, B.tbits, B.key_bits, (int)B.rl.vcap, g->G, g->K, g->use_topo, g->use_rank_reuse,
+                      results, (int)g->sim_block, (int)g->sim_grid, (int)g->sim_grid_topo, (int)g->sim_cpw};
+  std::vector<char> key(sizeof b + sizeof ptrs + sizeof ints);
+  memcpy(key.data(), &b, sizeof b);
+  memcpy(key.data() + sizeof b, ptrs, sizeof ptrs);
+  memcpy(key.data() + sizeof b + sizeof ptrs, ints, sizeof ints);
+  if (!g->dl_exec || g->dl_key != key) {
+    if (getenv("FASTT_HOST_TRACE") && g->dl_key.size() == key.size()) {
+      char msg[96];
+      for (size_t k = 0; k < key.size(); k++)
+        if (key[k] != g->dl_key[k]) {
+          snprintf(msg, sizeof msg, "loop: key differs at byte %zu (SimArgs %zu bytes)", k, sizeof b);
+          host_trace(msg);
+          break;
+        }
+    }
+    if (g->dl_exec) {  // retire: destroyed once its last launch completed
+      g->dl_retired.push_back({g->dl_exec, g->dl_ev});
+      g->dl_exec = nullptr;
+      g->dl_ev = nullptr;
+      CK(cudaEventCreateWithFlags(&g->dl_ev, cudaEventDisableTiming));
+    }
+    TRY(build_defer_graph(g, B, b, cap, results, n_main, ndefer, &g->dl_exec));
+    g->dl_key.swap(key);
+  }
+  host_trace("loop: setup + graph");
+  CK(cudaGraphLaunch(g->dl_exec, st));
+  host_trace("loop: graph launch");
+  CK(cudaEventRecord(g->dl_ev, st));
+  g->launches += 2;  // setup + begin (the rounds: fastt_last_timing)
+  CK(cudaMemcpyAsync(g->dl_sum, g->dblk, sizeof(DeferBlock), cudaMemcpyDeviceToHost, st));
+  CK(cudaEventRecord(g->dl_sum_ev, st));
+  g->dl_sum_pending = true;
+  g->dl_ran = true;
+  return FASTT_OK;
+}
+
 // ------------------------------------------------- overlapped evaluation
 // A start-step-sorted candidate list classified on the device (launch_t0_sort
 // with T0Classify: the candidates that need their own prepared graph sorted
@@ -961,6 +1211,7 @@ static fastt_status run_overlapped(fastt_graph *g, Base &B, SimArgs a, int64_t n
   launch_slots(g, b, B.tbits, cap, sp);
   g->launches += NL_SIM;
   CK(cudaGetLastError());
+  host_trace("overlap: prep stream launches");
   CK(cudaEventRecord(g->ov_ev[2], sp));
   // the main launch (the call's stream)
   a.preclassified = 1;
@@ -984,54 +1235,15 @@ static fastt_status run_overlapped(fastt_graph *g, Base &B, SimArgs a, int64_t n
   return FASTT_OK;
 }
 
-// after the join (host-synchronising): a tail longer than the arena and the
-// main launch's packed-key deferrals, sequentially on st
+// after the join: a tail longer than the arena and the main launch's
+// packed-key deferrals, sequentially on st (the device-driven loop)
 static fastt_status finish_overlapped(fastt_graph *g, Base &B, SimArgs a, int64_t n, cudaStream_t st, bool results,
-                                      int cap, int wmain, unsigned long long *nd_total) {
-  uint32_t w[2] = {0, 0};
-  unsigned long long pkd = 0;
-  CK(cudaMemcpyAsync(w, g->ov_words, 8, cudaMemcpyDeviceToHost, st));
-  CK(cudaMemcpyAsync(&pkd, g->counters + 1, sizeof pkd, cudaMemcpyDeviceToHost, st));
-  CK(cudaStreamSynchronize(st));
-  const int64_t tail = n - (int64_t)w[0];
-  g->pin_defer_hint = tail;
-  *nd_total = (unsigned long long)tail + pkd;
+                                      int cap, int wmain) {
   SimArgs b = a;
-  b.slots = g->slot_pgs_dev;
-  b.cands = g->slot_cands;
-  b.slot_index = results ? nullptr : g->slot_index;
-  b.slot_result = results ? g->slot_result : nullptr;
   b.wbest = g->wbest + 2 * (int64_t)wmain;
   b.slab = g->slab_mg;
-  b.lane_batches = 0;
-  b.preclassified = 0;
-  b.stat = nullptr;
   b.n_dev = nullptr;
-  for (int64_t off = cap; off < tail; off += cap) {  // the tail past the arena
-    const int nc = (int)std::min<int64_t>(cap, tail - off);
-    launch_gather_tail(g->srt_c, g->srt_i, results ? g->srt_res : nullptr, g->ov_words, n, off, cap, g->slot_cands,
-                       g->slot_index, results ? g->slot_result : nullptr, g->ov_words + 1, st);
-    g->launches += NL_GATHER + NL_SIM;
-    TRY(run_prep(g, B, nc, st));
-    CK(cudaMemsetAsync(g->counters2, 0, sizeof(unsigned long long), st));
-    b.counter = g->counters2;
-    b.n = nc;
-    launch_slots(g, b, B.tbits, nc, st);
-    CK(cudaGetLastError());
-  }
-  for (int64_t c0 = 0; c0 < (int64_t)pkd; c0 += cap) {  // packed-key deferrals of the main launch
-    const int nc = (int)std::min<int64_t>(cap, (int64_t)pkd - c0);
-    launch_gather_sorted(g->srt_c, g->srt_i, results ? g->srt_res : nullptr, g->defer_q + c0, nc, g->slot_cands,
-                         results ? nullptr : g->slot_index, results ? g->slot_result : nullptr, st);
-    g->launches += NL_GATHER + NL_SIM;
-    TRY(run_prep(g, B, nc, st));
-    CK(cudaMemsetAsync(g->counters2, 0, sizeof(unsigned long long), st));
-    b.counter = g->counters2;
-    b.n = nc;
-    launch_slots(g, b, B.tbits, nc, st);
-    CK(cudaGetLastError());
-  }
-  return FASTT_OK;
+  return run_defer_loop(g, B, b, cap, 0, true, n, nullptr, nullptr, 0, 1, results, g->counters + 1, st);
 }
 
 struct DevOut {
@@ -1114,13 +1326,13 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
     }
     TRY(run_overlapped(g, B, a, n, flags, st, true, cap, wmain));
     timing_mark(g, flags, 2, st);
-    unsigned long long ndo = 0;
-    TRY(finish_overlapped(g, B, a, n, st, true, cap, wmain, &ndo));
-    g->last_nd = (int64_t)ndo;
-    if (o.order) return fail(FASTT_EINVAL, "order output on the overlapped path");  // (excluded above)
-    CK(cudaStreamSynchronize(st));
+    TRY(finish_overlapped(g, B, a, n, st, true, cap, wmain));
+    if (!(flags & FASTT_F_ASYNC)) CK(cudaStreamSynchronize(st));
     return FASTT_OK;
   }
+  // the arena of the deferral rounds (sized before the launch: the count is
+  // only known on the device)
+  TRY(ensure_arena(g, B, st, std::max<int64_t>(256, std::min<int64_t>(g->pin_defer_hint, 8192))));
   if (sorted) {
     // order the list by BASE-prefix start step (results keep their index)
     TRY(ensure_sort_buf(g, n));
@@ -1144,57 +1356,34 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
   g->launches += NL_SIM;
   CK(cudaGetLastError());
   timing_mark(g, flags, 1, st);
-  unsigned long long nd = 0;
-  CK(cudaMemcpyAsync(&nd, g->counters + 1, sizeof nd, cudaMemcpyDeviceToHost, st));
-  CK(cudaStreamSynchronize(st));
-  if (nd > 0) {
-    TRY(ensure_arena(g, B, st, (int64_t)nd));
-    for (int64_t c0 = 0; c0 < (int64_t)nd; c0 += g->arena_slots) {
-      int nc = (int)std::min<int64_t>(g->arena_slots, (int64_t)nd - c0);
-      if (sorted) launch_gather_sorted(g->srt_c, g->srt_i, g->srt_res, g->defer_q + c0, nc, g->slot_cands, nullptr,
-                                       g->slot_result, st);
-      else launch_gather_cands(d_cands, g->defer_q + c0, nc, g->slot_cands, g->slot_result, st);
-      g->launches += NL_GATHER + NL_SIM;
-      TRY(run_prep(g, B, nc, st));
-      CK(cudaMemsetAsync(g->counters, 0, sizeof(unsigned long long), st));
-      SimArgs b = a;
-      b.slots = g->slot_pgs_dev;
-      b.cands = g->slot_cands;
-      b.slot_result = g->slot_result;
-      b.slot_index = nullptr;
-      b.n = nc;
-      launch_slots(g, b, B.tbits, nc, st);
-      CK(cudaGetLastError());
-    }
-  }
+  TRY(run_defer_loop(g, B, a, g->arena_slots, sorted ? 0 : 1, false, n, d_cands, nullptr, 0, 1, true,
+                     g->counters + 1, st));
   timing_mark(g, flags, 2, st);
   if (o.order) {
-    // execution order list A (R17): per-result stable sort of the dequeue list by start
-    int64_t chunk = 256;
-    uint64_t *k0, *k1;
-    uint32_t *v0, *v1;
-    CK(cudaMalloc(&k0, (size_t)chunk * o.vmax * 8));
-    CK(cudaMalloc(&k1, (size_t)chunk * o.vmax * 8));
-    CK(cudaMalloc(&v0, (size_t)chunk * o.vmax * 4));
-    CK(cudaMalloc(&v1, (size_t)chunk * o.vmax * 4));
-    std::vector<int64_t> idx(chunk);
-    int64_t *d_idx;
-    CK(cudaMalloc(&d_idx, sizeof(int64_t) * chunk));
+    // execution order list A (R17): per-result stable sort of the dequeue
+    // list by start, 256 results per launch (stream-ordered scratch)
+    const int64_t chunk = 256;
+    uint64_t *k0 = nullptr, *k1 = nullptr;
+    uint32_t *v0 = nullptr, *v1 = nullptr;
+    int64_t *d_idx = nullptr;
+    CK(cudaMallocAsync(&k0, (size_t)chunk * o.vmax * 8, st));
+    CK(cudaMallocAsync(&k1, (size_t)chunk * o.vmax * 8, st));
+    CK(cudaMallocAsync(&v0, (size_t)chunk * o.vmax * 4, st));
+    CK(cudaMallocAsync(&v1, (size_t)chunk * o.vmax * 4, st));
+    CK(cudaMallocAsync(&d_idx, sizeof(int64_t) * n, st));
+    launch_iota_i64(d_idx, n, st);
     for (int64_t c0 = 0; c0 < n; c0 += chunk) {
-      int64_t nc = std::min(chunk, n - c0);
-      for (int64_t k = 0; k < nc; k++) idx[k] = c0 + k;
-      CK(cudaMemcpyAsync(d_idx, idx.data(), sizeof(int64_t) * nc, cudaMemcpyHostToDevice, st));
-      launch_order_chunk(o.deq, o.start, o.order, d_idx, nc, o.vmax, B.key_bits, k0, k1, v0, v1, st);
+      const int64_t nc = std::min(chunk, n - c0);
+      launch_order_chunk(o.deq, o.start, o.order, d_idx + c0, nc, o.vmax, B.key_bits, k0, k1, v0, v1, st);
       g->launches += NL_ORDER;
-      CK(cudaStreamSynchronize(st));
     }
-    cudaFree(k0);
-    cudaFree(k1);
-    cudaFree(v0);
-    cudaFree(v1);
-    cudaFree(d_idx);
+    CK(cudaFreeAsync(k0, st));
+    CK(cudaFreeAsync(k1, st));
+    CK(cudaFreeAsync(v0, st));
+    CK(cudaFreeAsync(v1, st));
+    CK(cudaFreeAsync(d_idx, st));
   }
-  CK(cudaStreamSynchronize(st));
+  if (!(flags & FASTT_F_ASYNC)) CK(cudaStreamSynchronize(st));
   return FASTT_OK;
 }
 
@@ -1256,7 +1445,7 @@ static fastt_status ensure_stream(fastt_graph *g, uint32_t flags, int pow2, cuda
   o.status = d_st;
   o.place = S.base_place;
   o.vmax = vm;
-  TRY(eval_batch(g, B, d_c, 1, flags, st, o));
+  TRY(eval_batch(g, B, d_c, 1, flags & ~FASTT_F_ASYNC, st, o));  // (one-time setup: blocking)
   uint8_t hst = 0;
   CK(cudaMemcpy(&hst, d_st, 1, cudaMemcpyDeviceToHost));
   std::vector<int32_t> list;
@@ -1605,6 +1794,7 @@ void fastt_free_graph(fastt_graph *g) {
   if (!g) return;
   {
     Dev guard(g->dev);
+    cudaDeviceSynchronize();  // (in-flight asynchronous calls)
     g->base.release();
     for (auto &s : g->streams) s.release();
     cudaFree(g->gc_dev);
@@ -1637,6 +1827,15 @@ void fastt_free_graph(fastt_graph *g) {
     cudaFree(g->counters2);
     cudaFree(g->ov_words);
     cudaFree(g->slot_bm);
+    reap_defer(g, true);
+    if (g->dl_exec) cudaGraphExecDestroy(g->dl_exec);
+    if (g->dl_ev) cudaEventDestroy(g->dl_ev);
+    if (g->dl_sum_ev) cudaEventDestroy(g->dl_sum_ev);
+    if (g->done_ev) cudaEventDestroy(g->done_ev);
+    if (g->st_cap) cudaStreamDestroy(g->st_cap);
+    cudaFreeHost(g->dl_sum);
+    cudaFree(g->dblk);
+    cudaFree(g->dwords);
   }
   delete g;
 }
@@ -1684,6 +1883,7 @@ fastt_status fastt_rank(const fastt_graph *gc_, const fastt_candidate *cand, con
   std::lock_guard<std::mutex> lk(g->mu);
   Dev guard(g->dev);
   cudaStream_t st = stream_of(opts);
+  CallGuard cg(g, st);  // (blocking: the ranks come back through the host)
   Base &B = g->base;
   const int64_t vm = g->v_max;
   std::vector<uint64_t> r(B.rl.vcap, ~0ull);
@@ -1744,11 +1944,11 @@ fastt_status fastt_schedule_batch(const fastt_graph *gc_, const fastt_candidate 
   std::lock_guard<std::mutex> lk(g->mu);
   Dev guard(g->dev);
   cudaStream_t st = stream_of(opts);
+  TRY(call_begin(g, st));
   Base &B = g->base;
   const int64_t vm = g->v_max;
   const bool outdev = (flags & FASTT_F_OUT_DEVICE) != 0;
   Cand *d_c;
-  bool own_c = false;
   if (flags & FASTT_F_IN_DEVICE) {
     d_c = (Cand *)cands;
   } else {
@@ -1759,11 +1959,11 @@ fastt_status fastt_schedule_batch(const fastt_graph *gc_, const fastt_candidate 
   DevOut o;
   o.vmax = vm;
   std::vector<void *> tmp;
-  auto dalloc = [&](void *user, size_t bytes, bool need) -> void * {
+  auto dalloc = [&](void *user, size_t bytes, bool need) -> void * {  // stream-ordered scratch
     if (!need) return nullptr;
     if (outdev && user) return user;
     void *p = nullptr;
-    if (cudaMalloc(&p, bytes) != cudaSuccess) return nullptr;
+    if (cudaMallocAsync(&p, bytes, st) != cudaSuccess) return nullptr;
     tmp.push_back(p);
     return p;
   };
@@ -1779,15 +1979,8 @@ fastt_status fastt_schedule_batch(const fastt_graph *gc_, const fastt_candidate 
   if (!o.makespan || !o.status || (peak_mem && !o.peak) || (want_sched && (!o.place || !o.start)) ||
       (order && (!o.deq || !o.order)))
     rc = fail(FASTT_ENOMEM, "device output buffers");
-  unsigned long long nd0 = 0;
   if (rc == FASTT_OK) rc = timing_begin(g, flags, st);
-  g->last_nd = -1;
-  if (rc == FASTT_OK) rc = eval_batch(g, B, d_c, n, flags, st, o);
-  if (rc == FASTT_OK && g->last_nd >= 0) nd0 = (unsigned long long)g->last_nd;  // (overlapped path)
-  else if (rc == FASTT_OK &&
-           (cudaMemcpyAsync(&nd0, g->counters + 1, sizeof nd0, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
-            cudaStreamSynchronize(st) != cudaSuccess))
-    rc = fail(FASTT_ECUDA, "deferred count");
+  if (rc == FASTT_OK) rc = eval_batch(g, B, d_c, n, flags | FASTT_F_ASYNC, st, o);
   if (rc == FASTT_OK && !outdev) {
     auto back = [&](void *h, void *dd, size_t bytes) {
       if (h && dd && cudaMemcpyAsync(h, dd, bytes, cudaMemcpyDeviceToHost, st) != cudaSuccess)
@@ -1800,11 +1993,9 @@ fastt_status fastt_schedule_batch(const fastt_graph *gc_, const fastt_candidate 
     back(start_ns, o.start, 8 * (size_t)n * vm);
     back(order, o.order, 4 * (size_t)n * vm);
   }
-  if (rc == FASTT_OK) rc = timing_end(g, flags, st, n, (int64_t)nd0);
-  if (cudaStreamSynchronize(st) != cudaSuccess && rc == FASTT_OK) rc = fail(FASTT_ECUDA, "synchronize");
-  for (void *p : tmp) cudaFree(p);
-  if (own_c) cudaFree(d_c);
-  return rc;
+  for (void *p : tmp) cudaFreeAsync(p, st);
+  if (rc == FASTT_OK) rc = timing_end(g, flags, st, n);
+  return call_end(g, flags, st, rc);
 }
 
 fastt_status fastt_stream_info(const fastt_graph *gc_, const fastt_gen_params *gen, const fastt_opts *opts,
@@ -1813,6 +2004,7 @@ fastt_status fastt_stream_info(const fastt_graph *gc_, const fastt_gen_params *g
   if (!g || !gen || !n_split) return fail(FASTT_EINVAL, "NULL argument");
   std::lock_guard<std::mutex> lk(g->mu);
   Dev guard(g->dev);
+  CallGuard cg(g, stream_of(opts));
   StreamCache *S;
   TRY(ensure_stream(g, flags_of(opts), gen->n_pow2_only, stream_of(opts), &S));
   *n_split = S->n_split;
@@ -1826,6 +2018,7 @@ fastt_status fastt_generate_candidates(const fastt_graph *gc_, const fastt_gen_p
   std::lock_guard<std::mutex> lk(g->mu);
   Dev guard(g->dev);
   cudaStream_t st = stream_of(opts);
+  TRY(call_begin(g, st));
   StreamCache *S;
   TRY(ensure_stream(g, flags_of(opts), gen->n_pow2_only, st, &S));
   TRY(check_gen(g, *S, gen, first, n, 1));
@@ -1833,15 +2026,14 @@ fastt_status fastt_generate_candidates(const fastt_graph *gc_, const fastt_gen_p
   StreamState ss = stream_state(g, *S, gen);
   const bool outdev = (flags_of(opts) & FASTT_F_OUT_DEVICE) != 0;
   Cand *d = (Cand *)out;
-  if (!outdev) CK(cudaMalloc(&d, sizeof(Cand) * n));
+  if (!outdev) CK(cudaMallocAsync(&d, sizeof(Cand) * n, st));
   launch_candgen(ss, first, n, d, st);
   CK(cudaGetLastError());
-  CK(cudaStreamSynchronize(st));
   if (!outdev) {
-    CK(cudaMemcpy(out, d, sizeof(Cand) * n, cudaMemcpyDeviceToHost));
-    cudaFree(d);
+    CK(cudaMemcpyAsync(out, d, sizeof(Cand) * n, cudaMemcpyDeviceToHost, st));
+    CK(cudaFreeAsync(d, st));
   }
-  return FASTT_OK;
+  return call_end(g, flags_of(opts), st, FASTT_OK);
 }
 
 fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *gen, const fastt_opts *opts,
@@ -1852,12 +2044,18 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
   std::lock_guard<std::mutex> lk(g->mu);
   Dev guard(g->dev);
   cudaStream_t st = stream_of(opts);
+  host_trace("sweep: enter");
+  TRY(call_begin(g, st));
+  host_trace("sweep: call_begin");
   StreamCache *S;
   TRY(ensure_stream(g, flags, gen->n_pow2_only, st, &S));
   TRY(check_gen(g, *S, gen, first, n, stride));
   Base &B = g->base;
+  host_trace("sweep: stream");
   TRY(ensure_sim(g, B, n, flags));
+  host_trace("sweep: sim");
   if (g->share) TRY(ensure_snapshot(g, B, flags, st));
+  host_trace("sweep: snapshot");
   int64_t nwarps = max_slots(g);  // candidate slots (per-warp bests)
   SimArgs a = sim_args(g, B, flags);
   a.mode = 0;
@@ -1896,13 +2094,16 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
       main_shape(g, B, t, gr, sm);
       wmain = lane_warps(g, t);
     }
+    host_trace("sweep: arena");
     TRY(ensure_overlap(g, B, cap, wmain));
+    host_trace("sweep: overlap bufs");
     nwarps = (int64_t)wmain + cap + 64;
   } else {
     launch_init_best(g->wbest, nwarps, st);
   }
+  // (the non-overlapped path's deferral rounds: arena sized before the launch)
+  if (!ovl && n > 0) TRY(ensure_arena(g, B, st, std::max<int64_t>(256, std::min<int64_t>(g->pin_defer_hint, 8192))));
   TRY(timing_begin(g, flags, st));
-  unsigned long long nd = 0;
   if (n > 0 && ovl) {
     CK(cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), st));
     TRY(ensure_sort_buf(g, n));
@@ -1920,9 +2121,12 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
       size_t sm;
       main_shape(g, B, a, gr, sm);
     }
+    host_trace("sweep: sort");
     TRY(run_overlapped(g, B, a, n, flags, st, false, cap, wmain));
+    host_trace("sweep: overlapped launches");
     timing_mark(g, flags, 2, st);
-    TRY(finish_overlapped(g, B, a, n, st, false, cap, wmain, &nd));
+    TRY(finish_overlapped(g, B, a, n, st, false, cap, wmain));
+    host_trace("sweep: deferral loop");
   } else if (n > 0) {
     CK(cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), st));
     if (a.snap_mode == 2) {
@@ -1945,28 +2149,8 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
     g->launches += NL_SIM;
     CK(cudaGetLastError());
     timing_mark(g, flags, 1, st);
-    CK(cudaMemcpyAsync(&nd, g->counters + 1, sizeof nd, cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    if (nd > 0) {
-      TRY(ensure_arena(g, B, st, (int64_t)nd));
-      for (int64_t c0 = 0; c0 < (int64_t)nd; c0 += g->arena_slots) {
-        int nc = (int)std::min<int64_t>(g->arena_slots, (int64_t)nd - c0);
-        if (a.mode == 3) launch_gather_sorted(g->srt_c, g->srt_i, nullptr, g->defer_q + c0, nc, g->slot_cands,
-                                              g->slot_index, nullptr, st);
-        else launch_candgen_idx(a.stream, first, stride, g->defer_q + c0, nc, g->slot_cands, g->slot_index, st);
-        g->launches += NL_CANDGEN + NL_SIM;
-        TRY(run_prep(g, B, nc, st));
-        CK(cudaMemsetAsync(g->counters, 0, sizeof(unsigned long long), st));
-        SimArgs b = a;
-        b.slots = g->slot_pgs_dev;
-        b.cands = g->slot_cands;
-        b.slot_result = nullptr;
-        b.slot_index = g->slot_index;
-        b.n = nc;
-        launch_slots(g, b, B.tbits, nc, st);
-        CK(cudaGetLastError());
-      }
-    }
+    TRY(run_defer_loop(g, B, a, g->arena_slots, a.mode == 3 ? 0 : 2, false, n, nullptr, &a.stream, first, stride,
+                       false, g->counters + 1, st));
     timing_mark(g, flags, 2, st);
   } else {
     timing_mark(g, flags, 1, st);
@@ -1980,14 +2164,16 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
   } else {
     CK(cudaMemcpyAsync(best, g->best_dev, 16, cudaMemcpyDeviceToHost, st));
   }
-  TRY(timing_end(g, flags, st, n, (int64_t)nd));
+  TRY(timing_end(g, flags, st, n));
   if (ovl && (flags & FASTT_F_TIMING)) {  // the concurrent preparation stream's own duration
     float mp = 0;
     CK(cudaEventElapsedTime(&mp, g->ov_ev[1], g->ov_ev[2]));
     g->last.ms_prep = mp;
   }
-  CK(cudaStreamSynchronize(st));
-  return FASTT_OK;
+  host_trace("sweep: argmin");
+  const fastt_status rc = call_end(g, flags, st, FASTT_OK);
+  host_trace("sweep: exit");
+  return rc;
 }
 
 // materialise an accepted split into a new base with room for one more split
@@ -2045,6 +2231,7 @@ fastt_status fastt_split_search(const fastt_graph *gc_, const fastt_opts *opts, 
   std::lock_guard<std::mutex> lk(g->mu);
   Dev guard(g->dev);
   cudaStream_t st = stream_of(opts);
+  CallGuard cg(g, st);  // (blocking: Alg. 2's accept/stop decisions are taken on the host)
   std::deque<Base> owned;  // bases created by accepted splits (stable addresses)
   Base *cur = &g->base;
   // Alg. 2 line 3: DPOS of the input graph
@@ -2503,6 +2690,16 @@ fastt_status fastt_link_model(int32_t G, const int64_t *alpha, const int64_t *be
     link_beta[k] = kb[k];
   }
   return FASTT_OK;
+}
+
+fastt_status fastt_sync(const fastt_graph *gc_, const fastt_opts *opts) {
+  fastt_graph *g = (fastt_graph *)gc_;
+  if (!g) return fail(FASTT_EINVAL, "NULL argument");
+  std::lock_guard<std::mutex> lk(g->mu);
+  Dev guard(g->dev);
+  cudaStream_t st = stream_of(opts);
+  if (g->done_rec) CK(cudaStreamWaitEvent(st, g->done_ev, 0));
+  return call_end(g, 0, st, FASTT_OK);
 }
 
 fastt_status fastt_last_timing(const fastt_graph *g, fastt_timing *out) {

@@ -330,6 +330,43 @@ void launch_gather_tail(const Cand *src, const int64_t *sidx, const int64_t *sre
 void launch_init_best(int64_t *wb, int64_t nw, cudaStream_t st);
 void launch_gather_sorted(const Cand *src, const int64_t *sidx, const int64_t *sres, const int64_t *qs, int64_t n,
                           Cand *dst, int64_t *didx, int64_t *dres, cudaStream_t st);
+// Device-driven deferral loop (the ABI's asynchronous contract, fastt.h):
+// the candidates a main launch hands to the preparation pipeline -- the
+// tail of a classified sorted list past the arena (phase 0) and the
+// deferral queue defer_q[0 .. *ndefer) (phase 1) -- are gathered into the
+// arena in rounds of at most cap slots by a CUDA-graph WHILE node whose
+// condition the kernels below set on the device, so no host round trip
+// decides how many rounds run.
+struct DeferBlock {
+  // per call (k_defer_setup)
+  int64_t n;            // sorted list length (phase 0 source)
+  int32_t cap;          // arena slots per round
+  int32_t src;          // phase-1 source: 0 sorted list, 1 candidate list (cands), 2 the stream
+  int32_t do_tail;      // phase 0 runs (overlapped path)
+  int32_t results;      // slot_result gets the result index (schedule_batch), else slot_index the stream index
+  const Cand *cands;    // src 1
+  StreamState ss;       // src 2
+  int64_t first, stride;
+  // k_defer_begin
+  int64_t n_main;       // classified main-list length (do_tail), else -1
+  int64_t tail_lo;      // first tail position (n_main + cap)
+  int64_t n_defer;      // *ndefer when the loop starts
+  int64_t total;        // candidates the loop evaluates (tail + deferrals)
+  // cursor (k_defer_plan)
+  int32_t phase;
+  uint32_t nact;        // slots of this round (the preparation kernels' device count)
+  int64_t off;          // consumed entries of the current phase
+  int64_t q_lo, q_cnt;  // this round: positions (phase 0) or defer_q entries (phase 1)
+  int32_t q_phase;      // this round's phase
+};
+void launch_defer_setup(DeferBlock *blk, int64_t n, int cap, int src, int do_tail, int results, const Cand *cands,
+                        const StreamState &ss, int64_t first, int64_t stride, cudaStream_t st);
+void launch_defer_begin(DeferBlock *blk, const uint32_t *n_main, const unsigned long long *ndefer,
+                        cudaGraphConditionalHandle h, cudaStream_t st);
+void launch_defer_plan(DeferBlock *blk, cudaGraphConditionalHandle h, cudaStream_t st);
+void launch_defer_gather(const DeferBlock *blk, int cap, const Cand *srt_c, const int64_t *srt_i,
+                         const int64_t *srt_res, const int64_t *defer_q, Cand *dst, int64_t *didx, int64_t *dres,
+                         cudaStream_t st);
 int sim_occupancy(int tbits, int gshift, int block, size_t smem, bool topo);
 void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st);
 int lane_occupancy(int tbits, int gshift, int mm, bool pk);
@@ -349,5 +386,6 @@ void launch_cost_table(int32_t V, int G, int64_t n, const int32_t *op, const uin
                        void *scratch, unsigned *err, int64_t *cost, int sms, cudaStream_t st);
 cudaError_t sim_set_smem(int tbits, int gshift, size_t smem);
 void launch_fill_i64(int64_t *p, int64_t n, int64_t v, cudaStream_t st);
+void launch_iota_i64(int64_t *p, int64_t n, cudaStream_t st);
 
 }  // namespace fastt

@@ -223,6 +223,112 @@ void launch_gather_tail(const Cand *src, const int64_t *sidx, const int64_t *sre
   const int blocks = (cap + 255) / 256 < 1024 ? (cap + 255) / 256 : 1024;
   k_gather_tail<<<blocks > 0 ? blocks : 1, 256, 0, st>>>(src, sidx, sres, n_main, n, off, cap, dst, didx, dres, nslot);
 }
+// ------------------------------------------------- device deferral loop
+__global__ void k_defer_setup(DeferBlock *b, int64_t n, int cap, int src, int do_tail, int results, const Cand *cands,
+                              StreamState ss, int64_t first, int64_t stride) {
+  b->n = n;
+  b->cap = cap;
+  b->src = src;
+  b->do_tail = do_tail;
+  b->results = results;
+  b->cands = cands;
+  b->ss = ss;
+  b->first = first;
+  b->stride = stride;
+}
+void launch_defer_setup(DeferBlock *blk, int64_t n, int cap, int src, int do_tail, int results, const Cand *cands,
+                        const StreamState &ss, int64_t first, int64_t stride, cudaStream_t st) {
+  k_defer_setup<<<1, 1, 0, st>>>(blk, n, cap, src, do_tail, results, cands, ss, first, stride);
+}
+// the loop's entry: the tail past the arena (the arena held [n_main, n_main
+// + cap)) and the deferral count; the WHILE condition = any work left
+__global__ void k_defer_begin(DeferBlock *b, const uint32_t *n_main, const unsigned long long *ndefer,
+                              cudaGraphConditionalHandle h) {
+  b->n_main = b->do_tail ? (int64_t)*n_main : -1;
+  b->tail_lo = b->do_tail ? b->n_main + b->cap : b->n;
+  if (b->tail_lo > b->n) b->tail_lo = b->n;
+  b->n_defer = (int64_t)*ndefer;
+  b->total = (b->n - b->tail_lo) + b->n_defer;
+  b->phase = b->tail_lo < b->n ? 0 : 1;
+  b->off = 0;
+  b->nact = 0;
+  cudaGraphSetConditional(h, b->total > 0 ? 1u : 0u);
+}
+void launch_defer_begin(DeferBlock *blk, const uint32_t *n_main, const unsigned long long *ndefer,
+                        cudaGraphConditionalHandle h, cudaStream_t st) {
+  k_defer_begin<<<1, 1, 0, st>>>(blk, n_main, ndefer, h);
+}
+// one round: the next at most cap entries; the condition = entries left after it
+__global__ void k_defer_plan(DeferBlock *b, cudaGraphConditionalHandle h) {
+  int64_t lo, cnt;
+  if (b->phase == 0) {
+    lo = b->tail_lo + b->off;
+    cnt = b->n - lo;
+  } else {
+    lo = b->off;
+    cnt = b->n_defer - lo;
+  }
+  if (cnt > b->cap) cnt = b->cap;
+  if (cnt < 0) cnt = 0;
+  b->q_lo = lo;
+  b->q_cnt = cnt;
+  b->q_phase = b->phase;
+  b->nact = (uint32_t)cnt;
+  b->off += cnt;
+  bool more;
+  if (b->phase == 0) {
+    if (b->tail_lo + b->off >= b->n) {  // the tail is done: the deferral queue next
+      b->phase = 1;
+      b->off = 0;
+      more = b->n_defer > 0;
+    } else {
+      more = true;
+    }
+  } else {
+    more = b->off < b->n_defer;
+  }
+  cudaGraphSetConditional(h, more ? 1u : 0u);
+}
+void launch_defer_plan(DeferBlock *blk, cudaGraphConditionalHandle h, cudaStream_t st) {
+  k_defer_plan<<<1, 1, 0, st>>>(blk, h);
+}
+// the round's candidates into the preparation slots (phase 0: sorted
+// positions; phase 1: defer_q entries of the sorted list, the candidate list
+// or the stream)
+__global__ void k_defer_gather(const DeferBlock *b, const Cand *srt_c, const int64_t *srt_i, const int64_t *srt_res,
+                               const int64_t *defer_q, Cand *dst, int64_t *didx, int64_t *dres) {
+  const int64_t cnt = b->q_cnt, lo = b->q_lo;
+  const bool tail = b->q_phase == 0;
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < cnt; k += (int64_t)gridDim.x * blockDim.x) {
+    Cand c;
+    int64_t sidx, res;
+    if (tail || b->src == 0) {
+      const int64_t q = tail ? lo + k : defer_q[lo + k];
+      c = srt_c[q];
+      sidx = srt_i[q];
+      res = srt_res ? srt_res[q] : -1;
+    } else if (b->src == 1) {
+      const int64_t q = defer_q[lo + k];
+      c = b->cands[q];
+      sidx = q;
+      res = q;
+    } else {
+      const int64_t q = defer_q[lo + k];
+      sidx = b->first + q * b->stride;
+      c = stream_cand(b->ss, sidx);
+      res = -1;
+    }
+    dst[k] = c;
+    if (didx) didx[k] = sidx;
+    if (dres) dres[k] = res;
+  }
+}
+void launch_defer_gather(const DeferBlock *blk, int cap, const Cand *srt_c, const int64_t *srt_i,
+                         const int64_t *srt_res, const int64_t *defer_q, Cand *dst, int64_t *didx, int64_t *dres,
+                         cudaStream_t st) {
+  const int blocks = (cap + 255) / 256 < 1024 ? (cap + 255) / 256 : 1024;
+  k_defer_gather<<<blocks > 0 ? blocks : 1, 256, 0, st>>>(blk, srt_c, srt_i, srt_res, defer_q, dst, didx, dres);
+}
 // per-warp best pairs (makespan, index) := (INT64_MAX, -1)
 __global__ void k_init_best(int64_t *wb, int64_t nw) {
   for (int64_t w = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; w < nw; w += (int64_t)gridDim.x * blockDim.x) {
@@ -283,6 +389,12 @@ void launch_argmin(const int64_t *wbest, int64_t nwarps, int64_t *best_dev, cuda
 
 __global__ void k_fill_i64(int64_t *p, int64_t n, int64_t v) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = v;
+}
+__global__ void k_iota_i64(int64_t *p, int64_t n) {
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x) p[k] = k;
+}
+void launch_iota_i64(int64_t *p, int64_t n, cudaStream_t st) {
+  if (n > 0) k_iota_i64<<<(int)((n + 255) / 256 < 1024 ? (n + 255) / 256 : 1024), 256, 0, st>>>(p, n);
 }
 void launch_fill_i64(int64_t *p, int64_t n, int64_t v, cudaStream_t st) {
   if (n <= 0) return;

@@ -66,11 +66,12 @@ class fastt_timing(C.Structure):
 SYMBOLS = ["fastt_load_graph", "fastt_free_graph", "fastt_graph_info", "fastt_rank", "fastt_schedule_batch",
            "fastt_stream_info", "fastt_generate_candidates", "fastt_sweep_best", "fastt_split_search",
            "fastt_free_split_result", "fastt_last_timing", "fastt_last_error", "fastt_version",
-           "fastt_fit_comm", "fastt_link_model", "fastt_cost_table"]
+           "fastt_fit_comm", "fastt_link_model", "fastt_cost_table", "fastt_sync"]
 F_TIMING = 16
 F_SPLIT_BEST = 32
 F_MEM_LIVE = 64
 F_SPLIT_MULTI = 128
+F_ASYNC = 256  # return once enqueued on the stream; Graph.sync() (or the stream) completes it
 
 _lib = None
 
@@ -112,6 +113,8 @@ def lib():
     L.fastt_link_model.argtypes = [i32, P, P, P, P, P, P]
     L.fastt_cost_table.restype = i32
     L.fastt_cost_table.argtypes = [i32, i32, i64, P, P, P, C.c_int, C.POINTER(fastt_opts), P]
+    L.fastt_sync.restype = i32
+    L.fastt_sync.argtypes = [P, C.POINTER(fastt_opts)]
     _lib = L
     return L
 
@@ -282,11 +285,23 @@ class Graph:
         _check(lib().fastt_stream_info(self.h, C.byref(gen), C.byref(o), C.byref(ns)))
         return int(ns.value)
 
-    def generate_candidates(self, gen, first, n, flags=0, stream=None):
-        out = np.zeros(n, CANDIDATE_DTYPE)
-        o = _opts(flags, stream)
+    def generate_candidates(self, gen, first, n, flags=0, stream=None, out=None):
+        """The stream's candidates [first, first + n): numpy records, or into
+        `out` (a torch CUDA uint8 tensor [n, 32]) on the device."""
+        fl = int(flags)
+        if out is None:
+            out = np.zeros(n, CANDIDATE_DTYPE)
+        elif _is_dev(out):
+            fl |= F_OUT_DEVICE
+        o = _opts(fl, stream)
         _check(lib().fastt_generate_candidates(self.h, C.byref(gen), C.byref(o), int(first), int(n), _ptr(out)))
         return out
+
+    def sync(self, stream=None):
+        """fastt_sync: completes every asynchronous call on this graph and
+        reports a deferred device-side error."""
+        o = _opts(0, stream)
+        _check(lib().fastt_sync(self.h, C.byref(o)))
 
     def sweep_best(self, gen, first, n, stride=1, flags=0, stream=None, out=None):
         """Returns (best makespan, best index); with `out` (a torch CUDA int64
