@@ -182,8 +182,11 @@ typedef struct {
 /* Load + encode: validates (acyclic, ranges), merges
  * parallel edges, builds both CSRs, computes the device-side base ranks and
  * priority order.  Supported envelope: G <= 32, K <= 16, in/out degree
- * < 65535, V + largest split overlay <= 32768 ops (EUNSUP beyond: the ready
- * set bitmap of one candidate lives in shared memory); int64 guard
+ * < 65535, V + largest split overlay <= 2^23 ops; above 32,768 ops the base
+ * priority order must be topological (EUNSUP otherwise: the ready-set
+ * kernel's bitmap of one candidate lives in shared memory; a candidate whose
+ * order is not topological on such a graph fails the call, see fastt_sync);
+ * int64 guard
  * sum_i (max cost + G) + sum_e (max comm + copy cost) * (G+2) < 2^58 and
  * sum_i mem * (G+1) < 2^60 (ERANGE beyond; the oracle applies the same rule).
  * cuda_device: the CUDA device ordinal to use. */

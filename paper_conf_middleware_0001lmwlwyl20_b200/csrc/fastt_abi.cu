@@ -195,6 +195,7 @@ struct Base {
     int round_dev = -1;
     char *buf = nullptr;  // dq | avail | ms | rec | rounds | used | used + reserved | keys
     uint32_t *dq = nullptr, *key = nullptr;  // key: the records as packed keys FT << gshift | place (PK)
+    uint32_t *key2 = nullptr;                // the keys doubled (k_lane_pk, two candidates per lane)
     void *avail = nullptr, *ms = nullptr, *rec = nullptr, *used = nullptr, *ur = nullptr;
     int32_t *rounds = nullptr;
   } snap[2];
@@ -271,6 +272,7 @@ struct fastt_graph {
   bool use_rank_reuse = true;  // FASTT_NO_RANK_REUSE=1: SPLIT slots recompute every rank (A/B parity)
   bool use_pk = true;      // FASTT_NO_PK=1: the lane kernel without packed device keys (A/B parity)
   bool use_pk_tma = true;  // FASTT_NO_PK_TMA=1: packed keys on k_sim_lane instead of k_lane_pk (A/B parity)
+  int pk_cpl = 2;          // FASTT_PK_CPL=1: one candidate per lane in the makespan-only k_lane_pk (A/B)
   uint32_t pk_lim_cap = 0xFFFFFFFFu;  // FASTT_PK_LIM=<ns>: lower the deferral bound (tests of the deferral path)
   bool use_lane = true;   // FASTT_NO_LANE=1 keeps position-order launches on the group kernel (A/B parity)
   int last_topo = 0;      // the last main launch: 0 ready-set kernel, 1 group position-order, 2 lane position-order
@@ -307,14 +309,25 @@ struct fastt_graph {
   int64_t *srt_tmp_i = nullptr, *srt_i = nullptr, *srt_res = nullptr;
   uint32_t *srt_key = nullptr, *srt_hist = nullptr;
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+  cudaEvent_t ev_main = nullptr;  // the main launch's start when it waits for the preparation kernels
+  bool ev_main_rec = false;
   // overlapped preparation: the deferred tail of a classified list is
   // prepared and simulated on a high-priority stream while the main launch
   // (non-persistent, on the call's stream) runs
   bool use_overlap = true;  // FASTT_NO_OVERLAP=1 (A/B parity)
-  int lane_batches = 1;     // FASTT_LANE_BATCHES: batches per warp of the non-persistent main launch (0: persistent)
+  int lane_batches = 0;     // FASTT_LANE_BATCHES: batches per warp of a non-persistent main launch (0: persistent)
   int main_bps = 0;         // FASTT_MAIN_BPS: resident blocks per SM of a persistent overlapped main launch (0: all)
+  // FASTT_OVL_MODE: 1 (default) the main launch starts once the preparation
+  // kernels are done and overlaps the slot simulations; 0 it starts at once
+  // (all three run together); 2 main_bps blocks per SM start at once, the
+  // rest after the preparation kernels (measured on C5, 1e6 candidates:
+  // 106 / 108.7 (LANE_BATCHES=2) / 123-179 ms per sweep: a latency-bound
+  // preparation chain co-running with the issue-bound main launch slows by
+  // more than the main launch gains)
+  int ovl_mode = 1;
   cudaStream_t st_prep = nullptr;
-  cudaEvent_t ov_ev[4] = {nullptr, nullptr, nullptr, nullptr};  // classified, prep start, prep done, main done
+  cudaEvent_t ov_ev[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};  // classified, prep start, slots done, prepared, main 2 done
+  cudaStream_t st_main2 = nullptr;  // the second main launch (ovl_mode 2)
   void *slab_mg = nullptr;  // slab columns of the concurrent slot launches
   int64_t slab_mg_cols = 0;
   unsigned long long *counters2 = nullptr;  // work counter of the concurrent slot launches
@@ -323,6 +336,7 @@ struct fastt_graph {
   int32_t slot_bm_bits = 0;
   int64_t wbest_cap = 0;        // wbest entries allocated
   int64_t pin_defer_hint = 256; // rank-changing PINs seen by the last classified call
+  int64_t seq_defer_hint = 256; // deferred candidates of the last sequential (non-overlapped) evaluation
   // device-driven deferral loop (run_defer_loop): a cached CUDA graph with a
   // WHILE node over the preparation rounds, rebuilt when its arguments change
   DeferBlock *dblk = nullptr;
@@ -368,6 +382,8 @@ static fastt_status timing_begin(fastt_graph *g, uint32_t flags, cudaStream_t st
   if (g->counters) CK(cudaMemsetAsync(g->counters + 2, 0, 2 * sizeof(unsigned long long), st));
   for (auto &e : g->ev)
     if (!e) CK(cudaEventCreate(&e));
+  if (!g->ev_main) CK(cudaEventCreate(&g->ev_main));
+  g->ev_main_rec = false;
   CK(cudaEventRecord(g->ev[0], st));
   return FASTT_OK;
 }
@@ -416,7 +432,7 @@ static fastt_status timing_end(fastt_graph *g, uint32_t flags, cudaStream_t st, 
     g->last.lane_steps = (int64_t)ws[1];
   }
   float a = 0, b = 0, c = 0;
-  CK(cudaEventElapsedTime(&a, g->ev[0], g->ev[1]));
+  CK(cudaEventElapsedTime(&a, g->ev_main_rec ? g->ev_main : g->ev[0], g->ev[1]));
   CK(cudaEventElapsedTime(&b, g->ev[1], g->ev[2]));
   CK(cudaEventElapsedTime(&c, g->ev[0], g->ev[3]));
   g->last.ms_sim = a;
@@ -602,6 +618,9 @@ static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st,
   return FASTT_OK;
 }
 
+// candidates per lane of the makespan-only k_lane_pk launch
+static int pk_cpl(const fastt_graph *g) { return g->use_pk_tma && g->pk_cpl == 2 ? 2 : 1; }
+
 static int gshift_of(int G) {
   int gsh = 0;
   while ((1 << gsh) < G) gsh++;
@@ -637,7 +656,8 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     g->sim_grid_topo = g->sms * std::max(1, sim_occupancy(B.tbits, gsh, g->sim_block, 0, true));
     for (int mm = 0; mm < 3; mm++)
       for (int pk = 0; pk < 2; pk++)
-        g->sim_grid_lane[mm][pk] = g->sms * std::max(1, lane_occupancy(B.tbits, gsh, mm, pk != 0));
+        g->sim_grid_lane[mm][pk] =
+            g->sms * std::max(1, lane_occupancy(B.tbits, gsh, mm, pk != 0, mm == 0 && pk ? pk_cpl(g) : 1));
     g->sim_smem = smem;
     g->sim_cpw = cpw;
     g->sim_bm_stride = stride;
@@ -731,6 +751,7 @@ static void main_shape(fastt_graph *g, const Base &B, SimArgs &a, int &grid, siz
     // (the packed-key variant: 32-bit time, one link class, keys prepared)
     const bool pk = B.tbits == 32 && g->K == 1 && a.costk != nullptr && a.pk_lim > 0;
     grid = g->sim_grid_lane[a.lane_mm][pk ? 1 : 0];
+    a.pk_cpl = pk && a.pkc && a.lane_mm == 0 ? pk_cpl(g) : 1;
     smem = 0;
   } else if (topo) {
     a.topo = 1;
@@ -825,7 +846,7 @@ static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cud
   const size_t o_dq = 0, o_av = al16(4 * n), o_ms = o_av + al16(tb * (n + 1) * g->G),
                o_rec = o_ms + al16(tb * (n + 1)), o_rd = o_rec + al16((B.tbits == 32 ? 8 : 16) * n),
                o_us = o_rd + 64, o_ur = o_us + al16(8 * (n + 1) * g->G), o_k = o_ur + al16(8 * (n + 1) * g->G),
-               tot = o_k + al16(4 * n);
+               o_k2 = o_k + al16(4 * n), tot = o_k2 + al16(8 * n);
   CK(cudaMalloc(&S.buf, tot));
   S.dq = (uint32_t *)(S.buf + o_dq);
   S.avail = S.buf + o_av;
@@ -835,6 +856,7 @@ static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cud
   S.used = S.buf + o_us;
   S.ur = S.buf + o_ur;
   S.key = (uint32_t *)(S.buf + o_k);
+  S.key2 = (uint32_t *)(S.buf + o_k2);
   CK(cudaMemsetAsync(S.rounds, 0, 16, st));
   Cand c;
   memset(&c, 0, sizeof c);
@@ -882,7 +904,7 @@ static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cud
   cudaFree(d_st);
   if (hst != FASTT_CAND_OK) return FASTT_OK;  // an infeasible BASE (caps): no sharing
   if (B.tbits == 32) {
-    launch_snap_keys(S.rec, B.n, gshift_of(g->G), S.key, st);
+    launch_snap_keys(S.rec, B.n, gshift_of(g->G), S.key, S.key2, st);
     CK(cudaGetLastError());
   }
   S.round_dev = (rd[0] == 1 && rd[2] == 0 && rd[3] == B.cp_len) ? rd[1] : -1;
@@ -898,6 +920,7 @@ static void use_snapshot(const Base &B, uint32_t flags, SimArgs &a) {
   a.snap_used = S.used;
   a.snap_ur = S.ur;
   a.snap_key = S.key;
+  a.snap_key2 = S.key2;
   a.snap_round_dev = S.round_dev;
   a.snap_dq = S.dq;
   a.snap_avail = S.avail;
@@ -1007,6 +1030,13 @@ static void read_defer_summary(fastt_graph *g) {
   if (!g->dl_sum_pending || cudaEventQuery(g->dl_sum_ev) != cudaSuccess) return;
   g->dl_sum_pending = false;
   if (g->dl_sum->do_tail && g->dl_sum->n_main >= 0) g->pin_defer_hint = g->dl_sum->n - g->dl_sum->n_main;
+  else g->seq_defer_hint = g->dl_sum->n_defer;
+}
+
+// arena slots of a sequential (non-overlapped) evaluation: the last such
+// call's deferral count (one round when the count repeats), at least `lo`
+static int64_t seq_arena_want(const fastt_graph *g, int64_t lo) {
+  return std::max<int64_t>(std::max<int64_t>(256, lo), std::min<int64_t>(g->seq_defer_hint, 8192));
 }
 
 static fastt_status build_defer_graph(fastt_graph *g, Base &B, const SimArgs &b, int cap, bool results,
@@ -1146,6 +1176,7 @@ static fastt_status ensure_overlap(fastt_graph *g, const Base &B, int cap, int w
     int lo = 0, hi = 0;
     CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
     CK(cudaStreamCreateWithPriority(&g->st_prep, cudaStreamNonBlocking, hi));
+    CK(cudaStreamCreateWithFlags(&g->st_main2, cudaStreamNonBlocking));
     for (auto &e : g->ov_ev) CK(cudaEventCreate(&e));
     CK(cudaMalloc(&g->counters2, 2 * sizeof(unsigned long long)));
     CK(cudaMalloc(&g->ov_words, 16));
@@ -1194,6 +1225,7 @@ static fastt_status run_overlapped(fastt_graph *g, Base &B, SimArgs a, int64_t n
                      g->slot_index, results ? g->slot_result : nullptr, g->ov_words + 1, sp);
   g->launches += NL_GATHER;
   TRY(run_prep(g, B, cap, sp, g->ov_words + 1));
+  if (g->ovl_mode >= 1) CK(cudaEventRecord(g->ov_ev[3], sp));  // (prepared: the main launch may start)
   SimArgs b = a;
   b.slots = g->slot_pgs_dev;
   b.cands = g->slot_cands;
@@ -1221,13 +1253,40 @@ static fastt_status run_overlapped(fastt_graph *g, Base &B, SimArgs a, int64_t n
   a.n_slab_slots = wmain;
   int64_t blocks;
   if (g->lane_batches > 0) {
-    const int64_t warps = (n + 31) / 32;
+    const int64_t rw = 32 * (int64_t)std::max(1, a.pk_cpl);  // candidates per warp batch
+    const int64_t warps = (n + rw - 1) / rw;
     blocks = (warps + (int64_t)g->lane_batches * (LANE_BLOCK / 32) - 1) / ((int64_t)g->lane_batches * (LANE_BLOCK / 32));
   } else {  // persistent, optionally leaving block slots to the preparation stream
     blocks = wmain / (LANE_BLOCK / 32);
     if (g->main_bps > 0) blocks = std::min<int64_t>(blocks, (int64_t)g->sms * g->main_bps);
   }
-  launch_sim(a, B.tbits, (int)std::max<int64_t>(1, std::min<int64_t>(blocks, 1 << 30)), LANE_BLOCK, 0, st);
+  if (g->ovl_mode == 2 && g->lane_batches == 0) {
+    // two persistent launches on one work queue: main_bps blocks per SM at
+    // once (beside the preparation kernels), the rest of the resident
+    // blocks once the preparation kernels are done (their own slab columns
+    // and wbest entries: gwarp_off)
+    const int64_t ba = std::min<int64_t>(blocks, (int64_t)g->sms * std::max(1, g->main_bps));
+    a.gwarp_off = 0;
+    launch_sim(a, B.tbits, (int)std::max<int64_t>(1, ba), LANE_BLOCK, 0, st);
+    if (blocks > ba) {
+      CK(cudaStreamWaitEvent(g->st_main2, g->ov_ev[3], 0));
+      SimArgs a2 = a;
+      a2.gwarp_off = (int32_t)(ba * (LANE_BLOCK / 32));
+      launch_sim(a2, B.tbits, (int)(blocks - ba), LANE_BLOCK, 0, g->st_main2);
+      CK(cudaEventRecord(g->ov_ev[4], g->st_main2));
+      CK(cudaStreamWaitEvent(st, g->ov_ev[4], 0));
+      g->launches += NL_SIM;
+    }
+  } else {
+    if (g->ovl_mode == 1) {
+      CK(cudaStreamWaitEvent(st, g->ov_ev[3], 0));
+      if (flags & FASTT_F_TIMING) {  // ms_sim: the main launch's own duration
+        CK(cudaEventRecord(g->ev_main, st));
+        g->ev_main_rec = true;
+      }
+    }
+    launch_sim(a, B.tbits, (int)std::max<int64_t>(1, std::min<int64_t>(blocks, 1 << 30)), LANE_BLOCK, 0, st);
+  }
   g->launches += NL_SIM;
   CK(cudaGetLastError());
   timing_mark(g, flags, 1, st);
@@ -1332,7 +1391,7 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
   }
   // the arena of the deferral rounds (sized before the launch: the count is
   // only known on the device)
-  TRY(ensure_arena(g, B, st, std::max<int64_t>(256, std::min<int64_t>(g->pin_defer_hint, 8192))));
+  TRY(ensure_arena(g, B, st, seq_arena_want(g, 0)));
   if (sorted) {
     // order the list by BASE-prefix start step (results keep their index)
     TRY(ensure_sort_buf(g, n));
@@ -1714,6 +1773,10 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     if (e && e[0]) g->lane_batches = std::max(0, atoi(e));
     e = getenv("FASTT_MAIN_BPS");
     if (e && e[0]) g->main_bps = std::max(0, atoi(e));
+    e = getenv("FASTT_OVL_MODE");
+    if (e && e[0]) g->ovl_mode = atoi(e);
+    e = getenv("FASTT_PK_CPL");
+    if (e && e[0]) g->pk_cpl = atoi(e) == 1 ? 1 : 2;
     e = getenv("FASTT_PK_LIM");
     if (e && e[0]) g->pk_lim_cap = (uint32_t)std::max(1ll, std::min(0xFFFFFFFFll, atoll(e)));
   }
@@ -1822,7 +1885,9 @@ void fastt_free_graph(fastt_graph *g) {
       if (e) cudaEventDestroy(e);
     for (auto &e : g->ov_ev)
       if (e) cudaEventDestroy(e);
+    if (g->ev_main) cudaEventDestroy(g->ev_main);
     if (g->st_prep) cudaStreamDestroy(g->st_prep);
+    if (g->st_main2) cudaStreamDestroy(g->st_main2);
     cudaFree(g->slab_mg);
     cudaFree(g->counters2);
     cudaFree(g->ov_words);
@@ -2102,7 +2167,17 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
     launch_init_best(g->wbest, nwarps, st);
   }
   // (the non-overlapped path's deferral rounds: arena sized before the launch)
-  if (!ovl && n > 0) TRY(ensure_arena(g, B, st, std::max<int64_t>(256, std::min<int64_t>(g->pin_defer_hint, 8192))));
+  if (!ovl && n > 0) {
+    // the window's SPLIT and device-subset candidates are deferred for sure
+    const int64_t hi = a.stream.n_split + a.stream.n_subset;
+    int64_t nsp = 0;
+    if (hi >= 1 && first <= hi) {
+      const int64_t q_lo = first >= 1 ? 0 : (1 - first + stride - 1) / stride;
+      const int64_t q_hi = std::min<int64_t>(n - 1, (hi - first) / stride);
+      nsp = q_hi >= q_lo ? q_hi - q_lo + 1 : 0;
+    }
+    TRY(ensure_arena(g, B, st, seq_arena_want(g, nsp)));
+  }
   TRY(timing_begin(g, flags, st));
   if (n > 0 && ovl) {
     CK(cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), st));

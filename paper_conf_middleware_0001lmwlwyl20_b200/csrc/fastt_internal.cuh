@@ -272,6 +272,11 @@ struct SimArgs {
   // INSERT on the lane kernel: per lane and device gap_cap idle slots
   void *gap_lane;
   int32_t gap_cap;
+  // k_lane_pk with two candidates per lane: the BASE keys doubled ([2n],
+  // key s at words 2s and 2s + 1, so an aligned 8-B load gives it to both)
+  const uint32_t *snap_key2;
+  int32_t pk_cpl;  // candidates per lane of the k_lane_pk launch (1 or 2)
+  int32_t gwarp_off;  // persistent k_lane_pk: first slab column block / wbest entry of this launch
 };
 
 // one idle slot [a, b) of a device under INSERT
@@ -289,7 +294,7 @@ FASTT_DECL_SIM_FN(0) FASTT_DECL_SIM_FN(1) FASTT_DECL_SIM_FN(2) FASTT_DECL_SIM_FN
 FASTT_DECL_SIM_FN(5)
 #undef FASTT_DECL_SIM_FN
 #define FASTT_DECL_LANE_FN(N, M) const void *lane_fn_g##N##_m##M(int tbits, int cm, bool exact, bool mg, bool pk);
-#define FASTT_DECL_PK_FN(N) const void *lane_pk_fn_g##N(int mm, bool exact); \
+#define FASTT_DECL_PK_FN(N) const void *lane_pk_fn_g##N(int mm, bool exact, int cpl); \
   const void *lane_ins_fn_g##N(int tbits, int cm, bool exact);
 FASTT_DECL_PK_FN(0) FASTT_DECL_PK_FN(1) FASTT_DECL_PK_FN(2) FASTT_DECL_PK_FN(3) FASTT_DECL_PK_FN(4) FASTT_DECL_PK_FN(5)
 #undef FASTT_DECL_PK_FN
@@ -369,7 +374,7 @@ void launch_defer_gather(const DeferBlock *blk, int cap, const Cand *srt_c, cons
                          cudaStream_t st);
 int sim_occupancy(int tbits, int gshift, int block, size_t smem, bool topo);
 void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st);
-int lane_occupancy(int tbits, int gshift, int mm, bool pk);
+int lane_occupancy(int tbits, int gshift, int mm, bool pk, int cpl = 1);
 // costk[p][d] = (cost[p][d] << gshift) | d over n positions; mx[0] = max
 // cost, mx[1] = max edge comm (one link class) of the prepared graph
 void launch_pack_costs(const PrepGraph *pg_dev, int32_t n, int G, int gshift, int64_t E, uint32_t *costk,
@@ -377,7 +382,7 @@ void launch_pack_costs(const PrepGraph *pg_dev, int32_t n, int G, int gshift, in
 // words of one compact PK card (k_lane_pk.cuh)
 int pk_card_words_host(int gshift);
 // BASE records (uint32 time: FT | place << 32) -> packed keys FT << gshift | place
-void launch_snap_keys(const void *rec, int32_t n, int gshift, uint32_t *key, cudaStream_t st);
+void launch_snap_keys(const void *rec, int32_t n, int gshift, uint32_t *key, uint32_t *key2, cudaStream_t st);
 void launch_fit(int G, int64_t n, const uint8_t *src, const uint8_t *dst, const int64_t *bytes, const int64_t *tns,
                 void *sums, unsigned *err, int64_t *alpha, int64_t *beta, int64_t *count, int sms, cudaStream_t st);
 size_t fit_sums_bytes(int G);

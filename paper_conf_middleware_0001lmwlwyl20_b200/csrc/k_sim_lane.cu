@@ -129,14 +129,19 @@ void launch_pack_costs(const PrepGraph *pg_dev, int32_t n, int G, int gshift, in
   k_pack_costs<<<148, 256, 0, st>>>(pg_dev, n, G, gshift, E, costk, commk, pkc, pk_card_words(1 << gshift), mx);
 }
 
-__global__ void k_snap_keys(const unsigned long long *rec, int32_t n, int gshift, uint32_t *key) {
+// BASE records as packed keys, and doubled (key2[2p] = key2[2p + 1] =
+// key[p]) for the two-candidates-per-lane kernel
+__global__ void k_snap_keys(const unsigned long long *rec, int32_t n, int gshift, uint32_t *key, uint2 *key2) {
   for (int32_t p = blockIdx.x * blockDim.x + threadIdx.x; p < n; p += gridDim.x * blockDim.x) {
     const unsigned long long w = rec[p];
-    key[p] = ((uint32_t)w << gshift) | (uint32_t)(w >> 32);
+    const uint32_t k = ((uint32_t)w << gshift) | (uint32_t)(w >> 32);
+    key[p] = k;
+    key2[p] = make_uint2(k, k);
   }
 }
-void launch_snap_keys(const void *rec, int32_t n, int gshift, uint32_t *key, cudaStream_t st) {
-  if (n > 0) k_snap_keys<<<(n + 255) / 256, 256, 0, st>>>((const unsigned long long *)rec, n, gshift, key);
+void launch_snap_keys(const void *rec, int32_t n, int gshift, uint32_t *key, uint32_t *key2, cudaStream_t st) {
+  if (n > 0)
+    k_snap_keys<<<(n + 255) / 256, 256, 0, st>>>((const unsigned long long *)rec, n, gshift, key, (uint2 *)key2);
 }
 
 int lane_comm_mode(const SimArgs &a, int tbits) {
@@ -147,28 +152,29 @@ int lane_comm_mode(const SimArgs &a, int tbits) {
 // a.lane: 1 = candidates of the base graph (LANE_BLOCK threads per block),
 // 2 = prepared slots, one per lane (one warp per block; grid = warps)
 // the packed-key kernel k_lane_pk (k_lane_pk.cuh) and its shared memory
-static const void *lane_pk_fn(int gshift, int mm, bool exact) {
+static const void *lane_pk_fn(int gshift, int mm, bool exact, int cpl) {
   switch (gshift) {
-    case 0: return lane_pk_fn_g0(mm, exact);
-    case 1: return lane_pk_fn_g1(mm, exact);
-    case 2: return lane_pk_fn_g2(mm, exact);
-    case 3: return lane_pk_fn_g3(mm, exact);
-    case 4: return lane_pk_fn_g4(mm, exact);
-    default: return lane_pk_fn_g5(mm, exact);
+    case 0: return lane_pk_fn_g0(mm, exact, cpl);
+    case 1: return lane_pk_fn_g1(mm, exact, cpl);
+    case 2: return lane_pk_fn_g2(mm, exact, cpl);
+    case 3: return lane_pk_fn_g3(mm, exact, cpl);
+    case 4: return lane_pk_fn_g4(mm, exact, cpl);
+    default: return lane_pk_fn_g5(mm, exact, cpl);
   }
 }
-template <int GP> static size_t pk_smem_w(int mm) {
+template <int GP> static size_t pk_smem_w(int mm, int cpl) {
+  if (cpl == 2) return pk_smem_per_warp<GP, 0, 2>();
   return mm == 0 ? pk_smem_per_warp<GP, 0>() : mm == 1 ? pk_smem_per_warp<GP, 1>() : pk_smem_per_warp<GP, 2>();
 }
-static size_t lane_pk_smem(int gshift, int mm) {
+static size_t lane_pk_smem(int gshift, int mm, int cpl) {
   size_t w;
   switch (gshift) {
-    case 0: w = pk_smem_w<1>(mm); break;
-    case 1: w = pk_smem_w<2>(mm); break;
-    case 2: w = pk_smem_w<4>(mm); break;
-    case 3: w = pk_smem_w<8>(mm); break;
-    case 4: w = pk_smem_w<16>(mm); break;
-    default: w = pk_smem_w<32>(mm); break;
+    case 0: w = pk_smem_w<1>(mm, cpl); break;
+    case 1: w = pk_smem_w<2>(mm, cpl); break;
+    case 2: w = pk_smem_w<4>(mm, cpl); break;
+    case 3: w = pk_smem_w<8>(mm, cpl); break;
+    case 4: w = pk_smem_w<16>(mm, cpl); break;
+    default: w = pk_smem_w<32>(mm, cpl); break;
   }
   return (LANE_BLOCK / 32) * w;
 }
@@ -198,8 +204,9 @@ void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
   }
   const bool pk = !mg && tbits == 32 && cm != 2 && a.costk != nullptr && a.pk_lim > 0;
   if (pk && a.pkc) {  // the base-graph sweep kernel: TMA-staged packed-key cards
-    const void *f = lane_pk_fn(a.gshift, a.lane_mm, a.G == (1 << a.gshift));
-    const size_t sm = lane_pk_smem(a.gshift, a.lane_mm);
+    const int cpl = a.pk_cpl == 2 && a.lane_mm == 0 ? 2 : 1;
+    const void *f = lane_pk_fn(a.gshift, a.lane_mm, a.G == (1 << a.gshift), cpl);
+    const size_t sm = lane_pk_smem(a.gshift, a.lane_mm, cpl);
     SimArgs aa = a;
     void *args[] = {&aa};
     cudaLaunchKernel(f, dim3(grid), dim3(LANE_BLOCK), args, sm, st);
@@ -216,13 +223,14 @@ void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
 // resident blocks per SM of the base-graph launch of memory mode mm and
 // packed keys pk (the minimum over the comm / exactness variants); sets their
 // dynamic shared memory limit
-int lane_occupancy(int tbits, int gshift, int mm, bool pk) {
+int lane_occupancy(int tbits, int gshift, int mm, bool pk, int cpl) {
   int nb = 1 << 30, x = 0;
   if (pk && tbits != 32) return 0;
   if (pk) {  // k_lane_pk
-    const size_t sm = lane_pk_smem(gshift, mm);
+    if (mm != 0) cpl = 1;
+    const size_t sm = lane_pk_smem(gshift, mm, cpl);
     for (int ex = 0; ex < 2; ex++) {
-      const void *f = lane_pk_fn(gshift, mm, ex != 0);
+      const void *f = lane_pk_fn(gshift, mm, ex != 0, cpl);
       cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, f, LANE_BLOCK, sm);
       nb = x < nb ? x : nb;
