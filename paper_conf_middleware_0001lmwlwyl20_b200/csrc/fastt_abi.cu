@@ -273,6 +273,7 @@ struct fastt_graph {
   bool use_pk = true;      // FASTT_NO_PK=1: the lane kernel without packed device keys (A/B parity)
   bool use_pk_tma = true;  // FASTT_NO_PK_TMA=1: packed keys on k_sim_lane instead of k_lane_pk (A/B parity)
   int pk_cpl = 2;          // FASTT_PK_CPL=1: one candidate per lane in the makespan-only k_lane_pk (A/B)
+  bool pk_cpl_peak = false;  // FASTT_PK_CPL_PEAK=1: two per lane with per-device peak memory too
   uint32_t pk_lim_cap = 0xFFFFFFFFu;  // FASTT_PK_LIM=<ns>: lower the deferral bound (tests of the deferral path)
   bool use_lane = true;   // FASTT_NO_LANE=1 keeps position-order launches on the group kernel (A/B parity)
   int last_topo = 0;      // the last main launch: 0 ready-set kernel, 1 group position-order, 2 lane position-order
@@ -618,8 +619,13 @@ static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st,
   return FASTT_OK;
 }
 
-// candidates per lane of the makespan-only k_lane_pk launch
-static int pk_cpl(const fastt_graph *g) { return g->use_pk_tma && g->pk_cpl == 2 ? 2 : 1; }
+// candidates per lane of a k_lane_pk launch in memory mode mm: two for
+// makespan-only sweeps; with per-device peak memory (mm 1) only on request
+// (FASTT_PK_CPL_PEAK=1: its 4 KB more shared memory per warp leave 2 blocks
+// per SM, measured 101.5 vs 90.8 ms for one candidate per lane on C5)
+static int pk_cpl(const fastt_graph *g, int mm) {
+  return g->use_pk_tma && g->pk_cpl == 2 && (mm == 0 || (mm == 1 && g->pk_cpl_peak)) ? 2 : 1;
+}
 
 static int gshift_of(int G) {
   int gsh = 0;
@@ -657,7 +663,7 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     for (int mm = 0; mm < 3; mm++)
       for (int pk = 0; pk < 2; pk++)
         g->sim_grid_lane[mm][pk] =
-            g->sms * std::max(1, lane_occupancy(B.tbits, gsh, mm, pk != 0, mm == 0 && pk ? pk_cpl(g) : 1));
+            g->sms * std::max(1, lane_occupancy(B.tbits, gsh, mm, pk != 0, pk ? pk_cpl(g, mm) : 1));
     g->sim_smem = smem;
     g->sim_cpw = cpw;
     g->sim_bm_stride = stride;
@@ -751,7 +757,7 @@ static void main_shape(fastt_graph *g, const Base &B, SimArgs &a, int &grid, siz
     // (the packed-key variant: 32-bit time, one link class, keys prepared)
     const bool pk = B.tbits == 32 && g->K == 1 && a.costk != nullptr && a.pk_lim > 0;
     grid = g->sim_grid_lane[a.lane_mm][pk ? 1 : 0];
-    a.pk_cpl = pk && a.pkc && a.lane_mm == 0 ? pk_cpl(g) : 1;
+    a.pk_cpl = pk && a.pkc ? pk_cpl(g, a.lane_mm) : 1;
     smem = 0;
   } else if (topo) {
     a.topo = 1;
@@ -1773,6 +1779,8 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     if (e && e[0]) g->lane_batches = std::max(0, atoi(e));
     e = getenv("FASTT_MAIN_BPS");
     if (e && e[0]) g->main_bps = std::max(0, atoi(e));
+    e = getenv("FASTT_PK_CPL_PEAK");
+    g->pk_cpl_peak = e && e[0] == '1';
     e = getenv("FASTT_OVL_MODE");
     if (e && e[0]) g->ovl_mode = atoi(e);
     e = getenv("FASTT_PK_CPL");

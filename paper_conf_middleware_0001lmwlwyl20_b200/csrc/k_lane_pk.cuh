@@ -53,7 +53,7 @@ template <int GP, int MM, int CPL = 1> __host__ __device__ constexpr size_t pk_m
          (size_t)PK_CR * pk_card_bytes(GP) + (size_t)32 * GP * 4 * CPL;
 }
 template <int GP, int MM, int CPL = 1> __host__ __device__ constexpr size_t pk_smem_per_warp() {
-  return pk_mm_off<GP, MM, CPL>() + (MM >= 1 ? (size_t)32 * GP * 8 : 0) + (MM == 2 ? (size_t)32 * GP * 8 : 0);
+  return pk_mm_off<GP, MM, CPL>() + (MM >= 1 ? (size_t)32 * GP * 8 * CPL : 0) + (MM == 2 ? (size_t)32 * GP * 8 : 0);
 }
 
 __device__ __forceinline__ void mbar_init(uint32_t a, uint32_t count) {
@@ -95,7 +95,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, CPL == 1 ? LANE_MINB : 3) k_lane_p
   constexpr int CB = pk_card_bytes(GP);
   constexpr int RW = 32 * CPL;  // keys per record row
   static_assert((D & (D - 1)) == 0 && CB % 16 == 0, "pipeline slots");
-  static_assert(CPL == 1 || (CPL == 2 && MM == 0), "two candidates per lane: makespan-only mode");
+  static_assert(CPL == 1 || (CPL == 2 && MM <= 1), "two candidates per lane: makespan (+ peak memory)");
   const int lane = threadIdx.x & 31;
   int64_t gwarp = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5) + a.gwarp_off;
   if (a.lane_batches > 0) {
@@ -145,7 +145,9 @@ __global__ void __launch_bounds__(LANE_BLOCK, CPL == 1 ? LANE_MINB : 3) k_lane_p
   auto avk_at = [&](int j, uint32_t d) -> uint32_t & {
     return GP >= 2 ? avk_j(j)[(d >> 1) * 64 + (d & 1)] : avk_j(j)[0];
   };
+  // memory state (MM >= 1) of candidate j: mv_j(j)[d * 32]
   int64_t *const mv = (int64_t *)(wsm + pk_mm_off<GP, MM, CPL>()) + lane;
+  auto mv_j = [&](int j) -> int64_t * { return mv + j * 32 * GP; };
   uint32_t *const s32b =
       (uint32_t *)(wsm + pk_mm_off<GP, MM, CPL>() + (size_t)32 * GP * 8) + (GP >= 4 ? 4 * lane : lane);
   uint32_t *const rnd = (uint32_t *)(wsm + pk_mm_off<GP, MM, CPL>() + (size_t)32 * GP * 12) + lane;
@@ -254,7 +256,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, CPL == 1 ? LANE_MINB : 3) k_lane_p
       dead[j] = false;
       if (MM && run[j]) {
 #pragma unroll
-        for (int d = 0; d < GP; d++) mv[d * 32] = (MM == 2 && d < G) ? gc.cap[d] : 0;
+        for (int d = 0; d < GP; d++) mv_j(j)[d * 32] = (MM == 2 && d < G) ? gc.cap[d] : 0;
       }
       if (run[j] && cp_on && cpl > 0) {
         uint32_t pc[MAXPINS];
@@ -331,7 +333,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, CPL == 1 ? LANE_MINB : 3) k_lane_p
           if (d < G) avk_at(j, d) = __ldg(sa + d) << GSH;
         ms[j] = __ldg((const uint32_t *)a.snap_ms + lo);
         if (MM == 1)
-          for (int d = 0; d < G; d++) mv[d * 32] = __ldg((const int64_t *)a.snap_used + (size_t)lo * G + d);
+          for (int d = 0; d < G; d++) mv_j(j)[d * 32] = __ldg((const int64_t *)a.snap_used + (size_t)lo * G + d);
         if (MM == 2)
           for (int d = 0; d < G; d++)
             mv[d * 32] = gc.cap[d] - __ldg((const int64_t *)a.snap_ur + (size_t)lo * G + d);
@@ -590,7 +592,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, CPL == 1 ? LANE_MINB : 3) k_lane_p
         rec[j] = bk[j];
         if (go) {
           const uint32_t dc = bk[j] & GMK;
-          if (MM == 1) mv[dc * 32] += mem64;
+          if (MM == 1) mv_j(j)[dc * 32] += mem64;
           if (MM == 2 && !cpf[j]) {
             const int64_t v = mv[dc * 32] - mem64;
             mv[dc * 32] = v;
@@ -631,7 +633,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, CPL == 1 ? LANE_MINB : 3) k_lane_p
           a.out.status[res_idx[j]] = dead[j] ? 1 : 0;
           if (MM && a.out.peak)
             for (int d = 0; d < G; d++)
-              a.out.peak[res_idx[j] * G + d] = dead[j] ? -1 : (MM == 1 ? mv[d * 32] : gc.cap[d] - mv[d * 32]);
+              a.out.peak[res_idx[j] * G + d] = dead[j] ? -1 : (MM == 1 ? mv_j(j)[d * 32] : gc.cap[d] - mv[d * 32]);
         }
         if (!dead[j] && ((int64_t)ms[j] < bms || ((int64_t)ms[j] == bms && sidx[j] < bidx))) {
           bms = (int64_t)ms[j];

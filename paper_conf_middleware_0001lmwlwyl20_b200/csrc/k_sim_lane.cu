@@ -163,7 +163,7 @@ static const void *lane_pk_fn(int gshift, int mm, bool exact, int cpl) {
   }
 }
 template <int GP> static size_t pk_smem_w(int mm, int cpl) {
-  if (cpl == 2) return pk_smem_per_warp<GP, 0, 2>();
+  if (cpl == 2 && mm <= 1) return mm == 0 ? pk_smem_per_warp<GP, 0, 2>() : pk_smem_per_warp<GP, 1, 2>();
   return mm == 0 ? pk_smem_per_warp<GP, 0>() : mm == 1 ? pk_smem_per_warp<GP, 1>() : pk_smem_per_warp<GP, 2>();
 }
 static size_t lane_pk_smem(int gshift, int mm, int cpl) {
@@ -204,7 +204,7 @@ void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
   }
   const bool pk = !mg && tbits == 32 && cm != 2 && a.costk != nullptr && a.pk_lim > 0;
   if (pk && a.pkc) {  // the base-graph sweep kernel: TMA-staged packed-key cards
-    const int cpl = a.pk_cpl == 2 && a.lane_mm == 0 ? 2 : 1;
+    const int cpl = a.pk_cpl == 2 && a.lane_mm <= 1 ? 2 : 1;
     const void *f = lane_pk_fn(a.gshift, a.lane_mm, a.G == (1 << a.gshift), cpl);
     const size_t sm = lane_pk_smem(a.gshift, a.lane_mm, cpl);
     SimArgs aa = a;
@@ -227,7 +227,7 @@ int lane_occupancy(int tbits, int gshift, int mm, bool pk, int cpl) {
   int nb = 1 << 30, x = 0;
   if (pk && tbits != 32) return 0;
   if (pk) {  // k_lane_pk
-    if (mm != 0) cpl = 1;
+    if (mm > 1) cpl = 1;
     const size_t sm = lane_pk_smem(gshift, mm, cpl);
     for (int ex = 0; ex < 2; ex++) {
       const void *f = lane_pk_fn(gshift, mm, ex != 0, cpl);

@@ -31,8 +31,9 @@ SHAPES = [
     {"FASTT_PK_CPL": "2", "FASTT_OVL_MODE": "2", "FASTT_LANE_BATCHES": "0", "FASTT_MAIN_BPS": "1"},
     {"FASTT_PK_CPL": "1", "FASTT_OVL_MODE": "2", "FASTT_LANE_BATCHES": "0", "FASTT_MAIN_BPS": "2"},
     {"FASTT_PK_CPL": "2", "FASTT_NO_OVERLAP": "1"},
+    {"FASTT_PK_CPL": "2", "FASTT_PK_CPL_PEAK": "1"},
 ]
-KEYS = ("FASTT_PK_CPL", "FASTT_OVL_MODE", "FASTT_LANE_BATCHES", "FASTT_MAIN_BPS", "FASTT_NO_OVERLAP")
+KEYS = ("FASTT_PK_CPL", "FASTT_OVL_MODE", "FASTT_LANE_BATCHES", "FASTT_MAIN_BPS", "FASTT_NO_OVERLAP", "FASTT_PK_CPL_PEAK")
 
 
 def _graph(desc, env):
@@ -54,16 +55,19 @@ def _graph(desc, env):
 def test_shapes_agree(cfg, n):
     desc = synth.config(cfg)
     gen = F.gen_params(seed=0xFA57)
-    ref_best = ref_ms = None
+    ref_best = ref_ms = ref_peak = None
     for env in SHAPES:
         g = _graph(desc, env)
         ns = g.stream_info(gen, flags=F.F_CP_PIN)
         best = g.sweep_best(gen, 0, n, flags=F.F_CP_PIN)
         cands = g.generate_candidates(gen, 0, min(n, ns + 20_000), flags=F.F_CP_PIN)
         ms = g.schedule_batch(cands, flags=F.F_CP_PIN, peak=False)["makespan"]
+        rp = g.schedule_batch(cands, flags=F.F_CP_PIN, peak=True)  # (memory mode 1 of the lane kernel)
+        assert np.array_equal(rp["makespan"], ms), env
         if ref_best is None:
-            ref_best, ref_ms = best, ms
+            ref_best, ref_ms, ref_peak = best, ms, rp["peak_mem"]
             c = g.generate_candidates(gen, best[1], 1, flags=F.F_CP_PIN)
             assert O.OracleGraph(desc).schedule(c[0], flags=O.F_CP_PIN, outputs=False)["makespan"] == best[0]
         assert best == ref_best, env
         assert np.array_equal(ms, ref_ms), env
+        assert np.array_equal(rp["peak_mem"], ref_peak), env
