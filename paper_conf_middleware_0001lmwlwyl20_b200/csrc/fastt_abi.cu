@@ -263,6 +263,8 @@ struct fastt_graph {
   bool use_topo = true;   // FASTT_NO_TOPO=1 forces the ready-set path (A/B parity)
   // resident blocks of the lane-per-candidate kernel per memory mode and packed keys
   int sim_grid_lane[3][2] = {{0, 0}, {0, 0}, {0, 0}};
+  int lane_wpb[3][2] = {{4, 4}, {4, 4}, {4, 4}};  // warps per block of those launches (k_lane_pk: 1, 2 or 4)
+  int pk_wpb_env = 0;  // FASTT_PK_WPB: force k_lane_pk's warps per block
   // device staging buffers of fastt_schedule_batch (host candidates in,
   // makespan/status out), kept across calls and grown on demand
   struct IoBuf {
@@ -273,7 +275,7 @@ struct fastt_graph {
   bool use_pk = true;      // FASTT_NO_PK=1: the lane kernel without packed device keys (A/B parity)
   bool use_pk_tma = true;  // FASTT_NO_PK_TMA=1: packed keys on k_sim_lane instead of k_lane_pk (A/B parity)
   int pk_cpl = 2;          // FASTT_PK_CPL=1: one candidate per lane in the makespan-only k_lane_pk (A/B)
-  bool pk_cpl_peak = false;  // FASTT_PK_CPL_PEAK=1: two per lane with per-device peak memory too
+  bool pk_cpl_peak = true;  // FASTT_PK_CPL_PEAK=0: one per lane with per-device peak memory
   uint32_t pk_lim_cap = 0xFFFFFFFFu;  // FASTT_PK_LIM=<ns>: lower the deferral bound (tests of the deferral path)
   bool use_lane = true;   // FASTT_NO_LANE=1 keeps position-order launches on the group kernel (A/B parity)
   int last_topo = 0;      // the last main launch: 0 ready-set kernel, 1 group position-order, 2 lane position-order
@@ -593,8 +595,9 @@ static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st,
   size_t freeb = 0, totb = 0;
   CK(cudaMemGetInfo(&freeb, &totb));
   size_t per = rt + pt;
-  // at most 40 % of the free and 25 % of the total device memory per graph
-  int64_t slots = std::min<int64_t>(want, (int64_t)(std::min(freeb * 2 / 5, totb / 4) / per));
+  // at most 60 % of the free and 30 % of the total device memory per graph
+  // (a wave that does not fit costs one more latency-bound preparation round)
+  int64_t slots = std::min<int64_t>(want, (int64_t)(std::min(freeb * 3 / 5, totb * 3 / 10) / per));
   if (slots < 1) return fail(FASTT_ENOMEM, "device memory too small for one preparation slot (%zu bytes)", per);
   g->arena_slots = (int)slots;
   CK(cudaMalloc(&g->arena, per * slots));
@@ -620,9 +623,10 @@ static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st,
 }
 
 // candidates per lane of a k_lane_pk launch in memory mode mm: two for
-// makespan-only sweeps; with per-device peak memory (mm 1) only on request
-// (FASTT_PK_CPL_PEAK=1: its 4 KB more shared memory per warp leave 2 blocks
-// per SM, measured 101.5 vs 90.8 ms for one candidate per lane on C5)
+// makespan-only sweeps and with per-device peak memory (mm 1; FASTT_PK_CPL_PEAK=0
+// keeps one: its 4 KB more shared memory per warp need blocks of 1-2 warps to
+// keep 10 warps per SM, measured 88.9 vs 90.8 ms for one candidate per lane
+// on C5, 101.5 ms with 4-warp blocks)
 static int pk_cpl(const fastt_graph *g, int mm) {
   return g->use_pk_tma && g->pk_cpl == 2 && (mm == 0 || (mm == 1 && g->pk_cpl_peak)) ? 2 : 1;
 }
@@ -661,16 +665,34 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
     g->sim_grid = g->sms * per_sm;
     g->sim_grid_topo = g->sms * std::max(1, sim_occupancy(B.tbits, gsh, g->sim_block, 0, true));
     for (int mm = 0; mm < 3; mm++)
-      for (int pk = 0; pk < 2; pk++)
-        g->sim_grid_lane[mm][pk] =
-            g->sms * std::max(1, lane_occupancy(B.tbits, gsh, mm, pk != 0, pk ? pk_cpl(g, mm) : 1));
+      for (int pk = 0; pk < 2; pk++) {
+        // k_lane_pk: the block size (1, 2 or 4 warps) with the most resident
+        // warps (its shared memory per warp need not divide an SM's by 4)
+        int best_w = 4, best_b = std::max(1, lane_occupancy(B.tbits, gsh, mm, pk != 0, pk ? pk_cpl(g, mm) : 1, 4));
+        if (pk && B.tbits == 32)
+          for (int w : {2, 1}) {
+            if (g->pk_wpb_env > 0 && w != g->pk_wpb_env) continue;
+            const int b = lane_occupancy(B.tbits, gsh, mm, true, pk_cpl(g, mm), w);
+            if (b * w > best_b * best_w || (g->pk_wpb_env == w && b > 0)) {
+              best_b = b;
+              best_w = w;
+            }
+          }
+        g->sim_grid_lane[mm][pk] = g->sms * best_b;
+        g->lane_wpb[mm][pk] = best_w;
+        if (getenv("FASTT_HOST_TRACE")) {
+          char msg[96];
+          snprintf(msg, sizeof msg, "lane launch mm %d pk %d: %d blocks/SM x %d warps", mm, pk, best_b, best_w);
+          host_trace(msg);
+        }
+      }
     g->sim_smem = smem;
     g->sim_cpw = cpw;
     g->sim_bm_stride = stride;
     int64_t nslot = (int64_t)std::max(g->sim_grid, g->sim_grid_topo) * (g->sim_block / 32) * cpw;
     for (int mm = 0; mm < 3; mm++)
       for (int pk = 0; pk < 2; pk++)
-        nslot = std::max<int64_t>(nslot, (int64_t)g->sim_grid_lane[mm][pk] * LANE_BLOCK);  // one column per lane
+        nslot = std::max<int64_t>(nslot, (int64_t)g->sim_grid_lane[mm][pk] * 32 * g->lane_wpb[mm][pk]);  // a column per lane
     size_t rec = B.tbits == 32 ? 8 : 16;
     CK(cudaMalloc(&g->slab, (size_t)nslot * ncap * rec));
     CK(cudaMalloc(&g->wbest, sizeof(int64_t) * 2 * nslot));
@@ -758,6 +780,7 @@ static void main_shape(fastt_graph *g, const Base &B, SimArgs &a, int &grid, siz
     const bool pk = B.tbits == 32 && g->K == 1 && a.costk != nullptr && a.pk_lim > 0;
     grid = g->sim_grid_lane[a.lane_mm][pk ? 1 : 0];
     a.pk_cpl = pk && a.pkc ? pk_cpl(g, a.lane_mm) : 1;
+    a.pk_wpb = g->lane_wpb[a.lane_mm][pk ? 1 : 0];
     smem = 0;
   } else if (topo) {
     a.topo = 1;
@@ -770,9 +793,10 @@ static void main_shape(fastt_graph *g, const Base &B, SimArgs &a, int &grid, siz
   }
 }
 static int max_slots(const fastt_graph *g) {
-  int gl = 0;
-  for (int mm = 0; mm < 3; mm++) gl = std::max(gl, std::max(g->sim_grid_lane[mm][0], g->sim_grid_lane[mm][1]));
-  return std::max(std::max(g->sim_grid, g->sim_grid_topo) * (g->sim_block / 32) * g->sim_cpw, gl * (LANE_BLOCK / 32));
+  int gl = 0;  // resident warps of the lane launches
+  for (int mm = 0; mm < 3; mm++)
+    for (int pk = 0; pk < 2; pk++) gl = std::max(gl, g->sim_grid_lane[mm][pk] * g->lane_wpb[mm][pk]);
+  return std::max(std::max(g->sim_grid, g->sim_grid_topo) * (g->sim_block / 32) * g->sim_cpw, gl);
 }
 
 static SimArgs sim_args(fastt_graph *g, const Base &B, uint32_t flags) {
@@ -1212,7 +1236,9 @@ static fastt_status ensure_overlap(fastt_graph *g, const Base &B, int cap, int w
 }
 
 // resident warps of the main lane launch (its slab slots and wbest entries)
-static int lane_warps(const fastt_graph *g, const SimArgs &a) { return g->sim_grid_lane[a.lane_mm][1] * (LANE_BLOCK / 32); }
+static int lane_warps(const fastt_graph *g, const SimArgs &a) {
+  return g->sim_grid_lane[a.lane_mm][1] * g->lane_wpb[a.lane_mm][1];
+}
 
 // the overlapped launches after the classified sort (a: the main launch's
 // arguments, mode 3 over g->srt_*); results: per-candidate outputs through
@@ -1261,9 +1287,10 @@ static fastt_status run_overlapped(fastt_graph *g, Base &B, SimArgs a, int64_t n
   if (g->lane_batches > 0) {
     const int64_t rw = 32 * (int64_t)std::max(1, a.pk_cpl);  // candidates per warp batch
     const int64_t warps = (n + rw - 1) / rw;
-    blocks = (warps + (int64_t)g->lane_batches * (LANE_BLOCK / 32) - 1) / ((int64_t)g->lane_batches * (LANE_BLOCK / 32));
+    const int64_t wpb = std::max(1, a.pk_wpb);
+    blocks = (warps + (int64_t)g->lane_batches * wpb - 1) / ((int64_t)g->lane_batches * wpb);
   } else {  // persistent, optionally leaving block slots to the preparation stream
-    blocks = wmain / (LANE_BLOCK / 32);
+    blocks = wmain / std::max(1, a.pk_wpb);
     if (g->main_bps > 0) blocks = std::min<int64_t>(blocks, (int64_t)g->sms * g->main_bps);
   }
   if (g->ovl_mode == 2 && g->lane_batches == 0) {
@@ -1277,7 +1304,7 @@ static fastt_status run_overlapped(fastt_graph *g, Base &B, SimArgs a, int64_t n
     if (blocks > ba) {
       CK(cudaStreamWaitEvent(g->st_main2, g->ov_ev[3], 0));
       SimArgs a2 = a;
-      a2.gwarp_off = (int32_t)(ba * (LANE_BLOCK / 32));
+      a2.gwarp_off = (int32_t)(ba * std::max(1, a.pk_wpb));
       launch_sim(a2, B.tbits, (int)(blocks - ba), LANE_BLOCK, 0, g->st_main2);
       CK(cudaEventRecord(g->ov_ev[4], g->st_main2));
       CK(cudaStreamWaitEvent(st, g->ov_ev[4], 0));
@@ -1779,8 +1806,10 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     if (e && e[0]) g->lane_batches = std::max(0, atoi(e));
     e = getenv("FASTT_MAIN_BPS");
     if (e && e[0]) g->main_bps = std::max(0, atoi(e));
+    e = getenv("FASTT_PK_WPB");
+    if (e && e[0]) g->pk_wpb_env = (atoi(e) == 1 || atoi(e) == 2) ? atoi(e) : 4;
     e = getenv("FASTT_PK_CPL_PEAK");
-    g->pk_cpl_peak = e && e[0] == '1';
+    if (e && e[0]) g->pk_cpl_peak = e[0] == '1';
     e = getenv("FASTT_OVL_MODE");
     if (e && e[0]) g->ovl_mode = atoi(e);
     e = getenv("FASTT_PK_CPL");

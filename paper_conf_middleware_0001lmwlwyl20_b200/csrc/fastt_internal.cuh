@@ -277,6 +277,7 @@ struct SimArgs {
   const uint32_t *snap_key2;
   int32_t pk_cpl;  // candidates per lane of the k_lane_pk launch (1 or 2)
   int32_t gwarp_off;  // persistent k_lane_pk: first slab column block / wbest entry of this launch
+  int32_t pk_wpb;     // k_lane_pk: warps per block (1, 2 or 4; 0 = 4)
 };
 
 // one idle slot [a, b) of a device under INSERT
@@ -374,7 +375,7 @@ void launch_defer_gather(const DeferBlock *blk, int cap, const Cand *srt_c, cons
                          cudaStream_t st);
 int sim_occupancy(int tbits, int gshift, int block, size_t smem, bool topo);
 void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st);
-int lane_occupancy(int tbits, int gshift, int mm, bool pk, int cpl = 1);
+int lane_occupancy(int tbits, int gshift, int mm, bool pk, int cpl = 1, int wpb = 4);
 // costk[p][d] = (cost[p][d] << gshift) | d over n positions; mx[0] = max
 // cost, mx[1] = max edge comm (one link class) of the prepared graph
 void launch_pack_costs(const PrepGraph *pg_dev, int32_t n, int G, int gshift, int64_t E, uint32_t *costk,

@@ -166,7 +166,7 @@ template <int GP> static size_t pk_smem_w(int mm, int cpl) {
   if (cpl == 2 && mm <= 1) return mm == 0 ? pk_smem_per_warp<GP, 0, 2>() : pk_smem_per_warp<GP, 1, 2>();
   return mm == 0 ? pk_smem_per_warp<GP, 0>() : mm == 1 ? pk_smem_per_warp<GP, 1>() : pk_smem_per_warp<GP, 2>();
 }
-static size_t lane_pk_smem(int gshift, int mm, int cpl) {
+static size_t lane_pk_smem(int gshift, int mm, int cpl, int wpb) {
   size_t w;
   switch (gshift) {
     case 0: w = pk_smem_w<1>(mm, cpl); break;
@@ -176,7 +176,7 @@ static size_t lane_pk_smem(int gshift, int mm, int cpl) {
     case 4: w = pk_smem_w<16>(mm, cpl); break;
     default: w = pk_smem_w<32>(mm, cpl); break;
   }
-  return (LANE_BLOCK / 32) * w;
+  return (size_t)wpb * w;
 }
 
 static const void *lane_ins_fn(int tbits, int gshift, int cm, bool exact) {
@@ -205,11 +205,13 @@ void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
   const bool pk = !mg && tbits == 32 && cm != 2 && a.costk != nullptr && a.pk_lim > 0;
   if (pk && a.pkc) {  // the base-graph sweep kernel: TMA-staged packed-key cards
     const int cpl = a.pk_cpl == 2 && a.lane_mm <= 1 ? 2 : 1;
+    const int wpb = a.pk_wpb > 0 ? a.pk_wpb : LANE_BLOCK / 32;
     const void *f = lane_pk_fn(a.gshift, a.lane_mm, a.G == (1 << a.gshift), cpl);
-    const size_t sm = lane_pk_smem(a.gshift, a.lane_mm, cpl);
+    const size_t sm = lane_pk_smem(a.gshift, a.lane_mm, cpl, wpb);
+    cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     SimArgs aa = a;
     void *args[] = {&aa};
-    cudaLaunchKernel(f, dim3(grid), dim3(LANE_BLOCK), args, sm, st);
+    cudaLaunchKernel(f, dim3(grid), dim3(32 * wpb), args, sm, st);
     return;
   }
   const void *f = lane_fn(tbits, a.gshift, cm, a.G == (1 << a.gshift), mg, pk, a.lane_mm);
@@ -223,16 +225,16 @@ void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
 // resident blocks per SM of the base-graph launch of memory mode mm and
 // packed keys pk (the minimum over the comm / exactness variants); sets their
 // dynamic shared memory limit
-int lane_occupancy(int tbits, int gshift, int mm, bool pk, int cpl) {
+int lane_occupancy(int tbits, int gshift, int mm, bool pk, int cpl, int wpb) {
   int nb = 1 << 30, x = 0;
   if (pk && tbits != 32) return 0;
-  if (pk) {  // k_lane_pk
+  if (pk) {  // k_lane_pk (blocks of wpb warps)
     if (mm > 1) cpl = 1;
-    const size_t sm = lane_pk_smem(gshift, mm, cpl);
+    const size_t sm = lane_pk_smem(gshift, mm, cpl, wpb);
     for (int ex = 0; ex < 2; ex++) {
       const void *f = lane_pk_fn(gshift, mm, ex != 0, cpl);
       cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, f, LANE_BLOCK, sm);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&x, f, 32 * wpb, sm);
       nb = x < nb ? x : nb;
     }
     return nb;
