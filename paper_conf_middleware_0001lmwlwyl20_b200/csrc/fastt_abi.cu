@@ -196,6 +196,7 @@ struct Base {
     char *buf = nullptr;  // dq | avail | ms | rec | rounds | used | used + reserved | keys
     uint32_t *dq = nullptr, *key = nullptr;  // key: the records as packed keys FT << gshift | place (PK)
     uint32_t *key2 = nullptr;                // the keys doubled (k_lane_pk, two candidates per lane)
+    uint32_t *key4 = nullptr;                // ... and four times (four candidates per lane)
     void *avail = nullptr, *ms = nullptr, *rec = nullptr, *used = nullptr, *ur = nullptr;
     int32_t *rounds = nullptr;
   } snap[2];
@@ -628,7 +629,9 @@ static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st,
 // keep 10 warps per SM, measured 88.9 vs 90.8 ms for one candidate per lane
 // on C5, 101.5 ms with 4-warp blocks)
 static int pk_cpl(const fastt_graph *g, int mm) {
-  return g->use_pk_tma && g->pk_cpl == 2 && (mm == 0 || (mm == 1 && g->pk_cpl_peak)) ? 2 : 1;
+  if (!g->use_pk_tma || g->pk_cpl < 2) return 1;
+  if (mm == 0) return g->pk_cpl;
+  return mm == 1 && g->pk_cpl_peak ? 2 : 1;
 }
 
 static int gshift_of(int G) {
@@ -876,7 +879,7 @@ static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cud
   const size_t o_dq = 0, o_av = al16(4 * n), o_ms = o_av + al16(tb * (n + 1) * g->G),
                o_rec = o_ms + al16(tb * (n + 1)), o_rd = o_rec + al16((B.tbits == 32 ? 8 : 16) * n),
                o_us = o_rd + 64, o_ur = o_us + al16(8 * (n + 1) * g->G), o_k = o_ur + al16(8 * (n + 1) * g->G),
-               o_k2 = o_k + al16(4 * n), tot = o_k2 + al16(8 * n);
+               o_k2 = o_k + al16(4 * n), o_k4 = o_k2 + al16(8 * n), tot = o_k4 + al16(16 * n);
   CK(cudaMalloc(&S.buf, tot));
   S.dq = (uint32_t *)(S.buf + o_dq);
   S.avail = S.buf + o_av;
@@ -887,6 +890,7 @@ static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cud
   S.ur = S.buf + o_ur;
   S.key = (uint32_t *)(S.buf + o_k);
   S.key2 = (uint32_t *)(S.buf + o_k2);
+  S.key4 = (uint32_t *)(S.buf + o_k4);
   CK(cudaMemsetAsync(S.rounds, 0, 16, st));
   Cand c;
   memset(&c, 0, sizeof c);
@@ -934,7 +938,7 @@ static fastt_status ensure_snapshot(fastt_graph *g, Base &B, uint32_t flags, cud
   cudaFree(d_st);
   if (hst != FASTT_CAND_OK) return FASTT_OK;  // an infeasible BASE (caps): no sharing
   if (B.tbits == 32) {
-    launch_snap_keys(S.rec, B.n, gshift_of(g->G), S.key, S.key2, st);
+    launch_snap_keys(S.rec, B.n, gshift_of(g->G), S.key, S.key2, S.key4, st);
     CK(cudaGetLastError());
   }
   S.round_dev = (rd[0] == 1 && rd[2] == 0 && rd[3] == B.cp_len) ? rd[1] : -1;
@@ -951,6 +955,7 @@ static void use_snapshot(const Base &B, uint32_t flags, SimArgs &a) {
   a.snap_ur = S.ur;
   a.snap_key = S.key;
   a.snap_key2 = S.key2;
+  a.snap_key4 = S.key4;
   a.snap_round_dev = S.round_dev;
   a.snap_dq = S.dq;
   a.snap_avail = S.avail;
@@ -1813,7 +1818,7 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     e = getenv("FASTT_OVL_MODE");
     if (e && e[0]) g->ovl_mode = atoi(e);
     e = getenv("FASTT_PK_CPL");
-    if (e && e[0]) g->pk_cpl = atoi(e) == 1 ? 1 : 2;
+    if (e && e[0]) g->pk_cpl = atoi(e) == 1 ? 1 : atoi(e) == 4 ? 4 : 2;
     e = getenv("FASTT_PK_LIM");
     if (e && e[0]) g->pk_lim_cap = (uint32_t)std::max(1ll, std::min(0xFFFFFFFFll, atoll(e)));
   }

@@ -275,6 +275,7 @@ struct SimArgs {
   // k_lane_pk with two candidates per lane: the BASE keys doubled ([2n],
   // key s at words 2s and 2s + 1, so an aligned 8-B load gives it to both)
   const uint32_t *snap_key2;
+  const uint32_t *snap_key4;  // ... and four times ([4n], CPL 4)
   int32_t pk_cpl;  // candidates per lane of the k_lane_pk launch (1 or 2)
   int32_t gwarp_off;  // persistent k_lane_pk: first slab column block / wbest entry of this launch
   int32_t pk_wpb;     // k_lane_pk: warps per block (1, 2 or 4; 0 = 4)
@@ -383,7 +384,8 @@ void launch_pack_costs(const PrepGraph *pg_dev, int32_t n, int G, int gshift, in
 // words of one compact PK card (k_lane_pk.cuh)
 int pk_card_words_host(int gshift);
 // BASE records (uint32 time: FT | place << 32) -> packed keys FT << gshift | place
-void launch_snap_keys(const void *rec, int32_t n, int gshift, uint32_t *key, uint32_t *key2, cudaStream_t st);
+void launch_snap_keys(const void *rec, int32_t n, int gshift, uint32_t *key, uint32_t *key2, uint32_t *key4,
+                      cudaStream_t st);
 void launch_fit(int G, int64_t n, const uint8_t *src, const uint8_t *dst, const int64_t *bytes, const int64_t *tns,
                 void *sums, unsigned *err, int64_t *alpha, int64_t *beta, int64_t *count, int sms, cudaStream_t st);
 size_t fit_sums_bytes(int G);

@@ -88,14 +88,15 @@ __device__ __forceinline__ void cp16_if(bool p, uint32_t saddr, const void *g) {
 // EX: G == GP.  MM: memory mode (0 none, 1 peak, 2 caps; k_sim_lane).
 // CPL: candidates per lane (2 only with MM 0).
 template <int GSH, bool EX, int MM, int CPL>
-__global__ void __launch_bounds__(LANE_BLOCK, CPL == 1 ? LANE_MINB : 3) k_lane_pk(SimArgs a) {
+__global__ void __launch_bounds__(LANE_BLOCK, CPL == 1 ? LANE_MINB : CPL == 2 ? 3 : 2) k_lane_pk(SimArgs a) {
   constexpr int GP = 1 << GSH;
   constexpr uint32_t GMK = GP - 1;
   constexpr int D = LANE_D, P = D - 1;
   constexpr int CB = pk_card_bytes(GP);
   constexpr int RW = 32 * CPL;  // keys per record row
   static_assert((D & (D - 1)) == 0 && CB % 16 == 0, "pipeline slots");
-  static_assert(CPL == 1 || (CPL == 2 && MM <= 1), "two candidates per lane: makespan (+ peak memory)");
+  static_assert(CPL == 1 || (CPL == 2 && MM <= 1) || (CPL == 4 && MM == 0),
+                "two candidates per lane: makespan (+ peak memory); four: makespan only");
   const int lane = threadIdx.x & 31;
   int64_t gwarp = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5) + a.gwarp_off;
   if (a.lane_batches > 0) {
@@ -169,7 +170,9 @@ __global__ void __launch_bounds__(LANE_BLOCK, CPL == 1 ? LANE_MINB : 3) k_lane_p
   const uint32_t *pkc = a.pkc;
   const int32_t n = pg->n, cpl = pg->cp_len;
   const uint32_t *__restrict__ snap = a.snap_key;
-  const uint32_t *__restrict__ snapx = CPL == 1 ? a.snap_key : a.snap_key2;  // (CPL 2: each key twice)
+  // (CPL 2 / 4: each BASE key twice / four times, so an aligned 8-/16-B load
+  // gives it to every candidate of a lane)
+  const uint32_t *__restrict__ snapx = CPL == 1 ? a.snap_key : CPL == 2 ? a.snap_key2 : a.snap_key4;
   const bool cp_on = (a.flags & 1u) != 0;
   int64_t bms = I64MAX, bidx = -1;
   uint32_t zc = 0;  // card chunks issued by this warp so far (barrier zc & 3, phase (zc >> 2) & 1)
@@ -381,7 +384,7 @@ __global__ void __launch_bounds__(LANE_BLOCK, CPL == 1 ? LANE_MINB : 3) k_lane_p
       const bool staged = u < n && (uint32_t)pk_k < npu && (int32_t)s < thr;
       const bool base_rec = (int32_t)s < lo;  // the BASE record: one 16-B chunk holds it
       const uint32_t row = stage_sa + (slot * 4 + (uint32_t)pk_k) * (4 * RW);
-      const uint32_t sw = CPL == 1 ? s : 2 * s;  // the BASE key's word (CPL 2: the doubled array, 8-B pairs)
+      const uint32_t sw = CPL * s;  // the BASE key's word in the CPL-fold array
 #pragma unroll
       for (int i = 0; i < CPL; i++) {
         const int cc = pk_c + 8 * i;
@@ -449,10 +452,16 @@ __global__ void __launch_bounds__(LANE_BLOCK, CPL == 1 ? LANE_MINB : 3) k_lane_p
         for (int k = 0; k < 4; k++) {
           if (CPL == 1) {
             rk[0][k] = *(const uint32_t *)__cvta_shared_to_generic(ad[k]);
-          } else {  // (a BASE record is a doubled pair: the same key for both)
+          } else if (CPL == 2) {  // (a BASE record is a doubled pair: the same key for both)
             const uint2 x = *(const uint2 *)__cvta_shared_to_generic(ad[k]);
             rk[0][k] = x.x;
             rk[CPL - 1][k] = x.y;
+          } else {
+            const uint4 x = *(const uint4 *)__cvta_shared_to_generic(ad[k]);
+            rk[0][k] = x.x;
+            rk[1 % CPL][k] = x.y;
+            rk[2 % CPL][k] = x.z;
+            rk[3 % CPL][k] = x.w;
           }
         }
       }
@@ -610,10 +619,14 @@ __global__ void __launch_bounds__(LANE_BLOCK, CPL == 1 ? LANE_MINB : 3) k_lane_p
           col[(size_t)t * RW] = rec[0];
           ring[(t & (D - 1)) * RW] = rec[0];
         }
-      } else {
+      } else if (CPL == 2) {
         const uint2 r2 = make_uint2(rec[0], rec[CPL - 1]);
         *(uint2 *)(col + (size_t)t * RW) = r2;
         *(uint2 *)(ring + (t & (D - 1)) * RW) = r2;
+      } else {
+        const uint4 r4 = make_uint4(rec[0], rec[1 % CPL], rec[2 % CPL], rec[3 % CPL]);
+        *(uint4 *)(col + (size_t)t * RW) = r4;
+        *(uint4 *)(ring + (t & (D - 1)) * RW) = r4;
       }
     }
     // drain: nothing may land in the stage or card slots after this batch

@@ -10,7 +10,9 @@
 namespace fastt {
 
 const void *FASTT_CAT(lane_pk_fn_g, FASTT_GSH)(int mm, bool exact, int cpl) {
-  if (cpl == 2 && mm <= 1)  // (two candidates per lane: makespan, + per-device peak memory)
+  if (cpl == 4 && mm == 0)  // (four candidates per lane: makespan only)
+    return exact ? (const void *)k_lane_pk<FASTT_GSH, true, 0, 4> : (const void *)k_lane_pk<FASTT_GSH, false, 0, 4>;
+  if (cpl >= 2 && mm <= 1)  // (two candidates per lane: makespan, + per-device peak memory)
     return exact ? (mm == 0 ? (const void *)k_lane_pk<FASTT_GSH, true, 0, 2> : (const void *)k_lane_pk<FASTT_GSH, true, 1, 2>)
                  : (mm == 0 ? (const void *)k_lane_pk<FASTT_GSH, false, 0, 2>
                             : (const void *)k_lane_pk<FASTT_GSH, false, 1, 2>);

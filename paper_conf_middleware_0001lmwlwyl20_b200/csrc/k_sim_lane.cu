@@ -131,17 +131,21 @@ void launch_pack_costs(const PrepGraph *pg_dev, int32_t n, int G, int gshift, in
 
 // BASE records as packed keys, and doubled (key2[2p] = key2[2p + 1] =
 // key[p]) for the two-candidates-per-lane kernel
-__global__ void k_snap_keys(const unsigned long long *rec, int32_t n, int gshift, uint32_t *key, uint2 *key2) {
+__global__ void k_snap_keys(const unsigned long long *rec, int32_t n, int gshift, uint32_t *key, uint2 *key2,
+                            uint4 *key4) {
   for (int32_t p = blockIdx.x * blockDim.x + threadIdx.x; p < n; p += gridDim.x * blockDim.x) {
     const unsigned long long w = rec[p];
     const uint32_t k = ((uint32_t)w << gshift) | (uint32_t)(w >> 32);
     key[p] = k;
     key2[p] = make_uint2(k, k);
+    key4[p] = make_uint4(k, k, k, k);
   }
 }
-void launch_snap_keys(const void *rec, int32_t n, int gshift, uint32_t *key, uint32_t *key2, cudaStream_t st) {
+void launch_snap_keys(const void *rec, int32_t n, int gshift, uint32_t *key, uint32_t *key2, uint32_t *key4,
+                      cudaStream_t st) {
   if (n > 0)
-    k_snap_keys<<<(n + 255) / 256, 256, 0, st>>>((const unsigned long long *)rec, n, gshift, key, (uint2 *)key2);
+    k_snap_keys<<<(n + 255) / 256, 256, 0, st>>>((const unsigned long long *)rec, n, gshift, key, (uint2 *)key2,
+                                                  (uint4 *)key4);
 }
 
 int lane_comm_mode(const SimArgs &a, int tbits) {
@@ -163,7 +167,8 @@ static const void *lane_pk_fn(int gshift, int mm, bool exact, int cpl) {
   }
 }
 template <int GP> static size_t pk_smem_w(int mm, int cpl) {
-  if (cpl == 2 && mm <= 1) return mm == 0 ? pk_smem_per_warp<GP, 0, 2>() : pk_smem_per_warp<GP, 1, 2>();
+  if (cpl == 4 && mm == 0) return pk_smem_per_warp<GP, 0, 4>();
+  if (cpl >= 2 && mm <= 1) return mm == 0 ? pk_smem_per_warp<GP, 0, 2>() : pk_smem_per_warp<GP, 1, 2>();
   return mm == 0 ? pk_smem_per_warp<GP, 0>() : mm == 1 ? pk_smem_per_warp<GP, 1>() : pk_smem_per_warp<GP, 2>();
 }
 static size_t lane_pk_smem(int gshift, int mm, int cpl, int wpb) {
@@ -204,7 +209,7 @@ void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st) {
   }
   const bool pk = !mg && tbits == 32 && cm != 2 && a.costk != nullptr && a.pk_lim > 0;
   if (pk && a.pkc) {  // the base-graph sweep kernel: TMA-staged packed-key cards
-    const int cpl = a.pk_cpl == 2 && a.lane_mm <= 1 ? 2 : 1;
+    const int cpl = a.pk_cpl == 4 && a.lane_mm == 0 ? 4 : a.pk_cpl >= 2 && a.lane_mm <= 1 ? 2 : 1;
     const int wpb = a.pk_wpb > 0 ? a.pk_wpb : LANE_BLOCK / 32;
     const void *f = lane_pk_fn(a.gshift, a.lane_mm, a.G == (1 << a.gshift), cpl);
     const size_t sm = lane_pk_smem(a.gshift, a.lane_mm, cpl, wpb);
@@ -230,6 +235,7 @@ int lane_occupancy(int tbits, int gshift, int mm, bool pk, int cpl, int wpb) {
   if (pk && tbits != 32) return 0;
   if (pk) {  // k_lane_pk (blocks of wpb warps)
     if (mm > 1) cpl = 1;
+    if (mm == 1 && cpl > 2) cpl = 2;
     const size_t sm = lane_pk_smem(gshift, mm, cpl, wpb);
     for (int ex = 0; ex < 2; ex++) {
       const void *f = lane_pk_fn(gshift, mm, ex != 0, cpl);
