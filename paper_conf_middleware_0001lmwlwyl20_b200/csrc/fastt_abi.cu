@@ -273,6 +273,7 @@ struct fastt_graph {
     size_t cap = 0;
   } io[3];
   bool use_rank_reuse = true;  // FASTT_NO_RANK_REUSE=1: SPLIT slots recompute every rank (A/B parity)
+  bool use_cost_hole = true;   // FASTT_NO_COST_HOLE=1: split slots copy the base cost table too (A/B parity)
   bool use_pk = true;      // FASTT_NO_PK=1: the lane kernel without packed device keys (A/B parity)
   bool use_pk_tma = true;  // FASTT_NO_PK_TMA=1: packed keys on k_sim_lane instead of k_lane_pk (A/B parity)
   int pk_cpl = 2;          // FASTT_PK_CPL=1: one candidate per lane in the makespan-only k_lane_pk (A/B)
@@ -855,15 +856,22 @@ static fastt_status run_prep(fastt_graph *g, const Base &B, int nslots, cudaStre
                              const uint32_t *nact = nullptr) {
   g->launches += NL_PREP;
   launch_slot_setup(g->slot_cands, g->tmpl_dev, B.raw_dev, g->slot_raws_dev, nslots, st);
+  // the slot copy skips the base cost, mem and param tables (layout slots
+  // 10-12, contiguous): k_rank, k_cards_pred and k_cards_hdr read a base op's
+  // rows from the base graph; k_patch_split writes the overlay rows
+  const RawGraph Rb = raw_struct(B.raw_block, B.rl, B.V, B.n_live, B.E);
+  const int64_t c_lo = (int64_t)B.rl.o[10], c_hi = (int64_t)B.rl.o[13];
+  const bool hole = g->use_cost_hole && (c_hi & 15) == 0 && (c_lo & 15) == 0;
   launch_copy_block(B.raw_block, g->arena, (int64_t)(g->arena_raw_total + g->arena_prep_total), (int64_t)B.rl.total,
-                    g->slot_cands, nslots, st, nact);
+                    g->slot_cands, nslots, st, nact, hole ? c_lo : 0, hole ? c_hi : 0);
   launch_patch_split(B.raw_dev, g->slot_raws_dev, g->gc_dev, g->slot_cands, nslots, st, nact);
   launch_rank(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, g->slot_cands, nslots, g->G, st,
-              g->use_rank_reuse ? prep_struct(B.prep_block, B.pl, B.tbits).rank : nullptr, nact);
+              g->use_rank_reuse ? prep_struct(B.prep_block, B.pl, B.tbits).rank : nullptr, nact,
+              hole ? Rb.cost : nullptr);
   launch_sort(g->slot_pgs_dev, g->slot_raws_dev, nslots, B.key_bits, (int)B.rl.vcap, st, nact);
   // (successor lists only for slots the ready-set kernel will run: see launch_slots)
   launch_cards(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, nslots, (int)B.rl.vcap, g->G, g->K, B.tbits, st,
-               !g->use_topo, nact);
+               !g->use_topo, nact, hole ? Rb.cost : nullptr, hole ? Rb.mem : nullptr, hole ? Rb.param : nullptr);
   launch_cp(g->slot_raws_dev, g->slot_pgs_dev, nslots, g->G, B.tbits, st, nact);
   CK(cudaGetLastError());
   return FASTT_OK;
@@ -1797,6 +1805,8 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     g->use_lane = !(e && e[0] == '1');
     e = getenv("FASTT_NO_RANK_REUSE");
     g->use_rank_reuse = !(e && e[0] == '1');
+    e = getenv("FASTT_NO_COST_HOLE");
+    g->use_cost_hole = !(e && e[0] == '1');
     e = getenv("FASTT_NO_PK");
     g->use_pk = !(e && e[0] == '1');
     e = getenv("FASTT_NO_PK_TMA");

@@ -160,17 +160,25 @@ __host__ __device__ inline int64_t part_bytes(int64_t b, int n, int k) { return 
 // nact (all prep launchers, nullable): device count of the active slots; the
 // grid covers nslots, slots at or past *nact exit at once (a preparation
 // wave sized on the device, without a host round trip)
+// base_cost (nullable): a split slot's base-op cost rows are read from the
+// base graph (the slot copy skips the cost table; the overlay rows are the
+// slot's own)
 void launch_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, const Cand *cands, int nslots,
-                 int G, cudaStream_t st, const uint64_t *base_rank = nullptr, const uint32_t *nact = nullptr);
+                 int G, cudaStream_t st, const uint64_t *base_rank = nullptr, const uint32_t *nact = nullptr,
+                 const int64_t *base_cost = nullptr);
 void launch_heights(RawGraph *raw_dev, int32_t *scratch, int64_t vcap, cudaStream_t st);
 void launch_sort(PrepGraph *pgs, const RawGraph *raws, int nslots, int key_bits, int max_n, cudaStream_t st,
                  const uint32_t *nact = nullptr);
 void launch_cards(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, int nslots, int max_n, int G, int K,
-                  int tbits, cudaStream_t st, bool succ_all, const uint32_t *nact = nullptr);
+                  int tbits, cudaStream_t st, bool succ_all, const uint32_t *nact = nullptr,
+                  const int64_t *base_cost = nullptr, const int64_t *base_mem = nullptr,
+                  const int64_t *base_param = nullptr);
 void launch_cp(const RawGraph *raws, PrepGraph *pgs, int nslots, int G, int tbits, cudaStream_t st,
                const uint32_t *nact = nullptr);
+// (hole_lo, hole_hi: a byte range of the block not copied, 16-B aligned)
 void launch_copy_block(const void *src, void *dst, int64_t slot_stride_bytes, int64_t bytes, const Cand *cands,
-                       int nslots, cudaStream_t st, const uint32_t *nact = nullptr);
+                       int nslots, cudaStream_t st, const uint32_t *nact = nullptr, int64_t hole_lo = 0,
+                       int64_t hole_hi = 0);
 void launch_patch_split(const RawGraph *base, RawGraph *raws, const GraphConst *gc, const Cand *cands, int nslots,
                         cudaStream_t st, const uint32_t *nact = nullptr);
 void launch_bound(const RawGraph *raw, const GraphConst *gc, int G, unsigned long long *out /* [2] */,

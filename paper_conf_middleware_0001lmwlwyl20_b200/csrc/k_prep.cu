@@ -28,12 +28,18 @@ __device__ __forceinline__ uint32_t warp_min_u32(uint32_t v) { return __reduce_m
 
 // Bulk copy of the base raw block into every SPLIT slot (same layout, contiguous).
 // (nact: device count of active slots, nullable -- slots at or past it exit)
+// Words [hole_lo, hole_hi) are skipped (the cost, mem and param tables:
+// split slots read a base op's from the base graph, only the overlay rows
+// -- written by k_patch_split -- are their own).
 __global__ void k_copy_block(const uint4 *src, uint4 *dst_base, int64_t slot_stride_words, int64_t words,
-                             const Cand *cands, const uint32_t *nact) {
+                             const Cand *cands, const uint32_t *nact, int64_t hole_lo, int64_t hole_hi) {
   if ((nact && blockIdx.y >= *nact) || cands[blockIdx.y].kind != 2) return;
   uint4 *dst = dst_base + (int64_t)blockIdx.y * slot_stride_words;
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += (int64_t)gridDim.x * blockDim.x)
+  const int64_t hole = hole_hi - hole_lo, n = words - hole;
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = k < hole_lo ? k : k + hole;
     dst[i] = src[i];
+  }
 }
 
 // remove `o` from a sorted adjacency list and append `nw` (larger than every id)
@@ -193,10 +199,12 @@ __global__ void k_patch_split(const RawGraph *base_p, RawGraph *raws, const Grap
 
 // host-visible entry points used by the ABI (declared in the .cpp)
 void launch_copy_block(const void *src, void *dst, int64_t slot_stride_bytes, int64_t bytes, const Cand *cands,
-                       int nslots, cudaStream_t st, const uint32_t *nact) {
+                       int nslots, cudaStream_t st, const uint32_t *nact, int64_t hole_lo, int64_t hole_hi) {
   int64_t words = (bytes + 15) / 16;
-  dim3 grid((unsigned)((words + 255) / 256 > 1024 ? 1024 : (words + 255) / 256), (unsigned)nslots);
-  k_copy_block<<<grid, 256, 0, st>>>((const uint4 *)src, (uint4 *)dst, slot_stride_bytes / 16, words, cands, nact);
+  const int64_t copied = words - (hole_hi - hole_lo) / 16;
+  dim3 grid((unsigned)((copied + 255) / 256 > 1024 ? 1024 : (copied + 255) / 256), (unsigned)nslots);
+  k_copy_block<<<grid, 256, 0, st>>>((const uint4 *)src, (uint4 *)dst, slot_stride_bytes / 16, words, cands, nact,
+                                     hole_lo / 16, hole_hi / 16);
 }
 void launch_patch_split(const RawGraph *base, RawGraph *raws, const GraphConst *gc, const Cand *cands, int nslots,
                         cudaStream_t st, const uint32_t *nact) {
@@ -248,16 +256,16 @@ __device__ __forceinline__ int pin_of(int32_t u, const int32_t *po, const int32_
 
 // rank of one op u evaluated by one lane: w_u over the allowed
 // devices + max over successors of (c_uv + rank_v)
-__device__ __forceinline__ void rank_one(const RawGraph &R, const GraphConst &gc, uint64_t *rank, int32_t u,
-                                         const int32_t *po, const int32_t *pd, int np, uint32_t dset,
+__device__ __forceinline__ void rank_one(const RawGraph &R, const int64_t *cost, const GraphConst &gc, uint64_t *rank,
+                                         int32_t u, const int32_t *po, const int32_t *pd, int np, uint32_t dset,
                                          uint32_t offm) {
   const int G = gc.G;
   const int pu = pin_of(u, po, pd, np);
   int64_t w = 0;
-  if (pu >= 0) w = R.cost[(int64_t)u * G + pu];
+  if (pu >= 0) w = cost[(int64_t)u * G + pu];
   else
     for (int d = 0; d < G; d++) {
-      const int64_t c = R.cost[(int64_t)u * G + d];
+      const int64_t c = cost[(int64_t)u * G + d];
       w = ((dset >> d) & 1u) && c > w ? c : w;
     }
   const uint32_t off = R.succ_off[u], cnt_s = R.succ_cnt[u];
@@ -276,7 +284,7 @@ __device__ __forceinline__ void rank_one(const RawGraph &R, const GraphConst &gc
 // independent, one lane each.  A split slot inserts its concat nodes before
 // level h(o), its sub-ops with level h(o) and its split nodes after it.
 __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gcp, const Cand *cands, int nslots,
-                       const uint64_t *base_rank, const uint32_t *nact) {
+                       const uint64_t *base_rank, const uint32_t *nact, const int64_t *base_cost) {
   const int lane = threadIdx.x & 31;
   const int slot = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (slot >= nslots || (nact && (uint32_t)slot >= *nact)) return;
@@ -332,7 +340,8 @@ __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *g
       const int32_t extra = (phase == 1 && split && lev == ho) ? R.ov_n : 0;
       for (int32_t q = lane; q < cnt + extra; q += 32) {
         int32_t u = q < cnt ? (list ? list[q] : lo + q) : R.ov_base + R.ov_P + (q - cnt);
-        if (R.alive[u]) rank_one(R, gc, rank, u, po, pd, np, dset, offm);
+        if (R.alive[u]) rank_one(R, split && base_cost && u < R.ov_base ? base_cost : R.cost, gc, rank, u, po, pd, np,
+                                 dset, offm);
       }
       __syncwarp();
     }
@@ -340,11 +349,11 @@ __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *g
 }
 
 void launch_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, const Cand *cands, int nslots, int G,
-                 cudaStream_t st, const uint64_t *base_rank, const uint32_t *nact) {
+                 cudaStream_t st, const uint64_t *base_rank, const uint32_t *nact, const int64_t *base_cost) {
   (void)G;
   int warps_per_block = 4;
   int blocks = (nslots + warps_per_block - 1) / warps_per_block;
-  k_rank<<<blocks, warps_per_block * 32, 0, st>>>(raws, pgs, gc, cands, nslots, base_rank, nact);
+  k_rank<<<blocks, warps_per_block * 32, 0, st>>>(raws, pgs, gc, cands, nslots, base_rank, nact, base_cost);
 }
 
 __device__ uint32_t cta_exscan(uint32_t v, uint32_t *total, uint32_t *s_w);
@@ -590,9 +599,12 @@ void launch_sort(PrepGraph *pgs, const RawGraph *raws, int nslots, int key_bits,
 // ----------------------------------------------------------------- cards
 
 // One CTA per slot: degree scans in position order + card headers.
-__global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, PrepGraph *pgs, const uint32_t *nact) {
+__global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, PrepGraph *pgs, const uint32_t *nact,
+                                                      const int64_t *base_mem, const int64_t *base_param) {
   if (nact && blockIdx.x >= *nact) return;
   const RawGraph R = raws[blockIdx.x];  // (by value: see k_rank)
+  // (a split slot's base-op memory from the base graph: see k_copy_block)
+  const bool bm = base_mem && R.ov_P >= 0;
   PrepGraph &P = pgs[blockIdx.x];
   __shared__ uint64_t s_w[33];
   const int32_t n = P.n;
@@ -616,12 +628,14 @@ __global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, Prep
       c[CW_PBASE] = runp + bp;
       c[CW_SBASE] = runs + bs;
       c[CW_CPIDX] = NONE;
-      uint64_t m = (uint64_t)R.mem[u];
+      const bool fb = bm && (int32_t)u < R.ov_base;
+      const int64_t mu = fb ? base_mem[u] : R.mem[u], pu = fb ? base_param[u] : R.param[u];
+      uint64_t m = (uint64_t)mu;
       c[CW_MEMLO] = (uint32_t)m;
       c[CW_MEMHI] = (uint32_t)(m >> 32);
       c[CW_UID] = u;
       c[CW_FLAGS] = 0;
-      P.act[p] = R.mem[u] - R.param[u];
+      P.act[p] = mu - pu;
       P.npred[p] = np_;
       if (np_ == 0) atomicOr(&P.srcbits[p >> 5], 1u << (p & 31));
     }
@@ -648,7 +662,8 @@ __global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, Prep
 // the inline predecessor entries of the card (words 8-15); clears P.topo on
 // an edge that does not go from a lower to a higher position.
 template <typename T>
-__global__ void k_cards_pred(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gcp, const uint32_t *nact) {
+__global__ void k_cards_pred(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gcp, const uint32_t *nact,
+                             const int64_t *base_cost) {
   const int slot = blockIdx.y;
   if (nact && (uint32_t)slot >= *nact) return;
   const RawGraph R = raws[slot];  // (by value: see k_rank)
@@ -664,7 +679,8 @@ __global__ void k_cards_pred(const RawGraph *raws, PrepGraph *pgs, const GraphCo
     const uint32_t u = P.uid[p];
     const uint2 dp = *(const uint2 *)c;  // CW_DEG, CW_PBASE (k_cards_hdr)
     const uint32_t np_ = dp.x & 0xFFFF, pb = dp.y;
-    for (int d = 0; d < G; d++) costp[(int64_t)p * G + d] = (T)R.cost[(int64_t)u * G + d];
+    const int64_t *cr = base_cost && R.ov_P >= 0 && (int32_t)u < R.ov_base ? base_cost : R.cost;  // (see k_copy_block)
+    for (int d = 0; d < G; d++) costp[(int64_t)p * G + d] = (T)cr[(int64_t)u * G + d];
     const uint32_t po = R.pred_off[u];
     uint32_t inl[P_IN] = {0, 0, 0, 0}, icm[P_IN] = {0, 0, 0, 0};  // unused slots hold position 0
 #pragma unroll
@@ -726,12 +742,13 @@ __global__ void k_cards_succ(const RawGraph *raws, PrepGraph *pgs, int all, cons
 }
 
 void launch_cards(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, int nslots, int max_n, int G, int K,
-                  int tbits, cudaStream_t st, bool succ_all, const uint32_t *nact) {
+                  int tbits, cudaStream_t st, bool succ_all, const uint32_t *nact, const int64_t *base_cost,
+                  const int64_t *base_mem, const int64_t *base_param) {
   (void)G; (void)K;
-  k_cards_hdr<<<nslots, SORT_T, 0, st>>>(raws, pgs, nact);
+  k_cards_hdr<<<nslots, SORT_T, 0, st>>>(raws, pgs, nact, base_mem, base_param);
   dim3 gp((unsigned)std::max(1, std::min((max_n + 255) / 256, 1024)), nslots);
-  if (tbits == 32) k_cards_pred<uint32_t><<<gp, 256, 0, st>>>(raws, pgs, gc, nact);
-  else k_cards_pred<uint64_t><<<gp, 256, 0, st>>>(raws, pgs, gc, nact);
+  if (tbits == 32) k_cards_pred<uint32_t><<<gp, 256, 0, st>>>(raws, pgs, gc, nact, base_cost);
+  else k_cards_pred<uint64_t><<<gp, 256, 0, st>>>(raws, pgs, gc, nact, base_cost);
   int blocks = (max_n * 32 + 255) / 256;
   if (blocks > 2048) blocks = 2048;
   // (only the rare non-topological slots do work unless succ_all: a full-width
