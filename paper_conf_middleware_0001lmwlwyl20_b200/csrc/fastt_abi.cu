@@ -188,6 +188,7 @@ struct Base {
   uint32_t *costk = nullptr;  // [n][G] cost << gshift | d, then commk [n][4] (inline comm << gshift)
   uint32_t *commk = nullptr;
   uint32_t *pkc = nullptr;  // compact PK cards of k_lane_pk (same allocation)
+  LvlRec *lvlrec = nullptr;  // k_rank's level records (LvlRec, n_live)
   uint32_t pk_lim = 0;
   // recorded BASE schedule for prefix sharing, per CP-pin flag value
   struct Snap {
@@ -206,6 +207,8 @@ struct Base {
     cudaFree(prep_block);
     cudaFree(pg_dev);
     cudaFree(costk);
+    cudaFree(lvlrec);
+    lvlrec = nullptr;
     costk = nullptr;
     commk = nullptr;
     pkc = nullptr;
@@ -274,6 +277,7 @@ struct fastt_graph {
   } io[3];
   bool use_rank_reuse = true;  // FASTT_NO_RANK_REUSE=1: SPLIT slots recompute every rank (A/B parity)
   bool use_cost_hole = true;   // FASTT_NO_COST_HOLE=1: split slots copy the base cost table too (A/B parity)
+  bool use_lvlrec = true;      // FASTT_NO_LVLREC=1: k_rank recomputes every op's terms on its chain (A/B parity)
   bool use_pk = true;      // FASTT_NO_PK=1: the lane kernel without packed device keys (A/B parity)
   bool use_pk_tma = true;  // FASTT_NO_PK_TMA=1: packed keys on k_sim_lane instead of k_lane_pk (A/B parity)
   int pk_cpl = 2;          // FASTT_PK_CPL=1: one candidate per lane in the makespan-only k_lane_pk (A/B)
@@ -518,6 +522,14 @@ static fastt_status prepare_base(fastt_graph *g, Base &B, cudaStream_t st) {
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(st));
     cudaFree(scratch);
+  }
+  // k_rank's level records (fast path of the preparation slots)
+  cudaFree(B.lvlrec);
+  B.lvlrec = nullptr;
+  if (B.n_live > 0) {
+    CK(cudaMalloc(&B.lvlrec, sizeof(LvlRec) * (size_t)B.n_live));
+    launch_lvlrec(B.raw_dev, g->gc_dev, B.n_live, B.lvlrec, st);
+    CK(cudaGetLastError());
   }
   unsigned long long *d_b = nullptr;
   CK(cudaMalloc(&d_b, 16));
@@ -867,7 +879,7 @@ static fastt_status run_prep(fastt_graph *g, const Base &B, int nslots, cudaStre
   launch_patch_split(B.raw_dev, g->slot_raws_dev, g->gc_dev, g->slot_cands, nslots, st, nact);
   launch_rank(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, g->slot_cands, nslots, g->G, st,
               g->use_rank_reuse ? prep_struct(B.prep_block, B.pl, B.tbits).rank : nullptr, nact,
-              hole ? Rb.cost : nullptr);
+              hole ? Rb.cost : nullptr, g->use_lvlrec ? B.lvlrec : nullptr);
   launch_sort(g->slot_pgs_dev, g->slot_raws_dev, nslots, B.key_bits, (int)B.rl.vcap, st, nact);
   // (successor lists only for slots the ready-set kernel will run: see launch_slots)
   launch_cards(g->slot_raws_dev, g->slot_pgs_dev, g->gc_dev, nslots, (int)B.rl.vcap, g->G, g->K, B.tbits, st,
@@ -1807,6 +1819,8 @@ fastt_status fastt_load_graph(const fastt_graph_desc *d, int cuda_device, fastt_
     g->use_rank_reuse = !(e && e[0] == '1');
     e = getenv("FASTT_NO_COST_HOLE");
     g->use_cost_hole = !(e && e[0] == '1');
+    e = getenv("FASTT_NO_LVLREC");
+    g->use_lvlrec = !(e && e[0] == '1');
     e = getenv("FASTT_NO_PK");
     g->use_pk = !(e && e[0] == '1');
     e = getenv("FASTT_NO_PK_TMA");

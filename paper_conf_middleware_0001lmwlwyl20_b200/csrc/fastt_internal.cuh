@@ -160,12 +160,24 @@ __host__ __device__ inline int64_t part_bytes(int64_t b, int n, int k) { return 
 // nact (all prep launchers, nullable): device count of the active slots; the
 // grid covers nslots, slots at or past *nact exit at once (a preparation
 // wave sized on the device, without a host round trip)
+// Level records of a base graph (k_rank's fast path): per op in level order
+// (lvl_ops), its unpinned, full-device-set rank terms -- w = max cost, the
+// first 4 successors and their c (R5) -- so a slot's level walk
+// reads one 64-B record per op instead of recomputing them on its chain.
+struct LvlRec {
+  int32_t u, ns;    // op id (-1: dead), successor count
+  int64_t w;
+  int32_t s[4];     // successors (-1 past ns)
+  int64_t c[4];
+};
+static_assert(sizeof(LvlRec) == 64, "level record");
+void launch_lvlrec(const RawGraph *raw, const GraphConst *gc, int32_t n_live, LvlRec *out, cudaStream_t st);
 // base_cost (nullable): a split slot's base-op cost rows are read from the
 // base graph (the slot copy skips the cost table; the overlay rows are the
 // slot's own)
 void launch_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, const Cand *cands, int nslots,
                  int G, cudaStream_t st, const uint64_t *base_rank = nullptr, const uint32_t *nact = nullptr,
-                 const int64_t *base_cost = nullptr);
+                 const int64_t *base_cost = nullptr, const LvlRec *lvlrec = nullptr);
 void launch_heights(RawGraph *raw_dev, int32_t *scratch, int64_t vcap, cudaStream_t st);
 void launch_sort(PrepGraph *pgs, const RawGraph *raws, int nslots, int key_bits, int max_n, cudaStream_t st,
                  const uint32_t *nact = nullptr);

@@ -283,8 +283,40 @@ __device__ __forceinline__ void rank_one(const RawGraph &R, const int64_t *cost,
 // successor of an op sits on a lower level); the ops of a level are
 // independent, one lane each.  A split slot inserts its concat nodes before
 // level h(o), its sub-ops with level h(o) and its split nodes after it.
+// the level records of a base graph (LvlRec): one thread per level-order index
+__global__ void k_lvlrec(const RawGraph *rp, const GraphConst *gcp, int32_t n_live, LvlRec *out) {
+  const RawGraph R = *rp;
+  const GraphConst &gc = *gcp;
+  const int G = gc.G;
+  const uint32_t all = all_devices(G);
+  for (int32_t q = blockIdx.x * blockDim.x + threadIdx.x; q < n_live; q += gridDim.x * blockDim.x) {
+    LvlRec r;
+    const int32_t u = R.lvl_ops[q];
+    r.u = R.alive[u] ? u : -1;
+    r.ns = (int32_t)R.succ_cnt[u];
+    int64_t w = 0;
+    for (int d = 0; d < G; d++) {
+      const int64_t c = R.cost[(int64_t)u * G + d];
+      w = c > w ? c : w;
+    }
+    r.w = w;
+    const uint32_t so = R.succ_off[u];
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+      const bool ok = k < r.ns;
+      r.s[k] = ok ? R.succ_dst[so + k] : -1;
+      r.c[k] = ok ? c_allowed(gc, R.succ_bytes[so + k], -1, -1, all, gc.offdiag_mask) : 0;
+    }
+    out[q] = r;
+  }
+}
+void launch_lvlrec(const RawGraph *raw, const GraphConst *gc, int32_t n_live, LvlRec *out, cudaStream_t st) {
+  if (n_live > 0) k_lvlrec<<<(n_live + 255) / 256, 256, 0, st>>>(raw, gc, n_live, out);
+}
+
 __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gcp, const Cand *cands, int nslots,
-                       const uint64_t *base_rank, const uint32_t *nact, const int64_t *base_cost) {
+                       const uint64_t *base_rank, const uint32_t *nact, const int64_t *base_cost,
+                       const LvlRec *lrec) {
   const int lane = threadIdx.x & 31;
   const int slot = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (slot >= nslots || (nact && (uint32_t)slot >= *nact)) return;
@@ -323,7 +355,63 @@ __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *g
     __syncwarp();
     lev0 = ho;
   }
+  // Fast path (lrec): a level above the split op's (every level of a PIN
+  // slot) reads one base record per op -- its w and the first 4 successors'
+  // c are the base graph's unless the op or that successor is pinned, or the
+  // op is a predecessor of the split op (its successor list now holds a
+  // split node): those take rank_one on the slot's lists, as do successors
+  // past the 4th (from the slot's lists, unchanged for these ops) and the
+  // ops past a level's first 32.
+  const bool fast = lrec != nullptr && dset == all_devices(gc.G);
+  int32_t opre[8];
+  int32_t nopre = 0;
+  if (fast && split) {
+    nopre = R.ov_P <= 8 ? R.ov_P : -1;
+    for (int k = 0; k < 8; k++)  // (split node a's single predecessor is the split op's a-th)
+      opre[k] = k < nopre ? R.pred_src[R.pred_off[R.ov_base + k]] : -1;
+  }
   for (int32_t lev = lev0; lev <= R.H; lev++) {
+    if (fast && !(split && lev == ho) && nopre >= 0) {
+      const int32_t lo = R.lvl_off[lev], cnt = R.lvl_off[lev + 1] - lo;
+      if (lane < cnt) {
+        const LvlRec r = lrec[lo + lane];
+        const int32_t u = r.u;
+        const bool skip = u < 0 || (split && u == R.ov_o);  // (dead)
+        bool own = false;
+#pragma unroll
+        for (int k = 0; k < MAXPINS; k++) own |= k < np && (po[k] == u || po[k] == r.s[0] || po[k] == r.s[1] ||
+                                                           po[k] == r.s[2] || po[k] == r.s[3]);
+#pragma unroll
+        for (int a = 0; a < 8; a++) own |= opre[a] == u;
+        if (!skip && !own) {
+          uint64_t best = 0;
+#pragma unroll
+          for (int k = 0; k < 4; k++) {
+            const uint64_t v = k < r.ns ? (uint64_t)r.c[k] + rank[r.s[k]] : 0;
+            best = v > best ? v : best;
+          }
+          if (r.ns > 4) {  // the rest from the slot's lists (they hold the split node already)
+            const uint32_t off = R.succ_off[u];
+            for (int32_t j = 4; j < r.ns; j++) {
+              const int32_t sj = R.succ_dst[off + j];
+              const uint64_t v =
+                  (uint64_t)c_allowed(gc, R.succ_bytes[off + j], -1, pin_of(sj, po, pd, np), dset, offm) + rank[sj];
+              best = v > best ? v : best;
+            }
+          }
+          rank[u] = (uint64_t)r.w + best;
+        } else if (!skip) {
+          rank_one(R, split && base_cost && u < R.ov_base ? base_cost : R.cost, gc, rank, u, po, pd, np, dset, offm);
+        }
+      }
+      for (int32_t q = lane + 32; q < cnt; q += 32) {
+        const int32_t u = R.lvl_ops[lo + q];
+        if (R.alive[u])
+          rank_one(R, split && base_cost && u < R.ov_base ? base_cost : R.cost, gc, rank, u, po, pd, np, dset, offm);
+      }
+      __syncwarp();
+      continue;
+    }
     for (int phase = 0; phase < 3; phase++) {
       // phase 0: concat nodes (label 4h(o)-2), 1: the level (+ sub-ops at h(o)), 2: split nodes (4h(o)+2)
       int32_t lo, cnt;
@@ -349,11 +437,12 @@ __global__ void k_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *g
 }
 
 void launch_rank(const RawGraph *raws, PrepGraph *pgs, const GraphConst *gc, const Cand *cands, int nslots, int G,
-                 cudaStream_t st, const uint64_t *base_rank, const uint32_t *nact, const int64_t *base_cost) {
+                 cudaStream_t st, const uint64_t *base_rank, const uint32_t *nact, const int64_t *base_cost,
+                 const LvlRec *lvlrec) {
   (void)G;
   int warps_per_block = 4;
   int blocks = (nslots + warps_per_block - 1) / warps_per_block;
-  k_rank<<<blocks, warps_per_block * 32, 0, st>>>(raws, pgs, gc, cands, nslots, base_rank, nact, base_cost);
+  k_rank<<<blocks, warps_per_block * 32, 0, st>>>(raws, pgs, gc, cands, nslots, base_rank, nact, base_cost, lvlrec);
 }
 
 __device__ uint32_t cta_exscan(uint32_t v, uint32_t *total, uint32_t *s_w);

@@ -35,11 +35,12 @@ SHAPES = [
     {"FASTT_PK_CPL": "2", "FASTT_PK_WPB": "1"},
     {"FASTT_PK_CPL": "4"},
     {"FASTT_NO_COST_HOLE": "1"},
+    {"FASTT_NO_LVLREC": "1"},
     {"FASTT_PK_CPL": "4", "FASTT_PK_WPB": "2", "FASTT_OVL_MODE": "0", "FASTT_LANE_BATCHES": "1"},
     {"FASTT_PK_CPL": "2", "FASTT_PK_WPB": "4", "FASTT_OVL_MODE": "0", "FASTT_LANE_BATCHES": "2"},
 ]
 KEYS = ("FASTT_PK_CPL", "FASTT_OVL_MODE", "FASTT_LANE_BATCHES", "FASTT_MAIN_BPS", "FASTT_NO_OVERLAP", "FASTT_PK_CPL_PEAK",
-        "FASTT_PK_WPB", "FASTT_NO_COST_HOLE")
+        "FASTT_PK_WPB", "FASTT_NO_COST_HOLE", "FASTT_NO_LVLREC")
 
 
 def _graph(desc, env):
