@@ -689,7 +689,10 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
           for (int w : {2, 1}) {
             if (g->pk_wpb_env > 0 && w != g->pk_wpb_env) continue;
             const int b = lane_occupancy(B.tbits, gsh, mm, true, pk_cpl(g, mm), w);
-            if (b * w > best_b * best_w || (g->pk_wpb_env == w && b > 0)) {
+            // (ties: two candidates per lane run better in 1-warp blocks,
+            // measured 70.5 vs 71.9 ms on C5 at equal resident warps)
+            const bool tie_small = pk_cpl(g, mm) >= 2 && w == 1 && b * w == best_b * best_w;
+            if (b * w > best_b * best_w || tie_small || (g->pk_wpb_env == w && b > 0)) {
               best_b = b;
               best_w = w;
             }
