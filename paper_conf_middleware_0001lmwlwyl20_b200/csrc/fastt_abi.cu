@@ -274,7 +274,7 @@ struct fastt_graph {
   struct IoBuf {
     void *p = nullptr;
     size_t cap = 0;
-  } io[3];
+  } io[4];  // candidates in, makespan, status, per-device peak memory out
   bool use_rank_reuse = true;  // FASTT_NO_RANK_REUSE=1: SPLIT slots recompute every rank (A/B parity)
   bool use_cost_hole = true;   // FASTT_NO_COST_HOLE=1: split slots copy the base cost table too (A/B parity)
   bool use_lvlrec = true;      // FASTT_NO_LVLREC=1: k_rank recomputes every op's terms on its chain (A/B parity)
@@ -2103,7 +2103,11 @@ fastt_status fastt_schedule_batch(const fastt_graph *gc_, const fastt_candidate 
   };
   o.makespan = (int64_t *)(outdev ? dalloc(makespan, 8 * (size_t)n, true) : io_buf(g, 1, 8 * (size_t)n));
   o.status = (uint8_t *)(outdev ? dalloc(status, (size_t)n, true) : io_buf(g, 2, (size_t)n));
-  o.peak = (int64_t *)dalloc(peak_mem, 8 * (size_t)n * g->G, peak_mem != nullptr);
+  // (host outputs: the graph's staging buffers, kept across calls -- a
+  // stream-ordered allocation per call would return its pages to the OS at
+  // every synchronisation)
+  o.peak = (int64_t *)(outdev || !peak_mem ? dalloc(peak_mem, 8 * (size_t)n * g->G, peak_mem != nullptr)
+                                           : io_buf(g, 3, 8 * (size_t)n * g->G));
   const bool want_sched = placement || order || start_ns;
   o.place = (uint8_t *)dalloc(placement, (size_t)n * vm, want_sched);
   o.start = (int64_t *)dalloc(start_ns, 8 * (size_t)n * vm, want_sched);
@@ -2160,13 +2164,13 @@ fastt_status fastt_generate_candidates(const fastt_graph *gc_, const fastt_gen_p
   StreamState ss = stream_state(g, *S, gen);
   const bool outdev = (flags_of(opts) & FASTT_F_OUT_DEVICE) != 0;
   Cand *d = (Cand *)out;
-  if (!outdev) CK(cudaMallocAsync(&d, sizeof(Cand) * n, st));
+  if (!outdev) {  // (the graph's candidate staging buffer, kept across calls)
+    d = (Cand *)io_buf(g, 0, sizeof(Cand) * (size_t)(n + 1));
+    if (!d) return fail(FASTT_ENOMEM, "candidate staging buffer");
+  }
   launch_candgen(ss, first, n, d, st);
   CK(cudaGetLastError());
-  if (!outdev) {
-    CK(cudaMemcpyAsync(out, d, sizeof(Cand) * n, cudaMemcpyDeviceToHost, st));
-    CK(cudaFreeAsync(d, st));
-  }
+  if (!outdev) CK(cudaMemcpyAsync(out, d, sizeof(Cand) * n, cudaMemcpyDeviceToHost, st));
   return call_end(g, flags_of(opts), st, FASTT_OK);
 }
 
