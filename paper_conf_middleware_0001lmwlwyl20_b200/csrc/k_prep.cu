@@ -713,17 +713,14 @@ __global__ void __launch_bounds__(SORT_T) k_cards_hdr(const RawGraph *raws, Prep
     const uint32_t totp = (uint32_t)tot2, tots = (uint32_t)(tot2 >> 32);
     if (p < n) {
       uint32_t *c = P.card + (int64_t)p * CARD_WORDS;
-      c[CW_DEG] = np_ | (ns_ << 16);
-      c[CW_PBASE] = runp + bp;
-      c[CW_SBASE] = runs + bs;
-      c[CW_CPIDX] = NONE;
       const bool fb = bm && (int32_t)u < R.ov_base;
       const int64_t mu = fb ? base_mem[u] : R.mem[u], pu = fb ? base_param[u] : R.param[u];
-      uint64_t m = (uint64_t)mu;
-      c[CW_MEMLO] = (uint32_t)m;
-      c[CW_MEMHI] = (uint32_t)(m >> 32);
-      c[CW_UID] = u;
-      c[CW_FLAGS] = 0;
+      const uint64_t m = (uint64_t)mu;
+      // the header words 0-7 (CW_DEG .. CW_FLAGS) as two 16-B stores
+      static_assert(CW_DEG == 0 && CW_PBASE == 1 && CW_SBASE == 2 && CW_CPIDX == 3 && CW_MEMLO == 4 &&
+                        CW_MEMHI == 5 && CW_UID == 6 && CW_FLAGS == 7, "card header layout");
+      *(uint4 *)c = make_uint4(np_ | (ns_ << 16), runp + bp, runs + bs, NONE);
+      *(uint4 *)(c + 4) = make_uint4((uint32_t)m, (uint32_t)(m >> 32), u, 0u);
       P.act[p] = mu - pu;
       P.npred[p] = np_;
       if (np_ == 0) atomicOr(&P.srcbits[p >> 5], 1u << (p & 31));
@@ -769,7 +766,15 @@ __global__ void k_cards_pred(const RawGraph *raws, PrepGraph *pgs, const GraphCo
     const uint2 dp = *(const uint2 *)c;  // CW_DEG, CW_PBASE (k_cards_hdr)
     const uint32_t np_ = dp.x & 0xFFFF, pb = dp.y;
     const int64_t *cr = base_cost && R.ov_P >= 0 && (int32_t)u < R.ov_base ? base_cost : R.cost;  // (see k_copy_block)
-    for (int d = 0; d < G; d++) costp[(int64_t)p * G + d] = (T)cr[(int64_t)u * G + d];
+    if (sizeof(T) == 4 && (G & 3) == 0) {  // 16-B stores of the row (4 devices each)
+      for (int d = 0; d < G; d += 4) {
+        const longlong2 a = *(const longlong2 *)(cr + (int64_t)u * G + d);
+        const longlong2 b = *(const longlong2 *)(cr + (int64_t)u * G + d + 2);
+        *(uint4 *)(costp + (int64_t)p * G + d) = make_uint4((uint32_t)a.x, (uint32_t)a.y, (uint32_t)b.x, (uint32_t)b.y);
+      }
+    } else {
+      for (int d = 0; d < G; d++) costp[(int64_t)p * G + d] = (T)cr[(int64_t)u * G + d];
+    }
     const uint32_t po = R.pred_off[u];
     uint32_t inl[P_IN] = {0, 0, 0, 0}, icm[P_IN] = {0, 0, 0, 0};  // unused slots hold position 0
 #pragma unroll
