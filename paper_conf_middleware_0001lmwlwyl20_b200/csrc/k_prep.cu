@@ -592,8 +592,10 @@ __global__ void __launch_bounds__(SORT_T) k_sort(PrepGraph *pgs, const RawGraph 
   PrepGraph &P = pgs[blockIdx.x];
   const RawGraph &R = raws[blockIdx.x];
   __shared__ uint32_t s_w[33];
-  __shared__ uint32_t s_base[256], s_tot[256];
+  __shared__ uint32_t s_base[256], s_tot[256], s_cst[256];
   __shared__ uint32_t s_cnt[SORT_T / 32][257];
+  __shared__ uint64_t s_k[SORT_T];  // a chunk in digit order (coalesced write-out)
+  __shared__ uint32_t s_v[SORT_T];
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const uint64_t maxk = key_bits >= 64 ? ~0ull : ((1ull << key_bits) - 1);
   // compaction of live uids in ascending order
@@ -657,10 +659,35 @@ __global__ void __launch_bounds__(SORT_T) k_sort(PrepGraph *pgs, const RawGraph 
         s_tot[tid] = r;
       }
       __syncthreads();
+      if (wid == 0) {  // the chunk's digit starts: exclusive scan of s_tot (8 per lane)
+        uint32_t loc[8], sm = 0;
+#pragma unroll
+        for (int q = 0; q < 8; q++) { loc[q] = s_tot[lane * 8 + q]; sm += loc[q]; }
+        uint32_t x = sm;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t y = __shfl_up_sync(FULL, x, o);
+          if (lane >= o) x += y;
+        }
+        uint32_t e = x - sm;
+#pragma unroll
+        for (int q = 0; q < 8; q++) { s_cst[lane * 8 + q] = e; e += loc[q]; }
+      }
+      __syncthreads();
+      // stable within the chunk: digit, then warp, then lane
       if (valid) {
-        uint32_t dst = s_base[dg] + s_cnt[wid][dg] + rk;
-        kout[dst] = k;
-        vout[dst] = v;
+        const uint32_t l = s_cst[dg] + s_cnt[wid][dg] + rk;
+        s_k[l] = k;
+        s_v[l] = v;
+      }
+      __syncthreads();
+      // write-out in chunk order: a digit's keys land contiguously
+      if (i < n) {
+        const uint64_t kk = s_k[tid];
+        const uint32_t d = (uint32_t)((kk >> sh) & 255);
+        const uint32_t dst = s_base[d] + ((uint32_t)tid - s_cst[d]);
+        kout[dst] = kk;
+        vout[dst] = s_v[tid];
       }
       __syncthreads();
       if (tid < 256) s_base[tid] += s_tot[tid];
