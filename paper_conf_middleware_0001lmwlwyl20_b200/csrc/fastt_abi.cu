@@ -703,6 +703,11 @@ static fastt_status ensure_sim(fastt_graph *g, const Base &B, int64_t defer_need
           char msg[96];
           snprintf(msg, sizeof msg, "lane launch mm %d pk %d: %d blocks/SM x %d warps", mm, pk, best_b, best_w);
           host_trace(msg);
+          if (pk && B.tbits == 32) {
+            char att[512] = "";
+            lane_pk_attrs(gsh, mm, pk_cpl(g, mm), att, sizeof att);
+            host_trace(att);
+          }
         }
       }
     g->sim_smem = smem;

@@ -397,6 +397,7 @@ void launch_defer_gather(const DeferBlock *blk, int cap, const Cand *srt_c, cons
 int sim_occupancy(int tbits, int gshift, int block, size_t smem, bool topo);
 void launch_sim_lane(const SimArgs &a, int tbits, int grid, cudaStream_t st);
 int lane_occupancy(int tbits, int gshift, int mm, bool pk, int cpl = 1, int wpb = 4);
+void lane_pk_attrs(int gshift, int mm, int cpl, char *buf, size_t len);
 // costk[p][d] = (cost[p][d] << gshift) | d over n positions; mx[0] = max
 // cost, mx[1] = max edge comm (one link class) of the prepared graph
 void launch_pack_costs(const PrepGraph *pg_dev, int32_t n, int G, int gshift, int64_t E, uint32_t *costk,

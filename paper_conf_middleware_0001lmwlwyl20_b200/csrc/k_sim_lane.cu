@@ -38,6 +38,8 @@
 // The kernel itself is in k_sim_lane_body.cuh (instances: k_sim_lane_inst.cu).
 #include "k_sim_lane_body.cuh"
 #include "k_lane_pk.cuh"
+#include <cstdio>
+#include <cstring>
 
 namespace fastt {
 
@@ -256,4 +258,17 @@ int lane_occupancy(int tbits, int gshift, int mm, bool pk, int cpl, int wpb) {
   return nb;
 }
 
+}  // namespace fastt
+
+namespace fastt {
+// (FASTT_HOST_TRACE) registers and shared memory of a k_lane_pk instance
+void lane_pk_attrs(int gshift, int mm, int cpl, char *buf, size_t len) {
+  cudaFuncAttributes fa;
+  for (int ex = 0; ex < 2; ex++) {
+    if (cudaFuncGetAttributes(&fa, lane_pk_fn(gshift, mm, ex != 0, cpl)) != cudaSuccess) continue;
+    const size_t o = strlen(buf);
+    snprintf(buf + o, len - o, " [ex %d: %d regs, %zu static smem, %d max dyn smem, %zu local]", ex, fa.numRegs,
+             fa.sharedSizeBytes, fa.maxDynamicSharedSizeBytes, fa.localSizeBytes);
+  }
+}
 }  // namespace fastt
