@@ -383,7 +383,7 @@ def main():
         roof = {"bound": "hbm", "achieved": hbm_gbs, "peak": peak, "unit": "GB/s", "frac": hbm_gbs / peak,
                 "traffic": traffic, "peak_source": peak_src, "bytes_per_candidate": bpc}
     pk = lane and g.time_bits == 32 and int(len(desc.alpha)) == 1
-    roof.update({"kernel": ("k_lane_pk<GSH=3, EX, MM=0>" if pk else "k_sim_lane" if lane else "k_sim") + " (sweep launch)",
+    roof.update({"kernel": ("k_lane_pk<GSH=3, EX, MM=0, CPL=2> (two candidates per lane)" if pk else "k_sim_lane" if lane else "k_sim") + " (sweep launch)",
                  "candidates_per_launch": fast, "launch_ms": sim_ms, "prep_ms_per_step": prep_ms})
     launches = sum(x["launches"] for x in tms)
 
