@@ -168,3 +168,53 @@ def test_two_graphs_overlap_on_two_streams():
     ga.sync(stream=sa)
     gb.sync(stream=sb)
     assert tuple(oa.tolist()) == ra and tuple(ob.tolist()) == rb
+
+
+@pytest.mark.parametrize("cfg,extra,n", [("C4", "insert", 3000), ("C2", "live", 3000), ("C1", "insert", 20000)])
+def test_async_other_paths(cfg, extra, n):
+    """the sequential (non-overlapped) evaluations -- INSERT (R1i), liveness
+    memory (R24): unsorted stream deferrals (source 2 of the loop) -- are
+    asynchronous too and equal their blocking results"""
+    desc = synth.config(cfg)
+    gen = F.gen_params(seed=SEED, n_pow2_only=(cfg == "C4"))
+    fl = F.F_CP_PIN | (F.F_POLICY_INSERT if extra == "insert" else F.F_MEM_LIVE)
+    g = F.Graph(desc)
+    ref = g.sweep_best(gen, 0, n, flags=fl)
+    s = torch.cuda.Stream()
+    out = torch.empty(2, dtype=torch.int64, device="cuda")
+    for _ in range(2):
+        g.sweep_best(gen, 0, n, flags=fl | F.F_ASYNC, stream=s, out=out)
+    g.sync(stream=s)
+    assert tuple(out.tolist()) == ref
+
+
+def test_async_per_op_outputs():
+    """placement / start / order outputs (an unsorted candidate list: source
+    1 of the loop, and the order sort's stream-ordered scratch) on a device
+    stream equal the blocking host-buffer results and the oracle's"""
+    desc = synth.config("C1")
+    gen = F.gen_params(seed=SEED)
+    g = F.Graph(desc)
+    ns = g.stream_info(gen, flags=F.F_CP_PIN)
+    cands = g.generate_candidates(gen, 0, ns + 300, flags=F.F_CP_PIN)
+    ref = g.schedule_batch(cands, flags=F.F_CP_PIN, placement=True, order=True, start=True)
+    n, vm = len(cands), g.v_max
+    out = {"makespan": torch.empty(n, dtype=torch.int64, device="cuda"),
+           "status": torch.empty(n, dtype=torch.uint8, device="cuda"),
+           "peak_mem": torch.empty(n * g.G, dtype=torch.int64, device="cuda"),
+           "placement": torch.empty(n * vm, dtype=torch.uint8, device="cuda"),
+           "order": torch.empty(n * vm, dtype=torch.int32, device="cuda"),
+           "start": torch.empty(n * vm, dtype=torch.int64, device="cuda")}
+    s = torch.cuda.Stream()
+    g.schedule_batch(_dev_cands(cands), flags=F.F_CP_PIN | F.F_ASYNC, stream=s, out=out)
+    g.sync(stream=s)
+    assert (out["makespan"].cpu().numpy() == ref["makespan"]).all()
+    assert (out["placement"].cpu().numpy().reshape(n, vm) == ref["placement"]).all()
+    assert (out["order"].cpu().numpy().reshape(n, vm) == ref["order"]).all()
+    assert (out["start"].cpu().numpy().reshape(n, vm) == ref["start"]).all()
+    og = O.OracleGraph(desc)
+    for k in range(0, n, 37):
+        r = og.schedule(cands[k], flags=O.F_CP_PIN)
+        assert int(ref["makespan"][k]) == r["makespan"]
+        if r["status"] == 0:
+            assert (ref["order"][k] == r["order"]).all()
