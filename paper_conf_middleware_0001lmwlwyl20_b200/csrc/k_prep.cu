@@ -586,6 +586,7 @@ __device__ uint64_t cta_exscan64(uint64_t v, uint64_t *total, uint64_t *s_w) {
 
 // One CTA per slot: order live ops by (rank desc, uid asc) with a stable LSD
 // radix sort of key = (2^key_bits - 1 - rank) over values initially in uid order.
+template <typename KT>  // key type: uint32_t when key_bits <= 32 (half the key traffic), else uint64_t
 __global__ void __launch_bounds__(SORT_T) k_sort(PrepGraph *pgs, const RawGraph *raws, int key_bits,
                                                  const uint32_t *nact) {
   if (nact && blockIdx.x >= *nact) return;
@@ -594,7 +595,7 @@ __global__ void __launch_bounds__(SORT_T) k_sort(PrepGraph *pgs, const RawGraph 
   __shared__ uint32_t s_w[33];
   __shared__ uint32_t s_base[256], s_tot[256], s_cst[256];
   __shared__ uint32_t s_cnt[SORT_T / 32][257];
-  __shared__ uint64_t s_k[SORT_T];  // a chunk in digit order (coalesced write-out)
+  __shared__ KT s_k[SORT_T];  // a chunk in digit order (coalesced write-out)
   __shared__ uint32_t s_v[SORT_T];
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const uint64_t maxk = key_bits >= 64 ? ~0ull : ((1ull << key_bits) - 1);
@@ -606,14 +607,14 @@ __global__ void __launch_bounds__(SORT_T) k_sort(PrepGraph *pgs, const RawGraph 
     uint32_t tot;
     uint32_t pre = cta_exscan(live, &tot, s_w);
     if (live) {
-      P.key0[run + pre] = maxk - P.rank[u];
+      ((KT *)P.key0)[run + pre] = (KT)(maxk - P.rank[u]);
       P.val0[run + pre] = (uint32_t)u;
     }
     run += tot;
   }
   const int32_t n = (int32_t)run;
   if (tid == 0) P.n = n;
-  uint64_t *kin = P.key0, *kout = P.key1;
+  KT *kin = (KT *)P.key0, *kout = (KT *)P.key1;
   uint32_t *vin = P.val0, *vout = P.val1;
   const unsigned lt = (1u << lane) - 1;
   for (int sh = 0; sh < key_bits; sh += 8) {
@@ -642,7 +643,7 @@ __global__ void __launch_bounds__(SORT_T) k_sort(PrepGraph *pgs, const RawGraph 
       __syncthreads();
       int32_t i = t0 + tid;
       bool valid = i < n;
-      uint64_t k = valid ? kin[i] : 0;
+      KT k = valid ? kin[i] : (KT)0;
       uint32_t v = valid ? vin[i] : 0;
       uint32_t dg = valid ? (uint32_t)((k >> sh) & 255) : 256u;
       unsigned peers = __match_any_sync(FULL, dg);
@@ -683,7 +684,7 @@ __global__ void __launch_bounds__(SORT_T) k_sort(PrepGraph *pgs, const RawGraph 
       __syncthreads();
       // write-out in chunk order: a digit's keys land contiguously
       if (i < n) {
-        const uint64_t kk = s_k[tid];
+        const KT kk = s_k[tid];
         const uint32_t d = (uint32_t)((kk >> sh) & 255);
         const uint32_t dst = s_base[d] + ((uint32_t)tid - s_cst[d]);
         kout[dst] = kk;
@@ -693,7 +694,7 @@ __global__ void __launch_bounds__(SORT_T) k_sort(PrepGraph *pgs, const RawGraph 
       if (tid < 256) s_base[tid] += s_tot[tid];
       __syncthreads();
     }
-    uint64_t *tk = kin; kin = kout; kout = tk;
+    KT *tk = kin; kin = kout; kout = tk;
     uint32_t *tv = vin; vin = vout; vout = tv;
   }
   // positions
@@ -709,7 +710,8 @@ __global__ void __launch_bounds__(SORT_T) k_sort(PrepGraph *pgs, const RawGraph 
 void launch_sort(PrepGraph *pgs, const RawGraph *raws, int nslots, int key_bits, int max_n, cudaStream_t st,
                  const uint32_t *nact) {
   (void)max_n;
-  k_sort<<<nslots, SORT_T, 0, st>>>(pgs, raws, key_bits, nact);
+  if (key_bits <= 32) k_sort<uint32_t><<<nslots, SORT_T, 0, st>>>(pgs, raws, key_bits, nact);
+  else k_sort<uint64_t><<<nslots, SORT_T, 0, st>>>(pgs, raws, key_bits, nact);
 }
 
 // ----------------------------------------------------------------- cards
