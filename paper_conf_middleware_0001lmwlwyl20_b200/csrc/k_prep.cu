@@ -522,7 +522,7 @@ void launch_heights(RawGraph *raw_dev, int32_t *scratch, int64_t vcap, cudaStrea
 
 // ------------------------------------------------------------- radix sort
 
-constexpr int SORT_T = 1024;
+constexpr int SORT_T = 512;
 
 // CTA exclusive scan of one value per thread; returns the prefix, *total = sum
 __device__ uint32_t cta_exscan(uint32_t v, uint32_t *total, uint32_t *s_w) {
