@@ -453,7 +453,8 @@ def main():
                              "candidates_per_s": cps, "ops_per_s": cps * d2.n_ops, "ms_per_sweep": ms2,
                              "kernel": ("k_lane_pk" if g2.time_bits == 32 and len(d2.alpha) == 1 else "k_sim_lane")
                              if tm2["topo"] == 2 else "k_sim",
-                             "deferred_to_prep": tm2["deferred"]}
+                             "deferred_to_prep": tm2["deferred"], "launches": tm2["launches"],
+                             "free_device_gb": torch.cuda.mem_get_info()[0] / 1e9}
             del g2
         # C5 under the paper's insertion policy (R1i): the same
         # stream, 100k candidates (the group kernel, a lane per device)

@@ -609,9 +609,10 @@ static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st,
   size_t freeb = 0, totb = 0;
   CK(cudaMemGetInfo(&freeb, &totb));
   size_t per = rt + pt;
-  // at most 60 % of the free and 30 % of the total device memory per graph
-  // (a wave that does not fit costs one more latency-bound preparation round)
-  int64_t slots = std::min<int64_t>(want, (int64_t)(std::min(freeb * 3 / 5, totb * 3 / 10) / per));
+  // at most 60 % of the free and 40 % of the total device memory per graph
+  // (a wave that does not fit costs one more latency-bound preparation round;
+  // C5R8's 4,038 split slots take ~53 GB)
+  int64_t slots = std::min<int64_t>(want, (int64_t)(std::min(freeb * 3 / 5, totb * 2 / 5) / per));
   if (slots < 1) return fail(FASTT_ENOMEM, "device memory too small for one preparation slot (%zu bytes)", per);
   g->arena_slots = (int)slots;
   CK(cudaMalloc(&g->arena, per * slots));
