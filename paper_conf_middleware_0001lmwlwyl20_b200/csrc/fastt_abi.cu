@@ -592,11 +592,14 @@ static fastt_status prepare_base(fastt_graph *g, Base &B, cudaStream_t st) {
 // ------------------------------------------------------------- workspaces
 
 // preparation slots for `need` deferred candidates: sized to the batch (a
-// C5 sweep's ~4k split candidates prepare in one wave), capped at 8192 slots
-// and 40 % of free HBM, and kept for later calls with the same layout
+// C5 sweep's ~4k split candidates prepare in one wave), capped at
+// ARENA_MAX_SLOTS (small graphs' frequent deferrals -- C1 defers ~10 % of
+// its candidates -- take fewer rounds) and by memory (below), and kept for
+// later calls with the same layout
+constexpr int64_t ARENA_MAX_SLOTS = 32768;  // (slot-indexed launches put the slot in gridDim.y)
 static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st, int64_t need) {
   size_t rt = B.rl.total, pt = B.pl.total;
-  const int64_t want = std::min<int64_t>(std::max<int64_t>(need, 64), 8192);
+  const int64_t want = std::min<int64_t>(std::max<int64_t>(need, 64), ARENA_MAX_SLOTS);
   if (g->arena && g->arena_raw_total == rt && g->arena_prep_total == pt && g->arena_slots >= want) return FASTT_OK;
   cudaFree(g->arena);
   cudaFree(g->tmpl_dev);
@@ -1100,7 +1103,7 @@ static void read_defer_summary(fastt_graph *g) {
 // arena slots of a sequential (non-overlapped) evaluation: the last such
 // call's deferral count (one round when the count repeats), at least `lo`
 static int64_t seq_arena_want(const fastt_graph *g, int64_t lo) {
-  return std::max<int64_t>(std::max<int64_t>(256, lo), std::min<int64_t>(g->seq_defer_hint, 8192));
+  return std::max<int64_t>(std::max<int64_t>(256, lo), std::min<int64_t>(g->seq_defer_hint, ARENA_MAX_SLOTS));
 }
 
 static fastt_status build_defer_graph(fastt_graph *g, Base &B, const SimArgs &b, int cap, bool results,
@@ -1422,7 +1425,7 @@ static fastt_status eval_batch(fastt_graph *g, Base &B, const Cand *d_cands, int
     ovl = t.lane == 1;
   }
   if (ovl) {
-    TRY(ensure_arena(g, B, st, std::max<int64_t>(256, std::min<int64_t>(g->pin_defer_hint, 8192))));
+    TRY(ensure_arena(g, B, st, std::max<int64_t>(256, std::min<int64_t>(g->pin_defer_hint, ARENA_MAX_SLOTS))));
     const int cap = g->arena_slots;
     int wmain;
     {
@@ -2229,7 +2232,7 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
       const int64_t q_hi = std::min<int64_t>(n - 1, (hi - first) / stride);
       nsp = q_hi >= q_lo ? q_hi - q_lo + 1 : 0;
     }
-    TRY(ensure_arena(g, B, st, std::max<int64_t>(nsp + 256, std::min<int64_t>(g->pin_defer_hint, 8192))));
+    TRY(ensure_arena(g, B, st, std::max<int64_t>(nsp + 256, std::min<int64_t>(g->pin_defer_hint, ARENA_MAX_SLOTS))));
     cap = g->arena_slots;
     {
       SimArgs t = a;
