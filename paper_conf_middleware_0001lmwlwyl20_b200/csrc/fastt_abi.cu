@@ -256,6 +256,7 @@ struct fastt_graph {
   // arena (per base layout)
   size_t arena_raw_total = 0, arena_prep_total = 0;
   int arena_slots = 0;
+  bool arena_capped = false;  // the last allocation was limited by the memory cap
   char *arena = nullptr;
   RawGraph *tmpl_dev = nullptr, *slot_raws_dev = nullptr;
   PrepGraph *slot_pgs_dev = nullptr;
@@ -600,7 +601,12 @@ constexpr int64_t ARENA_MAX_SLOTS = 32768;  // (slot-indexed launches put the sl
 static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st, int64_t need) {
   size_t rt = B.rl.total, pt = B.pl.total;
   const int64_t want = std::min<int64_t>(std::max<int64_t>(need, 64), ARENA_MAX_SLOTS);
-  if (g->arena && g->arena_raw_total == rt && g->arena_prep_total == pt && g->arena_slots >= want) return FASTT_OK;
+  const bool same = g->arena && g->arena_raw_total == rt && g->arena_prep_total == pt;
+  if (same && g->arena_slots >= want) return FASTT_OK;
+  // (an arena the memory cap already limited is not re-allocated for a
+  // larger request of the same layout: the cap would bind again, and each
+  // attempt frees and re-allocates tens of GB; more rounds run instead)
+  if (same && g->arena_capped) return FASTT_OK;
   cudaFree(g->arena);
   cudaFree(g->tmpl_dev);
   cudaFree(g->slot_raws_dev);
@@ -618,6 +624,7 @@ static fastt_status ensure_arena(fastt_graph *g, const Base &B, cudaStream_t st,
   int64_t slots = std::min<int64_t>(want, (int64_t)(std::min(freeb * 3 / 5, totb * 2 / 5) / per));
   if (slots < 1) return fail(FASTT_ENOMEM, "device memory too small for one preparation slot (%zu bytes)", per);
   g->arena_slots = (int)slots;
+  g->arena_capped = slots < want;
   CK(cudaMalloc(&g->arena, per * slots));
   std::vector<RawGraph> tm(slots);
   std::vector<PrepGraph> pg(slots);
@@ -2259,6 +2266,7 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
       nsp = q_hi >= q_lo ? q_hi - q_lo + 1 : 0;
     }
     TRY(ensure_arena(g, B, st, seq_arena_want(g, nsp)));
+    host_trace("sweep: arena (sequential path)");
   }
   TRY(timing_begin(g, flags, st));
   if (n > 0 && ovl) {
@@ -2297,6 +2305,7 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
       a.slot_index = g->srt_i;
       a.slot_result = nullptr;
     }
+    host_trace("sweep: sorted (sequential path)");
     {
       int grid;
       size_t smem;
@@ -2305,6 +2314,7 @@ fastt_status fastt_sweep_best(const fastt_graph *gc_, const fastt_gen_params *ge
     }
     g->launches += NL_SIM;
     CK(cudaGetLastError());
+    host_trace("sweep: main launch (sequential path)");
     timing_mark(g, flags, 1, st);
     TRY(run_defer_loop(g, B, a, g->arena_slots, a.mode == 3 ? 0 : 2, false, n, nullptr, &a.stream, first, stride,
                        false, g->counters + 1, st));
