@@ -330,8 +330,8 @@ struct fastt_graph {
   // FASTT_OVL_MODE: 1 (default) the main launch starts once the preparation
   // kernels are done and overlaps the slot simulations; 0 it starts at once
   // (all three run together); 2 main_bps blocks per SM start at once, the
-  // rest after the preparation kernels (measured on C5, 1e6 candidates:
-  // 106 / 108.7 (LANE_BATCHES=2) / 123-179 ms per sweep: a latency-bound
+  // rest after the preparation kernels (measured on C5, 1e6 candidates, final
+  // code: 93.6 / 103-104 / 97.7-107 ms per sweep: a latency-bound
   // preparation chain co-running with the issue-bound main launch slows by
   // more than the main launch gains)
   int ovl_mode = 1;
@@ -1335,7 +1335,7 @@ static fastt_status run_overlapped(fastt_graph *g, Base &B, SimArgs a, int64_t n
     blocks = (warps + (int64_t)g->lane_batches * wpb - 1) / ((int64_t)g->lane_batches * wpb);
   } else {  // persistent, optionally leaving block slots to the preparation stream
     blocks = wmain / std::max(1, a.pk_wpb);
-    if (g->main_bps > 0) blocks = std::min<int64_t>(blocks, (int64_t)g->sms * g->main_bps);
+    if (g->main_bps > 0 && g->ovl_mode != 2) blocks = std::min<int64_t>(blocks, (int64_t)g->sms * g->main_bps);
   }
   if (g->ovl_mode == 2 && g->lane_batches == 0) {
     // two persistent launches on one work queue: main_bps blocks per SM at
